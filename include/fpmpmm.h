@@ -1,0 +1,268 @@
+/* fpmpmm.h -- C ABI of libfpmpmm.so: FPM-partitioned column-based parallel
+ * matrix multiplication on B200 (sm_100a).
+ *
+ * Method: Zhong, Rychkov, Lastovetsky, "Data Partitioning on Heterogeneous
+ * Multicore and Multi-GPU Systems Using Functional Performance Models of
+ * Data-Parallel Applications", Cluster 2012.  Citations "P:<line>" refer to
+ * the paper text; "Q<n>" to the readings listed in DESIGN.md.
+ *
+ * The application "takes the FPMs of heterogeneous processors as input,
+ * partitions the matrices using the FPM-based data partitioning algorithm, and
+ * performs the blocked matrix multiplication, using the GEMM kernel".
+ * The four calls of that statement are fpm_sample, fpm_partition,
+ * colpart_arrange and pmm_run.
+ *
+ * Conventions
+ *  - Every function returns an int status: FPM_OK (0) on success, a negative
+ *    FPM_E* code on failure.  No C++ exception crosses the ABI.  The message of
+ *    the last failure on the calling thread is returned by fpm_last_error().
+ *  - "blocks" are b x b blocks of the N x N matrices; n = N / b, T = n * n.
+ *  - Host matrices are row-major.  Pointers passed in are owned by the caller,
+ *    read (or written) only for the duration of the call; the library never
+ *    keeps them.
+ *  - The library owns everything it allocates inside a pmm_ctx (device
+ *    buffers, streams, events, green contexts, NCCL communicators); all of it
+ *    is released by pmm_destroy.
+ *  - fpm_partition, colpart_arrange, colpart_plan_step and fpm_model_speed are
+ *    pure host functions: no GPU, no context, thread-safe.  Calls on one
+ *    pmm_ctx must be serialised by the caller.
+ */
+#ifndef FPMPMM_H
+#define FPMPMM_H
+
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define FPM_OK            0
+#define FPM_EINVAL       -1   /* invalid argument (shape, model, arrangement, ...) */
+#define FPM_ENOMEM       -2   /* host or device allocation failed                 */
+#define FPM_ECUDA        -3   /* CUDA runtime / driver error (message has detail)  */
+#define FPM_ENCCL        -4   /* NCCL error                                        */
+#define FPM_EUNSUPPORTED -5   /* configuration not supported (e.g. SM cap)         */
+#define FPM_ESTATE       -6   /* call out of order (e.g. pmm_compute before setup) */
+
+#define FPM_MAX_DEVICES  16
+
+typedef enum { FPM_F32 = 0, FPM_F64 = 1 } fpm_dtype;
+typedef enum { FPM_DIST_PM1 = 0, FPM_DIST_INT = 1 } fpm_dist;
+
+/* Functional performance model of one device (P:8 "represents the processor
+ * speed by a function of problem size"; P:18 built from timed kernel runs on
+ * sqrt(x) x sqrt(x) submatrices).  x[j]: problem size in blocks, strictly
+ * increasing, >= 1.  s[j]: speed in flop/s, finite, > 0.  npts >= 1.
+ * Evaluation (reading Q4): piecewise linear in s between points, constant
+ * beyond both ends; t(x) = x / s(x). */
+typedef struct {
+    int32_t        npts;
+    const int64_t* x;
+    const double*  s;
+} fpm_model;
+
+/* One device's rectangle of the column-based arrangement (Fig. 1(a)),
+ * in blocks: column index `col` (-1 for an empty rectangle), top-left block
+ * (row0, col0), height h and width w. */
+typedef struct {
+    int32_t col;
+    int64_t row0, col0, h, w;
+} colpart_rect;
+
+/* One pivot transfer of iteration k (reading Q12), in blocks.
+ * A moves: device src sends rows [begin, end) of block-column k to dst.
+ * B moves: device src sends cols [begin, end) of block-row k to dst.
+ * src == dst marks a local use (no transfer). */
+typedef struct {
+    int32_t src, dst;
+    int64_t begin, end;
+} colpart_move;
+
+/* Statistics of one pmm_compute / pmm_run.  Times in seconds, measured with
+ * CUDA events on the launching streams. */
+typedef struct {
+    double  t_compute_s;                        /* k-loop, first event to last, max over devices  */
+    double  t_upload_s;                         /* host -> device scatter (pmm_run only)          */
+    double  t_download_s;                       /* device -> host gather  (pmm_run only)          */
+    double  per_dev_compute_s[FPM_MAX_DEVICES]; /* sum of split + update kernel time per device   */
+    double  per_dev_update_s[FPM_MAX_DEVICES];  /* sum of rank-b update kernel time per device    */
+    double  gflops;                             /* 2 N^3 / t_compute_s / 1e9                      */
+    double  imbalance;                          /* max/mean - 1 of per_dev_compute_s (area > 0)   */
+    int64_t iters;                              /* n = N / b                                      */
+    int64_t comm_bytes;                         /* pivot bytes received by this process's devices */
+    int64_t kernel_launches;                    /* library kernels launched in the k-loop         */
+} pmm_stats;
+
+typedef struct pmm_ctx pmm_ctx;
+
+/* ---------------------------------------------------------------- misc */
+const char* fpm_last_error(void);  /* thread-local, never NULL */
+int32_t     fpm_abi_version(void); /* 1 */
+
+/* ------------------------------------------------ host algorithms (pure) */
+
+/* s(x) of one model (P:8, reading Q4).  FPM_EINVAL if the model is invalid
+ * or x < 0. */
+int fpm_model_speed(const fpm_model* model, int64_t x, double* s_out);
+
+/* FPM-based data partitioning (P:9 "all processors complete their work
+ * within the same time"; algorithm of [5]; readings Q1-Q3).
+ * Computes integer areas d[0..p) with sum d = total_blocks such that the
+ * times d_i / s_i(d_i) are balanced, by the geometric method: bisection of
+ * the line through the origin (slope = 1 / time) over the speed graphs,
+ * followed by an exact integer phase.  The result is bit-identical to the
+ * canonical definition (give blocks one at a time to the device with the
+ * smallest t_i(d_i + 1), ties to the lowest index), which is min-max optimal
+ * whenever each t_i is non-decreasing.
+ * models: p entries (1 <= p <= FPM_MAX_DEVICES).  d_out: p int64, written.
+ * iters_out (nullable): bisection iterations used.
+ * Errors: FPM_EINVAL on p out of range, total_blocks < 0, invalid model. */
+int fpm_partition(int64_t total_blocks, int32_t p, const fpm_model* models,
+                  int64_t* d_out, int32_t* iters_out);
+
+/* Column-based arrangement ("arranges the submatrices to be as square as
+ * possible, minimising the total volume of communications"; [17] P:144;
+ * reading Q10): rectangles of areas close to d_i tiling the n x n grid,
+ * minimising the sum of half-perimeters.  d: p areas with sum = n*n.
+ * rects_out: p entries.  Achieved areas h_i * w_i differ from d_i by the
+ * integer rounding of widths/heights.  Zero areas give empty rectangles
+ * (col = -1).  Errors: FPM_EINVAL if sum d != n*n, any d < 0, n < 1. */
+int colpart_arrange(int64_t n, int32_t p, const int64_t* d, colpart_rect* rects_out);
+
+/* Delivery plan of iteration k ("pivot column of matrix A and pivot row
+ * of matrix B are broadcast horizontally and vertically"; reading Q12).
+ * Writes at most a_cap / b_cap moves, sorted by (src, dst, begin); the counts
+ * are always written.  FPM_EINVAL if the rectangles do not tile the grid, k
+ * out of range, or a capacity is too small (counts still written). */
+int colpart_plan_step(int64_t n, int32_t p, const colpart_rect* rects, int64_t k,
+                      colpart_move* a_moves, int32_t a_cap, int32_t* a_count,
+                      colpart_move* b_moves, int32_t b_cap, int32_t* b_count);
+
+/* ------------------------------------------------------------- runtime */
+
+/* Single-process context driving p "devices".  Device i runs on CUDA ordinal
+ * cuda_devices[i]; several devices may share one GPU.  sm_caps (nullable):
+ * 0 = the whole GPU, else a cap on SMs (multiple of 8, >= 8) realised with a
+ * green context (heterogeneity emulation, BASELINE north_star).  Pivot
+ * transfers between devices are device-to-device copies on the receivers'
+ * communication streams.  Errors: FPM_EINVAL, FPM_ECUDA, FPM_EUNSUPPORTED. */
+int pmm_create_local(int32_t p, const int32_t* cuda_devices, const int32_t* sm_caps,
+                     pmm_ctx** out);
+
+/* Multi-process context: one process per GPU (rank `rank` of `world`), pivot
+ * broadcasts over NCCL (libnccl.so.2 loaded at run time): vertical B pivot
+ * rows with ncclBroadcast on per-column communicators, horizontal A pivot
+ * slices with grouped ncclSend/ncclRecv.  nccl_id: 128 bytes from
+ * pmm_nccl_unique_id() on rank 0, distributed by the caller. */
+int pmm_nccl_unique_id(uint8_t id_out[128]);
+int pmm_create_nccl(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm_cap,
+                    const uint8_t nccl_id[128], pmm_ctx** out);
+
+int pmm_destroy(pmm_ctx* ctx);
+
+/* Fix the problem: N x N matrices, blocking factor b ("blocking factor
+ * b"), arrangement rects[p] (p = devices of the context, or world size in
+ * NCCL mode), dtype.  Allocates the resident A_i, B_i, C_i of the devices this
+ * process drives plus pivot staging.  Requires b | N, b % 32 == 0 (FP32) or
+ * b % 8 == 0 (FP64), rects tiling the n x n grid.
+ * Layout in HBM: A_i as w_i block-columns, each (h_i b) x b row-major
+ * (K-major pivot panels); B_i as h_i block-rows, each b x (w_i b) row-major;
+ * C_i (h_i b) x (w_i b) row-major. */
+int pmm_setup(pmm_ctx* ctx, int64_t N, int64_t b, int32_t p, const colpart_rect* rects,
+              fpm_dtype dt);
+
+/* Copy this process's rectangles of A and B from host windows (untimed
+ * distribution, P:8 "Data partitioning algorithms map all data to processors
+ * and do not redistribute it").  The host arrays hold the global rows
+ * [row_base, ...) and columns [col_base, ...) with leading dimension ld
+ * (elements); every local rectangle must lie inside the window.  Element type
+ * = the dtype of pmm_setup.  Zeroes C_i. */
+int pmm_upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld,
+               int64_t row_base, int64_t col_base);
+
+/* Fill the resident A_i, B_i with the seeded counter-based generator of
+ * synth/__init__.py (global element index row*N + col), zero C_i. */
+int pmm_fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int32_t dist);
+
+/* Run the N/b iterations on resident data: per iteration pivot exchange
+ * (look-ahead one iteration, on communication streams) and the rank-b update
+ * C_i += A(b) x B(b) on each device.  Starts from C_i = 0 (zeroed by
+ * upload / fill / the previous download when zero_c != 0).  Blocks until done. */
+int pmm_compute(pmm_ctx* ctx, int32_t zero_c, pmm_stats* stats);
+
+/* Copy this process's C_i into a host window (same convention as upload). */
+int pmm_download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base);
+
+/* Copy the global block C[r0 : r0+rows, c0 : c0+cols] (must lie inside one
+ * rectangle held by this process) into host memory (row stride ld elements).
+ * For sampled checks at full size without gathering all of C. */
+int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t rows, int64_t cols, void* C_host,
+                       int64_t ld);
+
+/* Whole call on host matrices: setup (if the problem changed) + upload +
+ * compute + download.  A, B, C are host windows as for pmm_upload.  Upload and
+ * download times are reported in stats. */
+int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int64_t b,
+            int32_t p, const colpart_rect* rects, fpm_dtype dt, int64_t ld,
+            int64_t row_base, int64_t col_base, pmm_stats* stats);
+
+/* Build a speed function (P:9 kernel-based benchmarking, P:10 (iii) repeated
+ * until statistically reliable, P:18 sqrt(x) x sqrt(x) submatrices): for each
+ * x = sizes[j] (must be a perfect square m^2), time the computational kernel
+ * C += A(b) x B(b) (pivot split + rank-b update) on an (m b) x (m b) C on
+ * device `dev` of the context (its SM cap applies) and return
+ * speeds_out[j] = 2 x b^3 / t in flop/s.  Repeats until the 95% confidence
+ * half-width is <= 2.5% of the mean (>= 5, <= 50 repetitions, reading Q8).
+ * rel_ci95_out / reps_out nullable. */
+int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t* sizes,
+               int32_t nsizes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out);
+
+/* Tuning / selection knobs (all optional):
+ *   "f32_scheme": 0 = F16X3 (default: x 2^e = h0 + h1 in fp16, per-row
+ *                 power-of-two scales, 3 kind::f16 MMAs), 1 = TF32X3
+ *                 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  DESIGN.md Q15.
+ *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
+ * FPM_EINVAL on unknown key or value. */
+int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value);
+
+/* --------------------------------------- kernel-level entry points (tests)
+ * Device pointers on the current CUDA device, launched asynchronously on
+ * `stream` (a cudaStream_t; NULL = the legacy default stream). */
+
+/* FP32 operand split of a rows x K panel (row stride ld, elements) for the
+ * tensor cores (reading Q15).  scheme 0 (F16X3): hi/lo are fp16 rows x K,
+ * inv_scale[rows] receives 2^-e of each row.  scheme 1 (TF32X3): hi/lo are
+ * fp32 rows x K holding tf32 values; inv_scale unused (may be NULL).
+ * K % 4 == 0, ld % 4 == 0. */
+int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64_t K, int32_t scheme,
+                    void* hi, void* lo, float* inv_scale, void* stream);
+
+/* dst (cols x rows, contiguous) = transpose of src (rows x cols, row stride
+ * ld); dt = FPM_F32 or FPM_F64.  Used for the K-major B pivot panel. */
+int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64_t cols, void* dst,
+                    void* stream);
+
+/* Rank-b update C (M x Nc, row-major, ldc) += A (M x K) x B with B
+ * given as Bt (Nc x K, K-major), operands as produced by fpm_k_split_f32 with
+ * the same scheme (sa / sb: inverse row scales of A and Bt for F16X3, NULL
+ * for TF32X3).  cta_group 1 or 2; num_sms = persistent grid (0 = all SMs).
+ * Requires K % 8 == 0, ldc % 4 == 0. */
+int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
+                     const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
+                     int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, void* stream);
+
+/* Rank-b update in FP64 on DMMA: C (M x Nc, ldc) += A (M x K, lda) x Bt^T,
+ * Bt (Nc x K). */
+int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
+                     int64_t K, int64_t ldc, void* stream);
+
+/* Fill a rows x cols window (ld elements) of the seeded global N x N matrix
+ * starting at global (r0, c0); dt = FPM_F32 or FPM_F64; dist = fpm_dist. */
+int fpm_k_fill_synthetic(void* dst, int32_t dt, int64_t ld, uint64_t seed, int64_t N, int64_t r0,
+                         int64_t c0, int64_t rows, int64_t cols, int32_t dist, void* stream);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* FPMPMM_H */

@@ -1,0 +1,58 @@
+// Internal launcher interface of the sm_100a kernels (C++ only, not the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "../common.hpp"
+
+namespace fpm {
+
+// How an FP32 operand is represented on the tensor cores (reading Q15).
+enum class SplitScheme : int {
+    F16X3 = 0,   // x 2^e = h0 + h1 in fp16, per-row power-of-two scale, 3 x kind::f16
+    TF32X3 = 1,  // x = hi + lo in tf32, 3 x kind::tf32
+};
+
+struct UpdateArgs {
+    const void* a_hi;   // M x K, K-major (row-major, ld = K), fp16 or tf32-in-fp32
+    const void* a_lo;
+    const void* bt_hi;  // Nc x K, K-major
+    const void* bt_lo;
+    const float* sa;    // per-row inverse scale of A (F16X3), M floats
+    const float* sb;    // per-row inverse scale of Bt (F16X3), Nc floats
+    float* C;           // M x Nc, ld = ldc
+    int64_t M, Nc, K, ldc;
+    SplitScheme scheme;
+    int cta_group;      // 1 or 2
+    int num_sms;        // SMs the persistent grid may use
+};
+
+// C += A . Bt^T  (the rank-b update)
+void launch_update_f32(const UpdateArgs& a, cudaStream_t st);
+
+// Split an FP32 panel (rows x K, row stride ld) into the two operand halves.
+// F16X3: hi/lo are __half[rows*K], inv_scale[rows] written.
+// TF32X3: hi/lo are float[rows*K], inv_scale untouched (may be null).
+void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, SplitScheme s, void* hi,
+                       void* lo, float* inv_scale, cudaStream_t st);
+
+// dst (cols x rows, K-major) = transpose of src (rows x cols, ld).
+void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t cols, float* dst,
+                          cudaStream_t st);
+void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t cols, double* dst,
+                          cudaStream_t st);
+
+// C (M x Nc, ldc) += A (M x K, lda) . Bt^T, Bt (Nc x K), FP64 on DMMA.
+void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
+                       int64_t K, int64_t ldc, cudaStream_t st);
+
+// Seeded counter-based generator (same bits as synth/__init__.py).
+void launch_fill_synthetic(void* dst, bool f64, int64_t ld, uint64_t seed, int64_t N, int64_t r0, int64_t c0,
+                           int64_t rows, int64_t cols, int dist, cudaStream_t st);
+
+// Panel copy (rows x cols elements of `elem` bytes) between strided buffers.
+void launch_zero(void* dst, size_t bytes, cudaStream_t st);
+
+}  // namespace fpm

@@ -1,0 +1,251 @@
+// Pivot staging kernels: the FP32 operand split for the tensor
+// cores, the B pivot-row transpose to a K-major panel, the FP64 update on DMMA,
+// and the seeded synthetic-input generator.  All HBM-bound except the FP64
+// update; vectorised, coalesced, grid sized in multiples of the SM count.
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.hpp"
+
+namespace fpm {
+
+namespace {
+
+__device__ __forceinline__ float tf32_rna(float x) {
+    uint32_t r;
+    asm("cvt.rna.tf32.f32 %0, %1;" : "=r"(r) : "f"(x));
+    return __uint_as_float(r);
+}
+
+__device__ __forceinline__ float warp_max(float v) {
+#pragma unroll
+    for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
+    return v;
+}
+
+// One warp per row.  F16X3: choose 2^s with the row max scaled into [2^14, 2^15),
+// h0 = fp16(x 2^s), h1 = fp16(x 2^s - h0); inv_scale = 2^-s.
+__global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ src, int64_t ld, int64_t rows,
+                                                      int64_t K, __half* __restrict__ hi, __half* __restrict__ lo,
+                                                      float* __restrict__ inv_scale) {
+    const int64_t row = (int64_t)blockIdx.x * 8 + threadIdx.x / 32;
+    const int lane = threadIdx.x % 32;
+    if (row >= rows) return;
+    const float4* s4 = reinterpret_cast<const float4*>(src + row * ld);
+    const int64_t n4 = K / 4;
+    float m = 0.0f;
+    for (int64_t i = lane; i < n4; i += 32) {
+        const float4 v = s4[i];
+        m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+    }
+    m = warp_max(m);
+    int e = 0;
+    if (m > 0.0f) {
+        frexpf(m, &e);  // m < 2^e
+    }
+    int s = (m > 0.0f) ? 15 - e : 0;
+    s = s < -126 ? -126 : (s > 127 ? 127 : s);
+    const float scale = ldexpf(1.0f, s);
+    if (lane == 0) inv_scale[row] = ldexpf(1.0f, -s);
+    __half2* h2 = reinterpret_cast<__half2*>(hi + row * K);
+    __half2* l2 = reinterpret_cast<__half2*>(lo + row * K);
+    for (int64_t i = lane; i < n4; i += 32) {
+        const float4 v = s4[i];
+        const float x[4] = {v.x * scale, v.y * scale, v.z * scale, v.w * scale};
+        __half h[4], l[4];
+#pragma unroll
+        for (int j = 0; j < 4; ++j) {
+            h[j] = __float2half_rn(x[j]);
+            l[j] = __float2half_rn(x[j] - __half2float(h[j]));
+        }
+        h2[2 * i] = __halves2half2(h[0], h[1]);
+        h2[2 * i + 1] = __halves2half2(h[2], h[3]);
+        l2[2 * i] = __halves2half2(l[0], l[1]);
+        l2[2 * i + 1] = __halves2half2(l[2], l[3]);
+    }
+}
+
+__global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__ src, int64_t ld, int64_t rows,
+                                                       int64_t K, float* __restrict__ hi, float* __restrict__ lo) {
+    const int64_t n4 = K / 4;
+    const int64_t total = rows * n4;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = idx / n4, c = idx - r * n4;
+        const float4 v = reinterpret_cast<const float4*>(src + r * ld)[c];
+        float4 h, l;
+        h.x = tf32_rna(v.x); l.x = tf32_rna(v.x - h.x);
+        h.y = tf32_rna(v.y); l.y = tf32_rna(v.y - h.y);
+        h.z = tf32_rna(v.z); l.z = tf32_rna(v.z - h.z);
+        h.w = tf32_rna(v.w); l.w = tf32_rna(v.w - h.w);
+        reinterpret_cast<float4*>(hi + r * K)[c] = h;
+        reinterpret_cast<float4*>(lo + r * K)[c] = l;
+    }
+}
+
+template <class T>
+__global__ void __launch_bounds__(256) transpose_k(const T* __restrict__ src, int64_t ld, int64_t rows,
+                                                   int64_t cols, T* __restrict__ dst) {
+    __shared__ T tile[32][33];
+    const int64_t r0 = (int64_t)blockIdx.y * 32, c0 = (int64_t)blockIdx.x * 32;
+    for (int j = threadIdx.y; j < 32; j += 8) {
+        const int64_t r = r0 + j, c = c0 + threadIdx.x;
+        if (r < rows && c < cols) tile[j][threadIdx.x] = src[r * ld + c];
+    }
+    __syncthreads();
+    for (int j = threadIdx.y; j < 32; j += 8) {
+        const int64_t c = c0 + j, r = r0 + threadIdx.x;
+        if (r < rows && c < cols) dst[c * rows + r] = tile[threadIdx.x][j];
+    }
+}
+
+// ---- seeded generator: identical bits to synth/__init__.py
+__device__ __forceinline__ uint64_t synth_hash(uint64_t seed, uint64_t idx) {
+    uint64_t z = seed * 0xD1B54A32D192ED03ull + (idx + 1ull) * 0x9E3779B97F4A7C15ull;
+    z = (z ^ (z >> 30)) * 0xBF58476D1CE4E5B9ull;
+    z = (z ^ (z >> 27)) * 0x94D049BB133111EBull;
+    return z ^ (z >> 31);
+}
+
+template <class T>
+__global__ void __launch_bounds__(256) fill_k(T* dst, int64_t ld, uint64_t seed, int64_t N, int64_t r0, int64_t c0,
+                                              int64_t rows, int64_t cols, int dist) {
+    const int64_t total = rows * cols;
+    for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
+         idx += (int64_t)gridDim.x * blockDim.x) {
+        const int64_t r = idx / cols, c = idx - r * cols;
+        const uint64_t z = synth_hash(seed, (uint64_t)(r0 + r) * (uint64_t)N + (uint64_t)(c0 + c));
+        double x;
+        if (dist == FPM_DIST_PM1) x = (double)(z >> 40) * (1.0 / 8388608.0) - 1.0;
+        else x = (double)((z >> 32) % 17ull) - 8.0;
+        dst[r * ld + c] = (T)x;
+    }
+}
+
+// ---- FP64 rank-b update on DMMA (mma.sync m8n8k4 f64).  64 x 64 CTA tile,
+// 4 warps of 32 x 32, K staged through shared memory in steps of 16.
+__global__ void __launch_bounds__(128) update_f64_k(const double* __restrict__ A, int64_t lda,
+                                                    const double* __restrict__ Bt, double* __restrict__ C,
+                                                    int64_t M, int64_t Nc, int64_t K, int64_t ldc) {
+    __shared__ double As[64][17];
+    __shared__ double Bs[64][17];
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int64_t m0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 64;
+    const int wm = (warp / 2) * 32, wn = (warp % 2) * 32;
+    double acc[4][4][2];
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+    for (int64_t k0 = 0; k0 < K; k0 += 16) {
+        for (int idx = threadIdx.x; idx < 64 * 16; idx += 128) {
+            const int r = idx / 16, c = idx % 16;
+            const int64_t gm = m0 + r, gn = n0 + r, gk = k0 + c;
+            As[r][c] = (gm < M && gk < K) ? A[gm * lda + gk] : 0.0;
+            Bs[r][c] = (gn < Nc && gk < K) ? Bt[gn * K + gk] : 0.0;
+        }
+        __syncthreads();
+#pragma unroll
+        for (int kk = 0; kk < 16; kk += 4) {
+            double a[4], b[4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i) a[i] = As[wm + i * 8 + lane / 4][kk + lane % 4];
+#pragma unroll
+            for (int j = 0; j < 4; ++j) b[j] = Bs[wn + j * 8 + lane / 4][kk + lane % 4];
+#pragma unroll
+            for (int i = 0; i < 4; ++i)
+#pragma unroll
+                for (int j = 0; j < 4; ++j)
+                    asm volatile(
+                        "mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                        : "+d"(acc[i][j][0]), "+d"(acc[i][j][1])
+                        : "d"(a[i]), "d"(b[j]));
+        }
+        __syncthreads();
+    }
+#pragma unroll
+    for (int i = 0; i < 4; ++i)
+#pragma unroll
+        for (int j = 0; j < 4; ++j)
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+                const int64_t gm = m0 + wm + i * 8 + lane / 4;
+                const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4) + h;
+                if (gm < M && gn < Nc) C[gm * ldc + gn] += acc[i][j][h];
+            }
+}
+
+int grid_for(int64_t work, int threads) {
+    int dev = 0, sms = 148;
+    cudaGetDevice(&dev);
+    cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    int64_t blocks = (work + threads - 1) / threads;
+    const int64_t cap = (int64_t)sms * 8;  // 8 resident 256-thread CTAs per SM
+    if (blocks > cap) blocks = cap;
+    return (int)(blocks < 1 ? 1 : blocks);
+}
+
+void check_launch(const char* what) {
+    cudaError_t e = cudaGetLastError();
+    if (e != cudaSuccess) fail(FPM_ECUDA, "%s launch: %s", what, cudaGetErrorString(e));
+}
+
+}  // namespace
+
+void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, SplitScheme s, void* hi, void* lo,
+                       float* inv_scale, cudaStream_t st) {
+    if (rows <= 0 || K <= 0) return;
+    FPM_CHECK_ARG(K % 4 == 0 && ld % 4 == 0, "split: K and ld must be multiples of 4");
+    if (s == SplitScheme::F16X3) {
+        const int64_t blocks = (rows + 7) / 8;
+        split_rows_f16<<<(unsigned)blocks, 256, 0, st>>>(src, ld, rows, K, static_cast<__half*>(hi),
+                                                         static_cast<__half*>(lo), inv_scale);
+        check_launch("split_rows_f16");
+    } else {
+        split_rows_tf32<<<grid_for(rows * K / 4, 256), 256, 0, st>>>(src, ld, rows, K, static_cast<float*>(hi),
+                                                                      static_cast<float*>(lo));
+        check_launch("split_rows_tf32");
+    }
+}
+
+void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t cols, float* dst, cudaStream_t st) {
+    if (rows <= 0 || cols <= 0) return;
+    dim3 grid((unsigned)((cols + 31) / 32), (unsigned)((rows + 31) / 32));
+    transpose_k<float><<<grid, dim3(32, 8), 0, st>>>(src, ld, rows, cols, dst);
+    check_launch("transpose_f32");
+}
+
+void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t cols, double* dst,
+                          cudaStream_t st) {
+    if (rows <= 0 || cols <= 0) return;
+    dim3 grid((unsigned)((cols + 31) / 32), (unsigned)((rows + 31) / 32));
+    transpose_k<double><<<grid, dim3(32, 8), 0, st>>>(src, ld, rows, cols, dst);
+    check_launch("transpose_f64");
+}
+
+void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
+                       int64_t K, int64_t ldc, cudaStream_t st) {
+    if (M <= 0 || Nc <= 0 || K <= 0) return;
+    dim3 grid((unsigned)((Nc + 63) / 64), (unsigned)((M + 63) / 64));
+    update_f64_k<<<grid, 128, 0, st>>>(A, lda, Bt, C, M, Nc, K, ldc);
+    check_launch("update_f64");
+}
+
+void launch_fill_synthetic(void* dst, bool f64, int64_t ld, uint64_t seed, int64_t N, int64_t r0, int64_t c0,
+                           int64_t rows, int64_t cols, int dist, cudaStream_t st) {
+    if (rows <= 0 || cols <= 0) return;
+    FPM_CHECK_ARG(dist == FPM_DIST_PM1 || dist == FPM_DIST_INT, "unknown dist %d", dist);
+    const int g = grid_for(rows * cols, 256);
+    if (f64) fill_k<double><<<g, 256, 0, st>>>(static_cast<double*>(dst), ld, seed, N, r0, c0, rows, cols, dist);
+    else fill_k<float><<<g, 256, 0, st>>>(static_cast<float*>(dst), ld, seed, N, r0, c0, rows, cols, dist);
+    check_launch("fill_synthetic");
+}
+
+void launch_zero(void* dst, size_t bytes, cudaStream_t st) {
+    cudaError_t e = cudaMemsetAsync(dst, 0, bytes, st);
+    if (e != cudaSuccess) fail(FPM_ECUDA, "cudaMemsetAsync: %s", cudaGetErrorString(e));
+}
+
+}  // namespace fpm

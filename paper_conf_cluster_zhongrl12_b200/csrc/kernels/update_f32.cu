@@ -1,0 +1,390 @@
+// Rank-b update C_i += A(b) x B(b) (Fig. 1(b)) in FP32 precision
+// on the sm_100a tensor cores.
+//
+// tcgen05 has no FP32 kind, so each FP32 operand arrives split in two
+// (reading Q15):
+//   * F16X3  (default): x * 2^e = h0 + h1 with h0 = fp16_rn(x 2^e),
+//                       h1 = fp16_rn(x 2^e - h0), 2^e a per-row power of two
+//                       (A rows, B columns) that puts the row maximum in
+//                       [2^14, 2^15).  C += 2^-(ea_i+eb_j) (h0 h0' + h0 h1' + h1 h0')
+//                       -> 22 significant bits per operand, 3 MMAs of kind::f16.
+//   * TF32X3:           x = hi + lo, hi = tf32_rna(x), lo = tf32_rna(x - hi);
+//                       C += hi hi' + hi lo' + lo hi' -> 3 MMAs of kind::tf32
+//                       (half the f16 rate).
+// Both keep FP32 accumulation in TMEM.
+//
+// Structure (warp-specialised persistent kernel, one CTA per SM or CTA pair):
+//   warp 0      TMA producer: A_hi/A_lo/B_hi/B_lo k-blocks of 128 B rows, 128B swizzle
+//   warp 1      TMEM allocator + single-thread tcgen05.mma issuer (leader CTA)
+//   warps 2-5   epilogue: TMEM -> registers, C chunk (128 x 32 fp32) TMA-loaded
+//               into smem, C += scale * acc, TMA-stored back (C read-modify-write
+//               every iteration, "accumulating the intermediate results")
+// Two TMEM accumulators (2 x BN columns) let the epilogue of tile t overlap the
+// mainloop of tile t+1.  CG = 2 pairs two SMs on a 256-row tile (cta_group::2).
+#include <cuda.h>
+#include <cuda_fp16.h>
+#include <cuda_runtime.h>
+
+#include <cstdint>
+
+#include "kernels.hpp"
+#include "ptx.cuh"
+
+namespace fpm {
+
+template <int CG, bool TF32, int BN, int STAGES>
+struct UpdCfg {
+    static constexpr int BM = 128;                 // rows of C per CTA
+    static constexpr int TILE_M = BM * CG;         // rows per MMA tile
+    static constexpr int BN_CTA = BN / CG;         // B^T rows loaded per CTA
+    static constexpr int ELEM = TF32 ? 4 : 2;      // operand bytes
+    static constexpr int BK = 128 / ELEM;          // k elements per 128-B row
+    static constexpr int A_BYTES = BM * 128;       // one operand half (hi or lo)
+    static constexpr int B_BYTES = BN_CTA * 128;
+    static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
+    static constexpr int C_CHUNK_BYTES = BM * 128; // 128 rows x 32 fp32
+    static constexpr int N_CHUNKS = BN / 32;
+    static constexpr int TMEM_COLS = 2 * BN;
+    static constexpr int BAR_BYTES = 256;
+    static constexpr int SMEM = 1024 /*align slack*/ + STAGES * STAGE_BYTES + 2 * C_CHUNK_BYTES + BAR_BYTES;
+    static constexpr uint32_t IDESC = ptx::idesc_f32acc(TILE_M, BN, TF32);
+    static constexpr int THREADS = 192;
+    static_assert(TMEM_COLS == 256 || TMEM_COLS == 512, "TMEM columns must be a power of two");
+    static_assert(SMEM <= 232448, "shared memory budget");
+};
+
+struct UpdParams {
+    int M, Nc, K;
+    int tiles_m, tiles_n, num_tiles;
+    const float* sa;  // per-row inverse scales of A (F16X3) or nullptr
+    const float* sb;  // per-column inverse scales of B (F16X3) or nullptr
+};
+
+// Grouped raster over tiles so concurrently running CTAs share A / B tiles in L2.
+__device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int& tm, int& tn) {
+    constexpr int G = 16;
+    const int per_group = G * tiles_n;
+    const int g = t / per_group;
+    const int first_m = g * G;
+    const int gm = min(tiles_m - first_m, G);
+    const int r = t - g * per_group;
+    tm = first_m + r % gm;
+    tn = r / gm;
+}
+
+template <int CG, bool TF32, int BN, int STAGES>
+__global__ void __launch_bounds__(192, 1)
+    update_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
+                  const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
+                  const __grid_constant__ CUtensorMap tmC, const UpdParams P) {
+    using Cfg = UpdCfg<CG, TF32, BN, STAGES>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* stage_base = smem;
+    uint8_t* cbuf = smem + STAGES * Cfg::STAGE_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + 2 * Cfg::C_CHUNK_BYTES);
+    uint64_t* full = bars;                       // [STAGES]
+    uint64_t* empty = bars + STAGES;             // [STAGES]
+    uint64_t* tfull = bars + 2 * STAGES;         // [2]
+    uint64_t* tempty = bars + 2 * STAGES + 2;    // [2]
+    uint64_t* cfull = bars + 2 * STAGES + 4;     // [2]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
+
+    const uint32_t warp = threadIdx.x / 32;
+    const uint32_t lane = threadIdx.x % 32;
+    const uint32_t rank = (CG == 2) ? ptx::cluster_ctarank() : 0;
+    const bool leader = rank == 0;
+    const int cluster_id = blockIdx.x / CG;
+    const int num_clusters = gridDim.x / CG;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            ptx::mbar_init(&full[s], 1);
+            ptx::mbar_init(&empty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            ptx::mbar_init(&tfull[a], 1);
+            ptx::mbar_init(&tempty[a], 4 * CG);  // one arrival per epilogue warp of each CTA
+            ptx::mbar_init(&cfull[a], 1);
+        }
+        ptx::fence_mbar_init();
+    }
+    if (warp == 0 && lane == 0) {
+        ptx::tma_prefetch_desc(&tmA_hi);
+        ptx::tma_prefetch_desc(&tmA_lo);
+        ptx::tma_prefetch_desc(&tmB_hi);
+        ptx::tma_prefetch_desc(&tmB_lo);
+        ptx::tma_prefetch_desc(&tmC);
+    }
+    if (warp == 1) {
+        ptx::tmem_alloc<CG>(tmem_slot, Cfg::TMEM_COLS);
+        ptx::tmem_relinquish<CG>();
+    }
+    ptx::tc_fence_before();
+    __syncthreads();
+    if constexpr (CG == 2) ptx::cluster_sync();
+    ptx::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int num_kb = (P.K + Cfg::BK - 1) / Cfg::BK;
+
+    if (warp == 0) {
+        // ------------------------------------------------------------ producer
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+                int tm, tn;
+                tile_coords(t, P.tiles_m, P.tiles_n, tm, tn);
+                const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
+                const int n0 = tn * BN + (int)rank * Cfg::BN_CTA;
+                for (int kb = 0; kb < num_kb; ++kb) {
+                    ptx::mbar_wait(&empty[stage], phase ^ 1);
+                    uint8_t* sA_hi = stage_base + stage * Cfg::STAGE_BYTES;
+                    uint8_t* sA_lo = sA_hi + Cfg::A_BYTES;
+                    uint8_t* sB_hi = sA_lo + Cfg::A_BYTES;
+                    uint8_t* sB_lo = sB_hi + Cfg::B_BYTES;
+                    const int k0 = kb * Cfg::BK;
+                    if constexpr (CG == 1) {
+                        ptx::mbar_arrive_expect_tx(&full[stage], Cfg::STAGE_BYTES);
+                        ptx::tma_load_2d(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
+                        ptx::tma_load_2d(sA_lo, &tmA_lo, &full[stage], k0, m0, ptx::kEvictLast);
+                        ptx::tma_load_2d(sB_hi, &tmB_hi, &full[stage], k0, n0, ptx::kEvictLast);
+                        ptx::tma_load_2d(sB_lo, &tmB_lo, &full[stage], k0, n0, ptx::kEvictLast);
+                    } else {
+                        if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
+                        ptx::tma_load_2d_cg2(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
+                        ptx::tma_load_2d_cg2(sA_lo, &tmA_lo, &full[stage], k0, m0, ptx::kEvictLast);
+                        ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, ptx::kEvictLast);
+                        ptx::tma_load_2d_cg2(sB_lo, &tmB_lo, &full[stage], k0, n0, ptx::kEvictLast);
+                    }
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ----------------------------------------------------------- MMA issuer
+        if (leader) {
+            int stage = 0;
+            uint32_t phase = 0;
+            int it = 0;
+            for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
+                const int acc = it & 1;
+                const uint32_t acc_par = (it >> 1) & 1;
+                ptx::mbar_wait(&tempty[acc], acc_par ^ 1);
+                ptx::tc_fence_after();
+                const uint32_t d_tmem = tmem_base + acc * BN;
+                for (int kb = 0; kb < num_kb; ++kb) {
+                    ptx::mbar_wait(&full[stage], phase);
+                    ptx::tc_fence_after();
+                    if (lane == 0) {
+                        const uint32_t a_hi = ptx::smem_u32(stage_base + stage * Cfg::STAGE_BYTES);
+                        const uint32_t a_lo = a_hi + Cfg::A_BYTES;
+                        const uint32_t b_hi = a_lo + Cfg::A_BYTES;
+                        const uint32_t b_lo = b_hi + Cfg::B_BYTES;
+                        const uint64_t dA_hi = ptx::sdesc_k_sw128(a_hi), dA_lo = ptx::sdesc_k_sw128(a_lo);
+                        const uint64_t dB_hi = ptx::sdesc_k_sw128(b_hi), dB_lo = ptx::sdesc_k_sw128(b_lo);
+#pragma unroll
+                        for (int k = 0; k < 4; ++k) {
+                            const uint64_t off = (uint64_t)(k * 32) >> 4;  // 32 B per MMA k-step
+                            ptx::umma<CG, TF32>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC, (kb | k) != 0);
+                            ptx::umma<CG, TF32>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
+                            ptx::umma<CG, TF32>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
+                        }
+                        ptx::umma_commit<CG>(&empty[stage]);
+                    }
+                    __syncwarp();
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+                if (lane == 0) ptx::umma_commit<CG>(&tfull[acc]);
+                __syncwarp();
+            }
+        }
+    } else {
+        // -------------------------------------------------------------- epilogue
+        const uint32_t e = threadIdx.x - 64;   // 0..127
+        const uint32_t q = warp & 3;           // TMEM lane quarter this warp may access
+        const uint32_t r = q * 32 + lane;      // row of the CTA tile
+        uint32_t cpar = 0;  // bit b = parity of cfull[b]
+        int it = 0;
+        for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
+            int tm, tn;
+            tile_coords(t, P.tiles_m, P.tiles_n, tm, tn);
+            const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
+            const int n0 = tn * BN;
+            const int acc = it & 1;
+            const uint32_t acc_par = (it >> 1) & 1;
+            if (e == 0) {
+                ptx::bulk_wait_read0();
+                for (int c = 0; c < 2 && c < Cfg::N_CHUNKS; ++c) {
+                    ptx::mbar_arrive_expect_tx(&cfull[c], Cfg::C_CHUNK_BYTES);
+                    ptx::tma_load_2d(cbuf + c * Cfg::C_CHUNK_BYTES, &tmC, &cfull[c], n0 + 32 * c, m0,
+                                     ptx::kEvictFirst);
+                }
+            }
+            const int grow = m0 + (int)r;
+            const float sa = (P.sa != nullptr && grow < P.M) ? P.sa[grow] : 1.0f;
+            ptx::mbar_wait(&tfull[acc], acc_par);
+            ptx::tc_fence_after();
+            const uint32_t t_row = tmem_base + ((q * 32) << 16) + acc * BN;
+#pragma unroll 1
+            for (int c = 0; c < Cfg::N_CHUNKS; ++c) {
+                const int buf = c & 1;
+                float v[32];
+                ptx::tmem_ld_32x32b_x32(t_row + 32 * c, v);
+                if (c == Cfg::N_CHUNKS - 1) {
+                    // accumulator fully read: hand it back to the MMA warp
+                    ptx::tc_fence_before();
+                    __syncwarp();
+                    if (lane == 0) {
+                        if constexpr (CG == 1) ptx::mbar_arrive(&tempty[acc]);
+                        else ptx::mbar_arrive_cluster(&tempty[acc], 0);
+                    }
+                }
+                if (P.sb != nullptr) {
+                    const int gc = n0 + 32 * c;
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) {
+                        const float sbj = (gc + j < P.Nc) ? __ldg(P.sb + gc + j) : 0.0f;
+                        v[j] *= sa * sbj;
+                    }
+                }
+                ptx::mbar_wait(&cfull[buf], (cpar >> buf) & 1u);
+                cpar ^= 1u << buf;
+                uint8_t* rowp = cbuf + buf * Cfg::C_CHUNK_BYTES + r * 128;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    float4* p4 = reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4));
+                    float4 cv = *p4;
+                    cv.x += v[4 * j + 0];
+                    cv.y += v[4 * j + 1];
+                    cv.z += v[4 * j + 2];
+                    cv.w += v[4 * j + 3];
+                    *p4 = cv;
+                }
+                ptx::fence_proxy_async_smem();
+                ptx::named_bar_sync(1, 128);
+                if (e == 0) {
+                    ptx::tma_store_2d(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0);
+                    ptx::bulk_commit();
+                    if (c + 2 < Cfg::N_CHUNKS) {
+                        ptx::bulk_wait_read0();
+                        ptx::mbar_arrive_expect_tx(&cfull[buf], Cfg::C_CHUNK_BYTES);
+                        ptx::tma_load_2d(cbuf + buf * Cfg::C_CHUNK_BYTES, &tmC, &cfull[buf], n0 + 32 * (c + 2), m0,
+                                         ptx::kEvictFirst);
+                    }
+                }
+            }
+        }
+        if (e == 0) ptx::bulk_wait0();
+    }
+
+    ptx::tc_fence_before();
+    __syncthreads();
+    if constexpr (CG == 2) ptx::cluster_sync();
+    if (warp == 1) {
+        ptx::tc_fence_after();
+        ptx::tmem_dealloc<CG>(tmem_base, Cfg::TMEM_COLS);
+    }
+}
+
+// ------------------------------------------------------------------- host side
+namespace {
+
+using EncodeTiledFn = CUresult (*)(CUtensorMap*, CUtensorMapDataType, cuuint32_t, void*, const cuuint64_t*,
+                                   const cuuint64_t*, const cuuint32_t*, const cuuint32_t*, CUtensorMapInterleave,
+                                   CUtensorMapSwizzle, CUtensorMapL2promotion, CUtensorMapFloatOOBfill);
+
+EncodeTiledFn get_encode() {
+    static EncodeTiledFn fn = nullptr;
+    if (!fn) {
+        cudaDriverEntryPointQueryResult q;
+        void* p = nullptr;
+        cudaError_t err = cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q);
+        if (err != cudaSuccess || q != cudaDriverEntryPointSuccess || !p)
+            fail(FPM_ECUDA, "cuTensorMapEncodeTiled unavailable (%s)", cudaGetErrorString(err));
+        fn = reinterpret_cast<EncodeTiledFn>(p);
+    }
+    return fn;
+}
+
+}  // namespace
+
+// Row-major rows x cols matrix (ld elements), 128B-swizzled box of box_cols x box_rows.
+CUtensorMap make_tmap_2d(const void* base, CUtensorMapDataType dt, int elem_bytes, int64_t rows, int64_t cols,
+                         int64_t ld, int box_cols, int box_rows) {
+    CUtensorMap m;
+    cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+    cuuint64_t strides[1] = {(cuuint64_t)(ld * elem_bytes)};
+    cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
+    cuuint32_t estr[2] = {1, 1};
+    CUresult r = get_encode()(&m, dt, 2, const_cast<void*>(base), dims, strides, box, estr,
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+    if (r != CUDA_SUCCESS)
+        fail(FPM_ECUDA, "cuTensorMapEncodeTiled failed (%d) rows=%lld cols=%lld ld=%lld", (int)r,
+             (long long)rows, (long long)cols, (long long)ld);
+    return m;
+}
+
+template <int CG, bool TF32, int BN, int STAGES>
+static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
+    using Cfg = UpdCfg<CG, TF32, BN, STAGES>;
+    const CUtensorMapDataType odt = TF32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+    const CUtensorMap tAh = make_tmap_2d(a.a_hi, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
+    const CUtensorMap tAl = make_tmap_2d(a.a_lo, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
+    const CUtensorMap tBh = make_tmap_2d(a.bt_hi, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+    const CUtensorMap tBl = make_tmap_2d(a.bt_lo, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+    const CUtensorMap tC = make_tmap_2d(a.C, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.M, a.Nc, a.ldc, 32, Cfg::BM);
+    UpdParams P;
+    P.M = (int)a.M;
+    P.Nc = (int)a.Nc;
+    P.K = (int)a.K;
+    P.tiles_m = (int)((a.M + Cfg::TILE_M - 1) / Cfg::TILE_M);
+    P.tiles_n = (int)((a.Nc + BN - 1) / BN);
+    P.num_tiles = P.tiles_m * P.tiles_n;
+    P.sa = a.sa;
+    P.sb = a.sb;
+    auto kern = update_kernel<CG, TF32, BN, STAGES>;
+    static uint64_t attr_done = 0;  // one bit per CUDA device
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(attr_done & (1ull << dev))) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+        attr_done |= 1ull << dev;
+    }
+    int clusters = a.num_sms / CG;
+    if (clusters > P.num_tiles) clusters = P.num_tiles;
+    if (clusters < 1) clusters = 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(clusters * CG);
+    cfg.blockDim = dim3(Cfg::THREADS);
+    cfg.dynamicSmemBytes = Cfg::SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = CG;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tAh, tAl, tBh, tBl, tC, P);
+    if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
+}
+
+void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
+    if (a.M <= 0 || a.Nc <= 0 || a.K <= 0) return;
+    FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
+    FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
+    FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
+    const bool tf32 = a.scheme == SplitScheme::TF32X3;
+    if (a.cta_group == 2) {
+        if (tf32) launch_update_t<2, true, 256, 3>(a, st);
+        else launch_update_t<2, false, 256, 3>(a, st);
+    } else {
+        if (tf32) launch_update_t<1, true, 256, 2>(a, st);
+        else launch_update_t<1, false, 256, 2>(a, st);
+    }
+}
+
+}  // namespace fpm

@@ -1,0 +1,936 @@
+// Runtime of the FPM-partitioned column-based parallel matrix multiplication
+// (§IV): device contexts, resident data layout, the N/b
+// iteration loop with look-ahead pivot exchange, kernel-based speed sampling
+// (fpm_sample) and the C ABI of the runtime part.
+//
+// Per device and iteration k (slot = k mod 2, look-ahead one iteration):
+//   comm stream:    wait free[slot] -> receive A(rows_i, k), B(k, cols_i)
+//                   (local copies or NCCL) -> split / transpose into the slot's
+//                   operand buffers -> record ready[slot]
+//   compute stream: wait ready[slot] -> rank-b update C_i += A(b) B(b) ->
+//                   record free[slot]
+// so the exchange and staging of k+1 run under the update of k (P:40/P:68
+// overlap principle; "broadcast horizontally and vertically").
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <string>
+#include <vector>
+
+#include "../common.hpp"
+#include "../host/host_algos.hpp"
+#include "../kernels/kernels.hpp"
+#include "nccl_loader.hpp"
+
+#define CU(expr)                                                                                        \
+    do {                                                                                                \
+        cudaError_t _e = (expr);                                                                        \
+        if (_e != cudaSuccess)                                                                          \
+            ::fpm::fail(FPM_ECUDA, "%s: %s (%s:%d)", #expr, cudaGetErrorString(_e), __FILE__, __LINE__); \
+    } while (0)
+#define NC(expr)                                                                                   \
+    do {                                                                                           \
+        ncclResult_t _r = (expr);                                                                  \
+        if (_r != ncclSuccess)                                                                     \
+            ::fpm::fail(FPM_ENCCL, "%s: %s", #expr, ::fpm::nccl().GetErrorString(_r));             \
+    } while (0)
+
+namespace fpm {
+
+struct Device {
+    int idx = 0;       // index in the arrangement (= rank in NCCL mode)
+    int cuda_dev = 0;
+    int sm_cap = 0;    // 0 = all SMs
+    int num_sms = 0;   // persistent grid of the update kernel
+    cudaStream_t s_comp = nullptr, s_comm = nullptr;
+    cudaEvent_t ev_ready[2] = {}, ev_free[2] = {};
+    cudaEvent_t ev_start = nullptr, ev_stop = nullptr, ev_io0 = nullptr, ev_io1 = nullptr;
+    std::vector<cudaEvent_t> ev_pack0, ev_pack1, ev_upd0, ev_upd1;
+
+    // problem state
+    colpart_rect rect{-1, 0, 0, 0, 0};
+    int64_t H = 0, W = 0;  // rectangle in elements
+    void* A = nullptr;     // w block-columns, each H x b row-major (K-major panels)
+    void* B = nullptr;     // H x W row-major (h block-rows of b x W)
+    void* C = nullptr;     // H x W row-major
+    void* a_recv[2] = {}, *b_recv[2] = {};
+    void* bt[2] = {};                       // W x b (K-major) transposed B pivot row
+    void* a_hi[2] = {}, *a_lo[2] = {}, *b_hi[2] = {}, *b_lo[2] = {};
+    float* sa[2] = {}, *sb[2] = {};
+    const void* a_op[2] = {};               // FP64: A operand of the slot
+    std::vector<void*> allocs;
+
+    bool live() const { return H > 0 && W > 0; }
+};
+
+}  // namespace fpm
+
+struct pmm_ctx {
+    bool nccl_mode = false;
+    int rank = 0, world = 1;
+    std::vector<fpm::Device> devs;
+    ncclComm_t world_comm = nullptr;
+    ncclComm_t col_comm = nullptr;
+    std::vector<int> col_members;  // global ranks of my column, sorted
+
+    bool have_problem = false;
+    int64_t N = 0, b = 0, n = 0;
+    int p = 0;
+    fpm_dtype dt = FPM_F32;
+    std::vector<colpart_rect> rects;
+    std::vector<std::vector<fpm::Move>> plan_a, plan_b;
+
+    int f32_scheme = 0;  // fpm::SplitScheme
+    int cta_group = 2;
+};
+
+namespace fpm {
+namespace {
+
+size_t esize(fpm_dtype dt) { return dt == FPM_F64 ? 8 : 4; }
+
+void* dalloc(Device& d, size_t bytes) {
+    if (bytes == 0) return nullptr;
+    void* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(FPM_ENOMEM, "cudaMalloc(%zu) on device %d: %s", bytes, d.cuda_dev, cudaGetErrorString(e));
+    }
+    d.allocs.push_back(p);
+    return p;
+}
+
+void free_problem(Device& d) {
+    cudaSetDevice(d.cuda_dev);
+    for (void* p : d.allocs) cudaFree(p);
+    d.allocs.clear();
+    for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1}) {
+        for (cudaEvent_t e : *v) cudaEventDestroy(e);
+        v->clear();
+    }
+    d.A = d.B = d.C = nullptr;
+    for (int s = 0; s < 2; ++s) {
+        d.a_recv[s] = d.b_recv[s] = d.bt[s] = d.a_hi[s] = d.a_lo[s] = d.b_hi[s] = d.b_lo[s] = nullptr;
+        d.sa[s] = d.sb[s] = nullptr;
+        d.a_op[s] = nullptr;
+    }
+    d.H = d.W = 0;
+}
+
+void init_device(Device& d) {
+    CU(cudaSetDevice(d.cuda_dev));
+    int sms = 0;
+    CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d.cuda_dev));
+    if (d.sm_cap != 0) {
+        if (d.sm_cap < 8 || d.sm_cap % 8 != 0 || d.sm_cap > sms)
+            fail(FPM_EUNSUPPORTED, "SM cap %d not achievable (multiple of 8 in [8, %d])", d.sm_cap, sms);
+        d.num_sms = d.sm_cap;
+    } else {
+        d.num_sms = sms;
+    }
+    CU(cudaStreamCreateWithFlags(&d.s_comp, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&d.s_comm, cudaStreamNonBlocking));
+    for (int s = 0; s < 2; ++s) {
+        CU(cudaEventCreateWithFlags(&d.ev_ready[s], cudaEventDisableTiming));
+        CU(cudaEventCreateWithFlags(&d.ev_free[s], cudaEventDisableTiming));
+    }
+    CU(cudaEventCreate(&d.ev_start));
+    CU(cudaEventCreate(&d.ev_stop));
+    CU(cudaEventCreate(&d.ev_io0));
+    CU(cudaEventCreate(&d.ev_io1));
+}
+
+void destroy_device(Device& d) {
+    free_problem(d);
+    cudaSetDevice(d.cuda_dev);
+    for (int s = 0; s < 2; ++s) {
+        if (d.ev_ready[s]) cudaEventDestroy(d.ev_ready[s]);
+        if (d.ev_free[s]) cudaEventDestroy(d.ev_free[s]);
+    }
+    for (cudaEvent_t e : {d.ev_start, d.ev_stop, d.ev_io0, d.ev_io1})
+        if (e) cudaEventDestroy(e);
+    if (d.s_comp) cudaStreamDestroy(d.s_comp);
+    if (d.s_comm) cudaStreamDestroy(d.s_comm);
+}
+
+float elapsed_ms(cudaEvent_t a, cudaEvent_t b) {
+    float ms = 0.0f;
+    CU(cudaEventElapsedTime(&ms, a, b));
+    return ms;
+}
+
+Device* local_dev(pmm_ctx* ctx, int idx) {
+    for (auto& d : ctx->devs)
+        if (d.idx == idx) return &d;
+    return nullptr;
+}
+
+// ---------------------------------------------------------------- setup
+void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects, fpm_dtype dt) {
+    FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype %d", (int)dt);
+    FPM_CHECK_ARG(N >= 1 && b >= 1 && N % b == 0, "b must divide N (N=%lld, b=%lld)", (long long)N,
+                  (long long)b);
+    FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 : b % 32 == 0, "b must be a multiple of %d",
+                  dt == FPM_F64 ? 8 : 32);
+    const int expect_p = ctx->nccl_mode ? ctx->world : (int)ctx->devs.size();
+    FPM_CHECK_ARG(p == expect_p, "arrangement has %d devices, context drives %d", p, expect_p);
+    FPM_CHECK_ARG(rects != nullptr, "null rects");
+    const int64_t n = N / b;
+    validate_rects(n, p, rects);
+
+    for (auto& d : ctx->devs) free_problem(d);
+    ctx->have_problem = false;
+    ctx->N = N;
+    ctx->b = b;
+    ctx->n = n;
+    ctx->p = p;
+    ctx->dt = dt;
+    ctx->rects.assign(rects, rects + p);
+    ctx->plan_a.assign(n, {});
+    ctx->plan_b.assign(n, {});
+    for (int64_t k = 0; k < n; ++k) plan_step(n, p, rects, k, ctx->plan_a[k], ctx->plan_b[k]);
+
+    const size_t es = esize(dt);
+    for (auto& d : ctx->devs) {
+        CU(cudaSetDevice(d.cuda_dev));
+        d.rect = rects[d.idx];
+        d.H = d.rect.h * b;
+        d.W = d.rect.w * b;
+        if (!d.live()) {
+            d.H = d.W = 0;
+            continue;
+        }
+        const size_t HW = (size_t)d.H * d.W;
+        d.A = dalloc(d, HW * es);
+        d.B = dalloc(d, HW * es);
+        d.C = dalloc(d, HW * es);
+        const size_t op = (dt == FPM_F64) ? 0 : (ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4);
+        for (int s = 0; s < 2; ++s) {
+            d.a_recv[s] = dalloc(d, (size_t)d.H * b * es);
+            d.b_recv[s] = dalloc(d, (size_t)b * d.W * es);
+            d.bt[s] = dalloc(d, (size_t)d.W * b * es);
+            if (dt == FPM_F32) {
+                d.a_hi[s] = dalloc(d, (size_t)d.H * b * op);
+                d.a_lo[s] = dalloc(d, (size_t)d.H * b * op);
+                d.b_hi[s] = dalloc(d, (size_t)d.W * b * op);
+                d.b_lo[s] = dalloc(d, (size_t)d.W * b * op);
+                d.sa[s] = static_cast<float*>(dalloc(d, (size_t)d.H * sizeof(float)));
+                d.sb[s] = static_cast<float*>(dalloc(d, (size_t)d.W * sizeof(float)));
+            }
+        }
+        for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1}) {
+            v->resize(n);
+            for (auto& e : *v) CU(cudaEventCreate(&e));
+        }
+        CU(cudaMemsetAsync(d.C, 0, HW * es, d.s_comp));
+    }
+
+    if (ctx->nccl_mode) {
+        // per-column communicators for the vertical B broadcast
+        if (ctx->col_comm) {
+            nccl().CommDestroy(ctx->col_comm);
+            ctx->col_comm = nullptr;
+        }
+        const colpart_rect& me = rects[ctx->rank];
+        const bool live = me.h > 0 && me.w > 0;
+        ctx->col_members.clear();
+        for (int q = 0; q < p; ++q)
+            if (rects[q].h > 0 && rects[q].w > 0 && live && rects[q].col == me.col) ctx->col_members.push_back(q);
+        const int color = live ? me.col : NCCL_SPLIT_NOCOLOR;
+        NC(nccl().CommSplit(ctx->world_comm, color, ctx->rank, &ctx->col_comm, nullptr));
+    }
+    for (auto& d : ctx->devs) {
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaDeviceSynchronize());
+    }
+    ctx->have_problem = true;
+}
+
+// ------------------------------------------------------------ iteration parts
+ncclDataType_t nccl_dtype(fpm_dtype dt) { return dt == FPM_F64 ? ncclFloat64 : ncclFloat32; }
+
+// Exchange + staging of iteration k on device d's comm stream.
+int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use) {
+    const size_t es = esize(ctx->dt);
+    const int64_t b = ctx->b;
+    int64_t bytes = 0;
+    CU(cudaSetDevice(d.cuda_dev));
+    if (!first_use) CU(cudaStreamWaitEvent(d.s_comm, d.ev_free[slot], 0));
+    const colpart_rect& r = d.rect;
+
+    // ---- A(rows_i, k): local if this device's column holds block-column k
+    const bool holder = r.col0 <= k && k < r.col0 + r.w;
+    const void* a_src;
+    if (holder) {
+        a_src = static_cast<const char*>(d.A) + (size_t)(k - r.col0) * d.H * b * es;
+    } else {
+        a_src = d.a_recv[slot];
+        if (!ctx->nccl_mode) {
+            for (const Move& m : ctx->plan_a[k]) {
+                if (m.dst != d.idx) continue;
+                Device* q = local_dev(ctx, m.src);
+                const colpart_rect& qr = ctx->rects[m.src];
+                const size_t cnt = (size_t)(m.end - m.begin) * b * b;
+                const char* src = static_cast<const char*>(q->A) +
+                                  ((size_t)(k - qr.col0) * q->H * b + (size_t)(m.begin - qr.row0) * b * b) * es;
+                char* dst = static_cast<char*>(d.a_recv[slot]) + (size_t)(m.begin - r.row0) * b * b * es;
+                CU(cudaMemcpyAsync(dst, src, cnt * es, cudaMemcpyDefault, d.s_comm));
+                bytes += (int64_t)(cnt * es);
+            }
+        }
+    }
+    // ---- B(k, cols_i): local if this device's rows hold block-row k
+    const bool owner = r.row0 <= k && k < r.row0 + r.h;
+    const void* b_src;
+    if (owner) {
+        b_src = static_cast<const char*>(d.B) + (size_t)(k - r.row0) * b * d.W * es;
+    } else {
+        b_src = d.b_recv[slot];
+        if (!ctx->nccl_mode) {
+            for (const Move& m : ctx->plan_b[k]) {
+                if (m.dst != d.idx) continue;
+                Device* o = local_dev(ctx, m.src);
+                const colpart_rect& orr = ctx->rects[m.src];
+                const char* src = static_cast<const char*>(o->B) + (size_t)(k - orr.row0) * b * o->W * es;
+                CU(cudaMemcpyAsync(d.b_recv[slot], src, (size_t)b * d.W * es, cudaMemcpyDefault, d.s_comm));
+                bytes += (int64_t)((size_t)b * d.W * es);
+            }
+        }
+    }
+    if (ctx->nccl_mode) {
+        const NcclApi& nc = nccl();
+        const ncclDataType_t ndt = nccl_dtype(ctx->dt);
+        NC(nc.GroupStart());
+        for (const Move& m : ctx->plan_a[k]) {
+            if (m.src == m.dst) continue;
+            const size_t cnt = (size_t)(m.end - m.begin) * b * b;
+            if (m.src == d.idx) {
+                const char* src = static_cast<const char*>(d.A) +
+                                  ((size_t)(k - r.col0) * d.H * b + (size_t)(m.begin - r.row0) * b * b) * es;
+                NC(nc.Send(src, cnt, ndt, m.dst, ctx->world_comm, d.s_comm));
+            } else if (m.dst == d.idx) {
+                char* dst = static_cast<char*>(d.a_recv[slot]) + (size_t)(m.begin - r.row0) * b * b * es;
+                NC(nc.Recv(dst, cnt, ndt, m.src, ctx->world_comm, d.s_comm));
+                bytes += (int64_t)(cnt * es);
+            }
+        }
+        NC(nc.GroupEnd());
+        if (ctx->col_members.size() > 1) {
+            int owner_rank = -1;
+            for (const Move& m : ctx->plan_b[k])
+                if (m.dst == d.idx) owner_rank = m.src;
+            const int root = (int)(std::find(ctx->col_members.begin(), ctx->col_members.end(), owner_rank) -
+                                   ctx->col_members.begin());
+            void* buf = owner ? const_cast<void*>(b_src) : d.b_recv[slot];
+            NC(nc.Broadcast(buf, buf, (size_t)b * d.W, ndt, root, ctx->col_comm, d.s_comm));
+            if (!owner) bytes += (int64_t)((size_t)b * d.W * es);
+        }
+    }
+
+    // ---- staging: K-major operands for the update
+    CU(cudaEventRecord(d.ev_pack0[k], d.s_comm));
+    if (ctx->dt == FPM_F32) {
+        const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
+        launch_split_rows(static_cast<const float*>(a_src), b, d.H, b, sch, d.a_hi[slot], d.a_lo[slot], d.sa[slot],
+                          d.s_comm);
+        launch_transpose_f32(static_cast<const float*>(b_src), d.W, b, d.W, static_cast<float*>(d.bt[slot]),
+                             d.s_comm);
+        launch_split_rows(static_cast<const float*>(d.bt[slot]), b, d.W, b, sch, d.b_hi[slot], d.b_lo[slot],
+                          d.sb[slot], d.s_comm);
+    } else {
+        d.a_op[slot] = a_src;
+        launch_transpose_f64(static_cast<const double*>(b_src), d.W, b, d.W, static_cast<double*>(d.bt[slot]),
+                             d.s_comm);
+    }
+    CU(cudaEventRecord(d.ev_pack1[k], d.s_comm));
+    CU(cudaEventRecord(d.ev_ready[slot], d.s_comm));
+    return bytes;
+}
+
+void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
+    CU(cudaSetDevice(d.cuda_dev));
+    CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
+    CU(cudaEventRecord(d.ev_upd0[k], d.s_comp));
+    if (ctx->dt == FPM_F32) {
+        UpdateArgs a;
+        a.a_hi = d.a_hi[slot];
+        a.a_lo = d.a_lo[slot];
+        a.bt_hi = d.b_hi[slot];
+        a.bt_lo = d.b_lo[slot];
+        const bool f16 = ctx->f32_scheme == (int)SplitScheme::F16X3;
+        a.sa = f16 ? d.sa[slot] : nullptr;
+        a.sb = f16 ? d.sb[slot] : nullptr;
+        a.C = static_cast<float*>(d.C);
+        a.M = d.H;
+        a.Nc = d.W;
+        a.K = ctx->b;
+        a.ldc = d.W;
+        a.scheme = (SplitScheme)ctx->f32_scheme;
+        a.cta_group = ctx->cta_group;
+        a.num_sms = d.num_sms;
+        launch_update_f32(a, d.s_comp);
+    } else {
+        launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
+                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, d.s_comp);
+    }
+    CU(cudaEventRecord(d.ev_upd1[k], d.s_comp));
+    CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
+}
+
+void compute(pmm_ctx* ctx, bool zero_c, pmm_stats* st) {
+    if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
+    const size_t es = esize(ctx->dt);
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        CU(cudaSetDevice(d.cuda_dev));
+        if (zero_c) CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
+        CU(cudaStreamSynchronize(d.s_comp));
+        CU(cudaStreamSynchronize(d.s_comm));
+    }
+    for (auto& d : ctx->devs) {
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaEventRecord(d.ev_start, d.s_comp));
+        CU(cudaStreamWaitEvent(d.s_comm, d.ev_start, 0));
+    }
+    int64_t bytes = 0, launches = 0;
+    const int per_iter = ctx->dt == FPM_F32 ? 4 : 2;
+    for (int64_t k = 0; k < ctx->n; ++k) {
+        const int slot = (int)(k & 1);
+        if (ctx->nccl_mode) {
+            // every rank takes part in the NCCL calls, live or not
+            Device& d = ctx->devs[0];
+            if (d.live()) {
+                bytes += issue_comm(ctx, d, k, slot, k < 2);
+                issue_update(ctx, d, k, slot);
+                launches += per_iter;
+            } else {
+                NC(nccl().GroupStart());
+                NC(nccl().GroupEnd());
+            }
+            continue;
+        }
+        for (auto& d : ctx->devs)
+            if (d.live()) bytes += issue_comm(ctx, d, k, slot, k < 2);
+        for (auto& d : ctx->devs)
+            if (d.live()) {
+                issue_update(ctx, d, k, slot);
+                launches += per_iter;
+            }
+    }
+    for (auto& d : ctx->devs) {
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaEventRecord(d.ev_stop, d.s_comp));
+    }
+    double t_max = 0.0;
+    for (auto& d : ctx->devs) {
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaEventSynchronize(d.ev_stop));
+        CU(cudaStreamSynchronize(d.s_comm));
+        t_max = std::max(t_max, (double)elapsed_ms(d.ev_start, d.ev_stop) * 1e-3);
+    }
+    if (st) {
+        std::memset(st, 0, sizeof(*st));
+        st->t_compute_s = t_max;
+        st->iters = ctx->n;
+        st->comm_bytes = bytes;
+        st->kernel_launches = launches;
+        st->gflops = t_max > 0 ? 2.0 * (double)ctx->N * (double)ctx->N * (double)ctx->N / t_max * 1e-9 : 0.0;
+        double mx = 0.0, sum = 0.0;
+        int cnt = 0;
+        for (auto& d : ctx->devs) {
+            if (!d.live()) continue;
+            double comp = 0.0, upd = 0.0;
+            for (int64_t k = 0; k < ctx->n; ++k) {
+                const double u = elapsed_ms(d.ev_upd0[k], d.ev_upd1[k]) * 1e-3;
+                comp += u + elapsed_ms(d.ev_pack0[k], d.ev_pack1[k]) * 1e-3;
+                upd += u;
+            }
+            if (d.idx < FPM_MAX_DEVICES) {
+                st->per_dev_compute_s[d.idx] = comp;
+                st->per_dev_update_s[d.idx] = upd;
+            }
+            mx = std::max(mx, comp);
+            sum += comp;
+            ++cnt;
+        }
+        st->imbalance = (cnt > 0 && sum > 0) ? mx / (sum / cnt) - 1.0 : 0.0;
+    }
+}
+
+// ------------------------------------------------------------ host transfers
+void check_window(pmm_ctx* ctx, const Device& d, int64_t ld, int64_t row_base, int64_t col_base) {
+    const int64_t R0 = d.rect.row0 * ctx->b, C0 = d.rect.col0 * ctx->b;
+    FPM_CHECK_ARG(row_base >= 0 && col_base >= 0 && R0 >= row_base && C0 >= col_base &&
+                      C0 - col_base + d.W <= ld,
+                  "device %d rectangle outside the host window (ld=%lld)", d.idx, (long long)ld);
+}
+
+void upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld, int64_t row_base, int64_t col_base,
+            double* t_out) {
+    if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_upload before pmm_setup");
+    FPM_CHECK_ARG(A && B, "null host matrix");
+    const size_t es = esize(ctx->dt);
+    const int64_t b = ctx->b;
+    double t = 0.0;
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        check_window(ctx, d, ld, row_base, col_base);
+        CU(cudaSetDevice(d.cuda_dev));
+        const int64_t R0 = d.rect.row0 * b - row_base, C0 = d.rect.col0 * b - col_base;
+        CU(cudaEventRecord(d.ev_io0, d.s_comp));
+        for (int64_t c = 0; c < d.rect.w; ++c) {
+            const char* src = static_cast<const char*>(A) + ((size_t)R0 * ld + (size_t)(C0 + c * b)) * es;
+            char* dst = static_cast<char*>(d.A) + (size_t)c * d.H * b * es;
+            CU(cudaMemcpy2DAsync(dst, b * es, src, ld * es, b * es, d.H, cudaMemcpyHostToDevice, d.s_comp));
+        }
+        const char* srcB = static_cast<const char*>(B) + ((size_t)R0 * ld + (size_t)C0) * es;
+        CU(cudaMemcpy2DAsync(d.B, d.W * es, srcB, ld * es, d.W * es, d.H, cudaMemcpyHostToDevice, d.s_comp));
+        CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
+        CU(cudaEventRecord(d.ev_io1, d.s_comp));
+    }
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaEventSynchronize(d.ev_io1));
+        t = std::max(t, (double)elapsed_ms(d.ev_io0, d.ev_io1) * 1e-3);
+    }
+    if (t_out) *t_out = t;
+}
+
+void download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base, double* t_out) {
+    if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_download before pmm_setup");
+    FPM_CHECK_ARG(C, "null host matrix");
+    const size_t es = esize(ctx->dt);
+    const int64_t b = ctx->b;
+    double t = 0.0;
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        check_window(ctx, d, ld, row_base, col_base);
+        CU(cudaSetDevice(d.cuda_dev));
+        const int64_t R0 = d.rect.row0 * b - row_base, C0 = d.rect.col0 * b - col_base;
+        CU(cudaEventRecord(d.ev_io0, d.s_comp));
+        char* dst = static_cast<char*>(C) + ((size_t)R0 * ld + (size_t)C0) * es;
+        CU(cudaMemcpy2DAsync(dst, ld * es, d.C, d.W * es, d.W * es, d.H, cudaMemcpyDeviceToHost, d.s_comp));
+        CU(cudaEventRecord(d.ev_io1, d.s_comp));
+    }
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaEventSynchronize(d.ev_io1));
+        t = std::max(t, (double)elapsed_ms(d.ev_io0, d.ev_io1) * 1e-3);
+    }
+    if (t_out) *t_out = t;
+}
+
+void fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int dist) {
+    if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_fill_synthetic before pmm_setup");
+    const size_t es = esize(ctx->dt);
+    const bool f64 = ctx->dt == FPM_F64;
+    const int64_t b = ctx->b;
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        CU(cudaSetDevice(d.cuda_dev));
+        const int64_t R0 = d.rect.row0 * b, C0 = d.rect.col0 * b;
+        for (int64_t c = 0; c < d.rect.w; ++c)
+            launch_fill_synthetic(static_cast<char*>(d.A) + (size_t)c * d.H * b * es, f64, b, seed_a, ctx->N, R0,
+                                  C0 + c * b, d.H, b, dist, d.s_comp);
+        launch_fill_synthetic(d.B, f64, d.W, seed_b, ctx->N, R0, C0, d.H, d.W, dist, d.s_comp);
+        CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
+    }
+    for (auto& d : ctx->devs) {
+        if (!d.live()) continue;
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaStreamSynchronize(d.s_comp));
+    }
+}
+
+// ------------------------------------------------------------ speed sampling
+double t975(int df) {
+    static const double tab[] = {0,      12.706, 4.303, 3.182, 2.776, 2.571, 2.447, 2.365, 2.306, 2.262, 2.228,
+                                 2.201, 2.179,  2.160, 2.145, 2.131, 2.120, 2.110, 2.101, 2.093, 2.086};
+    if (df <= 20) return tab[df < 1 ? 1 : df];
+    if (df <= 30) return 2.086 + (2.042 - 2.086) * (df - 20) / 10.0;
+    if (df <= 60) return 2.042 + (2.000 - 2.042) * (df - 30) / 30.0;
+    return 1.96;
+}
+
+// P:9 "The speed function of the application can be built more efficiently by
+// timing this kernel"; P:10 (iii) "experiments are repeated multiple times
+// until the results are statistically reliable"; P:18 kernel Ci += A(b) x B(b)
+// on sqrt(x) x sqrt(x) submatrices.  Speed = 2 x b^3 flop / time (Q7, Q8).
+void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes, int nsizes, double* speeds,
+            double* ci, int32_t* reps_out) {
+    Device* d = local_dev(ctx, dev);
+    FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
+    FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype");
+    FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 && b >= 8 : b % 32 == 0 && b >= 32, "bad block size b");
+    FPM_CHECK_ARG(nsizes >= 1 && sizes && speeds, "bad sizes");
+    int64_t mmax = 0;
+    std::vector<int64_t> ms(nsizes);
+    for (int j = 0; j < nsizes; ++j) {
+        const int64_t x = sizes[j];
+        FPM_CHECK_ARG(x >= 1, "size must be >= 1");
+        int64_t m = (int64_t)std::llround(std::sqrt((double)x));
+        while (m * m > x) --m;
+        while ((m + 1) * (m + 1) <= x) ++m;
+        FPM_CHECK_ARG(m * m == x, "size %lld is not a perfect square (P:18 sqrt(x) x sqrt(x))", (long long)x);
+        ms[j] = m;
+        mmax = std::max(mmax, m);
+    }
+    CU(cudaSetDevice(d->cuda_dev));
+    const int64_t L = mmax * b;
+    const size_t es = dt == FPM_F64 ? 8 : 4;
+    const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
+    const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
+    Device tmp;  // owns the scratch allocations
+    tmp.cuda_dev = d->cuda_dev;
+    struct Guard {
+        Device& t;
+        ~Guard() { free_problem(t); }
+    } guard{tmp};
+    void* C = dalloc(tmp, (size_t)L * L * es);
+    void* Ap = dalloc(tmp, (size_t)L * b * es);
+    void* Bp = dalloc(tmp, (size_t)b * L * es);
+    void* Bt = dalloc(tmp, (size_t)L * b * es);
+    void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
+    float *sa = nullptr, *sb = nullptr;
+    if (dt == FPM_F32) {
+        ah = dalloc(tmp, (size_t)L * b * op);
+        al = dalloc(tmp, (size_t)L * b * op);
+        bh = dalloc(tmp, (size_t)L * b * op);
+        bl = dalloc(tmp, (size_t)L * b * op);
+        sa = static_cast<float*>(dalloc(tmp, (size_t)L * 4));
+        sb = static_cast<float*>(dalloc(tmp, (size_t)L * 4));
+    }
+    cudaStream_t s = d->s_comp;
+    launch_fill_synthetic(Ap, dt == FPM_F64, b, 101, L, 0, 0, L, b, FPM_DIST_PM1, s);
+    launch_fill_synthetic(Bp, dt == FPM_F64, L, 102, L, 0, 0, b, L, FPM_DIST_PM1, s);
+    CU(cudaMemsetAsync(C, 0, (size_t)L * L * es, s));
+    cudaEvent_t e0, e1;
+    CU(cudaEventCreate(&e0));
+    CU(cudaEventCreate(&e1));
+    struct EvGuard {
+        cudaEvent_t a, b;
+        ~EvGuard() { cudaEventDestroy(a); cudaEventDestroy(b); }
+    } evg{e0, e1};
+
+    for (int j = 0; j < nsizes; ++j) {
+        const int64_t Lx = ms[j] * b;
+        auto run = [&]() {
+            if (dt == FPM_F32) {
+                launch_split_rows(static_cast<const float*>(Ap), b, Lx, b, sch, ah, al, sa, s);
+                launch_transpose_f32(static_cast<const float*>(Bp), L, b, Lx, static_cast<float*>(Bt), s);
+                launch_split_rows(static_cast<const float*>(Bt), b, Lx, b, sch, bh, bl, sb, s);
+                UpdateArgs a;
+                a.a_hi = ah; a.a_lo = al; a.bt_hi = bh; a.bt_lo = bl;
+                a.sa = sch == SplitScheme::F16X3 ? sa : nullptr;
+                a.sb = sch == SplitScheme::F16X3 ? sb : nullptr;
+                a.C = static_cast<float*>(C);
+                a.M = Lx; a.Nc = Lx; a.K = b; a.ldc = Lx;
+                a.scheme = sch;
+                a.cta_group = ctx->cta_group;
+                a.num_sms = d->num_sms;
+                launch_update_f32(a, s);
+            } else {
+                launch_transpose_f64(static_cast<const double*>(Bp), L, b, Lx, static_cast<double*>(Bt), s);
+                launch_update_f64(static_cast<const double*>(Ap), b, static_cast<const double*>(Bt),
+                                  static_cast<double*>(C), Lx, Lx, b, Lx, s);
+            }
+        };
+        for (int w = 0; w < 2; ++w) run();
+        std::vector<double> ts;
+        double mean = 0.0, half = 0.0;
+        for (int r = 0; r < 50; ++r) {
+            CU(cudaEventRecord(e0, s));
+            run();
+            CU(cudaEventRecord(e1, s));
+            CU(cudaEventSynchronize(e1));
+            ts.push_back(elapsed_ms(e0, e1) * 1e-3);
+            const int nr = (int)ts.size();
+            mean = 0.0;
+            for (double t : ts) mean += t;
+            mean /= nr;
+            double var = 0.0;
+            for (double t : ts) var += (t - mean) * (t - mean);
+            var = nr > 1 ? var / (nr - 1) : 0.0;
+            half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
+            if (nr >= 5 && half <= 0.025 * mean) break;
+        }
+        const double x = (double)(ms[j] * ms[j]);
+        speeds[j] = 2.0 * x * (double)b * (double)b * (double)b / mean;
+        if (ci) ci[j] = mean > 0 ? half / mean : 0.0;
+        if (reps_out) reps_out[j] = (int32_t)ts.size();
+    }
+}
+
+}  // namespace
+}  // namespace fpm
+
+// =================================================================== C ABI
+using fpm::guarded;
+
+extern "C" int pmm_create_local(int32_t p, const int32_t* cuda_devices, const int32_t* sm_caps, pmm_ctx** out) {
+    return guarded([&] {
+        FPM_CHECK_ARG(out != nullptr, "null out");
+        *out = nullptr;
+        FPM_CHECK_ARG(p >= 1 && p <= FPM_MAX_DEVICES, "p = %d out of [1, %d]", p, FPM_MAX_DEVICES);
+        FPM_CHECK_ARG(cuda_devices != nullptr, "null cuda_devices");
+        int count = 0;
+        CU(cudaGetDeviceCount(&count));
+        auto ctx = std::make_unique<pmm_ctx>();
+        ctx->devs.resize(p);
+        try {
+            for (int i = 0; i < p; ++i) {
+                FPM_CHECK_ARG(cuda_devices[i] >= 0 && cuda_devices[i] < count, "CUDA device %d out of range",
+                              cuda_devices[i]);
+                ctx->devs[i].idx = i;
+                ctx->devs[i].cuda_dev = cuda_devices[i];
+                ctx->devs[i].sm_cap = sm_caps ? sm_caps[i] : 0;
+                fpm::init_device(ctx->devs[i]);
+            }
+            // peer access between distinct GPUs (pivot copies over NVLink)
+            for (int i = 0; i < p; ++i)
+                for (int j = 0; j < p; ++j) {
+                    const int a = cuda_devices[i], c = cuda_devices[j];
+                    if (a == c) continue;
+                    int can = 0;
+                    cudaDeviceCanAccessPeer(&can, a, c);
+                    if (can) {
+                        cudaSetDevice(a);
+                        cudaDeviceEnablePeerAccess(c, 0);
+                        cudaGetLastError();  // already enabled is fine
+                    }
+                }
+        } catch (...) {
+            for (auto& d : ctx->devs) fpm::destroy_device(d);
+            throw;
+        }
+        *out = ctx.release();
+    });
+}
+
+extern "C" int pmm_nccl_unique_id(uint8_t id_out[128]) {
+    return guarded([&] {
+        FPM_CHECK_ARG(id_out != nullptr, "null id");
+        ncclUniqueId id;
+        NC(fpm::nccl().GetUniqueId(&id));
+        static_assert(sizeof(id) == 128, "ncclUniqueId size");
+        std::memcpy(id_out, &id, 128);
+    });
+}
+
+extern "C" int pmm_create_nccl(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm_cap,
+                               const uint8_t nccl_id[128], pmm_ctx** out) {
+    return guarded([&] {
+        FPM_CHECK_ARG(out != nullptr && nccl_id != nullptr, "null argument");
+        *out = nullptr;
+        FPM_CHECK_ARG(world >= 1 && world <= FPM_MAX_DEVICES && rank >= 0 && rank < world, "bad rank/world");
+        int count = 0;
+        CU(cudaGetDeviceCount(&count));
+        FPM_CHECK_ARG(cuda_device >= 0 && cuda_device < count, "CUDA device %d out of range", cuda_device);
+        auto ctx = std::make_unique<pmm_ctx>();
+        ctx->nccl_mode = true;
+        ctx->rank = rank;
+        ctx->world = world;
+        ctx->devs.resize(1);
+        ctx->devs[0].idx = rank;
+        ctx->devs[0].cuda_dev = cuda_device;
+        ctx->devs[0].sm_cap = sm_cap;
+        fpm::init_device(ctx->devs[0]);
+        ncclUniqueId id;
+        std::memcpy(&id, nccl_id, 128);
+        CU(cudaSetDevice(cuda_device));
+        ncclResult_t r = fpm::nccl().CommInitRank(&ctx->world_comm, world, id, rank);
+        if (r != ncclSuccess) {
+            fpm::destroy_device(ctx->devs[0]);
+            fpm::fail(FPM_ENCCL, "ncclCommInitRank: %s", fpm::nccl().GetErrorString(r));
+        }
+        *out = ctx.release();
+    });
+}
+
+extern "C" int pmm_destroy(pmm_ctx* ctx) {
+    return guarded([&] {
+        if (!ctx) return;
+        for (auto& d : ctx->devs) fpm::destroy_device(d);
+        if (ctx->nccl_mode) {
+            if (ctx->col_comm) fpm::nccl().CommDestroy(ctx->col_comm);
+            if (ctx->world_comm) fpm::nccl().CommDestroy(ctx->world_comm);
+        }
+        delete ctx;
+    });
+}
+
+extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx && key, "null argument");
+        const std::string k(key);
+        if (k == "f32_scheme") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "f32_scheme must be 0 or 1");
+            if (ctx->f32_scheme != (int)value) ctx->have_problem = false;  // operand buffers change size
+            ctx->f32_scheme = (int)value;
+        } else if (k == "cta_group") {
+            FPM_CHECK_ARG(value == 1 || value == 2, "cta_group must be 1 or 2");
+            ctx->cta_group = (int)value;
+        } else {
+            fpm::fail(FPM_EINVAL, "unknown option '%s'", key);
+        }
+    });
+}
+
+extern "C" int pmm_setup(pmm_ctx* ctx, int64_t N, int64_t b, int32_t p, const colpart_rect* rects, fpm_dtype dt) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        fpm::setup(ctx, N, b, p, rects, dt);
+    });
+}
+
+extern "C" int pmm_upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld, int64_t row_base,
+                          int64_t col_base) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        fpm::upload(ctx, A, B, ld, row_base, col_base, nullptr);
+    });
+}
+
+extern "C" int pmm_fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int32_t dist) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        fpm::fill_synthetic(ctx, seed_a, seed_b, dist);
+    });
+}
+
+extern "C" int pmm_compute(pmm_ctx* ctx, int32_t zero_c, pmm_stats* stats) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        fpm::compute(ctx, zero_c != 0, stats);
+    });
+}
+
+extern "C" int pmm_download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        fpm::download(ctx, C, ld, row_base, col_base, nullptr);
+    });
+}
+
+extern "C" int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t rows, int64_t cols, void* C_host,
+                                  int64_t ld) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr && C_host != nullptr, "null argument");
+        if (!ctx->have_problem) fpm::fail(FPM_ESTATE, "pmm_download_block before pmm_setup");
+        FPM_CHECK_ARG(rows >= 0 && cols >= 0 && ld >= cols, "bad block shape");
+        if (rows == 0 || cols == 0) return;
+        const int64_t b = ctx->b;
+        const size_t es = ctx->dt == FPM_F64 ? 8 : 4;
+        for (auto& d : ctx->devs) {
+            if (!d.live()) continue;
+            const int64_t R0 = d.rect.row0 * b, C0 = d.rect.col0 * b;
+            if (r0 >= R0 && c0 >= C0 && r0 + rows <= R0 + d.H && c0 + cols <= C0 + d.W) {
+                CU(cudaSetDevice(d.cuda_dev));
+                CU(cudaStreamSynchronize(d.s_comp));
+                const char* src = static_cast<const char*>(d.C) + ((size_t)(r0 - R0) * d.W + (size_t)(c0 - C0)) * es;
+                CU(cudaMemcpy2D(C_host, ld * es, src, d.W * es, cols * es, rows, cudaMemcpyDeviceToHost));
+                return;
+            }
+        }
+        fpm::fail(FPM_EINVAL, "block not inside one local rectangle");
+    });
+}
+
+extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int64_t b, int32_t p,
+                       const colpart_rect* rects, fpm_dtype dt, int64_t ld, int64_t row_base, int64_t col_base,
+                       pmm_stats* stats) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        bool same = ctx->have_problem && ctx->N == N && ctx->b == b && ctx->p == p && ctx->dt == dt;
+        if (same)
+            for (int i = 0; i < p; ++i) {
+                const colpart_rect &x = ctx->rects[i], &y = rects[i];
+                same = same && x.col == y.col && x.row0 == y.row0 && x.col0 == y.col0 && x.h == y.h && x.w == y.w;
+            }
+        if (!same) fpm::setup(ctx, N, b, p, rects, dt);
+        double tu = 0.0, td = 0.0;
+        fpm::upload(ctx, A, B, ld, row_base, col_base, &tu);
+        pmm_stats local;
+        fpm::compute(ctx, false, &local);
+        fpm::download(ctx, C, ld, row_base, col_base, &td);
+        local.t_upload_s = tu;
+        local.t_download_s = td;
+        if (stats) *stats = local;
+    });
+}
+
+extern "C" int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t* sizes,
+                          int32_t nsizes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr, "null ctx");
+        fpm::sample(ctx, dev, dt, b, sizes, nsizes, speeds_out, rel_ci95_out, reps_out);
+    });
+}
+
+// ------------------------------------------------------- kernel-level ABI
+extern "C" int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64_t K, int32_t scheme, void* hi,
+                               void* lo, float* inv_scale, void* stream) {
+    return guarded([&] {
+        FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
+        FPM_CHECK_ARG(scheme == 1 || inv_scale != nullptr, "F16X3 needs inv_scale");
+        fpm::launch_split_rows(src, ld, rows, K, (fpm::SplitScheme)scheme, hi, lo, inv_scale,
+                               static_cast<cudaStream_t>(stream));
+    });
+}
+
+extern "C" int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64_t cols, void* dst,
+                               void* stream) {
+    return guarded([&] {
+        FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "bad dtype");
+        if (dt == FPM_F32)
+            fpm::launch_transpose_f32(static_cast<const float*>(src), ld, rows, cols, static_cast<float*>(dst),
+                                      static_cast<cudaStream_t>(stream));
+        else
+            fpm::launch_transpose_f64(static_cast<const double*>(src), ld, rows, cols, static_cast<double*>(dst),
+                                      static_cast<cudaStream_t>(stream));
+    });
+}
+
+extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
+                                const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
+                                int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, void* stream) {
+    return guarded([&] {
+        FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
+        FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
+        FPM_CHECK_ARG(scheme == 1 || (sa && sb), "F16X3 needs sa and sb");
+        fpm::UpdateArgs a;
+        a.a_hi = a_hi; a.a_lo = a_lo; a.bt_hi = bt_hi; a.bt_lo = bt_lo;
+        a.sa = scheme == 0 ? sa : nullptr;
+        a.sb = scheme == 0 ? sb : nullptr;
+        a.C = C; a.M = M; a.Nc = Nc; a.K = K; a.ldc = ldc;
+        a.scheme = (fpm::SplitScheme)scheme;
+        a.cta_group = cta_group;
+        int dev = 0, sms = 0;
+        CU(cudaGetDevice(&dev));
+        CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
+        a.num_sms = (num_sms > 0 && num_sms < sms) ? num_sms : sms;
+        fpm::launch_update_f32(a, static_cast<cudaStream_t>(stream));
+    });
+}
+
+extern "C" int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
+                                int64_t K, int64_t ldc, void* stream) {
+    return guarded([&] {
+        fpm::launch_update_f64(A, lda, Bt, C, M, Nc, K, ldc, static_cast<cudaStream_t>(stream));
+    });
+}
+
+extern "C" int fpm_k_fill_synthetic(void* dst, int32_t dt, int64_t ld, uint64_t seed, int64_t N, int64_t r0,
+                                    int64_t c0, int64_t rows, int64_t cols, int32_t dist, void* stream) {
+    return guarded([&] {
+        FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "bad dtype");
+        fpm::launch_fill_synthetic(dst, dt == FPM_F64, ld, seed, N, r0, c0, rows, cols, dist,
+                                   static_cast<cudaStream_t>(stream));
+    });
+}

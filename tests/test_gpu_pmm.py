@@ -1,0 +1,172 @@
+"""End-to-end parity of the hot path on the GPU, through the C ABI:
+fpm_partition -> colpart_arrange -> pmm_run (pivot exchange + staging + rank-b
+updates) vs the oracle GEMM; fpm_sample procedure checks; full-size sampled
+parity at the bench configuration."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import fpm as ofpm
+from oracle import gemm as og
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+import paper_conf_cluster_zhongrl12_b200 as pkg  # noqa: E402
+
+
+@pytest.fixture(autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    yield
+
+
+def _models(seed, p):
+    return synth.random_models(np.random.default_rng(seed), p, monotone_time=True, max_m=12)
+
+
+def _run(ctx, N, b, rects, dt, dist=synth.DIST_PM1, seeds=(1, 2)):
+    npdt = np.float32 if dt == pkg.FPM_F32 else np.float64
+    A = synth.rect(seeds[0], N, 0, 0, N, N, dist, npdt)
+    B = synth.rect(seeds[1], N, 0, 0, N, N, dist, npdt)
+    C = np.full((N, N), np.nan, dtype=npdt)
+    st = ctx.run(A, B, C, N, b, rects, dt)
+    return A, B, C, st
+
+
+@pytest.mark.parametrize("dt,tol", [(pkg.FPM_F32, 1e-5), (pkg.FPM_F64, 1e-12)])
+@pytest.mark.parametrize("N,b", [(512, 64), (1024, 128), (768, 256)])
+def test_p1(dt, tol, N, b):
+    with pkg.Context.local([0]) as ctx:
+        A, B, C, st = _run(ctx, N, b, [(0, 0, 0, N // b, N // b)], dt)
+        assert og.rel_fro(C, og.gemm(A, B)) <= tol
+        assert st.iters == N // b and st.t_compute_s > 0 and st.kernel_launches > 0
+
+
+@pytest.mark.parametrize("p", [2, 3, 4, 5])
+@pytest.mark.parametrize("dt", [pkg.FPM_F32, pkg.FPM_F64])
+def test_local_multi_device_parity(p, dt):
+    """p emulated devices on one GPU: FPM partition, arrangement, pivot exchange."""
+    N, b = 768, 64
+    n = N // b
+    models = _models(100 + p, p)
+    d = pkg.fpm_partition(n * n, models)
+    assert d == ofpm.partition(n * n, models)
+    rects = pkg.colpart_arrange(n, d)
+    assert rects == ofpm.arrange(n, d)
+    with pkg.Context.local([0] * p) as ctx:
+        A, B, C, st = _run(ctx, N, b, rects, dt)
+        tol = 1e-5 if dt == pkg.FPM_F32 else 1e-12
+        assert og.rel_fro(C, og.gemm(A, B)) <= tol
+        live = [i for i, r in enumerate(rects) if r[3] * r[4] > 0]
+        assert all(st.per_dev_compute_s[i] > 0 for i in live)
+        if len(live) > 1:
+            assert st.comm_bytes > 0
+
+
+@pytest.mark.parametrize("p", [1, 2, 4, 8])
+def test_integer_inputs_bit_exact_and_p_invariant(p):
+    N, b = 1024, 128
+    n = N // b
+    d = pkg.fpm_partition(n * n, [([1], [1.0 + i % 3])] * p) if p > 1 else [n * n]
+    rects = pkg.colpart_arrange(n, d)
+    ref = None
+    for dt in (pkg.FPM_F32, pkg.FPM_F64):
+        with pkg.Context.local([0] * p) as ctx:
+            A, B, C, _ = _run(ctx, N, b, rects, dt, dist=synth.DIST_INT, seeds=(11, 12))
+        exact = og.gemm(A, B)
+        assert np.array_equal(C.astype(np.float64), exact)
+        ref = exact if ref is None else ref
+
+
+def test_tf32x3_scheme_and_cta_group1():
+    N, b = 1024, 128
+    rects = pkg.colpart_arrange(N // b, [32, 32])
+    for scheme, cg in [(pkg.SCHEME_TF32X3, 2), (pkg.SCHEME_F16X3, 1), (pkg.SCHEME_TF32X3, 1)]:
+        with pkg.Context.local([0, 0]) as ctx:
+            ctx.set_option("f32_scheme", scheme)
+            ctx.set_option("cta_group", cg)
+            A, B, C, _ = _run(ctx, N, b, rects, pkg.FPM_F32)
+            assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+def test_zero_area_device_and_sm_caps():
+    N, b = 512, 64
+    n = N // b
+    d = [n * n - 5, 5, 0]
+    rects = pkg.colpart_arrange(n, d)
+    with pkg.Context.local([0, 0, 0], sm_caps=[64, 16, 8]) as ctx:
+        A, B, C, st = _run(ctx, N, b, rects, pkg.FPM_F32)
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+def test_invalid_arguments_fail_loudly():
+    with pkg.Context.local([0]) as ctx:
+        with pytest.raises(pkg.FpmError):
+            ctx.setup(500, 64, [(0, 0, 0, 7, 7)])        # b does not divide N
+        with pytest.raises(pkg.FpmError):
+            ctx.setup(512, 64, [(0, 0, 0, 8, 7)])        # does not tile
+        with pytest.raises(pkg.FpmError):
+            ctx.compute()                                 # no problem set
+    with pytest.raises(pkg.FpmError):
+        pkg.Context.local([0], sm_caps=[12])              # not a multiple of 8
+
+
+def test_fpm_sample_procedure():
+    """Speed points are positive, meet the CI stop rule or the repetition cap (P:10 (iii))."""
+    with pkg.Context.local([0]) as ctx:
+        sizes = [1, 4, 16, 64]
+        sp, ci, reps = ctx.sample(0, 256, sizes, pkg.FPM_F32)
+        assert all(s > 0 for s in sp)
+        assert all(5 <= r <= 50 for r in reps)
+        assert all(c <= 0.025 or r == 50 for c, r in zip(ci, reps))
+        sp64, _, _ = ctx.sample(0, 64, [1, 4, 9], pkg.FPM_F64)
+        assert all(s > 0 for s in sp64)
+        with pytest.raises(pkg.FpmError):
+            ctx.sample(0, 256, [3])                        # not a perfect square
+
+
+def test_config1_fp64_two_capped_devices():
+    """BASELINE config 1: N=512, b=64, FP64, two devices with SM caps {144, 48}:
+    FPMs from 8 sample sizes -> partition -> arrangement -> multiply."""
+    N, b = 512, 64
+    n = N // b
+    sizes = [m * m for m in range(1, 9)]
+    with pkg.Context.local([0, 0], sm_caps=[144, 48]) as ctx:
+        models = []
+        for dev in range(2):
+            sp, _, _ = ctx.sample(dev, b, sizes, pkg.FPM_F64)
+            models.append((sizes, sp))
+        d = pkg.fpm_partition(n * n, models)
+        assert sum(d) == n * n
+        rects = pkg.colpart_arrange(n, d)
+        A, B, C, _ = _run(ctx, N, b, rects, pkg.FPM_F64, seeds=(1, 2))
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-12
+
+
+@pytest.mark.parametrize("N,b", [(16384, 512), (49152, 1024)])
+def test_full_size_sampled_parity(N, b):
+    """Bench configurations (c3 at p=1, c5 at p=1): synthetic inputs generated on
+    the device by the shared counter-based generator, sampled blocks of C
+    (corners, interior, ragged tile edges) vs the oracle on the same entries."""
+    free, _ = torch.cuda.mem_get_info(0)
+    if free < 3.3 * 3 * N * N * 4:
+        pytest.skip("not enough device memory")
+    n = N // b
+    with pkg.Context.local([0]) as ctx:
+        ctx.setup(N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+        ctx.fill_synthetic(1, 2, pkg.FPM_DIST_PM1)
+        st = ctx.compute(zero_c=True)
+        assert st.t_compute_s > 0
+        rng = np.random.default_rng(N)
+        blocks = [(0, 0), (N - 16, N - 64), (0, N - 64), (N - 16, 0)]
+        blocks += [(int(r), int(c)) for r, c in zip(rng.integers(0, N - 16, 4), rng.integers(0, N - 64, 4))]
+        B_cols = {}
+        for (r0, c0) in blocks:
+            got = ctx.download_block(r0, c0, 16, 64)
+            A_rows = synth.rect(1, N, r0, 0, 16, N)
+            if c0 not in B_cols:
+                B_cols[c0] = synth.rect(2, N, 0, c0, N, 64)
+            ref = og.gemm(A_rows, B_cols[c0])
+            assert og.rel_fro(got, ref) <= 1e-5, (r0, c0, og.rel_fro(got, ref))
