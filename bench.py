@@ -1,0 +1,376 @@
+#!/usr/bin/env python
+"""Benchmark of the FPM-partitioned column-based parallel matrix multiplication.
+
+    python bench.py --gpus N --steps K --warmup W [--impl ours|reference]
+
+One process per GPU (torchrun for N > 1: RANK / WORLD_SIZE / LOCAL_RANK), the
+pivot exchange over NCCL inside libfpmpmm, torch.distributed (gloo) only for the
+control plane (unique id, barriers, max-over-ranks of device times).
+
+Workload (BASELINE.json config 5): N = 49152, b = 1024, FP32,
+square U[-1,1) matrices from the shared counter-based generator, p = N GPUs,
+strong scaling.  A step = fpm_partition + colpart_arrange + pmm_compute (the
+N/b iterations of pivot exchange, staging and rank-b update) on inputs resident
+in HBM; `value` = 2 N^3 K / sum of per-step device times (max over ranks).
+`e2e` = the same through pmm_run on pinned host buffers (H2D + D2H inside).
+`--impl reference` times the CPU oracle (plain triple loop) on a bounded
+sample of the same workload (rank 0 only).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "partitioned GEMM GFLOPS & % tensor peak at 1/2/4/8 B200; FPM load imbalance %"
+UNIT = "GFLOP/s"
+N_DEFAULT, B_DEFAULT = 49152, 1024
+ORACLE_ROWS, ORACLE_COLS = 64, 1024   # bounded sample for the CPU oracle
+
+
+def log(*a):
+    print(*a, file=sys.stderr, flush=True)
+
+
+# ----------------------------------------------------------------- clocks
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, gpu: int):
+        self.gpu = gpu
+        self.rows = []
+        self.proc = None
+
+    def start(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.gpu), f"--query-gpu={self.FIELDS}", "--format=csv,noheader,nounits",
+                 "-lms", "200"], stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.thread = threading.Thread(target=self._read, daemon=True)
+            self.thread.start()
+        except Exception as e:  # pragma: no cover
+            log("clock sampler unavailable:", e)
+            self.proc = None
+
+    def _read(self):
+        for line in self.proc.stdout:
+            parts = [p.strip() for p in line.split(",")]
+            if len(parts) == 7:
+                self.rows.append(parts)
+
+    def stop(self) -> dict:
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        self.proc.terminate()
+        try:
+            self.proc.wait(timeout=5)
+        except Exception:
+            self.proc.kill()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        sms, mx, reasons, power = [], None, set(), []
+        for r in self.rows:
+            try:
+                sms.append(float(r[0]))
+                mx = float(r[1])
+                power.append(float(r[2]))
+            except ValueError:
+                continue
+            for nm, v in zip(names, r[3:]):
+                if v.lower().startswith("active"):
+                    reasons.add(nm)
+        loaded = [s for s, p in zip(sms, power) if p > 200.0] or sms
+        return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": mx,
+                "reasons": sorted(reasons), "samples": len(sms)}
+
+
+# ----------------------------------------------------------------- peaks
+def measured_peaks() -> dict:
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(path):
+        with open(path) as f:
+            d = json.load(f)
+        return {"bf16_burst": d.get("bf16_tflops", 1590.0), "bf16_sustained": d.get("bf16_tflops_sustained", 1400.0),
+                "hbm_gbs": d.get("hbm_gbs", 6650.0), "source": "measured"}
+    return {"bf16_burst": 1590.0, "bf16_sustained": 1400.0, "hbm_gbs": 6650.0, "source": "fallback"}
+
+
+# ----------------------------------------------------------------- oracle
+def oracle_sample(N: int, reps: int = 1):
+    """Time the CPU oracle (plain triple loop, FP64 accumulation) on the block
+    C[0:R, 0:S] = A[0:R, :] B[:, 0:S] of the workload; returns (GFLOP/s, cores, desc)."""
+    import synth
+    from oracle import gemm as og
+    R, S = ORACLE_ROWS, ORACLE_COLS
+    sa, sb = synth.seeds_for_config(4)
+    A = synth.rect(sa, N, 0, 0, R, N)
+    B = synth.rect(sb, N, 0, 0, N, S)
+    og.gemm(A[:2, :64], B[:64, :8])  # build / load outside the timing
+    ts = []
+    for _ in range(reps):
+        t0 = time.perf_counter()
+        og.gemm(A, B)
+        ts.append(time.perf_counter() - t0)
+    t = min(ts)
+    flops = 2.0 * R * S * N
+    desc = (f"C[0:{R},0:{S}] = A[0:{R},:] B[:,0:{S}] of the N={N} workload (K={N}); "
+            f"{flops / 1e9:.2f} GFLOP per step, oracle triple loop (gcc -O2, OpenMP, FP64 accumulation)")
+    return flops / t / 1e9, og.num_threads(), desc, t
+
+
+# ----------------------------------------------------------------- main arms
+def run_reference(args, rank: int):
+    if rank != 0:
+        return
+    N = args.N
+    vals, times = [], []
+    for i in range(args.warmup + args.steps):
+        g, cores, desc, t = oracle_sample(N)
+        if i >= args.warmup:
+            vals.append(g)
+            times.append(t)
+    value = statistics.median(vals)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.median(times),
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic",
+        "config": {"workload": f"c5: N={N}, b={args.b}, FP32 inputs (oracle accumulates in FP64)",
+                   "N": N, "b": args.b, "sample": desc},
+        "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc},
+        "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def run_ours(args, rank: int, world: int, local_rank: int, dist):
+    import numpy as np
+    import torch
+
+    import paper_conf_cluster_zhongrl12_b200 as pkg
+
+    torch.cuda.set_device(local_rank)
+    N, b = args.N, args.b
+    n = N // b
+    p = world
+
+    # ---- context (NCCL over NVLink for N > 1)
+    if world > 1:
+        obj = [pkg.Context.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        ctx = pkg.Context.nccl(rank, world, local_rank, obj[0])
+    else:
+        ctx = pkg.Context.local([local_rank])
+    if args.scheme == "tf32x3":
+        ctx.set_option("f32_scheme", pkg.SCHEME_TF32X3)
+    ctx.set_option("cta_group", args.cta_group)
+
+    # ---- FPMs (offline): sample this GPU's speed function once;
+    # every rank's model is gathered so all ranks partition identically.
+    sizes = [m * m for m in (1, 2, 4, 8, 12, 16)]
+    t0 = time.perf_counter()
+    sp, ci, reps = ctx.sample(rank, b, sizes, pkg.FPM_F32)
+    t_sample = time.perf_counter() - t0
+    models_all = [None] * world
+    if world > 1:
+        dist.all_gather_object(models_all, (sizes, sp))
+    else:
+        models_all = [(sizes, sp)]
+
+    def plan():
+        d = pkg.fpm_partition(n * n, models_all)
+        return d, pkg.colpart_arrange(n, d)
+
+    d, rects = plan()
+    ctx.setup(N, b, rects, pkg.FPM_F32)
+    import synth
+    sa, sb = synth.seeds_for_config(4)   # config 5 (index 4): seeds 5 and 6
+    ctx.fill_synthetic(sa, sb, pkg.FPM_DIST_PM1)
+
+    def barrier():
+        torch.cuda.synchronize()
+        if world > 1:
+            dist.barrier()
+
+    def max_over_ranks(x: float) -> float:
+        if world == 1:
+            return x
+        t = torch.tensor([x], dtype=torch.float64)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        return float(t.item())
+
+    # ---- device-resident steps
+    for _ in range(args.warmup):
+        d, rects = plan()
+        ctx.compute(zero_c=True)
+    barrier()
+    clocks = ClockSampler(local_rank)
+    clocks.start()
+    step_times, upd_times, comp_times, launches, comm = [], [], [], 0, 0
+    wall0 = time.perf_counter()
+    for _ in range(args.steps):
+        d, rects = plan()
+        st = ctx.compute(zero_c=True)
+        step_times.append(max_over_ranks(st.t_compute_s))
+        upd_times.append(st.per_dev_update_s[rank])
+        comp_times.append(st.per_dev_compute_s[rank])
+        launches += st.kernel_launches
+        comm += st.comm_bytes
+    barrier()
+    wall = time.perf_counter() - wall0
+    clk = clocks.stop()
+    total_t = sum(step_times)
+    flops = 2.0 * N ** 3
+    value = flops * args.steps / total_t / 1e9
+
+    # per-rank computation time (Fig. 6 metric) -> measured imbalance
+    comp_all = [statistics.median(comp_times)]
+    if world > 1:
+        comp_all = [None] * world
+        dist.all_gather_object(comp_all, statistics.median(comp_times))
+    live = [c for c, r in zip(comp_all, rects) if r[3] * r[4] > 0]
+    imb_meas = max(live) / (sum(live) / len(live)) - 1.0 if live else 0.0
+    areas = [r[3] * r[4] for r in rects]
+    pred_t = [a / pkg.fpm_model_speed(m, a) if a > 0 else 0.0 for a, m in zip(areas, models_all)]
+    live_t = [t for t in pred_t if t > 0]
+    imb_pred = max(live_t) / (sum(live_t) / len(live_t)) - 1.0 if live_t else 0.0
+
+    # ---- roofline of the dominant kernel (rank-b update): algorithmic flops per
+    # launch = 2 H W b, over the mean launch duration (CUDA events on its stream).
+    peaks = measured_peaks()
+    r = rects[rank]
+    H, W = r[3] * b, r[4] * b
+    upd_mean = statistics.median(upd_times) / n
+    achieved = 2.0 * H * W * b / upd_mean / 1e12 if upd_mean > 0 else 0.0
+    mma_per_mac = 3.0  # F16X3 and TF32X3 both issue three tensor-core products per FP32 MAC
+    dense_peak = peaks["bf16_sustained"] if args.scheme == "f16x3" else peaks["bf16_sustained"] / 2.0
+    peak = dense_peak / mma_per_mac
+    roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
+                "frac": achieved / peak if peak else None, "traffic": args.traffic,
+                "peak_basis": (f"{'fp16' if args.scheme == 'f16x3' else 'tf32'} dense tensor peak "
+                               f"({peaks['source']} {dense_peak:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC"),
+                "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None}
+
+    # ---- end to end through pmm_run with pinned host buffers
+    e2e = None
+    if args.e2e_steps > 0:
+        try:
+            e2e = run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier)
+        except Exception as ex:  # report, do not hide
+            log("e2e failed:", repr(ex))
+            e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:200]}
+
+    cpu = None
+    if rank == 0 and not args.no_cpu_baseline:
+        g, cores, desc, _ = oracle_sample(N)
+        cpu = {"value": g, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
+            "warmup": args.warmup, "ms_per_step": 1e3 * total_t / args.steps, "higher_is_better": True,
+            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "config": {
+                "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
+                "N": N, "b": b, "p": p, "partition": d, "rects": rects,
+                "f32_scheme": args.scheme, "cta_group": args.cta_group,
+                "l2": "inputs larger than L2 (A, B, C 9.7 GB each)",
+                "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
+                "imbalance_pct_measured": 100.0 * imb_meas, "imbalance_pct_predicted": 100.0 * imb_pred,
+                "fpm_sample_s": t_sample, "fpm_sizes": sizes,
+                "comm_bytes_per_step": comm // max(1, args.steps),
+                "wall_s_timed_region": wall,
+            },
+            "roofline": roofline,
+            "cpu_baseline": cpu,
+            "e2e": e2e,
+            "gpu_launches": launches,
+            "clocks": clk,
+        }
+        print(json.dumps(line), flush=True)
+    ctx.close()
+
+
+def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier):
+    import torch
+
+    import paper_conf_cluster_zhongrl12_b200 as pkg
+    N, b = args.N, args.b
+    r = rects[rank]
+    H, W = r[3] * b, r[4] * b
+    R0, C0 = r[1] * b, r[2] * b
+    if H * W == 0:
+        return None
+    # host windows = this rank's rectangle (generated on the device once, untimed)
+    hA = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
+    hB = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
+    hC = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
+    tmp = torch.empty((H, W), dtype=torch.float32, device="cuda")
+    pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 5, N, R0, C0, H, W)  # seeds_for_config(4)
+    hA.copy_(tmp)
+    pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 6, N, R0, C0, H, W)
+    hB.copy_(tmp)
+    del tmp
+    torch.cuda.empty_cache()
+    barrier()
+    ts = []
+    for i in range(args.e2e_steps + 1):
+        t0 = time.perf_counter()
+        st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32, ld=W, row_base=R0, col_base=C0)
+        t_host = time.perf_counter() - t0
+        t_dev = st.t_upload_s + st.t_compute_s + st.t_download_s
+        if i > 0:  # first call is a warm-up
+            ts.append(max_over_ranks(max(t_host, t_dev)))
+    t = statistics.median(ts)
+    return {"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
+            "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
+            "upload_s": st.t_upload_s, "download_s": st.t_download_s}
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
+    ap.add_argument("--N", type=int, default=N_DEFAULT)
+    ap.add_argument("--b", type=int, default=B_DEFAULT)
+    ap.add_argument("--scheme", choices=["f16x3", "tf32x3"], default="f16x3")
+    ap.add_argument("--cta-group", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--traffic", type=float, default=None,
+                    help="dram bytes per update launch from an ncu --set full capture")
+    args = ap.parse_args()
+    if args.N % args.b:
+        ap.error("b must divide N")
+
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    dist = None
+    if world > 1:
+        import torch.distributed as dist
+        os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        dist.init_process_group("gloo", rank=rank, world_size=world)
+    if args.impl == "reference":
+        run_reference(args, rank)
+    else:
+        run_ours(args, rank, world, local_rank, dist)
+    if dist is not None:
+        dist.barrier()
+        dist.destroy_process_group()
+
+
+if __name__ == "__main__":
+    main()

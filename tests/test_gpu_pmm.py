@@ -69,7 +69,7 @@ def test_local_multi_device_parity(p, dt):
 def test_integer_inputs_bit_exact_and_p_invariant(p):
     N, b = 1024, 128
     n = N // b
-    d = pkg.fpm_partition(n * n, [([1], [1.0 + i % 3])] * p) if p > 1 else [n * n]
+    d = pkg.fpm_partition(n * n, [([1], [1.0 + i % 3]) for i in range(p)])
     rects = pkg.colpart_arrange(n, d)
     ref = None
     for dt in (pkg.FPM_F32, pkg.FPM_F64):
