@@ -179,7 +179,10 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     # every rank's model is gathered so all ranks partition identically.
     sizes = [m * m for m in (1, 2, 4, 8, 12, 16)]
     t0 = time.perf_counter()
-    sp, ci, reps = ctx.sample(rank, b, sizes, pkg.FPM_F32)
+    if args.no_sample:  # profiling runs: identical constant models, predictable launch order
+        sp = [1.0] * len(sizes)
+    else:
+        sp, ci, reps = ctx.sample(rank, b, sizes, pkg.FPM_F32)
     t_sample = time.perf_counter() - t0
     models_all = [None] * world
     if world > 1:
@@ -349,6 +352,7 @@ def main():
     ap.add_argument("--cta-group", type=int, default=2)
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")
     ap.add_argument("--traffic", type=float, default=None,
                     help="dram bytes per update launch from an ncu --set full capture")
     args = ap.parse_args()

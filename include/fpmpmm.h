@@ -142,8 +142,9 @@ int colpart_plan_step(int64_t n, int32_t p, const colpart_rect* rects, int64_t k
 
 /* Single-process context driving p "devices".  Device i runs on CUDA ordinal
  * cuda_devices[i]; several devices may share one GPU.  sm_caps (nullable):
- * 0 = the whole GPU, else a cap on SMs (multiple of 8, >= 8) realised with a
- * green context (heterogeneity emulation, BASELINE north_star).  Pivot
+ * 0 = the whole GPU, else a cap on SMs (even, >= 2) for heterogeneity
+ * emulation (BASELINE north_star): the persistent rank-b update kernel, which
+ * holds one SM per CTA, runs with a grid of `cap` CTAs.  Pivot
  * transfers between devices are device-to-device copies on the receivers'
  * communication streams.  Errors: FPM_EINVAL, FPM_ECUDA, FPM_EUNSUPPORTED. */
 int pmm_create_local(int32_t p, const int32_t* cuda_devices, const int32_t* sm_caps,
@@ -186,8 +187,9 @@ int pmm_fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int32_t d
 
 /* Run the N/b iterations on resident data: per iteration pivot exchange
  * (look-ahead one iteration, on communication streams) and the rank-b update
- * C_i += A(b) x B(b) on each device.  Starts from C_i = 0 (zeroed by
- * upload / fill / the previous download when zero_c != 0).  Blocks until done. */
+ * C_i += A(b) x B(b) on each device.  Iteration 0 writes C_i = A(0) B(0)
+ * (no zeroing pass), so every call leaves C_i = (A B)_i.  zero_c is accepted
+ * for compatibility and has no effect.  Blocks until done. */
 int pmm_compute(pmm_ctx* ctx, int32_t zero_c, pmm_stats* stats);
 
 /* Copy this process's C_i into a host window (same convention as upload). */
@@ -199,9 +201,13 @@ int pmm_download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t co
 int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t rows, int64_t cols, void* C_host,
                        int64_t ld);
 
-/* Whole call on host matrices: setup (if the problem changed) + upload +
- * compute + download.  A, B, C are host windows as for pmm_upload.  Upload and
- * download times are reported in stats. */
+/* Whole call on host matrices: setup (if the problem changed), then the N/b
+ * iterations with the inputs streamed from the host windows (block-column k of
+ * A and block-row k of B are copied host -> device on the communication stream
+ * just ahead of iteration k, overlapping earlier updates), then the download
+ * of C.  A, B, C are host windows as for pmm_upload (pinned memory gives
+ * asynchronous copies).  stats: t_compute_s includes the streamed upload,
+ * t_upload_s = time until the last panel landed, t_download_s. */
 int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int64_t b,
             int32_t p, const colpart_rect* rects, fpm_dtype dt, int64_t ld,
             int64_t row_base, int64_t col_base, pmm_stats* stats);
@@ -237,6 +243,12 @@ int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value);
 int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64_t K, int32_t scheme,
                     void* hi, void* lo, float* inv_scale, void* stream);
 
+/* The same split applied to the transpose of a B pivot row: src is K x W
+ * (row stride ld), hi/lo receive W x K (K-major), inv_scale[W] the per-column
+ * scales of src.  One pass, no shared memory.  K % 8 == 0, W % 4 == 0. */
+int fpm_k_split_cols_f32(const float* src, int64_t ld, int64_t K, int64_t W, int32_t scheme,
+                         void* hi, void* lo, float* inv_scale, void* stream);
+
 /* dst (cols x rows, contiguous) = transpose of src (rows x cols, row stride
  * ld); dt = FPM_F32 or FPM_F64.  Used for the K-major B pivot panel. */
 int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64_t cols, void* dst,
@@ -246,15 +258,17 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * given as Bt (Nc x K, K-major), operands as produced by fpm_k_split_f32 with
  * the same scheme (sa / sb: inverse row scales of A and Bt for F16X3, NULL
  * for TF32X3).  cta_group 1 or 2; num_sms = persistent grid (0 = all SMs).
+ * accumulate = 0 writes C = A x B without reading C.
  * Requires K % 8 == 0, ldc % 4 == 0. */
 int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
                      const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
-                     int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, void* stream);
+                     int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms,
+                     int32_t accumulate, void* stream);
 
-/* Rank-b update in FP64 on DMMA: C (M x Nc, ldc) += A (M x K, lda) x Bt^T,
- * Bt (Nc x K). */
+/* Rank-b update in FP64 on DMMA: C (M x Nc, ldc) (+)= A (M x K, lda) x Bt^T,
+ * Bt (Nc x K); accumulate = 0 overwrites C. */
 int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                     int64_t K, int64_t ldc, void* stream);
+                     int64_t K, int64_t ldc, int32_t accumulate, void* stream);
 
 /* Fill a rows x cols window (ld elements) of the seeded global N x N matrix
  * starting at global (r0, c0); dt = FPM_F32 or FPM_F64; dist = fpm_dist. */

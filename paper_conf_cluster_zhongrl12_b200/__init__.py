@@ -191,19 +191,25 @@ def k_split_f32(src, ld, rows, K, scheme, hi, lo, inv_scale=None, stream=None):
                               _lib._ptr(inv_scale), _stream(stream)))
 
 
+def k_split_cols_f32(src, ld, K, W, scheme, hi, lo, inv_scale=None, stream=None):
+    check(lib.fpm_k_split_cols_f32(_lib._ptr(src), ld, K, W, scheme, _lib._ptr(hi), _lib._ptr(lo),
+                                   _lib._ptr(inv_scale), _stream(stream)))
+
+
 def k_transpose(src, dtype, ld, rows, cols, dst, stream=None):
     check(lib.fpm_k_transpose(_lib._ptr(src), dtype, ld, rows, cols, _lib._ptr(dst), _stream(stream)))
 
 
 def k_update_f32(a_hi, a_lo, bt_hi, bt_lo, sa, sb, C, M, Nc, K, ldc, scheme=SCHEME_F16X3, cta_group=2,
-                 num_sms=0, stream=None):
+                 num_sms=0, accumulate=True, stream=None):
     check(lib.fpm_k_update_f32(_lib._ptr(a_hi), _lib._ptr(a_lo), _lib._ptr(bt_hi), _lib._ptr(bt_lo),
                                _lib._ptr(sa), _lib._ptr(sb), _lib._ptr(C), M, Nc, K, ldc, scheme, cta_group,
-                               num_sms, _stream(stream)))
+                               num_sms, 1 if accumulate else 0, _stream(stream)))
 
 
-def k_update_f64(A, lda, Bt, C, M, Nc, K, ldc, stream=None):
-    check(lib.fpm_k_update_f64(_lib._ptr(A), lda, _lib._ptr(Bt), _lib._ptr(C), M, Nc, K, ldc, _stream(stream)))
+def k_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate=True, stream=None):
+    check(lib.fpm_k_update_f64(_lib._ptr(A), lda, _lib._ptr(Bt), _lib._ptr(C), M, Nc, K, ldc,
+                               1 if accumulate else 0, _stream(stream)))
 
 
 def k_fill_synthetic(dst, dtype, ld, seed, N, r0, c0, rows, cols, dist=FPM_DIST_PM1, stream=None):

@@ -27,6 +27,7 @@ struct UpdateArgs {
     SplitScheme scheme;
     int cta_group;      // 1 or 2
     int num_sms;        // SMs the persistent grid may use
+    bool accumulate = true;  // false: C = A . Bt^T (no read of C)
 };
 
 // C += A . Bt^T  (the rank-b update)
@@ -38,6 +39,11 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st);
 void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, SplitScheme s, void* hi,
                        void* lo, float* inv_scale, cudaStream_t st);
 
+// B pivot row src (K x W, row stride ld) -> split halves of its transpose
+// (W x K, K-major), per-row (= per-column of src) inverse scales for F16X3.
+void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,
+                       float* inv_scale, cudaStream_t st);
+
 // dst (cols x rows, K-major) = transpose of src (rows x cols, ld).
 void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t cols, float* dst,
                           cudaStream_t st);
@@ -46,7 +52,7 @@ void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t c
 
 // C (M x Nc, ldc) += A (M x K, lda) . Bt^T, Bt (Nc x K), FP64 on DMMA.
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                       int64_t K, int64_t ldc, cudaStream_t st);
+                       int64_t K, int64_t ldc, bool accumulate, cudaStream_t st);
 
 // Seeded counter-based generator (same bits as synth/__init__.py).
 void launch_fill_synthetic(void* dst, bool f64, int64_t ld, uint64_t seed, int64_t N, int64_t r0, int64_t c0,

@@ -85,6 +85,75 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
     }
 }
 
+// B pivot row (K rows x W cols, row stride ld) -> K-major operand halves of its
+// transpose (W rows x K), split as in split_rows_*.  No shared memory (so it can
+// co-reside with the persistent update kernel): a warp owns 128 columns, lane
+// l columns 4l..4l+3; pass 1 takes the column maxima (F16X3), pass 2 re-reads
+// 8 rows at a time (coalesced float4) and writes 16 B of each of its 4 output
+// rows per half.
+template <bool F16>
+__global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
+                                                    void* __restrict__ hi, void* __restrict__ lo,
+                                                    float* __restrict__ inv_scale) {
+    const int64_t col0 = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 128 + (threadIdx.x % 32) * 4;
+    if (col0 >= W) return;
+    float scale[4] = {1.f, 1.f, 1.f, 1.f};
+    if constexpr (F16) {
+        float m[4] = {0.f, 0.f, 0.f, 0.f};
+        for (int64_t r = 0; r < K; ++r) {
+            const float4 v = *reinterpret_cast<const float4*>(src + r * ld + col0);
+            m[0] = fmaxf(m[0], fabsf(v.x));
+            m[1] = fmaxf(m[1], fabsf(v.y));
+            m[2] = fmaxf(m[2], fabsf(v.z));
+            m[3] = fmaxf(m[3], fabsf(v.w));
+        }
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            int e = 0;
+            if (m[c] > 0.0f) frexpf(m[c], &e);
+            int s = (m[c] > 0.0f) ? 15 - e : 0;
+            s = s < -126 ? -126 : (s > 127 ? 127 : s);
+            scale[c] = ldexpf(1.0f, s);
+            inv_scale[col0 + c] = ldexpf(1.0f, -s);
+        }
+    }
+    for (int64_t r0 = 0; r0 < K; r0 += 8) {
+        float x[8][4];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const float4 v = *reinterpret_cast<const float4*>(src + (r0 + i) * ld + col0);
+            x[i][0] = v.x; x[i][1] = v.y; x[i][2] = v.z; x[i][3] = v.w;
+        }
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            if constexpr (F16) {
+                __align__(16) __half h[8], l[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const float xs = x[i][c] * scale[c];
+                    h[i] = __float2half_rn(xs);
+                    l[i] = __float2half_rn(xs - __half2float(h[i]));
+                }
+                *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + (col0 + c) * K + r0) = *reinterpret_cast<uint4*>(h);
+                *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + (col0 + c) * K + r0) = *reinterpret_cast<uint4*>(l);
+            } else {
+                __align__(16) float h[8], l[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    h[i] = tf32_rna(x[i][c]);
+                    l[i] = tf32_rna(x[i][c] - h[i]);
+                }
+                float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + (col0 + c) * K + r0);
+                float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + (col0 + c) * K + r0);
+                hp[0] = *reinterpret_cast<float4*>(h);
+                hp[1] = *reinterpret_cast<float4*>(h + 4);
+                lp[0] = *reinterpret_cast<float4*>(l);
+                lp[1] = *reinterpret_cast<float4*>(l + 4);
+            }
+        }
+    }
+}
+
 template <class T>
 __global__ void __launch_bounds__(256) transpose_k(const T* __restrict__ src, int64_t ld, int64_t rows,
                                                    int64_t cols, T* __restrict__ dst) {
@@ -128,7 +197,8 @@ __global__ void __launch_bounds__(256) fill_k(T* dst, int64_t ld, uint64_t seed,
 // 4 warps of 32 x 32, K staged through shared memory in steps of 16.
 __global__ void __launch_bounds__(128) update_f64_k(const double* __restrict__ A, int64_t lda,
                                                     const double* __restrict__ Bt, double* __restrict__ C,
-                                                    int64_t M, int64_t Nc, int64_t K, int64_t ldc) {
+                                                    int64_t M, int64_t Nc, int64_t K, int64_t ldc,
+                                                    int accumulate) {
     __shared__ double As[64][17];
     __shared__ double Bs[64][17];
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
@@ -173,7 +243,7 @@ __global__ void __launch_bounds__(128) update_f64_k(const double* __restrict__ A
             for (int h = 0; h < 2; ++h) {
                 const int64_t gm = m0 + wm + i * 8 + lane / 4;
                 const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4) + h;
-                if (gm < M && gn < Nc) C[gm * ldc + gn] += acc[i][j][h];
+                if (gm < M && gn < Nc) C[gm * ldc + gn] = (accumulate ? C[gm * ldc + gn] : 0.0) + acc[i][j][h];
             }
 }
 
@@ -210,6 +280,20 @@ void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, Sp
     }
 }
 
+void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,
+                       float* inv_scale, cudaStream_t st) {
+    if (K <= 0 || W <= 0) return;
+    FPM_CHECK_ARG(K % 8 == 0 && W % 4 == 0 && ld % 4 == 0, "split_cols: K % 8, W % 4, ld % 4 must be 0");
+    const unsigned blocks = (unsigned)((W + 1023) / 1024);  // 8 warps x 128 columns
+    if (s == SplitScheme::F16X3) {
+        FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
+        split_cols_k<true><<<blocks, 256, 0, st>>>(src, ld, K, W, hi, lo, inv_scale);
+    } else {
+        split_cols_k<false><<<blocks, 256, 0, st>>>(src, ld, K, W, hi, lo, inv_scale);
+    }
+    check_launch("split_cols");
+}
+
 void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t cols, float* dst, cudaStream_t st) {
     if (rows <= 0 || cols <= 0) return;
     dim3 grid((unsigned)((cols + 31) / 32), (unsigned)((rows + 31) / 32));
@@ -226,10 +310,10 @@ void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t c
 }
 
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                       int64_t K, int64_t ldc, cudaStream_t st) {
+                       int64_t K, int64_t ldc, bool accumulate, cudaStream_t st) {
     if (M <= 0 || Nc <= 0 || K <= 0) return;
     dim3 grid((unsigned)((Nc + 63) / 64), (unsigned)((M + 63) / 64));
-    update_f64_k<<<grid, 128, 0, st>>>(A, lda, Bt, C, M, Nc, K, ldc);
+    update_f64_k<<<grid, 128, 0, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
     check_launch("update_f64");
 }
 

@@ -58,6 +58,7 @@ struct UpdParams {
     int tiles_m, tiles_n, num_tiles;
     const float* sa;  // per-row inverse scales of A (F16X3) or nullptr
     const float* sb;  // per-column inverse scales of B (F16X3) or nullptr
+    int load_c;       // 1: C += A B^T (read-modify-write), 0: C = A B^T (first iteration)
 };
 
 // Grouped raster over tiles so concurrently running CTAs share A / B tiles in L2.
@@ -213,7 +214,7 @@ __global__ void __launch_bounds__(192, 1)
             const int n0 = tn * BN;
             const int acc = it & 1;
             const uint32_t acc_par = (it >> 1) & 1;
-            if (e == 0) {
+            if (e == 0 && P.load_c) {
                 ptx::bulk_wait_read0();
                 for (int c = 0; c < 2 && c < Cfg::N_CHUNKS; ++c) {
                     ptx::mbar_arrive_expect_tx(&cfull[c], Cfg::C_CHUNK_BYTES);
@@ -248,13 +249,21 @@ __global__ void __launch_bounds__(192, 1)
                         v[j] *= sa * sbj;
                     }
                 }
-                ptx::mbar_wait(&cfull[buf], (cpar >> buf) & 1u);
-                cpar ^= 1u << buf;
+                if (P.load_c) {
+                    ptx::mbar_wait(&cfull[buf], (cpar >> buf) & 1u);
+                    cpar ^= 1u << buf;
+                } else {
+                    // overwrite (first iteration, C = A(0) B(0)): only wait until the
+                    // store that last used this buffer has read it
+                    if (e == 0) ptx::bulk_wait_read1();
+                    ptx::named_bar_sync(1, 128);
+                }
                 uint8_t* rowp = cbuf + buf * Cfg::C_CHUNK_BYTES + r * 128;
 #pragma unroll
                 for (int j = 0; j < 8; ++j) {
                     float4* p4 = reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4));
-                    float4 cv = *p4;
+                    float4 cv = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (P.load_c) cv = *p4;
                     cv.x += v[4 * j + 0];
                     cv.y += v[4 * j + 1];
                     cv.z += v[4 * j + 2];
@@ -266,7 +275,7 @@ __global__ void __launch_bounds__(192, 1)
                 if (e == 0) {
                     ptx::tma_store_2d(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0);
                     ptx::bulk_commit();
-                    if (c + 2 < Cfg::N_CHUNKS) {
+                    if (P.load_c && c + 2 < Cfg::N_CHUNKS) {
                         ptx::bulk_wait_read0();
                         ptx::mbar_arrive_expect_tx(&cfull[buf], Cfg::C_CHUNK_BYTES);
                         ptx::tma_load_2d(cbuf + buf * Cfg::C_CHUNK_BYTES, &tmC, &cfull[buf], n0 + 32 * (c + 2), m0,
@@ -344,6 +353,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.num_tiles = P.tiles_m * P.tiles_n;
     P.sa = a.sa;
     P.sb = a.sb;
+    P.load_c = a.accumulate ? 1 : 0;
     auto kern = update_kernel<CG, TF32, BN, STAGES>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;

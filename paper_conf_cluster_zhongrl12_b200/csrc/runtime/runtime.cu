@@ -48,7 +48,7 @@ struct Device {
     cudaStream_t s_comp = nullptr, s_comm = nullptr;
     cudaEvent_t ev_ready[2] = {}, ev_free[2] = {};
     cudaEvent_t ev_start = nullptr, ev_stop = nullptr, ev_io0 = nullptr, ev_io1 = nullptr;
-    std::vector<cudaEvent_t> ev_pack0, ev_pack1, ev_upd0, ev_upd1;
+    std::vector<cudaEvent_t> ev_pack0, ev_pack1, ev_upd0, ev_upd1, ev_up;
 
     // problem state
     colpart_rect rect{-1, 0, 0, 0, 0};
@@ -108,7 +108,7 @@ void free_problem(Device& d) {
     cudaSetDevice(d.cuda_dev);
     for (void* p : d.allocs) cudaFree(p);
     d.allocs.clear();
-    for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1}) {
+    for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1, &d.ev_up}) {
         for (cudaEvent_t e : *v) cudaEventDestroy(e);
         v->clear();
     }
@@ -126,8 +126,8 @@ void init_device(Device& d) {
     int sms = 0;
     CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d.cuda_dev));
     if (d.sm_cap != 0) {
-        if (d.sm_cap < 8 || d.sm_cap % 8 != 0 || d.sm_cap > sms)
-            fail(FPM_EUNSUPPORTED, "SM cap %d not achievable (multiple of 8 in [8, %d])", d.sm_cap, sms);
+        if (d.sm_cap < 2 || d.sm_cap % 2 != 0 || d.sm_cap > sms)
+            fail(FPM_EUNSUPPORTED, "SM cap %d not achievable (even, in [2, %d]: CTA pairs)", d.sm_cap, sms);
         d.num_sms = d.sm_cap;
     } else {
         d.num_sms = sms;
@@ -212,7 +212,7 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         for (int s = 0; s < 2; ++s) {
             d.a_recv[s] = dalloc(d, (size_t)d.H * b * es);
             d.b_recv[s] = dalloc(d, (size_t)b * d.W * es);
-            d.bt[s] = dalloc(d, (size_t)d.W * b * es);
+            if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * b * es);
             if (dt == FPM_F32) {
                 d.a_hi[s] = dalloc(d, (size_t)d.H * b * op);
                 d.a_lo[s] = dalloc(d, (size_t)d.H * b * op);
@@ -222,7 +222,7 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
                 d.sb[s] = static_cast<float*>(dalloc(d, (size_t)d.W * sizeof(float)));
             }
         }
-        for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1}) {
+        for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1, &d.ev_up}) {
             v->resize(n);
             for (auto& e : *v) CU(cudaEventCreate(&e));
         }
@@ -253,8 +253,38 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
 // ------------------------------------------------------------ iteration parts
 ncclDataType_t nccl_dtype(fpm_dtype dt) { return dt == FPM_F64 ? ncclFloat64 : ncclFloat32; }
 
+// Host windows streamed into the resident rectangles during the k-loop
+// (pmm_run): block-column k of A and block-row k of B are copied just before
+// iteration k needs them, so host->device traffic overlaps earlier updates.
+struct HostSrc {
+    const void* A;
+    const void* B;
+    int64_t ld, row_base, col_base;
+};
+
+void issue_upload(pmm_ctx* ctx, Device& d, int64_t k, const HostSrc& h) {
+    const size_t es = esize(ctx->dt);
+    const int64_t b = ctx->b;
+    const colpart_rect& r = d.rect;
+    CU(cudaSetDevice(d.cuda_dev));
+    const int64_t R0 = r.row0 * b - h.row_base, C0 = r.col0 * b - h.col_base;
+    if (r.col0 <= k && k < r.col0 + r.w) {
+        const int64_t c = k - r.col0;
+        const char* src = static_cast<const char*>(h.A) + ((size_t)R0 * h.ld + (size_t)(C0 + c * b)) * es;
+        char* dst = static_cast<char*>(d.A) + (size_t)c * d.H * b * es;
+        CU(cudaMemcpy2DAsync(dst, b * es, src, h.ld * es, b * es, d.H, cudaMemcpyHostToDevice, d.s_comm));
+    }
+    if (r.row0 <= k && k < r.row0 + r.h) {
+        const int64_t rr = k - r.row0;
+        const char* src = static_cast<const char*>(h.B) + ((size_t)(R0 + rr * b) * h.ld + (size_t)C0) * es;
+        char* dst = static_cast<char*>(d.B) + (size_t)rr * b * d.W * es;
+        CU(cudaMemcpy2DAsync(dst, d.W * es, src, h.ld * es, d.W * es, b, cudaMemcpyHostToDevice, d.s_comm));
+    }
+    CU(cudaEventRecord(d.ev_up[k], d.s_comm));
+}
+
 // Exchange + staging of iteration k on device d's comm stream.
-int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use) {
+int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use, bool streamed) {
     const size_t es = esize(ctx->dt);
     const int64_t b = ctx->b;
     int64_t bytes = 0;
@@ -278,6 +308,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use)
                 const char* src = static_cast<const char*>(q->A) +
                                   ((size_t)(k - qr.col0) * q->H * b + (size_t)(m.begin - qr.row0) * b * b) * es;
                 char* dst = static_cast<char*>(d.a_recv[slot]) + (size_t)(m.begin - r.row0) * b * b * es;
+                if (streamed) CU(cudaStreamWaitEvent(d.s_comm, q->ev_up[k], 0));
                 CU(cudaMemcpyAsync(dst, src, cnt * es, cudaMemcpyDefault, d.s_comm));
                 bytes += (int64_t)(cnt * es);
             }
@@ -296,6 +327,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use)
                 Device* o = local_dev(ctx, m.src);
                 const colpart_rect& orr = ctx->rects[m.src];
                 const char* src = static_cast<const char*>(o->B) + (size_t)(k - orr.row0) * b * o->W * es;
+                if (streamed) CU(cudaStreamWaitEvent(d.s_comm, o->ev_up[k], 0));
                 CU(cudaMemcpyAsync(d.b_recv[slot], src, (size_t)b * d.W * es, cudaMemcpyDefault, d.s_comm));
                 bytes += (int64_t)((size_t)b * d.W * es);
             }
@@ -337,9 +369,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use)
         const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
         launch_split_rows(static_cast<const float*>(a_src), b, d.H, b, sch, d.a_hi[slot], d.a_lo[slot], d.sa[slot],
                           d.s_comm);
-        launch_transpose_f32(static_cast<const float*>(b_src), d.W, b, d.W, static_cast<float*>(d.bt[slot]),
-                             d.s_comm);
-        launch_split_rows(static_cast<const float*>(d.bt[slot]), b, d.W, b, sch, d.b_hi[slot], d.b_lo[slot],
+        launch_split_cols(static_cast<const float*>(b_src), d.W, b, d.W, sch, d.b_hi[slot], d.b_lo[slot],
                           d.sb[slot], d.s_comm);
     } else {
         d.a_op[slot] = a_src;
@@ -372,22 +402,24 @@ void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
         a.scheme = (SplitScheme)ctx->f32_scheme;
         a.cta_group = ctx->cta_group;
         a.num_sms = d.num_sms;
+        a.accumulate = k != 0;  // iteration 0 writes C = A(0) B(0): no zeroing, no read of C
         launch_update_f32(a, d.s_comp);
     } else {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
-                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, d.s_comp);
+                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k != 0, d.s_comp);
     }
     CU(cudaEventRecord(d.ev_upd1[k], d.s_comp));
     CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
 }
 
-void compute(pmm_ctx* ctx, bool zero_c, pmm_stats* st) {
+// The N/b iterations.  Iteration 0 writes C_i = A(0) B(0), so C needs no
+// zeroing.  With `host` set, the pivot panels are streamed from host memory one
+// iteration ahead of their use (pmm_run).
+void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
-    const size_t es = esize(ctx->dt);
     for (auto& d : ctx->devs) {
         if (!d.live()) continue;
         CU(cudaSetDevice(d.cuda_dev));
-        if (zero_c) CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
         CU(cudaStreamSynchronize(d.s_comp));
         CU(cudaStreamSynchronize(d.s_comm));
     }
@@ -396,15 +428,19 @@ void compute(pmm_ctx* ctx, bool zero_c, pmm_stats* st) {
         CU(cudaEventRecord(d.ev_start, d.s_comp));
         CU(cudaStreamWaitEvent(d.s_comm, d.ev_start, 0));
     }
+    const bool streamed = host != nullptr;
     int64_t bytes = 0, launches = 0;
-    const int per_iter = ctx->dt == FPM_F32 ? 4 : 2;
+    const int per_iter = ctx->dt == FPM_F32 ? 3 : 2;  // split A, split B^T, update | transpose, update
     for (int64_t k = 0; k < ctx->n; ++k) {
         const int slot = (int)(k & 1);
+        if (streamed)
+            for (auto& d : ctx->devs)
+                if (d.live()) issue_upload(ctx, d, k, *host);
         if (ctx->nccl_mode) {
             // every rank takes part in the NCCL calls, live or not
             Device& d = ctx->devs[0];
             if (d.live()) {
-                bytes += issue_comm(ctx, d, k, slot, k < 2);
+                bytes += issue_comm(ctx, d, k, slot, k < 2, streamed);
                 issue_update(ctx, d, k, slot);
                 launches += per_iter;
             } else {
@@ -414,7 +450,7 @@ void compute(pmm_ctx* ctx, bool zero_c, pmm_stats* st) {
             continue;
         }
         for (auto& d : ctx->devs)
-            if (d.live()) bytes += issue_comm(ctx, d, k, slot, k < 2);
+            if (d.live()) bytes += issue_comm(ctx, d, k, slot, k < 2, streamed);
         for (auto& d : ctx->devs)
             if (d.live()) {
                 issue_update(ctx, d, k, slot);
@@ -435,6 +471,12 @@ void compute(pmm_ctx* ctx, bool zero_c, pmm_stats* st) {
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->t_compute_s = t_max;
+        if (streamed) {
+            double tu = 0.0;  // until the last host->device panel landed
+            for (auto& d : ctx->devs)
+                if (d.live()) tu = std::max(tu, (double)elapsed_ms(d.ev_start, d.ev_up[ctx->n - 1]) * 1e-3);
+            st->t_upload_s = tu;
+        }
         st->iters = ctx->n;
         st->comm_bytes = bytes;
         st->kernel_launches = launches;
@@ -623,8 +665,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         auto run = [&]() {
             if (dt == FPM_F32) {
                 launch_split_rows(static_cast<const float*>(Ap), b, Lx, b, sch, ah, al, sa, s);
-                launch_transpose_f32(static_cast<const float*>(Bp), L, b, Lx, static_cast<float*>(Bt), s);
-                launch_split_rows(static_cast<const float*>(Bt), b, Lx, b, sch, bh, bl, sb, s);
+                launch_split_cols(static_cast<const float*>(Bp), L, b, Lx, sch, bh, bl, sb, s);
                 UpdateArgs a;
                 a.a_hi = ah; a.a_lo = al; a.bt_hi = bh; a.bt_lo = bl;
                 a.sa = sch == SplitScheme::F16X3 ? sa : nullptr;
@@ -638,7 +679,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             } else {
                 launch_transpose_f64(static_cast<const double*>(Bp), L, b, Lx, static_cast<double*>(Bt), s);
                 launch_update_f64(static_cast<const double*>(Ap), b, static_cast<const double*>(Bt),
-                                  static_cast<double*>(C), Lx, Lx, b, Lx, s);
+                                  static_cast<double*>(C), Lx, Lx, b, Lx, true, s);
             }
         };
         for (int w = 0; w < 2; ++w) run();
@@ -807,7 +848,8 @@ extern "C" int pmm_fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b
 extern "C" int pmm_compute(pmm_ctx* ctx, int32_t zero_c, pmm_stats* stats) {
     return guarded([&] {
         FPM_CHECK_ARG(ctx != nullptr, "null ctx");
-        fpm::compute(ctx, zero_c != 0, stats);
+        (void)zero_c;  // every compute produces C = A B (iteration 0 overwrites C)
+        fpm::compute(ctx, stats);
     });
 }
 
@@ -854,12 +896,14 @@ extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int6
                 same = same && x.col == y.col && x.row0 == y.row0 && x.col0 == y.col0 && x.h == y.h && x.w == y.w;
             }
         if (!same) fpm::setup(ctx, N, b, p, rects, dt);
-        double tu = 0.0, td = 0.0;
-        fpm::upload(ctx, A, B, ld, row_base, col_base, &tu);
+        FPM_CHECK_ARG(A && B && C, "null host matrix");
+        for (auto& d : ctx->devs)
+            if (d.live()) fpm::check_window(ctx, d, ld, row_base, col_base);
+        const fpm::HostSrc host{A, B, ld, row_base, col_base};
         pmm_stats local;
-        fpm::compute(ctx, false, &local);
+        fpm::compute(ctx, &local, &host);  // host panels streamed under the updates
+        double td = 0.0;
         fpm::download(ctx, C, ld, row_base, col_base, &td);
-        local.t_upload_s = tu;
         local.t_download_s = td;
         if (stats) *stats = local;
     });
@@ -884,6 +928,15 @@ extern "C" int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64
     });
 }
 
+extern "C" int fpm_k_split_cols_f32(const float* src, int64_t ld, int64_t K, int64_t W, int32_t scheme, void* hi,
+                                    void* lo, float* inv_scale, void* stream) {
+    return guarded([&] {
+        FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
+        fpm::launch_split_cols(src, ld, K, W, (fpm::SplitScheme)scheme, hi, lo, inv_scale,
+                               static_cast<cudaStream_t>(stream));
+    });
+}
+
 extern "C" int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64_t cols, void* dst,
                                void* stream) {
     return guarded([&] {
@@ -899,7 +952,8 @@ extern "C" int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t 
 
 extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
                                 const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
-                                int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, void* stream) {
+                                int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, int32_t accumulate,
+                                void* stream) {
     return guarded([&] {
         FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
@@ -915,14 +969,15 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
         CU(cudaGetDevice(&dev));
         CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
         a.num_sms = (num_sms > 0 && num_sms < sms) ? num_sms : sms;
+        a.accumulate = accumulate != 0;
         fpm::launch_update_f32(a, static_cast<cudaStream_t>(stream));
     });
 }
 
 extern "C" int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                                int64_t K, int64_t ldc, void* stream) {
+                                int64_t K, int64_t ldc, int32_t accumulate, void* stream) {
     return guarded([&] {
-        fpm::launch_update_f64(A, lda, Bt, C, M, Nc, K, ldc, static_cast<cudaStream_t>(stream));
+        fpm::launch_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate != 0, static_cast<cudaStream_t>(stream));
     });
 }
 

@@ -1,0 +1,122 @@
+#!/usr/bin/env python
+"""Heterogeneity study (BASELINE config 4 analogue) on ONE B200.
+
+p emulated devices share the GPU, each capped to a number of SMs (the
+persistent update kernel's grid), with caps proportional to config 4's
+{144, 128, 112, 96, 80, 64, 48, 32} scaled to fit 148 SMs.  For each device an
+FPM is sampled with fpm_sample (exclusive, as the paper measures GPUs);
+then the same multiply runs under four partitions:
+
+  fpm          fpm_partition on the sampled speed functions ([5])
+  cpm_ncal     constant models = speed at the even share of a smaller
+               calibration problem N_cal ("when some workload is
+               distributed evenly"; P:107 the CPM used speeds measured while the
+               problem was small) -- reading Q9
+  cpm_self     constant models calibrated at this run's even share
+  homogeneous  equal areas
+
+Reported per partition: total time and GFLOPS, per-device computation time
+(Fig. 6 metric), measured imbalance max/mean - 1, and the imbalance the
+FPMs predict for the achieved areas.  Writes JSON (default profiles/hetero_c4_r01.json).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import sys
+import time
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+sys.path.insert(0, ROOT)
+
+import paper_conf_cluster_zhongrl12_b200 as pkg  # noqa: E402
+
+
+def imbalance(ts):
+    live = [t for t in ts if t > 0]
+    return max(live) / (sum(live) / len(live)) - 1.0 if live else 0.0
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--N", type=int, default=32768)
+    ap.add_argument("--b", type=int, default=512)
+    ap.add_argument("--caps", default="30,26,24,20,16,14,10,6")
+    ap.add_argument("--ncal", type=int, default=8192)
+    ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--sizes", default="1,2,3,4,6,8,12,16,20,24,28,32,40")
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
+    args = ap.parse_args()
+    caps = [int(c) for c in args.caps.split(",")]
+    p, N, b = len(caps), args.N, args.b
+    n = N // b
+    T = n * n
+    sizes = [int(m) ** 2 for m in args.sizes.split(",")]
+
+    ctx = pkg.Context.local([0] * p, sm_caps=caps)
+    t0 = time.perf_counter()
+    models, sample_info = [], []
+    for dev in range(p):
+        sp, ci, reps = ctx.sample(dev, b, sizes, pkg.FPM_F32)
+        models.append((sizes, sp))
+        sample_info.append({"cap": caps[dev], "speeds_gflops": [s / 1e9 for s in sp], "rel_ci95": ci, "reps": reps})
+    t_sample = time.perf_counter() - t0
+
+    x_cal = max(1, (args.ncal // b) ** 2 // p)
+    x_even = T // p
+    parts = {
+        "fpm": pkg.fpm_partition(T, models),
+        "cpm_ncal": pkg.fpm_partition(T, [([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models]),
+        "cpm_self": pkg.fpm_partition(T, [([1], [pkg.fpm_model_speed(m, x_even)]) for m in models]),
+        "homogeneous": pkg.fpm_partition(T, [([1], [1.0])] * p),
+    }
+    results = {}
+    for name, d in parts.items():
+        rects = pkg.colpart_arrange(n, d)
+        ctx.setup(N, b, rects, pkg.FPM_F32)
+        ctx.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
+        ctx.compute()
+        best = None
+        for _ in range(args.reps):
+            st = ctx.compute()
+            if best is None or st.t_compute_s < best.t_compute_s:
+                best = st
+        areas = [r[3] * r[4] for r in rects]
+        per_dev = list(best.per_dev_compute_s[:p])
+        pred = [a / pkg.fpm_model_speed(m, a) if a > 0 else 0.0 for a, m in zip(areas, models)]
+        results[name] = {
+            "d": d, "areas": areas, "rects": rects,
+            "t_total_s": best.t_compute_s, "gflops": best.gflops,
+            "per_dev_compute_s": per_dev,
+            "imbalance_measured": imbalance(per_dev), "imbalance_predicted": imbalance(pred),
+            "predicted_time_s": max(pred),
+            "comm_bytes": best.comm_bytes,
+        }
+        print(f"{name:12s} t={best.t_compute_s:8.4f}s  {best.gflops / 1e3:8.1f} TFLOP/s  "
+              f"imb meas={100 * imbalance(per_dev):6.2f}%  pred={100 * imbalance(pred):6.2f}%  d={d}",
+              flush=True)
+    ctx.close()
+
+    # reference: the whole GPU as one device (upper bound of the aggregate)
+    with pkg.Context.local([0]) as one:
+        one.setup(N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+        one.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
+        one.compute()
+        st1 = one.compute()
+    out = {
+        "config": {"N": N, "b": b, "p": p, "sm_caps": caps, "ncal": args.ncal, "x_cal": x_cal, "x_even": x_even,
+                   "sizes": sizes, "dtype": "f32 (F16X3)", "gpu": "1x B200, devices emulated by SM caps"},
+        "fpm_sample_s": t_sample, "models": sample_info, "partitions": results,
+        "whole_gpu": {"t_s": st1.t_compute_s, "gflops": st1.gflops},
+        "fpm_vs_cpm_ncal_time_delta": results["fpm"]["t_total_s"] / results["cpm_ncal"]["t_total_s"] - 1.0,
+        "fpm_vs_homogeneous_time_delta": results["fpm"]["t_total_s"] / results["homogeneous"]["t_total_s"] - 1.0,
+    }
+    os.makedirs(os.path.dirname(args.out), exist_ok=True)
+    with open(args.out, "w") as f:
+        json.dump(out, f, indent=1)
+    print(json.dumps({k: out[k] for k in ("fpm_vs_cpm_ncal_time_delta", "fpm_vs_homogeneous_time_delta")}))
+
+
+if __name__ == "__main__":
+    main()

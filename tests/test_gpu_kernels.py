@@ -69,6 +69,57 @@ def test_split_f16x3_reconstructs():
     assert np.all(hm[nz] >= 2.0 ** 14) and np.all(hm[nz] <= 2.0 ** 15)
 
 
+def _np_split_f16(x):
+    """Reading Q15 written out in numpy: per row, 2^s puts the row max in
+    [2^14, 2^15); h0 = fp16_rn(x 2^s), h1 = fp16_rn(x 2^s - h0) in fp32."""
+    m = np.abs(x).max(axis=1)
+    _, e = np.frexp(m)
+    s = np.where(m > 0, np.clip(15 - e, -126, 127), 0).astype(np.int32)
+    xs = (x * np.ldexp(np.float32(1), s)[:, None]).astype(np.float32)
+    h0 = xs.astype(np.float16)
+    h1 = (xs - h0.astype(np.float32)).astype(np.float16)
+    return h0, h1, np.ldexp(np.float32(1), -s).astype(np.float32)
+
+
+def test_split_rows_f16x3_bit_exact_vs_numpy():
+    rows, K = 130, 256
+    x = _scaled_rows(rows, K, 5)
+    hi = torch.empty((rows, K), dtype=torch.float16, device="cuda")
+    lo = torch.empty_like(hi)
+    inv = torch.empty(rows, dtype=torch.float32, device="cuda")
+    pkg.k_split_f32(T(x), K, rows, K, pkg.SCHEME_F16X3, hi, lo, inv)
+    torch.cuda.synchronize()
+    h0, h1, s = _np_split_f16(x)
+    assert np.array_equal(hi.cpu().numpy().view(np.uint16), h0.view(np.uint16))
+    assert np.array_equal(lo.cpu().numpy().view(np.uint16), h1.view(np.uint16))
+    assert np.array_equal(inv.cpu().numpy(), s)
+
+
+@pytest.mark.parametrize("K,W,ld", [(64, 256, 256), (512, 1000, 1004), (32, 4, 8)])
+def test_split_cols_bit_exact_vs_numpy(K, W, ld):
+    """B pivot row K x W -> split halves of its transpose (W x K)."""
+    src = _scaled_rows(W, K, 6).T.copy()           # K x W with per-column scales
+    src = np.pad(src, ((0, 0), (0, ld - W)), constant_values=7.0)
+    for scheme in (pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3):
+        odt = torch.float16 if scheme == pkg.SCHEME_F16X3 else torch.float32
+        hi = torch.empty((W, K), dtype=odt, device="cuda")
+        lo = torch.empty_like(hi)
+        inv = torch.empty(W, dtype=torch.float32, device="cuda")
+        pkg.k_split_cols_f32(T(src), ld, K, W, scheme, hi, lo, inv)
+        torch.cuda.synchronize()
+        xt = np.ascontiguousarray(src[:, :W].T)
+        if scheme == pkg.SCHEME_F16X3:
+            h0, h1, s = _np_split_f16(xt)
+            assert np.array_equal(hi.cpu().numpy().view(np.uint16), h0.view(np.uint16))
+            assert np.array_equal(lo.cpu().numpy().view(np.uint16), h1.view(np.uint16))
+            assert np.array_equal(inv.cpu().numpy(), s)
+        else:
+            hb = hi.cpu().numpy()
+            assert np.all(hb.view(np.uint32) & 0x1FFF == 0)
+            rec = hb.astype(np.float64) + lo.cpu().numpy().astype(np.float64)
+            assert np.all(np.abs(rec - xt) <= 2.0 ** -21 * np.abs(xt.astype(np.float64)) + 1e-300)
+
+
 def test_split_tf32x3_reconstructs():
     rows, K = 257, 96
     x = _scaled_rows(rows, K, 4)
@@ -96,7 +147,7 @@ def test_transpose_bit_exact(dt, rows, cols):
     assert np.array_equal(out.cpu().numpy(), x[:, :cols].T)
 
 
-def _update_f32(A, B, C0, scheme, cg, num_sms=0):
+def _update_f32(A, B, C0, scheme, cg, num_sms=0, accumulate=True):
     M, K = A.shape
     Nc = B.shape[1]
     half = scheme == pkg.SCHEME_F16X3
@@ -107,10 +158,13 @@ def _update_f32(A, B, C0, scheme, cg, num_sms=0):
     sa = torch.empty(M, dtype=torch.float32, device="cuda")
     sb = torch.empty(Nc, dtype=torch.float32, device="cuda")
     pkg.k_split_f32(T(A), K, M, K, scheme, a_hi, a_lo, sa)
-    pkg.k_split_f32(T(Bt), K, Nc, K, scheme, b_hi, b_lo, sb)
+    if Nc % 4 == 0:   # the product path: split of the transposed B pivot row in one pass
+        pkg.k_split_cols_f32(T(B), Nc, K, Nc, scheme, b_hi, b_lo, sb)
+    else:
+        pkg.k_split_f32(T(Bt), K, Nc, K, scheme, b_hi, b_lo, sb)
     C = T(C0)
     pkg.k_update_f32(a_hi, a_lo, b_hi, b_lo, sa if half else None, sb if half else None, C, M, Nc, K,
-                     C0.shape[1], scheme, cg, num_sms)
+                     C0.shape[1], scheme, cg, num_sms, accumulate)
     torch.cuda.synchronize()
     return C.cpu().numpy()
 
@@ -141,6 +195,21 @@ def test_update_f32_integer_exact(scheme, cg):
     C0 = synth.rect(6, 4096, 0, 0, M, Nc, synth.DIST_INT)
     C = _update_f32(A, B, C0, scheme, cg)
     assert np.array_equal(C.astype(np.float64), C0.astype(np.float64) + og.gemm(A, B))
+
+
+@pytest.mark.parametrize("scheme", [pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])
+@pytest.mark.parametrize("cg", [1, 2])
+def test_update_f32_overwrite_ignores_c(scheme, cg):
+    """accumulate = 0 (iteration 0): C = A B, the old C (NaN here) is never read."""
+    M, Nc, K = 700, 520, 128
+    A = synth.rect(1, 4096, 0, 0, M, K)
+    B = synth.rect(2, 4096, 0, 0, K, Nc)
+    C = _update_f32(A, B, np.full((M, Nc), np.nan, np.float32), scheme, cg, accumulate=False)
+    assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+    Ai = synth.rect(4, 4096, 0, 0, M, K, synth.DIST_INT)
+    Bi = synth.rect(5, 4096, 0, 0, K, Nc, synth.DIST_INT)
+    Ci = _update_f32(Ai, Bi, np.full((M, Nc), np.nan, np.float32), scheme, cg, accumulate=False)
+    assert np.array_equal(Ci.astype(np.float64), og.gemm(Ai, Bi))
 
 
 def test_update_f32_identity_and_sm_cap():
@@ -177,7 +246,7 @@ def test_update_f64(M, Nc, K):
     assert og.rel_fro(C.cpu().numpy(), ref) <= 1e-12
     Ai = synth.rect(4, 4096, 0, 0, M, K, synth.DIST_INT, np.float64)
     Bi = synth.rect(5, 4096, 0, 0, K, Nc, synth.DIST_INT, np.float64)
-    Ci = torch.zeros((M, Nc), dtype=torch.float64, device="cuda")
-    pkg.k_update_f64(T(Ai), K, T(np.ascontiguousarray(Bi.T)), Ci, M, Nc, K, Nc)
+    Ci = torch.full((M, Nc), float("nan"), dtype=torch.float64, device="cuda")
+    pkg.k_update_f64(T(Ai), K, T(np.ascontiguousarray(Bi.T)), Ci, M, Nc, K, Nc, accumulate=False)
     torch.cuda.synchronize()
     assert np.array_equal(Ci.cpu().numpy(), og.gemm(Ai, Bi))

@@ -101,6 +101,42 @@ def test_zero_area_device_and_sm_caps():
         assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
 
 
+def test_nccl_mode_single_rank():
+    """The NCCL context (dlopen'ed libnccl, world communicator, column split) on
+    one rank: exercises the multi-process code path end to end on one GPU."""
+    nid = pkg.Context.nccl_unique_id()
+    with pkg.Context.nccl(0, 1, 0, nid) as ctx:
+        A, B, C, st = _run(ctx, 512, 64, [(0, 0, 0, 8, 8)], pkg.FPM_F32)
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+def test_run_streams_host_windows():
+    """pmm_run with a host window that is only one device's rectangle (the
+    multi-process usage) and with pinned host memory."""
+    N, b = 1024, 128
+    n = N // b
+    rects = pkg.colpart_arrange(n, [40, 24])
+    A = synth.rect(1, N, 0, 0, N, N)
+    B = synth.rect(2, N, 0, 0, N, N)
+    hA = torch.from_numpy(A).pin_memory()
+    hB = torch.from_numpy(B).pin_memory()
+    hC = torch.full((N, N), float("nan")).pin_memory()
+    with pkg.Context.local([0, 0]) as ctx:
+        st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32)
+        assert st.t_upload_s > 0 and st.t_download_s > 0
+    assert og.rel_fro(hC.numpy(), og.gemm(A, B)) <= 1e-5
+    # host arrays with a leading dimension larger than N (padded rows)
+    pad = 24
+    Ap = np.full((N, N + pad), 5.0, np.float32)
+    Bp = np.full((N, N + pad), 5.0, np.float32)
+    Ap[:, :N], Bp[:, :N] = A, B
+    Cp = np.full((N, N + pad), np.nan, dtype=np.float32)
+    with pkg.Context.local([0]) as ctx:
+        ctx.run(Ap, Bp, Cp, N, b, [(0, 0, 0, n, n)], pkg.FPM_F32, ld=N + pad)
+    assert og.rel_fro(Cp[:, :N], og.gemm(A, B)) <= 1e-5
+    assert np.all(np.isnan(Cp[:, N:]))
+
+
 def test_invalid_arguments_fail_loudly():
     with pkg.Context.local([0]) as ctx:
         with pytest.raises(pkg.FpmError):
@@ -110,7 +146,7 @@ def test_invalid_arguments_fail_loudly():
         with pytest.raises(pkg.FpmError):
             ctx.compute()                                 # no problem set
     with pytest.raises(pkg.FpmError):
-        pkg.Context.local([0], sm_caps=[12])              # not a multiple of 8
+        pkg.Context.local([0], sm_caps=[13])              # odd: CTA pairs need an even cap
 
 
 def test_fpm_sample_procedure():
