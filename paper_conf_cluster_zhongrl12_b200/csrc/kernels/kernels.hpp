@@ -28,6 +28,8 @@ struct UpdateArgs {
     int cta_group;      // 1 or 2
     int num_sms;        // SMs the persistent grid may use
     bool accumulate = true;  // false: C = A . Bt^T (no read of C)
+    int raster_group = 16;   // tile-rows per raster group (L2 reuse)
+    int l2_hint_b = 0;       // B^T tile L2 policy: 0 evict_normal, 1 evict_first, 2 evict_last
 };
 
 // C += A . Bt^T  (the rank-b update)

@@ -86,70 +86,68 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
 }
 
 // B pivot row (K rows x W cols, row stride ld) -> K-major operand halves of its
-// transpose (W rows x K), split as in split_rows_*.  No shared memory (so it can
-// co-reside with the persistent update kernel): a warp owns 128 columns, lane
-// l columns 4l..4l+3; pass 1 takes the column maxima (F16X3), pass 2 re-reads
-// 8 rows at a time (coalesced float4) and writes 16 B of each of its 4 output
-// rows per half.
+// transpose (W rows x K), split as in split_rows_*.  A block owns 32 columns
+// (lane = column, coalesced 128 B row reads); its 8 warps take interleaved
+// 8-row chunks.  Pass 1: column maxima, reduced across the warps through 1 KB of
+// shared memory (small enough to co-reside with the persistent update kernel,
+// which leaves ~2.8 KB per SM).  Pass 2: each lane converts its column's 8 rows
+// of a chunk and writes them as 16 B of output row (col, k0..k0+7).
 template <bool F16>
 __global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
                                                     void* __restrict__ hi, void* __restrict__ lo,
                                                     float* __restrict__ inv_scale) {
-    const int64_t col0 = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 128 + (threadIdx.x % 32) * 4;
-    if (col0 >= W) return;
-    float scale[4] = {1.f, 1.f, 1.f, 1.f};
+    __shared__ float red[8][32];
+    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
+    const int64_t col = (int64_t)blockIdx.x * 32 + lane;
+    const bool in = col < W;
+    const int64_t nchunks = K / 8;
+    float scale = 1.0f;
     if constexpr (F16) {
-        float m[4] = {0.f, 0.f, 0.f, 0.f};
-        for (int64_t r = 0; r < K; ++r) {
-            const float4 v = *reinterpret_cast<const float4*>(src + r * ld + col0);
-            m[0] = fmaxf(m[0], fabsf(v.x));
-            m[1] = fmaxf(m[1], fabsf(v.y));
-            m[2] = fmaxf(m[2], fabsf(v.z));
-            m[3] = fmaxf(m[3], fabsf(v.w));
-        }
+        float m = 0.0f;
+        if (in)
+            for (int64_t ch = warp; ch < nchunks; ch += 8)
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            int e = 0;
-            if (m[c] > 0.0f) frexpf(m[c], &e);
-            int s = (m[c] > 0.0f) ? 15 - e : 0;
-            s = s < -126 ? -126 : (s > 127 ? 127 : s);
-            scale[c] = ldexpf(1.0f, s);
-            inv_scale[col0 + c] = ldexpf(1.0f, -s);
-        }
+                for (int i = 0; i < 8; ++i) m = fmaxf(m, fabsf(src[(ch * 8 + i) * ld + col]));
+        red[warp][lane] = m;
+        __syncthreads();
+        m = red[0][lane];
+#pragma unroll
+        for (int w = 1; w < 8; ++w) m = fmaxf(m, red[w][lane]);
+        int e = 0;
+        if (m > 0.0f) frexpf(m, &e);
+        int s = (m > 0.0f) ? 15 - e : 0;
+        s = s < -126 ? -126 : (s > 127 ? 127 : s);
+        scale = ldexpf(1.0f, s);
+        if (warp == 0 && in) inv_scale[col] = ldexpf(1.0f, -s);
     }
-    for (int64_t r0 = 0; r0 < K; r0 += 8) {
-        float x[8][4];
+    if (!in) return;
+    for (int64_t ch = warp; ch < nchunks; ch += 8) {
+        float x[8];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            const float4 v = *reinterpret_cast<const float4*>(src + (r0 + i) * ld + col0);
-            x[i][0] = v.x; x[i][1] = v.y; x[i][2] = v.z; x[i][3] = v.w;
-        }
+        for (int i = 0; i < 8; ++i) x[i] = src[(ch * 8 + i) * ld + col];
+        if constexpr (F16) {
+            __align__(16) __half h[8], l[8];
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            if constexpr (F16) {
-                __align__(16) __half h[8], l[8];
-#pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    const float xs = x[i][c] * scale[c];
-                    h[i] = __float2half_rn(xs);
-                    l[i] = __float2half_rn(xs - __half2float(h[i]));
-                }
-                *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + (col0 + c) * K + r0) = *reinterpret_cast<uint4*>(h);
-                *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + (col0 + c) * K + r0) = *reinterpret_cast<uint4*>(l);
-            } else {
-                __align__(16) float h[8], l[8];
-#pragma unroll
-                for (int i = 0; i < 8; ++i) {
-                    h[i] = tf32_rna(x[i][c]);
-                    l[i] = tf32_rna(x[i][c] - h[i]);
-                }
-                float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + (col0 + c) * K + r0);
-                float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + (col0 + c) * K + r0);
-                hp[0] = *reinterpret_cast<float4*>(h);
-                hp[1] = *reinterpret_cast<float4*>(h + 4);
-                lp[0] = *reinterpret_cast<float4*>(l);
-                lp[1] = *reinterpret_cast<float4*>(l + 4);
+            for (int i = 0; i < 8; ++i) {
+                const float xs = x[i] * scale;
+                h[i] = __float2half_rn(xs);
+                l[i] = __float2half_rn(xs - __half2float(h[i]));
             }
+            *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + col * K + ch * 8) = *reinterpret_cast<uint4*>(h);
+            *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + col * K + ch * 8) = *reinterpret_cast<uint4*>(l);
+        } else {
+            __align__(16) float h[8], l[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                h[i] = tf32_rna(x[i]);
+                l[i] = tf32_rna(x[i] - h[i]);
+            }
+            float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + col * K + ch * 8);
+            float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + col * K + ch * 8);
+            hp[0] = *reinterpret_cast<float4*>(h);
+            hp[1] = *reinterpret_cast<float4*>(h + 4);
+            lp[0] = *reinterpret_cast<float4*>(l);
+            lp[1] = *reinterpret_cast<float4*>(l + 4);
         }
     }
 }
@@ -283,8 +281,8 @@ void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, Sp
 void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,
                        float* inv_scale, cudaStream_t st) {
     if (K <= 0 || W <= 0) return;
-    FPM_CHECK_ARG(K % 8 == 0 && W % 4 == 0 && ld % 4 == 0, "split_cols: K % 8, W % 4, ld % 4 must be 0");
-    const unsigned blocks = (unsigned)((W + 1023) / 1024);  // 8 warps x 128 columns
+    FPM_CHECK_ARG(K % 8 == 0, "split_cols: K must be a multiple of 8");
+    const unsigned blocks = (unsigned)((W + 31) / 32);  // 32 columns per block
     if (s == SplitScheme::F16X3) {
         FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
         split_cols_k<true><<<blocks, 256, 0, st>>>(src, ld, K, W, hi, lo, inv_scale);

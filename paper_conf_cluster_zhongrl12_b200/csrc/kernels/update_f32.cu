@@ -59,11 +59,14 @@ struct UpdParams {
     const float* sa;  // per-row inverse scales of A (F16X3) or nullptr
     const float* sb;  // per-column inverse scales of B (F16X3) or nullptr
     int load_c;       // 1: C += A B^T (read-modify-write), 0: C = A B^T (first iteration)
+    int group;        // raster group (tile-rows)
+    uint64_t hint_b;  // L2 policy of the B^T tiles (A tiles: evict_last, C: evict_first)
 };
 
-// Grouped raster over tiles so concurrently running CTAs share A / B tiles in L2.
-__device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int& tm, int& tn) {
-    constexpr int G = 16;
+// Grouped raster over tiles so concurrently running CTAs share A / B tiles in L2:
+// groups of G tile-rows, column-major inside a group (A rows of the group stay
+// resident while the B^T tiles stream once per group).
+__device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int G, int& tm, int& tn) {
     const int per_group = G * tiles_n;
     const int g = t / per_group;
     const int first_m = g * G;
@@ -135,7 +138,7 @@ __global__ void __launch_bounds__(192, 1)
             uint32_t phase = 0;
             for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
                 int tm, tn;
-                tile_coords(t, P.tiles_m, P.tiles_n, tm, tn);
+                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
                 const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
                 const int n0 = tn * BN + (int)rank * Cfg::BN_CTA;
                 for (int kb = 0; kb < num_kb; ++kb) {
@@ -149,14 +152,14 @@ __global__ void __launch_bounds__(192, 1)
                         ptx::mbar_arrive_expect_tx(&full[stage], Cfg::STAGE_BYTES);
                         ptx::tma_load_2d(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
                         ptx::tma_load_2d(sA_lo, &tmA_lo, &full[stage], k0, m0, ptx::kEvictLast);
-                        ptx::tma_load_2d(sB_hi, &tmB_hi, &full[stage], k0, n0, ptx::kEvictLast);
-                        ptx::tma_load_2d(sB_lo, &tmB_lo, &full[stage], k0, n0, ptx::kEvictLast);
+                        ptx::tma_load_2d(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
+                        ptx::tma_load_2d(sB_lo, &tmB_lo, &full[stage], k0, n0, P.hint_b);
                     } else {
                         if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
                         ptx::tma_load_2d_cg2(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
                         ptx::tma_load_2d_cg2(sA_lo, &tmA_lo, &full[stage], k0, m0, ptx::kEvictLast);
-                        ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, ptx::kEvictLast);
-                        ptx::tma_load_2d_cg2(sB_lo, &tmB_lo, &full[stage], k0, n0, ptx::kEvictLast);
+                        ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
+                        ptx::tma_load_2d_cg2(sB_lo, &tmB_lo, &full[stage], k0, n0, P.hint_b);
                     }
                     if (++stage == STAGES) { stage = 0; phase ^= 1; }
                 }
@@ -209,7 +212,7 @@ __global__ void __launch_bounds__(192, 1)
         int it = 0;
         for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
             int tm, tn;
-            tile_coords(t, P.tiles_m, P.tiles_n, tm, tn);
+            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
             const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
             const int n0 = tn * BN;
             const int acc = it & 1;
@@ -273,7 +276,8 @@ __global__ void __launch_bounds__(192, 1)
                 ptx::fence_proxy_async_smem();
                 ptx::named_bar_sync(1, 128);
                 if (e == 0) {
-                    ptx::tma_store_2d(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0);
+                    ptx::tma_store_2d_hint(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
+                                           ptx::kEvictFirst);
                     ptx::bulk_commit();
                     if (P.load_c && c + 2 < Cfg::N_CHUNKS) {
                         ptx::bulk_wait_read0();
@@ -354,6 +358,8 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.sa = a.sa;
     P.sb = a.sb;
     P.load_c = a.accumulate ? 1 : 0;
+    P.group = a.raster_group > 0 ? a.raster_group : 16;
+    P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
     auto kern = update_kernel<CG, TF32, BN, STAGES>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;

@@ -85,6 +85,8 @@ struct pmm_ctx {
 
     int f32_scheme = 0;  // fpm::SplitScheme
     int cta_group = 2;
+    int raster_group = 16;
+    int l2_hint_b = 0;
 };
 
 namespace fpm {
@@ -403,6 +405,8 @@ void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
         a.cta_group = ctx->cta_group;
         a.num_sms = d.num_sms;
         a.accumulate = k != 0;  // iteration 0 writes C = A(0) B(0): no zeroing, no read of C
+        a.raster_group = ctx->raster_group;
+        a.l2_hint_b = ctx->l2_hint_b;
         launch_update_f32(a, d.s_comp);
     } else {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
@@ -817,6 +821,12 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
         } else if (k == "cta_group") {
             FPM_CHECK_ARG(value == 1 || value == 2, "cta_group must be 1 or 2");
             ctx->cta_group = (int)value;
+        } else if (k == "l2_hint_b") {
+            FPM_CHECK_ARG(value >= 0 && value <= 2, "l2_hint_b must be 0 (normal), 1 (first) or 2 (last)");
+            ctx->l2_hint_b = (int)value;
+        } else if (k == "raster_group") {
+            FPM_CHECK_ARG(value >= 1 && value <= 4096, "raster_group must be in [1, 4096]");
+            ctx->raster_group = (int)value;
         } else {
             fpm::fail(FPM_EINVAL, "unknown option '%s'", key);
         }
