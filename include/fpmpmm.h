@@ -159,6 +159,20 @@ int pmm_nccl_unique_id(uint8_t id_out[128]);
 int pmm_create_nccl(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm_cap,
                     const uint8_t nccl_id[128], pmm_ctx** out);
 
+/* Multi-process context without NCCL: one process per GPU (rank of world),
+ * pivots pulled one-sidedly from the peers' resident A_q / B_q through CUDA IPC
+ * mappings (NVLink for peers on other GPUs), fused into the staging kernels that
+ * split them for the tensor cores.  The inputs never change during the
+ * iteration loop, so pulls need no synchronisation with the owner.  Protocol:
+ * pmm_setup -> pmm_ipc_export (every rank) -> all-gather of the blobs by the
+ * caller -> pmm_ipc_import -> pmm_upload / pmm_fill_synthetic -> caller
+ * barrier -> pmm_compute -> pmm_download.  pmm_run returns FPM_EUNSUPPORTED. */
+#define FPM_IPC_BLOB_BYTES 256
+int pmm_create_ipc(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm_cap, pmm_ctx** out);
+int pmm_ipc_export(pmm_ctx* ctx, uint8_t blob_out[FPM_IPC_BLOB_BYTES]);
+/* blobs: world x FPM_IPC_BLOB_BYTES, rank order. */
+int pmm_ipc_import(pmm_ctx* ctx, const uint8_t* blobs, int32_t world);
+
 int pmm_destroy(pmm_ctx* ctx);
 
 /* Fix the problem: N x N matrices, blocking factor b ("blocking factor

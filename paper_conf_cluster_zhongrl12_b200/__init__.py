@@ -98,6 +98,22 @@ class Context:
         check(lib.pmm_create_nccl(rank, world, cuda_device, sm_cap, nccl_id, ctypes.byref(h)))
         return cls(h.value, world)
 
+    @classmethod
+    def ipc(cls, rank: int, world: int, cuda_device: int, sm_cap: int = 0) -> "Context":
+        """One process per GPU, pivots pulled from peers' memory (CUDA IPC)."""
+        h = ctypes.c_void_p()
+        check(lib.pmm_create_ipc(rank, world, cuda_device, sm_cap, ctypes.byref(h)))
+        return cls(h.value, world)
+
+    def ipc_export(self) -> bytes:
+        buf = ctypes.create_string_buffer(_lib.FPM_IPC_BLOB_BYTES)
+        check(lib.pmm_ipc_export(self._h, buf))
+        return buf.raw
+
+    def ipc_import(self, blobs: Sequence[bytes]) -> None:
+        joined = b"".join(blobs)
+        check(lib.pmm_ipc_import(self._h, joined, len(blobs)))
+
     def close(self) -> None:
         if self._h:
             check(lib.pmm_destroy(self._h))

@@ -20,6 +20,7 @@ FPM_ENCCL = -4
 FPM_EUNSUPPORTED = -5
 FPM_ESTATE = -6
 FPM_MAX_DEVICES = 16
+FPM_IPC_BLOB_BYTES = 256
 
 FPM_F32 = 0
 FPM_F64 = 1
@@ -87,6 +88,9 @@ _SIGS = {
     "pmm_create_local": ([i32, ctypes.POINTER(i32), ctypes.POINTER(i32), ctypes.POINTER(vp)], ctypes.c_int),
     "pmm_nccl_unique_id": ([ctypes.c_char_p], ctypes.c_int),
     "pmm_create_nccl": ([i32, i32, i32, i32, ctypes.c_char_p, ctypes.POINTER(vp)], ctypes.c_int),
+    "pmm_create_ipc": ([i32, i32, i32, i32, ctypes.POINTER(vp)], ctypes.c_int),
+    "pmm_ipc_export": ([vp, ctypes.c_char_p], ctypes.c_int),
+    "pmm_ipc_import": ([vp, ctypes.c_char_p, i32], ctypes.c_int),
     "pmm_destroy": ([vp], ctypes.c_int),
     "pmm_set_option": ([vp, ctypes.c_char_p, i64], ctypes.c_int),
     "pmm_setup": ([vp, i64, i64, i32, ctypes.POINTER(ColpartRect), ctypes.c_int], ctypes.c_int),

@@ -62,6 +62,7 @@ struct Device {
     float* sa[2] = {}, *sb[2] = {};
     const void* a_op[2] = {};               // FP64: A operand of the slot
     std::vector<void*> allocs;
+    int64_t launches = 0;                   // library kernels launched (running count)
 
     bool live() const { return H > 0 && W > 0; }
 };
@@ -69,12 +70,16 @@ struct Device {
 }  // namespace fpm
 
 struct pmm_ctx {
-    bool nccl_mode = false;
+    bool nccl_mode = false;  // one process per GPU, pivots over NCCL
+    bool ipc_mode = false;   // one process per GPU, pivots pulled from peers' memory (CUDA IPC)
     int rank = 0, world = 1;
     std::vector<fpm::Device> devs;
     ncclComm_t world_comm = nullptr;
     ncclComm_t col_comm = nullptr;
     std::vector<int> col_members;  // global ranks of my column, sorted
+    // IPC mode: peers' resident A_q, B_q mapped into this process
+    std::vector<void*> peer_A, peer_B;
+    bool peers_ready = false;
 
     bool have_problem = false;
     int64_t N = 0, b = 0, n = 0;
@@ -171,6 +176,30 @@ Device* local_dev(pmm_ctx* ctx, int idx) {
     return nullptr;
 }
 
+// ------------------------------------------------------------------ IPC peers
+void close_peers(pmm_ctx* ctx) {
+    if (!ctx->ipc_mode) return;
+    if (!ctx->devs.empty()) cudaSetDevice(ctx->devs[0].cuda_dev);
+    for (auto* v : {&ctx->peer_A, &ctx->peer_B})
+        for (void*& ptr : *v) {
+            if (ptr) cudaIpcCloseMemHandle(ptr);
+            ptr = nullptr;
+        }
+    ctx->peers_ready = false;
+}
+
+// Resident A_q / B_q of device q: local devices directly, IPC peers through the
+// mapped handles.  These buffers are written only by upload/fill, never during
+// the k-loop, so a pull needs no synchronisation with the owner.
+const void* src_A(pmm_ctx* ctx, int q) {
+    if (ctx->ipc_mode) return q == ctx->rank ? ctx->devs[0].A : ctx->peer_A[q];
+    return local_dev(ctx, q)->A;
+}
+const void* src_B(pmm_ctx* ctx, int q) {
+    if (ctx->ipc_mode) return q == ctx->rank ? ctx->devs[0].B : ctx->peer_B[q];
+    return local_dev(ctx, q)->B;
+}
+
 // ---------------------------------------------------------------- setup
 void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects, fpm_dtype dt) {
     FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype %d", (int)dt);
@@ -178,12 +207,13 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
                   (long long)b);
     FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 : b % 32 == 0, "b must be a multiple of %d",
                   dt == FPM_F64 ? 8 : 32);
-    const int expect_p = ctx->nccl_mode ? ctx->world : (int)ctx->devs.size();
+    const int expect_p = (ctx->nccl_mode || ctx->ipc_mode) ? ctx->world : (int)ctx->devs.size();
     FPM_CHECK_ARG(p == expect_p, "arrangement has %d devices, context drives %d", p, expect_p);
     FPM_CHECK_ARG(rects != nullptr, "null rects");
     const int64_t n = N / b;
     validate_rects(n, p, rects);
 
+    close_peers(ctx);
     for (auto& d : ctx->devs) free_problem(d);
     ctx->have_problem = false;
     ctx->N = N;
@@ -211,9 +241,14 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         d.B = dalloc(d, HW * es);
         d.C = dalloc(d, HW * es);
         const size_t op = (dt == FPM_F64) ? 0 : (ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4);
+        // receive buffers: NCCL lands pivots in them; FP64 copies peers' pivots into
+        // them.  FP32 in local / IPC mode stages straight from the peers' memory.
+        const bool need_recv = ctx->nccl_mode || dt == FPM_F64;
         for (int s = 0; s < 2; ++s) {
-            d.a_recv[s] = dalloc(d, (size_t)d.H * b * es);
-            d.b_recv[s] = dalloc(d, (size_t)b * d.W * es);
+            if (need_recv) {
+                d.a_recv[s] = dalloc(d, (size_t)d.H * b * es);
+                d.b_recv[s] = dalloc(d, (size_t)b * d.W * es);
+            }
             if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * b * es);
             if (dt == FPM_F32) {
                 d.a_hi[s] = dalloc(d, (size_t)d.H * b * op);
@@ -294,45 +329,61 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use,
     if (!first_use) CU(cudaStreamWaitEvent(d.s_comm, d.ev_free[slot], 0));
     const colpart_rect& r = d.rect;
 
+    // FP32 in local / IPC mode: the staging kernels read the pivot straight from
+    // the holder's / owner's resident buffer (peer memory over NVLink, or the same
+    // GPU), so the transfer is fused into the split -- no receive buffer, no copy.
+    const bool fused = ctx->dt == FPM_F32 && !ctx->nccl_mode;
+    struct Piece {
+        const void* src;
+        int64_t row_off, rows;  // in elements (rows of my H x b panel)
+    };
+    std::vector<Piece> a_pieces;
+
     // ---- A(rows_i, k): local if this device's column holds block-column k
     const bool holder = r.col0 <= k && k < r.col0 + r.w;
-    const void* a_src;
+    const void* a_src = nullptr;
     if (holder) {
         a_src = static_cast<const char*>(d.A) + (size_t)(k - r.col0) * d.H * b * es;
-    } else {
+    } else if (ctx->nccl_mode) {
         a_src = d.a_recv[slot];
-        if (!ctx->nccl_mode) {
-            for (const Move& m : ctx->plan_a[k]) {
-                if (m.dst != d.idx) continue;
-                Device* q = local_dev(ctx, m.src);
-                const colpart_rect& qr = ctx->rects[m.src];
-                const size_t cnt = (size_t)(m.end - m.begin) * b * b;
-                const char* src = static_cast<const char*>(q->A) +
-                                  ((size_t)(k - qr.col0) * q->H * b + (size_t)(m.begin - qr.row0) * b * b) * es;
+    } else {
+        for (const Move& m : ctx->plan_a[k]) {
+            if (m.dst != d.idx) continue;
+            const colpart_rect& qr = ctx->rects[m.src];
+            const size_t cnt = (size_t)(m.end - m.begin) * b * b;
+            const char* src = static_cast<const char*>(src_A(ctx, m.src)) +
+                              ((size_t)(k - qr.col0) * qr.h * b * b + (size_t)(m.begin - qr.row0) * b * b) * es;
+            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[k], 0));
+            if (fused) {
+                a_pieces.push_back(Piece{src, (m.begin - r.row0) * b, (m.end - m.begin) * b});
+            } else {
                 char* dst = static_cast<char*>(d.a_recv[slot]) + (size_t)(m.begin - r.row0) * b * b * es;
-                if (streamed) CU(cudaStreamWaitEvent(d.s_comm, q->ev_up[k], 0));
                 CU(cudaMemcpyAsync(dst, src, cnt * es, cudaMemcpyDefault, d.s_comm));
-                bytes += (int64_t)(cnt * es);
+                a_src = d.a_recv[slot];
             }
+            bytes += (int64_t)(cnt * es);
         }
     }
     // ---- B(k, cols_i): local if this device's rows hold block-row k
     const bool owner = r.row0 <= k && k < r.row0 + r.h;
-    const void* b_src;
+    const void* b_src = nullptr;
     if (owner) {
         b_src = static_cast<const char*>(d.B) + (size_t)(k - r.row0) * b * d.W * es;
-    } else {
+    } else if (ctx->nccl_mode) {
         b_src = d.b_recv[slot];
-        if (!ctx->nccl_mode) {
-            for (const Move& m : ctx->plan_b[k]) {
-                if (m.dst != d.idx) continue;
-                Device* o = local_dev(ctx, m.src);
-                const colpart_rect& orr = ctx->rects[m.src];
-                const char* src = static_cast<const char*>(o->B) + (size_t)(k - orr.row0) * b * o->W * es;
-                if (streamed) CU(cudaStreamWaitEvent(d.s_comm, o->ev_up[k], 0));
+    } else {
+        for (const Move& m : ctx->plan_b[k]) {
+            if (m.dst != d.idx) continue;
+            const colpart_rect& orr = ctx->rects[m.src];
+            const char* src = static_cast<const char*>(src_B(ctx, m.src)) + (size_t)(k - orr.row0) * b * d.W * es;
+            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[k], 0));
+            if (fused) {
+                b_src = src;
+            } else {
                 CU(cudaMemcpyAsync(d.b_recv[slot], src, (size_t)b * d.W * es, cudaMemcpyDefault, d.s_comm));
-                bytes += (int64_t)((size_t)b * d.W * es);
+                b_src = d.b_recv[slot];
             }
+            bytes += (int64_t)((size_t)b * d.W * es);
         }
     }
     if (ctx->nccl_mode) {
@@ -369,14 +420,26 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use,
     CU(cudaEventRecord(d.ev_pack0[k], d.s_comm));
     if (ctx->dt == FPM_F32) {
         const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
-        launch_split_rows(static_cast<const float*>(a_src), b, d.H, b, sch, d.a_hi[slot], d.a_lo[slot], d.sa[slot],
-                          d.s_comm);
+        const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
+        d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + 1;
+        if (a_src) {
+            launch_split_rows(static_cast<const float*>(a_src), b, d.H, b, sch, d.a_hi[slot], d.a_lo[slot],
+                              d.sa[slot], d.s_comm);
+        } else {
+            for (const Piece& pc : a_pieces)
+                launch_split_rows(static_cast<const float*>(pc.src), b, pc.rows, b, sch,
+                                  static_cast<char*>(d.a_hi[slot]) + (size_t)pc.row_off * b * op,
+                                  static_cast<char*>(d.a_lo[slot]) + (size_t)pc.row_off * b * op,
+                                  d.sa[slot] + pc.row_off, d.s_comm);
+        }
+        FPM_CHECK_ARG(b_src != nullptr, "no source of block-row %lld for device %d", (long long)k, d.idx);
         launch_split_cols(static_cast<const float*>(b_src), d.W, b, d.W, sch, d.b_hi[slot], d.b_lo[slot],
                           d.sb[slot], d.s_comm);
     } else {
         d.a_op[slot] = a_src;
         launch_transpose_f64(static_cast<const double*>(b_src), d.W, b, d.W, static_cast<double*>(d.bt[slot]),
                              d.s_comm);
+        d.launches += 1;
     }
     CU(cudaEventRecord(d.ev_pack1[k], d.s_comm));
     CU(cudaEventRecord(d.ev_ready[slot], d.s_comm));
@@ -412,6 +475,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
                           static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k != 0, d.s_comp);
     }
+    d.launches += 1;
     CU(cudaEventRecord(d.ev_upd1[k], d.s_comp));
     CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
 }
@@ -421,6 +485,11 @@ void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
 // iteration ahead of their use (pmm_run).
 void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
+    if (ctx->ipc_mode && !ctx->peers_ready)
+        fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
+    FPM_CHECK_ARG(!(ctx->ipc_mode && host), "IPC mode has no streamed host input (peers cannot be ordered)");
+    int64_t launches0 = 0;
+    for (auto& d : ctx->devs) launches0 += d.launches;
     for (auto& d : ctx->devs) {
         if (!d.live()) continue;
         CU(cudaSetDevice(d.cuda_dev));
@@ -433,8 +502,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         CU(cudaStreamWaitEvent(d.s_comm, d.ev_start, 0));
     }
     const bool streamed = host != nullptr;
-    int64_t bytes = 0, launches = 0;
-    const int per_iter = ctx->dt == FPM_F32 ? 3 : 2;  // split A, split B^T, update | transpose, update
+    int64_t bytes = 0;
     for (int64_t k = 0; k < ctx->n; ++k) {
         const int slot = (int)(k & 1);
         if (streamed)
@@ -446,7 +514,6 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
             if (d.live()) {
                 bytes += issue_comm(ctx, d, k, slot, k < 2, streamed);
                 issue_update(ctx, d, k, slot);
-                launches += per_iter;
             } else {
                 NC(nccl().GroupStart());
                 NC(nccl().GroupEnd());
@@ -456,11 +523,10 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         for (auto& d : ctx->devs)
             if (d.live()) bytes += issue_comm(ctx, d, k, slot, k < 2, streamed);
         for (auto& d : ctx->devs)
-            if (d.live()) {
-                issue_update(ctx, d, k, slot);
-                launches += per_iter;
-            }
+            if (d.live()) issue_update(ctx, d, k, slot);
     }
+    int64_t launches = -launches0;
+    for (auto& d : ctx->devs) launches += d.launches;
     for (auto& d : ctx->devs) {
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventRecord(d.ev_stop, d.s_comp));
@@ -798,9 +864,92 @@ extern "C" int pmm_create_nccl(int32_t rank, int32_t world, int32_t cuda_device,
     });
 }
 
+extern "C" int pmm_create_ipc(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm_cap, pmm_ctx** out) {
+    return guarded([&] {
+        FPM_CHECK_ARG(out != nullptr, "null argument");
+        *out = nullptr;
+        FPM_CHECK_ARG(world >= 1 && world <= FPM_MAX_DEVICES && rank >= 0 && rank < world, "bad rank/world");
+        int count = 0;
+        CU(cudaGetDeviceCount(&count));
+        FPM_CHECK_ARG(cuda_device >= 0 && cuda_device < count, "CUDA device %d out of range", cuda_device);
+        auto ctx = std::make_unique<pmm_ctx>();
+        ctx->ipc_mode = true;
+        ctx->rank = rank;
+        ctx->world = world;
+        ctx->peer_A.assign(world, nullptr);
+        ctx->peer_B.assign(world, nullptr);
+        ctx->devs.resize(1);
+        ctx->devs[0].idx = rank;
+        ctx->devs[0].cuda_dev = cuda_device;
+        ctx->devs[0].sm_cap = sm_cap;
+        fpm::init_device(ctx->devs[0]);
+        *out = ctx.release();
+    });
+}
+
+namespace {
+constexpr uint32_t kIpcMagic = 0x46504d31;  // "FPM1"
+struct IpcBlob {
+    uint32_t magic;
+    int32_t rank;
+    int32_t live;
+    int32_t pad;
+    int64_t N, b;
+    cudaIpcMemHandle_t A, B;
+};
+static_assert(sizeof(IpcBlob) <= FPM_IPC_BLOB_BYTES, "IPC blob size");
+}  // namespace
+
+extern "C" int pmm_ipc_export(pmm_ctx* ctx, uint8_t blob_out[FPM_IPC_BLOB_BYTES]) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx && blob_out, "null argument");
+        FPM_CHECK_ARG(ctx->ipc_mode, "not an IPC context");
+        if (!ctx->have_problem) fpm::fail(FPM_ESTATE, "pmm_ipc_export before pmm_setup");
+        IpcBlob blob;
+        std::memset(&blob, 0, sizeof(blob));
+        blob.magic = kIpcMagic;
+        blob.rank = ctx->rank;
+        blob.N = ctx->N;
+        blob.b = ctx->b;
+        fpm::Device& d = ctx->devs[0];
+        blob.live = d.live() ? 1 : 0;
+        if (d.live()) {
+            CU(cudaSetDevice(d.cuda_dev));
+            CU(cudaIpcGetMemHandle(&blob.A, d.A));
+            CU(cudaIpcGetMemHandle(&blob.B, d.B));
+        }
+        std::memset(blob_out, 0, FPM_IPC_BLOB_BYTES);
+        std::memcpy(blob_out, &blob, sizeof(blob));
+    });
+}
+
+extern "C" int pmm_ipc_import(pmm_ctx* ctx, const uint8_t* blobs, int32_t world) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx && blobs, "null argument");
+        FPM_CHECK_ARG(ctx->ipc_mode, "not an IPC context");
+        FPM_CHECK_ARG(world == ctx->world, "expected %d blobs", ctx->world);
+        if (!ctx->have_problem) fpm::fail(FPM_ESTATE, "pmm_ipc_import before pmm_setup");
+        fpm::close_peers(ctx);
+        CU(cudaSetDevice(ctx->devs[0].cuda_dev));
+        for (int q = 0; q < world; ++q) {
+            IpcBlob blob;
+            std::memcpy(&blob, blobs + (size_t)q * FPM_IPC_BLOB_BYTES, sizeof(blob));
+            FPM_CHECK_ARG(blob.magic == kIpcMagic && blob.rank == q, "blob %d is not rank %d's export", q, q);
+            FPM_CHECK_ARG(blob.N == ctx->N && blob.b == ctx->b, "rank %d set up a different problem", q);
+            const colpart_rect& r = ctx->rects[q];
+            FPM_CHECK_ARG((blob.live != 0) == (r.h > 0 && r.w > 0), "rank %d liveness differs from the arrangement", q);
+            if (q == ctx->rank || !blob.live) continue;
+            CU(cudaIpcOpenMemHandle(&ctx->peer_A[q], blob.A, cudaIpcMemLazyEnablePeerAccess));
+            CU(cudaIpcOpenMemHandle(&ctx->peer_B[q], blob.B, cudaIpcMemLazyEnablePeerAccess));
+        }
+        ctx->peers_ready = true;
+    });
+}
+
 extern "C" int pmm_destroy(pmm_ctx* ctx) {
     return guarded([&] {
         if (!ctx) return;
+        fpm::close_peers(ctx);
         for (auto& d : ctx->devs) fpm::destroy_device(d);
         if (ctx->nccl_mode) {
             if (ctx->col_comm) fpm::nccl().CommDestroy(ctx->col_comm);
@@ -905,6 +1054,9 @@ extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int6
                 const colpart_rect &x = ctx->rects[i], &y = rects[i];
                 same = same && x.col == y.col && x.row0 == y.row0 && x.col0 == y.col0 && x.h == y.h && x.w == y.w;
             }
+        if (ctx->ipc_mode)
+            fpm::fail(FPM_EUNSUPPORTED, "pmm_run is not available on IPC contexts: use pmm_upload, a barrier across "
+                                        "the ranks, pmm_compute, pmm_download");
         if (!same) fpm::setup(ctx, N, b, p, rects, dt);
         FPM_CHECK_ARG(A && B && C, "null host matrix");
         for (auto& d : ctx->devs)
