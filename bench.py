@@ -164,11 +164,15 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     n = N // b
     p = world
 
-    # ---- context (NCCL over NVLink for N > 1)
-    if world > 1:
+    # ---- context: N > 1 -> one process per GPU, pivots pulled from the peers'
+    # memory over NVLink (ipc, default) or exchanged with NCCL (nccl)
+    ipc = world > 1 and args.transport == "ipc"
+    if world > 1 and not ipc:
         obj = [pkg.Context.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         ctx = pkg.Context.nccl(rank, world, local_rank, obj[0])
+    elif ipc:
+        ctx = pkg.Context.ipc(rank, world, local_rank)
     else:
         ctx = pkg.Context.local([local_rank])
     if args.scheme == "tf32x3":
@@ -196,16 +200,21 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         d = pkg.fpm_partition(n * n, models_all)
         return d, pkg.colpart_arrange(n, d)
 
-    d, rects = plan()
-    ctx.setup(N, b, rects, pkg.FPM_F32)
-    import synth
-    sa, sb = synth.seeds_for_config(4)   # config 5 (index 4): seeds 5 and 6
-    ctx.fill_synthetic(sa, sb, pkg.FPM_DIST_PM1)
-
     def barrier():
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
+
+    d, rects = plan()
+    ctx.setup(N, b, rects, pkg.FPM_F32)
+    if ipc:
+        blobs = [None] * world
+        dist.all_gather_object(blobs, ctx.ipc_export())
+        ctx.ipc_import(blobs)
+    import synth
+    sa, sb = synth.seeds_for_config(4)   # config 5 (index 4): seeds 5 and 6
+    ctx.fill_synthetic(sa, sb, pkg.FPM_DIST_PM1)
+    barrier()                            # every rank's inputs resident before any pull
 
     def max_over_ranks(x: float) -> float:
         if world == 1:
@@ -289,6 +298,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
                 "N": N, "b": b, "p": p, "partition": d, "rects": rects,
                 "f32_scheme": args.scheme, "cta_group": args.cta_group, "raster_group": args.raster_group,
+                "transport": (args.transport if world > 1 else "none (p = 1)"),
                 "l2": "inputs larger than L2 (A, B, C 9.7 GB each)",
                 "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
                 "imbalance_pct_measured": 100.0 * imb_meas, "imbalance_pct_predicted": 100.0 * imb_pred,
@@ -303,6 +313,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             "clocks": clk,
         }
         print(json.dumps(line), flush=True)
+    barrier()  # no rank frees buffers a peer may still read (IPC)
     ctx.close()
 
 
@@ -314,34 +325,46 @@ def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier):
     r = rects[rank]
     H, W = r[3] * b, r[4] * b
     R0, C0 = r[1] * b, r[2] * b
-    if H * W == 0:
-        return None
+    live = H * W > 0
+    ipc = args.transport == "ipc" and args.gpus > 1
     # host windows = this rank's rectangle (generated on the device once, untimed)
-    hA = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
-    hB = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
-    hC = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
-    tmp = torch.empty((H, W), dtype=torch.float32, device="cuda")
-    pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 5, N, R0, C0, H, W)  # seeds_for_config(4)
-    hA.copy_(tmp)
-    pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 6, N, R0, C0, H, W)
-    hB.copy_(tmp)
-    del tmp
-    torch.cuda.empty_cache()
+    if live:
+        hA = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
+        hB = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
+        hC = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
+        tmp = torch.empty((H, W), dtype=torch.float32, device="cuda")
+        pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 5, N, R0, C0, H, W)  # seeds_for_config(4)
+        hA.copy_(tmp)
+        pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 6, N, R0, C0, H, W)
+        hB.copy_(tmp)
+        del tmp
+        torch.cuda.empty_cache()
     barrier()
-    ts = []
+    ts, st = [], None
     for i in range(args.e2e_steps + 1):
         barrier()
         t0 = time.perf_counter()
-        # blocking call: H2D streamed under the updates, k-loop, D2H of C
-        st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32, ld=W, row_base=R0, col_base=C0)
+        if ipc:
+            # peers pull from each other's resident inputs: upload, barrier, k-loop, download
+            if live:
+                ctx.upload(hA, hB, W, R0, C0)
+            barrier()
+            st = ctx.compute()
+            if live:
+                ctx.download(hC, W, R0, C0)
+        elif live:
+            # blocking call: H2D streamed under the updates, k-loop, D2H of C
+            st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32, ld=W, row_base=R0, col_base=C0)
         t_host = time.perf_counter() - t0
+        t_all = max_over_ranks(t_host)
         if i > 0:  # first call is a warm-up
-            ts.append(max_over_ranks(t_host))
+            ts.append(t_all)
     t = statistics.median(ts)
     return {"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
             "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
-            "device_kloop_incl_streamed_h2d_s": st.t_compute_s, "download_s": st.t_download_s,
-            "timing": "host wall clock around the blocking pmm_run call, max over ranks"}
+            "device_kloop_s": st.t_compute_s if st else None, "download_s": st.t_download_s if st else None,
+            "timing": ("host wall clock: upload + barrier + pmm_compute + download (IPC), max over ranks"
+                       if ipc else "host wall clock around the blocking pmm_run call, max over ranks")}
 
 
 def main():
@@ -353,12 +376,16 @@ def main():
     ap.add_argument("--N", type=int, default=N_DEFAULT)
     ap.add_argument("--b", type=int, default=B_DEFAULT)
     ap.add_argument("--scheme", choices=["f16x3", "tf32x3"], default="f16x3")
+    ap.add_argument("--transport", choices=["ipc", "nccl"], default="ipc",
+                    help="N > 1: pull pivots from peers' memory (ipc) or exchange them with NCCL")
     ap.add_argument("--cta-group", type=int, default=2)
     ap.add_argument("--raster-group", type=int, default=16)
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")
+    ap.add_argument("--same-gpu", action="store_true",
+                    help="testing only: put every rank on cuda:0 (IPC transport works within one GPU)")
     ap.add_argument("--traffic", type=float, default=None,
                     help="dram bytes per update launch from an ncu --set full capture")
     args = ap.parse_args()
@@ -368,6 +395,8 @@ def main():
     world = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
+    if args.same_gpu:
+        local_rank = 0
     dist = None
     if world > 1:
         import torch.distributed as dist
