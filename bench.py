@@ -180,6 +180,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     ctx.set_option("cta_group", args.cta_group)
     ctx.set_option("raster_group", args.raster_group)
     ctx.set_option("l2_hint_b", args.l2_hint_b)
+    ctx.set_option("kernel_variant", args.kernel_variant)
 
     # ---- FPMs (offline): sample this GPU's speed function once;
     # every rank's model is gathered so all ranks partition identically.
@@ -298,6 +299,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
                 "N": N, "b": b, "p": p, "partition": d, "rects": rects,
                 "f32_scheme": args.scheme, "cta_group": args.cta_group, "raster_group": args.raster_group,
+                "kernel_variant": args.kernel_variant,
                 "transport": (args.transport if world > 1 else "none (p = 1)"),
                 "l2": "inputs larger than L2 (A, B, C 9.7 GB each)",
                 "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
@@ -381,6 +383,7 @@ def main():
     ap.add_argument("--cta-group", type=int, default=2)
     ap.add_argument("--raster-group", type=int, default=16)
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
+    ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")

@@ -242,6 +242,10 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 power-of-two scales, 3 kind::f16 MMAs), 1 = TF32X3
  *                 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  DESIGN.md Q15.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
+ *   "kernel_variant": -1 (auto, default) or 0..3, see fpm_k_update_f32.
+ *   "raster_group": tile-rows per L2 raster group of the update (default 16).
+ *   "l2_hint_b":  L2 policy of the B^T operand tiles: 0 normal (default),
+ *                 1 evict-first, 2 evict-last.
  * FPM_EINVAL on unknown key or value. */
 int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value);
 
@@ -272,12 +276,15 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * given as Bt (Nc x K, K-major), operands as produced by fpm_k_split_f32 with
  * the same scheme (sa / sb: inverse row scales of A and Bt for F16X3, NULL
  * for TF32X3).  cta_group 1 or 2; num_sms = persistent grid (0 = all SMs).
- * accumulate = 0 writes C = A x B without reading C.
+ * accumulate = 0 writes C = A x B without reading C.  variant (cta_group 2):
+ * shared-memory split between the operand ring and the C ring: 0 = 128-byte
+ * k-blocks x 3 stages + 2 C chunks in flight, 1 = 64-byte x 4 + 6, 2 = 128-byte
+ * x 2 + 6, 3 = 64-byte x 5 + 4; -1 = auto (= 2, measured best).
  * Requires K % 8 == 0, ldc % 4 == 0. */
 int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
                      const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
                      int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms,
-                     int32_t accumulate, void* stream);
+                     int32_t accumulate, int32_t variant, void* stream);
 
 /* Rank-b update in FP64 on DMMA: C (M x Nc, ldc) (+)= A (M x K, lda) x Bt^T,
  * Bt (Nc x K); accumulate = 0 overwrites C. */

@@ -217,10 +217,10 @@ def k_transpose(src, dtype, ld, rows, cols, dst, stream=None):
 
 
 def k_update_f32(a_hi, a_lo, bt_hi, bt_lo, sa, sb, C, M, Nc, K, ldc, scheme=SCHEME_F16X3, cta_group=2,
-                 num_sms=0, accumulate=True, stream=None):
+                 num_sms=0, accumulate=True, variant=-1, stream=None):
     check(lib.fpm_k_update_f32(_lib._ptr(a_hi), _lib._ptr(a_lo), _lib._ptr(bt_hi), _lib._ptr(bt_lo),
                                _lib._ptr(sa), _lib._ptr(sb), _lib._ptr(C), M, Nc, K, ldc, scheme, cta_group,
-                               num_sms, 1 if accumulate else 0, _stream(stream)))
+                               num_sms, 1 if accumulate else 0, variant, _stream(stream)))
 
 
 def k_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate=True, stream=None):

@@ -106,7 +106,8 @@ _SIGS = {
     "fpm_k_split_f32": ([vp, i64, i64, i64, i32, vp, vp, vp, vp], ctypes.c_int),
     "fpm_k_split_cols_f32": ([vp, i64, i64, i64, i32, vp, vp, vp, vp], ctypes.c_int),
     "fpm_k_transpose": ([vp, i32, i64, i64, i64, vp, vp], ctypes.c_int),
-    "fpm_k_update_f32": ([vp, vp, vp, vp, vp, vp, vp, i64, i64, i64, i64, i32, i32, i32, i32, vp], ctypes.c_int),
+    "fpm_k_update_f32": ([vp, vp, vp, vp, vp, vp, vp, i64, i64, i64, i64, i32, i32, i32, i32, i32, vp],
+                         ctypes.c_int),
     "fpm_k_update_f64": ([vp, i64, vp, vp, i64, i64, i64, i64, i32, vp], ctypes.c_int),
     "fpm_k_fill_synthetic": ([vp, i32, i64, u64, i64, i64, i64, i64, i64, i32, vp], ctypes.c_int),
 }

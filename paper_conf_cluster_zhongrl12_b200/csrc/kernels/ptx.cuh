@@ -120,6 +120,10 @@ __device__ __forceinline__ void bulk_wait_read0() {
 __device__ __forceinline__ void bulk_wait_read1() {
     asm volatile("cp.async.bulk.wait_group.read 1;" ::: "memory");
 }
+template <int N>
+__device__ __forceinline__ void bulk_wait_read_n() {
+    asm volatile("cp.async.bulk.wait_group.read %0;" ::"n"(N) : "memory");
+}
 __device__ __forceinline__ void bulk_wait0() { asm volatile("cp.async.bulk.wait_group 0;" ::: "memory"); }
 __device__ __forceinline__ void fence_proxy_async_smem() {
     asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
@@ -227,15 +231,18 @@ __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, float (&v)[32
     for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
-// Shared-memory matrix descriptor, K-major operand with 128-byte swizzle:
-// rows of 128 B, 8-row atoms of 1024 B (SBO), LBO unused (1), version 1.
-__device__ __forceinline__ uint64_t sdesc_k_sw128(uint32_t smem_addr) {
+// Shared-memory matrix descriptor, K-major operand with SW-byte swizzle
+// (SW = 128 or 64): rows of SW bytes, 8-row atoms of 8*SW bytes (SBO), LBO
+// unused (1), version 1, layout type 2 (128B) / 4 (64B).
+template <int SW>
+__device__ __forceinline__ uint64_t sdesc_k(uint32_t smem_addr) {
+    static_assert(SW == 128 || SW == 64, "swizzle");
     uint64_t d = 0;
     d |= (uint64_t)((smem_addr & 0x3FFFF) >> 4);  // start address
     d |= (uint64_t)1 << 16;                        // leading byte offset (ignored)
-    d |= (uint64_t)(1024 >> 4) << 32;              // stride byte offset
+    d |= (uint64_t)((8 * SW) >> 4) << 32;          // stride byte offset
     d |= (uint64_t)1 << 46;                        // descriptor version (sm_100)
-    d |= (uint64_t)2 << 61;                        // SWIZZLE_128B
+    d |= (uint64_t)(SW == 128 ? 2 : 4) << 61;      // SWIZZLE_128B / SWIZZLE_64B
     return d;
 }
 

@@ -14,13 +14,20 @@
 // Both keep FP32 accumulation in TMEM.
 //
 // Structure (warp-specialised persistent kernel, one CTA per SM or CTA pair):
-//   warp 0      TMA producer: A_hi/A_lo/B_hi/B_lo k-blocks of 128 B rows, 128B swizzle
+//   warp 0      TMA producer: A_hi/A_lo/B_hi/B_lo k-blocks of SW-byte rows (SW-byte swizzle)
 //   warp 1      TMEM allocator + single-thread tcgen05.mma issuer (leader CTA)
-//   warps 2-5   epilogue: TMEM -> registers, C chunk (128 x 32 fp32) TMA-loaded
-//               into smem, C += scale * acc, TMA-stored back (C read-modify-write
-//               every iteration, "accumulating the intermediate results")
+//   warps 2-5   epilogue: TMEM -> registers, C chunks (128 x 32 fp32) TMA-loaded
+//               into an NCB-deep smem ring, C += scale * acc, TMA-stored back (C
+//               read-modify-write every iteration, "accumulating the
+//               intermediate results")
 // Two TMEM accumulators (2 x BN columns) let the epilogue of tile t overlap the
 // mainloop of tile t+1.  CG = 2 pairs two SMs on a 256-row tile (cta_group::2).
+//
+// Shared memory is the budget that decides the balance between the operand ring
+// (STAGES x SW-byte k-blocks) and the C ring (NCB chunks in flight); variant 1
+// (SW = 64, 4 stages, 6 C chunks) keeps ~96 KB of C in flight, which the short
+// mainloops of b = 512 need; variant 0 (SW = 128, 3 stages, 2 C chunks) is the
+// round-1 layout.
 #include <cuda.h>
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
@@ -32,23 +39,26 @@
 
 namespace fpm {
 
-template <int CG, bool TF32, int BN, int STAGES>
+template <int CG, bool TF32, int BN, int STAGES, int SW, int NCB>
 struct UpdCfg {
     static constexpr int BM = 128;                 // rows of C per CTA
     static constexpr int TILE_M = BM * CG;         // rows per MMA tile
     static constexpr int BN_CTA = BN / CG;         // B^T rows loaded per CTA
     static constexpr int ELEM = TF32 ? 4 : 2;      // operand bytes
-    static constexpr int BK = 128 / ELEM;          // k elements per 128-B row
-    static constexpr int A_BYTES = BM * 128;       // one operand half (hi or lo)
-    static constexpr int B_BYTES = BN_CTA * 128;
+    static constexpr int BK = SW / ELEM;           // k elements per SW-byte row
+    static constexpr int KSTEPS = SW / 32;         // MMA k-steps (32 B each) per k-block
+    static constexpr int A_BYTES = BM * SW;        // one operand half (hi or lo)
+    static constexpr int B_BYTES = BN_CTA * SW;
     static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
     static constexpr int C_CHUNK_BYTES = BM * 128; // 128 rows x 32 fp32
     static constexpr int N_CHUNKS = BN / 32;
     static constexpr int TMEM_COLS = 2 * BN;
-    static constexpr int BAR_BYTES = 256;
-    static constexpr int SMEM = 1024 /*align slack*/ + STAGES * STAGE_BYTES + 2 * C_CHUNK_BYTES + BAR_BYTES;
+    static constexpr int BAR_BYTES = 8 * (2 * STAGES + 4 + NCB) + 16;
+    static constexpr int SMEM = 1024 /*align slack*/ + STAGES * STAGE_BYTES + NCB * C_CHUNK_BYTES + BAR_BYTES;
     static constexpr uint32_t IDESC = ptx::idesc_f32acc(TILE_M, BN, TF32);
     static constexpr int THREADS = 192;
+    static_assert(SW == 128 || SW == 64, "swizzle width");
+    static_assert(NCB >= 2 && NCB <= 8, "C ring depth");
     static_assert(TMEM_COLS == 256 || TMEM_COLS == 512, "TMEM columns must be a power of two");
     static_assert(SMEM <= 232448, "shared memory budget");
 };
@@ -76,23 +86,23 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
     tn = r / gm;
 }
 
-template <int CG, bool TF32, int BN, int STAGES>
+template <int CG, bool TF32, int BN, int STAGES, int SW, int NCB>
 __global__ void __launch_bounds__(192, 1)
     update_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
                   const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
                   const __grid_constant__ CUtensorMap tmC, const UpdParams P) {
-    using Cfg = UpdCfg<CG, TF32, BN, STAGES>;
+    using Cfg = UpdCfg<CG, TF32, BN, STAGES, SW, NCB>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint8_t* stage_base = smem;
     uint8_t* cbuf = smem + STAGES * Cfg::STAGE_BYTES;
-    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + 2 * Cfg::C_CHUNK_BYTES);
+    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + NCB * Cfg::C_CHUNK_BYTES);
     uint64_t* full = bars;                       // [STAGES]
     uint64_t* empty = bars + STAGES;             // [STAGES]
     uint64_t* tfull = bars + 2 * STAGES;         // [2]
     uint64_t* tempty = bars + 2 * STAGES + 2;    // [2]
-    uint64_t* cfull = bars + 2 * STAGES + 4;     // [2]
-    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
+    uint64_t* cfull = bars + 2 * STAGES + 4;     // [NCB]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 4 + NCB);
 
     const uint32_t warp = threadIdx.x / 32;
     const uint32_t lane = threadIdx.x % 32;
@@ -109,8 +119,8 @@ __global__ void __launch_bounds__(192, 1)
         for (int a = 0; a < 2; ++a) {
             ptx::mbar_init(&tfull[a], 1);
             ptx::mbar_init(&tempty[a], 4 * CG);  // one arrival per epilogue warp of each CTA
-            ptx::mbar_init(&cfull[a], 1);
         }
+        for (int c = 0; c < NCB; ++c) ptx::mbar_init(&cfull[c], 1);
         ptx::fence_mbar_init();
     }
     if (warp == 0 && lane == 0) {
@@ -185,10 +195,10 @@ __global__ void __launch_bounds__(192, 1)
                         const uint32_t a_lo = a_hi + Cfg::A_BYTES;
                         const uint32_t b_hi = a_lo + Cfg::A_BYTES;
                         const uint32_t b_lo = b_hi + Cfg::B_BYTES;
-                        const uint64_t dA_hi = ptx::sdesc_k_sw128(a_hi), dA_lo = ptx::sdesc_k_sw128(a_lo);
-                        const uint64_t dB_hi = ptx::sdesc_k_sw128(b_hi), dB_lo = ptx::sdesc_k_sw128(b_lo);
+                        const uint64_t dA_hi = ptx::sdesc_k<SW>(a_hi), dA_lo = ptx::sdesc_k<SW>(a_lo);
+                        const uint64_t dB_hi = ptx::sdesc_k<SW>(b_hi), dB_lo = ptx::sdesc_k<SW>(b_lo);
 #pragma unroll
-                        for (int k = 0; k < 4; ++k) {
+                        for (int k = 0; k < Cfg::KSTEPS; ++k) {
                             const uint64_t off = (uint64_t)(k * 32) >> 4;  // 32 B per MMA k-step
                             ptx::umma<CG, TF32>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC, (kb | k) != 0);
                             ptx::umma<CG, TF32>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
@@ -205,10 +215,14 @@ __global__ void __launch_bounds__(192, 1)
         }
     } else {
         // -------------------------------------------------------------- epilogue
+        // C ring: chunk c of a tile lives in buffer c % NCB.  NCB chunks are
+        // loaded when a tile starts; after chunk c >= 1 is stored, chunk
+        // c - 1 + NCB is loaded into the buffer of chunk c - 1 (whose store has
+        // then almost surely finished reading), so NCB - 1 loads stay in flight.
         const uint32_t e = threadIdx.x - 64;   // 0..127
         const uint32_t q = warp & 3;           // TMEM lane quarter this warp may access
         const uint32_t r = q * 32 + lane;      // row of the CTA tile
-        uint32_t cpar = 0;  // bit b = parity of cfull[b]
+        uint32_t cpar = 0;                     // bit b = parity of cfull[b]
         int it = 0;
         for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
             int tm, tn;
@@ -219,7 +233,7 @@ __global__ void __launch_bounds__(192, 1)
             const uint32_t acc_par = (it >> 1) & 1;
             if (e == 0 && P.load_c) {
                 ptx::bulk_wait_read0();
-                for (int c = 0; c < 2 && c < Cfg::N_CHUNKS; ++c) {
+                for (int c = 0; c < NCB && c < Cfg::N_CHUNKS; ++c) {
                     ptx::mbar_arrive_expect_tx(&cfull[c], Cfg::C_CHUNK_BYTES);
                     ptx::tma_load_2d(cbuf + c * Cfg::C_CHUNK_BYTES, &tmC, &cfull[c], n0 + 32 * c, m0,
                                      ptx::kEvictFirst);
@@ -232,7 +246,7 @@ __global__ void __launch_bounds__(192, 1)
             const uint32_t t_row = tmem_base + ((q * 32) << 16) + acc * BN;
 #pragma unroll 1
             for (int c = 0; c < Cfg::N_CHUNKS; ++c) {
-                const int buf = c & 1;
+                const int buf = c % NCB;
                 float v[32];
                 ptx::tmem_ld_32x32b_x32(t_row + 32 * c, v);
                 if (c == Cfg::N_CHUNKS - 1) {
@@ -246,19 +260,31 @@ __global__ void __launch_bounds__(192, 1)
                 }
                 if (P.sb != nullptr) {
                     const int gc = n0 + 32 * c;
+                    if (gc + 32 <= P.Nc) {
+                        const float4* sb4 = reinterpret_cast<const float4*>(P.sb + gc);
 #pragma unroll
-                    for (int j = 0; j < 32; ++j) {
-                        const float sbj = (gc + j < P.Nc) ? __ldg(P.sb + gc + j) : 0.0f;
-                        v[j] *= sa * sbj;
+                        for (int j = 0; j < 8; ++j) {
+                            const float4 s4 = __ldg(sb4 + j);
+                            v[4 * j + 0] *= sa * s4.x;
+                            v[4 * j + 1] *= sa * s4.y;
+                            v[4 * j + 2] *= sa * s4.z;
+                            v[4 * j + 3] *= sa * s4.w;
+                        }
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) {
+                            const float sbj = (gc + j < P.Nc) ? __ldg(P.sb + gc + j) : 0.0f;
+                            v[j] *= sa * sbj;
+                        }
                     }
                 }
                 if (P.load_c) {
                     ptx::mbar_wait(&cfull[buf], (cpar >> buf) & 1u);
                     cpar ^= 1u << buf;
                 } else {
-                    // overwrite (first iteration, C = A(0) B(0)): only wait until the
-                    // store that last used this buffer has read it
-                    if (e == 0) ptx::bulk_wait_read1();
+                    // overwrite (first iteration, C = A(0) B(0)): wait until the store
+                    // that last used this buffer (chunk c - NCB) has read it
+                    if (e == 0) ptx::bulk_wait_read_n<NCB - 1>();
                     ptx::named_bar_sync(1, 128);
                 }
                 uint8_t* rowp = cbuf + buf * Cfg::C_CHUNK_BYTES + r * 128;
@@ -279,10 +305,12 @@ __global__ void __launch_bounds__(192, 1)
                     ptx::tma_store_2d_hint(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
                                            ptx::kEvictFirst);
                     ptx::bulk_commit();
-                    if (P.load_c && c + 2 < Cfg::N_CHUNKS) {
-                        ptx::bulk_wait_read0();
-                        ptx::mbar_arrive_expect_tx(&cfull[buf], Cfg::C_CHUNK_BYTES);
-                        ptx::tma_load_2d(cbuf + buf * Cfg::C_CHUNK_BYTES, &tmC, &cfull[buf], n0 + 32 * (c + 2), m0,
+                    const int nxt = c - 1 + NCB;  // refill the buffer of chunk c - 1
+                    if (P.load_c && c >= 1 && nxt < Cfg::N_CHUNKS) {
+                        const int nb = (c - 1) % NCB;
+                        ptx::bulk_wait_read1();  // store of chunk c - 1 has read its buffer
+                        ptx::mbar_arrive_expect_tx(&cfull[nb], Cfg::C_CHUNK_BYTES);
+                        ptx::tma_load_2d(cbuf + nb * Cfg::C_CHUNK_BYTES, &tmC, &cfull[nb], n0 + 32 * nxt, m0,
                                          ptx::kEvictFirst);
                     }
                 }
@@ -322,7 +350,8 @@ EncodeTiledFn get_encode() {
 
 }  // namespace
 
-// Row-major rows x cols matrix (ld elements), 128B-swizzled box of box_cols x box_rows.
+// Row-major rows x cols matrix (ld elements), swizzled box of box_cols x box_rows
+// (box_cols * elem_bytes = the swizzle width: 128 or 64 bytes).
 CUtensorMap make_tmap_2d(const void* base, CUtensorMapDataType dt, int elem_bytes, int64_t rows, int64_t cols,
                          int64_t ld, int box_cols, int box_rows) {
     CUtensorMap m;
@@ -330,18 +359,22 @@ CUtensorMap make_tmap_2d(const void* base, CUtensorMapDataType dt, int elem_byte
     cuuint64_t strides[1] = {(cuuint64_t)(ld * elem_bytes)};
     cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
     cuuint32_t estr[2] = {1, 1};
+    const int row_bytes = box_cols * elem_bytes;
+    const CUtensorMapSwizzle sw = row_bytes == 128 ? CU_TENSOR_MAP_SWIZZLE_128B
+                                  : row_bytes == 64 ? CU_TENSOR_MAP_SWIZZLE_64B
+                                                    : CU_TENSOR_MAP_SWIZZLE_32B;
     CUresult r = get_encode()(&m, dt, 2, const_cast<void*>(base), dims, strides, box, estr,
-                              CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
-                              CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+                              CU_TENSOR_MAP_INTERLEAVE_NONE, sw, CU_TENSOR_MAP_L2_PROMOTION_L2_256B,
+                              CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
     if (r != CUDA_SUCCESS)
         fail(FPM_ECUDA, "cuTensorMapEncodeTiled failed (%d) rows=%lld cols=%lld ld=%lld", (int)r,
              (long long)rows, (long long)cols, (long long)ld);
     return m;
 }
 
-template <int CG, bool TF32, int BN, int STAGES>
+template <int CG, bool TF32, int BN, int STAGES, int SW, int NCB>
 static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
-    using Cfg = UpdCfg<CG, TF32, BN, STAGES>;
+    using Cfg = UpdCfg<CG, TF32, BN, STAGES, SW, NCB>;
     const CUtensorMapDataType odt = TF32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
     const CUtensorMap tAh = make_tmap_2d(a.a_hi, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
     const CUtensorMap tAl = make_tmap_2d(a.a_lo, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
@@ -360,7 +393,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.load_c = a.accumulate ? 1 : 0;
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
-    auto kern = update_kernel<CG, TF32, BN, STAGES>;
+    auto kern = update_kernel<CG, TF32, BN, STAGES, SW, NCB>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;
     cudaGetDevice(&dev);
@@ -393,13 +426,32 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
+    FPM_CHECK_ARG(a.variant >= -1 && a.variant <= 3, "kernel variant must be -1 (auto) or 0..3");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
+    // auto: variant 2 (two 64-KB operand stages, six C chunks in flight) measured
+    // best at both K = 512 and K = 1024 on B200 (profiles/README.md)
+    const int variant = a.variant >= 0 ? a.variant : 2;
     if (a.cta_group == 2) {
-        if (tf32) launch_update_t<2, true, 256, 3>(a, st);
-        else launch_update_t<2, false, 256, 3>(a, st);
+        switch (variant) {
+            case 1:  // 64-B k-blocks x 4 stages, 6 C chunks in flight
+                if (tf32) launch_update_t<2, true, 256, 4, 64, 6>(a, st);
+                else launch_update_t<2, false, 256, 4, 64, 6>(a, st);
+                break;
+            case 2:  // 128-B k-blocks x 2 stages, 6 C chunks
+                if (tf32) launch_update_t<2, true, 256, 2, 128, 6>(a, st);
+                else launch_update_t<2, false, 256, 2, 128, 6>(a, st);
+                break;
+            case 3:  // 64-B k-blocks x 5 stages, 4 C chunks
+                if (tf32) launch_update_t<2, true, 256, 5, 64, 4>(a, st);
+                else launch_update_t<2, false, 256, 5, 64, 4>(a, st);
+                break;
+            default:  // 128-B k-blocks x 3 stages, 2 C chunks
+                if (tf32) launch_update_t<2, true, 256, 3, 128, 2>(a, st);
+                else launch_update_t<2, false, 256, 3, 128, 2>(a, st);
+        }
     } else {
-        if (tf32) launch_update_t<1, true, 256, 2>(a, st);
-        else launch_update_t<1, false, 256, 2>(a, st);
+        if (tf32) launch_update_t<1, true, 256, 2, 128, 2>(a, st);
+        else launch_update_t<1, false, 256, 2, 128, 2>(a, st);
     }
 }
 

@@ -92,6 +92,7 @@ struct pmm_ctx {
     int cta_group = 2;
     int raster_group = 16;
     int l2_hint_b = 0;
+    int kernel_variant = -1;  // auto (by K)
 };
 
 namespace fpm {
@@ -470,6 +471,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
         a.accumulate = k != 0;  // iteration 0 writes C = A(0) B(0): no zeroing, no read of C
         a.raster_group = ctx->raster_group;
         a.l2_hint_b = ctx->l2_hint_b;
+        a.variant = ctx->kernel_variant;
         launch_update_f32(a, d.s_comp);
     } else {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
@@ -745,6 +747,9 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.scheme = sch;
                 a.cta_group = ctx->cta_group;
                 a.num_sms = d->num_sms;
+                a.raster_group = ctx->raster_group;
+                a.l2_hint_b = ctx->l2_hint_b;
+                a.variant = ctx->kernel_variant;
                 launch_update_f32(a, s);
             } else {
                 launch_transpose_f64(static_cast<const double*>(Bp), L, b, Lx, static_cast<double*>(Bt), s);
@@ -970,6 +975,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
         } else if (k == "cta_group") {
             FPM_CHECK_ARG(value == 1 || value == 2, "cta_group must be 1 or 2");
             ctx->cta_group = (int)value;
+        } else if (k == "kernel_variant") {
+            FPM_CHECK_ARG(value >= -1 && value <= 3, "kernel_variant must be -1 (auto) or 0..3");
+            ctx->kernel_variant = (int)value;
         } else if (k == "l2_hint_b") {
             FPM_CHECK_ARG(value >= 0 && value <= 2, "l2_hint_b must be 0 (normal), 1 (first) or 2 (last)");
             ctx->l2_hint_b = (int)value;
@@ -1115,10 +1123,11 @@ extern "C" int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t 
 extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
                                 const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
                                 int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, int32_t accumulate,
-                                void* stream) {
+                                int32_t variant, void* stream) {
     return guarded([&] {
         FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
+        FPM_CHECK_ARG(variant >= -1 && variant <= 3, "variant must be -1 (auto) or 0..3");
         FPM_CHECK_ARG(scheme == 1 || (sa && sb), "F16X3 needs sa and sb");
         fpm::UpdateArgs a;
         a.a_hi = a_hi; a.a_lo = a_lo; a.bt_hi = bt_hi; a.bt_lo = bt_lo;
@@ -1132,6 +1141,7 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
         CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev));
         a.num_sms = (num_sms > 0 && num_sms < sms) ? num_sms : sms;
         a.accumulate = accumulate != 0;
+        a.variant = variant;
         fpm::launch_update_f32(a, static_cast<cudaStream_t>(stream));
     });
 }

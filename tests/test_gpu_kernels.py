@@ -147,7 +147,13 @@ def test_transpose_bit_exact(dt, rows, cols):
     assert np.array_equal(out.cpu().numpy(), x[:, :cols].T)
 
 
+KCFG = ["1", "2v0", "2v1"]   # cta_group 1; cta_group 2 with smem variants 0 and 1
+
+
 def _update_f32(A, B, C0, scheme, cg, num_sms=0, accumulate=True):
+    cg = str(cg)
+    variant = int(cg[2]) if "v" in cg else 1
+    cg = int(cg[0])
     M, K = A.shape
     Nc = B.shape[1]
     half = scheme == pkg.SCHEME_F16X3
@@ -164,7 +170,7 @@ def _update_f32(A, B, C0, scheme, cg, num_sms=0, accumulate=True):
         pkg.k_split_f32(T(Bt), K, Nc, K, scheme, b_hi, b_lo, sb)
     C = T(C0)
     pkg.k_update_f32(a_hi, a_lo, b_hi, b_lo, sa if half else None, sb if half else None, C, M, Nc, K,
-                     C0.shape[1], scheme, cg, num_sms, accumulate)
+                     C0.shape[1], scheme, cg, num_sms, accumulate, variant)
     torch.cuda.synchronize()
     return C.cpu().numpy()
 
@@ -174,7 +180,7 @@ SHAPES = [(128, 256, 64), (300, 520, 96), (1000, 1000, 512), (64, 40, 32), (1, 8
 
 
 @pytest.mark.parametrize("scheme", [pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])
-@pytest.mark.parametrize("cg", [1, 2])
+@pytest.mark.parametrize("cg", KCFG)
 @pytest.mark.parametrize("M,Nc,K", SHAPES)
 def test_update_f32_random(scheme, cg, M, Nc, K):
     A = synth.rect(1, 4096, 0, 0, M, K)
@@ -187,7 +193,7 @@ def test_update_f32_random(scheme, cg, M, Nc, K):
 
 
 @pytest.mark.parametrize("scheme", [pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])
-@pytest.mark.parametrize("cg", [1, 2])
+@pytest.mark.parametrize("cg", KCFG)
 def test_update_f32_integer_exact(scheme, cg):
     M, Nc, K = 520, 776, 512
     A = synth.rect(4, 4096, 0, 0, M, K, synth.DIST_INT)
@@ -198,7 +204,7 @@ def test_update_f32_integer_exact(scheme, cg):
 
 
 @pytest.mark.parametrize("scheme", [pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])
-@pytest.mark.parametrize("cg", [1, 2])
+@pytest.mark.parametrize("cg", KCFG)
 def test_update_f32_overwrite_ignores_c(scheme, cg):
     """accumulate = 0 (iteration 0): C = A B, the old C (NaN here) is never read."""
     M, Nc, K = 700, 520, 128
