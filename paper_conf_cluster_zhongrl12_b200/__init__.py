@@ -73,9 +73,10 @@ def colpart_plan_step(n: int, rects: Sequence[Rect], k: int):
 class Context:
     """Owns a pmm_ctx: devices, streams, resident buffers, NCCL communicators."""
 
-    def __init__(self, handle: int, p: int):
+    def __init__(self, handle: int, p: int, local_devices: int = 1):
         self._h = ctypes.c_void_p(handle)
-        self.p = p
+        self.p = p                          # devices of the arrangement
+        self.local_devices = local_devices  # devices driven by this process
 
     @classmethod
     def local(cls, cuda_devices: Sequence[int], sm_caps: Sequence[int] | None = None) -> "Context":
@@ -84,7 +85,7 @@ class Context:
         caps = (ctypes.c_int32 * p)(*(sm_caps or [0] * p))
         h = ctypes.c_void_p()
         check(lib.pmm_create_local(p, devs, caps, ctypes.byref(h)))
-        return cls(h.value, p)
+        return cls(h.value, p, p)
 
     @staticmethod
     def nccl_unique_id() -> bytes:
@@ -171,13 +172,19 @@ class Context:
         return st
 
     def sample(self, dev: int, b: int, sizes: Sequence[int], dtype: int = FPM_F32):
+        """Speed points of device `dev`; dev = -1 samples all local devices at once
+        and returns lists of per-device lists."""
         n = len(sizes)
+        rows = self.local_devices if dev == -1 else 1
         xs = (ctypes.c_int64 * n)(*[int(x) for x in sizes])
-        sp = (ctypes.c_double * n)()
-        ci = (ctypes.c_double * n)()
-        reps = (ctypes.c_int32 * n)()
+        sp = (ctypes.c_double * (n * rows))()
+        ci = (ctypes.c_double * (n * rows))()
+        reps = (ctypes.c_int32 * (n * rows))()
         check(lib.fpm_sample(self._h, int(dev), int(dtype), int(b), xs, n, sp, ci, reps))
-        return list(sp), list(ci), list(reps)
+        if dev != -1:
+            return list(sp), list(ci), list(reps)
+        cut = lambda a: [list(a[i * n:(i + 1) * n]) for i in range(rows)]  # noqa: E731
+        return cut(sp), cut(ci), cut(reps)
 
 
 def fpm_sample(ctx: Context, dev: int, b: int, sizes: Sequence[int], dtype: int = FPM_F32):

@@ -676,13 +676,25 @@ double t975(int df) {
 // timing this kernel"; P:10 (iii) "experiments are repeated multiple times
 // until the results are statistically reliable"; P:18 kernel Ci += A(b) x B(b)
 // on sqrt(x) x sqrt(x) submatrices.  Speed = 2 x b^3 flop / time (Q7, Q8).
+//
+// dev = -1 samples every device of the context at the same time (P:10 (ii):
+// "Processes are synchronised ... ensures that the resources will be shared
+// between the maximum number of processes"), which captures the contention of
+// devices emulated on one GPU; each repetition launches the kernel on all
+// devices and times each on its own stream.  Outputs are then p x nsizes.
 void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes, int nsizes, double* speeds,
             double* ci, int32_t* reps_out) {
-    Device* d = local_dev(ctx, dev);
-    FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
     FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype");
     FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 && b >= 8 : b % 32 == 0 && b >= 32, "bad block size b");
     FPM_CHECK_ARG(nsizes >= 1 && sizes && speeds, "bad sizes");
+    std::vector<Device*> devs;
+    if (dev == -1) {
+        for (auto& d : ctx->devs) devs.push_back(&d);
+    } else {
+        Device* d = local_dev(ctx, dev);
+        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
+        devs.push_back(d);
+    }
     int64_t mmax = 0;
     std::vector<int64_t> ms(nsizes);
     for (int j = 0; j < nsizes; ++j) {
@@ -695,91 +707,122 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         ms[j] = m;
         mmax = std::max(mmax, m);
     }
-    CU(cudaSetDevice(d->cuda_dev));
     const int64_t L = mmax * b;
     const size_t es = dt == FPM_F64 ? 8 : 4;
     const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
     const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
-    Device tmp;  // owns the scratch allocations
-    tmp.cuda_dev = d->cuda_dev;
-    struct Guard {
-        Device& t;
-        ~Guard() { free_problem(t); }
-    } guard{tmp};
-    void* C = dalloc(tmp, (size_t)L * L * es);
-    void* Ap = dalloc(tmp, (size_t)L * b * es);
-    void* Bp = dalloc(tmp, (size_t)b * L * es);
-    void* Bt = dalloc(tmp, (size_t)L * b * es);
-    void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
-    float *sa = nullptr, *sb = nullptr;
-    if (dt == FPM_F32) {
-        ah = dalloc(tmp, (size_t)L * b * op);
-        al = dalloc(tmp, (size_t)L * b * op);
-        bh = dalloc(tmp, (size_t)L * b * op);
-        bl = dalloc(tmp, (size_t)L * b * op);
-        sa = static_cast<float*>(dalloc(tmp, (size_t)L * 4));
-        sb = static_cast<float*>(dalloc(tmp, (size_t)L * 4));
+
+    struct Scratch {
+        Device* d = nullptr;
+        Device mem;  // owns the allocations
+        void *C = nullptr, *Ap = nullptr, *Bp = nullptr, *Bt = nullptr;
+        void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
+        float *sa = nullptr, *sb = nullptr;
+        cudaEvent_t e0 = nullptr, e1 = nullptr;
+        std::vector<double> ts;
+        double mean = 0.0, half = 0.0;
+        bool done = false;
+        ~Scratch() {
+            free_problem(mem);
+            if (e0) cudaEventDestroy(e0);
+            if (e1) cudaEventDestroy(e1);
+        }
+    };
+    std::vector<std::unique_ptr<Scratch>> S;
+    for (Device* d : devs) {
+        S.emplace_back(new Scratch);
+        Scratch& s = *S.back();
+        s.d = d;
+        s.mem.cuda_dev = d->cuda_dev;
+        CU(cudaSetDevice(d->cuda_dev));
+        s.C = dalloc(s.mem, (size_t)L * L * es);
+        s.Ap = dalloc(s.mem, (size_t)L * b * es);
+        s.Bp = dalloc(s.mem, (size_t)b * L * es);
+        s.Bt = dalloc(s.mem, (size_t)L * b * es);
+        if (dt == FPM_F32) {
+            s.ah = dalloc(s.mem, (size_t)L * b * op);
+            s.al = dalloc(s.mem, (size_t)L * b * op);
+            s.bh = dalloc(s.mem, (size_t)L * b * op);
+            s.bl = dalloc(s.mem, (size_t)L * b * op);
+            s.sa = static_cast<float*>(dalloc(s.mem, (size_t)L * 4));
+            s.sb = static_cast<float*>(dalloc(s.mem, (size_t)L * 4));
+        }
+        CU(cudaEventCreate(&s.e0));
+        CU(cudaEventCreate(&s.e1));
+        launch_fill_synthetic(s.Ap, dt == FPM_F64, b, 101, L, 0, 0, L, b, FPM_DIST_PM1, d->s_comp);
+        launch_fill_synthetic(s.Bp, dt == FPM_F64, L, 102, L, 0, 0, b, L, FPM_DIST_PM1, d->s_comp);
+        CU(cudaMemsetAsync(s.C, 0, (size_t)L * L * es, d->s_comp));
     }
-    cudaStream_t s = d->s_comp;
-    launch_fill_synthetic(Ap, dt == FPM_F64, b, 101, L, 0, 0, L, b, FPM_DIST_PM1, s);
-    launch_fill_synthetic(Bp, dt == FPM_F64, L, 102, L, 0, 0, b, L, FPM_DIST_PM1, s);
-    CU(cudaMemsetAsync(C, 0, (size_t)L * L * es, s));
-    cudaEvent_t e0, e1;
-    CU(cudaEventCreate(&e0));
-    CU(cudaEventCreate(&e1));
-    struct EvGuard {
-        cudaEvent_t a, b;
-        ~EvGuard() { cudaEventDestroy(a); cudaEventDestroy(b); }
-    } evg{e0, e1};
 
     for (int j = 0; j < nsizes; ++j) {
         const int64_t Lx = ms[j] * b;
-        auto run = [&]() {
+        auto run = [&](Scratch& s) {
+            const cudaStream_t st = s.d->s_comp;
             if (dt == FPM_F32) {
-                launch_split_rows(static_cast<const float*>(Ap), b, Lx, b, sch, ah, al, sa, s);
-                launch_split_cols(static_cast<const float*>(Bp), L, b, Lx, sch, bh, bl, sb, s);
+                launch_split_rows(static_cast<const float*>(s.Ap), b, Lx, b, sch, s.ah, s.al, s.sa, st);
+                launch_split_cols(static_cast<const float*>(s.Bp), L, b, Lx, sch, s.bh, s.bl, s.sb, st);
                 UpdateArgs a;
-                a.a_hi = ah; a.a_lo = al; a.bt_hi = bh; a.bt_lo = bl;
-                a.sa = sch == SplitScheme::F16X3 ? sa : nullptr;
-                a.sb = sch == SplitScheme::F16X3 ? sb : nullptr;
-                a.C = static_cast<float*>(C);
+                a.a_hi = s.ah; a.a_lo = s.al; a.bt_hi = s.bh; a.bt_lo = s.bl;
+                a.sa = sch == SplitScheme::F16X3 ? s.sa : nullptr;
+                a.sb = sch == SplitScheme::F16X3 ? s.sb : nullptr;
+                a.C = static_cast<float*>(s.C);
                 a.M = Lx; a.Nc = Lx; a.K = b; a.ldc = Lx;
                 a.scheme = sch;
                 a.cta_group = ctx->cta_group;
-                a.num_sms = d->num_sms;
+                a.num_sms = s.d->num_sms;
                 a.raster_group = ctx->raster_group;
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
-                launch_update_f32(a, s);
+                launch_update_f32(a, st);
             } else {
-                launch_transpose_f64(static_cast<const double*>(Bp), L, b, Lx, static_cast<double*>(Bt), s);
-                launch_update_f64(static_cast<const double*>(Ap), b, static_cast<const double*>(Bt),
-                                  static_cast<double*>(C), Lx, Lx, b, Lx, true, s);
+                launch_transpose_f64(static_cast<const double*>(s.Bp), L, b, Lx, static_cast<double*>(s.Bt), st);
+                launch_update_f64(static_cast<const double*>(s.Ap), b, static_cast<const double*>(s.Bt),
+                                  static_cast<double*>(s.C), Lx, Lx, b, Lx, true, st);
             }
         };
-        for (int w = 0; w < 2; ++w) run();
-        std::vector<double> ts;
-        double mean = 0.0, half = 0.0;
+        for (auto& sp : S) {
+            sp->ts.clear();
+            sp->done = false;
+        }
+        for (int w = 0; w < 2; ++w)
+            for (auto& sp : S) {
+                CU(cudaSetDevice(sp->d->cuda_dev));
+                run(*sp);
+            }
         for (int r = 0; r < 50; ++r) {
-            CU(cudaEventRecord(e0, s));
-            run();
-            CU(cudaEventRecord(e1, s));
-            CU(cudaEventSynchronize(e1));
-            ts.push_back(elapsed_ms(e0, e1) * 1e-3);
-            const int nr = (int)ts.size();
-            mean = 0.0;
-            for (double t : ts) mean += t;
-            mean /= nr;
-            double var = 0.0;
-            for (double t : ts) var += (t - mean) * (t - mean);
-            var = nr > 1 ? var / (nr - 1) : 0.0;
-            half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
-            if (nr >= 5 && half <= 0.025 * mean) break;
+            // all devices run every repetition, so contention stays the same until the last converges
+            for (auto& sp : S) {
+                CU(cudaSetDevice(sp->d->cuda_dev));
+                CU(cudaEventRecord(sp->e0, sp->d->s_comp));
+                run(*sp);
+                CU(cudaEventRecord(sp->e1, sp->d->s_comp));
+            }
+            bool all_done = true;
+            for (auto& sp : S) {
+                Scratch& s = *sp;
+                CU(cudaSetDevice(s.d->cuda_dev));
+                CU(cudaEventSynchronize(s.e1));
+                s.ts.push_back(elapsed_ms(s.e0, s.e1) * 1e-3);
+                const int nr = (int)s.ts.size();
+                s.mean = 0.0;
+                for (double t : s.ts) s.mean += t;
+                s.mean /= nr;
+                double var = 0.0;
+                for (double t : s.ts) var += (t - s.mean) * (t - s.mean);
+                var = nr > 1 ? var / (nr - 1) : 0.0;
+                s.half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
+                s.done = nr >= 5 && s.half <= 0.025 * s.mean;
+                all_done = all_done && s.done;
+            }
+            if (all_done) break;
         }
         const double x = (double)(ms[j] * ms[j]);
-        speeds[j] = 2.0 * x * (double)b * (double)b * (double)b / mean;
-        if (ci) ci[j] = mean > 0 ? half / mean : 0.0;
-        if (reps_out) reps_out[j] = (int32_t)ts.size();
+        for (size_t i = 0; i < S.size(); ++i) {
+            const Scratch& s = *S[i];
+            speeds[i * nsizes + j] = 2.0 * x * (double)b * (double)b * (double)b / s.mean;
+            if (ci) ci[i * nsizes + j] = s.mean > 0 ? s.half / s.mean : 0.0;
+            if (reps_out) reps_out[i * nsizes + j] = (int32_t)s.ts.size();
+        }
     }
 }
 

@@ -46,6 +46,8 @@ def main():
     ap.add_argument("--ncal", type=int, default=8192)
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--sizes", default="1,2,3,4,6,8,12,16,20,24,28,32,40")
+    ap.add_argument("--concurrent", dest="exclusive", action="store_false",
+                    help="sample all devices at once (P:10 (ii)) instead of each alone (P:11, default)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
     args = ap.parse_args()
     caps = [int(c) for c in args.caps.split(",")]
@@ -57,8 +59,12 @@ def main():
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
     t0 = time.perf_counter()
     models, sample_info = [], []
-    for dev in range(p):
-        sp, ci, reps = ctx.sample(dev, b, sizes, pkg.FPM_F32)
+    if args.exclusive:   # each device alone (how the paper measured its GPUs)
+        per_dev = [ctx.sample(dev, b, sizes, pkg.FPM_F32) for dev in range(p)]
+    else:                # all devices at once (P:10 (ii)): contention as in the run
+        sps, cis, repss = ctx.sample(-1, b, sizes, pkg.FPM_F32)
+        per_dev = list(zip(sps, cis, repss))
+    for dev, (sp, ci, reps) in enumerate(per_dev):
         models.append((sizes, sp))
         sample_info.append({"cap": caps[dev], "speeds_gflops": [s / 1e9 for s in sp], "rel_ci95": ci, "reps": reps})
     t_sample = time.perf_counter() - t0
@@ -106,7 +112,8 @@ def main():
         st1 = one.compute()
     out = {
         "config": {"N": N, "b": b, "p": p, "sm_caps": caps, "ncal": args.ncal, "x_cal": x_cal, "x_even": x_even,
-                   "sizes": sizes, "dtype": "f32 (F16X3)", "gpu": "1x B200, devices emulated by SM caps"},
+                   "sizes": sizes, "dtype": "f32 (F16X3)", "gpu": "1x B200, devices emulated by SM caps",
+                   "sampling": "exclusive" if args.exclusive else "concurrent (all devices at once)"},
         "fpm_sample_s": t_sample, "models": sample_info, "partitions": results,
         "whole_gpu": {"t_s": st1.t_compute_s, "gflops": st1.gflops},
         "fpm_vs_cpm_ncal_time_delta": results["fpm"]["t_total_s"] / results["cpm_ncal"]["t_total_s"] - 1.0,

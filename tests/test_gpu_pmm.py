@@ -163,6 +163,16 @@ def test_fpm_sample_procedure():
             ctx.sample(0, 256, [3])                        # not a perfect square
 
 
+def test_fpm_sample_all_devices_concurrently():
+    """dev = -1: every device sampled at once (P:10 (ii)); a device capped to
+    fewer SMs must come out slower at a size that fills the GPU."""
+    with pkg.Context.local([0, 0], sm_caps=[96, 32]) as ctx:
+        sp, ci, reps = ctx.sample(-1, 512, [64, 256], pkg.FPM_F32)
+        assert len(sp) == 2 and all(len(r) == 2 for r in sp)
+        assert all(s > 0 for row in sp for s in row)
+        assert sp[0][1] > 1.5 * sp[1][1]
+
+
 def test_config1_fp64_two_capped_devices():
     """BASELINE config 1: N=512, b=64, FP64, two devices with SM caps {144, 48}:
     FPMs from 8 sample sizes -> partition -> arrangement -> multiply."""
