@@ -191,39 +191,76 @@ __global__ void __launch_bounds__(256) fill_k(T* dst, int64_t ld, uint64_t seed,
     }
 }
 
-// ---- FP64 rank-b update on DMMA (mma.sync m8n8k4 f64).  64 x 64 CTA tile,
-// 4 warps of 32 x 32, K staged through shared memory in steps of 16.
-__global__ void __launch_bounds__(128) update_f64_k(const double* __restrict__ A, int64_t lda,
-                                                    const double* __restrict__ Bt, double* __restrict__ C,
-                                                    int64_t M, int64_t Nc, int64_t K, int64_t ldc,
-                                                    int accumulate) {
-    __shared__ double As[64][17];
-    __shared__ double Bs[64][17];
+// ---- FP64 rank-b update on the FP64 tensor path (mma.sync m8n8k4 f64 ->
+// SASS DMMA.8x8x4).  128 x 128 CTA tile, 8 warps of 64 x 32 (8 x 4 DMMA tiles,
+// 64 accumulators per lane), K staged through shared memory in chunks of 32
+// with cp.async double buffering.  Smem rows are padded to 36 doubles so the
+// fragment loads (lane -> row lane/4, column lane%4) hit 16 distinct 8-byte
+// bank pairs per half-warp.
+constexpr int F64_BM = 128, F64_BN = 128, F64_BK = 32, F64_LD = 36;
+constexpr int F64_SMEM = 2 * (F64_BM + F64_BN) * F64_LD * 8;  // 147456 B
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool valid) {
+    const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
+    const int n = valid ? 16 : 0;  // src-size 0 -> zero fill
+    asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
+}
+
+__global__ void __launch_bounds__(256, 1) update_f64_k(const double* __restrict__ A, int64_t lda,
+                                                       const double* __restrict__ Bt, double* __restrict__ C,
+                                                       int64_t M, int64_t Nc, int64_t K, int64_t ldc,
+                                                       int accumulate) {
+    extern __shared__ double sm64[];
+    double* As = sm64;                                  // [2][BM][LD]
+    double* Bs = sm64 + 2 * F64_BM * F64_LD;            // [2][BN][LD]
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int64_t m0 = (int64_t)blockIdx.y * 64, n0 = (int64_t)blockIdx.x * 64;
-    const int wm = (warp / 2) * 32, wn = (warp % 2) * 32;
-    double acc[4][4][2];
+    const int64_t m0 = (int64_t)blockIdx.y * F64_BM, n0 = (int64_t)blockIdx.x * F64_BN;
+    const int wm = (warp / 4) * 64, wn = (warp % 4) * 32;
+    double acc[8][4][2];
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < 8; ++i)
 #pragma unroll
         for (int j = 0; j < 4; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
-    for (int64_t k0 = 0; k0 < K; k0 += 16) {
-        for (int idx = threadIdx.x; idx < 64 * 16; idx += 128) {
-            const int r = idx / 16, c = idx % 16;
-            const int64_t gm = m0 + r, gn = n0 + r, gk = k0 + c;
-            As[r][c] = (gm < M && gk < K) ? A[gm * lda + gk] : 0.0;
-            Bs[r][c] = (gn < Nc && gk < K) ? Bt[gn * K + gk] : 0.0;
+
+    // 128 rows x 32 doubles = 2048 16-B chunks per operand per stage; 8 per thread
+    auto load_stage = [&](int stage, int64_t k0) {
+#pragma unroll
+        for (int it = 0; it < 8; ++it) {
+            const int idx = threadIdx.x + it * 256;
+            const int r = idx / 16, c2 = (idx % 16) * 2;
+            const int64_t gk = k0 + c2;
+            const int64_t gm = m0 + r, gn = n0 + r;
+            const bool ka = gk < K;  // K % 8 == 0, so a 2-element chunk is all in or all out
+            cp_async16(As + (stage * F64_BM + r) * F64_LD + c2, A + (ka && gm < M ? gm * lda + gk : 0),
+                       ka && gm < M);
+            cp_async16(Bs + (stage * F64_BN + r) * F64_LD + c2, Bt + (ka && gn < Nc ? gn * K + gk : 0),
+                       ka && gn < Nc);
+        }
+        asm volatile("cp.async.commit_group;" ::: "memory");
+    };
+
+    const int64_t nk = (K + F64_BK - 1) / F64_BK;
+    load_stage(0, 0);
+    for (int64_t kb = 0; kb < nk; ++kb) {
+        const int st = (int)(kb & 1);
+        if (kb + 1 < nk) {
+            load_stage(st ^ 1, (kb + 1) * F64_BK);
+            asm volatile("cp.async.wait_group 1;" ::: "memory");
+        } else {
+            asm volatile("cp.async.wait_group 0;" ::: "memory");
         }
         __syncthreads();
+        const double* as = As + st * F64_BM * F64_LD;
+        const double* bs = Bs + st * F64_BN * F64_LD;
 #pragma unroll
-        for (int kk = 0; kk < 16; kk += 4) {
-            double a[4], b[4];
+        for (int kk = 0; kk < F64_BK; kk += 4) {
+            double a[8], b[4];
 #pragma unroll
-            for (int i = 0; i < 4; ++i) a[i] = As[wm + i * 8 + lane / 4][kk + lane % 4];
+            for (int i = 0; i < 8; ++i) a[i] = as[(wm + i * 8 + lane / 4) * F64_LD + kk + lane % 4];
 #pragma unroll
-            for (int j = 0; j < 4; ++j) b[j] = Bs[wn + j * 8 + lane / 4][kk + lane % 4];
+            for (int j = 0; j < 4; ++j) b[j] = bs[(wn + j * 8 + lane / 4) * F64_LD + kk + lane % 4];
 #pragma unroll
-            for (int i = 0; i < 4; ++i)
+            for (int i = 0; i < 8; ++i)
 #pragma unroll
                 for (int j = 0; j < 4; ++j)
                     asm volatile(
@@ -234,15 +271,24 @@ __global__ void __launch_bounds__(128) update_f64_k(const double* __restrict__ A
         __syncthreads();
     }
 #pragma unroll
-    for (int i = 0; i < 4; ++i)
+    for (int i = 0; i < 8; ++i)
 #pragma unroll
-        for (int j = 0; j < 4; ++j)
+        for (int j = 0; j < 4; ++j) {
+            const int64_t gm = m0 + wm + i * 8 + lane / 4;
+            const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4);
+            if (gm >= M) continue;
+            double* cp = C + gm * ldc + gn;
+            if (gn + 1 < Nc && (reinterpret_cast<uintptr_t>(cp) & 15) == 0) {
+                double2 c = accumulate ? *reinterpret_cast<double2*>(cp) : make_double2(0.0, 0.0);
+                c.x += acc[i][j][0];
+                c.y += acc[i][j][1];
+                *reinterpret_cast<double2*>(cp) = c;
+            } else {
 #pragma unroll
-            for (int h = 0; h < 2; ++h) {
-                const int64_t gm = m0 + wm + i * 8 + lane / 4;
-                const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4) + h;
-                if (gm < M && gn < Nc) C[gm * ldc + gn] = (accumulate ? C[gm * ldc + gn] : 0.0) + acc[i][j][h];
+                for (int h = 0; h < 2; ++h)
+                    if (gn + h < Nc) cp[h] = (accumulate ? cp[h] : 0.0) + acc[i][j][h];
             }
+        }
 }
 
 int grid_for(int64_t work, int threads) {
@@ -310,8 +356,19 @@ void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t c
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
                        int64_t K, int64_t ldc, bool accumulate, cudaStream_t st) {
     if (M <= 0 || Nc <= 0 || K <= 0) return;
-    dim3 grid((unsigned)((Nc + 63) / 64), (unsigned)((M + 63) / 64));
-    update_f64_k<<<grid, 128, 0, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
+    FPM_CHECK_ARG(K % 8 == 0 && lda % 2 == 0, "FP64 update: K % 8 == 0 and even lda required");
+    FPM_CHECK_ARG((reinterpret_cast<uintptr_t>(A) & 15) == 0 && (reinterpret_cast<uintptr_t>(Bt) & 15) == 0,
+                  "FP64 update: A and Bt must be 16-byte aligned");
+    static uint64_t attr_done = 0;  // one bit per CUDA device
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(attr_done & (1ull << dev))) {
+        cudaError_t e = cudaFuncSetAttribute(update_f64_k, cudaFuncAttributeMaxDynamicSharedMemorySize, F64_SMEM);
+        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute(update_f64): %s", cudaGetErrorString(e));
+        attr_done |= 1ull << dev;
+    }
+    dim3 grid((unsigned)((Nc + F64_BN - 1) / F64_BN), (unsigned)((M + F64_BM - 1) / F64_BM));
+    update_f64_k<<<grid, 256, F64_SMEM, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
     check_launch("update_f64");
 }
 
