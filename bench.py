@@ -105,6 +105,18 @@ def measured_peaks() -> dict:
     return {"bf16_burst": 1590.0, "bf16_sustained": 1400.0, "hbm_gbs": 6650.0, "source": "fallback"}
 
 
+def committed_traffic(N: int, b: int, args):
+    """DRAM bytes per update launch from the committed ncu capture of the same
+    configuration (profiles/ncu_traffic.json), else None."""
+    path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    variant = 2 if args.kernel_variant < 0 else args.kernel_variant
+    key = f"{N}_{b}_{args.scheme}_v{variant}"
+    if args.gpus != 1 or not os.path.exists(path):
+        return None
+    entry = json.load(open(path)).get(key)
+    return entry["dram_bytes_per_launch"] if entry else None
+
+
 # ----------------------------------------------------------------- oracle
 def oracle_sample(N: int, reps: int = 1):
     """Time the CPU oracle (plain triple loop, FP64 accumulation) on the block
@@ -271,7 +283,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     dense_peak = peaks["bf16_sustained"] if args.scheme == "f16x3" else peaks["bf16_sustained"] / 2.0
     peak = dense_peak / mma_per_mac
     roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
-                "frac": achieved / peak if peak else None, "traffic": args.traffic,
+                "frac": achieved / peak if peak else None,
+                "traffic": args.traffic if args.traffic is not None else committed_traffic(N, b, args),
                 "peak_basis": (f"{'fp16' if args.scheme == 'f16x3' else 'tf32'} dense tensor peak "
                                f"({peaks['source']} {dense_peak:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC"),
                 "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None}
