@@ -110,7 +110,8 @@ def committed_traffic(N: int, b: int, args):
     configuration (profiles/ncu_traffic.json), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     variant = 2 if args.kernel_variant < 0 else args.kernel_variant
-    key = f"{N}_{b}_{args.scheme}_v{variant}"
+    fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
+    key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}")
     if args.gpus != 1 or not os.path.exists(path):
         return None
     entry = json.load(open(path)).get(key)
@@ -193,6 +194,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     ctx.set_option("raster_group", args.raster_group)
     ctx.set_option("l2_hint_b", args.l2_hint_b)
     ctx.set_option("kernel_variant", args.kernel_variant)
+    ctx.set_option("fuse", args.fuse)
 
     # ---- FPMs (offline): sample this GPU's speed function once;
     # every rank's model is gathered so all ranks partition identically.
@@ -272,13 +274,15 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     live_t = [t for t in pred_t if t > 0]
     imb_pred = max(live_t) / (sum(live_t) / len(live_t)) - 1.0 if live_t else 0.0
 
-    # ---- roofline of the dominant kernel (rank-b update): algorithmic flops per
-    # launch = 2 H W b, over the mean launch duration (CUDA events on its stream).
+    # ---- roofline of the dominant kernel (rank-(f b) update): algorithmic flops per
+    # launch = 2 H W f b, over the launch duration (CUDA events on its stream);
+    # per step: 2 H W b n flop over the summed update time.
     peaks = measured_peaks()
     r = rects[rank]
     H, W = r[3] * b, r[4] * b
-    upd_mean = statistics.median(upd_times) / n
-    achieved = 2.0 * H * W * b / upd_mean / 1e12 if upd_mean > 0 else 0.0
+    upd_launches = st.updates
+    upd_step = statistics.median(upd_times)
+    achieved = 2.0 * H * W * b * n / upd_step / 1e12 if upd_step > 0 else 0.0
     mma_per_mac = 3.0  # F16X3 and TF32X3 both issue three tensor-core products per FP32 MAC
     dense_peak = peaks["bf16_sustained"] if args.scheme == "f16x3" else peaks["bf16_sustained"] / 2.0
     peak = dense_peak / mma_per_mac
@@ -312,7 +316,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
                 "N": N, "b": b, "p": p, "partition": d, "rects": rects,
                 "f32_scheme": args.scheme, "cta_group": args.cta_group, "raster_group": args.raster_group,
-                "kernel_variant": args.kernel_variant,
+                "kernel_variant": args.kernel_variant, "fuse": args.fuse,
+                "update_launches_per_step": upd_launches,
                 "transport": (args.transport if world > 1 else "none (p = 1)"),
                 "l2": "inputs larger than L2 (A, B, C 9.7 GB each)",
                 "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
@@ -397,6 +402,7 @@ def main():
     ap.add_argument("--raster-group", type=int, default=16)
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
+    ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")

@@ -91,6 +91,7 @@ typedef struct {
     int64_t iters;                              /* n = N / b                                      */
     int64_t comm_bytes;                         /* pivot bytes received by this process's devices */
     int64_t kernel_launches;                    /* library kernels launched in the k-loop         */
+    int64_t updates;                            /* rank-(f b) update launches (f pivots fused)    */
 } pmm_stats;
 
 typedef struct pmm_ctx pmm_ctx;
@@ -246,6 +247,12 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  DESIGN.md Q15.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
  *   "kernel_variant": -1 (auto, default) or 0..3, see fpm_k_update_f32.
+ *   "fuse":       pivots fused into one rank-(f b) update (FP32): 0 = auto
+ *                 (f = min(8, max(1, 2048 / b))), else 1..8.  Groups never
+ *                 straddle a column or row boundary of the arrangement, so a
+ *                 group's exchange is its first pivot's plan with f-times longer
+ *                 panels; the F16X3 scales are taken over the fused rows.  Halves
+ *                 (f = 2) the C read-modify-write traffic of the iteration loop.
  *   "raster_group": tile-rows per L2 raster group of the update (default 16).
  *   "l2_hint_b":  L2 policy of the B^T operand tiles: 0 normal (default),
  *                 1 evict-first, 2 evict-last.

@@ -50,7 +50,7 @@ class PmmStats(ctypes.Structure):
         ("t_compute_s", dbl), ("t_upload_s", dbl), ("t_download_s", dbl),
         ("per_dev_compute_s", dbl * FPM_MAX_DEVICES), ("per_dev_update_s", dbl * FPM_MAX_DEVICES),
         ("gflops", dbl), ("imbalance", dbl), ("iters", i64), ("comm_bytes", i64),
-        ("kernel_launches", i64),
+        ("kernel_launches", i64), ("updates", i64),
     ]
 
     def as_dict(self, p: int | None = None) -> dict:
@@ -61,7 +61,7 @@ class PmmStats(ctypes.Structure):
             "per_dev_compute_s": list(self.per_dev_compute_s[:p]),
             "per_dev_update_s": list(self.per_dev_update_s[:p]),
             "gflops": self.gflops, "imbalance": self.imbalance, "iters": self.iters,
-            "comm_bytes": self.comm_bytes, "kernel_launches": self.kernel_launches,
+            "comm_bytes": self.comm_bytes, "kernel_launches": self.kernel_launches, "updates": self.updates,
         }
 
 

@@ -44,6 +44,12 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st);
 void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, SplitScheme s, void* hi,
                        void* lo, float* inv_scale, cudaStream_t st);
 
+// Fused pivots: row r of the operand is nseg segments of K elements, segment j
+// at src + j*seg_stride + r*ld; output row stride ld_out (>= nseg*K); the F16X3
+// scale is taken over the whole fused row.
+void launch_split_rows_seg(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t rows, int64_t K,
+                           int64_t ld_out, SplitScheme s, void* hi, void* lo, float* inv_scale, cudaStream_t st);
+
 // B pivot row src (K x W, row stride ld) -> split halves of its transpose
 // (W x K, K-major), per-row (= per-column of src) inverse scales for F16X3.
 void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,

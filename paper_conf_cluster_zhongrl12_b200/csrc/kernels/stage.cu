@@ -25,20 +25,26 @@ __device__ __forceinline__ float warp_max(float v) {
     return v;
 }
 
-// One warp per row.  F16X3: choose 2^s with the row max scaled into [2^14, 2^15),
-// h0 = fp16(x 2^s), h1 = fp16(x 2^s - h0); inv_scale = 2^-s.
-__global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ src, int64_t ld, int64_t rows,
-                                                      int64_t K, __half* __restrict__ hi, __half* __restrict__ lo,
+// One warp per row.  A row of the operand is nseg segments of K elements, segment
+// j at src + j * seg_stride + row * ld (the panels of nseg consecutive pivots
+// fused into one update); it is written to out + row * ld_out + j * K.
+// F16X3: choose 2^s with the maximum of the whole (fused) row scaled into
+// [2^14, 2^15), h0 = fp16(x 2^s), h1 = fp16(x 2^s - h0); inv_scale = 2^-s.
+__global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ src, int64_t ld, int64_t seg_stride,
+                                                      int nseg, int64_t rows, int64_t K, int64_t ld_out,
+                                                      __half* __restrict__ hi, __half* __restrict__ lo,
                                                       float* __restrict__ inv_scale) {
     const int64_t row = (int64_t)blockIdx.x * 8 + threadIdx.x / 32;
     const int lane = threadIdx.x % 32;
     if (row >= rows) return;
-    const float4* s4 = reinterpret_cast<const float4*>(src + row * ld);
     const int64_t n4 = K / 4;
     float m = 0.0f;
-    for (int64_t i = lane; i < n4; i += 32) {
-        const float4 v = s4[i];
-        m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+    for (int j = 0; j < nseg; ++j) {
+        const float4* s4 = reinterpret_cast<const float4*>(src + j * seg_stride + row * ld);
+        for (int64_t i = lane; i < n4; i += 32) {
+            const float4 v = s4[i];
+            m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+        }
     }
     m = warp_max(m);
     int e = 0;
@@ -49,39 +55,45 @@ __global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ 
     s = s < -126 ? -126 : (s > 127 ? 127 : s);
     const float scale = ldexpf(1.0f, s);
     if (lane == 0) inv_scale[row] = ldexpf(1.0f, -s);
-    __half2* h2 = reinterpret_cast<__half2*>(hi + row * K);
-    __half2* l2 = reinterpret_cast<__half2*>(lo + row * K);
-    for (int64_t i = lane; i < n4; i += 32) {
-        const float4 v = s4[i];
-        const float x[4] = {v.x * scale, v.y * scale, v.z * scale, v.w * scale};
-        __half h[4], l[4];
+    for (int j = 0; j < nseg; ++j) {
+        const float4* s4 = reinterpret_cast<const float4*>(src + j * seg_stride + row * ld);
+        __half2* h2 = reinterpret_cast<__half2*>(hi + row * ld_out + j * K);
+        __half2* l2 = reinterpret_cast<__half2*>(lo + row * ld_out + j * K);
+        for (int64_t i = lane; i < n4; i += 32) {
+            const float4 v = s4[i];
+            const float x[4] = {v.x * scale, v.y * scale, v.z * scale, v.w * scale};
+            __half h[4], l[4];
 #pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            h[j] = __float2half_rn(x[j]);
-            l[j] = __float2half_rn(x[j] - __half2float(h[j]));
+            for (int q = 0; q < 4; ++q) {
+                h[q] = __float2half_rn(x[q]);
+                l[q] = __float2half_rn(x[q] - __half2float(h[q]));
+            }
+            h2[2 * i] = __halves2half2(h[0], h[1]);
+            h2[2 * i + 1] = __halves2half2(h[2], h[3]);
+            l2[2 * i] = __halves2half2(l[0], l[1]);
+            l2[2 * i + 1] = __halves2half2(l[2], l[3]);
         }
-        h2[2 * i] = __halves2half2(h[0], h[1]);
-        h2[2 * i + 1] = __halves2half2(h[2], h[3]);
-        l2[2 * i] = __halves2half2(l[0], l[1]);
-        l2[2 * i + 1] = __halves2half2(l[2], l[3]);
     }
 }
 
-__global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__ src, int64_t ld, int64_t rows,
-                                                       int64_t K, float* __restrict__ hi, float* __restrict__ lo) {
+__global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__ src, int64_t ld, int64_t seg_stride,
+                                                       int nseg, int64_t rows, int64_t K, int64_t ld_out,
+                                                       float* __restrict__ hi, float* __restrict__ lo) {
     const int64_t n4 = K / 4;
-    const int64_t total = rows * n4;
+    const int64_t per_row = nseg * n4;
+    const int64_t total = rows * per_row;
     for (int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; idx < total;
          idx += (int64_t)gridDim.x * blockDim.x) {
-        const int64_t r = idx / n4, c = idx - r * n4;
-        const float4 v = reinterpret_cast<const float4*>(src + r * ld)[c];
+        const int64_t r = idx / per_row, rem = idx - r * per_row;
+        const int64_t j = rem / n4, c = rem - j * n4;
+        const float4 v = reinterpret_cast<const float4*>(src + j * seg_stride + r * ld)[c];
         float4 h, l;
         h.x = tf32_rna(v.x); l.x = tf32_rna(v.x - h.x);
         h.y = tf32_rna(v.y); l.y = tf32_rna(v.y - h.y);
         h.z = tf32_rna(v.z); l.z = tf32_rna(v.z - h.z);
         h.w = tf32_rna(v.w); l.w = tf32_rna(v.w - h.w);
-        reinterpret_cast<float4*>(hi + r * K)[c] = h;
-        reinterpret_cast<float4*>(lo + r * K)[c] = l;
+        reinterpret_cast<float4*>(hi + r * ld_out + j * K)[c] = h;
+        reinterpret_cast<float4*>(lo + r * ld_out + j * K)[c] = l;
     }
 }
 
@@ -308,20 +320,27 @@ void check_launch(const char* what) {
 
 }  // namespace
 
-void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, SplitScheme s, void* hi, void* lo,
-                       float* inv_scale, cudaStream_t st) {
-    if (rows <= 0 || K <= 0) return;
-    FPM_CHECK_ARG(K % 4 == 0 && ld % 4 == 0, "split: K and ld must be multiples of 4");
+void launch_split_rows_seg(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t rows, int64_t K,
+                           int64_t ld_out, SplitScheme s, void* hi, void* lo, float* inv_scale, cudaStream_t st) {
+    if (rows <= 0 || K <= 0 || nseg <= 0) return;
+    FPM_CHECK_ARG(K % 4 == 0 && ld % 4 == 0 && seg_stride % 4 == 0 && ld_out % 4 == 0 && ld_out >= nseg * K,
+                  "split: K, ld, seg_stride, ld_out must be multiples of 4 and ld_out >= nseg*K");
     if (s == SplitScheme::F16X3) {
         const int64_t blocks = (rows + 7) / 8;
-        split_rows_f16<<<(unsigned)blocks, 256, 0, st>>>(src, ld, rows, K, static_cast<__half*>(hi),
-                                                         static_cast<__half*>(lo), inv_scale);
+        split_rows_f16<<<(unsigned)blocks, 256, 0, st>>>(src, ld, seg_stride, nseg, rows, K, ld_out,
+                                                         static_cast<__half*>(hi), static_cast<__half*>(lo),
+                                                         inv_scale);
         check_launch("split_rows_f16");
     } else {
-        split_rows_tf32<<<grid_for(rows * K / 4, 256), 256, 0, st>>>(src, ld, rows, K, static_cast<float*>(hi),
-                                                                      static_cast<float*>(lo));
+        split_rows_tf32<<<grid_for(rows * nseg * K / 4, 256), 256, 0, st>>>(
+            src, ld, seg_stride, nseg, rows, K, ld_out, static_cast<float*>(hi), static_cast<float*>(lo));
         check_launch("split_rows_tf32");
     }
+}
+
+void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, SplitScheme s, void* hi, void* lo,
+                       float* inv_scale, cudaStream_t st) {
+    launch_split_rows_seg(src, ld, 0, 1, rows, K, K, s, hi, lo, inv_scale, st);
 }
 
 void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,

@@ -92,7 +92,10 @@ struct pmm_ctx {
     int cta_group = 2;
     int raster_group = 16;
     int l2_hint_b = 0;
-    int kernel_variant = -1;  // auto (by K)
+    int kernel_variant = -1;  // auto
+    int fuse = 0;             // pivots per update (0 = auto)
+    int fuse_max = 1;         // resolved for the current problem
+    std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
 };
 
 namespace fpm {
@@ -201,6 +204,15 @@ const void* src_B(pmm_ctx* ctx, int q) {
     return local_dev(ctx, q)->B;
 }
 
+// Pivots fused per update (FP32 only): option "fuse", 0 = auto = K of about 2048
+// (measured on B200: f = 2 at b = 1024 gives 419 vs 392 TFLOP/s unfused and
+// beats f = 3, 4; at b = 512, f = 2..8 give 404-406 vs 332 unfused).
+int fuse_factor(pmm_ctx* ctx, fpm_dtype dt, int64_t b) {
+    if (dt != FPM_F32) return 1;
+    if (ctx->fuse > 0) return ctx->fuse;
+    return (int)std::max<int64_t>(1, std::min<int64_t>(8, 2048 / b));
+}
+
 // ---------------------------------------------------------------- setup
 void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects, fpm_dtype dt) {
     FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype %d", (int)dt);
@@ -227,6 +239,27 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
     ctx->plan_b.assign(n, {});
     for (int64_t k = 0; k < n; ++k) plan_step(n, p, rects, k, ctx->plan_a[k], ctx->plan_b[k]);
 
+    // Update groups: f consecutive pivots fused into one rank-(f b) update, never
+    // across a column boundary (one set of A holders per group) nor a row
+    // boundary of any device (one B owner per column per group), so a group's
+    // exchange is the plan of its first pivot with longer panels.
+    const int f = fuse_factor(ctx, dt, b);
+    std::vector<int64_t> cuts;
+    for (int q = 0; q < p; ++q)
+        if (rects[q].h > 0 && rects[q].w > 0) {
+            cuts.push_back(rects[q].col0);
+            cuts.push_back(rects[q].row0);
+        }
+    ctx->groups.clear();
+    for (int64_t k = 0; k < n;) {
+        int64_t size = std::min<int64_t>(f, n - k);
+        for (int64_t c : cuts)
+            if (c > k && c < k + size) size = c - k;
+        ctx->groups.push_back({k, (int)size});
+        k += size;
+    }
+    ctx->fuse_max = f;
+
     const size_t es = esize(dt);
     for (auto& d : ctx->devs) {
         CU(cudaSetDevice(d.cuda_dev));
@@ -245,17 +278,18 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         // receive buffers: NCCL lands pivots in them; FP64 copies peers' pivots into
         // them.  FP32 in local / IPC mode stages straight from the peers' memory.
         const bool need_recv = ctx->nccl_mode || dt == FPM_F64;
+        const size_t fb = (size_t)f * b;  // K of a fused update
         for (int s = 0; s < 2; ++s) {
             if (need_recv) {
-                d.a_recv[s] = dalloc(d, (size_t)d.H * b * es);
-                d.b_recv[s] = dalloc(d, (size_t)b * d.W * es);
+                d.a_recv[s] = dalloc(d, (size_t)d.H * fb * es);  // f panels of H x b
+                d.b_recv[s] = dalloc(d, fb * d.W * es);          // f block-rows of b x W
             }
             if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * b * es);
             if (dt == FPM_F32) {
-                d.a_hi[s] = dalloc(d, (size_t)d.H * b * op);
-                d.a_lo[s] = dalloc(d, (size_t)d.H * b * op);
-                d.b_hi[s] = dalloc(d, (size_t)d.W * b * op);
-                d.b_lo[s] = dalloc(d, (size_t)d.W * b * op);
+                d.a_hi[s] = dalloc(d, (size_t)d.H * fb * op);
+                d.a_lo[s] = dalloc(d, (size_t)d.H * fb * op);
+                d.b_hi[s] = dalloc(d, (size_t)d.W * fb * op);
+                d.b_lo[s] = dalloc(d, (size_t)d.W * fb * op);
                 d.sa[s] = static_cast<float*>(dalloc(d, (size_t)d.H * sizeof(float)));
                 d.sb[s] = static_cast<float*>(dalloc(d, (size_t)d.W * sizeof(float)));
             }
@@ -321,120 +355,135 @@ void issue_upload(pmm_ctx* ctx, Device& d, int64_t k, const HostSrc& h) {
     CU(cudaEventRecord(d.ev_up[k], d.s_comm));
 }
 
-// Exchange + staging of iteration k on device d's comm stream.
-int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use, bool streamed) {
+// Exchange + staging of update group g (pivots k0 .. k0+f-1) on device d's comm
+// stream.  All pivots of a group share their holders and owners (setup), so the
+// group moves as the plan of k0 with f-times longer panels.
+int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, bool streamed) {
     const size_t es = esize(ctx->dt);
     const int64_t b = ctx->b;
+    const int64_t k0 = ctx->groups[g].first;
+    const int f = ctx->groups[g].second;
+    const int64_t kl = k0 + f - 1;  // last pivot of the group
+    const int64_t fb = (int64_t)f * b;
     int64_t bytes = 0;
     CU(cudaSetDevice(d.cuda_dev));
     if (!first_use) CU(cudaStreamWaitEvent(d.s_comm, d.ev_free[slot], 0));
     const colpart_rect& r = d.rect;
 
-    // FP32 in local / IPC mode: the staging kernels read the pivot straight from
+    // FP32 in local / IPC mode: the staging kernels read the pivots straight from
     // the holder's / owner's resident buffer (peer memory over NVLink, or the same
     // GPU), so the transfer is fused into the split -- no receive buffer, no copy.
     const bool fused = ctx->dt == FPM_F32 && !ctx->nccl_mode;
     struct Piece {
-        const void* src;
-        int64_t row_off, rows;  // in elements (rows of my H x b panel)
+        const void* src;        // first pivot's rows; pivot j at src + j * seg_stride
+        int64_t seg_stride;     // elements between consecutive pivot panels of the holder
+        int64_t row_off, rows;  // in elements (rows of my H x b panels)
     };
     std::vector<Piece> a_pieces;
 
-    // ---- A(rows_i, k): local if this device's column holds block-column k
-    const bool holder = r.col0 <= k && k < r.col0 + r.w;
-    const void* a_src = nullptr;
+    // ---- A(rows_i, k0..kl): local if this device's column holds the block-columns
+    const bool holder = r.col0 <= k0 && k0 < r.col0 + r.w;
+    const void* a_src = nullptr;  // f contiguous H x b panels (holder / received)
     if (holder) {
-        a_src = static_cast<const char*>(d.A) + (size_t)(k - r.col0) * d.H * b * es;
+        a_src = static_cast<const char*>(d.A) + (size_t)(k0 - r.col0) * d.H * b * es;
     } else if (ctx->nccl_mode) {
         a_src = d.a_recv[slot];
     } else {
-        for (const Move& m : ctx->plan_a[k]) {
+        for (const Move& m : ctx->plan_a[k0]) {
             if (m.dst != d.idx) continue;
             const colpart_rect& qr = ctx->rects[m.src];
+            const int64_t qH = qr.h * b;
             const size_t cnt = (size_t)(m.end - m.begin) * b * b;
             const char* src = static_cast<const char*>(src_A(ctx, m.src)) +
-                              ((size_t)(k - qr.col0) * qr.h * b * b + (size_t)(m.begin - qr.row0) * b * b) * es;
-            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[k], 0));
+                              ((size_t)(k0 - qr.col0) * qH * b + (size_t)(m.begin - qr.row0) * b * b) * es;
+            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[kl], 0));
             if (fused) {
-                a_pieces.push_back(Piece{src, (m.begin - r.row0) * b, (m.end - m.begin) * b});
-            } else {
-                char* dst = static_cast<char*>(d.a_recv[slot]) + (size_t)(m.begin - r.row0) * b * b * es;
-                CU(cudaMemcpyAsync(dst, src, cnt * es, cudaMemcpyDefault, d.s_comm));
+                a_pieces.push_back(Piece{src, qH * b, (m.begin - r.row0) * b, (m.end - m.begin) * b});
+            } else {  // FP64: copy the f panels' rows into the receive buffer
+                for (int j = 0; j < f; ++j) {
+                    char* dst = static_cast<char*>(d.a_recv[slot]) +
+                                ((size_t)j * d.H * b + (size_t)(m.begin - r.row0) * b * b) * es;
+                    CU(cudaMemcpyAsync(dst, src + (size_t)j * qH * b * es, cnt * es, cudaMemcpyDefault, d.s_comm));
+                }
                 a_src = d.a_recv[slot];
             }
-            bytes += (int64_t)(cnt * es);
+            bytes += (int64_t)(cnt * es) * f;
         }
     }
-    // ---- B(k, cols_i): local if this device's rows hold block-row k
-    const bool owner = r.row0 <= k && k < r.row0 + r.h;
-    const void* b_src = nullptr;
+    // ---- B(k0..kl, cols_i): local if this device's rows hold the block-rows
+    const bool owner = r.row0 <= k0 && k0 < r.row0 + r.h;
+    const void* b_src = nullptr;  // f b x W rows, contiguous
     if (owner) {
-        b_src = static_cast<const char*>(d.B) + (size_t)(k - r.row0) * b * d.W * es;
+        b_src = static_cast<const char*>(d.B) + (size_t)(k0 - r.row0) * b * d.W * es;
     } else if (ctx->nccl_mode) {
         b_src = d.b_recv[slot];
     } else {
-        for (const Move& m : ctx->plan_b[k]) {
+        for (const Move& m : ctx->plan_b[k0]) {
             if (m.dst != d.idx) continue;
             const colpart_rect& orr = ctx->rects[m.src];
-            const char* src = static_cast<const char*>(src_B(ctx, m.src)) + (size_t)(k - orr.row0) * b * d.W * es;
-            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[k], 0));
+            const char* src = static_cast<const char*>(src_B(ctx, m.src)) + (size_t)(k0 - orr.row0) * b * d.W * es;
+            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[kl], 0));
             if (fused) {
                 b_src = src;
             } else {
-                CU(cudaMemcpyAsync(d.b_recv[slot], src, (size_t)b * d.W * es, cudaMemcpyDefault, d.s_comm));
+                CU(cudaMemcpyAsync(d.b_recv[slot], src, (size_t)fb * d.W * es, cudaMemcpyDefault, d.s_comm));
                 b_src = d.b_recv[slot];
             }
-            bytes += (int64_t)((size_t)b * d.W * es);
+            bytes += (int64_t)((size_t)fb * d.W * es);
         }
     }
     if (ctx->nccl_mode) {
         const NcclApi& nc = nccl();
         const ncclDataType_t ndt = nccl_dtype(ctx->dt);
         NC(nc.GroupStart());
-        for (const Move& m : ctx->plan_a[k]) {
-            if (m.src == m.dst) continue;
-            const size_t cnt = (size_t)(m.end - m.begin) * b * b;
-            if (m.src == d.idx) {
-                const char* src = static_cast<const char*>(d.A) +
-                                  ((size_t)(k - r.col0) * d.H * b + (size_t)(m.begin - r.row0) * b * b) * es;
-                NC(nc.Send(src, cnt, ndt, m.dst, ctx->world_comm, d.s_comm));
-            } else if (m.dst == d.idx) {
-                char* dst = static_cast<char*>(d.a_recv[slot]) + (size_t)(m.begin - r.row0) * b * b * es;
-                NC(nc.Recv(dst, cnt, ndt, m.src, ctx->world_comm, d.s_comm));
-                bytes += (int64_t)(cnt * es);
+        for (int j = 0; j < f; ++j) {
+            const int64_t k = k0 + j;
+            for (const Move& m : ctx->plan_a[k]) {
+                if (m.src == m.dst) continue;
+                const size_t cnt = (size_t)(m.end - m.begin) * b * b;
+                if (m.src == d.idx) {
+                    const char* src = static_cast<const char*>(d.A) +
+                                      ((size_t)(k - r.col0) * d.H * b + (size_t)(m.begin - r.row0) * b * b) * es;
+                    NC(nc.Send(src, cnt, ndt, m.dst, ctx->world_comm, d.s_comm));
+                } else if (m.dst == d.idx) {
+                    char* dst = static_cast<char*>(d.a_recv[slot]) +
+                                ((size_t)j * d.H * b + (size_t)(m.begin - r.row0) * b * b) * es;
+                    NC(nc.Recv(dst, cnt, ndt, m.src, ctx->world_comm, d.s_comm));
+                    bytes += (int64_t)(cnt * es);
+                }
             }
         }
         NC(nc.GroupEnd());
         if (ctx->col_members.size() > 1) {
             int owner_rank = -1;
-            for (const Move& m : ctx->plan_b[k])
+            for (const Move& m : ctx->plan_b[k0])
                 if (m.dst == d.idx) owner_rank = m.src;
             const int root = (int)(std::find(ctx->col_members.begin(), ctx->col_members.end(), owner_rank) -
                                    ctx->col_members.begin());
             void* buf = owner ? const_cast<void*>(b_src) : d.b_recv[slot];
-            NC(nc.Broadcast(buf, buf, (size_t)b * d.W, ndt, root, ctx->col_comm, d.s_comm));
-            if (!owner) bytes += (int64_t)((size_t)b * d.W * es);
+            NC(nc.Broadcast(buf, buf, (size_t)fb * d.W, ndt, root, ctx->col_comm, d.s_comm));
+            if (!owner) bytes += (int64_t)((size_t)fb * d.W * es);
         }
     }
 
-    // ---- staging: K-major operands for the update
-    CU(cudaEventRecord(d.ev_pack0[k], d.s_comm));
+    // ---- staging: K-major operands of the fused update (K = f b)
+    CU(cudaEventRecord(d.ev_pack0[g], d.s_comm));
     if (ctx->dt == FPM_F32) {
         const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
         const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
         d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + 1;
-        if (a_src) {
-            launch_split_rows(static_cast<const float*>(a_src), b, d.H, b, sch, d.a_hi[slot], d.a_lo[slot],
-                              d.sa[slot], d.s_comm);
+        if (a_src) {  // own or received panels: f consecutive H x b panels
+            launch_split_rows_seg(static_cast<const float*>(a_src), b, d.H * b, f, d.H, b, fb, sch,
+                                  d.a_hi[slot], d.a_lo[slot], d.sa[slot], d.s_comm);
         } else {
             for (const Piece& pc : a_pieces)
-                launch_split_rows(static_cast<const float*>(pc.src), b, pc.rows, b, sch,
-                                  static_cast<char*>(d.a_hi[slot]) + (size_t)pc.row_off * b * op,
-                                  static_cast<char*>(d.a_lo[slot]) + (size_t)pc.row_off * b * op,
-                                  d.sa[slot] + pc.row_off, d.s_comm);
+                launch_split_rows_seg(static_cast<const float*>(pc.src), b, pc.seg_stride, f, pc.rows, b, fb, sch,
+                                      static_cast<char*>(d.a_hi[slot]) + (size_t)pc.row_off * fb * op,
+                                      static_cast<char*>(d.a_lo[slot]) + (size_t)pc.row_off * fb * op,
+                                      d.sa[slot] + pc.row_off, d.s_comm);
         }
-        FPM_CHECK_ARG(b_src != nullptr, "no source of block-row %lld for device %d", (long long)k, d.idx);
-        launch_split_cols(static_cast<const float*>(b_src), d.W, b, d.W, sch, d.b_hi[slot], d.b_lo[slot],
+        FPM_CHECK_ARG(b_src != nullptr, "no source of block-row %lld for device %d", (long long)k0, d.idx);
+        launch_split_cols(static_cast<const float*>(b_src), d.W, fb, d.W, sch, d.b_hi[slot], d.b_lo[slot],
                           d.sb[slot], d.s_comm);
     } else {
         d.a_op[slot] = a_src;
@@ -442,15 +491,17 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int64_t k, int slot, bool first_use,
                              d.s_comm);
         d.launches += 1;
     }
-    CU(cudaEventRecord(d.ev_pack1[k], d.s_comm));
+    CU(cudaEventRecord(d.ev_pack1[g], d.s_comm));
     CU(cudaEventRecord(d.ev_ready[slot], d.s_comm));
     return bytes;
 }
 
-void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
+void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
+    const int64_t k0 = ctx->groups[g].first;
+    const int f = ctx->groups[g].second;
     CU(cudaSetDevice(d.cuda_dev));
     CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
-    CU(cudaEventRecord(d.ev_upd0[k], d.s_comp));
+    CU(cudaEventRecord(d.ev_upd0[g], d.s_comp));
     if (ctx->dt == FPM_F32) {
         UpdateArgs a;
         a.a_hi = d.a_hi[slot];
@@ -463,22 +514,22 @@ void issue_update(pmm_ctx* ctx, Device& d, int64_t k, int slot) {
         a.C = static_cast<float*>(d.C);
         a.M = d.H;
         a.Nc = d.W;
-        a.K = ctx->b;
+        a.K = (int64_t)f * ctx->b;
         a.ldc = d.W;
         a.scheme = (SplitScheme)ctx->f32_scheme;
         a.cta_group = ctx->cta_group;
         a.num_sms = d.num_sms;
-        a.accumulate = k != 0;  // iteration 0 writes C = A(0) B(0): no zeroing, no read of C
+        a.accumulate = k0 != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
         a.raster_group = ctx->raster_group;
         a.l2_hint_b = ctx->l2_hint_b;
         a.variant = ctx->kernel_variant;
         launch_update_f32(a, d.s_comp);
     } else {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
-                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k != 0, d.s_comp);
+                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k0 != 0, d.s_comp);
     }
     d.launches += 1;
-    CU(cudaEventRecord(d.ev_upd1[k], d.s_comp));
+    CU(cudaEventRecord(d.ev_upd1[g], d.s_comp));
     CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
 }
 
@@ -505,17 +556,20 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
     }
     const bool streamed = host != nullptr;
     int64_t bytes = 0;
-    for (int64_t k = 0; k < ctx->n; ++k) {
-        const int slot = (int)(k & 1);
+    const int ngroups = (int)ctx->groups.size();
+    for (int g = 0; g < ngroups; ++g) {
+        const int slot = g & 1;
+        const int64_t k0 = ctx->groups[g].first;
         if (streamed)
-            for (auto& d : ctx->devs)
-                if (d.live()) issue_upload(ctx, d, k, *host);
+            for (int64_t k = k0; k < k0 + ctx->groups[g].second; ++k)
+                for (auto& d : ctx->devs)
+                    if (d.live()) issue_upload(ctx, d, k, *host);
         if (ctx->nccl_mode) {
             // every rank takes part in the NCCL calls, live or not
             Device& d = ctx->devs[0];
             if (d.live()) {
-                bytes += issue_comm(ctx, d, k, slot, k < 2, streamed);
-                issue_update(ctx, d, k, slot);
+                bytes += issue_comm(ctx, d, g, slot, g < 2, streamed);
+                issue_update(ctx, d, g, slot);
             } else {
                 NC(nccl().GroupStart());
                 NC(nccl().GroupEnd());
@@ -523,9 +577,9 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
             continue;
         }
         for (auto& d : ctx->devs)
-            if (d.live()) bytes += issue_comm(ctx, d, k, slot, k < 2, streamed);
+            if (d.live()) bytes += issue_comm(ctx, d, g, slot, g < 2, streamed);
         for (auto& d : ctx->devs)
-            if (d.live()) issue_update(ctx, d, k, slot);
+            if (d.live()) issue_update(ctx, d, g, slot);
     }
     int64_t launches = -launches0;
     for (auto& d : ctx->devs) launches += d.launches;
@@ -550,6 +604,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
             st->t_upload_s = tu;
         }
         st->iters = ctx->n;
+        st->updates = ngroups;
         st->comm_bytes = bytes;
         st->kernel_launches = launches;
         st->gflops = t_max > 0 ? 2.0 * (double)ctx->N * (double)ctx->N * (double)ctx->N / t_max * 1e-9 : 0.0;
@@ -558,9 +613,9 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         for (auto& d : ctx->devs) {
             if (!d.live()) continue;
             double comp = 0.0, upd = 0.0;
-            for (int64_t k = 0; k < ctx->n; ++k) {
-                const double u = elapsed_ms(d.ev_upd0[k], d.ev_upd1[k]) * 1e-3;
-                comp += u + elapsed_ms(d.ev_pack0[k], d.ev_pack1[k]) * 1e-3;
+            for (int g = 0; g < ngroups; ++g) {
+                const double u = elapsed_ms(d.ev_upd0[g], d.ev_upd1[g]) * 1e-3;
+                comp += u + elapsed_ms(d.ev_pack0[g], d.ev_pack1[g]) * 1e-3;
                 upd += u;
             }
             if (d.idx < FPM_MAX_DEVICES) {
@@ -711,6 +766,9 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
     const size_t es = dt == FPM_F64 ? 8 : 4;
     const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
     const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
+    // the kernel as the k-loop runs it: f fused pivots per update (K = f b)
+    const int f = fuse_factor(ctx, dt, b);
+    const int64_t fb = (int64_t)f * b;
 
     struct Scratch {
         Device* d = nullptr;
@@ -736,21 +794,21 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         s.mem.cuda_dev = d->cuda_dev;
         CU(cudaSetDevice(d->cuda_dev));
         s.C = dalloc(s.mem, (size_t)L * L * es);
-        s.Ap = dalloc(s.mem, (size_t)L * b * es);
-        s.Bp = dalloc(s.mem, (size_t)b * L * es);
+        s.Ap = dalloc(s.mem, (size_t)L * fb * es);
+        s.Bp = dalloc(s.mem, (size_t)fb * L * es);
         s.Bt = dalloc(s.mem, (size_t)L * b * es);
         if (dt == FPM_F32) {
-            s.ah = dalloc(s.mem, (size_t)L * b * op);
-            s.al = dalloc(s.mem, (size_t)L * b * op);
-            s.bh = dalloc(s.mem, (size_t)L * b * op);
-            s.bl = dalloc(s.mem, (size_t)L * b * op);
+            s.ah = dalloc(s.mem, (size_t)L * fb * op);
+            s.al = dalloc(s.mem, (size_t)L * fb * op);
+            s.bh = dalloc(s.mem, (size_t)L * fb * op);
+            s.bl = dalloc(s.mem, (size_t)L * fb * op);
             s.sa = static_cast<float*>(dalloc(s.mem, (size_t)L * 4));
             s.sb = static_cast<float*>(dalloc(s.mem, (size_t)L * 4));
         }
         CU(cudaEventCreate(&s.e0));
         CU(cudaEventCreate(&s.e1));
-        launch_fill_synthetic(s.Ap, dt == FPM_F64, b, 101, L, 0, 0, L, b, FPM_DIST_PM1, d->s_comp);
-        launch_fill_synthetic(s.Bp, dt == FPM_F64, L, 102, L, 0, 0, b, L, FPM_DIST_PM1, d->s_comp);
+        launch_fill_synthetic(s.Ap, dt == FPM_F64, fb, 101, L, 0, 0, L, fb, FPM_DIST_PM1, d->s_comp);
+        launch_fill_synthetic(s.Bp, dt == FPM_F64, L, 102, L, 0, 0, fb, L, FPM_DIST_PM1, d->s_comp);
         CU(cudaMemsetAsync(s.C, 0, (size_t)L * L * es, d->s_comp));
     }
 
@@ -759,14 +817,14 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         auto run = [&](Scratch& s) {
             const cudaStream_t st = s.d->s_comp;
             if (dt == FPM_F32) {
-                launch_split_rows(static_cast<const float*>(s.Ap), b, Lx, b, sch, s.ah, s.al, s.sa, st);
-                launch_split_cols(static_cast<const float*>(s.Bp), L, b, Lx, sch, s.bh, s.bl, s.sb, st);
+                launch_split_rows(static_cast<const float*>(s.Ap), fb, Lx, fb, sch, s.ah, s.al, s.sa, st);
+                launch_split_cols(static_cast<const float*>(s.Bp), L, fb, Lx, sch, s.bh, s.bl, s.sb, st);
                 UpdateArgs a;
                 a.a_hi = s.ah; a.a_lo = s.al; a.bt_hi = s.bh; a.bt_lo = s.bl;
                 a.sa = sch == SplitScheme::F16X3 ? s.sa : nullptr;
                 a.sb = sch == SplitScheme::F16X3 ? s.sb : nullptr;
                 a.C = static_cast<float*>(s.C);
-                a.M = Lx; a.Nc = Lx; a.K = b; a.ldc = Lx;
+                a.M = Lx; a.Nc = Lx; a.K = fb; a.ldc = Lx;
                 a.scheme = sch;
                 a.cta_group = ctx->cta_group;
                 a.num_sms = s.d->num_sms;
@@ -819,7 +877,8 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         const double x = (double)(ms[j] * ms[j]);
         for (size_t i = 0; i < S.size(); ++i) {
             const Scratch& s = *S[i];
-            speeds[i * nsizes + j] = 2.0 * x * (double)b * (double)b * (double)b / s.mean;
+            // one timed run = f pivots of the x-block kernel: 2 x b^3 f flop
+            speeds[i * nsizes + j] = 2.0 * x * (double)b * (double)b * (double)fb / s.mean;
             if (ci) ci[i * nsizes + j] = s.mean > 0 ? s.half / s.mean : 0.0;
             if (reps_out) reps_out[i * nsizes + j] = (int32_t)s.ts.size();
         }
@@ -1018,6 +1077,10 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
         } else if (k == "cta_group") {
             FPM_CHECK_ARG(value == 1 || value == 2, "cta_group must be 1 or 2");
             ctx->cta_group = (int)value;
+        } else if (k == "fuse") {
+            FPM_CHECK_ARG(value >= 0 && value <= 8, "fuse must be 0 (auto) or 1..8");
+            if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
+            ctx->fuse = (int)value;
         } else if (k == "kernel_variant") {
             FPM_CHECK_ARG(value >= -1 && value <= 3, "kernel_variant must be -1 (auto) or 0..3");
             ctx->kernel_variant = (int)value;

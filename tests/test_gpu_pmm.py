@@ -80,6 +80,22 @@ def test_integer_inputs_bit_exact_and_p_invariant(p):
         ref = exact if ref is None else ref
 
 
+@pytest.mark.parametrize("fuse", [1, 2, 3, 8])
+def test_fused_pivot_groups(fuse):
+    """f pivots per update (groups cut at every column / row boundary), local
+    fused pulls, FP32: parity with the oracle, integer inputs bit-exact."""
+    N, b = 1536, 64
+    n = N // b
+    rects = pkg.colpart_arrange(n, [250, 170, 96, 60])
+    with pkg.Context.local([0] * 4) as ctx:
+        ctx.set_option("fuse", fuse)
+        A, B, C, st = _run(ctx, N, b, rects, pkg.FPM_F32)
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+        assert st.updates >= -(-n // fuse)
+        Ai, Bi, Ci, _ = _run(ctx, N, b, rects, pkg.FPM_F32, dist=synth.DIST_INT, seeds=(7, 8))
+        assert np.array_equal(Ci.astype(np.float64), og.gemm(Ai, Bi))
+
+
 def test_tf32x3_scheme_and_cta_group1():
     N, b = 1024, 128
     rects = pkg.colpart_arrange(N // b, [32, 32])
