@@ -179,22 +179,26 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
 
     # ---- context: N > 1 -> one process per GPU, pivots pulled from the peers'
     # memory over NVLink (ipc, default) or exchanged with NCCL (nccl)
-    ipc = world > 1 and args.transport == "ipc"
-    if world > 1 and not ipc:
-        obj = [pkg.Context.nccl_unique_id() if rank == 0 else None]
-        dist.broadcast_object_list(obj, src=0)
-        ctx = pkg.Context.nccl(rank, world, local_rank, obj[0])
-    elif ipc:
-        ctx = pkg.Context.ipc(rank, world, local_rank)
-    else:
-        ctx = pkg.Context.local([local_rank])
-    if args.scheme == "tf32x3":
-        ctx.set_option("f32_scheme", pkg.SCHEME_TF32X3)
-    ctx.set_option("cta_group", args.cta_group)
-    ctx.set_option("raster_group", args.raster_group)
-    ctx.set_option("l2_hint_b", args.l2_hint_b)
-    ctx.set_option("kernel_variant", args.kernel_variant)
-    ctx.set_option("fuse", args.fuse)
+    def make_ctx(transport: str):
+        if world > 1 and transport == "nccl":
+            obj = [pkg.Context.nccl_unique_id() if rank == 0 else None]
+            dist.broadcast_object_list(obj, src=0)
+            c = pkg.Context.nccl(rank, world, local_rank, obj[0])
+        elif world > 1:
+            c = pkg.Context.ipc(rank, world, local_rank)
+        else:
+            c = pkg.Context.local([local_rank])
+        if args.scheme == "tf32x3":
+            c.set_option("f32_scheme", pkg.SCHEME_TF32X3)
+        c.set_option("cta_group", args.cta_group)
+        c.set_option("raster_group", args.raster_group)
+        c.set_option("l2_hint_b", args.l2_hint_b)
+        c.set_option("kernel_variant", args.kernel_variant)
+        c.set_option("fuse", args.fuse)
+        return c
+
+    transport = args.transport if world > 1 else "none (p = 1)"
+    ctx = make_ctx(transport)
 
     # ---- FPMs (offline): sample this GPU's speed function once;
     # every rank's model is gathered so all ranks partition identically.
@@ -222,10 +226,24 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
 
     d, rects = plan()
     ctx.setup(N, b, rects, pkg.FPM_F32)
-    if ipc:
+    if transport == "ipc":
+        ok = 1
         blobs = [None] * world
         dist.all_gather_object(blobs, ctx.ipc_export())
-        ctx.ipc_import(blobs)
+        try:
+            ctx.ipc_import(blobs)
+        except pkg.FpmError as ex:  # e.g. no peer access between these GPUs
+            log(f"rank {rank}: IPC import failed ({ex}); falling back to NCCL")
+            ok = 0
+        flag = torch.tensor([ok], dtype=torch.int32)
+        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+        if int(flag.item()) == 0:
+            dist.barrier()
+            ctx.close()
+            transport = "nccl (ipc unavailable)"
+            ctx = make_ctx("nccl")
+            ctx.setup(N, b, rects, pkg.FPM_F32)
+    ipc = transport == "ipc"
     import synth
     sa, sb = synth.seeds_for_config(4)   # config 5 (index 4): seeds 5 and 6
     ctx.fill_synthetic(sa, sb, pkg.FPM_DIST_PM1)
@@ -297,7 +315,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     e2e = None
     if args.e2e_steps > 0:
         try:
-            e2e = run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier)
+            e2e = run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc)
         except Exception as ex:  # report, do not hide
             log("e2e failed:", repr(ex))
             e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:200]}
@@ -318,7 +336,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "f32_scheme": args.scheme, "cta_group": args.cta_group, "raster_group": args.raster_group,
                 "kernel_variant": args.kernel_variant, "fuse": args.fuse,
                 "update_launches_per_step": upd_launches,
-                "transport": (args.transport if world > 1 else "none (p = 1)"),
+                "transport": transport,
                 "l2": "inputs larger than L2 (A, B, C 9.7 GB each)",
                 "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
                 "imbalance_pct_measured": 100.0 * imb_meas, "imbalance_pct_predicted": 100.0 * imb_pred,
@@ -337,7 +355,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     ctx.close()
 
 
-def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier):
+def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc):
     import torch
 
     import paper_conf_cluster_zhongrl12_b200 as pkg
@@ -346,7 +364,6 @@ def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier):
     H, W = r[3] * b, r[4] * b
     R0, C0 = r[1] * b, r[2] * b
     live = H * W > 0
-    ipc = args.transport == "ipc" and args.gpus > 1
     # host windows = this rank's rectangle (generated on the device once, untimed)
     if live:
         hA = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
