@@ -337,7 +337,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "kernel_variant": args.kernel_variant, "fuse": args.fuse,
                 "update_launches_per_step": upd_launches,
                 "transport": transport,
-                "l2": "inputs larger than L2 (A, B, C 9.7 GB each)",
+                "l2": (f"inputs larger than L2 (A, B, C {N * N * 4 / 1e9:.2f} GB each)" if N * N * 4 > 126e6
+                       else "inputs fit in L2 (no flush between steps)"),
                 "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
                 "imbalance_pct_measured": 100.0 * imb_meas, "imbalance_pct_predicted": 100.0 * imb_pred,
                 "fpm_sample_s": t_sample, "fpm_sizes": sizes,
