@@ -21,8 +21,8 @@
  *    read (or written) only for the duration of the call; the library never
  *    keeps them.
  *  - The library owns everything it allocates inside a pmm_ctx (device
- *    buffers, streams, events, green contexts, NCCL communicators); all of it
- *    is released by pmm_destroy.
+ *    buffers, streams, events, IPC mappings, NCCL communicators); all of it is
+ *    released by pmm_destroy.
  *  - fpm_partition, colpart_arrange, colpart_plan_step and fpm_model_speed are
  *    pure host functions: no GPU, no context, thread-safe.  Calls on one
  *    pmm_ctx must be serialised by the caller.
@@ -289,7 +289,8 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * accumulate = 0 writes C = A x B without reading C.  variant (cta_group 2):
  * shared-memory split between the operand ring and the C ring: 0 = 128-byte
  * k-blocks x 3 stages + 2 C chunks in flight, 1 = 64-byte x 4 + 6, 2 = 128-byte
- * x 2 + 6, 3 = 64-byte x 5 + 4; -1 = auto (= 2, measured best).
+ * x 2 + 6, 3 = 64-byte x 5 + 4, 4 = 128-byte x 2 + 4 (leaves ~36 KB smem per
+ * SM for NCCL / staging kernels co-running with the update); -1 = auto (4).
  * Requires K % 8 == 0, ldc % 4 == 0. */
 int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
                      const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,

@@ -30,7 +30,7 @@ struct UpdateArgs {
     bool accumulate = true;  // false: C = A . Bt^T (no read of C)
     int raster_group = 16;   // tile-rows per raster group (L2 reuse)
     int l2_hint_b = 0;       // B^T tile L2 policy: 0 evict_normal, 1 evict_first, 2 evict_last
-    int variant = -1;        // smem split (cta_group 2): -1 auto (= 2),
+    int variant = -1;        // smem split (cta_group 2): -1 auto (= 4), 4 = SW128 x 2 + 4 C chunks,
                              // 0 = SW128 x 3 stages + 2 C chunks, 1 = SW64 x 4 + 6,
                              // 2 = SW128 x 2 + 6, 3 = SW64 x 5 + 4
 };
@@ -63,7 +63,7 @@ void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t c
 
 // C (M x Nc, ldc) += A (M x K, lda) . Bt^T, Bt (Nc x K), FP64 on DMMA.
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                       int64_t K, int64_t ldc, bool accumulate, cudaStream_t st);
+                       int64_t K, int64_t ldc, bool accumulate, int num_sms, cudaStream_t st);
 
 // Seeded counter-based generator (same bits as synth/__init__.py).
 void launch_fill_synthetic(void* dst, bool f64, int64_t ld, uint64_t seed, int64_t N, int64_t r0, int64_t c0,

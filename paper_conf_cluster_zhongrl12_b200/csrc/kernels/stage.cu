@@ -5,6 +5,7 @@
 #include <cuda_fp16.h>
 #include <cuda_runtime.h>
 
+#include <algorithm>
 #include <cstdint>
 
 #include "kernels.hpp"
@@ -98,42 +99,37 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
 }
 
 // B pivot row (K rows x W cols, row stride ld) -> K-major operand halves of its
-// transpose (W rows x K), split as in split_rows_*.  A block owns 32 columns
-// (lane = column, coalesced 128 B row reads); its 8 warps take interleaved
-// 8-row chunks.  Pass 1: column maxima, reduced across the warps through 1 KB of
-// shared memory (small enough to co-reside with the persistent update kernel,
-// which leaves ~2.8 KB per SM).  Pass 2: each lane converts its column's 8 rows
-// of a chunk and writes them as 16 B of output row (col, k0..k0+7).
+// transpose (W rows x K), split as in split_rows_*.  A warp owns 32 columns
+// (lane = column, coalesced 128 B row reads) over all K rows, so no shared
+// memory is needed: the staging kernels then co-reside with the persistent
+// update kernel (which leaves < 2 KB of shared memory per SM).  Pass 1: column
+// maxima; pass 2: each lane converts its column's 8-row chunks and writes them
+// as 16 B of output row (col, k0..k0+7).
 template <bool F16>
 __global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
                                                     void* __restrict__ hi, void* __restrict__ lo,
                                                     float* __restrict__ inv_scale) {
-    __shared__ float red[8][32];
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int64_t col = (int64_t)blockIdx.x * 32 + lane;
-    const bool in = col < W;
+    const int lane = threadIdx.x % 32;
+    const int64_t col = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 32 + lane;
+    if (col >= W) return;
     const int64_t nchunks = K / 8;
     float scale = 1.0f;
     if constexpr (F16) {
-        float m = 0.0f;
-        if (in)
-            for (int64_t ch = warp; ch < nchunks; ch += 8)
+        float m[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+        for (int64_t ch = 0; ch < nchunks; ++ch)
 #pragma unroll
-                for (int i = 0; i < 8; ++i) m = fmaxf(m, fabsf(src[(ch * 8 + i) * ld + col]));
-        red[warp][lane] = m;
-        __syncthreads();
-        m = red[0][lane];
+            for (int i = 0; i < 8; ++i) m[i] = fmaxf(m[i], fabsf(src[(ch * 8 + i) * ld + col]));
+        float mm = m[0];
 #pragma unroll
-        for (int w = 1; w < 8; ++w) m = fmaxf(m, red[w][lane]);
+        for (int i = 1; i < 8; ++i) mm = fmaxf(mm, m[i]);
         int e = 0;
-        if (m > 0.0f) frexpf(m, &e);
-        int s = (m > 0.0f) ? 15 - e : 0;
+        if (mm > 0.0f) frexpf(mm, &e);
+        int s = (mm > 0.0f) ? 15 - e : 0;
         s = s < -126 ? -126 : (s > 127 ? 127 : s);
         scale = ldexpf(1.0f, s);
-        if (warp == 0 && in) inv_scale[col] = ldexpf(1.0f, -s);
+        inv_scale[col] = ldexpf(1.0f, -s);
     }
-    if (!in) return;
-    for (int64_t ch = warp; ch < nchunks; ch += 8) {
+    for (int64_t ch = 0; ch < nchunks; ++ch) {
         float x[8];
 #pragma unroll
         for (int i = 0; i < 8; ++i) x[i] = src[(ch * 8 + i) * ld + col];
@@ -226,8 +222,12 @@ __global__ void __launch_bounds__(256, 1) update_f64_k(const double* __restrict_
     double* As = sm64;                                  // [2][BM][LD]
     double* Bs = sm64 + 2 * F64_BM * F64_LD;            // [2][BN][LD]
     const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int64_t m0 = (int64_t)blockIdx.y * F64_BM, n0 = (int64_t)blockIdx.x * F64_BN;
     const int wm = (warp / 4) * 64, wn = (warp % 4) * 32;
+    // persistent over tiles: the grid is capped at the device's SM cap
+    const int64_t tiles_n = (Nc + F64_BN - 1) / F64_BN;
+    const int64_t tiles = ((M + F64_BM - 1) / F64_BM) * tiles_n;
+    for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
+    const int64_t m0 = (t / tiles_n) * F64_BM, n0 = (t % tiles_n) * F64_BN;
     double acc[8][4][2];
 #pragma unroll
     for (int i = 0; i < 8; ++i)
@@ -301,6 +301,7 @@ __global__ void __launch_bounds__(256, 1) update_f64_k(const double* __restrict_
                     if (gn + h < Nc) cp[h] = (accumulate ? cp[h] : 0.0) + acc[i][j][h];
             }
         }
+    }  // tile loop
 }
 
 int grid_for(int64_t work, int threads) {
@@ -347,7 +348,7 @@ void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, Split
                        float* inv_scale, cudaStream_t st) {
     if (K <= 0 || W <= 0) return;
     FPM_CHECK_ARG(K % 8 == 0, "split_cols: K must be a multiple of 8");
-    const unsigned blocks = (unsigned)((W + 31) / 32);  // 32 columns per block
+    const unsigned blocks = (unsigned)((W + 255) / 256);  // 8 warps x 32 columns per block
     if (s == SplitScheme::F16X3) {
         FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
         split_cols_k<true><<<blocks, 256, 0, st>>>(src, ld, K, W, hi, lo, inv_scale);
@@ -373,7 +374,7 @@ void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t c
 }
 
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                       int64_t K, int64_t ldc, bool accumulate, cudaStream_t st) {
+                       int64_t K, int64_t ldc, bool accumulate, int num_sms, cudaStream_t st) {
     if (M <= 0 || Nc <= 0 || K <= 0) return;
     FPM_CHECK_ARG(K % 8 == 0 && lda % 2 == 0, "FP64 update: K % 8 == 0 and even lda required");
     FPM_CHECK_ARG((reinterpret_cast<uintptr_t>(A) & 15) == 0 && (reinterpret_cast<uintptr_t>(Bt) & 15) == 0,
@@ -386,7 +387,10 @@ void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C
         if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute(update_f64): %s", cudaGetErrorString(e));
         attr_done |= 1ull << dev;
     }
-    dim3 grid((unsigned)((Nc + F64_BN - 1) / F64_BN), (unsigned)((M + F64_BM - 1) / F64_BM));
+    const int64_t tiles = ((Nc + F64_BN - 1) / F64_BN) * ((M + F64_BM - 1) / F64_BM);
+    int sms = num_sms;
+    if (sms <= 0) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+    const unsigned grid = (unsigned)std::min<int64_t>(tiles, std::max(1, sms));  // 1 CTA per SM (147 KB smem)
     update_f64_k<<<grid, 256, F64_SMEM, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
     check_launch("update_f64");
 }

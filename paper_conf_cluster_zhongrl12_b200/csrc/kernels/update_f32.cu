@@ -426,11 +426,13 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
-    FPM_CHECK_ARG(a.variant >= -1 && a.variant <= 3, "kernel variant must be -1 (auto) or 0..3");
+    FPM_CHECK_ARG(a.variant >= -1 && a.variant <= 4, "kernel variant must be -1 (auto) or 0..4");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
-    // auto: variant 2 (two 64-KB operand stages, six C chunks in flight) measured
-    // best at both K = 512 and K = 1024 on B200 (profiles/README.md)
-    const int variant = a.variant >= 0 ? a.variant : 2;
+    // auto: variant 4 (two 64-KB operand stages, four C chunks in flight): as fast
+    // as variant 2 (six C chunks) at the fused K = 2048 (429 TFLOP/s both, c5) and
+    // leaves ~36 KB of shared memory per SM for kernels that must co-run with the
+    // persistent update (NCCL, staging of other emulated devices)
+    const int variant = a.variant >= 0 ? a.variant : 4;
     if (a.cta_group == 2) {
         switch (variant) {
             case 1:  // 64-B k-blocks x 4 stages, 6 C chunks in flight
@@ -444,6 +446,11 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
             case 3:  // 64-B k-blocks x 5 stages, 4 C chunks
                 if (tf32) launch_update_t<2, true, 256, 5, 64, 4>(a, st);
                 else launch_update_t<2, false, 256, 5, 64, 4>(a, st);
+                break;
+            case 4:  // 128-B k-blocks x 2 stages, 4 C chunks: leaves ~36 KB smem per SM for
+                     // NCCL kernels to co-run with the persistent update
+                if (tf32) launch_update_t<2, true, 256, 2, 128, 4>(a, st);
+                else launch_update_t<2, false, 256, 2, 128, 4>(a, st);
                 break;
             default:  // 128-B k-blocks x 3 stages, 2 C chunks
                 if (tf32) launch_update_t<2, true, 256, 3, 128, 2>(a, st);

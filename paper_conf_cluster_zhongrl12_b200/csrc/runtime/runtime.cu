@@ -522,11 +522,11 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
         a.accumulate = k0 != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
         a.raster_group = ctx->raster_group;
         a.l2_hint_b = ctx->l2_hint_b;
-        a.variant = ctx->kernel_variant;
+        a.variant = ctx->kernel_variant;  // -1: auto (variant 4, leaves smem for co-running kernels)
         launch_update_f32(a, d.s_comp);
     } else {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
-                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k0 != 0, d.s_comp);
+                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k0 != 0, d.num_sms, d.s_comp);
     }
     d.launches += 1;
     CU(cudaEventRecord(d.ev_upd1[g], d.s_comp));
@@ -835,7 +835,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             } else {
                 launch_transpose_f64(static_cast<const double*>(s.Bp), L, b, Lx, static_cast<double*>(s.Bt), st);
                 launch_update_f64(static_cast<const double*>(s.Ap), b, static_cast<const double*>(s.Bt),
-                                  static_cast<double*>(s.C), Lx, Lx, b, Lx, true, st);
+                                  static_cast<double*>(s.C), Lx, Lx, b, Lx, true, s.d->num_sms, st);
             }
         };
         for (auto& sp : S) {
@@ -1082,7 +1082,7 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
             ctx->fuse = (int)value;
         } else if (k == "kernel_variant") {
-            FPM_CHECK_ARG(value >= -1 && value <= 3, "kernel_variant must be -1 (auto) or 0..3");
+            FPM_CHECK_ARG(value >= -1 && value <= 4, "kernel_variant must be -1 (auto) or 0..4");
             ctx->kernel_variant = (int)value;
         } else if (k == "l2_hint_b") {
             FPM_CHECK_ARG(value >= 0 && value <= 2, "l2_hint_b must be 0 (normal), 1 (first) or 2 (last)");
@@ -1233,7 +1233,7 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
     return guarded([&] {
         FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
-        FPM_CHECK_ARG(variant >= -1 && variant <= 3, "variant must be -1 (auto) or 0..3");
+        FPM_CHECK_ARG(variant >= -1 && variant <= 4, "variant must be -1 (auto) or 0..4");
         FPM_CHECK_ARG(scheme == 1 || (sa && sb), "F16X3 needs sa and sb");
         fpm::UpdateArgs a;
         a.a_hi = a_hi; a.a_lo = a_lo; a.bt_hi = bt_hi; a.bt_lo = bt_lo;
@@ -1255,7 +1255,7 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
 extern "C" int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
                                 int64_t K, int64_t ldc, int32_t accumulate, void* stream) {
     return guarded([&] {
-        fpm::launch_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate != 0, static_cast<cudaStream_t>(stream));
+        fpm::launch_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate != 0, 0, static_cast<cudaStream_t>(stream));
     });
 }
 
