@@ -96,6 +96,29 @@ def test_fused_pivot_groups(fuse):
         assert np.array_equal(Ci.astype(np.float64), og.gemm(Ai, Bi))
 
 
+def test_single_iteration_b_equals_n():
+    """n = 1: one pivot, one update that overwrites C."""
+    N = b = 512
+    with pkg.Context.local([0]) as ctx:
+        for dt, tol in ((pkg.FPM_F32, 1e-5), (pkg.FPM_F64, 1e-12)):
+            A, B, C, st = _run(ctx, N, b, [(0, 0, 0, 1, 1)], dt)
+            assert og.rel_fro(C, og.gemm(A, B)) <= tol and st.iters == 1 and st.updates == 1
+
+
+def test_sixteen_devices_and_ragged_tiles():
+    """p = 16 (the ABI maximum) emulated devices; rectangle sides that are not
+    multiples of the 256-row tile (b = 96)."""
+    N, b = 96 * 20, 96
+    n = N // b
+    models = _models(77, 16)
+    d = pkg.fpm_partition(n * n, models)
+    assert d == ofpm.partition(n * n, models)
+    rects = pkg.colpart_arrange(n, d)
+    with pkg.Context.local([0] * 16) as ctx:
+        A, B, C, st = _run(ctx, N, b, rects, pkg.FPM_F32, dist=synth.DIST_INT, seeds=(3, 4))
+        assert np.array_equal(C.astype(np.float64), og.gemm(A, B))
+
+
 def test_tf32x3_scheme_and_cta_group1():
     N, b = 1024, 128
     rects = pkg.colpart_arrange(N // b, [32, 32])
