@@ -92,6 +92,8 @@ typedef struct {
     int64_t comm_bytes;                         /* pivot bytes received by this process's devices */
     int64_t kernel_launches;                    /* library kernels launched in the k-loop         */
     int64_t updates;                            /* rank-(f b) update launches (f pivots fused)    */
+    int64_t ooc_devices;                        /* bit i: device i held C_i out of core           */
+    int64_t ooc_bytes;                          /* C bytes streamed host <-> device (out of core) */
 } pmm_stats;
 
 typedef struct pmm_ctx pmm_ctx;
@@ -258,6 +260,23 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 1 evict-first, 2 evict-last.
  * FPM_EINVAL on unknown key or value. */
 int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value);
+
+/* Per-device knobs; `dev` is the device's index in the arrangement (must be
+ * driven by this context).  Takes effect at the next pmm_setup.
+ *   "c_cap_bytes": device memory C_i may occupy (0 = unlimited, default).
+ *                  When the H x W C_i of a problem is larger, C_i is held OUT OF
+ *                  CORE (PAPER.md P:34-40 GPU kernel versions 2-3): it
+ *                  lives in pinned host memory and every update streams it
+ *                  through two device band buffers ("C0 and C1") of at
+ *                  most c_cap_bytes / 2 each (whole multiples of 256 rows, at
+ *                  least 256), band j+1's host -> device copy and band j-1's
+ *                  device -> host copy overlapping band j's update on separate
+ *                  streams.  A_i, B_i and the pivot buffers stay resident.
+ *                  fpm_sample honours the cap (sizes whose C exceeds it are
+ *                  timed out of core), so the speed function shows the memory
+ *                  cliff that makes CPM fail (Table III).
+ * FPM_EINVAL on unknown key / device or bad value. */
+int pmm_set_device_option(pmm_ctx* ctx, int32_t dev, const char* key, int64_t value);
 
 /* --------------------------------------- kernel-level entry points (tests)
  * Device pointers on the current CUDA device, launched asynchronously on

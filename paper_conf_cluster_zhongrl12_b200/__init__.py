@@ -135,6 +135,11 @@ class Context:
     def set_option(self, key: str, value: int) -> None:
         check(lib.pmm_set_option(self._h, key.encode(), int(value)))
 
+    def set_device_option(self, dev: int, key: str, value: int) -> None:
+        """Per-device knob (include/fpmpmm.h pmm_set_device_option), e.g.
+        ``"c_cap_bytes"``: C_i above this size is held out of core."""
+        check(lib.pmm_set_device_option(self._h, int(dev), key.encode(), int(value)))
+
     def setup(self, N: int, b: int, rects: Sequence[Rect], dtype: int = FPM_F32) -> None:
         self._rects = list(rects)
         self._dtype = dtype

@@ -51,6 +51,7 @@ class PmmStats(ctypes.Structure):
         ("per_dev_compute_s", dbl * FPM_MAX_DEVICES), ("per_dev_update_s", dbl * FPM_MAX_DEVICES),
         ("gflops", dbl), ("imbalance", dbl), ("iters", i64), ("comm_bytes", i64),
         ("kernel_launches", i64), ("updates", i64),
+        ("ooc_devices", i64), ("ooc_bytes", i64),
     ]
 
     def as_dict(self, p: int | None = None) -> dict:
@@ -62,6 +63,7 @@ class PmmStats(ctypes.Structure):
             "per_dev_update_s": list(self.per_dev_update_s[:p]),
             "gflops": self.gflops, "imbalance": self.imbalance, "iters": self.iters,
             "comm_bytes": self.comm_bytes, "kernel_launches": self.kernel_launches, "updates": self.updates,
+            "ooc_devices": self.ooc_devices, "ooc_bytes": self.ooc_bytes,
         }
 
 
@@ -93,6 +95,7 @@ _SIGS = {
     "pmm_ipc_import": ([vp, ctypes.c_char_p, i32], ctypes.c_int),
     "pmm_destroy": ([vp], ctypes.c_int),
     "pmm_set_option": ([vp, ctypes.c_char_p, i64], ctypes.c_int),
+    "pmm_set_device_option": ([vp, i32, ctypes.c_char_p, i64], ctypes.c_int),
     "pmm_setup": ([vp, i64, i64, i32, ctypes.POINTER(ColpartRect), ctypes.c_int], ctypes.c_int),
     "pmm_upload": ([vp, vp, vp, i64, i64, i64], ctypes.c_int),
     "pmm_fill_synthetic": ([vp, u64, u64, i32], ctypes.c_int),

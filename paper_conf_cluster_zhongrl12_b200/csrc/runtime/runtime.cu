@@ -40,11 +40,34 @@
 
 namespace fpm {
 
+// Out-of-core C (GPU kernel versions 2/3): when C_i
+// exceeds the device's memory budget for it, C_i lives in pinned host memory and
+// every update streams it through the device in row bands, double buffered
+// ("C0 and C1"): H2D of band j+1 and D2H of band j-1 overlap the update
+// of band j on three streams.
+struct BandPipe {
+    cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+    cudaEvent_t in[2] = {}, done[2] = {}, out[2] = {};
+    void* buf[2] = {};
+    size_t buf_bytes = 0;
+    int ctr = 0;
+    bool used[2] = {false, false};
+    int last = -1;                        // buffer of the most recent device -> host copy
+    std::vector<cudaEvent_t> out_band;    // D2H of band j done (its host rows are current)
+    std::vector<char> band_used;
+    int64_t bytes = 0;                    // host <-> device bytes issued
+};
+
 struct Device {
     int idx = 0;       // index in the arrangement (= rank in NCCL mode)
     int cuda_dev = 0;
     int sm_cap = 0;    // 0 = all SMs
     int num_sms = 0;   // persistent grid of the update kernel
+    int64_t c_cap = 0;     // bytes of device memory C_i may use (0 = no limit)
+    bool ooc = false;      // C_i out of core for the current problem
+    float* hC = nullptr;   // pinned host C_i (H x W) when out of core
+    std::vector<void*> host_allocs;
+    BandPipe bp;
     cudaStream_t s_comp = nullptr, s_comm = nullptr;
     cudaEvent_t ev_ready[2] = {}, ev_free[2] = {};
     cudaEvent_t ev_start = nullptr, ev_stop = nullptr, ev_io0 = nullptr, ev_io1 = nullptr;
@@ -115,10 +138,119 @@ void* dalloc(Device& d, size_t bytes) {
     return p;
 }
 
+void* halloc(Device& d, size_t bytes) {
+    void* p = nullptr;
+    cudaError_t e = cudaHostAlloc(&p, bytes, cudaHostAllocPortable);
+    if (e != cudaSuccess) {
+        cudaGetLastError();
+        fail(FPM_ENOMEM, "cudaHostAlloc(%zu): %s", bytes, cudaGetErrorString(e));
+    }
+    d.host_allocs.push_back(p);
+    return p;
+}
+
+void bp_init(BandPipe& bp) {
+    CU(cudaStreamCreateWithFlags(&bp.s_h2d, cudaStreamNonBlocking));
+    CU(cudaStreamCreateWithFlags(&bp.s_d2h, cudaStreamNonBlocking));
+    for (int i = 0; i < 2; ++i)
+        for (cudaEvent_t* e : {&bp.in[i], &bp.done[i], &bp.out[i]})
+            CU(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
+}
+
+void bp_release_bands(BandPipe& bp) {
+    for (cudaEvent_t e : bp.out_band) cudaEventDestroy(e);
+    bp.out_band.clear();
+    bp.band_used.clear();
+    bp.buf[0] = bp.buf[1] = nullptr;
+    bp.buf_bytes = 0;
+    bp.used[0] = bp.used[1] = false;
+    bp.ctr = 0;
+    bp.last = -1;
+}
+
+void bp_destroy(BandPipe& bp) {
+    bp_release_bands(bp);
+    for (int i = 0; i < 2; ++i)
+        for (cudaEvent_t e : {bp.in[i], bp.done[i], bp.out[i]})
+            if (e) cudaEventDestroy(e);
+    if (bp.s_h2d) cudaStreamDestroy(bp.s_h2d);
+    if (bp.s_d2h) cudaStreamDestroy(bp.s_d2h);
+    bp = BandPipe{};
+}
+
+// Rows per band for a C of width W: half the cap, whole multiples of 256 rows
+// (one CTA-pair tile row), at least 256.
+int64_t band_rows_for(int64_t cap, int64_t W, size_t es) {
+    int64_t rows = cap / 2 / (W * (int64_t)es);
+    return std::max<int64_t>(256, rows / 256 * 256);
+}
+
+// Allocate the two band buffers (bytes each) and the per-band events.
+void bp_alloc_bands(Device& owner, BandPipe& bp, size_t bytes, int64_t nbands) {
+    bp_release_bands(bp);
+    bp.buf[0] = dalloc(owner, bytes);
+    bp.buf[1] = dalloc(owner, bytes);
+    bp.buf_bytes = bytes;
+    bp.out_band.resize(nbands);
+    for (auto& e : bp.out_band) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
+    bp.band_used.assign(nbands, 0);
+}
+
+// One out-of-core update of the host matrix hC (H rows of row_bytes, packed):
+// for each band of `band_rows` rows, H2D (only if `accumulate`) on s_h2d,
+// update on s_comp via launch(r0, rows, device band), D2H on s_d2h.  A band's
+// H2D waits for the previous D2H out of the same buffer (reuse) and for the
+// previous D2H of the same band (its host rows).  Returns the launches issued.
+template <class Launch>
+int64_t banded_update(BandPipe& bp, char* hC, int64_t H, size_t row_bytes, int64_t band_rows, bool accumulate,
+                      cudaStream_t s_comp, Launch&& launch) {
+    const int64_t nb = (H + band_rows - 1) / band_rows;
+    if ((int64_t)bp.out_band.size() < nb || (size_t)band_rows * row_bytes > bp.buf_bytes)
+        fail(FPM_ESTATE, "band pipeline not sized for %lld bands of %lld rows", (long long)nb,
+             (long long)band_rows);
+    int64_t launches = 0;
+    for (int64_t j = 0; j < nb; ++j) {
+        const int buf = bp.ctr++ & 1;
+        const int64_t r0 = j * band_rows, rows = std::min(band_rows, H - r0);
+        const size_t bytes = (size_t)rows * row_bytes;
+        if (bp.used[buf]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out[buf], 0));
+        if (accumulate) {
+            if (bp.band_used[j]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out_band[j], 0));
+            CU(cudaMemcpyAsync(bp.buf[buf], hC + (size_t)r0 * row_bytes, bytes, cudaMemcpyHostToDevice, bp.s_h2d));
+            bp.bytes += (int64_t)bytes;
+        }
+        CU(cudaEventRecord(bp.in[buf], bp.s_h2d));
+        CU(cudaStreamWaitEvent(s_comp, bp.in[buf], 0));
+        launch(r0, rows, bp.buf[buf]);
+        ++launches;
+        CU(cudaEventRecord(bp.done[buf], s_comp));
+        CU(cudaStreamWaitEvent(bp.s_d2h, bp.done[buf], 0));
+        CU(cudaMemcpyAsync(hC + (size_t)r0 * row_bytes, bp.buf[buf], bytes, cudaMemcpyDeviceToHost, bp.s_d2h));
+        bp.bytes += (int64_t)bytes;
+        CU(cudaEventRecord(bp.out[buf], bp.s_d2h));
+        CU(cudaEventRecord(bp.out_band[j], bp.s_d2h));
+        bp.used[buf] = true;
+        bp.band_used[j] = 1;
+        bp.last = buf;
+    }
+    return launches;
+}
+
+// Make `s` wait until every host copy of the band pipeline has landed.
+void bp_join(BandPipe& bp, cudaStream_t s) {
+    if (bp.last >= 0) CU(cudaStreamWaitEvent(s, bp.out[bp.last], 0));
+}
+
 void free_problem(Device& d) {
     cudaSetDevice(d.cuda_dev);
+    if (d.bp.s_d2h) cudaStreamSynchronize(d.bp.s_d2h);
+    bp_release_bands(d.bp);
     for (void* p : d.allocs) cudaFree(p);
     d.allocs.clear();
+    for (void* p : d.host_allocs) cudaFreeHost(p);
+    d.host_allocs.clear();
+    d.hC = nullptr;
+    d.ooc = false;
     for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1, &d.ev_up}) {
         for (cudaEvent_t e : *v) cudaEventDestroy(e);
         v->clear();
@@ -153,11 +285,13 @@ void init_device(Device& d) {
     CU(cudaEventCreate(&d.ev_stop));
     CU(cudaEventCreate(&d.ev_io0));
     CU(cudaEventCreate(&d.ev_io1));
+    bp_init(d.bp);
 }
 
 void destroy_device(Device& d) {
     free_problem(d);
     cudaSetDevice(d.cuda_dev);
+    bp_destroy(d.bp);
     for (int s = 0; s < 2; ++s) {
         if (d.ev_ready[s]) cudaEventDestroy(d.ev_ready[s]);
         if (d.ev_free[s]) cudaEventDestroy(d.ev_free[s]);
@@ -273,7 +407,14 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         const size_t HW = (size_t)d.H * d.W;
         d.A = dalloc(d, HW * es);
         d.B = dalloc(d, HW * es);
-        d.C = dalloc(d, HW * es);
+        d.ooc = d.c_cap > 0 && (int64_t)(HW * es) > d.c_cap;
+        if (d.ooc) {  // C_i in pinned host memory, streamed through two band buffers
+            const int64_t rows = std::min<int64_t>(band_rows_for(d.c_cap, d.W, es), d.H);
+            d.hC = static_cast<float*>(halloc(d, HW * es));
+            bp_alloc_bands(d, d.bp, (size_t)rows * d.W * es, (d.H + rows - 1) / rows);
+        } else {
+            d.C = dalloc(d, HW * es);
+        }
         const size_t op = (dt == FPM_F64) ? 0 : (ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4);
         // receive buffers: NCCL lands pivots in them; FP64 copies peers' pivots into
         // them.  FP32 in local / IPC mode stages straight from the peers' memory.
@@ -298,7 +439,10 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
             v->resize(n);
             for (auto& e : *v) CU(cudaEventCreate(&e));
         }
-        CU(cudaMemsetAsync(d.C, 0, HW * es, d.s_comp));
+        if (d.ooc)
+            std::memset(d.hC, 0, HW * es);
+        else
+            CU(cudaMemsetAsync(d.C, 0, HW * es, d.s_comp));
     }
 
     if (ctx->nccl_mode) {
@@ -523,12 +667,41 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
         a.raster_group = ctx->raster_group;
         a.l2_hint_b = ctx->l2_hint_b;
         a.variant = ctx->kernel_variant;  // -1: auto (variant 4, leaves smem for co-running kernels)
-        launch_update_f32(a, d.s_comp);
+        if (d.ooc) {
+            // out of core: the same update, one row band of C_i at a time (rows
+            // r0.. of the A operand and its scales, the band buffer as C)
+            const size_t op = a.scheme == SplitScheme::F16X3 ? 2 : 4;
+            const int64_t rows = (int64_t)(d.bp.buf_bytes / ((size_t)d.W * 4));
+            d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 4, rows, a.accumulate,
+                                        d.s_comp, [&](int64_t r0, int64_t m, void* band) {
+                                            UpdateArgs x = a;
+                                            x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * a.K * op;
+                                            x.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * a.K * op;
+                                            x.sa = a.sa ? a.sa + r0 : nullptr;
+                                            x.C = static_cast<float*>(band);
+                                            x.M = m;
+                                            launch_update_f32(x, d.s_comp);
+                                        });
+        } else {
+            launch_update_f32(a, d.s_comp);
+            d.launches += 1;
+        }
+    } else if (d.ooc) {
+        const int64_t rows = (int64_t)(d.bp.buf_bytes / ((size_t)d.W * 8));
+        const double* aop = static_cast<const double*>(d.a_op[slot]);
+        const int64_t b = ctx->b;
+        d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, rows, k0 != 0, d.s_comp,
+                                    [&](int64_t r0, int64_t m, void* band) {
+                                        launch_update_f64(aop + (size_t)r0 * b, b,
+                                                          static_cast<const double*>(d.bt[slot]),
+                                                          static_cast<double*>(band), m, d.W, b, d.W, k0 != 0,
+                                                          d.num_sms, d.s_comp);
+                                    });
     } else {
         launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
                           static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k0 != 0, d.num_sms, d.s_comp);
+        d.launches += 1;
     }
-    d.launches += 1;
     CU(cudaEventRecord(d.ev_upd1[g], d.s_comp));
     CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
 }
@@ -542,7 +715,10 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
     FPM_CHECK_ARG(!(ctx->ipc_mode && host), "IPC mode has no streamed host input (peers cannot be ordered)");
     int64_t launches0 = 0;
-    for (auto& d : ctx->devs) launches0 += d.launches;
+    for (auto& d : ctx->devs) {
+        launches0 += d.launches;
+        d.bp.bytes = 0;
+    }
     for (auto& d : ctx->devs) {
         if (!d.live()) continue;
         CU(cudaSetDevice(d.cuda_dev));
@@ -585,6 +761,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
     for (auto& d : ctx->devs) launches += d.launches;
     for (auto& d : ctx->devs) {
         CU(cudaSetDevice(d.cuda_dev));
+        if (d.ooc) bp_join(d.bp, d.s_comp);  // C_i is complete once its last band is back in host memory
         CU(cudaEventRecord(d.ev_stop, d.s_comp));
     }
     double t_max = 0.0;
@@ -605,6 +782,11 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         }
         st->iters = ctx->n;
         st->updates = ngroups;
+        for (auto& d : ctx->devs)
+            if (d.ooc) {
+                if (d.idx < 63) st->ooc_devices |= (int64_t)1 << d.idx;
+                st->ooc_bytes += d.bp.bytes;
+            }
         st->comm_bytes = bytes;
         st->kernel_launches = launches;
         st->gflops = t_max > 0 ? 2.0 * (double)ctx->N * (double)ctx->N * (double)ctx->N / t_max * 1e-9 : 0.0;
@@ -631,6 +813,12 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
 }
 
 // ------------------------------------------------------------ host transfers
+void copy_rows(void* dst, size_t dpitch, const void* src, size_t spitch, size_t width, int64_t rows) {
+    for (int64_t r = 0; r < rows; ++r)
+        std::memcpy(static_cast<char*>(dst) + (size_t)r * dpitch, static_cast<const char*>(src) + (size_t)r * spitch,
+                    width);
+}
+
 void check_window(pmm_ctx* ctx, const Device& d, int64_t ld, int64_t row_base, int64_t col_base) {
     const int64_t R0 = d.rect.row0 * ctx->b, C0 = d.rect.col0 * ctx->b;
     FPM_CHECK_ARG(row_base >= 0 && col_base >= 0 && R0 >= row_base && C0 >= col_base &&
@@ -658,7 +846,7 @@ void upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld, int64_t row_
         }
         const char* srcB = static_cast<const char*>(B) + ((size_t)R0 * ld + (size_t)C0) * es;
         CU(cudaMemcpy2DAsync(d.B, d.W * es, srcB, ld * es, d.W * es, d.H, cudaMemcpyHostToDevice, d.s_comp));
-        CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
+        if (!d.ooc) CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
         CU(cudaEventRecord(d.ev_io1, d.s_comp));
     }
     for (auto& d : ctx->devs) {
@@ -683,7 +871,12 @@ void download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_b
         const int64_t R0 = d.rect.row0 * b - row_base, C0 = d.rect.col0 * b - col_base;
         CU(cudaEventRecord(d.ev_io0, d.s_comp));
         char* dst = static_cast<char*>(C) + ((size_t)R0 * ld + (size_t)C0) * es;
-        CU(cudaMemcpy2DAsync(dst, ld * es, d.C, d.W * es, d.W * es, d.H, cudaMemcpyDeviceToHost, d.s_comp));
+        if (d.ooc) {  // C_i already in host memory (compute joined its band copies)
+            CU(cudaStreamSynchronize(d.bp.s_d2h));
+            copy_rows(dst, ld * es, d.hC, d.W * es, d.W * es, d.H);
+        } else {
+            CU(cudaMemcpy2DAsync(dst, ld * es, d.C, d.W * es, d.W * es, d.H, cudaMemcpyDeviceToHost, d.s_comp));
+        }
         CU(cudaEventRecord(d.ev_io1, d.s_comp));
     }
     for (auto& d : ctx->devs) {
@@ -708,7 +901,7 @@ void fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int dist) {
             launch_fill_synthetic(static_cast<char*>(d.A) + (size_t)c * d.H * b * es, f64, b, seed_a, ctx->N, R0,
                                   C0 + c * b, d.H, b, dist, d.s_comp);
         launch_fill_synthetic(d.B, f64, d.W, seed_b, ctx->N, R0, C0, d.H, d.W, dist, d.s_comp);
-        CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
+        if (!d.ooc) CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
     }
     for (auto& d : ctx->devs) {
         if (!d.live()) continue;
@@ -772,7 +965,8 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
 
     struct Scratch {
         Device* d = nullptr;
-        Device mem;  // owns the allocations
+        Device mem;  // owns the allocations (and the band pipeline of out-of-core sizes)
+        char* hC = nullptr;  // pinned host C for sizes above the device's C cap
         void *C = nullptr, *Ap = nullptr, *Bp = nullptr, *Bt = nullptr;
         void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
         float *sa = nullptr, *sb = nullptr;
@@ -782,10 +976,14 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         bool done = false;
         ~Scratch() {
             free_problem(mem);
+            bp_destroy(mem.bp);
             if (e0) cudaEventDestroy(e0);
             if (e1) cudaEventDestroy(e1);
         }
     };
+    // sizes whose C exceeds the device's C cap run out of core (as in the k-loop)
+    auto ooc_at = [&](const Device* d, int64_t Lx) { return d->c_cap > 0 && (int64_t)(Lx * Lx * es) > d->c_cap; };
+    auto rows_at = [&](const Device* d, int64_t Lx) { return std::min(band_rows_for(d->c_cap, Lx, es), Lx); };
     std::vector<std::unique_ptr<Scratch>> S;
     for (Device* d : devs) {
         S.emplace_back(new Scratch);
@@ -793,7 +991,26 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         s.d = d;
         s.mem.cuda_dev = d->cuda_dev;
         CU(cudaSetDevice(d->cuda_dev));
-        s.C = dalloc(s.mem, (size_t)L * L * es);
+        int64_t Lin = 0, Lout = 0, nbands = 0;
+        size_t band_bytes = 0;
+        for (int j = 0; j < nsizes; ++j) {
+            const int64_t Lx = ms[j] * b;
+            if (!ooc_at(d, Lx)) {
+                Lin = std::max(Lin, Lx);
+                continue;
+            }
+            Lout = std::max(Lout, Lx);
+            const int64_t rows = rows_at(d, Lx);
+            nbands = std::max(nbands, (Lx + rows - 1) / rows);
+            band_bytes = std::max(band_bytes, (size_t)rows * Lx * es);
+        }
+        s.C = dalloc(s.mem, (size_t)Lin * Lin * es);
+        if (Lout > 0) {
+            bp_init(s.mem.bp);
+            s.hC = static_cast<char*>(halloc(s.mem, (size_t)Lout * Lout * es));
+            std::memset(s.hC, 0, (size_t)Lout * Lout * es);
+            bp_alloc_bands(s.mem, s.mem.bp, band_bytes, nbands);
+        }
         s.Ap = dalloc(s.mem, (size_t)L * fb * es);
         s.Bp = dalloc(s.mem, (size_t)fb * L * es);
         s.Bt = dalloc(s.mem, (size_t)L * b * es);
@@ -809,13 +1026,14 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         CU(cudaEventCreate(&s.e1));
         launch_fill_synthetic(s.Ap, dt == FPM_F64, fb, 101, L, 0, 0, L, fb, FPM_DIST_PM1, d->s_comp);
         launch_fill_synthetic(s.Bp, dt == FPM_F64, L, 102, L, 0, 0, fb, L, FPM_DIST_PM1, d->s_comp);
-        CU(cudaMemsetAsync(s.C, 0, (size_t)L * L * es, d->s_comp));
+        if (s.C) CU(cudaMemsetAsync(s.C, 0, (size_t)Lin * Lin * es, d->s_comp));
     }
 
     for (int j = 0; j < nsizes; ++j) {
         const int64_t Lx = ms[j] * b;
         auto run = [&](Scratch& s) {
             const cudaStream_t st = s.d->s_comp;
+            const bool ooc = ooc_at(s.d, Lx);
             if (dt == FPM_F32) {
                 launch_split_rows(static_cast<const float*>(s.Ap), fb, Lx, fb, sch, s.ah, s.al, s.sa, st);
                 launch_split_cols(static_cast<const float*>(s.Bp), L, fb, Lx, sch, s.bh, s.bl, s.sb, st);
@@ -831,12 +1049,35 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.raster_group = ctx->raster_group;
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
-                launch_update_f32(a, st);
+                if (ooc) {
+                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 4, rows_at(s.d, Lx), true, st,
+                                  [&](int64_t r0, int64_t m, void* band) {
+                                      UpdateArgs x = a;
+                                      x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
+                                      x.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * fb * op;
+                                      x.sa = a.sa ? a.sa + r0 : nullptr;
+                                      x.C = static_cast<float*>(band);
+                                      x.M = m;
+                                      launch_update_f32(x, st);
+                                  });
+                } else {
+                    launch_update_f32(a, st);
+                }
             } else {
                 launch_transpose_f64(static_cast<const double*>(s.Bp), L, b, Lx, static_cast<double*>(s.Bt), st);
-                launch_update_f64(static_cast<const double*>(s.Ap), b, static_cast<const double*>(s.Bt),
-                                  static_cast<double*>(s.C), Lx, Lx, b, Lx, true, s.d->num_sms, st);
+                if (ooc) {
+                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 8, rows_at(s.d, Lx), true, st,
+                                  [&](int64_t r0, int64_t m, void* band) {
+                                      launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * b, b,
+                                                        static_cast<const double*>(s.Bt), static_cast<double*>(band),
+                                                        m, Lx, b, Lx, true, s.d->num_sms, st);
+                                  });
+                } else {
+                    launch_update_f64(static_cast<const double*>(s.Ap), b, static_cast<const double*>(s.Bt),
+                                      static_cast<double*>(s.C), Lx, Lx, b, Lx, true, s.d->num_sms, st);
+                }
             }
+            if (ooc) bp_join(s.mem.bp, st);  // the update is done when C is back in host memory
         };
         for (auto& sp : S) {
             sp->ts.clear();
@@ -1096,6 +1337,22 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
     });
 }
 
+extern "C" int pmm_set_device_option(pmm_ctx* ctx, int32_t dev, const char* key, int64_t value) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx && key, "null argument");
+        fpm::Device* d = fpm::local_dev(ctx, dev);
+        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
+        const std::string k(key);
+        if (k == "c_cap_bytes") {
+            FPM_CHECK_ARG(value >= 0, "c_cap_bytes must be >= 0");
+            if (d->c_cap != value) ctx->have_problem = false;  // C_i placement changes
+            d->c_cap = value;
+        } else {
+            fpm::fail(FPM_EINVAL, "unknown device option '%s'", key);
+        }
+    });
+}
+
 extern "C" int pmm_setup(pmm_ctx* ctx, int64_t N, int64_t b, int32_t p, const colpart_rect* rects, fpm_dtype dt) {
     return guarded([&] {
         FPM_CHECK_ARG(ctx != nullptr, "null ctx");
@@ -1148,8 +1405,15 @@ extern "C" int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t 
             if (r0 >= R0 && c0 >= C0 && r0 + rows <= R0 + d.H && c0 + cols <= C0 + d.W) {
                 CU(cudaSetDevice(d.cuda_dev));
                 CU(cudaStreamSynchronize(d.s_comp));
-                const char* src = static_cast<const char*>(d.C) + ((size_t)(r0 - R0) * d.W + (size_t)(c0 - C0)) * es;
-                CU(cudaMemcpy2D(C_host, ld * es, src, d.W * es, cols * es, rows, cudaMemcpyDeviceToHost));
+                const size_t off = ((size_t)(r0 - R0) * d.W + (size_t)(c0 - C0)) * es;
+                if (d.ooc) {
+                    CU(cudaStreamSynchronize(d.bp.s_d2h));
+                    fpm::copy_rows(C_host, ld * es, reinterpret_cast<const char*>(d.hC) + off, d.W * es, cols * es,
+                                   rows);
+                } else {
+                    CU(cudaMemcpy2D(C_host, ld * es, static_cast<const char*>(d.C) + off, d.W * es, cols * es, rows,
+                                    cudaMemcpyDeviceToHost));
+                }
                 return;
             }
         }
