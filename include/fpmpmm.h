@@ -255,6 +255,11 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 group's exchange is its first pivot's plan with f-times longer
  *                 panels; the F16X3 scales are taken over the fused rows.  Halves
  *                 (f = 2) the C read-modify-write traffic of the iteration loop.
+ *   "ooc_keep":   out-of-core devices (pmm_set_device_option "c_cap_bytes"):
+ *                 1 (default) = P:34's refinement: the band order reverses
+ *                 every other update and the last two bands of an update stay
+ *                 on the device for the next one (two transfers saved in each
+ *                 direction per update); 0 = every band in and out every update.
  *   "raster_group": tile-rows per L2 raster group of the update (default 16).
  *   "l2_hint_b":  L2 policy of the B^T operand tiles: 0 normal (default),
  *                 1 evict-first, 2 evict-last.

@@ -118,6 +118,7 @@ struct pmm_ctx {
     int kernel_variant = -1;  // auto
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
+    int ooc_keep = 1;         // out-of-core: keep the last two bands, reverse every other update
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
 };
 
@@ -200,36 +201,60 @@ void bp_alloc_bands(Device& owner, BandPipe& bp, size_t bytes, int64_t nbands) {
 // for each band of `band_rows` rows, H2D (only if `accumulate`) on s_h2d,
 // update on s_comp via launch(r0, rows, device band), D2H on s_d2h.  A band's
 // H2D waits for the previous D2H out of the same buffer (reuse) and for the
-// previous D2H of the same band (its host rows).  Returns the launches issued.
+// previous D2H of the same band (its host rows).
+//
+// P:34 "we keep the last two rectangles accumulating intermediate results in
+// the device in each iteration and reverse the updating order every other
+// iteration, which can save two transfers in each direction": `reverse` runs
+// the bands last to first; `keep_tail` leaves the last two bands of this call
+// in the buffers (no D2H); `kept_head` says the previous call kept its tail,
+// so this call (in the opposite order) starts on those two bands without H2D.
+// Returns the launches issued.
+struct BandCall {
+    bool accumulate = true;
+    bool reverse = false;
+    bool kept_head = false;
+    bool keep_tail = false;
+};
+
 template <class Launch>
-int64_t banded_update(BandPipe& bp, char* hC, int64_t H, size_t row_bytes, int64_t band_rows, bool accumulate,
+int64_t banded_update(BandPipe& bp, char* hC, int64_t H, size_t row_bytes, int64_t band_rows, const BandCall& bc,
                       cudaStream_t s_comp, Launch&& launch) {
     const int64_t nb = (H + band_rows - 1) / band_rows;
     if ((int64_t)bp.out_band.size() < nb || (size_t)band_rows * row_bytes > bp.buf_bytes)
         fail(FPM_ESTATE, "band pipeline not sized for %lld bands of %lld rows", (long long)nb,
              (long long)band_rows);
+    const int64_t nkeep = std::min<int64_t>(2, nb);
+    // the first band of this call is the last band of the previous one: same buffer
+    if (bc.kept_head) bp.ctr -= 1;
     int64_t launches = 0;
-    for (int64_t j = 0; j < nb; ++j) {
+    for (int64_t t = 0; t < nb; ++t) {
+        const int64_t j = bc.reverse ? nb - 1 - t : t;
         const int buf = bp.ctr++ & 1;
         const int64_t r0 = j * band_rows, rows = std::min(band_rows, H - r0);
         const size_t bytes = (size_t)rows * row_bytes;
-        if (bp.used[buf]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out[buf], 0));
-        if (accumulate) {
-            if (bp.band_used[j]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out_band[j], 0));
-            CU(cudaMemcpyAsync(bp.buf[buf], hC + (size_t)r0 * row_bytes, bytes, cudaMemcpyHostToDevice, bp.s_h2d));
-            bp.bytes += (int64_t)bytes;
+        const bool resident = bc.kept_head && t < nkeep;  // already in `buf`, current
+        if (!resident) {
+            if (bp.used[buf]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out[buf], 0));
+            if (bc.accumulate) {
+                if (bp.band_used[j]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out_band[j], 0));
+                CU(cudaMemcpyAsync(bp.buf[buf], hC + (size_t)r0 * row_bytes, bytes, cudaMemcpyHostToDevice,
+                                   bp.s_h2d));
+                bp.bytes += (int64_t)bytes;
+            }
+            CU(cudaEventRecord(bp.in[buf], bp.s_h2d));
+            CU(cudaStreamWaitEvent(s_comp, bp.in[buf], 0));
         }
-        CU(cudaEventRecord(bp.in[buf], bp.s_h2d));
-        CU(cudaStreamWaitEvent(s_comp, bp.in[buf], 0));
         launch(r0, rows, bp.buf[buf]);
         ++launches;
+        bp.used[buf] = true;
+        if (bc.keep_tail && t >= nb - nkeep) continue;  // stays in the buffer for the next call
         CU(cudaEventRecord(bp.done[buf], s_comp));
         CU(cudaStreamWaitEvent(bp.s_d2h, bp.done[buf], 0));
         CU(cudaMemcpyAsync(hC + (size_t)r0 * row_bytes, bp.buf[buf], bytes, cudaMemcpyDeviceToHost, bp.s_d2h));
         bp.bytes += (int64_t)bytes;
         CU(cudaEventRecord(bp.out[buf], bp.s_d2h));
         CU(cudaEventRecord(bp.out_band[j], bp.s_d2h));
-        bp.used[buf] = true;
         bp.band_used[j] = 1;
         bp.last = buf;
     }
@@ -646,6 +671,13 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
     CU(cudaSetDevice(d.cuda_dev));
     CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
     CU(cudaEventRecord(d.ev_upd0[g], d.s_comp));
+    // out-of-core band order: reversed every other update, the last two
+    // bands kept on the device between updates (option "ooc_keep")
+    BandCall bc;
+    bc.accumulate = k0 != 0;
+    bc.reverse = ctx->ooc_keep && (g & 1);
+    bc.kept_head = ctx->ooc_keep && g > 0;
+    bc.keep_tail = ctx->ooc_keep && g + 1 < (int)ctx->groups.size();
     if (ctx->dt == FPM_F32) {
         UpdateArgs a;
         a.a_hi = d.a_hi[slot];
@@ -672,7 +704,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
             // r0.. of the A operand and its scales, the band buffer as C)
             const size_t op = a.scheme == SplitScheme::F16X3 ? 2 : 4;
             const int64_t rows = (int64_t)(d.bp.buf_bytes / ((size_t)d.W * 4));
-            d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 4, rows, a.accumulate,
+            d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 4, rows, bc,
                                         d.s_comp, [&](int64_t r0, int64_t m, void* band) {
                                             UpdateArgs x = a;
                                             x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * a.K * op;
@@ -690,7 +722,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
         const int64_t rows = (int64_t)(d.bp.buf_bytes / ((size_t)d.W * 8));
         const double* aop = static_cast<const double*>(d.a_op[slot]);
         const int64_t b = ctx->b;
-        d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, rows, k0 != 0, d.s_comp,
+        d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, rows, bc, d.s_comp,
                                     [&](int64_t r0, int64_t m, void* band) {
                                         launch_update_f64(aop + (size_t)r0 * b, b,
                                                           static_cast<const double*>(d.bt[slot]),
@@ -972,6 +1004,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         float *sa = nullptr, *sb = nullptr;
         cudaEvent_t e0 = nullptr, e1 = nullptr;
         std::vector<double> ts;
+        int runs = 0;  // runs at the current size (out-of-core band order alternates)
         double mean = 0.0, half = 0.0;
         bool done = false;
         ~Scratch() {
@@ -1034,6 +1067,13 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         auto run = [&](Scratch& s) {
             const cudaStream_t st = s.d->s_comp;
             const bool ooc = ooc_at(s.d, Lx);
+            // out of core: the k-loop's steady state (bands kept and order reversed
+            // between consecutive updates)
+            BandCall bc;
+            bc.reverse = ctx->ooc_keep && (s.runs & 1);
+            bc.kept_head = ctx->ooc_keep && s.runs > 0;
+            bc.keep_tail = ctx->ooc_keep;
+            ++s.runs;
             if (dt == FPM_F32) {
                 launch_split_rows(static_cast<const float*>(s.Ap), fb, Lx, fb, sch, s.ah, s.al, s.sa, st);
                 launch_split_cols(static_cast<const float*>(s.Bp), L, fb, Lx, sch, s.bh, s.bl, s.sb, st);
@@ -1050,7 +1090,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
                 if (ooc) {
-                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 4, rows_at(s.d, Lx), true, st,
+                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 4, rows_at(s.d, Lx), bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
                                       UpdateArgs x = a;
                                       x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
@@ -1066,7 +1106,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             } else {
                 launch_transpose_f64(static_cast<const double*>(s.Bp), L, b, Lx, static_cast<double*>(s.Bt), st);
                 if (ooc) {
-                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 8, rows_at(s.d, Lx), true, st,
+                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 8, rows_at(s.d, Lx), bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
                                       launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * b, b,
                                                         static_cast<const double*>(s.Bt), static_cast<double*>(band),
@@ -1082,6 +1122,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         for (auto& sp : S) {
             sp->ts.clear();
             sp->done = false;
+            sp->runs = 0;
         }
         for (int w = 0; w < 2; ++w)
             for (auto& sp : S) {
@@ -1322,6 +1363,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= 0 && value <= 8, "fuse must be 0 (auto) or 1..8");
             if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
             ctx->fuse = (int)value;
+        } else if (k == "ooc_keep") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "ooc_keep must be 0 or 1");
+            ctx->ooc_keep = (int)value;
         } else if (k == "kernel_variant") {
             FPM_CHECK_ARG(value >= -1 && value <= 4, "kernel_variant must be -1 (auto) or 0..4");
             ctx->kernel_variant = (int)value;

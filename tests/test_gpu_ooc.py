@@ -33,9 +33,27 @@ def _cap_for_band_rows(rows, W, es):
     return 2 * rows * W * es
 
 
+def _expected_ooc_bytes(H, W, es, band_rows, updates, keep):
+    """Host <-> device C bytes of one k-loop, written from P:34 directly: every
+    update moves each band in (not the first update: it overwrites) and out;
+    with `keep` the order reverses every other update and the last two bands of
+    an update stay on the device for the next one (not after the last)."""
+    rows = [min(band_rows, H - r0) for r0 in range(0, H, band_rows)]
+    nb, nkeep = len(rows), min(2, len(rows))
+    total = 0
+    for g in range(updates):
+        order = list(range(nb))[::-1] if keep and g % 2 else list(range(nb))
+        head = set(order[:nkeep]) if keep and g > 0 else set()
+        tail = set(order[-nkeep:]) if keep and g + 1 < updates else set()
+        total += sum(rows[j] for j in order if g > 0 and j not in head)
+        total += sum(rows[j] for j in order if j not in tail)
+    return total * W * es
+
+
 @pytest.mark.parametrize("dt,tol", [(pkg.FPM_F32, 1e-5), (pkg.FPM_F64, 1e-12)])
 @pytest.mark.parametrize("band_rows", [256, 512, 0])
-def test_ooc_device_parity(dt, tol, band_rows):
+@pytest.mark.parametrize("keep", [1, 0])
+def test_ooc_device_parity(dt, tol, band_rows, keep):
     """Device 0 out of core with 1, 3 or 5 bands (ragged), device 1 resident."""
     N, b = 1440, 96          # rect 0 is 1056 x 1440: bands 4 x 256 + 32, 2 x 512 + 32
     n = N // b
@@ -47,13 +65,16 @@ def test_ooc_device_parity(dt, tol, band_rows):
     H0, W0 = r0[3] * b, r0[4] * b
     A, B, C = _inputs(N, dt)
     with pkg.Context.local([0, 0]) as ctx:
+        ctx.set_option("ooc_keep", keep)
         ctx.set_device_option(0, "c_cap_bytes", _cap_for_band_rows(band_rows, W0, es) if band_rows else 1)
         st = ctx.run(A, B, C, N, b, rects, dt)
     assert og.rel_fro(C, og.gemm(A, B)) <= tol
     assert st.ooc_devices == 1
-    # every update: D2H of all of C_0; every update but the first: H2D of all of C_0
-    assert st.ooc_bytes == H0 * W0 * es * (2 * st.updates - 1)
-    nb = -(-H0 // max(band_rows, 256))
+    br = max(band_rows, 256)
+    assert st.ooc_bytes == _expected_ooc_bytes(H0, W0, es, br, st.updates, keep)
+    if not keep:
+        assert st.ooc_bytes == H0 * W0 * es * (2 * st.updates - 1)
+    nb = -(-H0 // br)
     assert st.kernel_launches >= st.updates * (nb + 1)
 
 
@@ -64,10 +85,11 @@ def test_ooc_all_devices_integer_exact(fuse):
     N, b = 1024, 64
     n = N // b
     rects = pkg.colpart_arrange(n, [100, 80, 76])
-    for dt in (pkg.FPM_F32, pkg.FPM_F64):
+    for dt, keep in ((pkg.FPM_F32, 1), (pkg.FPM_F64, 1), (pkg.FPM_F32, 0)):
         A, B, C = _inputs(N, dt, dist=synth.DIST_INT, seeds=(11, 12))
         with pkg.Context.local([0, 0, 0]) as ctx:
             ctx.set_option("fuse", fuse)
+            ctx.set_option("ooc_keep", keep)
             for i in range(3):
                 ctx.set_device_option(i, "c_cap_bytes", 1)  # minimum bands: 256 rows
             st = ctx.run(A, B, C, N, b, rects, dt)
