@@ -257,9 +257,16 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 (f = 2) the C read-modify-write traffic of the iteration loop.
  *   "ooc_keep":   out-of-core devices (pmm_set_device_option "c_cap_bytes"):
  *                 1 (default) = P:34's refinement: the band order reverses
- *                 every other update and the last two bands of an update stay
- *                 on the device for the next one (two transfers saved in each
- *                 direction per update); 0 = every band in and out every update.
+ *                 every other update and the last R bands of an update stay
+ *                 on the device for the next one (the paper keeps two: R
+ *                 transfers saved in each direction per update); 0 = every
+ *                 band in and out every update.
+ *   "ooc_buffers": R, out-of-core band buffers sharing the C cap, 2..16
+ *                 (default 8; 2 = the paper's C0 / C1).  More, smaller bands
+ *                 overlap the two copy directions with each other and with the
+ *                 updates; with "ooc_keep" the per-update traffic stays C_i
+ *                 minus the cap in each direction.  Fewer buffers (not below
+ *                 2) are used when R bands of 256 rows exceed the cap.
  *   "raster_group": tile-rows per L2 raster group of the update (default 16).
  *   "l2_hint_b":  L2 policy of the B^T operand tiles: 0 normal (default),
  *                 1 evict-first, 2 evict-last.
@@ -272,11 +279,13 @@ int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value);
  *                  When the H x W C_i of a problem is larger, C_i is held OUT OF
  *                  CORE (PAPER.md P:34-40 GPU kernel versions 2-3): it
  *                  lives in pinned host memory and every update streams it
- *                  through two device band buffers ("C0 and C1") of at
- *                  most c_cap_bytes / 2 each (whole multiples of 256 rows, at
- *                  least 256), band j+1's host -> device copy and band j-1's
- *                  device -> host copy overlapping band j's update on separate
- *                  streams.  A_i, B_i and the pivot buffers stay resident.
+ *                  through a ring of R device band buffers (option
+ *                  "ooc_buffers"; R = 2 is the paper's "C0 and C1") of
+ *                  at most c_cap_bytes / R each (whole multiples of 256 rows,
+ *                  at least 256), the host -> device copy of a later band and
+ *                  the device -> host copy of an earlier one overlapping the
+ *                  update of the current band on separate streams.  A_i, B_i
+ *                  and the pivot buffers stay resident.
  *                  fpm_sample honours the cap (sizes whose C exceeds it are
  *                  timed out of core), so the speed function shows the memory
  *                  cliff that makes CPM fail (Table III).

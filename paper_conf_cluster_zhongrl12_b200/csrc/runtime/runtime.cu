@@ -42,17 +42,25 @@ namespace fpm {
 
 // Out-of-core C (GPU kernel versions 2/3): when C_i
 // exceeds the device's memory budget for it, C_i lives in pinned host memory and
-// every update streams it through the device in row bands, double buffered
-// ("C0 and C1"): H2D of band j+1 and D2H of band j-1 overlap the update
-// of band j on three streams.
+// every update streams it through the device in row bands held in a ring of R
+// device buffers (R = 2 is the paper's "C0 and C1"): the H2D of a later
+// band and the D2H of an earlier one overlap the update of the current band on
+// three streams.
+constexpr int kMaxBandBufs = 16;
+struct Ring {
+    int R;         // buffers in use
+    int64_t rows;  // rows per band
+};
 struct BandPipe {
     cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
-    cudaEvent_t in[2] = {}, done[2] = {}, out[2] = {};
-    void* buf[2] = {};
+    cudaEvent_t in[kMaxBandBufs] = {}, done[kMaxBandBufs] = {}, out[kMaxBandBufs] = {};
+    void* buf[kMaxBandBufs] = {};
+    bool used[kMaxBandBufs] = {};
+    int nbuf = 0;                         // R
     size_t buf_bytes = 0;
-    int ctr = 0;
-    bool used[2] = {false, false};
+    int next = 0, dir = 1;                // ring position and direction (reverses with the band order)
     int last = -1;                        // buffer of the most recent device -> host copy
+    int last_step = -1;                   // buffer used by the most recent update
     std::vector<cudaEvent_t> out_band;    // D2H of band j done (its host rows are current)
     std::vector<char> band_used;
     int64_t bytes = 0;                    // host <-> device bytes issued
@@ -68,6 +76,7 @@ struct Device {
     float* hC = nullptr;   // pinned host C_i (H x W) when out of core
     std::vector<void*> host_allocs;
     BandPipe bp;
+    Ring ring{0, 0};       // out-of-core band geometry of the current problem
     cudaStream_t s_comp = nullptr, s_comm = nullptr;
     cudaEvent_t ev_ready[2] = {}, ev_free[2] = {};
     cudaEvent_t ev_start = nullptr, ev_stop = nullptr, ev_io0 = nullptr, ev_io1 = nullptr;
@@ -118,7 +127,8 @@ struct pmm_ctx {
     int kernel_variant = -1;  // auto
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
-    int ooc_keep = 1;         // out-of-core: keep the last two bands, reverse every other update
+    int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
+    int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
 };
 
@@ -153,7 +163,7 @@ void* halloc(Device& d, size_t bytes) {
 void bp_init(BandPipe& bp) {
     CU(cudaStreamCreateWithFlags(&bp.s_h2d, cudaStreamNonBlocking));
     CU(cudaStreamCreateWithFlags(&bp.s_d2h, cudaStreamNonBlocking));
-    for (int i = 0; i < 2; ++i)
+    for (int i = 0; i < kMaxBandBufs; ++i)
         for (cudaEvent_t* e : {&bp.in[i], &bp.done[i], &bp.out[i]})
             CU(cudaEventCreateWithFlags(e, cudaEventDisableTiming));
 }
@@ -162,16 +172,20 @@ void bp_release_bands(BandPipe& bp) {
     for (cudaEvent_t e : bp.out_band) cudaEventDestroy(e);
     bp.out_band.clear();
     bp.band_used.clear();
-    bp.buf[0] = bp.buf[1] = nullptr;
+    for (int i = 0; i < kMaxBandBufs; ++i) {
+        bp.buf[i] = nullptr;
+        bp.used[i] = false;
+    }
+    bp.nbuf = 0;
     bp.buf_bytes = 0;
-    bp.used[0] = bp.used[1] = false;
-    bp.ctr = 0;
-    bp.last = -1;
+    bp.next = 0;
+    bp.dir = 1;
+    bp.last = bp.last_step = -1;
 }
 
 void bp_destroy(BandPipe& bp) {
     bp_release_bands(bp);
-    for (int i = 0; i < 2; ++i)
+    for (int i = 0; i < kMaxBandBufs; ++i)
         for (cudaEvent_t e : {bp.in[i], bp.done[i], bp.out[i]})
             if (e) cudaEventDestroy(e);
     if (bp.s_h2d) cudaStreamDestroy(bp.s_h2d);
@@ -179,18 +193,22 @@ void bp_destroy(BandPipe& bp) {
     bp = BandPipe{};
 }
 
-// Rows per band for a C of width W: half the cap, whole multiples of 256 rows
-// (one CTA-pair tile row), at least 256.
-int64_t band_rows_for(int64_t cap, int64_t W, size_t es) {
-    int64_t rows = cap / 2 / (W * (int64_t)es);
-    return std::max<int64_t>(256, rows / 256 * 256);
+// Ring geometry for an H x W C (element size es) in `cap` bytes with up to R
+// buffers: bands of whole multiples of 256 rows (one CTA-pair tile row), at
+// least 256; fewer buffers (not below 2) when R bands of 256 rows would not fit.
+Ring ring_for(int64_t cap, int64_t H, int64_t W, size_t es, int R) {
+    const int64_t row_bytes = W * (int64_t)es;
+    const int r = (int)std::min<int64_t>(R, std::max<int64_t>(2, cap / (256 * row_bytes)));
+    const int64_t rows = std::max<int64_t>(256, cap / r / row_bytes / 256 * 256);
+    return {r, std::min(rows, H)};
 }
 
-// Allocate the two band buffers (bytes each) and the per-band events.
-void bp_alloc_bands(Device& owner, BandPipe& bp, size_t bytes, int64_t nbands) {
+// Allocate the R band buffers (bytes each) and the per-band events.
+void bp_alloc_bands(Device& owner, BandPipe& bp, int R, size_t bytes, int64_t nbands) {
     bp_release_bands(bp);
-    bp.buf[0] = dalloc(owner, bytes);
-    bp.buf[1] = dalloc(owner, bytes);
+    FPM_CHECK_ARG(R >= 2 && R <= kMaxBandBufs, "out-of-core buffers must be in [2, %d]", kMaxBandBufs);
+    for (int i = 0; i < R; ++i) bp.buf[i] = dalloc(owner, bytes);
+    bp.nbuf = R;
     bp.buf_bytes = bytes;
     bp.out_band.resize(nbands);
     for (auto& e : bp.out_band) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
@@ -200,16 +218,18 @@ void bp_alloc_bands(Device& owner, BandPipe& bp, size_t bytes, int64_t nbands) {
 // One out-of-core update of the host matrix hC (H rows of row_bytes, packed):
 // for each band of `band_rows` rows, H2D (only if `accumulate`) on s_h2d,
 // update on s_comp via launch(r0, rows, device band), D2H on s_d2h.  A band's
-// H2D waits for the previous D2H out of the same buffer (reuse) and for the
+// H2D waits for the D2H of the buffer's previous occupant (reuse) and for the
 // previous D2H of the same band (its host rows).
 //
 // P:34 "we keep the last two rectangles accumulating intermediate results in
 // the device in each iteration and reverse the updating order every other
-// iteration, which can save two transfers in each direction": `reverse` runs
-// the bands last to first; `keep_tail` leaves the last two bands of this call
-// in the buffers (no D2H); `kept_head` says the previous call kept its tail,
-// so this call (in the opposite order) starts on those two bands without H2D.
-// Returns the launches issued.
+// iteration, which can save two transfers in each direction", generalised to
+// R buffers (the paper's R = 2): `reverse` runs the bands last to first;
+// `keep_tail` leaves the last min(R, bands) bands of this call in their buffers
+// (no D2H); `kept_head` says the previous call kept its tail, so this call (in
+// the opposite order) starts on those bands without H2D.  The ring then runs
+// backwards: the buffer freed first (its band updated and copied out first) is
+// the one the first non-resident band needs.  Returns the launches issued.
 struct BandCall {
     bool accumulate = true;
     bool reverse = false;
@@ -218,24 +238,33 @@ struct BandCall {
 };
 
 template <class Launch>
-int64_t banded_update(BandPipe& bp, char* hC, int64_t H, size_t row_bytes, int64_t band_rows, const BandCall& bc,
+int64_t banded_update(BandPipe& bp, const Ring& ring, char* hC, int64_t H, size_t row_bytes, const BandCall& bc,
                       cudaStream_t s_comp, Launch&& launch) {
+    const int R = ring.R;
+    const int64_t band_rows = ring.rows;
     const int64_t nb = (H + band_rows - 1) / band_rows;
-    if ((int64_t)bp.out_band.size() < nb || (size_t)band_rows * row_bytes > bp.buf_bytes)
+    if (R < 2 || R > bp.nbuf || (int64_t)bp.out_band.size() < nb || (size_t)band_rows * row_bytes > bp.buf_bytes)
         fail(FPM_ESTATE, "band pipeline not sized for %lld bands of %lld rows", (long long)nb,
              (long long)band_rows);
-    const int64_t nkeep = std::min<int64_t>(2, nb);
-    // the first band of this call is the last band of the previous one: same buffer
-    if (bc.kept_head) bp.ctr -= 1;
+    if (bp.next >= R) bp.next = 0;
+    const int64_t nkeep = std::min<int64_t>(R, nb);
+    if (bc.kept_head) {  // start on the previous call's last band, walk the ring the other way
+        bp.dir = -bp.dir;
+        bp.next = bp.last_step;
+    }
     int64_t launches = 0;
     for (int64_t t = 0; t < nb; ++t) {
         const int64_t j = bc.reverse ? nb - 1 - t : t;
-        const int buf = bp.ctr++ & 1;
+        const int buf = bp.next;
+        bp.next = ((bp.next + bp.dir) % R + R) % R;
         const int64_t r0 = j * band_rows, rows = std::min(band_rows, H - r0);
         const size_t bytes = (size_t)rows * row_bytes;
         const bool resident = bc.kept_head && t < nkeep;  // already in `buf`, current
         if (!resident) {
-            if (bp.used[buf]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out[buf], 0));
+            if (bp.used[buf]) {  // previous occupant updated and (unless kept) copied out
+                CU(cudaStreamWaitEvent(bp.s_h2d, bp.done[buf], 0));
+                CU(cudaStreamWaitEvent(bp.s_h2d, bp.out[buf], 0));
+            }
             if (bc.accumulate) {
                 if (bp.band_used[j]) CU(cudaStreamWaitEvent(bp.s_h2d, bp.out_band[j], 0));
                 CU(cudaMemcpyAsync(bp.buf[buf], hC + (size_t)r0 * row_bytes, bytes, cudaMemcpyHostToDevice,
@@ -248,8 +277,9 @@ int64_t banded_update(BandPipe& bp, char* hC, int64_t H, size_t row_bytes, int64
         launch(r0, rows, bp.buf[buf]);
         ++launches;
         bp.used[buf] = true;
-        if (bc.keep_tail && t >= nb - nkeep) continue;  // stays in the buffer for the next call
+        bp.last_step = buf;
         CU(cudaEventRecord(bp.done[buf], s_comp));
+        if (bc.keep_tail && t >= nb - nkeep) continue;  // stays in the buffer for the next call
         CU(cudaStreamWaitEvent(bp.s_d2h, bp.done[buf], 0));
         CU(cudaMemcpyAsync(hC + (size_t)r0 * row_bytes, bp.buf[buf], bytes, cudaMemcpyDeviceToHost, bp.s_d2h));
         bp.bytes += (int64_t)bytes;
@@ -434,9 +464,9 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         d.B = dalloc(d, HW * es);
         d.ooc = d.c_cap > 0 && (int64_t)(HW * es) > d.c_cap;
         if (d.ooc) {  // C_i in pinned host memory, streamed through two band buffers
-            const int64_t rows = std::min<int64_t>(band_rows_for(d.c_cap, d.W, es), d.H);
+            d.ring = ring_for(d.c_cap, d.H, d.W, es, ctx->ooc_buffers);
             d.hC = static_cast<float*>(halloc(d, HW * es));
-            bp_alloc_bands(d, d.bp, (size_t)rows * d.W * es, (d.H + rows - 1) / rows);
+            bp_alloc_bands(d, d.bp, d.ring.R, (size_t)d.ring.rows * d.W * es, (d.H + d.ring.rows - 1) / d.ring.rows);
         } else {
             d.C = dalloc(d, HW * es);
         }
@@ -703,8 +733,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
             // out of core: the same update, one row band of C_i at a time (rows
             // r0.. of the A operand and its scales, the band buffer as C)
             const size_t op = a.scheme == SplitScheme::F16X3 ? 2 : 4;
-            const int64_t rows = (int64_t)(d.bp.buf_bytes / ((size_t)d.W * 4));
-            d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 4, rows, bc,
+            d.launches += banded_update(d.bp, d.ring, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 4, bc,
                                         d.s_comp, [&](int64_t r0, int64_t m, void* band) {
                                             UpdateArgs x = a;
                                             x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * a.K * op;
@@ -719,10 +748,9 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
             d.launches += 1;
         }
     } else if (d.ooc) {
-        const int64_t rows = (int64_t)(d.bp.buf_bytes / ((size_t)d.W * 8));
         const double* aop = static_cast<const double*>(d.a_op[slot]);
         const int64_t b = ctx->b;
-        d.launches += banded_update(d.bp, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, rows, bc, d.s_comp,
+        d.launches += banded_update(d.bp, d.ring, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, bc, d.s_comp,
                                     [&](int64_t r0, int64_t m, void* band) {
                                         launch_update_f64(aop + (size_t)r0 * b, b,
                                                           static_cast<const double*>(d.bt[slot]),
@@ -1016,7 +1044,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
     };
     // sizes whose C exceeds the device's C cap run out of core (as in the k-loop)
     auto ooc_at = [&](const Device* d, int64_t Lx) { return d->c_cap > 0 && (int64_t)(Lx * Lx * es) > d->c_cap; };
-    auto rows_at = [&](const Device* d, int64_t Lx) { return std::min(band_rows_for(d->c_cap, Lx, es), Lx); };
+    auto ring_at = [&](const Device* d, int64_t Lx) { return ring_for(d->c_cap, Lx, Lx, es, ctx->ooc_buffers); };
     std::vector<std::unique_ptr<Scratch>> S;
     for (Device* d : devs) {
         S.emplace_back(new Scratch);
@@ -1033,7 +1061,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 continue;
             }
             Lout = std::max(Lout, Lx);
-            const int64_t rows = rows_at(d, Lx);
+            const int64_t rows = ring_at(d, Lx).rows;
             nbands = std::max(nbands, (Lx + rows - 1) / rows);
             band_bytes = std::max(band_bytes, (size_t)rows * Lx * es);
         }
@@ -1042,7 +1070,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             bp_init(s.mem.bp);
             s.hC = static_cast<char*>(halloc(s.mem, (size_t)Lout * Lout * es));
             std::memset(s.hC, 0, (size_t)Lout * Lout * es);
-            bp_alloc_bands(s.mem, s.mem.bp, band_bytes, nbands);
+            bp_alloc_bands(s.mem, s.mem.bp, ctx->ooc_buffers, band_bytes, nbands);
         }
         s.Ap = dalloc(s.mem, (size_t)L * fb * es);
         s.Bp = dalloc(s.mem, (size_t)fb * L * es);
@@ -1090,7 +1118,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
                 if (ooc) {
-                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 4, rows_at(s.d, Lx), bc, st,
+                    banded_update(s.mem.bp, ring_at(s.d, Lx), s.hC, Lx, (size_t)Lx * 4, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
                                       UpdateArgs x = a;
                                       x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
@@ -1106,7 +1134,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             } else {
                 launch_transpose_f64(static_cast<const double*>(s.Bp), L, b, Lx, static_cast<double*>(s.Bt), st);
                 if (ooc) {
-                    banded_update(s.mem.bp, s.hC, Lx, (size_t)Lx * 8, rows_at(s.d, Lx), bc, st,
+                    banded_update(s.mem.bp, ring_at(s.d, Lx), s.hC, Lx, (size_t)Lx * 8, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
                                       launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * b, b,
                                                         static_cast<const double*>(s.Bt), static_cast<double*>(band),
@@ -1363,6 +1391,11 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= 0 && value <= 8, "fuse must be 0 (auto) or 1..8");
             if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
             ctx->fuse = (int)value;
+        } else if (k == "ooc_buffers") {
+            FPM_CHECK_ARG(value >= 2 && value <= fpm::kMaxBandBufs, "ooc_buffers must be in [2, %d]",
+                          fpm::kMaxBandBufs);
+            if (ctx->ooc_buffers != (int)value) ctx->have_problem = false;  // band buffers change
+            ctx->ooc_buffers = (int)value;
         } else if (k == "ooc_keep") {
             FPM_CHECK_ARG(value == 0 || value == 1, "ooc_keep must be 0 or 1");
             ctx->ooc_keep = (int)value;

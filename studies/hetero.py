@@ -90,7 +90,9 @@ def main():
                 best = st
         areas = [r[3] * r[4] for r in rects]
         per_dev = list(best.per_dev_compute_s[:p])
-        pred = [a / pkg.fpm_model_speed(m, a) if a > 0 else 0.0 for a, m in zip(areas, models)]
+        # FPM-predicted k-loop time: 2 a b^2 N flop at the model's speed s(a)
+        pred = [2.0 * a * b * b * N / pkg.fpm_model_speed(m, a) if a > 0 else 0.0
+                for a, m in zip(areas, models)]
         results[name] = {
             "d": d, "areas": areas, "rects": rects,
             "t_total_s": best.t_compute_s, "gflops": best.gflops,

@@ -28,18 +28,19 @@ def _inputs(N, dt, dist=synth.DIST_PM1, seeds=(1, 2)):
     return A, B, np.full((N, N), np.nan, dtype=npdt)
 
 
-def _cap_for_band_rows(rows, W, es):
-    """c_cap_bytes that gives bands of `rows` rows (two buffers of rows x W)."""
-    return 2 * rows * W * es
+def _cap_for_band_rows(rows, W, es, R=2):
+    """c_cap_bytes that gives bands of `rows` rows (R buffers of rows x W)."""
+    return R * rows * W * es
 
 
-def _expected_ooc_bytes(H, W, es, band_rows, updates, keep):
+def _expected_ooc_bytes(H, W, es, band_rows, updates, keep, R=2):
     """Host <-> device C bytes of one k-loop, written from P:34 directly: every
     update moves each band in (not the first update: it overwrites) and out;
-    with `keep` the order reverses every other update and the last two bands of
-    an update stay on the device for the next one (not after the last)."""
+    with `keep` the order reverses every other update and the last R bands of
+    an update (the paper: two) stay on the device for the next one (not after
+    the last)."""
     rows = [min(band_rows, H - r0) for r0 in range(0, H, band_rows)]
-    nb, nkeep = len(rows), min(2, len(rows))
+    nb, nkeep = len(rows), min(R, len(rows))
     total = 0
     for g in range(updates):
         order = list(range(nb))[::-1] if keep and g % 2 else list(range(nb))
@@ -52,9 +53,10 @@ def _expected_ooc_bytes(H, W, es, band_rows, updates, keep):
 
 @pytest.mark.parametrize("dt,tol", [(pkg.FPM_F32, 1e-5), (pkg.FPM_F64, 1e-12)])
 @pytest.mark.parametrize("band_rows", [256, 512, 0])
-@pytest.mark.parametrize("keep", [1, 0])
-def test_ooc_device_parity(dt, tol, band_rows, keep):
-    """Device 0 out of core with 1, 3 or 5 bands (ragged), device 1 resident."""
+@pytest.mark.parametrize("keep,R", [(1, 2), (0, 2), (1, 3), (1, 8)])
+def test_ooc_device_parity(dt, tol, band_rows, keep, R):
+    """Device 0 out of core with 1, 3 or 5 bands (ragged), device 1 resident;
+    R band buffers (the paper's two, and rings of 3 and 8)."""
     N, b = 1440, 96          # rect 0 is 1056 x 1440: bands 4 x 256 + 32, 2 x 512 + 32
     n = N // b
     rects = pkg.colpart_arrange(n, [n * n - 60, 60])
@@ -64,14 +66,19 @@ def test_ooc_device_parity(dt, tol, band_rows, keep):
     r0 = rects[0]
     H0, W0 = r0[3] * b, r0[4] * b
     A, B, C = _inputs(N, dt)
+    cap = _cap_for_band_rows(band_rows, W0, es, R) if band_rows else 1
     with pkg.Context.local([0, 0]) as ctx:
         ctx.set_option("ooc_keep", keep)
-        ctx.set_device_option(0, "c_cap_bytes", _cap_for_band_rows(band_rows, W0, es) if band_rows else 1)
+        ctx.set_option("ooc_buffers", R)
+        ctx.set_device_option(0, "c_cap_bytes", cap)
         st = ctx.run(A, B, C, N, b, rects, dt)
     assert og.rel_fro(C, og.gemm(A, B)) <= tol
+    if cap >= H0 * W0 * es:           # C_0 fits the cap: stays resident
+        assert st.ooc_devices == 0 and st.ooc_bytes == 0
+        return
     assert st.ooc_devices == 1
     br = max(band_rows, 256)
-    assert st.ooc_bytes == _expected_ooc_bytes(H0, W0, es, br, st.updates, keep)
+    assert st.ooc_bytes == _expected_ooc_bytes(H0, W0, es, br, st.updates, keep, R)
     if not keep:
         assert st.ooc_bytes == H0 * W0 * es * (2 * st.updates - 1)
     nb = -(-H0 // br)
@@ -85,11 +92,12 @@ def test_ooc_all_devices_integer_exact(fuse):
     N, b = 1024, 64
     n = N // b
     rects = pkg.colpart_arrange(n, [100, 80, 76])
-    for dt, keep in ((pkg.FPM_F32, 1), (pkg.FPM_F64, 1), (pkg.FPM_F32, 0)):
+    for dt, keep, R in ((pkg.FPM_F32, 1, 2), (pkg.FPM_F64, 1, 2), (pkg.FPM_F32, 0, 2), (pkg.FPM_F32, 1, 3)):
         A, B, C = _inputs(N, dt, dist=synth.DIST_INT, seeds=(11, 12))
         with pkg.Context.local([0, 0, 0]) as ctx:
             ctx.set_option("fuse", fuse)
             ctx.set_option("ooc_keep", keep)
+            ctx.set_option("ooc_buffers", R)
             for i in range(3):
                 ctx.set_device_option(i, "c_cap_bytes", 1)  # minimum bands: 256 rows
             st = ctx.run(A, B, C, N, b, rects, dt)
@@ -148,6 +156,9 @@ def test_device_option_errors():
             ctx.set_device_option(0, "c_cap", 1)            # unknown key
         with pytest.raises(pkg.FpmError):
             ctx.set_device_option(0, "c_cap_bytes", -1)
+        for bad in (1, 17):
+            with pytest.raises(pkg.FpmError):
+                ctx.set_option("ooc_buffers", bad)
 
 
 def test_fpm_sample_shows_memory_cliff():
