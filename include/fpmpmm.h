@@ -267,6 +267,16 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 updates; with "ooc_keep" the per-update traffic stays C_i
  *                 minus the cap in each direction.  Fewer buffers (not below
  *                 2) are used when R bands of 256 rows exceed the cap.
+ *   "sm_partition": how an SM cap is enforced.  0 (default): the cap is the
+ *                 grid of the persistent update kernel (one CTA per SM); other
+ *                 kernels of the device are not confined, and devices sharing a
+ *                 GPU may have caps summing above its SM count.  1: every device
+ *                 gets a disjoint green-context partition of exactly its cap
+ *                 (CUDA driver green contexts, SM-pair granularity, one split per
+ *                 GPU) and all its kernels -- update, staging, NCCL -- run inside
+ *                 it.  Needs a cap on every device and the caps of the devices
+ *                 of one GPU to fit it (FPM_EUNSUPPORTED otherwise).  Rebuilds
+ *                 the devices' streams: set it before pmm_setup.
  *   "raster_group": tile-rows per L2 raster group of the update (default 16).
  *   "l2_hint_b":  L2 policy of the B^T operand tiles: 0 normal (default),
  *                 1 evict-first, 2 evict-last.

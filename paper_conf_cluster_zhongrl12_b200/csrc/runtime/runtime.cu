@@ -23,6 +23,7 @@
 #include "../common.hpp"
 #include "../host/host_algos.hpp"
 #include "../kernels/kernels.hpp"
+#include "green.hpp"
 #include "nccl_loader.hpp"
 
 #define CU(expr)                                                                                        \
@@ -71,6 +72,7 @@ struct Device {
     int cuda_dev = 0;
     int sm_cap = 0;    // 0 = all SMs
     int num_sms = 0;   // persistent grid of the update kernel
+    GreenPartition green;  // SM partition (option "sm_partition" = 1), else none
     int64_t c_cap = 0;     // bytes of device memory C_i may use (0 = no limit)
     bool ooc = false;      // C_i out of core for the current problem
     float* hC = nullptr;   // pinned host C_i (H x W) when out of core
@@ -128,6 +130,7 @@ struct pmm_ctx {
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
+    int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
 };
@@ -330,8 +333,14 @@ void init_device(Device& d) {
     } else {
         d.num_sms = sms;
     }
-    CU(cudaStreamCreateWithFlags(&d.s_comp, cudaStreamNonBlocking));
-    CU(cudaStreamCreateWithFlags(&d.s_comm, cudaStreamNonBlocking));
+    if (d.green.ctx) {  // every kernel of this device (update, staging, NCCL) inside its SMs
+        d.num_sms = d.green.sms;
+        d.s_comp = green_stream(d.green);
+        d.s_comm = green_stream(d.green);
+    } else {
+        CU(cudaStreamCreateWithFlags(&d.s_comp, cudaStreamNonBlocking));
+        CU(cudaStreamCreateWithFlags(&d.s_comm, cudaStreamNonBlocking));
+    }
     for (int s = 0; s < 2; ++s) {
         CU(cudaEventCreateWithFlags(&d.ev_ready[s], cudaEventDisableTiming));
         CU(cudaEventCreateWithFlags(&d.ev_free[s], cudaEventDisableTiming));
@@ -355,7 +364,12 @@ void destroy_device(Device& d) {
         if (e) cudaEventDestroy(e);
     if (d.s_comp) cudaStreamDestroy(d.s_comp);
     if (d.s_comm) cudaStreamDestroy(d.s_comm);
+    d.s_comp = d.s_comm = nullptr;
+    for (int s = 0; s < 2; ++s) d.ev_ready[s] = d.ev_free[s] = nullptr;
+    d.ev_start = d.ev_stop = d.ev_io0 = d.ev_io1 = nullptr;
+    green_destroy(d.green);
 }
+
 
 float elapsed_ms(cudaEvent_t a, cudaEvent_t b) {
     float ms = 0.0f;
@@ -379,6 +393,44 @@ void close_peers(pmm_ctx* ctx) {
             ptr = nullptr;
         }
     ctx->peers_ready = false;
+}
+
+// Option "sm_partition": rebuild every device's streams, inside disjoint
+// green-context SM partitions of its cap (on) or on the whole GPU (off).
+void set_sm_partition(pmm_ctx* ctx, bool green) {
+    // carve the partitions first: a failure leaves the context as it was
+    std::vector<GreenPartition> parts(ctx->devs.size());
+    if (green) {
+        for (auto& d : ctx->devs)
+            if (d.sm_cap == 0)
+                fail(FPM_EUNSUPPORTED, "sm_partition = 1 needs an SM cap on every device (device %d has none)", d.idx);
+        try {
+            std::vector<int> gpus;
+            for (auto& d : ctx->devs)
+                if (std::find(gpus.begin(), gpus.end(), d.cuda_dev) == gpus.end()) gpus.push_back(d.cuda_dev);
+            for (int g : gpus) {  // one split per GPU: the partitions of its devices are disjoint
+                std::vector<size_t> on;
+                std::vector<int> caps;
+                for (size_t i = 0; i < ctx->devs.size(); ++i)
+                    if (ctx->devs[i].cuda_dev == g) {
+                        on.push_back(i);
+                        caps.push_back(ctx->devs[i].sm_cap);
+                    }
+                std::vector<GreenPartition> got = green_partitions(g, caps);
+                for (size_t i = 0; i < on.size(); ++i) parts[on[i]] = got[i];
+            }
+        } catch (...) {
+            for (auto& gp : parts) green_destroy(gp);
+            throw;
+        }
+    }
+    close_peers(ctx);
+    for (auto& d : ctx->devs) destroy_device(d);
+    ctx->have_problem = false;
+    for (size_t i = 0; i < ctx->devs.size(); ++i) {
+        ctx->devs[i].green = parts[i];
+        init_device(ctx->devs[i]);
+    }
 }
 
 // Resident A_q / B_q of device q: local devices directly, IPC peers through the
@@ -1391,6 +1443,12 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= 0 && value <= 8, "fuse must be 0 (auto) or 1..8");
             if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
             ctx->fuse = (int)value;
+        } else if (k == "sm_partition") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "sm_partition must be 0 (grid caps) or 1 (green contexts)");
+            if (ctx->sm_partition != (int)value) {
+                fpm::set_sm_partition(ctx, value == 1);
+                ctx->sm_partition = (int)value;
+            }
         } else if (k == "ooc_buffers") {
             FPM_CHECK_ARG(value >= 2 && value <= fpm::kMaxBandBufs, "ooc_buffers must be in [2, %d]",
                           fpm::kMaxBandBufs);
