@@ -238,7 +238,10 @@ int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int6
  * half-width is <= 2.5% of the mean (>= 5, <= 50 repetitions, reading Q8).
  * dev = -1 samples every device of the context simultaneously (P:10 (ii)
  * "processes are synchronised", so shared resources are contended as in the
- * run); the outputs are then p x nsizes, device-major.
+ * run): after the warm-ups each device runs its kernel k_i = round(t_max /
+ * t_i) times (<= 64) per repetition, so all stay busy for the same window, and
+ * a run's time is the window / k_i.  The outputs are then p x nsizes,
+ * device-major.
  * rel_ci95_out / reps_out nullable. */
 int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t* sizes,
                int32_t nsizes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out);

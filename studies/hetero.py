@@ -48,6 +48,8 @@ def main():
     ap.add_argument("--sizes", default="1,2,3,4,6,8,12,16,20,24,28,32,40")
     ap.add_argument("--concurrent", dest="exclusive", action="store_false",
                     help="sample all devices at once (P:10 (ii)) instead of each alone (P:11, default)")
+    ap.add_argument("--sm-partition", type=int, default=0,
+                    help="1 = each device in its own green-context SM partition (all its kernels confined)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
     args = ap.parse_args()
     caps = [int(c) for c in args.caps.split(",")]
@@ -57,6 +59,7 @@ def main():
     sizes = [int(m) ** 2 for m in args.sizes.split(",")]
 
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
+    ctx.set_option("sm_partition", args.sm_partition)
     t0 = time.perf_counter()
     models, sample_info = [], []
     if args.exclusive:   # each device alone (how the paper measured its GPUs)
@@ -114,7 +117,7 @@ def main():
         st1 = one.compute()
     out = {
         "config": {"N": N, "b": b, "p": p, "sm_caps": caps, "ncal": args.ncal, "x_cal": x_cal, "x_even": x_even,
-                   "sizes": sizes, "dtype": "f32 (F16X3)", "gpu": "1x B200, devices emulated by SM caps",
+                   "sizes": sizes, "dtype": "f32 (F16X3)", "sm_partition": args.sm_partition, "gpu": "1x B200, devices emulated by SM caps",
                    "sampling": "exclusive" if args.exclusive else "concurrent (all devices at once)"},
         "fpm_sample_s": t_sample, "models": sample_info, "partitions": results,
         "whole_gpu": {"t_s": st1.t_compute_s, "gflops": st1.gflops},

@@ -92,6 +92,8 @@ def main():
     ap.add_argument("--concurrent", action="store_true",
                     help="sample all devices at once (P:10 (ii)): the out-of-core GPUs then share the "
                          "host link as they do in the run")
+    ap.add_argument("--sm-partition", type=int, default=0,
+                    help="1 = each device in its own green-context SM partition (all its kernels confined)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "memcap_table3_r01.json"))
     args = ap.parse_args()
     caps = [int(c) for c in args.caps.split(",")]
@@ -104,6 +106,7 @@ def main():
     pcie = pcie_bandwidth()
     print("pcie", pcie, flush=True)
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
+    ctx.set_option("sm_partition", args.sm_partition)
     ctx.set_option("ooc_keep", args.ooc_keep)
     ctx.set_option("ooc_buffers", args.ooc_buffers)
     for dev, cap in enumerate(c_caps):
@@ -165,7 +168,7 @@ def main():
         "config": {"b": b, "ns": ns, "p": p, "names": names, "sm_caps": caps, "c_cap_bytes": c_caps,
                    "ncal": args.ncal, "x_cal": x_cal, "sizes": sizes, "ooc_keep": args.ooc_keep, "ooc_buffers": args.ooc_buffers,
                    "sampling": "concurrent (all devices at once)" if args.concurrent else "exclusive",
-                   "dtype": "f32 (F16X3)",
+                   "dtype": "f32 (F16X3)", "sm_partition": args.sm_partition,
                    "gpu": "1x B200; devices emulated by SM caps, device memory by C caps (C_i out of core above)"},
         "pcie": pcie, "fpm_sample_s": t_sample, "models": sample_info, "table": table,
     }
