@@ -209,6 +209,15 @@ int pmm_fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int32_t d
  * for compatibility and has no effect.  Blocks until done. */
 int pmm_compute(pmm_ctx* ctx, int32_t zero_c, pmm_stats* stats);
 
+/* pmm_compute, then C_i into a host window (convention of pmm_download), with
+ * the device -> host copy overlapped with the last updates: the last L update
+ * groups (option "e2e_tail") run band-major over rows of C_i, and each band is
+ * copied out as soon as it is final.  Every element still receives the
+ * updates in k order.  Devices without a tail (FP64, out-of-core) are copied
+ * after the loop.  stats->t_download_s = copy time after the last update. */
+int pmm_compute_into(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base,
+                     pmm_stats* stats);
+
 /* Copy this process's C_i into a host window (same convention as upload). */
 int pmm_download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base);
 
@@ -222,7 +231,7 @@ int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t rows, int64
  * iterations with the inputs streamed from the host windows (block-column k of
  * A and block-row k of B are copied host -> device on the communication stream
  * just ahead of iteration k, overlapping earlier updates), then the download
- * of C.  A, B, C are host windows as for pmm_upload (pinned memory gives
+ * of C, overlapped with the last updates as in pmm_compute_into.  A, B, C are host windows as for pmm_upload (pinned memory gives
  * asynchronous copies).  stats: t_compute_s includes the streamed upload,
  * t_upload_s = time until the last panel landed, t_download_s. */
 int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int64_t b,
@@ -270,6 +279,10 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 updates; with "ooc_keep" the per-update traffic stays C_i
  *                 minus the cap in each direction.  Fewer buffers (not below
  *                 2) are used when R bands of 256 rows exceed the cap.
+ *   "e2e_tail":   update groups run band-major at the end of pmm_run /
+ *                 pmm_compute_into so the copy of C_i to the host overlaps them
+ *                 (FP32, resident C_i): -1 auto (default: enough groups to
+ *                 cover the copy at ~55 GB/s), 0 off, 1..16.
  *   "sm_partition": how an SM cap is enforced.  0 (default): the cap is the
  *                 grid of the persistent update kernel (one CTA per SM); other
  *                 kernels of the device are not confined, and devices sharing a

@@ -156,6 +156,14 @@ class Context:
         check(lib.pmm_compute(self._h, 1 if zero_c else 0, ctypes.byref(st)))
         return st
 
+    def compute_into(self, C, ld: int, row_base: int = 0, col_base: int = 0) -> PmmStats:
+        """pmm_compute + download of C_i into the host window, the copy
+        overlapped with the last updates (include/fpmpmm.h pmm_compute_into)."""
+        st = PmmStats()
+        check(lib.pmm_compute_into(self._h, _lib._ptr(C), int(ld), int(row_base), int(col_base),
+                                   ctypes.byref(st)))
+        return st
+
     def download(self, C, ld: int, row_base: int = 0, col_base: int = 0) -> None:
         check(lib.pmm_download(self._h, _lib._ptr(C), int(ld), int(row_base), int(col_base)))
 

@@ -95,6 +95,7 @@ _SIGS = {
     "pmm_ipc_import": ([vp, ctypes.c_char_p, i32], ctypes.c_int),
     "pmm_destroy": ([vp], ctypes.c_int),
     "pmm_set_option": ([vp, ctypes.c_char_p, i64], ctypes.c_int),
+    "pmm_compute_into": ([vp, vp, i64, i64, i64, ctypes.POINTER(PmmStats)], ctypes.c_int),
     "pmm_set_device_option": ([vp, i32, ctypes.c_char_p, i64], ctypes.c_int),
     "pmm_setup": ([vp, i64, i64, i32, ctypes.POINTER(ColpartRect), ctypes.c_int], ctypes.c_int),
     "pmm_upload": ([vp, vp, vp, i64, i64, i64], ctypes.c_int),

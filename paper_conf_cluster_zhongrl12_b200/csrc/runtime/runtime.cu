@@ -48,6 +48,8 @@ namespace fpm {
 // band and the D2H of an earlier one overlap the update of the current band on
 // three streams.
 constexpr int kMaxBandBufs = 16;
+constexpr int kMaxTail = 16;             // groups of the download-overlapped tail
+constexpr int kSlots = 2 + kMaxTail;     // operand slots per device
 struct Ring {
     int R;         // buffers in use
     int64_t rows;  // rows per band
@@ -80,7 +82,8 @@ struct Device {
     BandPipe bp;
     Ring ring{0, 0};       // out-of-core band geometry of the current problem
     cudaStream_t s_comp = nullptr, s_comm = nullptr;
-    cudaEvent_t ev_ready[2] = {}, ev_free[2] = {};
+    cudaStream_t s_up = nullptr;  // pmm_run: host -> device panel uploads, run ahead of the staging
+    cudaEvent_t ev_ready[kSlots] = {}, ev_free[kSlots] = {};
     cudaEvent_t ev_start = nullptr, ev_stop = nullptr, ev_io0 = nullptr, ev_io1 = nullptr;
     std::vector<cudaEvent_t> ev_pack0, ev_pack1, ev_upd0, ev_upd1, ev_up;
 
@@ -90,11 +93,14 @@ struct Device {
     void* A = nullptr;     // w block-columns, each H x b row-major (K-major panels)
     void* B = nullptr;     // H x W row-major (h block-rows of b x W)
     void* C = nullptr;     // H x W row-major
-    void* a_recv[2] = {}, *b_recv[2] = {};
-    void* bt[2] = {};                       // W x b (K-major) transposed B pivot row
-    void* a_hi[2] = {}, *a_lo[2] = {}, *b_hi[2] = {}, *b_lo[2] = {};
-    float* sa[2] = {}, *sb[2] = {};
-    const void* a_op[2] = {};               // FP64: A operand of the slot
+    // operand slots: 0, 1 double-buffer the k-loop; 2 .. 2+tail_slots-1 hold the
+    // groups of the download-overlapped tail (compute_into, allocated on demand)
+    void* a_recv[kSlots] = {}, *b_recv[kSlots] = {};
+    void* bt[kSlots] = {};                  // W x b (K-major) transposed B pivot row
+    void* a_hi[kSlots] = {}, *a_lo[kSlots] = {}, *b_hi[kSlots] = {}, *b_lo[kSlots] = {};
+    float* sa[kSlots] = {}, *sb[kSlots] = {};
+    const void* a_op[kSlots] = {};          // FP64: A operand of the slot
+    int tail_slots = 0;                     // slots 2.. allocated
     std::vector<void*> allocs;
     int64_t launches = 0;                   // library kernels launched (running count)
 
@@ -130,6 +136,7 @@ struct pmm_ctx {
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
+    int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
@@ -314,7 +321,8 @@ void free_problem(Device& d) {
         v->clear();
     }
     d.A = d.B = d.C = nullptr;
-    for (int s = 0; s < 2; ++s) {
+    d.tail_slots = 0;
+    for (int s = 0; s < kSlots; ++s) {
         d.a_recv[s] = d.b_recv[s] = d.bt[s] = d.a_hi[s] = d.a_lo[s] = d.b_hi[s] = d.b_lo[s] = nullptr;
         d.sa[s] = d.sb[s] = nullptr;
         d.a_op[s] = nullptr;
@@ -341,7 +349,8 @@ void init_device(Device& d) {
         CU(cudaStreamCreateWithFlags(&d.s_comp, cudaStreamNonBlocking));
         CU(cudaStreamCreateWithFlags(&d.s_comm, cudaStreamNonBlocking));
     }
-    for (int s = 0; s < 2; ++s) {
+    CU(cudaStreamCreateWithFlags(&d.s_up, cudaStreamNonBlocking));  // copies only: no SM partition
+    for (int s = 0; s < kSlots; ++s) {
         CU(cudaEventCreateWithFlags(&d.ev_ready[s], cudaEventDisableTiming));
         CU(cudaEventCreateWithFlags(&d.ev_free[s], cudaEventDisableTiming));
     }
@@ -356,7 +365,7 @@ void destroy_device(Device& d) {
     free_problem(d);
     cudaSetDevice(d.cuda_dev);
     bp_destroy(d.bp);
-    for (int s = 0; s < 2; ++s) {
+    for (int s = 0; s < kSlots; ++s) {
         if (d.ev_ready[s]) cudaEventDestroy(d.ev_ready[s]);
         if (d.ev_free[s]) cudaEventDestroy(d.ev_free[s]);
     }
@@ -364,8 +373,9 @@ void destroy_device(Device& d) {
         if (e) cudaEventDestroy(e);
     if (d.s_comp) cudaStreamDestroy(d.s_comp);
     if (d.s_comm) cudaStreamDestroy(d.s_comm);
-    d.s_comp = d.s_comm = nullptr;
-    for (int s = 0; s < 2; ++s) d.ev_ready[s] = d.ev_free[s] = nullptr;
+    if (d.s_up) cudaStreamDestroy(d.s_up);
+    d.s_comp = d.s_comm = d.s_up = nullptr;
+    for (int s = 0; s < kSlots; ++s) d.ev_ready[s] = d.ev_free[s] = nullptr;
     d.ev_start = d.ev_stop = d.ev_io0 = d.ev_io1 = nullptr;
     green_destroy(d.green);
 }
@@ -455,6 +465,30 @@ int fuse_factor(pmm_ctx* ctx, fpm_dtype dt, int64_t b) {
 }
 
 // ---------------------------------------------------------------- setup
+// Operand buffers of one slot: receive buffers (NCCL lands pivots in them;
+// FP64 copies peers' pivots into them -- FP32 in local / IPC mode stages
+// straight from the peers' memory) and the staged operands of a fused update.
+void alloc_slot(pmm_ctx* ctx, Device& d, int s) {
+    const fpm_dtype dt = ctx->dt;
+    const size_t es = esize(dt);
+    const size_t op = (dt == FPM_F64) ? 0 : (ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4);
+    const bool need_recv = ctx->nccl_mode || dt == FPM_F64;
+    const size_t fb = (size_t)ctx->fuse_max * ctx->b;  // K of a fused update
+    if (need_recv) {
+        d.a_recv[s] = dalloc(d, (size_t)d.H * fb * es);  // f panels of H x b
+        d.b_recv[s] = dalloc(d, fb * d.W * es);          // f block-rows of b x W
+    }
+    if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * ctx->b * es);
+    if (dt == FPM_F32) {
+        d.a_hi[s] = dalloc(d, (size_t)d.H * fb * op);
+        d.a_lo[s] = dalloc(d, (size_t)d.H * fb * op);
+        d.b_hi[s] = dalloc(d, (size_t)d.W * fb * op);
+        d.b_lo[s] = dalloc(d, (size_t)d.W * fb * op);
+        d.sa[s] = static_cast<float*>(dalloc(d, (size_t)d.H * sizeof(float)));
+        d.sb[s] = static_cast<float*>(dalloc(d, (size_t)d.W * sizeof(float)));
+    }
+}
+
 void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects, fpm_dtype dt) {
     FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype %d", (int)dt);
     FPM_CHECK_ARG(N >= 1 && b >= 1 && N % b == 0, "b must divide N (N=%lld, b=%lld)", (long long)N,
@@ -522,26 +556,7 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         } else {
             d.C = dalloc(d, HW * es);
         }
-        const size_t op = (dt == FPM_F64) ? 0 : (ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4);
-        // receive buffers: NCCL lands pivots in them; FP64 copies peers' pivots into
-        // them.  FP32 in local / IPC mode stages straight from the peers' memory.
-        const bool need_recv = ctx->nccl_mode || dt == FPM_F64;
-        const size_t fb = (size_t)f * b;  // K of a fused update
-        for (int s = 0; s < 2; ++s) {
-            if (need_recv) {
-                d.a_recv[s] = dalloc(d, (size_t)d.H * fb * es);  // f panels of H x b
-                d.b_recv[s] = dalloc(d, fb * d.W * es);          // f block-rows of b x W
-            }
-            if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * b * es);
-            if (dt == FPM_F32) {
-                d.a_hi[s] = dalloc(d, (size_t)d.H * fb * op);
-                d.a_lo[s] = dalloc(d, (size_t)d.H * fb * op);
-                d.b_hi[s] = dalloc(d, (size_t)d.W * fb * op);
-                d.b_lo[s] = dalloc(d, (size_t)d.W * fb * op);
-                d.sa[s] = static_cast<float*>(dalloc(d, (size_t)d.H * sizeof(float)));
-                d.sb[s] = static_cast<float*>(dalloc(d, (size_t)d.W * sizeof(float)));
-            }
-        }
+        for (int s = 0; s < 2; ++s) alloc_slot(ctx, d, s);
         for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1, &d.ev_up}) {
             v->resize(n);
             for (auto& e : *v) CU(cudaEventCreate(&e));
@@ -595,15 +610,15 @@ void issue_upload(pmm_ctx* ctx, Device& d, int64_t k, const HostSrc& h) {
         const int64_t c = k - r.col0;
         const char* src = static_cast<const char*>(h.A) + ((size_t)R0 * h.ld + (size_t)(C0 + c * b)) * es;
         char* dst = static_cast<char*>(d.A) + (size_t)c * d.H * b * es;
-        CU(cudaMemcpy2DAsync(dst, b * es, src, h.ld * es, b * es, d.H, cudaMemcpyHostToDevice, d.s_comm));
+        CU(cudaMemcpy2DAsync(dst, b * es, src, h.ld * es, b * es, d.H, cudaMemcpyHostToDevice, d.s_up));
     }
     if (r.row0 <= k && k < r.row0 + r.h) {
         const int64_t rr = k - r.row0;
         const char* src = static_cast<const char*>(h.B) + ((size_t)(R0 + rr * b) * h.ld + (size_t)C0) * es;
         char* dst = static_cast<char*>(d.B) + (size_t)rr * b * d.W * es;
-        CU(cudaMemcpy2DAsync(dst, d.W * es, src, h.ld * es, d.W * es, b, cudaMemcpyHostToDevice, d.s_comm));
+        CU(cudaMemcpy2DAsync(dst, d.W * es, src, h.ld * es, d.W * es, b, cudaMemcpyHostToDevice, d.s_up));
     }
-    CU(cudaEventRecord(d.ev_up[k], d.s_comm));
+    CU(cudaEventRecord(d.ev_up[k], d.s_up));
 }
 
 // Exchange + staging of update group g (pivots k0 .. k0+f-1) on device d's comm
@@ -619,6 +634,9 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     int64_t bytes = 0;
     CU(cudaSetDevice(d.cuda_dev));
     if (!first_use) CU(cudaStreamWaitEvent(d.s_comm, d.ev_free[slot], 0));
+    // streamed input: this device's own panels of the group have landed (the
+    // upload stream runs ahead, in k order)
+    if (streamed) CU(cudaStreamWaitEvent(d.s_comm, d.ev_up[kl], 0));
     const colpart_rect& r = d.rect;
 
     // FP32 in local / IPC mode: the staging kernels read the pivots straight from
@@ -747,6 +765,44 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     return bytes;
 }
 
+// FP32 update of group g from operand slot `slot` over all of C_i.
+UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
+    UpdateArgs a;
+    a.a_hi = d.a_hi[slot];
+    a.a_lo = d.a_lo[slot];
+    a.bt_hi = d.b_hi[slot];
+    a.bt_lo = d.b_lo[slot];
+    const bool f16 = ctx->f32_scheme == (int)SplitScheme::F16X3;
+    a.sa = f16 ? d.sa[slot] : nullptr;
+    a.sb = f16 ? d.sb[slot] : nullptr;
+    a.C = static_cast<float*>(d.C);
+    a.M = d.H;
+    a.Nc = d.W;
+    a.K = (int64_t)ctx->groups[g].second * ctx->b;
+    a.ldc = d.W;
+    a.scheme = (SplitScheme)ctx->f32_scheme;
+    a.cta_group = ctx->cta_group;
+    a.num_sms = d.num_sms;
+    a.accumulate = ctx->groups[g].first != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
+    a.raster_group = ctx->raster_group;
+    a.l2_hint_b = ctx->l2_hint_b;
+    a.variant = ctx->kernel_variant;  // -1: auto (variant 4, leaves smem for co-running kernels)
+    return a;
+}
+
+// The same update restricted to rows [r0, r0 + m) of C_i, written to `Cband`
+// (row stride W): rows r0.. of the A operand and of its scales.
+UpdateArgs band_args(const UpdateArgs& a, int64_t r0, int64_t m, float* Cband) {
+    const size_t op = a.scheme == SplitScheme::F16X3 ? 2 : 4;
+    UpdateArgs x = a;
+    x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * a.K * op;
+    x.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * a.K * op;
+    x.sa = a.sa ? a.sa + r0 : nullptr;
+    x.C = Cband;
+    x.M = m;
+    return x;
+}
+
 void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
     const int64_t k0 = ctx->groups[g].first;
     const int f = ctx->groups[g].second;
@@ -761,39 +817,14 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
     bc.kept_head = ctx->ooc_keep && g > 0;
     bc.keep_tail = ctx->ooc_keep && g + 1 < (int)ctx->groups.size();
     if (ctx->dt == FPM_F32) {
-        UpdateArgs a;
-        a.a_hi = d.a_hi[slot];
-        a.a_lo = d.a_lo[slot];
-        a.bt_hi = d.b_hi[slot];
-        a.bt_lo = d.b_lo[slot];
-        const bool f16 = ctx->f32_scheme == (int)SplitScheme::F16X3;
-        a.sa = f16 ? d.sa[slot] : nullptr;
-        a.sb = f16 ? d.sb[slot] : nullptr;
-        a.C = static_cast<float*>(d.C);
-        a.M = d.H;
-        a.Nc = d.W;
-        a.K = (int64_t)f * ctx->b;
-        a.ldc = d.W;
-        a.scheme = (SplitScheme)ctx->f32_scheme;
-        a.cta_group = ctx->cta_group;
-        a.num_sms = d.num_sms;
-        a.accumulate = k0 != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
-        a.raster_group = ctx->raster_group;
-        a.l2_hint_b = ctx->l2_hint_b;
-        a.variant = ctx->kernel_variant;  // -1: auto (variant 4, leaves smem for co-running kernels)
+        const UpdateArgs a = f32_args(ctx, d, g, slot);
         if (d.ooc) {
             // out of core: the same update, one row band of C_i at a time (rows
             // r0.. of the A operand and its scales, the band buffer as C)
-            const size_t op = a.scheme == SplitScheme::F16X3 ? 2 : 4;
             d.launches += banded_update(d.bp, d.ring, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 4, bc,
                                         d.s_comp, [&](int64_t r0, int64_t m, void* band) {
-                                            UpdateArgs x = a;
-                                            x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * a.K * op;
-                                            x.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * a.K * op;
-                                            x.sa = a.sa ? a.sa + r0 : nullptr;
-                                            x.C = static_cast<float*>(band);
-                                            x.M = m;
-                                            launch_update_f32(x, d.s_comp);
+                                            launch_update_f32(band_args(a, r0, m, static_cast<float*>(band)),
+                                                              d.s_comp);
                                         });
         } else {
             launch_update_f32(a, d.s_comp);
@@ -821,11 +852,90 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
 // The N/b iterations.  Iteration 0 writes C_i = A(0) B(0), so C needs no
 // zeroing.  With `host` set, the pivot panels are streamed from host memory one
 // iteration ahead of their use (pmm_run).
-void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
+// Host destination of C for compute_into / pmm_run.
+struct HostDst {
+    void* C;
+    int64_t ld, row_base, col_base;
+};
+
+// Groups of the download-overlapped tail (option "e2e_tail"; FP32, resident
+// C_i).  Auto: enough of the last updates to cover the device -> host copy of
+// C_i: per element of C_i the copy costs 4 B at ~55 GB/s, the k-loop 2 N flop
+// at ~3 TFLOP/s per SM (measured), so L = ceil(G * 1.15 * ratio).
+int tail_groups(pmm_ctx* ctx) {
+    const int G = (int)ctx->groups.size();
+    if (ctx->dt != FPM_F32 || ctx->e2e_tail == 0 || G == 0) return 0;
+    if (ctx->e2e_tail > 0) return std::min({ctx->e2e_tail, G, kMaxTail});
+    double r = 0.0;
+    for (auto& d : ctx->devs)
+        if (d.live() && !d.ooc) r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (3.0e12 * d.num_sms)));
+    if (r == 0.0) return 0;
+    return std::max(1, std::min({(int)std::ceil(G * 1.15 * r), G, kMaxTail}));
+}
+
+// Operand slots 2 .. 2+L-1 for the tail groups (allocated once per problem).
+void ensure_tail_slots(pmm_ctx* ctx, Device& d, int L) {
+    CU(cudaSetDevice(d.cuda_dev));
+    for (; d.tail_slots < L; ++d.tail_slots) alloc_slot(ctx, d, 2 + d.tail_slots);
+}
+
+// The tail of the k-loop, band-major: for each band of C_i rows, the updates of
+// the L tail groups (slots 2..), then its device -> host copy on the copy
+// stream -- band j's copy overlaps the updates of bands j+1.., so only the last
+// band's copy is exposed.  The same sums in the same order per element as the
+// group-major loop (each element still receives the groups in k order).
+void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
+    CU(cudaSetDevice(d.cuda_dev));
+    for (int t = 0; t < L; ++t) CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[2 + t], 0));
+    CU(cudaEventRecord(d.ev_upd0[g0], d.s_comp));
+    const int64_t band = std::min<int64_t>(d.H, 2048);  // whole CTA-pair tile rows
+    const int64_t b = ctx->b;
+    const int64_t R0 = d.rect.row0 * b - out.row_base, C0 = d.rect.col0 * b - out.col_base;
+    float* C = static_cast<float*>(d.C);
+    for (int64_t r0 = 0; r0 < d.H; r0 += band) {
+        const int64_t m = std::min(band, d.H - r0);
+        for (int t = 0; t < L; ++t) {
+            const UpdateArgs a = f32_args(ctx, d, g0 + t, 2 + t);
+            launch_update_f32(band_args(a, r0, m, C + (size_t)r0 * d.W), d.s_comp);
+            d.launches += 1;
+        }
+        CU(cudaEventRecord(d.bp.done[0], d.s_comp));
+        CU(cudaStreamWaitEvent(d.bp.s_d2h, d.bp.done[0], 0));
+        char* dst = static_cast<char*>(out.C) + ((size_t)(R0 + r0) * out.ld + (size_t)C0) * 4;
+        CU(cudaMemcpy2DAsync(dst, out.ld * 4, C + (size_t)r0 * d.W, d.W * 4, d.W * 4, m, cudaMemcpyDeviceToHost,
+                             d.bp.s_d2h));
+    }
+    CU(cudaEventRecord(d.ev_upd1[g0], d.s_comp));
+    for (int t = 1; t < L; ++t) {  // the tail's time is booked on its first group
+        CU(cudaEventRecord(d.ev_upd0[g0 + t], d.s_comp));
+        CU(cudaEventRecord(d.ev_upd1[g0 + t], d.s_comp));
+    }
+    for (int t = 0; t < L; ++t) CU(cudaEventRecord(d.ev_free[2 + t], d.s_comp));
+    CU(cudaEventRecord(d.ev_io1, d.bp.s_d2h));  // C_i in host memory
+}
+
+// The N/b iterations.  Iteration 0 writes C_i = A(0) B(0), so C needs no
+// zeroing.  With `host` set, the pivot panels are streamed from host memory one
+// iteration ahead of their use (pmm_run).  With `out` set, C_i is also copied
+// to host memory, overlapped with the last updates where possible (tail);
+// returns true for each device whose copy was done here (tail_done).
+void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const HostDst* out = nullptr,
+             std::vector<char>* tail_done = nullptr) {
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
     if (ctx->ipc_mode && !ctx->peers_ready)
         fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
     FPM_CHECK_ARG(!(ctx->ipc_mode && host), "IPC mode has no streamed host input (peers cannot be ordered)");
+    const int ngroups = (int)ctx->groups.size();
+    const int L = out ? tail_groups(ctx) : 0;
+    const int gt = ngroups - L;  // first tail group
+    if (tail_done) tail_done->assign(ctx->devs.size(), 0);
+    for (size_t i = 0; i < ctx->devs.size(); ++i) {
+        Device& d = ctx->devs[i];
+        if (L > 0 && d.live() && !d.ooc) {
+            ensure_tail_slots(ctx, d, L);  // before the timed region (cudaMalloc synchronises)
+            if (tail_done) (*tail_done)[i] = 1;
+        }
+    }
     int64_t launches0 = 0;
     for (auto& d : ctx->devs) {
         launches0 += d.launches;
@@ -841,12 +951,15 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventRecord(d.ev_start, d.s_comp));
         CU(cudaStreamWaitEvent(d.s_comm, d.ev_start, 0));
+        CU(cudaStreamWaitEvent(d.s_up, d.ev_start, 0));
     }
     const bool streamed = host != nullptr;
     int64_t bytes = 0;
-    const int ngroups = (int)ctx->groups.size();
+    // tail devices take tail groups from slots 2.. and update them band-major
+    // after the loop; everyone else (and every group before gt) as usual
+    auto in_tail = [&](const Device& d, int g) { return g >= gt && d.live() && !d.ooc; };
+    auto slot_of = [&](const Device& d, int g) { return in_tail(d, g) ? 2 + (g - gt) : (g & 1); };
     for (int g = 0; g < ngroups; ++g) {
-        const int slot = g & 1;
         const int64_t k0 = ctx->groups[g].first;
         if (streamed)
             for (int64_t k = k0; k < k0 + ctx->groups[g].second; ++k)
@@ -856,8 +969,9 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
             // every rank takes part in the NCCL calls, live or not
             Device& d = ctx->devs[0];
             if (d.live()) {
-                bytes += issue_comm(ctx, d, g, slot, g < 2, streamed);
-                issue_update(ctx, d, g, slot);
+                const int slot = slot_of(d, g);
+                bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed);
+                if (!in_tail(d, g)) issue_update(ctx, d, g, slot);
             } else {
                 NC(nccl().GroupStart());
                 NC(nccl().GroupEnd());
@@ -865,10 +979,16 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
             continue;
         }
         for (auto& d : ctx->devs)
-            if (d.live()) bytes += issue_comm(ctx, d, g, slot, g < 2, streamed);
+            if (d.live()) {
+                const int slot = slot_of(d, g);
+                bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed);
+            }
         for (auto& d : ctx->devs)
-            if (d.live()) issue_update(ctx, d, g, slot);
+            if (d.live() && !in_tail(d, g)) issue_update(ctx, d, g, g & 1);
     }
+    if (L > 0)
+        for (auto& d : ctx->devs)
+            if (d.live() && !d.ooc) issue_tail(ctx, d, gt, L, *out);
     int64_t launches = -launches0;
     for (auto& d : ctx->devs) launches += d.launches;
     for (auto& d : ctx->devs) {
@@ -876,16 +996,22 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr) {
         if (d.ooc) bp_join(d.bp, d.s_comp);  // C_i is complete once its last band is back in host memory
         CU(cudaEventRecord(d.ev_stop, d.s_comp));
     }
-    double t_max = 0.0;
-    for (auto& d : ctx->devs) {
+    double t_max = 0.0, t_tail_copy = 0.0;
+    for (size_t i = 0; i < ctx->devs.size(); ++i) {
+        Device& d = ctx->devs[i];
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventSynchronize(d.ev_stop));
         CU(cudaStreamSynchronize(d.s_comm));
         t_max = std::max(t_max, (double)elapsed_ms(d.ev_start, d.ev_stop) * 1e-3);
+        if (tail_done && (*tail_done)[i]) {  // copy still draining after the last update
+            CU(cudaEventSynchronize(d.ev_io1));
+            t_tail_copy = std::max(t_tail_copy, std::max(0.0, (double)elapsed_ms(d.ev_stop, d.ev_io1) * 1e-3));
+        }
     }
     if (st) {
         std::memset(st, 0, sizeof(*st));
         st->t_compute_s = t_max;
+        st->t_download_s = t_tail_copy;
         if (streamed) {
             double tu = 0.0;  // until the last host->device panel landed
             for (auto& d : ctx->devs)
@@ -970,14 +1096,18 @@ void upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld, int64_t row_
     if (t_out) *t_out = t;
 }
 
-void download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base, double* t_out) {
+void download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base, double* t_out,
+              const std::vector<char>* skip = nullptr) {
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_download before pmm_setup");
     FPM_CHECK_ARG(C, "null host matrix");
     const size_t es = esize(ctx->dt);
     const int64_t b = ctx->b;
     double t = 0.0;
-    for (auto& d : ctx->devs) {
-        if (!d.live()) continue;
+    std::vector<char> copied(ctx->devs.size(), 0);
+    for (size_t i = 0; i < ctx->devs.size(); ++i) {
+        Device& d = ctx->devs[i];
+        if (!d.live() || (skip && (*skip)[i])) continue;
+        copied[i] = 1;
         check_window(ctx, d, ld, row_base, col_base);
         CU(cudaSetDevice(d.cuda_dev));
         const int64_t R0 = d.rect.row0 * b - row_base, C0 = d.rect.col0 * b - col_base;
@@ -991,8 +1121,9 @@ void download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_b
         }
         CU(cudaEventRecord(d.ev_io1, d.s_comp));
     }
-    for (auto& d : ctx->devs) {
-        if (!d.live()) continue;
+    for (size_t i = 0; i < ctx->devs.size(); ++i) {
+        Device& d = ctx->devs[i];
+        if (!copied[i]) continue;
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventSynchronize(d.ev_io1));
         t = std::max(t, (double)elapsed_ms(d.ev_io0, d.ev_io1) * 1e-3);
@@ -1461,6 +1592,10 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= 0 && value <= 8, "fuse must be 0 (auto) or 1..8");
             if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
             ctx->fuse = (int)value;
+        } else if (k == "e2e_tail") {
+            FPM_CHECK_ARG(value >= -1 && value <= fpm::kMaxTail, "e2e_tail must be -1 (auto), 0 (off) or 1..%d",
+                          fpm::kMaxTail);
+            ctx->e2e_tail = (int)value;
         } else if (k == "sm_partition") {
             FPM_CHECK_ARG(value == 0 || value == 1, "sm_partition must be 0 (grid caps) or 1 (green contexts)");
             if (ctx->sm_partition != (int)value) {
@@ -1536,6 +1671,24 @@ extern "C" int pmm_compute(pmm_ctx* ctx, int32_t zero_c, pmm_stats* stats) {
     });
 }
 
+extern "C" int pmm_compute_into(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base,
+                                pmm_stats* stats) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr && C != nullptr, "null argument");
+        if (!ctx->have_problem) fpm::fail(FPM_ESTATE, "pmm_compute_into before pmm_setup");
+        for (auto& d : ctx->devs)
+            if (d.live()) fpm::check_window(ctx, d, ld, row_base, col_base);
+        const fpm::HostDst out{C, ld, row_base, col_base};
+        pmm_stats local;
+        std::vector<char> done;
+        fpm::compute(ctx, &local, nullptr, &out, &done);
+        double td = 0.0;
+        fpm::download(ctx, C, ld, row_base, col_base, &td, &done);
+        local.t_download_s = std::max(local.t_download_s, td);
+        if (stats) *stats = local;
+    });
+}
+
 extern "C" int pmm_download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_base) {
     return guarded([&] {
         FPM_CHECK_ARG(ctx != nullptr, "null ctx");
@@ -1593,11 +1746,13 @@ extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int6
         for (auto& d : ctx->devs)
             if (d.live()) fpm::check_window(ctx, d, ld, row_base, col_base);
         const fpm::HostSrc host{A, B, ld, row_base, col_base};
+        const fpm::HostDst out{C, ld, row_base, col_base};
         pmm_stats local;
-        fpm::compute(ctx, &local, &host);  // host panels streamed under the updates
+        std::vector<char> done;
+        fpm::compute(ctx, &local, &host, &out, &done);  // host panels streamed in, C streamed out
         double td = 0.0;
-        fpm::download(ctx, C, ld, row_base, col_base, &td);
-        local.t_download_s = td;
+        fpm::download(ctx, C, ld, row_base, col_base, &td, &done);  // devices without a tail
+        local.t_download_s = std::max(local.t_download_s, td);
         if (stats) *stats = local;
     });
 }

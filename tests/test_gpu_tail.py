@@ -1,0 +1,109 @@
+"""Download-overlapped tail (option "e2e_tail"; pmm_run / pmm_compute_into):
+the last update groups run band-major so C_i leaves the device band by band
+under the remaining updates.  Same sums per element, so parity with the oracle
+(bit-exact on integers) for every tail length, with resident and out-of-core
+devices mixed, through pmm_run and pmm_compute_into."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import gemm as og
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+import paper_conf_cluster_zhongrl12_b200 as pkg  # noqa: E402
+
+
+@pytest.fixture(autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    yield
+
+
+@pytest.mark.parametrize("tail", [-1, 0, 1, 3, 16])
+@pytest.mark.parametrize("p", [1, 3])
+def test_run_with_tail_parity(tail, p):
+    N, b = 2304, 96                  # n = 24 pivots, fused groups of 8 (K = 768); rects > 2048 rows: 2+ bands
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n - 100 * (p - 1)] + [100] * (p - 1))
+    A = synth.rect(1, N, 0, 0, N, N)
+    B = synth.rect(2, N, 0, 0, N, N)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0] * p) as ctx:
+        ctx.set_option("e2e_tail", tail)
+        st = ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+        assert st.updates >= 1
+    assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+@pytest.mark.parametrize("fuse", [1, 2])
+def test_tail_integer_exact_mixed_ooc(fuse):
+    N, b = 1536, 128
+    n = N // b
+    rects = pkg.colpart_arrange(n, [80, 40, 24])
+    A = synth.rect(11, N, 0, 0, N, N, synth.DIST_INT)
+    B = synth.rect(12, N, 0, 0, N, N, synth.DIST_INT)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0, 0, 0]) as ctx:
+        ctx.set_option("fuse", fuse)
+        ctx.set_option("e2e_tail", 4)
+        ctx.set_device_option(1, "c_cap_bytes", 1)   # device 1 out of core: no tail, copied after
+        st = ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+        assert st.ooc_devices == 2
+    assert np.array_equal(C.astype(np.float64), og.gemm(A, B))
+
+
+def test_single_group_all_tail():
+    """One update group (n = 4, f = 4): the whole k-loop is the tail and its
+    first (only) group overwrites C."""
+    N, b = 512, 128
+    A = synth.rect(3, N, 0, 0, N, N)
+    B = synth.rect(4, N, 0, 0, N, N)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0]) as ctx:
+        ctx.set_option("e2e_tail", 16)
+        st = ctx.run(A, B, C, N, b, [(0, 0, 0, 4, 4)], pkg.FPM_F32)
+        assert st.updates == 1
+    assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+def test_compute_into_pinned_windows():
+    """pmm_compute_into into a pinned host matrix, twice on the same context,
+    FP32 (tail) and FP64 (copied after the loop)."""
+    N, b = 2048, 128
+    n = N // b
+    rects = pkg.colpart_arrange(n, [160, 96])
+    for dt, tol in ((pkg.FPM_F32, 1e-5), (pkg.FPM_F64, 1e-12)):
+        npdt = np.float32 if dt == pkg.FPM_F32 else np.float64
+        tdt = torch.float32 if dt == pkg.FPM_F32 else torch.float64
+        A = synth.rect(5, N, 0, 0, N, N, synth.DIST_PM1, npdt)
+        B = synth.rect(6, N, 0, 0, N, N, synth.DIST_PM1, npdt)
+        ref = og.gemm(A, B)
+        with pkg.Context.local([0, 0]) as ctx:
+            ctx.setup(N, b, rects, dt)
+            ctx.fill_synthetic(5, 6)
+            for _ in range(2):
+                full = torch.full((N, N), float("nan"), dtype=tdt).pin_memory()
+                st = ctx.compute_into(full, N)
+                assert st.t_compute_s > 0
+                assert og.rel_fro(full.numpy(), ref) <= tol
+
+
+def test_nccl_single_rank_tail():
+    N, b = 1024, 128
+    A = synth.rect(7, N, 0, 0, N, N)
+    B = synth.rect(8, N, 0, 0, N, N)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.nccl(0, 1, 0, pkg.Context.nccl_unique_id()) as ctx:
+        ctx.set_option("e2e_tail", 2)
+        ctx.run(A, B, C, N, b, [(0, 0, 0, N // b, N // b)], pkg.FPM_F32)
+    assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+def test_e2e_tail_option_errors():
+    with pkg.Context.local([0]) as ctx:
+        for bad in (-2, 17):
+            with pytest.raises(pkg.FpmError):
+                ctx.set_option("e2e_tail", bad)
