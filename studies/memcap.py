@@ -1,5 +1,6 @@
 #!/usr/bin/env python
-"""Memory-cliff study (Table III analogue) on ONE B200.
+"""Memory-cliff study (Table III / Fig. 6 / Fig. 7 analogue, SURVEY §8(f)
+NEXT-1 and NEXT-2) on ONE B200.
 
 The paper's hybrid node: two GPUs whose device memory holds C_i only
 up to some problem size (GTX680 "G1", C870 "G2"), beyond which their
@@ -21,6 +22,10 @@ the multiply runs for n x n blocks, n in {40, 50, 60, 70}, under
   cpm   constant models = each device's speed at the even share of the 40 x 40
         problem (constants "obtained in advance, from the speed
         measurements when some workload is distributed evenly") -- reading Q9
+  homogeneous  equal areas ("data distributed evenly")
+
+Fig. 7 is the total time per n and partition (exchange included, P:107);
+Fig. 6 the per-device computation time at 60 x 60 (per_dev_compute_s).
 
 Reported per n and partition (Table III's columns): blocks per device, total
 time, per-device computation time, measured imbalance, whether each GPU ran out
@@ -80,7 +85,7 @@ def pcie_bandwidth(nbytes=1 << 30, reps=5):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--b", type=int, default=512)
-    ap.add_argument("--ns", default="40,50,60,70")
+    ap.add_argument("--ns", default="30,40,45,50,55,60,65,70")
     ap.add_argument("--caps", default="74,36,8,8,8,8")
     ap.add_argument("--names", default="G1,G2,S1,S2,S3,S4")
     ap.add_argument("--c-caps-mib", default="1024,512,0,0,0,0")
@@ -131,7 +136,7 @@ def main():
     for n in ns:
         N, T = n * b, n * n
         row = {"n": n, "N": N}
-        for name, mods in (("fpm", models), ("cpm", cpm_models)):
+        for name, mods in (("fpm", models), ("cpm", cpm_models), ("homogeneous", [([1], [1.0])] * p)):
             d = pkg.fpm_partition(T, mods)
             rects = pkg.colpart_arrange(n, d)
             ctx.setup(N, b, rects, pkg.FPM_F32)
@@ -161,6 +166,7 @@ def main():
                   + " ".join(f"{names[i]}={areas[i]}" for i in range(p))
                   + f"  ooc={row[name]['ooc']}", flush=True)
         row["fpm_vs_cpm_time_delta"] = row["fpm"]["t_total_s"] / row["cpm"]["t_total_s"] - 1.0
+        row["fpm_vs_homogeneous_time_delta"] = row["fpm"]["t_total_s"] / row["homogeneous"]["t_total_s"] - 1.0
         table.append(row)
     ctx.close()
 
@@ -175,7 +181,8 @@ def main():
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)
-    print(json.dumps([{"n": r["n"], "fpm_vs_cpm": r["fpm_vs_cpm_time_delta"]} for r in table]))
+    print(json.dumps([{"n": r["n"], "fpm_vs_cpm": r["fpm_vs_cpm_time_delta"],
+                       "fpm_vs_homogeneous": r["fpm_vs_homogeneous_time_delta"]} for r in table]))
 
 
 if __name__ == "__main__":
