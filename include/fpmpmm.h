@@ -279,6 +279,14 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 updates; with "ooc_keep" the per-update traffic stays C_i
  *                 minus the cap in each direction.  Fewer buffers (not below
  *                 2) are used when R bands of 256 rows exceed the cap.
+ *   "graph":      1 (default): pmm_compute captures the whole k-loop (every
+ *                 device's exchange, staging and update streams, forked from and
+ *                 joined into device 0's compute stream) into one CUDA graph on
+ *                 first use and replays it; timing events become event-record
+ *                 nodes so per-group statistics are kept.  Re-captured after
+ *                 pmm_setup, pmm_ipc_import or any option change.  NCCL
+ *                 contexts, pmm_run and pmm_compute_into issue eagerly.
+ *                 0: always eager.
  *   "e2e_tail":   update groups run band-major at the end of pmm_run /
  *                 pmm_compute_into so the copy of C_i to the host overlaps them
  *                 (FP32, resident C_i): -1 auto (default: enough groups to

@@ -81,6 +81,8 @@ struct Device {
     std::vector<void*> host_allocs;
     BandPipe bp;
     Ring ring{0, 0};       // out-of-core band geometry of the current problem
+    int64_t g_ooc_bytes = 0;        // out-of-core bytes of one captured k-loop
+    cudaEvent_t ev_join[4] = {};    // graph capture: join of this device's streams
     cudaStream_t s_comp = nullptr, s_comm = nullptr;
     cudaStream_t s_up = nullptr;  // pmm_run: host -> device panel uploads, run ahead of the staging
     cudaEvent_t ev_ready[kSlots] = {}, ev_free[kSlots] = {};
@@ -136,6 +138,10 @@ struct pmm_ctx {
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
+    int graph = 1;            // pmm_compute replays the k-loop as one CUDA graph
+    cudaGraphExec_t gexec = nullptr;
+    cudaEvent_t ev_fork = nullptr;  // on devs[0]'s device
+    int64_t g_bytes = 0, g_launches = 0;
     int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
@@ -358,6 +364,7 @@ void init_device(Device& d) {
     CU(cudaEventCreate(&d.ev_stop));
     CU(cudaEventCreate(&d.ev_io0));
     CU(cudaEventCreate(&d.ev_io1));
+    for (auto& e : d.ev_join) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     bp_init(d.bp);
 }
 
@@ -371,6 +378,10 @@ void destroy_device(Device& d) {
     }
     for (cudaEvent_t e : {d.ev_start, d.ev_stop, d.ev_io0, d.ev_io1})
         if (e) cudaEventDestroy(e);
+    for (auto& e : d.ev_join) {
+        if (e) cudaEventDestroy(e);
+        e = nullptr;
+    }
     if (d.s_comp) cudaStreamDestroy(d.s_comp);
     if (d.s_comm) cudaStreamDestroy(d.s_comm);
     if (d.s_up) cudaStreamDestroy(d.s_up);
@@ -380,6 +391,14 @@ void destroy_device(Device& d) {
     green_destroy(d.green);
 }
 
+
+// Timing events: while the k-loop is being captured into a CUDA graph they must
+// become event-record nodes (cudaEventRecordExternal), not capture-internal
+// dependencies, so that replays still time each group.
+bool g_capturing = false;
+void rec_t(cudaEvent_t e, cudaStream_t s) {
+    CU(cudaEventRecordWithFlags(e, s, g_capturing ? cudaEventRecordExternal : cudaEventRecordDefault));
+}
 
 float elapsed_ms(cudaEvent_t a, cudaEvent_t b) {
     float ms = 0.0f;
@@ -405,9 +424,16 @@ void close_peers(pmm_ctx* ctx) {
     ctx->peers_ready = false;
 }
 
+// The captured k-loop refers to the problem's buffers, events and options.
+void drop_graph(pmm_ctx* ctx) {
+    if (ctx->gexec) cudaGraphExecDestroy(ctx->gexec);
+    ctx->gexec = nullptr;
+}
+
 // Option "sm_partition": rebuild every device's streams, inside disjoint
 // green-context SM partitions of its cap (on) or on the whole GPU (off).
 void set_sm_partition(pmm_ctx* ctx, bool green) {
+    drop_graph(ctx);
     // carve the partitions first: a failure leaves the context as it was
     std::vector<GreenPartition> parts(ctx->devs.size());
     if (green) {
@@ -490,6 +516,7 @@ void alloc_slot(pmm_ctx* ctx, Device& d, int s) {
 }
 
 void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects, fpm_dtype dt) {
+    drop_graph(ctx);
     FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype %d", (int)dt);
     FPM_CHECK_ARG(N >= 1 && b >= 1 && N % b == 0, "b must divide N (N=%lld, b=%lld)", (long long)N,
                   (long long)b);
@@ -736,7 +763,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     }
 
     // ---- staging: K-major operands of the fused update (K = f b)
-    CU(cudaEventRecord(d.ev_pack0[g], d.s_comm));
+    rec_t(d.ev_pack0[g], d.s_comm);
     if (ctx->dt == FPM_F32) {
         const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
         const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
@@ -760,7 +787,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
                              d.s_comm);
         d.launches += 1;
     }
-    CU(cudaEventRecord(d.ev_pack1[g], d.s_comm));
+    rec_t(d.ev_pack1[g], d.s_comm);
     CU(cudaEventRecord(d.ev_ready[slot], d.s_comm));
     return bytes;
 }
@@ -808,7 +835,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
     const int f = ctx->groups[g].second;
     CU(cudaSetDevice(d.cuda_dev));
     CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
-    CU(cudaEventRecord(d.ev_upd0[g], d.s_comp));
+    rec_t(d.ev_upd0[g], d.s_comp);
     // out-of-core band order: reversed every other update, the last two
     // bands kept on the device between updates (option "ooc_keep")
     BandCall bc;
@@ -845,7 +872,7 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
                           static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k0 != 0, d.num_sms, d.s_comp);
         d.launches += 1;
     }
-    CU(cudaEventRecord(d.ev_upd1[g], d.s_comp));
+    rec_t(d.ev_upd1[g], d.s_comp);
     CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
 }
 
@@ -919,15 +946,18 @@ void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
 // iteration ahead of their use (pmm_run).  With `out` set, C_i is also copied
 // to host memory, overlapped with the last updates where possible (tail);
 // returns true for each device whose copy was done here (tail_done).
+void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, int64_t* bytes_out);
+void capture_kloop(pmm_ctx* ctx);
+void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<char>* tail_done, int64_t bytes,
+                  int64_t launches);
+
 void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const HostDst* out = nullptr,
              std::vector<char>* tail_done = nullptr) {
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
     if (ctx->ipc_mode && !ctx->peers_ready)
         fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
     FPM_CHECK_ARG(!(ctx->ipc_mode && host), "IPC mode has no streamed host input (peers cannot be ordered)");
-    const int ngroups = (int)ctx->groups.size();
     const int L = out ? tail_groups(ctx) : 0;
-    const int gt = ngroups - L;  // first tail group
     if (tail_done) tail_done->assign(ctx->devs.size(), 0);
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
@@ -947,11 +977,37 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
         CU(cudaStreamSynchronize(d.s_comp));
         CU(cudaStreamSynchronize(d.s_comm));
     }
+    // pmm_compute on resident inputs: the whole k-loop is one CUDA graph,
+    // captured on first use and replayed (option "graph")
+    const bool use_graph = ctx->graph && !host && !out && !ctx->nccl_mode;
+    int64_t bytes = 0, launches = 0;
+    if (use_graph) {
+        if (!ctx->gexec) capture_kloop(ctx);
+        Device& d0 = ctx->devs[0];
+        CU(cudaSetDevice(d0.cuda_dev));
+        CU(cudaGraphLaunch(ctx->gexec, d0.s_comp));
+        bytes = ctx->g_bytes;
+        launches = ctx->g_launches;
+        for (auto& d : ctx->devs) d.bp.bytes = d.g_ooc_bytes;
+    } else {
+        issue_kloop(ctx, host, out, L, &bytes);
+        launches = -launches0;
+        for (auto& d : ctx->devs) launches += d.launches;
+    }
+    finish_kloop(ctx, st, host != nullptr, tail_done, bytes, launches);
+}
+
+// Everything from ev_start to ev_stop of one k-loop, on the devices' streams.
+void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, int64_t* bytes_out) {
+    const int ngroups = (int)ctx->groups.size();
+    const int gt = ngroups - L;  // first tail group
     for (auto& d : ctx->devs) {
         CU(cudaSetDevice(d.cuda_dev));
-        CU(cudaEventRecord(d.ev_start, d.s_comp));
-        CU(cudaStreamWaitEvent(d.s_comm, d.ev_start, 0));
-        CU(cudaStreamWaitEvent(d.s_up, d.ev_start, 0));
+        rec_t(d.ev_start, d.s_comp);
+        if (!g_capturing) {  // (a capture forks every stream from its origin instead)
+            CU(cudaStreamWaitEvent(d.s_comm, d.ev_start, 0));
+            CU(cudaStreamWaitEvent(d.s_up, d.ev_start, 0));
+        }
     }
     const bool streamed = host != nullptr;
     int64_t bytes = 0;
@@ -989,13 +1045,86 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     if (L > 0)
         for (auto& d : ctx->devs)
             if (d.live() && !d.ooc) issue_tail(ctx, d, gt, L, *out);
-    int64_t launches = -launches0;
-    for (auto& d : ctx->devs) launches += d.launches;
     for (auto& d : ctx->devs) {
         CU(cudaSetDevice(d.cuda_dev));
         if (d.ooc) bp_join(d.bp, d.s_comp);  // C_i is complete once its last band is back in host memory
-        CU(cudaEventRecord(d.ev_stop, d.s_comp));
+        rec_t(d.ev_stop, d.s_comp);
     }
+    *bytes_out = bytes;
+}
+
+// Capture one k-loop into ctx->gexec: every stream of every device is forked
+// from device 0's compute stream and joined back into it.
+void capture_kloop(pmm_ctx* ctx) {
+    Device& d0 = ctx->devs[0];
+    for (auto& d : ctx->devs) {  // the graph starts from a clean band pipeline
+        d.bp.used[0] = false;
+        for (int i = 0; i < kMaxBandBufs; ++i) d.bp.used[i] = false;
+        std::fill(d.bp.band_used.begin(), d.bp.band_used.end(), 0);
+        d.bp.last = d.bp.last_step = -1;
+        d.bp.next = 0;
+        d.bp.dir = 1;
+        d.bp.bytes = 0;
+    }
+    int64_t launches0 = 0;
+    for (auto& d : ctx->devs) launches0 += d.launches;
+    CU(cudaSetDevice(d0.cuda_dev));
+    if (!ctx->ev_fork) CU(cudaEventCreateWithFlags(&ctx->ev_fork, cudaEventDisableTiming));
+    const cudaStream_t origin = d0.s_comp;
+    CU(cudaStreamBeginCapture(origin, cudaStreamCaptureModeRelaxed));
+    int64_t bytes = 0;
+    try {
+        CU(cudaEventRecord(ctx->ev_fork, origin));
+        for (auto& d : ctx->devs) {
+            CU(cudaSetDevice(d.cuda_dev));
+            for (cudaStream_t s : {d.s_comp, d.s_comm, d.bp.s_h2d, d.bp.s_d2h})
+                if (s != origin) CU(cudaStreamWaitEvent(s, ctx->ev_fork, 0));
+        }
+        g_capturing = true;
+        issue_kloop(ctx, nullptr, nullptr, 0, &bytes);
+        g_capturing = false;
+        for (auto& d : ctx->devs) {
+            CU(cudaSetDevice(d.cuda_dev));
+            int j = 0;
+            for (cudaStream_t s : {d.s_comp, d.s_comm, d.bp.s_h2d, d.bp.s_d2h}) {
+                if (s == origin) continue;
+                CU(cudaEventRecord(d.ev_join[j], s));
+                CU(cudaSetDevice(d0.cuda_dev));
+                CU(cudaStreamWaitEvent(origin, d.ev_join[j], 0));
+                CU(cudaSetDevice(d.cuda_dev));
+                ++j;
+            }
+        }
+    } catch (...) {
+        g_capturing = false;
+        cudaGraph_t junk = nullptr;
+        cudaSetDevice(d0.cuda_dev);
+        cudaStreamEndCapture(origin, &junk);
+        if (junk) cudaGraphDestroy(junk);
+        cudaGetLastError();
+        throw;
+    }
+    CU(cudaSetDevice(d0.cuda_dev));
+    cudaGraph_t graph = nullptr;
+    CU(cudaStreamEndCapture(origin, &graph));
+    cudaError_t e = cudaGraphInstantiate(&ctx->gexec, graph, 0);
+    cudaGraphDestroy(graph);
+    if (e != cudaSuccess) {
+        ctx->gexec = nullptr;
+        fail(FPM_ECUDA, "cudaGraphInstantiate: %s", cudaGetErrorString(e));
+    }
+    ctx->g_bytes = bytes;
+    ctx->g_launches = -launches0;
+    for (auto& d : ctx->devs) {
+        ctx->g_launches += d.launches;
+        d.g_ooc_bytes = d.bp.bytes;
+    }
+}
+
+// Wait for the k-loop and fill the statistics.
+void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<char>* tail_done, int64_t bytes,
+                  int64_t launches) {
+    const int ngroups = (int)ctx->groups.size();
     double t_max = 0.0, t_tail_copy = 0.0;
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
@@ -1548,6 +1677,7 @@ extern "C" int pmm_ipc_import(pmm_ctx* ctx, const uint8_t* blobs, int32_t world)
         FPM_CHECK_ARG(world == ctx->world, "expected %d blobs", ctx->world);
         if (!ctx->have_problem) fpm::fail(FPM_ESTATE, "pmm_ipc_import before pmm_setup");
         fpm::close_peers(ctx);
+        fpm::drop_graph(ctx);
         CU(cudaSetDevice(ctx->devs[0].cuda_dev));
         for (int q = 0; q < world; ++q) {
             IpcBlob blob;
@@ -1568,6 +1698,8 @@ extern "C" int pmm_destroy(pmm_ctx* ctx) {
     return guarded([&] {
         if (!ctx) return;
         fpm::close_peers(ctx);
+        fpm::drop_graph(ctx);
+        if (ctx->ev_fork) cudaEventDestroy(ctx->ev_fork);
         for (auto& d : ctx->devs) fpm::destroy_device(d);
         if (ctx->nccl_mode) {
             if (ctx->col_comm) fpm::nccl().CommDestroy(ctx->col_comm);
@@ -1580,8 +1712,12 @@ extern "C" int pmm_destroy(pmm_ctx* ctx) {
 extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
     return guarded([&] {
         FPM_CHECK_ARG(ctx && key, "null argument");
+        fpm::drop_graph(ctx);  // every option can change the captured k-loop
         const std::string k(key);
-        if (k == "f32_scheme") {
+        if (k == "graph") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "graph must be 0 or 1");
+            ctx->graph = (int)value;
+        } else if (k == "f32_scheme") {
             FPM_CHECK_ARG(value == 0 || value == 1, "f32_scheme must be 0 or 1");
             if (ctx->f32_scheme != (int)value) ctx->have_problem = false;  // operand buffers change size
             ctx->f32_scheme = (int)value;
@@ -1630,6 +1766,7 @@ extern "C" int pmm_set_device_option(pmm_ctx* ctx, int32_t dev, const char* key,
         FPM_CHECK_ARG(ctx && key, "null argument");
         fpm::Device* d = fpm::local_dev(ctx, dev);
         FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
+        fpm::drop_graph(ctx);
         const std::string k(key);
         if (k == "c_cap_bytes") {
             FPM_CHECK_ARG(value >= 0, "c_cap_bytes must be >= 0");
