@@ -200,13 +200,19 @@ __global__ void __launch_bounds__(256) fill_k(T* dst, int64_t ld, uint64_t seed,
 }
 
 // ---- FP64 rank-b update on the FP64 tensor path (mma.sync m8n8k4 f64 ->
-// SASS DMMA.8x8x4).  128 x 128 CTA tile, 8 warps of 64 x 32 (8 x 4 DMMA tiles,
-// 64 accumulators per lane), K staged through shared memory in chunks of 32
-// with cp.async double buffering.  Smem rows are padded to 36 doubles so the
-// fragment loads (lane -> row lane/4, column lane%4) hit 16 distinct 8-byte
-// bank pairs per half-warp.
-constexpr int F64_BM = 128, F64_BN = 128, F64_BK = 32, F64_LD = 36;
-constexpr int F64_SMEM = 2 * (F64_BM + F64_BN) * F64_LD * 8;  // 147456 B
+// SASS DMMA.8x8x4).  One persistent CTA per SM holds two independent groups of
+// 8 warps; each group walks its own sequence of 64 x 128 C tiles (warp tiles
+// 32 x 32: 4 x 4 DMMA tiles, 32 accumulators per lane) with its own 3-stage
+// cp.async ring (K chunks of 16) and its own named barrier, so one group's
+// epilogue (the C read-modify-write) overlaps the other's main loop -- what two
+// co-resident CTAs would do, without letting the hardware spread them over
+// more SMs than the device's cap.  Smem rows are padded to 20 doubles so the
+// fragment loads (lane -> row lane/4, column lane%4) are conflict-free per
+// half-warp.  Measured (ncu, L = 8192, K = 512): the previous 128 x 128
+// single-group design kept the DMMA pipe 73 % busy.
+constexpr int F64_BM = 64, F64_BN = 128, F64_BK = 16, F64_LD = 20, F64_ST = 3, F64_GROUPS = 2;
+constexpr int F64_GROUP_DOUBLES = F64_ST * (F64_BM + F64_BN) * F64_LD;
+constexpr int F64_SMEM = F64_GROUPS * F64_GROUP_DOUBLES * 8;  // 184320 B
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool valid) {
     const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
@@ -214,94 +220,117 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool va
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
 }
 
-__global__ void __launch_bounds__(256, 1) update_f64_k(const double* __restrict__ A, int64_t lda,
+__device__ __forceinline__ void group_bar(int id) { asm volatile("bar.sync %0, 256;" ::"r"(id) : "memory"); }
+
+__global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict__ A, int64_t lda,
                                                        const double* __restrict__ Bt, double* __restrict__ C,
                                                        int64_t M, int64_t Nc, int64_t K, int64_t ldc,
                                                        int accumulate) {
     extern __shared__ double sm64[];
-    double* As = sm64;                                  // [2][BM][LD]
-    double* Bs = sm64 + 2 * F64_BM * F64_LD;            // [2][BN][LD]
-    const int warp = threadIdx.x / 32, lane = threadIdx.x % 32;
-    const int wm = (warp / 4) * 64, wn = (warp % 4) * 32;
-    // persistent over tiles: the grid is capped at the device's SM cap
+    const int grp = threadIdx.x / 256, gtid = threadIdx.x % 256;
+    double* As = sm64 + grp * F64_GROUP_DOUBLES;       // [ST][BM][LD]
+    double* Bs = As + F64_ST * F64_BM * F64_LD;        // [ST][BN][LD]
+    const int warp = gtid / 32, lane = threadIdx.x % 32;
+    const int wm = (warp / 4) * 32, wn = (warp % 4) * 32;
     const int64_t tiles_n = (Nc + F64_BN - 1) / F64_BN;
     const int64_t tiles = ((M + F64_BM - 1) / F64_BM) * tiles_n;
-    for (int64_t t = blockIdx.x; t < tiles; t += gridDim.x) {
-    const int64_t m0 = (t / tiles_n) * F64_BM, n0 = (t % tiles_n) * F64_BN;
-    double acc[8][4][2];
-#pragma unroll
-    for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
-
-    // 128 rows x 32 doubles = 2048 16-B chunks per operand per stage; 8 per thread
-    auto load_stage = [&](int stage, int64_t k0) {
-#pragma unroll
-        for (int it = 0; it < 8; ++it) {
-            const int idx = threadIdx.x + it * 256;
-            const int r = idx / 16, c2 = (idx % 16) * 2;
-            const int64_t gk = k0 + c2;
-            const int64_t gm = m0 + r, gn = n0 + r;
-            const bool ka = gk < K;  // K % 8 == 0, so a 2-element chunk is all in or all out
-            cp_async16(As + (stage * F64_BM + r) * F64_LD + c2, A + (ka && gm < M ? gm * lda + gk : 0),
-                       ka && gm < M);
-            cp_async16(Bs + (stage * F64_BN + r) * F64_LD + c2, Bt + (ka && gn < Nc ? gn * K + gk : 0),
-                       ka && gn < Nc);
-        }
-        asm volatile("cp.async.commit_group;" ::: "memory");
-    };
-
     const int64_t nk = (K + F64_BK - 1) / F64_BK;
-    load_stage(0, 0);
-    for (int64_t kb = 0; kb < nk; ++kb) {
-        const int st = (int)(kb & 1);
-        if (kb + 1 < nk) {
-            load_stage(st ^ 1, (kb + 1) * F64_BK);
-            asm volatile("cp.async.wait_group 1;" ::: "memory");
-        } else {
-            asm volatile("cp.async.wait_group 0;" ::: "memory");
-        }
-        __syncthreads();
-        const double* as = As + st * F64_BM * F64_LD;
-        const double* bs = Bs + st * F64_BN * F64_LD;
+    // persistent over tiles (the grid is capped at the device's SM cap); the
+    // two groups of a CTA take alternate tiles
+    const int64_t first = 2 * (int64_t)blockIdx.x + grp, stride = 2 * (int64_t)gridDim.x;
+
+    // load cursor: (tile lt, chunk lkb) runs ST-1 chunks ahead of the compute
+    int64_t lt = first, lkb = 0;
+    int slot_l = 0;
+    auto advance_load = [&]() {
+        if (lt < tiles) {
+            const int64_t m0 = (lt / tiles_n) * F64_BM, n0 = (lt % tiles_n) * F64_BN, k0 = lkb * F64_BK;
+            // A: 64 rows x 16 doubles = 512 16-B chunks (2 per thread); B: 128 rows (4 per thread)
 #pragma unroll
-        for (int kk = 0; kk < F64_BK; kk += 4) {
-            double a[8], b[4];
-#pragma unroll
-            for (int i = 0; i < 8; ++i) a[i] = as[(wm + i * 8 + lane / 4) * F64_LD + kk + lane % 4];
-#pragma unroll
-            for (int j = 0; j < 4; ++j) b[j] = bs[(wn + j * 8 + lane / 4) * F64_LD + kk + lane % 4];
-#pragma unroll
-            for (int i = 0; i < 8; ++i)
-#pragma unroll
-                for (int j = 0; j < 4; ++j)
-                    asm volatile(
-                        "mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
-                        : "+d"(acc[i][j][0]), "+d"(acc[i][j][1])
-                        : "d"(a[i]), "d"(b[j]));
-        }
-        __syncthreads();
-    }
-#pragma unroll
-    for (int i = 0; i < 8; ++i)
-#pragma unroll
-        for (int j = 0; j < 4; ++j) {
-            const int64_t gm = m0 + wm + i * 8 + lane / 4;
-            const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4);
-            if (gm >= M) continue;
-            double* cp = C + gm * ldc + gn;
-            if (gn + 1 < Nc && (reinterpret_cast<uintptr_t>(cp) & 15) == 0) {
-                double2 c = accumulate ? *reinterpret_cast<double2*>(cp) : make_double2(0.0, 0.0);
-                c.x += acc[i][j][0];
-                c.y += acc[i][j][1];
-                *reinterpret_cast<double2*>(cp) = c;
-            } else {
-#pragma unroll
-                for (int h = 0; h < 2; ++h)
-                    if (gn + h < Nc) cp[h] = (accumulate ? cp[h] : 0.0) + acc[i][j][h];
+            for (int it = 0; it < 6; ++it) {
+                const int idx = gtid + it * 256;
+                const bool isA = it < 2;
+                const int j = isA ? idx : idx - 512;
+                const int r = j / 8, c2 = (j % 8) * 2;
+                const int64_t gk = k0 + c2;
+                const bool ka = gk < K;  // K even: a 2-element chunk is all in or all out
+                if (isA) {
+                    const int64_t gm = m0 + r;
+                    cp_async16(As + (slot_l * F64_BM + r) * F64_LD + c2, A + (ka && gm < M ? gm * lda + gk : 0),
+                               ka && gm < M);
+                } else {
+                    const int64_t gn = n0 + r;
+                    cp_async16(Bs + (slot_l * F64_BN + r) * F64_LD + c2, Bt + (ka && gn < Nc ? gn * K + gk : 0),
+                               ka && gn < Nc);
+                }
+            }
+            if (++lkb == nk) {
+                lkb = 0;
+                lt += stride;
             }
         }
+        asm volatile("cp.async.commit_group;" ::: "memory");  // (empty past the last tile)
+        slot_l = slot_l + 1 == F64_ST ? 0 : slot_l + 1;
+    };
+#pragma unroll
+    for (int s = 0; s < F64_ST - 1; ++s) advance_load();
+
+    int slot_c = 0;
+    for (int64_t t = first; t < tiles; t += stride) {
+        const int64_t m0 = (t / tiles_n) * F64_BM, n0 = (t % tiles_n) * F64_BN;
+        double acc[4][4][2];
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+
+        for (int64_t kb = 0; kb < nk; ++kb) {
+            asm volatile("cp.async.wait_group %0;" ::"n"(F64_ST - 2) : "memory");
+            group_bar(1 + grp);  // chunk visible to the group; the slot refilled next is free
+            advance_load();
+            const double* as = As + slot_c * F64_BM * F64_LD;
+            const double* bs = Bs + slot_c * F64_BN * F64_LD;
+#pragma unroll
+            for (int kk = 0; kk < F64_BK; kk += 4) {
+                double a[4], b[4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i) a[i] = as[(wm + i * 8 + lane / 4) * F64_LD + kk + lane % 4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) b[j] = bs[(wn + j * 8 + lane / 4) * F64_LD + kk + lane % 4];
+#pragma unroll
+                for (int i = 0; i < 4; ++i)
+#pragma unroll
+                    for (int j = 0; j < 4; ++j)
+                        asm volatile(
+                            "mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
+                            : "+d"(acc[i][j][0]), "+d"(acc[i][j][1])
+                            : "d"(a[i]), "d"(b[j]));
+            }
+            slot_c = slot_c + 1 == F64_ST ? 0 : slot_c + 1;
+        }
+        // epilogue: this group's next chunks are already in flight, the other
+        // group keeps the DMMA pipe busy
+#pragma unroll
+        for (int i = 0; i < 4; ++i)
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+                const int64_t gm = m0 + wm + i * 8 + lane / 4;
+                const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4);
+                if (gm >= M) continue;
+                double* cp = C + gm * ldc + gn;
+                if (gn + 1 < Nc && (reinterpret_cast<uintptr_t>(cp) & 15) == 0) {
+                    double2 c = accumulate ? *reinterpret_cast<double2*>(cp) : make_double2(0.0, 0.0);
+                    c.x += acc[i][j][0];
+                    c.y += acc[i][j][1];
+                    *reinterpret_cast<double2*>(cp) = c;
+                } else {
+#pragma unroll
+                    for (int h = 0; h < 2; ++h)
+                        if (gn + h < Nc) cp[h] = (accumulate ? cp[h] : 0.0) + acc[i][j][h];
+                }
+            }
     }  // tile loop
+    asm volatile("cp.async.wait_group 0;" ::: "memory");
 }
 
 int grid_for(int64_t work, int threads) {
@@ -390,8 +419,8 @@ void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C
     const int64_t tiles = ((Nc + F64_BN - 1) / F64_BN) * ((M + F64_BM - 1) / F64_BM);
     int sms = num_sms;
     if (sms <= 0) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
-    const unsigned grid = (unsigned)std::min<int64_t>(tiles, std::max(1, sms));  // 1 CTA per SM (147 KB smem)
-    update_f64_k<<<grid, 256, F64_SMEM, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
+    const unsigned grid = (unsigned)std::min<int64_t>((tiles + 1) / 2, std::max(1, sms));  // 1 CTA (2 tile groups) per SM
+    update_f64_k<<<grid, 512, F64_SMEM, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
     check_launch("update_f64");
 }
 
