@@ -285,7 +285,9 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 first use and replays it; timing events become event-record
  *                 nodes so per-group statistics are kept.  Re-captured after
  *                 pmm_setup, pmm_ipc_import or any option change.  NCCL
- *                 contexts, pmm_run and pmm_compute_into issue eagerly.
+ *                 contexts, green partitions ("sm_partition" = 1: replays
+ *                 were measured to lose the per-device SM confinement), pmm_run
+ *                 and pmm_compute_into issue eagerly.
  *                 0: always eager.
  *   "e2e_tail":   update groups run band-major at the end of pmm_run /
  *                 pmm_compute_into so the copy of C_i to the host overlaps them

@@ -979,7 +979,9 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     }
     // pmm_compute on resident inputs: the whole k-loop is one CUDA graph,
     // captured on first use and replayed (option "graph")
-    const bool use_graph = ctx->graph && !host && !out && !ctx->nccl_mode;
+    // (not with green partitions: measured, replays lose the per-device SM
+    // confinement -- c4 analogue 0.37 s replayed vs 0.23 s issued eagerly)
+    const bool use_graph = ctx->graph && !host && !out && !ctx->nccl_mode && !ctx->sm_partition;
     int64_t bytes = 0, launches = 0;
     if (use_graph) {
         if (!ctx->gexec) capture_kloop(ctx);

@@ -48,6 +48,9 @@ def main():
     ap.add_argument("--sizes", default="1,2,3,4,6,8,12,16,20,24,28,32,40")
     ap.add_argument("--concurrent", dest="exclusive", action="store_false",
                     help="sample all devices at once (P:10 (ii)) instead of each alone (P:11, default)")
+    ap.add_argument("--insitu", type=int, default=2,
+                    help="extra FPM partitions with models rescaled by the speeds achieved in the previous run")
+    ap.add_argument("--graph", type=int, default=1, help="pmm_compute as a replayed CUDA graph (option graph)")
     ap.add_argument("--sm-partition", type=int, default=0,
                     help="1 = each device in its own green-context SM partition (all its kernels confined)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
@@ -60,6 +63,7 @@ def main():
 
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
     ctx.set_option("sm_partition", args.sm_partition)
+    ctx.set_option("graph", args.graph)
     t0 = time.perf_counter()
     models, sample_info = [], []
     if args.exclusive:   # each device alone (how the paper measured its GPUs)
@@ -81,7 +85,30 @@ def main():
         "homogeneous": pkg.fpm_partition(T, [([1], [1.0])] * p),
     }
     results = {}
-    for name, d in parts.items():
+
+    def corrected(mods, res):
+        """Each device's model scaled by (speed it achieved in the run at its
+        area) / (model speed there): the models keep their shape (P:8), their
+        levels absorb the contention of the concurrent run.  The partition is
+        invariant to a common factor, so only the relative corrections act."""
+        out = []
+        for m, a, t in zip(mods, res["areas"], res["per_dev_compute_s"]):
+            if a <= 0 or t <= 0:
+                out.append(m)
+                continue
+            r = (2.0 * a * b * b * N / t) / pkg.fpm_model_speed(m, a)
+            out.append((m[0], [s * r for s in m[1]]))
+        return out
+
+    order = list(parts.items())
+    for it in range(args.insitu):
+        order.append((f"fpm_insitu{it + 1}", None))
+    cur_models = models
+    for name, d in order:
+        if d is None:   # in-situ corrected FPMs from the previous FPM run
+            prev = results["fpm" if name == "fpm_insitu1" else f"fpm_insitu{int(name[-1]) - 1}"]
+            cur_models = corrected(cur_models, prev)
+            d = pkg.fpm_partition(T, cur_models)
         rects = pkg.colpart_arrange(n, d)
         ctx.setup(N, b, rects, pkg.FPM_F32)
         ctx.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
@@ -95,7 +122,7 @@ def main():
         per_dev = list(best.per_dev_compute_s[:p])
         # FPM-predicted k-loop time: 2 a b^2 N flop at the model's speed s(a)
         pred = [2.0 * a * b * b * N / pkg.fpm_model_speed(m, a) if a > 0 else 0.0
-                for a, m in zip(areas, models)]
+                for a, m in zip(areas, cur_models if name.startswith("fpm_insitu") else models)]
         results[name] = {
             "d": d, "areas": areas, "rects": rects,
             "t_total_s": best.t_compute_s, "gflops": best.gflops,
