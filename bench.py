@@ -351,9 +351,44 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             "gpu_launches": launches,
             "clocks": clk,
         }
-        print(json.dumps(line), flush=True)
     barrier()  # no rank frees buffers a peer may still read (IPC)
     ctx.close()
+    if rank == 0:
+        if world == 1 and not args.no_hetero:
+            try:
+                line["hetero"] = run_hetero(peak)
+            except Exception as ex:  # report, do not hide
+                log("hetero failed:", repr(ex))
+                line["hetero"] = {"error": repr(ex)[:200]}
+        print(json.dumps(line), flush=True)
+
+
+def run_hetero(peak_tflops: float) -> dict:
+    """The metric's 'FPM load imbalance %' under emulated heterogeneity (SURVEY
+    §8(d) c4 analogue, studies/hetero.py): 8 devices on this GPU in disjoint
+    green-context SM partitions, FPMs sampled per device, the multiply under
+    FPM / CPM / homogeneous / in-situ corrected FPM partitions."""
+    import torch
+
+    from studies import hetero
+    caps = [30, 26, 24, 20, 16, 14, 10, 6]   # config 4's {144 .. 32} scaled to fit 148 SMs
+    t0 = time.perf_counter()
+    res = hetero.c4_study(caps, N=32768, b=512, reps=2, insitu=1, graph=0, sm_partition=1, log=log)
+    sms = torch.cuda.get_device_properties(0).multi_processor_count
+    capped_peak = peak_tflops * sum(caps) / sms
+    out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "
+                        f"SM partitions {caps}; FPMs sampled per device alone (P:11), "
+                        f"{len(res['config']['sizes'])} sizes"),
+           "capped_aggregate_peak_tflops": capped_peak, "fpm_sample_s": res["fpm_sample_s"]}
+    for name, r in res["partitions"].items():
+        out[name] = {"t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],
+                     "imbalance_pct_measured": 100.0 * r["imbalance_measured"],
+                     "imbalance_pct_predicted": 100.0 * r["imbalance_predicted"],
+                     "pct_of_capped_peak": 100.0 * r["gflops"] / 1e3 / capped_peak}
+    out["fpm_vs_cpm_time_delta_pct"] = 100.0 * res["fpm_vs_cpm_ncal_time_delta"]
+    out["fpm_vs_homogeneous_time_delta_pct"] = 100.0 * res["fpm_vs_homogeneous_time_delta"]
+    out["wall_s"] = time.perf_counter() - t0
+    return out
 
 
 def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc):
@@ -422,6 +457,8 @@ def main():
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--no-hetero", action="store_true",
+                    help="skip the emulated-heterogeneity measurement (c4 analogue) added at N = 1")
     ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")
     ap.add_argument("--same-gpu", action="store_true",
                     help="testing only: put every rank on cuda:0 (IPC transport works within one GPU)")

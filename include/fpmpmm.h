@@ -293,6 +293,8 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 pmm_compute_into so the copy of C_i to the host overlaps them
  *                 (FP32, resident C_i): -1 auto (default: enough groups to
  *                 cover the copy at ~55 GB/s), 0 off, 1..16.
+ *   "tail_band":  rows of C_i per band of that tail, a positive multiple of
+ *                 256 (default 2048); the last band's copy stays exposed.
  *   "sm_partition": how an SM cap is enforced.  0 (default): the cap is the
  *                 grid of the persistent update kernel (one CTA per SM); other
  *                 kernels of the device are not confined, and devices sharing a

@@ -143,9 +143,11 @@ struct pmm_ctx {
     cudaEvent_t ev_fork = nullptr;  // on devs[0]'s device
     int64_t g_bytes = 0, g_launches = 0;
     int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
+    int64_t tail_band = 2048; // rows of C_i per band of the tail (multiple of 256)
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
+    std::vector<std::pair<int64_t, int>> groups_streamed;  // the same for pmm_run (host-streamed inputs)
 };
 
 namespace fpm {
@@ -552,14 +554,21 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
             cuts.push_back(rects[q].col0);
             cuts.push_back(rects[q].row0);
         }
-    ctx->groups.clear();
-    for (int64_t k = 0; k < n;) {
-        int64_t size = std::min<int64_t>(f, n - k);
-        for (int64_t c : cuts)
-            if (c > k && c < k + size) size = c - k;
-        ctx->groups.push_back({k, (int)size});
-        k += size;
-    }
+    // Streamed runs (pmm_run) start with two single pivots: the first update
+    // waits for only one pivot's panels to cross the host link, and the second
+    // group's panels arrive under the first update.
+    auto build = [&](std::vector<std::pair<int64_t, int>>& out, int64_t singles) {
+        out.clear();
+        for (int64_t k = 0; k < n;) {
+            int64_t size = std::min<int64_t>(k < singles ? 1 : f, n - k);
+            for (int64_t c : cuts)
+                if (c > k && c < k + size) size = c - k;
+            out.push_back({k, (int)size});
+            k += size;
+        }
+    };
+    build(ctx->groups, 0);
+    build(ctx->groups_streamed, 2);
     ctx->fuse_max = f;
 
     const size_t es = esize(dt);
@@ -915,7 +924,7 @@ void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
     CU(cudaSetDevice(d.cuda_dev));
     for (int t = 0; t < L; ++t) CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[2 + t], 0));
     CU(cudaEventRecord(d.ev_upd0[g0], d.s_comp));
-    const int64_t band = std::min<int64_t>(d.H, 2048);  // whole CTA-pair tile rows
+    const int64_t band = std::min<int64_t>(d.H, ctx->tail_band);  // whole CTA-pair tile rows
     const int64_t b = ctx->b;
     const int64_t R0 = d.rect.row0 * b - out.row_base, C0 = d.rect.col0 * b - out.col_base;
     float* C = static_cast<float*>(d.C);
@@ -927,6 +936,7 @@ void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
             d.launches += 1;
         }
         CU(cudaEventRecord(d.bp.done[0], d.s_comp));
+        if (r0 + m >= d.H) CU(cudaEventRecord(d.ev_io0, d.s_comp));  // last band updated
         CU(cudaStreamWaitEvent(d.bp.s_d2h, d.bp.done[0], 0));
         char* dst = static_cast<char*>(out.C) + ((size_t)(R0 + r0) * out.ld + (size_t)C0) * 4;
         CU(cudaMemcpy2DAsync(dst, out.ld * 4, C + (size_t)r0 * d.W, d.W * 4, d.W * 4, m, cudaMemcpyDeviceToHost,
@@ -957,6 +967,17 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     if (ctx->ipc_mode && !ctx->peers_ready)
         fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
     FPM_CHECK_ARG(!(ctx->ipc_mode && host), "IPC mode has no streamed host input (peers cannot be ordered)");
+    // streamed input: the grouping that starts with single pivots (setup)
+    struct GroupSwap {
+        pmm_ctx* c;
+        bool on;
+        GroupSwap(pmm_ctx* c_, bool on_) : c(c_), on(on_) {
+            if (on) std::swap(c->groups, c->groups_streamed);
+        }
+        ~GroupSwap() {
+            if (on) std::swap(c->groups, c->groups_streamed);
+        }
+    } group_swap(ctx, host != nullptr);
     const int L = out ? tail_groups(ctx) : 0;
     if (tail_done) tail_done->assign(ctx->devs.size(), 0);
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
@@ -1136,7 +1157,9 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
         t_max = std::max(t_max, (double)elapsed_ms(d.ev_start, d.ev_stop) * 1e-3);
         if (tail_done && (*tail_done)[i]) {  // copy still draining after the last update
             CU(cudaEventSynchronize(d.ev_io1));
-            t_tail_copy = std::max(t_tail_copy, std::max(0.0, (double)elapsed_ms(d.ev_stop, d.ev_io1) * 1e-3));
+            // exposed copy: from the end of the last band's updates (a timing event
+            // recorded before its copy is issued) to the end of that copy
+            t_tail_copy = std::max(t_tail_copy, std::max(0.0, (double)elapsed_ms(d.ev_io0, d.ev_io1) * 1e-3));
         }
     }
     if (st) {
@@ -1734,6 +1757,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= -1 && value <= fpm::kMaxTail, "e2e_tail must be -1 (auto), 0 (off) or 1..%d",
                           fpm::kMaxTail);
             ctx->e2e_tail = (int)value;
+        } else if (k == "tail_band") {
+            FPM_CHECK_ARG(value >= 256 && value % 256 == 0, "tail_band must be a positive multiple of 256 rows");
+            ctx->tail_band = value;
         } else if (k == "sm_partition") {
             FPM_CHECK_ARG(value == 0 || value == 1, "sm_partition must be 0 (grid caps) or 1 (green contexts)");
             if (ctx->sm_partition != (int)value) {

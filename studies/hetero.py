@@ -38,45 +38,32 @@ def imbalance(ts):
     return max(live) / (sum(live) / len(live)) - 1.0 if live else 0.0
 
 
-def main():
-    ap = argparse.ArgumentParser()
-    ap.add_argument("--N", type=int, default=32768)
-    ap.add_argument("--b", type=int, default=512)
-    ap.add_argument("--caps", default="30,26,24,20,16,14,10,6")
-    ap.add_argument("--ncal", type=int, default=8192)
-    ap.add_argument("--reps", type=int, default=2)
-    ap.add_argument("--sizes", default="1,2,3,4,6,8,12,16,20,24,28,32,40")
-    ap.add_argument("--concurrent", dest="exclusive", action="store_false",
-                    help="sample all devices at once (P:10 (ii)) instead of each alone (P:11, default)")
-    ap.add_argument("--insitu", type=int, default=2,
-                    help="extra FPM partitions with models rescaled by the speeds achieved in the previous run")
-    ap.add_argument("--graph", type=int, default=1, help="pmm_compute as a replayed CUDA graph (option graph)")
-    ap.add_argument("--sm-partition", type=int, default=0,
-                    help="1 = each device in its own green-context SM partition (all its kernels confined)")
-    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
-    args = ap.parse_args()
-    caps = [int(c) for c in args.caps.split(",")]
-    p, N, b = len(caps), args.N, args.b
+def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, graph=1, sm_partition=0,
+             exclusive=True, log=print) -> dict:
+    """Sample each emulated device's FPM, then run the multiply under the FPM,
+    CPM (N_cal and self-calibrated), homogeneous and in-situ corrected FPM
+    partitions; returns the result dict written by main()."""
+    p = len(caps)
     n = N // b
     T = n * n
-    sizes = [int(m) ** 2 for m in args.sizes.split(",")]
+    sizes = sizes or [m * m for m in (1, 2, 3, 4, 6, 8, 12, 16, 20, 24, 28, 32, 40)]
 
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
-    ctx.set_option("sm_partition", args.sm_partition)
-    ctx.set_option("graph", args.graph)
+    ctx.set_option("sm_partition", sm_partition)
+    ctx.set_option("graph", graph)
     t0 = time.perf_counter()
     models, sample_info = [], []
-    if args.exclusive:   # each device alone (how the paper measured its GPUs)
+    if exclusive:   # each device alone (how the paper measured its GPUs, P:11)
         per_dev = [ctx.sample(dev, b, sizes, pkg.FPM_F32) for dev in range(p)]
-    else:                # all devices at once (P:10 (ii)): contention as in the run
+    else:           # all devices at once (P:10 (ii)): contention as in the run
         sps, cis, repss = ctx.sample(-1, b, sizes, pkg.FPM_F32)
         per_dev = list(zip(sps, cis, repss))
-    for dev, (sp, ci, reps) in enumerate(per_dev):
+    for dev, (sp, ci, nrep) in enumerate(per_dev):
         models.append((sizes, sp))
-        sample_info.append({"cap": caps[dev], "speeds_gflops": [s / 1e9 for s in sp], "rel_ci95": ci, "reps": reps})
+        sample_info.append({"cap": caps[dev], "speeds_gflops": [s / 1e9 for s in sp], "rel_ci95": ci, "reps": nrep})
     t_sample = time.perf_counter() - t0
 
-    x_cal = max(1, (args.ncal // b) ** 2 // p)
+    x_cal = max(1, (ncal // b) ** 2 // p)
     x_even = T // p
     parts = {
         "fpm": pkg.fpm_partition(T, models),
@@ -101,7 +88,7 @@ def main():
         return out
 
     order = list(parts.items())
-    for it in range(args.insitu):
+    for it in range(insitu):
         order.append((f"fpm_insitu{it + 1}", None))
     cur_models = models
     for name, d in order:
@@ -114,7 +101,7 @@ def main():
         ctx.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
         ctx.compute()
         best = None
-        for _ in range(args.reps):
+        for _ in range(reps):
             st = ctx.compute()
             if best is None or st.t_compute_s < best.t_compute_s:
                 best = st
@@ -131,9 +118,8 @@ def main():
             "predicted_time_s": max(pred),
             "comm_bytes": best.comm_bytes,
         }
-        print(f"{name:12s} t={best.t_compute_s:8.4f}s  {best.gflops / 1e3:8.1f} TFLOP/s  "
-              f"imb meas={100 * imbalance(per_dev):6.2f}%  pred={100 * imbalance(pred):6.2f}%  d={d}",
-              flush=True)
+        log(f"{name:12s} t={best.t_compute_s:8.4f}s  {best.gflops / 1e3:8.1f} TFLOP/s  "
+            f"imb meas={100 * imbalance(per_dev):6.2f}%  pred={100 * imbalance(pred):6.2f}%  d={d}")
     ctx.close()
 
     # reference: the whole GPU as one device (upper bound of the aggregate)
@@ -142,15 +128,38 @@ def main():
         one.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
         one.compute()
         st1 = one.compute()
-    out = {
-        "config": {"N": N, "b": b, "p": p, "sm_caps": caps, "ncal": args.ncal, "x_cal": x_cal, "x_even": x_even,
-                   "sizes": sizes, "dtype": "f32 (F16X3)", "sm_partition": args.sm_partition, "gpu": "1x B200, devices emulated by SM caps",
-                   "sampling": "exclusive" if args.exclusive else "concurrent (all devices at once)"},
+    return {
+        "config": {"N": N, "b": b, "p": p, "sm_caps": list(caps), "ncal": ncal, "x_cal": x_cal, "x_even": x_even,
+                   "sizes": sizes, "dtype": "f32 (F16X3)", "sm_partition": sm_partition,
+                   "gpu": "1x B200, devices emulated by SM caps",
+                   "sampling": "exclusive" if exclusive else "concurrent (all devices at once)"},
         "fpm_sample_s": t_sample, "models": sample_info, "partitions": results,
         "whole_gpu": {"t_s": st1.t_compute_s, "gflops": st1.gflops},
         "fpm_vs_cpm_ncal_time_delta": results["fpm"]["t_total_s"] / results["cpm_ncal"]["t_total_s"] - 1.0,
         "fpm_vs_homogeneous_time_delta": results["fpm"]["t_total_s"] / results["homogeneous"]["t_total_s"] - 1.0,
     }
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--N", type=int, default=32768)
+    ap.add_argument("--b", type=int, default=512)
+    ap.add_argument("--caps", default="30,26,24,20,16,14,10,6")
+    ap.add_argument("--ncal", type=int, default=8192)
+    ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--sizes", default="1,2,3,4,6,8,12,16,20,24,28,32,40")
+    ap.add_argument("--concurrent", dest="exclusive", action="store_false",
+                    help="sample all devices at once (P:10 (ii)) instead of each alone (P:11, default)")
+    ap.add_argument("--insitu", type=int, default=2,
+                    help="extra FPM partitions with models rescaled by the speeds achieved in the previous run")
+    ap.add_argument("--graph", type=int, default=1, help="pmm_compute as a replayed CUDA graph (option graph)")
+    ap.add_argument("--sm-partition", type=int, default=0,
+                    help="1 = each device in its own green-context SM partition (all its kernels confined)")
+    ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
+    args = ap.parse_args()
+    caps = [int(c) for c in args.caps.split(",")]
+    out = c4_study(caps, args.N, args.b, [int(m) ** 2 for m in args.sizes.split(",")], args.ncal, args.reps,
+                   args.insitu, args.graph, args.sm_partition, args.exclusive, log=lambda s: print(s, flush=True))
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)

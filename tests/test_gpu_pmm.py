@@ -96,6 +96,27 @@ def test_fused_pivot_groups(fuse):
         assert np.array_equal(Ci.astype(np.float64), og.gemm(Ai, Bi))
 
 
+def test_streamed_run_starts_with_single_pivots():
+    """pmm_run (host-streamed inputs) groups {0}, {1}, {2..9}, {10..15} at
+    n = 16, f = 8; pmm_compute on resident inputs {0..7}, {8..15}.  Same C
+    within tolerance, integer inputs bit-exact on both."""
+    N, b = 2048, 128
+    n = N // b
+    rects = [(0, 0, 0, n, n)]
+    with pkg.Context.local([0]) as ctx:
+        ctx.set_option("fuse", 8)
+        A, B, C, st = _run(ctx, N, b, rects, pkg.FPM_F32)
+        assert st.updates == 4
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+        ctx.upload(A, B, N)
+        assert ctx.compute().updates == 2
+        Cr = np.full((N, N), np.nan, np.float32)
+        ctx.download(Cr, N)
+        assert og.rel_fro(Cr, og.gemm(A, B)) <= 1e-5
+        Ai, Bi, Ci, st = _run(ctx, N, b, rects, pkg.FPM_F32, dist=synth.DIST_INT, seeds=(7, 8))
+        assert np.array_equal(Ci.astype(np.float64), og.gemm(Ai, Bi)) and st.updates == 4
+
+
 def test_single_iteration_b_equals_n():
     """n = 1: one pivot, one update that overwrites C."""
     N = b = 512

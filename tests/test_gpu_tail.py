@@ -56,8 +56,9 @@ def test_tail_integer_exact_mixed_ooc(fuse):
 
 
 def test_single_group_all_tail():
-    """One update group (n = 4, f = 4): the whole k-loop is the tail and its
-    first (only) group overwrites C."""
+    """n = 4, f = 4: pmm_run streams its inputs, so its groups are {0}, {1},
+    {2, 3} (two single pivots first, runtime.cu setup); the whole k-loop is the
+    tail and its first group overwrites C."""
     N, b = 512, 128
     A = synth.rect(3, N, 0, 0, N, N)
     B = synth.rect(4, N, 0, 0, N, N)
@@ -65,7 +66,7 @@ def test_single_group_all_tail():
     with pkg.Context.local([0]) as ctx:
         ctx.set_option("e2e_tail", 16)
         st = ctx.run(A, B, C, N, b, [(0, 0, 0, 4, 4)], pkg.FPM_F32)
-        assert st.updates == 1
+        assert st.updates == 3
     assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
 
 
