@@ -295,6 +295,11 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 cover the copy at ~55 GB/s), 0 off, 1..16.
  *   "tail_band":  rows of C_i per band of that tail, a positive multiple of
  *                 256 (default 2048); the last band's copy stays exposed.
+ *   "tail_fuse":  1 (default; FP32 local / IPC contexts): the tail's pivots are
+ *                 staged side by side as ONE operand with one F16X3 scale per
+ *                 row / column over all of them (maxima merged first), so each
+ *                 band takes a single update and one read-modify-write of C;
+ *                 0: one update per tail group and band.
  *   "sm_partition": how an SM cap is enforced.  0 (default): the cap is the
  *                 grid of the persistent update kernel (one CTA per SM); other
  *                 kernels of the device are not confined, and devices sharing a

@@ -47,13 +47,24 @@ void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, Sp
 // Fused pivots: row r of the operand is nseg segments of K elements, segment j
 // at src + j*seg_stride + r*ld; output row stride ld_out (>= nseg*K); the F16X3
 // scale is taken over the whole fused row.
+// With given_max (F16X3), the row maxima are taken from it (bits of non-negative
+// floats, e.g. from launch_rowmax_seg over a wider K) instead of this panel.
 void launch_split_rows_seg(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t rows, int64_t K,
-                           int64_t ld_out, SplitScheme s, void* hi, void* lo, float* inv_scale, cudaStream_t st);
+                           int64_t ld_out, SplitScheme s, void* hi, void* lo, float* inv_scale, cudaStream_t st,
+                           const unsigned* given_max = nullptr);
 
 // B pivot row src (K x W, row stride ld) -> split halves of its transpose
 // (W x K, K-major), per-row (= per-column of src) inverse scales for F16X3.
+// ld_out: row stride of the output (default K); given_max as above (per column).
 void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,
-                       float* inv_scale, cudaStream_t st);
+                       float* inv_scale, cudaStream_t st, int64_t ld_out = -1, const unsigned* given_max = nullptr);
+
+// m_bits[r] = max(m_bits[r], bits of max |x| over row r of the (fused) panel)
+// -- atomicMax on the bit patterns of non-negative floats; zero m_bits first.
+void launch_rowmax_seg(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t rows, int64_t K,
+                       unsigned* m_bits, cudaStream_t st);
+// m_bits[c] = max(m_bits[c], bits of max |x| over column c of a K x W block-row)
+void launch_colmax(const float* src, int64_t ld, int64_t K, int64_t W, unsigned* m_bits, cudaStream_t st);
 
 // dst (cols x rows, K-major) = transpose of src (rows x cols, ld).
 void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t cols, float* dst,

@@ -31,13 +31,10 @@ __device__ __forceinline__ float warp_max(float v) {
 // fused into one update); it is written to out + row * ld_out + j * K.
 // F16X3: choose 2^s with the maximum of the whole (fused) row scaled into
 // [2^14, 2^15), h0 = fp16(x 2^s), h1 = fp16(x 2^s - h0); inv_scale = 2^-s.
-__global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ src, int64_t ld, int64_t seg_stride,
-                                                      int nseg, int64_t rows, int64_t K, int64_t ld_out,
-                                                      __half* __restrict__ hi, __half* __restrict__ lo,
-                                                      float* __restrict__ inv_scale) {
-    const int64_t row = (int64_t)blockIdx.x * 8 + threadIdx.x / 32;
-    const int lane = threadIdx.x % 32;
-    if (row >= rows) return;
+// With `given` set, the row maximum is given[row] (bits of a non-negative float,
+// from rowmax_k over a wider K range) and the first pass is skipped.
+__device__ __forceinline__ float row_absmax(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t row,
+                                            int64_t K, int lane) {
     const int64_t n4 = K / 4;
     float m = 0.0f;
     for (int j = 0; j < nseg; ++j) {
@@ -47,7 +44,19 @@ __global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ 
             m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
         }
     }
-    m = warp_max(m);
+    return warp_max(m);
+}
+
+__global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ src, int64_t ld, int64_t seg_stride,
+                                                      int nseg, int64_t rows, int64_t K, int64_t ld_out,
+                                                      __half* __restrict__ hi, __half* __restrict__ lo,
+                                                      float* __restrict__ inv_scale,
+                                                      const unsigned* __restrict__ given) {
+    const int64_t row = (int64_t)blockIdx.x * 8 + threadIdx.x / 32;
+    const int lane = threadIdx.x % 32;
+    if (row >= rows) return;
+    const int64_t n4 = K / 4;
+    const float m = given ? __uint_as_float(given[row]) : row_absmax(src, ld, seg_stride, nseg, row, K, lane);
     int e = 0;
     if (m > 0.0f) {
         frexpf(m, &e);  // m < 2^e
@@ -105,23 +114,30 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
 // update kernel (which leaves < 2 KB of shared memory per SM).  Pass 1: column
 // maxima; pass 2: each lane converts its column's 8-row chunks and writes them
 // as 16 B of output row (col, k0..k0+7).
+__device__ __forceinline__ float col_absmax(const float* src, int64_t ld, int64_t K, int64_t col) {
+    float m[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
+    for (int64_t ch = 0; ch < K / 8; ++ch)
+#pragma unroll
+        for (int i = 0; i < 8; ++i) m[i] = fmaxf(m[i], fabsf(src[(ch * 8 + i) * ld + col]));
+    float mm = m[0];
+#pragma unroll
+    for (int i = 1; i < 8; ++i) mm = fmaxf(mm, m[i]);
+    return mm;
+}
+
+// Output row `col` is written at col * ld_out (ld_out >= K: the K rows land in
+// the first K elements, so a wider fused operand can be staged in pieces).
 template <bool F16>
 __global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
-                                                    void* __restrict__ hi, void* __restrict__ lo,
-                                                    float* __restrict__ inv_scale) {
+                                                    int64_t ld_out, void* __restrict__ hi, void* __restrict__ lo,
+                                                    float* __restrict__ inv_scale, const unsigned* __restrict__ given) {
     const int lane = threadIdx.x % 32;
     const int64_t col = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 32 + lane;
     if (col >= W) return;
     const int64_t nchunks = K / 8;
     float scale = 1.0f;
     if constexpr (F16) {
-        float m[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-        for (int64_t ch = 0; ch < nchunks; ++ch)
-#pragma unroll
-            for (int i = 0; i < 8; ++i) m[i] = fmaxf(m[i], fabsf(src[(ch * 8 + i) * ld + col]));
-        float mm = m[0];
-#pragma unroll
-        for (int i = 1; i < 8; ++i) mm = fmaxf(mm, m[i]);
+        const float mm = given ? __uint_as_float(given[col]) : col_absmax(src, ld, K, col);
         int e = 0;
         if (mm > 0.0f) frexpf(mm, &e);
         int s = (mm > 0.0f) ? 15 - e : 0;
@@ -141,8 +157,8 @@ __global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ sr
                 h[i] = __float2half_rn(xs);
                 l[i] = __float2half_rn(xs - __half2float(h[i]));
             }
-            *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + col * K + ch * 8) = *reinterpret_cast<uint4*>(h);
-            *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + col * K + ch * 8) = *reinterpret_cast<uint4*>(l);
+            *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + col * ld_out + ch * 8) = *reinterpret_cast<uint4*>(h);
+            *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + col * ld_out + ch * 8) = *reinterpret_cast<uint4*>(l);
         } else {
             __align__(16) float h[8], l[8];
 #pragma unroll
@@ -150,14 +166,33 @@ __global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ sr
                 h[i] = tf32_rna(x[i]);
                 l[i] = tf32_rna(x[i] - h[i]);
             }
-            float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + col * K + ch * 8);
-            float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + col * K + ch * 8);
+            float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + col * ld_out + ch * 8);
+            float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + col * ld_out + ch * 8);
             hp[0] = *reinterpret_cast<float4*>(h);
             hp[1] = *reinterpret_cast<float4*>(h + 4);
             lp[0] = *reinterpret_cast<float4*>(l);
             lp[1] = *reinterpret_cast<float4*>(l + 4);
         }
     }
+}
+
+// Maxima |x| of the rows of a (fused) panel / the columns of a block-row, merged
+// into m_bits with atomicMax on the bit patterns (non-negative floats order like
+// their bits): the common F16X3 scale of an operand staged in several pieces.
+__global__ void __launch_bounds__(256) rowmax_k(const float* __restrict__ src, int64_t ld, int64_t seg_stride,
+                                                int nseg, int64_t rows, int64_t K, unsigned* __restrict__ m_bits) {
+    const int64_t row = (int64_t)blockIdx.x * 8 + threadIdx.x / 32;
+    const int lane = threadIdx.x % 32;
+    if (row >= rows) return;
+    const float m = row_absmax(src, ld, seg_stride, nseg, row, K, lane);
+    if (lane == 0) atomicMax(m_bits + row, __float_as_uint(m));
+}
+
+__global__ void __launch_bounds__(256) colmax_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
+                                                unsigned* __restrict__ m_bits) {
+    const int64_t col = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 32 + threadIdx.x % 32;
+    if (col >= W) return;
+    atomicMax(m_bits + col, __float_as_uint(col_absmax(src, ld, K, col)));
 }
 
 template <class T>
@@ -351,7 +386,8 @@ void check_launch(const char* what) {
 }  // namespace
 
 void launch_split_rows_seg(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t rows, int64_t K,
-                           int64_t ld_out, SplitScheme s, void* hi, void* lo, float* inv_scale, cudaStream_t st) {
+                           int64_t ld_out, SplitScheme s, void* hi, void* lo, float* inv_scale, cudaStream_t st,
+                           const unsigned* given_max) {
     if (rows <= 0 || K <= 0 || nseg <= 0) return;
     FPM_CHECK_ARG(K % 4 == 0 && ld % 4 == 0 && seg_stride % 4 == 0 && ld_out % 4 == 0 && ld_out >= nseg * K,
                   "split: K, ld, seg_stride, ld_out must be multiples of 4 and ld_out >= nseg*K");
@@ -359,7 +395,7 @@ void launch_split_rows_seg(const float* src, int64_t ld, int64_t seg_stride, int
         const int64_t blocks = (rows + 7) / 8;
         split_rows_f16<<<(unsigned)blocks, 256, 0, st>>>(src, ld, seg_stride, nseg, rows, K, ld_out,
                                                          static_cast<__half*>(hi), static_cast<__half*>(lo),
-                                                         inv_scale);
+                                                         inv_scale, given_max);
         check_launch("split_rows_f16");
     } else {
         split_rows_tf32<<<grid_for(rows * nseg * K / 4, 256), 256, 0, st>>>(
@@ -374,17 +410,33 @@ void launch_split_rows(const float* src, int64_t ld, int64_t rows, int64_t K, Sp
 }
 
 void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, SplitScheme s, void* hi, void* lo,
-                       float* inv_scale, cudaStream_t st) {
+                       float* inv_scale, cudaStream_t st, int64_t ld_out, const unsigned* given_max) {
     if (K <= 0 || W <= 0) return;
-    FPM_CHECK_ARG(K % 8 == 0, "split_cols: K must be a multiple of 8");
+    if (ld_out < 0) ld_out = K;
+    FPM_CHECK_ARG(K % 8 == 0 && ld_out % 8 == 0 && ld_out >= K, "split_cols: K, ld_out multiples of 8, ld_out >= K");
     const unsigned blocks = (unsigned)((W + 255) / 256);  // 8 warps x 32 columns per block
     if (s == SplitScheme::F16X3) {
         FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
-        split_cols_k<true><<<blocks, 256, 0, st>>>(src, ld, K, W, hi, lo, inv_scale);
+        split_cols_k<true><<<blocks, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, inv_scale, given_max);
     } else {
-        split_cols_k<false><<<blocks, 256, 0, st>>>(src, ld, K, W, hi, lo, inv_scale);
+        split_cols_k<false><<<blocks, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, inv_scale, nullptr);
     }
     check_launch("split_cols");
+}
+
+void launch_rowmax_seg(const float* src, int64_t ld, int64_t seg_stride, int nseg, int64_t rows, int64_t K,
+                       unsigned* m_bits, cudaStream_t st) {
+    if (rows <= 0 || K <= 0 || nseg <= 0) return;
+    FPM_CHECK_ARG(K % 4 == 0 && ld % 4 == 0 && seg_stride % 4 == 0, "rowmax: K, ld, seg_stride multiples of 4");
+    rowmax_k<<<(unsigned)((rows + 7) / 8), 256, 0, st>>>(src, ld, seg_stride, nseg, rows, K, m_bits);
+    check_launch("rowmax");
+}
+
+void launch_colmax(const float* src, int64_t ld, int64_t K, int64_t W, unsigned* m_bits, cudaStream_t st) {
+    if (K <= 0 || W <= 0) return;
+    FPM_CHECK_ARG(K % 8 == 0, "colmax: K must be a multiple of 8");
+    colmax_k<<<(unsigned)((W + 255) / 256), 256, 0, st>>>(src, ld, K, W, m_bits);
+    check_launch("colmax");
 }
 
 void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t cols, float* dst, cudaStream_t st) {

@@ -49,7 +49,8 @@ namespace fpm {
 // three streams.
 constexpr int kMaxBandBufs = 16;
 constexpr int kMaxTail = 16;             // groups of the download-overlapped tail
-constexpr int kSlots = 2 + kMaxTail;     // operand slots per device
+constexpr int kSlots = 3 + kMaxTail;     // operand slots per device
+constexpr int kFusedSlot = kSlots - 1;  // the fused tail: all tail pivots as one operand
 struct Ring {
     int R;         // buffers in use
     int64_t rows;  // rows per band
@@ -103,6 +104,14 @@ struct Device {
     float* sa[kSlots] = {}, *sb[kSlots] = {};
     const void* a_op[kSlots] = {};          // FP64: A operand of the slot
     int tail_slots = 0;                     // slots 2.. allocated
+    // fused tail (kFusedSlot): the tail's pivots staged as one K = tail_K operand
+    // with common F16X3 scales (maxima merged in tmax_a / tmax_b first)
+    int64_t tail_K = 0, tail_K_alloc = 0;
+    unsigned* tmax_a = nullptr;
+    unsigned* tmax_b = nullptr;
+    std::vector<void*> tail_allocs;
+    cudaEvent_t ev_tpack0 = nullptr, ev_tpack1 = nullptr;  // staging of the fused tail (second pass)
+    bool tail_fused_run = false;  // the current k-loop stages its tail into kFusedSlot
     std::vector<void*> allocs;
     int64_t launches = 0;                   // library kernels launched (running count)
 
@@ -144,6 +153,7 @@ struct pmm_ctx {
     int64_t g_bytes = 0, g_launches = 0;
     int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
     int64_t tail_band = 2048; // rows of C_i per band of the tail (multiple of 256)
+    int tail_fuse = 1;        // local / IPC FP32: the tail as one fused operand (1) or per group (0)
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
@@ -330,6 +340,10 @@ void free_problem(Device& d) {
     }
     d.A = d.B = d.C = nullptr;
     d.tail_slots = 0;
+    for (void* p : d.tail_allocs) cudaFree(p);
+    d.tail_allocs.clear();
+    d.tail_K = d.tail_K_alloc = 0;
+    d.tmax_a = d.tmax_b = nullptr;
     for (int s = 0; s < kSlots; ++s) {
         d.a_recv[s] = d.b_recv[s] = d.bt[s] = d.a_hi[s] = d.a_lo[s] = d.b_hi[s] = d.b_lo[s] = nullptr;
         d.sa[s] = d.sb[s] = nullptr;
@@ -366,6 +380,8 @@ void init_device(Device& d) {
     CU(cudaEventCreate(&d.ev_stop));
     CU(cudaEventCreate(&d.ev_io0));
     CU(cudaEventCreate(&d.ev_io1));
+    CU(cudaEventCreate(&d.ev_tpack0));
+    CU(cudaEventCreate(&d.ev_tpack1));
     for (auto& e : d.ev_join) CU(cudaEventCreateWithFlags(&e, cudaEventDisableTiming));
     bp_init(d.bp);
 }
@@ -378,7 +394,7 @@ void destroy_device(Device& d) {
         if (d.ev_ready[s]) cudaEventDestroy(d.ev_ready[s]);
         if (d.ev_free[s]) cudaEventDestroy(d.ev_free[s]);
     }
-    for (cudaEvent_t e : {d.ev_start, d.ev_stop, d.ev_io0, d.ev_io1})
+    for (cudaEvent_t e : {d.ev_start, d.ev_stop, d.ev_io0, d.ev_io1, d.ev_tpack0, d.ev_tpack1})
         if (e) cudaEventDestroy(e);
     for (auto& e : d.ev_join) {
         if (e) cudaEventDestroy(e);
@@ -389,7 +405,7 @@ void destroy_device(Device& d) {
     if (d.s_up) cudaStreamDestroy(d.s_up);
     d.s_comp = d.s_comm = d.s_up = nullptr;
     for (int s = 0; s < kSlots; ++s) d.ev_ready[s] = d.ev_free[s] = nullptr;
-    d.ev_start = d.ev_stop = d.ev_io0 = d.ev_io1 = nullptr;
+    d.ev_start = d.ev_stop = d.ev_io0 = d.ev_io1 = d.ev_tpack0 = d.ev_tpack1 = nullptr;
     green_destroy(d.green);
 }
 
@@ -660,7 +676,17 @@ void issue_upload(pmm_ctx* ctx, Device& d, int64_t k, const HostSrc& h) {
 // Exchange + staging of update group g (pivots k0 .. k0+f-1) on device d's comm
 // stream.  All pivots of a group share their holders and owners (setup), so the
 // group moves as the plan of k0 with f-times longer panels.
-int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, bool streamed) {
+// Fused tail (kFusedSlot): phase 1 merges the group's row / column maxima into
+// tmax_a / tmax_b, phase 2 splits it with those maxima into K columns
+// [k_off, k_off + f b) of the tail operand (row stride tail_K).  Phase 0: the
+// ordinary staging into the slot.
+struct TailPhase {
+    int phase = 0;
+    int64_t k_off = 0;
+};
+
+int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, bool streamed,
+                   TailPhase tp = TailPhase{}) {
     const size_t es = esize(ctx->dt);
     const int64_t b = ctx->b;
     const int64_t k0 = ctx->groups[g].first;
@@ -772,33 +798,55 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     }
 
     // ---- staging: K-major operands of the fused update (K = f b)
-    rec_t(d.ev_pack0[g], d.s_comm);
+    if (tp.phase != 2) rec_t(d.ev_pack0[g], d.s_comm);
     if (ctx->dt == FPM_F32) {
         const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
-        const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
-        d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + 1;
-        if (a_src) {  // own or received panels: f consecutive H x b panels
-            launch_split_rows_seg(static_cast<const float*>(a_src), b, d.H * b, f, d.H, b, fb, sch,
-                                  d.a_hi[slot], d.a_lo[slot], d.sa[slot], d.s_comm);
-        } else {
-            for (const Piece& pc : a_pieces)
-                launch_split_rows_seg(static_cast<const float*>(pc.src), b, pc.seg_stride, f, pc.rows, b, fb, sch,
-                                      static_cast<char*>(d.a_hi[slot]) + (size_t)pc.row_off * fb * op,
-                                      static_cast<char*>(d.a_lo[slot]) + (size_t)pc.row_off * fb * op,
-                                      d.sa[slot] + pc.row_off, d.s_comm);
-        }
+        const bool f16 = sch == SplitScheme::F16X3;
+        const size_t op = f16 ? 2 : 4;
         FPM_CHECK_ARG(b_src != nullptr, "no source of block-row %lld for device %d", (long long)k0, d.idx);
-        launch_split_cols(static_cast<const float*>(b_src), d.W, fb, d.W, sch, d.b_hi[slot], d.b_lo[slot],
-                          d.sb[slot], d.s_comm);
+        if (tp.phase == 1) {  // maxima only (TF32X3 has no scales: nothing to do)
+            if (f16) {
+                d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + 1;
+                if (a_src) {
+                    launch_rowmax_seg(static_cast<const float*>(a_src), b, d.H * b, f, d.H, b, d.tmax_a, d.s_comm);
+                } else {
+                    for (const Piece& pc : a_pieces)
+                        launch_rowmax_seg(static_cast<const float*>(pc.src), b, pc.seg_stride, f, pc.rows, b,
+                                          d.tmax_a + pc.row_off, d.s_comm);
+                }
+                launch_colmax(static_cast<const float*>(b_src), d.W, fb, d.W, d.tmax_b, d.s_comm);
+            }
+        } else {
+            const int64_t ld_out = tp.phase == 2 ? d.tail_K : fb;
+            const size_t ko = (size_t)tp.k_off * op;
+            const unsigned* ga = (tp.phase == 2 && f16) ? d.tmax_a : nullptr;
+            const unsigned* gb = (tp.phase == 2 && f16) ? d.tmax_b : nullptr;
+            d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + 1;
+            if (a_src) {  // own or received panels: f consecutive H x b panels
+                launch_split_rows_seg(static_cast<const float*>(a_src), b, d.H * b, f, d.H, b, ld_out, sch,
+                                      static_cast<char*>(d.a_hi[slot]) + ko, static_cast<char*>(d.a_lo[slot]) + ko,
+                                      d.sa[slot], d.s_comm, ga);
+            } else {
+                for (const Piece& pc : a_pieces)
+                    launch_split_rows_seg(
+                        static_cast<const float*>(pc.src), b, pc.seg_stride, f, pc.rows, b, ld_out, sch,
+                        static_cast<char*>(d.a_hi[slot]) + (size_t)pc.row_off * ld_out * op + ko,
+                        static_cast<char*>(d.a_lo[slot]) + (size_t)pc.row_off * ld_out * op + ko,
+                        d.sa[slot] + pc.row_off, d.s_comm, ga ? ga + pc.row_off : nullptr);
+            }
+            launch_split_cols(static_cast<const float*>(b_src), d.W, fb, d.W, sch,
+                              static_cast<char*>(d.b_hi[slot]) + ko, static_cast<char*>(d.b_lo[slot]) + ko,
+                              d.sb[slot], d.s_comm, ld_out, gb);
+        }
     } else {
         d.a_op[slot] = a_src;
         launch_transpose_f64(static_cast<const double*>(b_src), d.W, b, d.W, static_cast<double*>(d.bt[slot]),
                              d.s_comm);
         d.launches += 1;
     }
-    rec_t(d.ev_pack1[g], d.s_comm);
-    CU(cudaEventRecord(d.ev_ready[slot], d.s_comm));
-    return bytes;
+    if (tp.phase != 2) rec_t(d.ev_pack1[g], d.s_comm);
+    if (tp.phase == 0) CU(cudaEventRecord(d.ev_ready[slot], d.s_comm));
+    return tp.phase == 2 ? 0 : bytes;
 }
 
 // FP32 update of group g from operand slot `slot` over all of C_i.
@@ -896,9 +944,11 @@ struct HostDst {
 
 // Groups of the download-overlapped tail (option "e2e_tail"; FP32, resident
 // C_i).  Auto: enough of the last updates to cover the device -> host copy of
-// C_i: per element of C_i the copy costs 4 B at ~55 GB/s, the k-loop 2 N flop
-// at ~3 TFLOP/s per SM (measured), so L = ceil(G * 1.15 * ratio).
-int tail_groups(pmm_ctx* ctx) {
+// C_i -- per element of C_i the copy costs 4 B at ~55 GB/s, the k-loop 2 N flop
+// at ~3 TFLOP/s per SM (measured) -- but, when the inputs are streamed in
+// (pmm_run), no more than leaves the uploads (8 B per element of C_i) under the
+// groups before the tail: the tail's staging needs its pivots on the device.
+int tail_groups(pmm_ctx* ctx, bool streamed) {
     const int G = (int)ctx->groups.size();
     if (ctx->dt != FPM_F32 || ctx->e2e_tail == 0 || G == 0) return 0;
     if (ctx->e2e_tail > 0) return std::min({ctx->e2e_tail, G, kMaxTail});
@@ -906,13 +956,53 @@ int tail_groups(pmm_ctx* ctx) {
     for (auto& d : ctx->devs)
         if (d.live() && !d.ooc) r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (3.0e12 * d.num_sms)));
     if (r == 0.0) return 0;
-    return std::max(1, std::min({(int)std::ceil(G * 1.15 * r), G, kMaxTail}));
+    int L = (int)std::ceil(G * 1.05 * r);
+    if (streamed) L = std::min(L, G - (int)std::ceil(G * 2.0 * r));
+    return std::max(1, std::min({L, G, kMaxTail}));
 }
 
 // Operand slots 2 .. 2+L-1 for the tail groups (allocated once per problem).
 void ensure_tail_slots(pmm_ctx* ctx, Device& d, int L) {
     CU(cudaSetDevice(d.cuda_dev));
     for (; d.tail_slots < L; ++d.tail_slots) alloc_slot(ctx, d, 2 + d.tail_slots);
+}
+
+// The tail as ONE operand (local / IPC FP32): the pivots of groups gt.. staged
+// side by side along K with common F16X3 row / column scales, so each band of
+// C_i takes one update of K = tail_K -- one read-modify-write of the band
+// instead of one per group.  The same sum per element as the group-major
+// loop, with one scale per row over the tail instead of one per group.
+bool use_fused_tail(const pmm_ctx* ctx) { return ctx->tail_fuse && ctx->dt == FPM_F32 && !ctx->nccl_mode; }
+
+void ensure_fused_tail(pmm_ctx* ctx, Device& d, int gt) {
+    int64_t K = 0;
+    for (size_t g = gt; g < ctx->groups.size(); ++g) K += (int64_t)ctx->groups[g].second * ctx->b;
+    d.tail_K = K;
+    if (K <= d.tail_K_alloc) return;
+    CU(cudaSetDevice(d.cuda_dev));
+    CU(cudaDeviceSynchronize());
+    for (void* p : d.tail_allocs) cudaFree(p);
+    d.tail_allocs.clear();
+    const size_t op = ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4;
+    auto get = [&](size_t bytes) {
+        void* p = nullptr;
+        if (cudaMalloc(&p, bytes) != cudaSuccess) {
+            cudaGetLastError();
+            fail(FPM_ENOMEM, "device %d: cannot allocate %zu bytes for the fused tail", d.cuda_dev, bytes);
+        }
+        d.tail_allocs.push_back(p);
+        return p;
+    };
+    const int s = kFusedSlot;
+    d.a_hi[s] = get((size_t)d.H * K * op);
+    d.a_lo[s] = get((size_t)d.H * K * op);
+    d.b_hi[s] = get((size_t)d.W * K * op);
+    d.b_lo[s] = get((size_t)d.W * K * op);
+    d.sa[s] = static_cast<float*>(get((size_t)d.H * sizeof(float)));
+    d.sb[s] = static_cast<float*>(get((size_t)d.W * sizeof(float)));
+    d.tmax_a = static_cast<unsigned*>(get((size_t)d.H * sizeof(unsigned)));
+    d.tmax_b = static_cast<unsigned*>(get((size_t)d.W * sizeof(unsigned)));
+    d.tail_K_alloc = K;
 }
 
 // The tail of the k-loop, band-major: for each band of C_i rows, the updates of
@@ -922,15 +1012,29 @@ void ensure_tail_slots(pmm_ctx* ctx, Device& d, int L) {
 // group-major loop (each element still receives the groups in k order).
 void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
     CU(cudaSetDevice(d.cuda_dev));
-    for (int t = 0; t < L; ++t) CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[2 + t], 0));
+    const bool fused = d.tail_fused_run;
+    if (fused) {
+        CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[kFusedSlot], 0));
+    } else {
+        for (int t = 0; t < L; ++t) CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[2 + t], 0));
+    }
     CU(cudaEventRecord(d.ev_upd0[g0], d.s_comp));
+    UpdateArgs fa;  // fused: all tail pivots in one operand of K = tail_K
+    if (fused) {
+        fa = f32_args(ctx, d, g0, kFusedSlot);
+        fa.K = d.tail_K;
+    }
     const int64_t band = std::min<int64_t>(d.H, ctx->tail_band);  // whole CTA-pair tile rows
     const int64_t b = ctx->b;
     const int64_t R0 = d.rect.row0 * b - out.row_base, C0 = d.rect.col0 * b - out.col_base;
     float* C = static_cast<float*>(d.C);
     for (int64_t r0 = 0; r0 < d.H; r0 += band) {
         const int64_t m = std::min(band, d.H - r0);
-        for (int t = 0; t < L; ++t) {
+        if (fused) {
+            launch_update_f32(band_args(fa, r0, m, C + (size_t)r0 * d.W), d.s_comp);
+            d.launches += 1;
+        }
+        for (int t = 0; t < L && !fused; ++t) {
             const UpdateArgs a = f32_args(ctx, d, g0 + t, 2 + t);
             launch_update_f32(band_args(a, r0, m, C + (size_t)r0 * d.W), d.s_comp);
             d.launches += 1;
@@ -947,7 +1051,11 @@ void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
         CU(cudaEventRecord(d.ev_upd0[g0 + t], d.s_comp));
         CU(cudaEventRecord(d.ev_upd1[g0 + t], d.s_comp));
     }
-    for (int t = 0; t < L; ++t) CU(cudaEventRecord(d.ev_free[2 + t], d.s_comp));
+    if (fused) {
+        CU(cudaEventRecord(d.ev_free[kFusedSlot], d.s_comp));
+    } else {
+        for (int t = 0; t < L; ++t) CU(cudaEventRecord(d.ev_free[2 + t], d.s_comp));
+    }
     CU(cudaEventRecord(d.ev_io1, d.bp.s_d2h));  // C_i in host memory
 }
 
@@ -978,12 +1086,19 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
             if (on) std::swap(c->groups, c->groups_streamed);
         }
     } group_swap(ctx, host != nullptr);
-    const int L = out ? tail_groups(ctx) : 0;
+    const int L = out ? tail_groups(ctx, host != nullptr) : 0;
     if (tail_done) tail_done->assign(ctx->devs.size(), 0);
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
+        d.tail_fused_run = false;
         if (L > 0 && d.live() && !d.ooc) {
-            ensure_tail_slots(ctx, d, L);  // before the timed region (cudaMalloc synchronises)
+            // before the timed region (cudaMalloc synchronises)
+            if (use_fused_tail(ctx)) {
+                ensure_fused_tail(ctx, d, (int)ctx->groups.size() - L);
+                d.tail_fused_run = true;
+            } else {
+                ensure_tail_slots(ctx, d, L);
+            }
             if (tail_done) (*tail_done)[i] = 1;
         }
     }
@@ -1037,7 +1152,9 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     // tail devices take tail groups from slots 2.. and update them band-major
     // after the loop; everyone else (and every group before gt) as usual
     auto in_tail = [&](const Device& d, int g) { return g >= gt && d.live() && !d.ooc; };
-    auto slot_of = [&](const Device& d, int g) { return in_tail(d, g) ? 2 + (g - gt) : (g & 1); };
+    auto slot_of = [&](const Device& d, int g) {
+        return in_tail(d, g) ? (d.tail_fused_run ? kFusedSlot : 2 + (g - gt)) : (g & 1);
+    };
     for (int g = 0; g < ngroups; ++g) {
         const int64_t k0 = ctx->groups[g].first;
         if (streamed)
@@ -1060,10 +1177,32 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
         for (auto& d : ctx->devs)
             if (d.live()) {
                 const int slot = slot_of(d, g);
-                bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed);
+                if (in_tail(d, g) && d.tail_fused_run) {  // fused tail, pass 1: merge the maxima
+                    if (g == gt) {
+                        CU(cudaMemsetAsync(d.tmax_a, 0, (size_t)d.H * sizeof(unsigned), d.s_comm));
+                        CU(cudaMemsetAsync(d.tmax_b, 0, (size_t)d.W * sizeof(unsigned), d.s_comm));
+                    }
+                    bytes += issue_comm(ctx, d, g, slot, false, streamed, TailPhase{1, 0});
+                } else {
+                    bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed);
+                }
             }
         for (auto& d : ctx->devs)
             if (d.live() && !in_tail(d, g)) issue_update(ctx, d, g, g & 1);
+    }
+    // fused tail, pass 2: split every tail group with the merged maxima into its
+    // K range of the tail operand
+    for (auto& d : ctx->devs) {
+        if (L == 0 || !d.live() || d.ooc || !d.tail_fused_run) continue;
+        CU(cudaSetDevice(d.cuda_dev));
+        rec_t(d.ev_tpack0, d.s_comm);
+        int64_t k_off = 0;
+        for (int g = gt; g < ngroups; ++g) {
+            issue_comm(ctx, d, g, kFusedSlot, false, streamed, TailPhase{2, k_off});
+            k_off += (int64_t)ctx->groups[g].second * ctx->b;
+        }
+        rec_t(d.ev_tpack1, d.s_comm);
+        CU(cudaEventRecord(d.ev_ready[kFusedSlot], d.s_comm));
     }
     if (L > 0)
         for (auto& d : ctx->devs)
@@ -1192,6 +1331,7 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
                 comp += u + elapsed_ms(d.ev_pack0[g], d.ev_pack1[g]) * 1e-3;
                 upd += u;
             }
+            if (d.tail_fused_run) comp += elapsed_ms(d.ev_tpack0, d.ev_tpack1) * 1e-3;
             if (d.idx < FPM_MAX_DEVICES) {
                 st->per_dev_compute_s[d.idx] = comp;
                 st->per_dev_update_s[d.idx] = upd;
@@ -1757,6 +1897,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= -1 && value <= fpm::kMaxTail, "e2e_tail must be -1 (auto), 0 (off) or 1..%d",
                           fpm::kMaxTail);
             ctx->e2e_tail = (int)value;
+        } else if (k == "tail_fuse") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "tail_fuse must be 0 or 1");
+            ctx->tail_fuse = (int)value;
         } else if (k == "tail_band") {
             FPM_CHECK_ARG(value >= 256 && value % 256 == 0, "tail_band must be a positive multiple of 256 rows");
             ctx->tail_band = value;

@@ -32,6 +32,7 @@ ap.add_argument("--b", type=int, default=1024)
 ap.add_argument("--fuse", type=int, nargs="+", default=[0, 4])
 ap.add_argument("--tail", type=int, nargs="+", default=[-1])
 ap.add_argument("--band", type=int, nargs="+", default=[2048])
+ap.add_argument("--tail-fuse", type=int, nargs="+", default=[1])
 ap.add_argument("--reps", type=int, default=2)
 ap.add_argument("--no-e2e", action="store_true")
 args = ap.parse_args()
@@ -63,9 +64,10 @@ for fuse in args.fuse:
     print(json.dumps({"fuse": fuse, "mode": "resident", "runs": res}), flush=True)
     if args.no_e2e:
         continue
-    for tail, band in [(t, bd) for t in args.tail for bd in args.band]:
+    for tail, band, tf in [(t, bd, tf) for t in args.tail for bd in args.band for tf in args.tail_fuse]:
         ctx.set_option("e2e_tail", tail)
         ctx.set_option("tail_band", band)
+        ctx.set_option("tail_fuse", tf)
         out = []
         for i in range(args.reps + 1):
             torch.cuda.synchronize()
@@ -74,5 +76,5 @@ for fuse in args.fuse:
             w = time.perf_counter() - t0
             if i:
                 out.append(stats_dict(st, w))
-        print(json.dumps({"fuse": fuse, "tail": tail, "band": band, "mode": "pmm_run", "runs": out}), flush=True)
+        print(json.dumps({"fuse": fuse, "tail": tail, "band": band, "tail_fuse": tf, "mode": "pmm_run", "runs": out}), flush=True)
 ctx.close()

@@ -22,9 +22,10 @@ def _cuda():
     yield
 
 
+@pytest.mark.parametrize("tail_fuse", [1, 0])
 @pytest.mark.parametrize("tail", [-1, 0, 1, 3, 16])
 @pytest.mark.parametrize("p", [1, 3])
-def test_run_with_tail_parity(tail, p):
+def test_run_with_tail_parity(tail, p, tail_fuse):
     N, b = 2304, 96                  # n = 24 pivots, fused groups of 8 (K = 768); rects > 2048 rows: 2+ bands
     n = N // b
     rects = pkg.colpart_arrange(n, [n * n - 100 * (p - 1)] + [100] * (p - 1))
@@ -33,13 +34,40 @@ def test_run_with_tail_parity(tail, p):
     C = np.full((N, N), np.nan, np.float32)
     with pkg.Context.local([0] * p) as ctx:
         ctx.set_option("e2e_tail", tail)
+        ctx.set_option("tail_fuse", tail_fuse)
         st = ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
         assert st.updates >= 1
     assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
 
 
+@pytest.mark.parametrize("scheme", [pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])
+def test_fused_tail_common_scale_over_groups(scheme):
+    """Fused tail: every row / column takes ONE F16X3 scale over all tail pivots
+    (maxima merged across groups and holders).  Block-columns of A and
+    block-rows of B scaled by 2^(+-6): a scale taken from one group alone
+    would overflow fp16 on another (|x| 2^s > 65504).  (A spread of 2^24 along
+    K would push the small values' lo halves into fp16 subnormals: DESIGN.md
+    Q15, the limit of one scale per row.)"""
+    N, b = 1536, 64
+    n = N // b
+    rects = pkg.colpart_arrange(n, [300, 160, 116])   # 3 devices, A slices pulled in pieces
+    A = synth.rect(3, N, 0, 0, N, N)
+    B = synth.rect(4, N, 0, 0, N, N)
+    for k in range(n):
+        A[:, k * b:(k + 1) * b] *= np.float32(2.0 ** (6 * ((k % 3) - 1)))
+        B[k * b:(k + 1) * b, :] *= np.float32(2.0 ** (-6 * ((k % 3) - 1)))
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0] * 3) as ctx:
+        ctx.set_option("f32_scheme", scheme)
+        ctx.set_option("fuse", 2)
+        ctx.set_option("e2e_tail", 6)
+        ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+    assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+@pytest.mark.parametrize("tail_fuse", [1, 0])
 @pytest.mark.parametrize("fuse", [1, 2])
-def test_tail_integer_exact_mixed_ooc(fuse):
+def test_tail_integer_exact_mixed_ooc(fuse, tail_fuse):
     N, b = 1536, 128
     n = N // b
     rects = pkg.colpart_arrange(n, [80, 40, 24])
@@ -48,6 +76,7 @@ def test_tail_integer_exact_mixed_ooc(fuse):
     C = np.full((N, N), np.nan, np.float32)
     with pkg.Context.local([0, 0, 0]) as ctx:
         ctx.set_option("fuse", fuse)
+        ctx.set_option("tail_fuse", tail_fuse)
         ctx.set_option("e2e_tail", 4)
         ctx.set_device_option(1, "c_cap_bytes", 1)   # device 1 out of core: no tail, copied after
         st = ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
