@@ -157,6 +157,114 @@ def arrange(n: int, d: Sequence[int]) -> List[Tuple[int, int, int, int, int]]:
     return rects
 
 
+def arrange_fpm(n: int, d: Sequence[int], models: Sequence[Model]) -> List[Tuple[int, int, int, int, int]]:
+    """Column-based arrangement whose integer widths and heights are chosen on the
+    FPMs (reading Q25; SURVEY §8(f) NEXT-4 "in-column FPM re-partition").
+
+    P:9: high performance "can be achieved when all processors complete their
+    work within the same time"; rectangles "as square as possible,
+    minimising the total volume of communications", with areas given by the
+    speed functions.  arrange() rounds the continuous quotas to integers, which
+    leaves a rounding imbalance (e.g. 132 vs 128 blocks at n = 32, p = 8).  Here
+    the equal-time condition decides the integers directly:
+
+      1. sort devices by (-d_i, i); devices with d_i = 0 get empty rectangles;
+      2. for every split of that order into consecutive columns:
+           column time T_j(w): heights h_i >= 0, sum n, given one row at a time
+             from zero to the device (position m in the column) minimising
+             (t_i((h_i + 1) w), m); T_j(w) = max_i t_i(h_i w)  (t(0) = 0);
+           widths w_j >= 0, sum n, given one column of blocks at a time from
+             zero to the column minimising (T_j(w_j + 1), j);
+           makespan = max_j T_j(w_j);
+           cost = sum over rectangles of positive area of (h_i + w_j);
+      3. choose min by (makespan, cost, #columns, tuple of column sizes);
+      4. columns of positive width left to right, numbered 0, 1, ...; devices
+         top to bottom in sorted order; a device left with zero area gets the
+         empty rectangle (-1, 0, 0, 0, 0) (reading Q11).
+
+    For non-decreasing times both greedy steps are min-max optimal (the
+    discrete equal-time solution of P:9 on the column's rows, then on the
+    columns' widths), and the family contains arrange()'s rounding, so the
+    makespan is never above arrange()'s.
+    """
+    p = len(d)
+    if sum(d) != n * n:
+        raise ValueError("sum(d) != n*n")
+    order = sorted(range(p), key=lambda i: (-d[i], i))
+    active = [i for i in order if d[i] > 0]
+    q = len(active)
+
+    def heights(g, w):
+        h = [0] * len(g)
+        for _ in range(n):
+            best_m = -1
+            best_t = 0.0
+            for m in range(len(g)):
+                t = time(models[g[m]], (h[m] + 1) * w)
+                if best_m < 0 or t < best_t:
+                    best_m, best_t = m, t
+            h[best_m] += 1
+        return h, max(time(models[g[m]], h[m] * w) for m in range(len(g)))
+
+    col_time = {}   # (first, last, w) -> T_j(w): plain memo, no change to the definition
+
+    def T(g, first, w):
+        key = (first, len(g), w)
+        if key not in col_time:
+            col_time[key] = heights(g, w)[1]
+        return col_time[key]
+
+    best_key = None
+    best = None
+    for mask in range(1 << (q - 1)):
+        groups, starts = [], []
+        cur, start = [active[0]], 0
+        for pos in range(1, q):
+            if mask & (1 << (pos - 1)):
+                groups.append(cur)
+                starts.append(start)
+                cur, start = [], pos
+            cur.append(active[pos])
+        groups.append(cur)
+        starts.append(start)
+        c = len(groups)
+        w = [0] * c
+        for _ in range(n):
+            best_j = -1
+            best_t = 0.0
+            for j in range(c):
+                t = T(groups[j], starts[j], w[j] + 1)
+                if best_j < 0 or t < best_t:
+                    best_j, best_t = j, t
+            w[best_j] += 1
+        makespan = max(T(groups[j], starts[j], w[j]) for j in range(c))
+        cost = 0
+        hs = []
+        for j in range(c):
+            h = heights(groups[j], w[j])[0]
+            hs.append(h)
+            cost += sum(x + w[j] for x in h if x * w[j] > 0)
+        key = (makespan, cost, c, tuple(len(g) for g in groups))
+        if best_key is None or key < best_key:
+            best_key, best = key, (groups, w, hs)
+
+    groups, w, hs = best
+    rects = [(-1, 0, 0, 0, 0)] * p
+    col0 = 0
+    col = 0
+    for j, g in enumerate(groups):
+        if w[j] == 0:
+            continue
+        row0 = 0
+        for i, h in zip(g, hs[j]):
+            if h > 0:
+                rects[i] = (col, row0, col0, h, w[j])
+            row0 += h
+        col0 += w[j]
+        col += 1
+    return rects
+
+
 def _largest_remainder(numerators: Sequence[int], denominator: int, total: int) -> List[int]:
     """Round quotas numerators[k] / denominator to integers summing to ``total``
     (Hamilton / largest remainder): floors, then +1 to the largest remainders,

@@ -161,3 +161,98 @@ def test_plan_delivers_every_pivot_exactly_once():
                     continue
                 assert np.array_equal(recvA[i], A[r0 * b:(r0 + h) * b, k * b:(k + 1) * b])
                 assert np.array_equal(recvB[i], B[k * b:(k + 1) * b, c0 * b:(c0 + w) * b])
+
+
+# ------------------------------------------------------------ arrange_fpm (Q25)
+import itertools
+
+import synth
+
+
+def _compositions(total, k):
+    """All k-tuples of integers >= 0 summing to total."""
+    if k == 1:
+        yield (total,)
+        return
+    for first in range(0, total + 1):
+        for rest in _compositions(total - first, k - 1):
+            yield (first,) + rest
+
+
+def _makespan(models, rects):
+    return max(fpm.time(models[i], r[3] * r[4]) for i, r in enumerate(rects) if r[3] * r[4] > 0)
+
+
+def _brute_force_min_makespan(n, d, models):
+    """Every split of the (-d_i, i) order into consecutive columns, every
+    integer width vector and every integer height vector (all >= 0)."""
+    order = [i for i in sorted(range(len(d)), key=lambda i: (-d[i], i)) if d[i] > 0]
+    q = len(order)
+    best = None
+    for mask in range(1 << (q - 1)):
+        groups, cur = [], [order[0]]
+        for pos in range(1, q):
+            if mask & (1 << (pos - 1)):
+                groups.append(cur)
+                cur = []
+            cur.append(order[pos])
+        groups.append(cur)
+        for ws in _compositions(n, len(groups)):
+            worst = 0.0
+            for g, w in zip(groups, ws):
+                col_best = min(max(fpm.time(models[i], h * w) for i, h in zip(g, hs))
+                               for hs in _compositions(n, len(g)))
+                worst = max(worst, col_best)
+            best = worst if best is None else min(best, worst)
+    return best
+
+
+def test_arrange_fpm_min_max_by_brute_force():
+    """For non-decreasing times the greedy widths / heights reach the minimum
+    makespan over every integer arrangement of the family (P:9 equal time)."""
+    rng = np.random.default_rng(25)
+    for trial in range(120):
+        n = int(rng.integers(1, 7))
+        p = int(rng.integers(1, min(4, n * n) + 1))
+        models = synth.random_models(rng, p, monotone_time=True, max_m=4)
+        d = fpm.partition(n * n, models)
+        if sum(1 for x in d if x > 0) > 3:
+            continue
+        rects = fpm.arrange_fpm(n, d, models)
+        _check_tiling(n, [r[3] * r[4] for r in rects], rects)
+        assert _makespan(models, rects) == _brute_force_min_makespan(n, d, models), (n, d, models)
+
+
+def test_arrange_fpm_never_worse_than_rounding():
+    """The same family as arrange(); its rounding is one of the candidates, so
+    with non-decreasing times the FPM-chosen integers are never slower."""
+    rng = np.random.default_rng(26)
+    for trial in range(80):
+        n = int(rng.integers(2, 24))
+        p = int(rng.integers(1, 7))
+        models = synth.random_models(rng, p, monotone_time=True, max_m=24)
+        d = fpm.partition(n * n, models)
+        r0 = fpm.arrange(n, d)
+        r1 = fpm.arrange_fpm(n, d, models)
+        _check_tiling(n, [r[3] * r[4] for r in r1], r1)
+        assert _makespan(models, r1) <= _makespan(models, r0)
+
+
+@pytest.mark.parametrize("n,p", [(32, 8), (64, 8), (48, 8), (32, 4), (48, 2)])
+def test_arrange_fpm_homogeneous_exact(n, p):
+    """Identical devices, p | n: every device gets exactly n^2 / p blocks
+    (arrange() leaves 132 / 128 at n = 32, p = 8 and 528 / 512 at n = 64)."""
+    models = [([1], [1.0])] * p
+    d = fpm.partition(n * n, models)
+    rects = fpm.arrange_fpm(n, d, models)
+    _check_tiling(n, d, rects)
+    assert all(r[3] * r[4] == n * n // p for r in rects)
+    assert rects == fpm.arrange_fpm(n, d, models)
+
+
+def test_arrange_fpm_zero_areas_and_single_device():
+    models = [([1], [1.0]), ([1], [2.0]), ([1], [3.0])]
+    rects = fpm.arrange_fpm(4, [0, 16, 0], models)
+    assert rects == [(-1, 0, 0, 0, 0), (0, 0, 0, 4, 4), (-1, 0, 0, 0, 0)]
+    rects = fpm.arrange_fpm(1, [1], [([1], [1.0])])
+    assert rects == [(0, 0, 0, 1, 1)]
