@@ -23,8 +23,9 @@
  *  - The library owns everything it allocates inside a pmm_ctx (device
  *    buffers, streams, events, IPC mappings, NCCL communicators); all of it is
  *    released by pmm_destroy.
- *  - fpm_partition, colpart_arrange, colpart_plan_step and fpm_model_speed are
- *    pure host functions: no GPU, no context, thread-safe.  Calls on one
+ *  - fpm_partition, colpart_arrange, colpart_arrange_fpm, colpart_plan_step
+ *    and fpm_model_speed are pure host functions: no GPU, no context,
+ *    thread-safe.  Calls on one
  *    pmm_ctx must be serialised by the caller.
  */
 #ifndef FPMPMM_H
@@ -131,6 +132,25 @@ int fpm_partition(int64_t total_blocks, int32_t p, const fpm_model* models,
  * integer rounding of widths/heights.  Zero areas give empty rectangles
  * (col = -1).  Errors: FPM_EINVAL if sum d != n*n, any d < 0, n < 1. */
 int colpart_arrange(int64_t n, int32_t p, const int64_t* d, colpart_rect* rects_out);
+
+/* Column-based arrangement whose integers come from the FPMs (reading Q25 in
+ * DESIGN.md).  P:9 "all processors complete their work
+ * within the same time" applied to the integer rectangles themselves instead
+ * of rounding continuous quotas: for every split of the devices, sorted by
+ * (-d_i, i), into consecutive columns, each column's heights (sum n) and then
+ * the columns' widths (sum n) are given out one unit at a time to whichever
+ * device / column would finish it earliest under the models; the split with
+ * the smallest (predicted makespan, sum of half-perimeters, #columns, column
+ * sizes) is returned.  Removes the rounding imbalance of colpart_arrange
+ * (e.g. 132 vs 128 blocks at n = 32, p = 8 equal devices).
+ * d: p areas with sum = n*n (they fix the device order and which devices take
+ * part); models: p speed functions as for fpm_partition.  rects_out: p
+ * entries; devices left without area get (-1, 0, 0, 0, 0); columns of positive
+ * width are numbered 0.. left to right.  Cost O(q^3 n^2) model evaluations for
+ * q devices with d_i > 0.  Errors: FPM_EINVAL if sum d != n*n, any d < 0,
+ * n outside [1, 1024], p out of range, invalid model. */
+int colpart_arrange_fpm(int64_t n, int32_t p, const int64_t* d, const fpm_model* models,
+                        colpart_rect* rects_out);
 
 /* Delivery plan of iteration k ("pivot column of matrix A and pivot row
  * of matrix B are broadcast horizontally and vertically"; reading Q12).

@@ -23,7 +23,7 @@ Model = Tuple[Sequence[int], Sequence[float]]
 Rect = Tuple[int, int, int, int, int]
 
 __all__ = [
-    "fpm_model_speed", "fpm_partition", "colpart_arrange", "colpart_plan_step", "Context",
+    "fpm_model_speed", "fpm_partition", "colpart_arrange", "colpart_arrange_fpm", "colpart_plan_step", "Context",
     "fpm_sample", "pmm_run", "FpmError", "FPM_F32", "FPM_F64", "FPM_DIST_PM1", "FPM_DIST_INT",
 ]
 
@@ -53,6 +53,17 @@ def colpart_arrange(n: int, d: Sequence[int]) -> List[Rect]:
     da = (ctypes.c_int64 * p)(*[int(v) for v in d])
     out = (_lib.ColpartRect * p)()
     check(lib.colpart_arrange(int(n), p, da, out))
+    return _lib.rects_from_c(out)
+
+
+def colpart_arrange_fpm(n: int, d: Sequence[int], models: Sequence[Model]) -> List[Rect]:
+    """Column-based rectangles with integer widths / heights chosen on the FPMs
+    (min-max predicted time, then half-perimeters; include/fpmpmm.h)."""
+    p = len(d)
+    da = (ctypes.c_int64 * p)(*[int(v) for v in d])
+    arr, keep = _lib._models(models)
+    out = (_lib.ColpartRect * p)()
+    check(lib.colpart_arrange_fpm(int(n), p, da, arr, out))
     return _lib.rects_from_c(out)
 
 

@@ -84,6 +84,8 @@ _SIGS = {
     "fpm_model_speed": ([ctypes.POINTER(FpmModel), i64, ctypes.POINTER(dbl)], ctypes.c_int),
     "fpm_partition": ([i64, i32, ctypes.POINTER(FpmModel), ctypes.POINTER(i64), ctypes.POINTER(i32)], ctypes.c_int),
     "colpart_arrange": ([i64, i32, ctypes.POINTER(i64), ctypes.POINTER(ColpartRect)], ctypes.c_int),
+    "colpart_arrange_fpm": ([i64, i32, ctypes.POINTER(i64), ctypes.POINTER(FpmModel), ctypes.POINTER(ColpartRect)],
+                            ctypes.c_int),
     "colpart_plan_step": ([i64, i32, ctypes.POINTER(ColpartRect), i64, ctypes.POINTER(ColpartMove), i32,
                            ctypes.POINTER(i32), ctypes.POINTER(ColpartMove), i32, ctypes.POINTER(i32)],
                           ctypes.c_int),

@@ -281,6 +281,125 @@ void arrange(int64_t n, int p, const int64_t* d, colpart_rect* out) {
     }
 }
 
+// FPM-chosen integers for the column-based arrangement (reading Q25, SURVEY
+// NEXT-4): every consecutive split of the (-d_i, i) order into columns; per
+// column and width w the heights come from the equal-time greedy on the rows
+// (P:9), the widths from the same greedy on the columns; the split with the
+// least (makespan, half-perimeter sum, #columns, column sizes) wins.
+// Column times are memoised per (first device, devices, width): O(q^3 n^2 / 6)
+// model evaluations for q live devices.
+void arrange_fpm(int64_t n, int p, const int64_t* d, const fpm_model* models, colpart_rect* out) {
+    FPM_CHECK_ARG(n >= 1 && n <= 1024, "n = %lld out of [1, 1024] for the FPM arrangement", (long long)n);
+    FPM_CHECK_ARG(p >= 1 && p <= FPM_MAX_DEVICES, "p = %d out of [1, %d]", p, FPM_MAX_DEVICES);
+    int64_t sum = 0;
+    for (int i = 0; i < p; ++i) {
+        FPM_CHECK_ARG(d[i] >= 0, "d[%d] < 0", i);
+        sum += d[i];
+        validate_model(models[i], i);
+    }
+    FPM_CHECK_ARG(sum == n * n, "sum of areas %lld != n*n = %lld", (long long)sum, (long long)(n * n));
+
+    std::vector<int> order(p);
+    for (int i = 0; i < p; ++i) order[i] = i;
+    std::sort(order.begin(), order.end(), [&](int a, int b) { return d[a] != d[b] ? d[a] > d[b] : a < b; });
+    std::vector<int> active;
+    for (int i : order)
+        if (d[i] > 0) active.push_back(i);
+    const int q = (int)active.size();
+
+    // heights of the column active[start .. start+len) at width w (rows from zero,
+    // one at a time to the least (t((h+1) w), position)); returns the column time
+    auto heights = [&](int start, int len, int64_t w, std::vector<int64_t>& h) {
+        h.assign(len, 0);
+        for (int64_t r = 0; r < n; ++r) {
+            int best = -1;
+            double bt = 0.0;
+            for (int m = 0; m < len; ++m) {
+                const double t = model_time(models[active[start + m]], (h[m] + 1) * w);
+                if (best < 0 || t < bt) {
+                    best = m;
+                    bt = t;
+                }
+            }
+            ++h[best];
+        }
+        double mx = 0.0;
+        for (int m = 0; m < len; ++m) mx = std::max(mx, model_time(models[active[start + m]], h[m] * w));
+        return mx;
+    };
+    std::vector<double> memo((size_t)q * q * (n + 1), -1.0);
+    std::vector<int64_t> scratch;
+    auto col_time = [&](int start, int len, int64_t w) {
+        double& v = memo[((size_t)start * q + (len - 1)) * (n + 1) + w];
+        if (v < 0.0) v = heights(start, len, w, scratch);
+        return v;
+    };
+
+    bool have = false;
+    double best_ms = 0.0;
+    int64_t best_cost = 0;
+    std::vector<int> best_sizes, best_starts;
+    std::vector<int64_t> best_w;
+    for (uint32_t mask = 0; mask < (1u << (q - 1)); ++mask) {
+        std::vector<int> starts{0}, sizes;
+        for (int pos = 1; pos < q; ++pos)
+            if (mask & (1u << (pos - 1))) starts.push_back(pos);
+        for (size_t j = 0; j < starts.size(); ++j)
+            sizes.push_back((j + 1 < starts.size() ? starts[j + 1] : q) - starts[j]);
+        const int c = (int)starts.size();
+        std::vector<int64_t> w(c, 0);
+        for (int64_t step = 0; step < n; ++step) {
+            int bj = -1;
+            double bt = 0.0;
+            for (int j = 0; j < c; ++j) {
+                const double t = col_time(starts[j], sizes[j], w[j] + 1);
+                if (bj < 0 || t < bt) {
+                    bj = j;
+                    bt = t;
+                }
+            }
+            ++w[bj];
+        }
+        double ms = 0.0;
+        int64_t cost = 0;
+        for (int j = 0; j < c; ++j) {
+            ms = std::max(ms, col_time(starts[j], sizes[j], w[j]));
+            heights(starts[j], sizes[j], w[j], scratch);
+            for (int64_t h : scratch)
+                if (h * w[j] > 0) cost += h + w[j];
+        }
+        const bool better = !have || ms < best_ms ||
+                            (ms == best_ms && (cost < best_cost ||
+                                               (cost == best_cost && (c < (int)best_sizes.size() ||
+                                                                      (c == (int)best_sizes.size() &&
+                                                                       sizes < best_sizes)))));
+        if (better) {
+            have = true;
+            best_ms = ms;
+            best_cost = cost;
+            best_sizes = sizes;
+            best_starts = starts;
+            best_w = w;
+        }
+    }
+
+    for (int i = 0; i < p; ++i) out[i] = colpart_rect{-1, 0, 0, 0, 0};
+    int64_t col0 = 0;
+    int32_t col = 0;
+    for (size_t j = 0; j < best_starts.size(); ++j) {
+        if (best_w[j] == 0) continue;
+        std::vector<int64_t> h;
+        heights(best_starts[j], best_sizes[j], best_w[j], h);
+        int64_t row0 = 0;
+        for (int m = 0; m < best_sizes[j]; ++m) {
+            if (h[m] > 0) out[active[best_starts[j] + m]] = colpart_rect{col, row0, col0, h[m], best_w[j]};
+            row0 += h[m];
+        }
+        col0 += best_w[j];
+        ++col;
+    }
+}
+
 void validate_rects(int64_t n, int p, const colpart_rect* r) {
     FPM_CHECK_ARG(n >= 1 && p >= 1 && p <= FPM_MAX_DEVICES, "bad n or p");
     // columns: same col0/w for all live members; widths partition [0, n); rows
@@ -374,6 +493,14 @@ extern "C" int colpart_arrange(int64_t n, int32_t p, const int64_t* d, colpart_r
     return fpm::guarded([&] {
         FPM_CHECK_ARG(d && rects_out, "null argument");
         fpm::arrange(n, p, d, rects_out);
+    });
+}
+
+extern "C" int colpart_arrange_fpm(int64_t n, int32_t p, const int64_t* d, const fpm_model* models,
+                                  colpart_rect* rects_out) {
+    return fpm::guarded([&] {
+        FPM_CHECK_ARG(d && models && rects_out, "null argument");
+        fpm::arrange_fpm(n, p, d, models, rects_out);
     });
 }
 

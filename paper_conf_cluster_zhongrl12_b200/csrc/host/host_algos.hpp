@@ -19,6 +19,9 @@ int partition(int64_t T, int p, const fpm_model* models, int64_t* d_out);
 // Column-based arrangement ([17] P:144).
 void arrange(int64_t n, int p, const int64_t* d, colpart_rect* out);
 
+// Column-based arrangement with FPM-chosen integer widths / heights (Q25).
+void arrange_fpm(int64_t n, int p, const int64_t* d, const fpm_model* models, colpart_rect* out);
+
 // Checks that rects form a column-based tiling of the n x n grid.
 void validate_rects(int64_t n, int p, const colpart_rect* rects);
 

@@ -75,12 +75,14 @@ def c1():
             "rel_fro": og.rel_fro(C, ref), "oracle_s": t_oracle, "oracle_threads": og.num_threads()}
 
 
-def run_device_resident(N, b, caps, reps=3):
+def run_device_resident(N, b, caps, reps=3, arrange="paper"):
     p = len(caps)
     n = N // b
     sa, sb = synth.seeds_for_config(2 if N == 16384 else 4)
-    d = pkg.fpm_partition(n * n, [([1], [float(c or 148)]) for c in caps])
-    rects = pkg.colpart_arrange(n, d)
+    models = [([1], [float(c or 148)]) for c in caps]
+    d = pkg.fpm_partition(n * n, models)
+    # paper: colpart_arrange (rounded quotas); fpm: colpart_arrange_fpm (reading Q25)
+    rects = pkg.colpart_arrange(n, d) if arrange == "paper" else pkg.colpart_arrange_fpm(n, d, models)
     with pkg.Context.local([0] * p, sm_caps=caps if p > 1 else None) as ctx:
         ctx.setup(N, b, rects, pkg.FPM_F32)
         ctx.fill_synthetic(sa, sb)
@@ -93,7 +95,7 @@ def run_device_resident(N, b, caps, reps=3):
         err = sampled_parity(ctx, N, (sa, sb), rects, b)
     per = list(best.per_dev_compute_s[:p])
     live = [t for t in per if t > 0]
-    return {"N": N, "b": b, "p": p, "sm_caps": caps, "partition": d, "rects": rects,
+    return {"N": N, "b": b, "p": p, "sm_caps": caps, "arrange": arrange, "partition": d, "rects": rects,
             "t_s": best.t_compute_s, "tflops": best.gflops / 1e3, "updates": best.updates,
             "imbalance": max(live) / (sum(live) / len(live)) - 1.0, "comm_bytes": best.comm_bytes,
             "sampled_rel_fro_max": err}
@@ -103,12 +105,12 @@ def main():
     out = {"c1": c1()}
     print("c1", {k: out["c1"][k] for k in ("partition", "rel_fro", "pmm_run_wall_s", "oracle_s")}, flush=True)
     out["c3"] = []
-    for p in (1, 2, 4, 8):
+    for p, arrange in ((1, "paper"), (2, "paper"), (4, "paper"), (8, "paper"), (8, "fpm")):
         caps = [0] if p == 1 else [148 // p // 2 * 2] * p
-        r = run_device_resident(16384, 512, caps)
+        r = run_device_resident(16384, 512, caps, arrange=arrange)
         out["c3"].append(r)
-        print("c3", p, round(r["tflops"], 1), "TFLOP/s", "imb %.2f%%" % (100 * r["imbalance"]),
-              "err %.1e" % r["sampled_rel_fro_max"], flush=True)
+        print("c3", p, arrange, round(r["tflops"], 1), "TFLOP/s", "imb %.2f%%" % (100 * r["imbalance"]),
+              "err %.1e" % r["sampled_rel_fro_max"], [x[3] * x[4] for x in r["rects"]], flush=True)
     r = run_device_resident(49152, 1024, [0])
     out["c5"] = r
     print("c5", round(r["tflops"], 1), "TFLOP/s", "err %.1e" % r["sampled_rel_fro_max"], flush=True)

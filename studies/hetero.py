@@ -87,16 +87,23 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
             out.append((m[0], [s * r for s in m[1]]))
         return out
 
-    order = list(parts.items())
+    # "_arr": the same partition arranged by colpart_arrange_fpm (integer widths
+    # and heights chosen on the models, reading Q25) instead of colpart_arrange
+    order = [("fpm", parts["fpm"]), ("fpm_arr", parts["fpm"])]
+    order += [(k, v) for k, v in parts.items() if k != "fpm"]
     for it in range(insitu):
-        order.append((f"fpm_insitu{it + 1}", None))
+        order += [(f"fpm_insitu{it + 1}", None), (f"fpm_insitu{it + 1}_arr", None)]
     cur_models = models
     for name, d in order:
-        if d is None:   # in-situ corrected FPMs from the previous FPM run
+        if d is None and not name.endswith("_arr"):   # in-situ corrected FPMs from the previous FPM run
             prev = results["fpm" if name == "fpm_insitu1" else f"fpm_insitu{int(name[-1]) - 1}"]
             cur_models = corrected(cur_models, prev)
+        if d is None:
             d = pkg.fpm_partition(T, cur_models)
-        rects = pkg.colpart_arrange(n, d)
+        if name.endswith("_arr"):
+            rects = pkg.colpart_arrange_fpm(n, d, cur_models if name.startswith("fpm_insitu") else models)
+        else:
+            rects = pkg.colpart_arrange(n, d)
         ctx.setup(N, b, rects, pkg.FPM_F32)
         ctx.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
         ctx.compute()

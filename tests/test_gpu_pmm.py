@@ -117,6 +117,23 @@ def test_streamed_run_starts_with_single_pivots():
         assert np.array_equal(Ci.astype(np.float64), og.gemm(Ai, Bi)) and st.updates == 4
 
 
+@pytest.mark.parametrize("seed", [3, 4])
+def test_run_on_fpm_arrangement(seed):
+    """colpart_arrange_fpm rectangles (integers chosen on the models, Q25):
+    same exchange and update path, parity with the oracle."""
+    N, b = 1536, 64
+    n = N // b
+    models = _models(seed, 5)
+    d = pkg.fpm_partition(n * n, models)
+    rects = pkg.colpart_arrange_fpm(n, d, models)
+    assert rects == ofpm.arrange_fpm(n, d, models)
+    with pkg.Context.local([0] * 5) as ctx:
+        A, B, C, st = _run(ctx, N, b, rects, pkg.FPM_F32)
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+        A, B, C, st = _run(ctx, N, b, rects, pkg.FPM_F64)
+        assert og.rel_fro(C, og.gemm(A, B)) <= 1e-12
+
+
 def test_single_iteration_b_equals_n():
     """n = 1: one pivot, one update that overwrites C."""
     N = b = 512

@@ -168,6 +168,48 @@ def test_arrange_config_cases():
     assert pkg.colpart_arrange(48, [288] * 8) == ofpm.arrange(48, [288] * 8)
 
 
+def test_arrange_fpm_bit_exact_random():
+    """colpart_arrange_fpm vs oracle arrange_fpm (Q25): same rectangles, bit for
+    bit, for monotone and non-monotone models, with zero areas."""
+    rng = np.random.default_rng(25)
+    for trial in range(400):
+        n = int(rng.integers(1, 28))
+        p = int(rng.integers(1, min(7, n * n) + 1))
+        models = synth.random_models(rng, p, monotone_time=bool(trial % 3), max_m=20)
+        d = ofpm.partition(n * n, models) if trial % 4 else _random_d(rng, n, p)
+        if trial % 7 == 0 and p > 2:
+            d[-1] += d[0]
+            d[0] = 0
+        assert pkg.colpart_arrange_fpm(n, d, models) == ofpm.arrange_fpm(n, d, models), (n, d)
+
+
+@pytest.mark.parametrize("caps", [[30, 26, 24, 20, 16, 14, 10, 6], [144, 128, 112, 96, 80, 64, 48, 32]])
+def test_arrange_fpm_config_models(caps):
+    """c4-shaped models (8 SM-capped devices, n = 64): bit-exact, and the
+    predicted makespan never above colpart_arrange's."""
+    n = 64
+    models = _sm_capped_models(caps)
+    d = pkg.fpm_partition(n * n, models)
+    r1 = pkg.colpart_arrange_fpm(n, d, models)
+    assert r1 == ofpm.arrange_fpm(n, d, models)
+    r0 = pkg.colpart_arrange(n, d)
+    ms = lambda rs: max(ofpm.time(m, r[3] * r[4]) for m, r in zip(models, rs) if r[3] * r[4] > 0)  # noqa: E731
+    assert ms(r1) <= ms(r0)
+
+
+def test_arrange_fpm_homogeneous_and_errors():
+    m8 = [([1], [1.0])] * 8
+    r = pkg.colpart_arrange_fpm(32, [128] * 8, m8)
+    assert r == ofpm.arrange_fpm(32, [128] * 8, m8)
+    assert all(x[3] * x[4] == 128 for x in r)
+    with pytest.raises(pkg.FpmError):
+        pkg.colpart_arrange_fpm(4, [10, 5], m8[:2])          # sum != n^2
+    with pytest.raises(pkg.FpmError):
+        pkg.colpart_arrange_fpm(4, [8, 8], [([1], [1.0]), ([2, 1], [1.0, 1.0])])  # bad model
+    with pytest.raises(pkg.FpmError):
+        pkg.colpart_arrange_fpm(2048, [2048 * 2048], m8[:1])  # n too large
+
+
 # ----------------------------------------------------------------------- plan
 def test_plan_bit_exact_random():
     rng = np.random.default_rng(17)
