@@ -26,6 +26,14 @@ __device__ __forceinline__ float warp_max(float v) {
     return v;
 }
 
+// Power-of-two F16X3 scale 2^s that puts the maximum m in [2^14, 2^15).
+__device__ __forceinline__ int f16x3_shift(float m) {
+    int e = 0;
+    if (m > 0.0f) frexpf(m, &e);  // m < 2^e
+    int s = (m > 0.0f) ? 15 - e : 0;
+    return s < -126 ? -126 : (s > 127 ? 127 : s);
+}
+
 // One warp per row.  A row of the operand is nseg segments of K elements, segment
 // j at src + j * seg_stride + row * ld (the panels of nseg consecutive pivots
 // fused into one update); it is written to out + row * ld_out + j * K.
@@ -57,12 +65,7 @@ __global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ 
     if (row >= rows) return;
     const int64_t n4 = K / 4;
     const float m = given ? __uint_as_float(given[row]) : row_absmax(src, ld, seg_stride, nseg, row, K, lane);
-    int e = 0;
-    if (m > 0.0f) {
-        frexpf(m, &e);  // m < 2^e
-    }
-    int s = (m > 0.0f) ? 15 - e : 0;
-    s = s < -126 ? -126 : (s > 127 ? 127 : s);
+    const int s = f16x3_shift(m);
     const float scale = ldexpf(1.0f, s);
     if (lane == 0) inv_scale[row] = ldexpf(1.0f, -s);
     for (int j = 0; j < nseg; ++j) {
@@ -108,72 +111,78 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
 }
 
 // B pivot row (K rows x W cols, row stride ld) -> K-major operand halves of its
-// transpose (W rows x K), split as in split_rows_*.  A warp owns 32 columns
-// (lane = column, coalesced 128 B row reads) over all K rows, so no shared
-// memory is needed: the staging kernels then co-reside with the persistent
-// update kernel (which leaves < 2 KB of shared memory per SM).  Pass 1: column
-// maxima; pass 2: each lane converts its column's 8-row chunks and writes them
-// as 16 B of output row (col, k0..k0+7).
-__device__ __forceinline__ float col_absmax(const float* src, int64_t ld, int64_t K, int64_t col) {
-    float m[8] = {0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f, 0.f};
-    for (int64_t ch = 0; ch < K / 8; ++ch)
-#pragma unroll
-        for (int i = 0; i < 8; ++i) m[i] = fmaxf(m[i], fabsf(src[(ch * 8 + i) * ld + col]));
-    float mm = m[0];
-#pragma unroll
-    for (int i = 1; i < 8; ++i) mm = fmaxf(mm, m[i]);
-    return mm;
+// transpose (W rows x K, row stride ld_out), split as in split_rows_*.
+// Three launches: column maxima (colmax_tile_k), the split + transpose
+// (split_cols_t), then the inverse scales (scale_from_max_k); with `given`
+// maxima (the fused tail) the first and last are skipped.  Both main kernels
+// are spread over the whole grid of (32 columns) x (K chunks), and use no
+// shared memory: kernels with shared memory were measured NOT to co-reside with
+// the persistent update kernel (they waited for it to finish, even with the
+// max-shared carveout and ~34 KB left per SM), while these must run under it.
+// A warp reads 8 rows x 32 columns (128 B coalesced per row; lane = column),
+// each lane writes its column's 8 values as 16 B of output row `column`; the 8
+// warps of a CTA fill 128 B of each output row, merged into full sectors in L2.
+constexpr int kColTileK = 64;   // rows of B (= K of the output) per CTA: 8 warps x 8 rows
+constexpr int kColMaxRows = 256;  // rows per CTA of the maxima pass: 8 warps x 32 rows
+
+// m_bits[c] = max(m_bits[c], bits of max |src[r][c]|): each warp 32 rows of 32
+// columns, one atomicMax per column per warp.
+__global__ void __launch_bounds__(256) colmax_tile_k(const float* __restrict__ src, int64_t ld, int64_t K,
+                                                     int64_t W, unsigned* __restrict__ m_bits) {
+    const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+    const int64_t col = (int64_t)blockIdx.x * 32 + lane;
+    const int64_t r0 = (int64_t)blockIdx.y * kColMaxRows + warp * 32;
+    if (col >= W || r0 >= K) return;
+    float m = 0.0f;
+    for (int i = 0; i < 32 && r0 + i < K; ++i) m = fmaxf(m, fabsf(src[(r0 + i) * ld + col]));
+    atomicMax(m_bits + col, __float_as_uint(m));
 }
 
-// Output row `col` is written at col * ld_out (ld_out >= K: the K rows land in
-// the first K elements, so a wider fused operand can be staged in pieces).
 template <bool F16>
-__global__ void __launch_bounds__(256) split_cols_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
+__global__ void __launch_bounds__(256) split_cols_t(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
                                                     int64_t ld_out, void* __restrict__ hi, void* __restrict__ lo,
-                                                    float* __restrict__ inv_scale, const unsigned* __restrict__ given) {
-    const int lane = threadIdx.x % 32;
-    const int64_t col = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 32 + lane;
-    if (col >= W) return;
-    const int64_t nchunks = K / 8;
-    float scale = 1.0f;
+                                                    const unsigned* __restrict__ m_bits,
+                                                    float* __restrict__ inv_scale) {
+    const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
+    const int64_t col = (int64_t)blockIdx.x * 32 + lane;
+    const int64_t kk = (int64_t)blockIdx.y * kColTileK + warp * 8;
+    if (col >= W || kk >= K) return;  // K % 8 == 0: a chunk of 8 rows is all in or all out
+    float x[8];
+#pragma unroll
+    for (int i = 0; i < 8; ++i) x[i] = src[(kk + i) * ld + col];
     if constexpr (F16) {
-        const float mm = given ? __uint_as_float(given[col]) : col_absmax(src, ld, K, col);
-        int e = 0;
-        if (mm > 0.0f) frexpf(mm, &e);
-        int s = (mm > 0.0f) ? 15 - e : 0;
-        s = s < -126 ? -126 : (s > 127 ? 127 : s);
-        scale = ldexpf(1.0f, s);
-        inv_scale[col] = ldexpf(1.0f, -s);
-    }
-    for (int64_t ch = 0; ch < nchunks; ++ch) {
-        float x[8];
+        const int s = f16x3_shift(__uint_as_float(m_bits[col]));
+        const float scale = ldexpf(1.0f, s);
+        if (inv_scale != nullptr && kk == 0) inv_scale[col] = ldexpf(1.0f, -s);
+        __align__(16) __half h[8], l[8];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) x[i] = src[(ch * 8 + i) * ld + col];
-        if constexpr (F16) {
-            __align__(16) __half h[8], l[8];
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                const float xs = x[i] * scale;
-                h[i] = __float2half_rn(xs);
-                l[i] = __float2half_rn(xs - __half2float(h[i]));
-            }
-            *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + col * ld_out + ch * 8) = *reinterpret_cast<uint4*>(h);
-            *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + col * ld_out + ch * 8) = *reinterpret_cast<uint4*>(l);
-        } else {
-            __align__(16) float h[8], l[8];
-#pragma unroll
-            for (int i = 0; i < 8; ++i) {
-                h[i] = tf32_rna(x[i]);
-                l[i] = tf32_rna(x[i] - h[i]);
-            }
-            float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + col * ld_out + ch * 8);
-            float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + col * ld_out + ch * 8);
-            hp[0] = *reinterpret_cast<float4*>(h);
-            hp[1] = *reinterpret_cast<float4*>(h + 4);
-            lp[0] = *reinterpret_cast<float4*>(l);
-            lp[1] = *reinterpret_cast<float4*>(l + 4);
+        for (int i = 0; i < 8; ++i) {
+            const float xs = x[i] * scale;
+            h[i] = __float2half_rn(xs);
+            l[i] = __float2half_rn(xs - __half2float(h[i]));
         }
+        *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + col * ld_out + kk) = *reinterpret_cast<uint4*>(h);
+        *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + col * ld_out + kk) = *reinterpret_cast<uint4*>(l);
+    } else {
+        __align__(16) float h[8], l[8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            h[i] = tf32_rna(x[i]);
+            l[i] = tf32_rna(x[i] - h[i]);
+        }
+        float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + col * ld_out + kk);
+        float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + col * ld_out + kk);
+        hp[0] = *reinterpret_cast<float4*>(h);
+        hp[1] = *reinterpret_cast<float4*>(h + 4);
+        lp[0] = *reinterpret_cast<float4*>(l);
+        lp[1] = *reinterpret_cast<float4*>(l + 4);
     }
+}
+
+// In place: maxima bits -> inverse F16X3 scales 2^-s (the buffer is inv_scale).
+__global__ void __launch_bounds__(256) scale_from_max_k(float* __restrict__ buf, int64_t W) {
+    const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+    if (c < W) buf[c] = ldexpf(1.0f, -f16x3_shift(buf[c]));
 }
 
 // Maxima |x| of the rows of a (fused) panel / the columns of a block-row, merged
@@ -186,13 +195,6 @@ __global__ void __launch_bounds__(256) rowmax_k(const float* __restrict__ src, i
     if (row >= rows) return;
     const float m = row_absmax(src, ld, seg_stride, nseg, row, K, lane);
     if (lane == 0) atomicMax(m_bits + row, __float_as_uint(m));
-}
-
-__global__ void __launch_bounds__(256) colmax_k(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
-                                                unsigned* __restrict__ m_bits) {
-    const int64_t col = ((int64_t)blockIdx.x * 8 + threadIdx.x / 32) * 32 + threadIdx.x % 32;
-    if (col >= W) return;
-    atomicMax(m_bits + col, __float_as_uint(col_absmax(src, ld, K, col)));
 }
 
 template <class T>
@@ -414,12 +416,22 @@ void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, Split
     if (K <= 0 || W <= 0) return;
     if (ld_out < 0) ld_out = K;
     FPM_CHECK_ARG(K % 8 == 0 && ld_out % 8 == 0 && ld_out >= K, "split_cols: K, ld_out multiples of 8, ld_out >= K");
-    const unsigned blocks = (unsigned)((W + 255) / 256);  // 8 warps x 32 columns per block
+    const dim3 grid((unsigned)((W + 31) / 32), (unsigned)((K + kColTileK - 1) / kColTileK));
     if (s == SplitScheme::F16X3) {
         FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
-        split_cols_k<true><<<blocks, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, inv_scale, given_max);
+        if (given_max) {
+            split_cols_t<true><<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, given_max, inv_scale);
+        } else {  // maxima into inv_scale (as bits), split, then bits -> inverse scales in place
+            unsigned* bits = reinterpret_cast<unsigned*>(inv_scale);
+            const cudaError_t e = cudaMemsetAsync(bits, 0, (size_t)W * sizeof(unsigned), st);
+            if (e != cudaSuccess) fail(FPM_ECUDA, "split_cols memset: %s", cudaGetErrorString(e));
+            launch_colmax(src, ld, K, W, bits, st);
+            split_cols_t<true><<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, bits, nullptr);
+            check_launch("split_cols");
+            scale_from_max_k<<<(unsigned)((W + 255) / 256), 256, 0, st>>>(inv_scale, W);
+        }
     } else {
-        split_cols_k<false><<<blocks, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, inv_scale, nullptr);
+        split_cols_t<false><<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, nullptr, nullptr);
     }
     check_launch("split_cols");
 }
@@ -435,7 +447,8 @@ void launch_rowmax_seg(const float* src, int64_t ld, int64_t seg_stride, int nse
 void launch_colmax(const float* src, int64_t ld, int64_t K, int64_t W, unsigned* m_bits, cudaStream_t st) {
     if (K <= 0 || W <= 0) return;
     FPM_CHECK_ARG(K % 8 == 0, "colmax: K must be a multiple of 8");
-    colmax_k<<<(unsigned)((W + 255) / 256), 256, 0, st>>>(src, ld, K, W, m_bits);
+    const dim3 grid((unsigned)((W + 31) / 32), (unsigned)((K + kColMaxRows - 1) / kColMaxRows));
+    colmax_tile_k<<<grid, 256, 0, st>>>(src, ld, K, W, m_bits);
     check_launch("colmax");
 }
 
