@@ -821,7 +821,8 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
             const size_t ko = (size_t)tp.k_off * op;
             const unsigned* ga = (tp.phase == 2 && f16) ? d.tmax_a : nullptr;
             const unsigned* gb = (tp.phase == 2 && f16) ? d.tmax_b : nullptr;
-            d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + 1;
+            // B rows: maxima, split, scales (F16X3 without given maxima) or the split alone
+            d.launches += (a_src ? 1 : (int64_t)a_pieces.size()) + ((f16 && gb == nullptr) ? 3 : 1);
             if (a_src) {  // own or received panels: f consecutive H x b panels
                 launch_split_rows_seg(static_cast<const float*>(a_src), b, d.H * b, f, d.H, b, ld_out, sch,
                                       static_cast<char*>(d.a_hi[slot]) + ko, static_cast<char*>(d.a_lo[slot]) + ko,

@@ -134,6 +134,26 @@ def test_run_on_fpm_arrangement(seed):
         assert og.rel_fro(C, og.gemm(A, B)) <= 1e-12
 
 
+def test_kernel_launch_count():
+    """pmm_stats.kernel_launches counts every library kernel of the k-loop: per
+    update group one A split, three B-row kernels (maxima, split, scales) for
+    F16X3 or one for TF32X3, and the update."""
+    N, b = 2048, 128
+    n = N // b
+    with pkg.Context.local([0]) as ctx:
+        ctx.set_option("fuse", 8)
+        ctx.setup(N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+        ctx.fill_synthetic(1, 2)
+        for graph in (0, 1):
+            ctx.set_option("graph", graph)
+            st = ctx.compute()
+            assert st.updates == 2 and st.kernel_launches == 2 * (1 + 3 + 1)
+        ctx.set_option("f32_scheme", pkg.SCHEME_TF32X3)
+        ctx.setup(N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+        ctx.fill_synthetic(1, 2)
+        assert ctx.compute().kernel_launches == 2 * (1 + 1 + 1)
+
+
 def test_single_iteration_b_equals_n():
     """n = 1: one pivot, one update that overwrites C."""
     N = b = 512
