@@ -263,11 +263,12 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     barrier()
     clocks = ClockSampler(local_rank)
     clocks.start()
-    step_times, upd_times, comp_times, launches, comm = [], [], [], 0, 0
+    step_times, upd_times, comp_times, own_times, launches, comm = [], [], [], [], 0, 0
     wall0 = time.perf_counter()
     for _ in range(args.steps):
         d, rects = plan()
         st = ctx.compute(zero_c=True)
+        own_times.append(st.t_compute_s)
         step_times.append(max_over_ranks(st.t_compute_s))
         upd_times.append(st.per_dev_update_s[rank])
         comp_times.append(st.per_dev_compute_s[rank])
@@ -291,6 +292,10 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     pred_t = [a / pkg.fpm_model_speed(m, a) if a > 0 else 0.0 for a, m in zip(areas, models_all)]
     live_t = [t for t in pred_t if t > 0]
     imb_pred = max(live_t) / (sum(live_t) / len(live_t)) - 1.0 if live_t else 0.0
+
+    stage = statistics.median(comp_times) - statistics.median(upd_times)
+    exposed = max(0.0, statistics.median(own_times) - statistics.median(upd_times))
+    overlap = 1.0 - exposed / stage if stage > 0 else None
 
     # ---- roofline of the dominant kernel (rank-(f b) update): algorithmic flops per
     # launch = 2 H W f b, over the launch duration (CUDA events on its stream);
@@ -343,6 +348,9 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "imbalance_pct_measured": 100.0 * imb_meas, "imbalance_pct_predicted": 100.0 * imb_pred,
                 "fpm_sample_s": t_sample, "fpm_sizes": sizes,
                 "comm_bytes_per_step": comm // max(1, args.steps),
+                # share of the exchange + staging time hidden under the updates (SURVEY §8(d) c5
+                # "broadcast/update overlap", from the CUDA events of this rank's streams)
+                "exchange_staging_overlap": overlap,
                 "wall_s_timed_region": wall,
             },
             "roofline": roofline,

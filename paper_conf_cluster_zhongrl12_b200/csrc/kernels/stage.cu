@@ -122,60 +122,85 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
 // A warp reads 8 rows x 32 columns (128 B coalesced per row; lane = column),
 // each lane writes its column's 8 values as 16 B of output row `column`; the 8
 // warps of a CTA fill 128 B of each output row, merged into full sectors in L2.
-constexpr int kColTileK = 64;   // rows of B (= K of the output) per CTA: 8 warps x 8 rows
+constexpr int kColTileK = 64;     // rows of B (= K of the output) per CTA: 8 warps x 8 rows
 constexpr int kColMaxRows = 256;  // rows per CTA of the maxima pass: 8 warps x 32 rows
+constexpr int kColsPerCta = 128;  // 32 lanes x 4 columns (float4 loads)
 
-// m_bits[c] = max(m_bits[c], bits of max |src[r][c]|): each warp 32 rows of 32
-// columns, one atomicMax per column per warp.
+// m_bits[c] = max(m_bits[c], bits of max |src[r][c]|): each warp 32 rows of 128
+// columns (a float4 per lane and row), one atomicMax per column per warp.
 __global__ void __launch_bounds__(256) colmax_tile_k(const float* __restrict__ src, int64_t ld, int64_t K,
                                                      int64_t W, unsigned* __restrict__ m_bits) {
     const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
-    const int64_t col = (int64_t)blockIdx.x * 32 + lane;
+    const int64_t col = (int64_t)blockIdx.x * kColsPerCta + 4 * lane;
     const int64_t r0 = (int64_t)blockIdx.y * kColMaxRows + warp * 32;
-    if (col >= W || r0 >= K) return;
-    float m = 0.0f;
-    for (int i = 0; i < 32 && r0 + i < K; ++i) m = fmaxf(m, fabsf(src[(r0 + i) * ld + col]));
-    atomicMax(m_bits + col, __float_as_uint(m));
+    if (col >= W || r0 >= K) return;  // W % 4 == 0: four columns are all in or all out
+    float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
+    const int rows = K - r0 < 32 ? (int)(K - r0) : 32;
+#pragma unroll 8
+    for (int i = 0; i < rows; ++i) {
+        const float4 v = *reinterpret_cast<const float4*>(src + (r0 + i) * ld + col);
+        m.x = fmaxf(m.x, fabsf(v.x));
+        m.y = fmaxf(m.y, fabsf(v.y));
+        m.z = fmaxf(m.z, fabsf(v.z));
+        m.w = fmaxf(m.w, fabsf(v.w));
+    }
+    atomicMax(m_bits + col + 0, __float_as_uint(m.x));
+    atomicMax(m_bits + col + 1, __float_as_uint(m.y));
+    atomicMax(m_bits + col + 2, __float_as_uint(m.z));
+    atomicMax(m_bits + col + 3, __float_as_uint(m.w));
 }
 
+// Split + transpose: warp w of a CTA reads rows kk .. kk+7 (kk = k0 + 8 w) of 128
+// columns (a float4 per lane and row); each lane then writes, for each of its 4
+// columns, the 8 values as 16 B of output row `column`.
 template <bool F16>
 __global__ void __launch_bounds__(256) split_cols_t(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
                                                     int64_t ld_out, void* __restrict__ hi, void* __restrict__ lo,
                                                     const unsigned* __restrict__ m_bits,
                                                     float* __restrict__ inv_scale) {
     const int lane = threadIdx.x % 32, warp = threadIdx.x / 32;
-    const int64_t col = (int64_t)blockIdx.x * 32 + lane;
+    const int64_t col = (int64_t)blockIdx.x * kColsPerCta + 4 * lane;
     const int64_t kk = (int64_t)blockIdx.y * kColTileK + warp * 8;
-    if (col >= W || kk >= K) return;  // K % 8 == 0: a chunk of 8 rows is all in or all out
-    float x[8];
+    if (col >= W || kk >= K) return;  // K % 8 == 0, W % 4 == 0: chunks are all in or all out
+    float x[4][8];
 #pragma unroll
-    for (int i = 0; i < 8; ++i) x[i] = src[(kk + i) * ld + col];
-    if constexpr (F16) {
-        const int s = f16x3_shift(__uint_as_float(m_bits[col]));
-        const float scale = ldexpf(1.0f, s);
-        if (inv_scale != nullptr && kk == 0) inv_scale[col] = ldexpf(1.0f, -s);
-        __align__(16) __half h[8], l[8];
+    for (int i = 0; i < 8; ++i) {
+        const float4 v = *reinterpret_cast<const float4*>(src + (kk + i) * ld + col);
+        x[0][i] = v.x;
+        x[1][i] = v.y;
+        x[2][i] = v.z;
+        x[3][i] = v.w;
+    }
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            const float xs = x[i] * scale;
-            h[i] = __float2half_rn(xs);
-            l[i] = __float2half_rn(xs - __half2float(h[i]));
+    for (int c = 0; c < 4; ++c) {
+        const int64_t orow = (col + c) * ld_out + kk;
+        if constexpr (F16) {
+            const int s = f16x3_shift(__uint_as_float(m_bits[col + c]));
+            const float scale = ldexpf(1.0f, s);
+            if (inv_scale != nullptr && kk == 0) inv_scale[col + c] = ldexpf(1.0f, -s);
+            __align__(16) __half h[8], l[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                const float xs = x[c][i] * scale;
+                h[i] = __float2half_rn(xs);
+                l[i] = __float2half_rn(xs - __half2float(h[i]));
+            }
+            *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + orow) = *reinterpret_cast<uint4*>(h);
+            *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + orow) = *reinterpret_cast<uint4*>(l);
+        } else {
+            __align__(16) float h[8], l[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) {
+                h[i] = tf32_rna(x[c][i]);
+                l[i] = tf32_rna(x[c][i] - h[i]);
+            }
+            float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + orow);
+            float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + orow);
+            hp[0] = *reinterpret_cast<float4*>(h);
+            hp[1] = *reinterpret_cast<float4*>(h + 4);
+            lp[0] = *reinterpret_cast<float4*>(l);
+            lp[1] = *reinterpret_cast<float4*>(l + 4);
         }
-        *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + col * ld_out + kk) = *reinterpret_cast<uint4*>(h);
-        *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + col * ld_out + kk) = *reinterpret_cast<uint4*>(l);
-    } else {
-        __align__(16) float h[8], l[8];
-#pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            h[i] = tf32_rna(x[i]);
-            l[i] = tf32_rna(x[i] - h[i]);
-        }
-        float4* hp = reinterpret_cast<float4*>(static_cast<float*>(hi) + col * ld_out + kk);
-        float4* lp = reinterpret_cast<float4*>(static_cast<float*>(lo) + col * ld_out + kk);
-        hp[0] = *reinterpret_cast<float4*>(h);
-        hp[1] = *reinterpret_cast<float4*>(h + 4);
-        lp[0] = *reinterpret_cast<float4*>(l);
-        lp[1] = *reinterpret_cast<float4*>(l + 4);
     }
 }
 
@@ -416,7 +441,9 @@ void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, Split
     if (K <= 0 || W <= 0) return;
     if (ld_out < 0) ld_out = K;
     FPM_CHECK_ARG(K % 8 == 0 && ld_out % 8 == 0 && ld_out >= K, "split_cols: K, ld_out multiples of 8, ld_out >= K");
-    const dim3 grid((unsigned)((W + 31) / 32), (unsigned)((K + kColTileK - 1) / kColTileK));
+    FPM_CHECK_ARG(W % 4 == 0 && ld % 4 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0,
+                  "split_cols: W and ld multiples of 4, src 16-byte aligned");
+    const dim3 grid((unsigned)((W + kColsPerCta - 1) / kColsPerCta), (unsigned)((K + kColTileK - 1) / kColTileK));
     if (s == SplitScheme::F16X3) {
         FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
         if (given_max) {
@@ -446,8 +473,9 @@ void launch_rowmax_seg(const float* src, int64_t ld, int64_t seg_stride, int nse
 
 void launch_colmax(const float* src, int64_t ld, int64_t K, int64_t W, unsigned* m_bits, cudaStream_t st) {
     if (K <= 0 || W <= 0) return;
-    FPM_CHECK_ARG(K % 8 == 0, "colmax: K must be a multiple of 8");
-    const dim3 grid((unsigned)((W + 31) / 32), (unsigned)((K + kColMaxRows - 1) / kColMaxRows));
+    FPM_CHECK_ARG(K % 8 == 0 && W % 4 == 0 && ld % 4 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0,
+                  "colmax: K multiple of 8, W and ld multiples of 4, src 16-byte aligned");
+    const dim3 grid((unsigned)((W + kColsPerCta - 1) / kColsPerCta), (unsigned)((K + kColMaxRows - 1) / kColMaxRows));
     colmax_tile_k<<<grid, 256, 0, st>>>(src, ld, K, W, m_bits);
     check_launch("colmax");
 }

@@ -95,7 +95,7 @@ def test_split_rows_f16x3_bit_exact_vs_numpy():
     assert np.array_equal(inv.cpu().numpy(), s)
 
 
-@pytest.mark.parametrize("K,W,ld", [(64, 256, 256), (512, 1000, 1004), (32, 4, 8)])
+@pytest.mark.parametrize("K,W,ld", [(64, 256, 256), (512, 1000, 1004), (32, 4, 8), (520, 388, 392)])
 def test_split_cols_bit_exact_vs_numpy(K, W, ld):
     """B pivot row K x W -> split halves of its transpose (W x K)."""
     src = _scaled_rows(W, K, 6).T.copy()           # K x W with per-column scales
