@@ -1011,6 +1011,29 @@ void ensure_fused_tail(pmm_ctx* ctx, Device& d, int gt) {
 // stream -- band j's copy overlaps the updates of bands j+1.., so only the last
 // band's copy is exposed.  The same sums in the same order per element as the
 // group-major loop (each element still receives the groups in k order).
+// Row bands of the tail: whole bands of `band` rows (multiples of 256, the
+// CTA-pair tile rows), the last one halved down to 256 rows (band, ..., band/2,
+// band/4, ..., 256, 256) so the copy left exposed after the last update is
+// small; the copy stream keeps pace with the updates, so earlier bands' copies
+// finish under the following bands.
+std::vector<std::pair<int64_t, int64_t>> tail_bands(int64_t H, int64_t band) {
+    std::vector<std::pair<int64_t, int64_t>> out;
+    int64_t r0 = 0;
+    while (H - r0 > band) {
+        out.push_back({r0, band});
+        r0 += band;
+    }
+    int64_t rest = H - r0;  // <= band: halve it while the halves stay >= 256 rows
+    while (rest > 512) {
+        const int64_t half = (rest / 2 + 255) / 256 * 256;
+        out.push_back({r0, half});
+        r0 += half;
+        rest -= half;
+    }
+    if (rest > 0) out.push_back({r0, rest});
+    return out;
+}
+
 void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
     CU(cudaSetDevice(d.cuda_dev));
     const bool fused = d.tail_fused_run;
@@ -1025,12 +1048,11 @@ void issue_tail(pmm_ctx* ctx, Device& d, int g0, int L, const HostDst& out) {
         fa = f32_args(ctx, d, g0, kFusedSlot);
         fa.K = d.tail_K;
     }
-    const int64_t band = std::min<int64_t>(d.H, ctx->tail_band);  // whole CTA-pair tile rows
     const int64_t b = ctx->b;
     const int64_t R0 = d.rect.row0 * b - out.row_base, C0 = d.rect.col0 * b - out.col_base;
     float* C = static_cast<float*>(d.C);
-    for (int64_t r0 = 0; r0 < d.H; r0 += band) {
-        const int64_t m = std::min(band, d.H - r0);
+    for (const auto& bd : tail_bands(d.H, ctx->tail_band)) {
+        const int64_t r0 = bd.first, m = bd.second;
         if (fused) {
             launch_update_f32(band_args(fa, r0, m, C + (size_t)r0 * d.W), d.s_comp);
             d.launches += 1;
