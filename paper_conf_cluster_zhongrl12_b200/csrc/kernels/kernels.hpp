@@ -72,9 +72,12 @@ void launch_transpose_f32(const float* src, int64_t ld, int64_t rows, int64_t co
 void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t cols, double* dst,
                           cudaStream_t st);
 
-// C (M x Nc, ldc) += A (M x K, lda) . Bt^T, Bt (Nc x K), FP64 on DMMA.
+// C (M x Nc, ldc) += A (M x K, lda) . Bt^T, Bt (Nc x K), FP64 on DMMA.  With
+// seg > 0, A is K / seg panels of M x seg (row stride lda) seg_stride elements
+// apart (the pivots of a fused group); seg <= 0: one M x K matrix.
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                       int64_t K, int64_t ldc, bool accumulate, int num_sms, cudaStream_t st);
+                       int64_t K, int64_t ldc, bool accumulate, int num_sms, cudaStream_t st, int64_t seg = 0,
+                       int64_t seg_stride = 0);
 
 // Seeded counter-based generator (same bits as synth/__init__.py).
 void launch_fill_synthetic(void* dst, bool f64, int64_t ld, uint64_t seed, int64_t N, int64_t r0, int64_t c0,

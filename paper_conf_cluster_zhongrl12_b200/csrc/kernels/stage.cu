@@ -284,10 +284,13 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool va
 
 __device__ __forceinline__ void group_bar(int id) { asm volatile("bar.sync %0, 256;" ::"r"(id) : "memory"); }
 
-__global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict__ A, int64_t lda,
-                                                       const double* __restrict__ Bt, double* __restrict__ C,
-                                                       int64_t M, int64_t Nc, int64_t K, int64_t ldc,
-                                                       int accumulate) {
+// A may be segmented along K (fused pivots, each pivot's H x b panel stored on
+// its own): element (r, k) at A + (k / seg) * seg_stride + r * lda + k % seg.
+// seg is even, so the two consecutive k of a 16-byte copy share a segment.
+__global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict__ A, int64_t lda, int64_t seg,
+                                                       int64_t seg_stride, const double* __restrict__ Bt,
+                                                       double* __restrict__ C, int64_t M, int64_t Nc, int64_t K,
+                                                       int64_t ldc, int accumulate) {
     extern __shared__ double sm64[];
     const int grp = threadIdx.x / 256, gtid = threadIdx.x % 256;
     double* As = sm64 + grp * F64_GROUP_DOUBLES;       // [ST][BM][LD]
@@ -318,8 +321,8 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
                 const bool ka = gk < K;  // K even: a 2-element chunk is all in or all out
                 if (isA) {
                     const int64_t gm = m0 + r;
-                    cp_async16(As + (slot_l * F64_BM + r) * F64_LD + c2, A + (ka && gm < M ? gm * lda + gk : 0),
-                               ka && gm < M);
+                    const int64_t off = (gk / seg) * seg_stride + gm * lda + gk % seg;
+                    cp_async16(As + (slot_l * F64_BM + r) * F64_LD + c2, A + (ka && gm < M ? off : 0), ka && gm < M);
                 } else {
                     const int64_t gn = n0 + r;
                     cp_async16(Bs + (slot_l * F64_BN + r) * F64_LD + c2, Bt + (ka && gn < Nc ? gn * K + gk : 0),
@@ -496,9 +499,15 @@ void launch_transpose_f64(const double* src, int64_t ld, int64_t rows, int64_t c
 }
 
 void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
-                       int64_t K, int64_t ldc, bool accumulate, int num_sms, cudaStream_t st) {
+                       int64_t K, int64_t ldc, bool accumulate, int num_sms, cudaStream_t st, int64_t seg,
+                       int64_t seg_stride) {
     if (M <= 0 || Nc <= 0 || K <= 0) return;
-    FPM_CHECK_ARG(K % 8 == 0 && lda % 2 == 0, "FP64 update: K % 8 == 0 and even lda required");
+    if (seg <= 0) {  // one contiguous row of K per A row
+        seg = K;
+        seg_stride = 0;
+    }
+    FPM_CHECK_ARG(K % 8 == 0 && lda % 2 == 0 && seg % 2 == 0 && seg_stride % 2 == 0 && (seg >= K || lda >= seg),
+                  "FP64 update: K % 8 == 0, even lda / seg / seg_stride, lda >= seg for segmented A");
     FPM_CHECK_ARG((reinterpret_cast<uintptr_t>(A) & 15) == 0 && (reinterpret_cast<uintptr_t>(Bt) & 15) == 0,
                   "FP64 update: A and Bt must be 16-byte aligned");
     static uint64_t attr_done = 0;  // one bit per CUDA device
@@ -513,7 +522,7 @@ void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C
     int sms = num_sms;
     if (sms <= 0) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const unsigned grid = (unsigned)std::min<int64_t>((tiles + 1) / 2, std::max(1, sms));  // 1 CTA (2 tile groups) per SM
-    update_f64_k<<<grid, 512, F64_SMEM, st>>>(A, lda, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
+    update_f64_k<<<grid, 512, F64_SMEM, st>>>(A, lda, seg, seg_stride, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
     check_launch("update_f64");
 }
 

@@ -503,7 +503,7 @@ const void* src_B(pmm_ctx* ctx, int q) {
 // (measured on B200: f = 2 at b = 1024 gives 419 vs 392 TFLOP/s unfused and
 // beats f = 3, 4; at b = 512, f = 2..8 give 404-406 vs 332 unfused).
 int fuse_factor(pmm_ctx* ctx, fpm_dtype dt, int64_t b) {
-    if (dt != FPM_F32) return 1;
+    (void)dt;  // FP32 and FP64 alike (FP64: the update reads the f panels as K segments)
     if (ctx->fuse > 0) return ctx->fuse;
     return (int)std::max<int64_t>(1, std::min<int64_t>(8, 2048 / b));
 }
@@ -522,7 +522,7 @@ void alloc_slot(pmm_ctx* ctx, Device& d, int s) {
         d.a_recv[s] = dalloc(d, (size_t)d.H * fb * es);  // f panels of H x b
         d.b_recv[s] = dalloc(d, fb * d.W * es);          // f block-rows of b x W
     }
-    if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * ctx->b * es);
+    if (dt == FPM_F64) d.bt[s] = dalloc(d, (size_t)d.W * fb * es);  // W x f b, K-major
     if (dt == FPM_F32) {
         d.a_hi[s] = dalloc(d, (size_t)d.H * fb * op);
         d.a_lo[s] = dalloc(d, (size_t)d.H * fb * op);
@@ -840,8 +840,8 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
                               d.sb[slot], d.s_comm, ld_out, gb);
         }
     } else {
-        d.a_op[slot] = a_src;
-        launch_transpose_f64(static_cast<const double*>(b_src), d.W, b, d.W, static_cast<double*>(d.bt[slot]),
+        d.a_op[slot] = a_src;  // f panels of H x b, H b apart (own block-columns or the receive buffer)
+        launch_transpose_f64(static_cast<const double*>(b_src), d.W, fb, d.W, static_cast<double*>(d.bt[slot]),
                              d.s_comm);
         d.launches += 1;
     }
@@ -915,20 +915,24 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
             launch_update_f32(a, d.s_comp);
             d.launches += 1;
         }
-    } else if (d.ooc) {
-        const double* aop = static_cast<const double*>(d.a_op[slot]);
-        const int64_t b = ctx->b;
-        d.launches += banded_update(d.bp, d.ring, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, bc, d.s_comp,
-                                    [&](int64_t r0, int64_t m, void* band) {
-                                        launch_update_f64(aop + (size_t)r0 * b, b,
-                                                          static_cast<const double*>(d.bt[slot]),
-                                                          static_cast<double*>(band), m, d.W, b, d.W, k0 != 0,
-                                                          d.num_sms, d.s_comp);
-                                    });
     } else {
-        launch_update_f64(static_cast<const double*>(d.a_op[slot]), ctx->b, static_cast<const double*>(d.bt[slot]),
-                          static_cast<double*>(d.C), d.H, d.W, ctx->b, d.W, k0 != 0, d.num_sms, d.s_comp);
-        d.launches += 1;
+        // FP64: the group's f panels (H x b each, H b apart) as K segments of one
+        // rank-(f b) update against the transposed block-rows (W x f b)
+        const double* aop = static_cast<const double*>(d.a_op[slot]);
+        const int64_t b = ctx->b, K = (int64_t)f * b;
+        if (d.ooc) {
+            d.launches += banded_update(d.bp, d.ring, reinterpret_cast<char*>(d.hC), d.H, (size_t)d.W * 8, bc,
+                                        d.s_comp, [&](int64_t r0, int64_t m, void* band) {
+                                            launch_update_f64(aop + (size_t)r0 * b, b,
+                                                              static_cast<const double*>(d.bt[slot]),
+                                                              static_cast<double*>(band), m, d.W, K, d.W, k0 != 0,
+                                                              d.num_sms, d.s_comp, b, d.H * b);
+                                        });
+        } else {
+            launch_update_f64(aop, b, static_cast<const double*>(d.bt[slot]), static_cast<double*>(d.C), d.H, d.W, K,
+                              d.W, k0 != 0, d.num_sms, d.s_comp, b, d.H * b);
+            d.launches += 1;
+        }
     }
     rec_t(d.ev_upd1[g], d.s_comp);
     CU(cudaEventRecord(d.ev_free[slot], d.s_comp));
@@ -1576,7 +1580,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         }
         s.Ap = dalloc(s.mem, (size_t)L * fb * es);
         s.Bp = dalloc(s.mem, (size_t)fb * L * es);
-        s.Bt = dalloc(s.mem, (size_t)L * b * es);
+        s.Bt = dalloc(s.mem, (size_t)L * fb * es);
         if (dt == FPM_F32) {
             s.ah = dalloc(s.mem, (size_t)L * fb * op);
             s.al = dalloc(s.mem, (size_t)L * fb * op);
@@ -1633,18 +1637,18 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 } else {
                     launch_update_f32(a, st);
                 }
-            } else {
-                launch_transpose_f64(static_cast<const double*>(s.Bp), L, b, Lx, static_cast<double*>(s.Bt), st);
+            } else {  // FP64: the fused update of the k-loop (K = f b, A rows contiguous here)
+                launch_transpose_f64(static_cast<const double*>(s.Bp), L, fb, Lx, static_cast<double*>(s.Bt), st);
                 if (ooc) {
                     banded_update(s.mem.bp, ring_at(s.d, Lx), s.hC, Lx, (size_t)Lx * 8, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
-                                      launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * b, b,
+                                      launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * fb, fb,
                                                         static_cast<const double*>(s.Bt), static_cast<double*>(band),
-                                                        m, Lx, b, Lx, true, s.d->num_sms, st);
+                                                        m, Lx, fb, Lx, true, s.d->num_sms, st);
                                   });
                 } else {
-                    launch_update_f64(static_cast<const double*>(s.Ap), b, static_cast<const double*>(s.Bt),
-                                      static_cast<double*>(s.C), Lx, Lx, b, Lx, true, s.d->num_sms, st);
+                    launch_update_f64(static_cast<const double*>(s.Ap), fb, static_cast<const double*>(s.Bt),
+                                      static_cast<double*>(s.C), Lx, Lx, fb, Lx, true, s.d->num_sms, st);
                 }
             }
             if (ooc) bp_join(s.mem.bp, st);  // the update is done when C is back in host memory
