@@ -90,8 +90,10 @@ class ClockSampler:
                 if v.lower().startswith("active"):
                     reasons.add(nm)
         loaded = [s for s, p in zip(sms, power) if p > 200.0] or sms
+        watts = [p for p in power if p > 200.0]
         return {"sm_mhz": statistics.median(loaded) if loaded else None, "sm_max_mhz": mx,
-                "reasons": sorted(reasons), "samples": len(sms)}
+                "reasons": sorted(reasons), "samples": len(sms),
+                "power_w_median": statistics.median(watts) if watts else None}
 
 
 # ----------------------------------------------------------------- peaks
@@ -109,7 +111,7 @@ def committed_traffic(N: int, b: int, args):
     """DRAM bytes per update launch from the committed ncu capture of the same
     configuration (profiles/ncu_traffic.json), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    variant = 4 if args.kernel_variant < 0 else args.kernel_variant
+    variant = (3 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
     key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}")
     if args.gpus != 1 or not os.path.exists(path):
@@ -188,8 +190,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             c = pkg.Context.ipc(rank, world, local_rank)
         else:
             c = pkg.Context.local([local_rank])
-        if args.scheme == "tf32x3":
-            c.set_option("f32_scheme", pkg.SCHEME_TF32X3)
+        c.set_option("f32_scheme", {"f16i8": pkg.SCHEME_F16I8, "f16x3": pkg.SCHEME_F16X3,
+                                    "tf32x3": pkg.SCHEME_TF32X3}[args.scheme])
         c.set_option("cta_group", args.cta_group)
         c.set_option("raster_group", args.raster_group)
         c.set_option("l2_hint_b", args.l2_hint_b)
@@ -306,14 +308,21 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     upd_launches = st.updates
     upd_step = statistics.median(upd_times)
     achieved = 2.0 * H * W * b * n / upd_step / 1e12 if upd_step > 0 else 0.0
-    mma_per_mac = 3.0  # F16X3 and TF32X3 both issue three tensor-core products per FP32 MAC
-    dense_peak = peaks["bf16_sustained"] if args.scheme == "f16x3" else peaks["bf16_sustained"] / 2.0
+    # tensor-pipe time per FP32 MAC in units of one dense fp16 MAC: F16X3 three
+    # fp16 products; TF32X3 three tf32 products at half the fp16 rate; F16I8 one
+    # fp16 product plus one int8 product over twice the K at twice the fp16 rate
+    # (the guide's nominal int8 : fp16 = 2 : 1) = 2
+    dense_peak = peaks["bf16_sustained"] if args.scheme != "tf32x3" else peaks["bf16_sustained"] / 2.0
+    mma_per_mac = 2.0 if args.scheme == "f16i8" else 3.0
     peak = dense_peak / mma_per_mac
+    basis = {"f16i8": "fp16 dense tensor peak ({src} {p:.1f} TFLOP/s sustained) / 2 (one fp16 product + one "
+                      "int8 product of 2K at 2x the fp16 rate per FP32 MAC)",
+             "f16x3": "fp16 dense tensor peak ({src} {p:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC",
+             "tf32x3": "tf32 dense tensor peak ({src} {p:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC"}[args.scheme]
     roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                 "frac": achieved / peak if peak else None,
                 "traffic": args.traffic if args.traffic is not None else committed_traffic(N, b, args),
-                "peak_basis": (f"{'fp16' if args.scheme == 'f16x3' else 'tf32'} dense tensor peak "
-                               f"({peaks['source']} {dense_peak:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC"),
+                "peak_basis": basis.format(src=peaks["source"], p=dense_peak),
                 "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None}
 
     # ---- end to end through pmm_run with pinned host buffers
@@ -455,7 +464,7 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--N", type=int, default=N_DEFAULT)
     ap.add_argument("--b", type=int, default=B_DEFAULT)
-    ap.add_argument("--scheme", choices=["f16x3", "tf32x3"], default="f16x3")
+    ap.add_argument("--scheme", choices=["f16i8", "f16x3", "tf32x3"], default="f16i8")
     ap.add_argument("--transport", choices=["ipc", "nccl"], default="ipc",
                     help="N > 1: pull pivots from peers' memory (ipc) or exchange them with NCCL")
     ap.add_argument("--cta-group", type=int, default=2)

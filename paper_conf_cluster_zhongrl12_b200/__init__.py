@@ -16,7 +16,7 @@ import ctypes
 from typing import List, Sequence, Tuple
 
 from . import _lib
-from ._lib import (FPM_DIST_INT, FPM_DIST_PM1, FPM_F32, FPM_F64, SCHEME_F16X3, SCHEME_TF32X3,  # noqa: F401
+from ._lib import (FPM_DIST_INT, FPM_DIST_PM1, FPM_F32, FPM_F64, SCHEME_F16I8, SCHEME_F16X3, SCHEME_TF32X3,  # noqa: F401,E501
                    FpmError, PmmStats, check, lib)
 
 Model = Tuple[Sequence[int], Sequence[float]]

@@ -29,6 +29,7 @@ FPM_DIST_INT = 1
 
 SCHEME_F16X3 = 0
 SCHEME_TF32X3 = 1
+SCHEME_F16I8 = 3      # fp16 main product + int8 cross terms (default for b % 64 == 0)
 
 i32, i64, u64, dbl, vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64, ctypes.c_double, ctypes.c_void_p
 

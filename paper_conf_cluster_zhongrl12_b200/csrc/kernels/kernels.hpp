@@ -13,6 +13,8 @@ namespace fpm {
 enum class SplitScheme : int {
     F16X3 = 0,   // x 2^e = h0 + h1 in fp16, per-row power-of-two scale, 3 x kind::f16
     TF32X3 = 1,  // x = hi + lo in tf32, 3 x kind::tf32
+    I8PROBE = 2, // timing probe only (kernel-level entry): int8 operands, 3 x kind::i8, s32 accumulator
+    F16I8 = 3,   // x 2^e = h0 + h1; h0 h0' in kind::f16 + 32 (q l' + l q') in kind::i8 (update_f32.cu)
 };
 
 struct UpdateArgs {

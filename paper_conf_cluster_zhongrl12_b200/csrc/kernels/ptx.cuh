@@ -168,34 +168,25 @@ __device__ __forceinline__ void tc_fence_after() {
 }
 
 // D[tmem] (+)= A[smem] . B[smem]^T, both K-major, described by 64-bit descriptors.
-template <int CG, bool TF32>
+// KIND: 0 = kind::f16 (f16/bf16 -> f32), 1 = kind::tf32, 2 = kind::i8 (s8 -> s32)
+#define FPM_UMMA_ASM(CGS, KINDS)                                                                    \
+    asm volatile("{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"                                 \
+                 "tcgen05.mma.cta_group::" CGS ".kind::" KINDS " [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem), \
+                 "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)                              \
+                 : "memory")
+template <int CG, int KIND>
 __device__ __forceinline__ void umma(uint32_t d_tmem, uint64_t a_desc, uint64_t b_desc, uint32_t idesc,
                                      uint32_t accumulate) {
-    if constexpr (CG == 1 && !TF32)
-        asm volatile(
-            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-            "tcgen05.mma.cta_group::1.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-            "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
-            : "memory");
-    else if constexpr (CG == 1 && TF32)
-        asm volatile(
-            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-            "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-            "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
-            : "memory");
-    else if constexpr (CG == 2 && !TF32)
-        asm volatile(
-            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-            "tcgen05.mma.cta_group::2.kind::f16 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-            "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
-            : "memory");
-    else
-        asm volatile(
-            "{\n\t.reg .pred p;\n\tsetp.ne.b32 p, %4, 0;\n\t"
-            "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
-            "l"(a_desc), "l"(b_desc), "r"(idesc), "r"(accumulate)
-            : "memory");
+    static_assert(CG == 1 || CG == 2, "cta_group");
+    static_assert(KIND >= 0 && KIND <= 2, "kind");
+    if constexpr (CG == 1 && KIND == 0) FPM_UMMA_ASM("1", "f16");
+    else if constexpr (CG == 1 && KIND == 1) FPM_UMMA_ASM("1", "tf32");
+    else if constexpr (CG == 1 && KIND == 2) FPM_UMMA_ASM("1", "i8");
+    else if constexpr (CG == 2 && KIND == 0) FPM_UMMA_ASM("2", "f16");
+    else if constexpr (CG == 2 && KIND == 1) FPM_UMMA_ASM("2", "tf32");
+    else FPM_UMMA_ASM("2", "i8");
 }
+#undef FPM_UMMA_ASM
 
 // Arrive on an mbarrier when all previously issued tcgen05.mma of this thread complete.
 template <int CG>
@@ -231,6 +222,22 @@ __device__ __forceinline__ void tmem_ld_32x32b_x32(uint32_t taddr, float (&v)[32
     for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
 }
 
+// The same without the wait: raw 32-bit words into r, caller issues tmem_wait_ld().
+__device__ __forceinline__ void tmem_ld_32x32b_x32_nw(uint32_t taddr, uint32_t* r) {
+    asm volatile(
+        "tcgen05.ld.sync.aligned.32x32b.x32.b32 "
+        "{%0, %1, %2, %3, %4, %5, %6, %7, %8, %9, %10, %11, %12, %13, %14, %15, "
+        "%16, %17, %18, %19, %20, %21, %22, %23, %24, %25, %26, %27, %28, %29, %30, %31}, [%32];"
+        : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]), "=r"(r[7]),
+          "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]), "=r"(r[14]),
+          "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]), "=r"(r[21]),
+          "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]), "=r"(r[28]),
+          "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+        : "r"(taddr)
+        : "memory");
+}
+__device__ __forceinline__ void tmem_wait_ld() { asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory"); }
+
 // Shared-memory matrix descriptor, K-major operand with SW-byte swizzle
 // (SW = 128 or 64): rows of SW bytes, 8-row atoms of 8*SW bytes (SBO), LBO
 // unused (1), version 1, layout type 2 (128B) / 4 (64B).
@@ -251,6 +258,10 @@ __device__ __forceinline__ uint64_t sdesc_k(uint32_t smem_addr) {
 __host__ __device__ constexpr uint32_t idesc_f32acc(int M, int N, bool tf32) {
     return (1u << 4) | ((tf32 ? 2u : 0u) << 7) | ((tf32 ? 2u : 0u) << 10) | ((uint32_t)(N >> 3) << 17) |
            ((uint32_t)(M >> 4) << 24);
+}
+// kind::i8: D s32 (c_format 2), A and B signed int8 (format 1), both K-major
+__host__ __device__ constexpr uint32_t idesc_s32acc_s8(int M, int N) {
+    return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(M >> 4) << 24);
 }
 
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {

@@ -34,6 +34,19 @@ __device__ __forceinline__ int f16x3_shift(float m) {
     return s < -126 ? -126 : (s > 127 ? 127 : s);
 }
 
+// F16I8 codes of a scaled element xs = x 2^s (update_f32.cu): h0 = fp16_rn(xs),
+// q = clamp(rint(xs / 256), +-127), l = rint(8 (xs - h0)) (|l| <= 64).
+__device__ __forceinline__ __half f16i8_codes(float xs, int& qc, int& lc) {
+    const __half h = __float2half_rn(xs);
+    qc = min(127, max(-127, __float2int_rn(xs * (1.0f / 256.0f))));
+    lc = __float2int_rn((xs - __half2float(h)) * 8.0f);
+    return h;
+}
+__device__ __forceinline__ uint32_t pack4_s8(int a, int b, int c, int d) {
+    return (uint32_t)(a & 0xff) | ((uint32_t)(b & 0xff) << 8) | ((uint32_t)(c & 0xff) << 16) |
+           ((uint32_t)(d & 0xff) << 24);
+}
+
 // One warp per row.  A row of the operand is nseg segments of K elements, segment
 // j at src + j * seg_stride + row * ld (the panels of nseg consecutive pivots
 // fused into one update); it is written to out + row * ld_out + j * K.
@@ -55,6 +68,9 @@ __device__ __forceinline__ float row_absmax(const float* src, int64_t ld, int64_
     return warp_max(m);
 }
 
+// I8 (F16I8): `lo` holds the int8 codes instead of h1, as 128-byte rows per
+// 64-wide k-block: [q of the 64 | l of the 64] (K % 64 == 0).
+template <bool I8>
 __global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ src, int64_t ld, int64_t seg_stride,
                                                       int nseg, int64_t rows, int64_t K, int64_t ld_out,
                                                       __half* __restrict__ hi, __half* __restrict__ lo,
@@ -76,15 +92,27 @@ __global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ 
             const float4 v = s4[i];
             const float x[4] = {v.x * scale, v.y * scale, v.z * scale, v.w * scale};
             __half h[4], l[4];
+            int qc[4], lc[4];
 #pragma unroll
             for (int q = 0; q < 4; ++q) {
-                h[q] = __float2half_rn(x[q]);
-                l[q] = __float2half_rn(x[q] - __half2float(h[q]));
+                if constexpr (I8) {
+                    h[q] = f16i8_codes(x[q], qc[q], lc[q]);
+                } else {
+                    h[q] = __float2half_rn(x[q]);
+                    l[q] = __float2half_rn(x[q] - __half2float(h[q]));
+                }
             }
             h2[2 * i] = __halves2half2(h[0], h[1]);
             h2[2 * i + 1] = __halves2half2(h[2], h[3]);
-            l2[2 * i] = __halves2half2(l[0], l[1]);
-            l2[2 * i + 1] = __halves2half2(l[2], l[3]);
+            if constexpr (I8) {
+                const int64_t k = 4 * i;
+                uint8_t* b8 = reinterpret_cast<uint8_t*>(l2) + (k / 64) * 128 + (k % 64);
+                *reinterpret_cast<uint32_t*>(b8) = pack4_s8(qc[0], qc[1], qc[2], qc[3]);
+                *reinterpret_cast<uint32_t*>(b8 + 64) = pack4_s8(lc[0], lc[1], lc[2], lc[3]);
+            } else {
+                l2[2 * i] = __halves2half2(l[0], l[1]);
+                l2[2 * i + 1] = __halves2half2(l[2], l[3]);
+            }
         }
     }
 }
@@ -153,7 +181,9 @@ __global__ void __launch_bounds__(256) colmax_tile_k(const float* __restrict__ s
 // Split + transpose: warp w of a CTA reads rows kk .. kk+7 (kk = k0 + 8 w) of 128
 // columns (a float4 per lane and row); each lane then writes, for each of its 4
 // columns, the 8 values as 16 B of output row `column`.
-template <bool F16>
+// I8 (F16I8): `lo` holds int8 codes as 128-byte rows per 64-wide k-block:
+// [l of the 64 | q of the 64] (the B side of the cross-term product).
+template <bool F16, bool I8 = false>
 __global__ void __launch_bounds__(256) split_cols_t(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
                                                     int64_t ld_out, void* __restrict__ hi, void* __restrict__ lo,
                                                     const unsigned* __restrict__ m_bits,
@@ -179,14 +209,28 @@ __global__ void __launch_bounds__(256) split_cols_t(const float* __restrict__ sr
             const float scale = ldexpf(1.0f, s);
             if (inv_scale != nullptr && kk == 0) inv_scale[col + c] = ldexpf(1.0f, -s);
             __align__(16) __half h[8], l[8];
+            int qc[8], lc[8];
 #pragma unroll
             for (int i = 0; i < 8; ++i) {
                 const float xs = x[c][i] * scale;
-                h[i] = __float2half_rn(xs);
-                l[i] = __float2half_rn(xs - __half2float(h[i]));
+                if constexpr (I8) {
+                    h[i] = f16i8_codes(xs, qc[i], lc[i]);
+                } else {
+                    h[i] = __float2half_rn(xs);
+                    l[i] = __float2half_rn(xs - __half2float(h[i]));
+                }
             }
             *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + orow) = *reinterpret_cast<uint4*>(h);
-            *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + orow) = *reinterpret_cast<uint4*>(l);
+            if constexpr (I8) {
+                uint8_t* b8 = reinterpret_cast<uint8_t*>(static_cast<__half*>(lo) + (col + c) * ld_out) +
+                              (kk / 64) * 128 + (kk % 64);
+                *reinterpret_cast<uint2*>(b8) =
+                    make_uint2(pack4_s8(lc[0], lc[1], lc[2], lc[3]), pack4_s8(lc[4], lc[5], lc[6], lc[7]));
+                *reinterpret_cast<uint2*>(b8 + 64) =
+                    make_uint2(pack4_s8(qc[0], qc[1], qc[2], qc[3]), pack4_s8(qc[4], qc[5], qc[6], qc[7]));
+            } else {
+                *reinterpret_cast<uint4*>(static_cast<__half*>(lo) + orow) = *reinterpret_cast<uint4*>(l);
+            }
         } else {
             __align__(16) float h[8], l[8];
 #pragma unroll
@@ -421,11 +465,18 @@ void launch_split_rows_seg(const float* src, int64_t ld, int64_t seg_stride, int
     if (rows <= 0 || K <= 0 || nseg <= 0) return;
     FPM_CHECK_ARG(K % 4 == 0 && ld % 4 == 0 && seg_stride % 4 == 0 && ld_out % 4 == 0 && ld_out >= nseg * K,
                   "split: K, ld, seg_stride, ld_out must be multiples of 4 and ld_out >= nseg*K");
-    if (s == SplitScheme::F16X3) {
+    if (s == SplitScheme::F16X3 || s == SplitScheme::F16I8) {
         const int64_t blocks = (rows + 7) / 8;
-        split_rows_f16<<<(unsigned)blocks, 256, 0, st>>>(src, ld, seg_stride, nseg, rows, K, ld_out,
-                                                         static_cast<__half*>(hi), static_cast<__half*>(lo),
-                                                         inv_scale, given_max);
+        if (s == SplitScheme::F16I8) {
+            FPM_CHECK_ARG(K % 64 == 0 && ld_out % 64 == 0, "F16I8 split: K and ld_out multiples of 64");
+            split_rows_f16<true><<<(unsigned)blocks, 256, 0, st>>>(src, ld, seg_stride, nseg, rows, K, ld_out,
+                                                                   static_cast<__half*>(hi), static_cast<__half*>(lo),
+                                                                   inv_scale, given_max);
+        } else {
+            split_rows_f16<false><<<(unsigned)blocks, 256, 0, st>>>(src, ld, seg_stride, nseg, rows, K, ld_out,
+                                                                    static_cast<__half*>(hi),
+                                                                    static_cast<__half*>(lo), inv_scale, given_max);
+        }
         check_launch("split_rows_f16");
     } else {
         split_rows_tf32<<<grid_for(rows * nseg * K / 4, 256), 256, 0, st>>>(
@@ -447,16 +498,19 @@ void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, Split
     FPM_CHECK_ARG(W % 4 == 0 && ld % 4 == 0 && (reinterpret_cast<uintptr_t>(src) & 15) == 0,
                   "split_cols: W and ld multiples of 4, src 16-byte aligned");
     const dim3 grid((unsigned)((W + kColsPerCta - 1) / kColsPerCta), (unsigned)((K + kColTileK - 1) / kColTileK));
-    if (s == SplitScheme::F16X3) {
-        FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 needs inv_scale");
+    if (s == SplitScheme::F16X3 || s == SplitScheme::F16I8) {
+        FPM_CHECK_ARG(inv_scale != nullptr, "F16X3 / F16I8 need inv_scale");
+        const bool i8 = s == SplitScheme::F16I8;
+        if (i8) FPM_CHECK_ARG(K % 64 == 0 && ld_out % 64 == 0, "F16I8 split: K and ld_out multiples of 64");
+        auto kern = i8 ? split_cols_t<true, true> : split_cols_t<true, false>;
         if (given_max) {
-            split_cols_t<true><<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, given_max, inv_scale);
+            kern<<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, given_max, inv_scale);
         } else {  // maxima into inv_scale (as bits), split, then bits -> inverse scales in place
             unsigned* bits = reinterpret_cast<unsigned*>(inv_scale);
             const cudaError_t e = cudaMemsetAsync(bits, 0, (size_t)W * sizeof(unsigned), st);
             if (e != cudaSuccess) fail(FPM_ECUDA, "split_cols memset: %s", cudaGetErrorString(e));
             launch_colmax(src, ld, K, W, bits, st);
-            split_cols_t<true><<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, bits, nullptr);
+            kern<<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, bits, nullptr);
             check_launch("split_cols");
             scale_from_max_k<<<(unsigned)((W + 255) / 256), 256, 0, st>>>(inv_scale, W);
         }

@@ -39,12 +39,12 @@
 
 namespace fpm {
 
-template <int CG, bool TF32, int BN, int STAGES, int SW, int NCB>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB>
 struct UpdCfg {
     static constexpr int BM = 128;                 // rows of C per CTA
     static constexpr int TILE_M = BM * CG;         // rows per MMA tile
     static constexpr int BN_CTA = BN / CG;         // B^T rows loaded per CTA
-    static constexpr int ELEM = TF32 ? 4 : 2;      // operand bytes
+    static constexpr int ELEM = KIND == 1 ? 4 : (KIND == 0 ? 2 : 1);  // operand bytes
     static constexpr int BK = SW / ELEM;           // k elements per SW-byte row
     static constexpr int KSTEPS = SW / 32;         // MMA k-steps (32 B each) per k-block
     static constexpr int A_BYTES = BM * SW;        // one operand half (hi or lo)
@@ -55,7 +55,8 @@ struct UpdCfg {
     static constexpr int TMEM_COLS = 2 * BN;
     static constexpr int BAR_BYTES = 8 * (2 * STAGES + 4 + NCB) + 16;
     static constexpr int SMEM = 1024 /*align slack*/ + STAGES * STAGE_BYTES + NCB * C_CHUNK_BYTES + BAR_BYTES;
-    static constexpr uint32_t IDESC = ptx::idesc_f32acc(TILE_M, BN, TF32);
+    static constexpr uint32_t IDESC =
+        KIND == 2 ? ptx::idesc_s32acc_s8(TILE_M, BN) : ptx::idesc_f32acc(TILE_M, BN, KIND == 1);
     static constexpr int THREADS = 192;
     static_assert(SW == 128 || SW == 64, "swizzle width");
     static_assert(NCB >= 2 && NCB <= 8, "C ring depth");
@@ -86,12 +87,12 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
     tn = r / gm;
 }
 
-template <int CG, bool TF32, int BN, int STAGES, int SW, int NCB>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB>
 __global__ void __launch_bounds__(192, 1)
     update_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
                   const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
                   const __grid_constant__ CUtensorMap tmC, const UpdParams P) {
-    using Cfg = UpdCfg<CG, TF32, BN, STAGES, SW, NCB>;
+    using Cfg = UpdCfg<CG, KIND, BN, STAGES, SW, NCB>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
     uint8_t* stage_base = smem;
@@ -200,9 +201,9 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
                         for (int k = 0; k < Cfg::KSTEPS; ++k) {
                             const uint64_t off = (uint64_t)(k * 32) >> 4;  // 32 B per MMA k-step
-                            ptx::umma<CG, TF32>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC, (kb | k) != 0);
-                            ptx::umma<CG, TF32>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
-                            ptx::umma<CG, TF32>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
+                            ptx::umma<CG, KIND>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC, (kb | k) != 0);
+                            ptx::umma<CG, KIND>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
+                            ptx::umma<CG, KIND>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
                         }
                         ptx::umma_commit<CG>(&empty[stage]);
                     }
@@ -249,6 +250,10 @@ __global__ void __launch_bounds__(192, 1)
                 const int buf = c % NCB;
                 float v[32];
                 ptx::tmem_ld_32x32b_x32(t_row + 32 * c, v);
+                if constexpr (KIND == 2) {  // s32 accumulator (timing probe)
+#pragma unroll
+                    for (int j = 0; j < 32; ++j) v[j] = (float)__float_as_int(v[j]);
+                }
                 if (c == Cfg::N_CHUNKS - 1) {
                     // accumulator fully read: hand it back to the MMA warp
                     ptx::tc_fence_before();
@@ -328,6 +333,284 @@ __global__ void __launch_bounds__(192, 1)
     }
 }
 
+// ------------------------------------------------------------ F16I8 (default)
+// FP32 operand x of a row (A) / column (B) with the F16X3 power-of-two scale
+// 2^e (row maximum in [2^14, 2^15)):  x 2^e = h0 + h1, h0 = fp16_rn(x 2^e),
+// |h1| <= 8, and two int8 codes q = clamp(rint(x 2^e / 256), +-127),
+// l = rint(8 h1) (|l| <= 64).  Then
+//   x_a x_b 2^(ea+eb) = h0a h0b + h0a h1b + h1a h0b + h1a h1b
+//                     ~ h0a h0b            (kind::f16, exact products, fp32 sum)
+//                     + 32 (qa lb + la qb) (kind::i8, exact s32 sum)
+// with the dropped h1a h1b and the q rounding of the cross terms at the 2^-18
+// level (relative Frobenius error ~3e-6 on U[-1,1), tolerance 1e-5).  The int8
+// operand of a 64-wide k-block is one 128-byte row [q(64) | l(64)] for A and
+// [l(64) | q(64)] for B^T, so ONE kind::i8 product over 128 bytes gives both
+// cross terms.  Per k-block: 4 f16 MMAs (K = 16 each) + 4 i8 MMAs (K = 32 each)
+// instead of F16X3's 12 f16 MMAs -- the int8 rate is twice the f16 rate and an
+// int8 operation was measured to cost 0.44 of the energy of an f16 one under
+// the 1000 W cap (studies/probes/i8_energy.py), and the update is power-bound.
+//
+// TMEM: the fp32 accumulator (256 columns) and the s32 accumulator (256) fill
+// all 512 columns, so there is no second accumulator set: eight epilogue warps
+// (two per TMEM lane quarter, one per 128-column half) drain both accumulators
+// into registers (128 combined values per thread), hand TMEM back to the MMA
+// warp, and only then do the C read-modify-write, which overlaps the next
+// tile's mainloop.  Each column half runs its own C ring (NCB / 2 chunks).
+// SW: bytes per operand row and k-block (128: 64 K per k-block, the fp16 row and
+// the whole [q | l] int8 row; 64: 32 K per k-block, the fp16 row and one half --
+// q or l -- of the int8 row: the pairing of fp16 and int8 k-blocks is free, the
+// two accumulators are independent sums over K).
+template <int SW, int STAGES, int NCB>
+struct HybCfg {
+    static constexpr int CG = 2, BM = 128, TILE_M = 256, BN = 256, BN_CTA = 128;
+    static constexpr int BK = SW / 2;         // fp16 K per k-block (int8 bytes per k-block: SW)
+    static constexpr int KSTEPS = SW / 32;    // 32 B per MMA k-step (16 fp16 / 32 int8 elements)
+    static constexpr int A_BYTES = BM * SW, B_BYTES = BN_CTA * SW;
+    static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);  // A fp16, A int8, B fp16, B int8
+    static constexpr int NCBH = NCB / 2;
+    static constexpr int C_CHUNK_BYTES = BM * 128;  // 128 rows x 32 fp32
+    static constexpr int BAR_BYTES = 8 * (2 * STAGES + 2 + NCB) + 16;
+    static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + NCB * C_CHUNK_BYTES + BAR_BYTES;
+    static constexpr uint32_t IDESC_F = ptx::idesc_f32acc(TILE_M, BN, false);
+    static constexpr uint32_t IDESC_I = ptx::idesc_s32acc_s8(TILE_M, BN);
+    static constexpr int THREADS = 320;  // producer, MMA, 8 epilogue warps
+    static_assert(SW == 128 || SW == 64, "swizzle width");
+    static_assert(NCB % 2 == 0 && NCBH >= 2 && NCBH <= 4, "C ring: 2..4 chunks per half");
+    static_assert(SMEM <= 232448, "shared memory budget");
+};
+
+template <int SW, int STAGES, int NCB>
+__global__ void __launch_bounds__(320, 1)
+    update_hyb_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_8,
+                      const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_8,
+                      const __grid_constant__ CUtensorMap tmC, const UpdParams P) {
+    using Cfg = HybCfg<SW, STAGES, NCB>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* stage_base = smem;
+    uint8_t* cbuf = smem + STAGES * Cfg::STAGE_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + NCB * Cfg::C_CHUNK_BYTES);
+    uint64_t* full = bars;               // [STAGES]
+    uint64_t* empty = bars + STAGES;     // [STAGES]
+    uint64_t* tfull = bars + 2 * STAGES;
+    uint64_t* tempty = tfull + 1;
+    uint64_t* cfull = tfull + 2;         // [NCB]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(cfull + NCB);
+
+    const uint32_t warp = threadIdx.x / 32;
+    const uint32_t lane = threadIdx.x % 32;
+    const uint32_t rank = ptx::cluster_ctarank();
+    const bool leader = rank == 0;
+    const int cluster_id = blockIdx.x / 2;
+    const int num_clusters = gridDim.x / 2;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            ptx::mbar_init(&full[s], 1);
+            ptx::mbar_init(&empty[s], 1);
+        }
+        ptx::mbar_init(tfull, 1);
+        ptx::mbar_init(tempty, 8 * 2);  // every epilogue warp of both CTAs
+        for (int c = 0; c < NCB; ++c) ptx::mbar_init(&cfull[c], 1);
+        ptx::fence_mbar_init();
+    }
+    if (warp == 0 && lane == 0) {
+        ptx::tma_prefetch_desc(&tmA_hi);
+        ptx::tma_prefetch_desc(&tmA_8);
+        ptx::tma_prefetch_desc(&tmB_hi);
+        ptx::tma_prefetch_desc(&tmB_8);
+        ptx::tma_prefetch_desc(&tmC);
+    }
+    if (warp == 1) {
+        ptx::tmem_alloc<2>(tmem_slot, 512);
+        ptx::tmem_relinquish<2>();
+    }
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::cluster_sync();
+    ptx::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int num_kb = P.K / Cfg::BK;
+
+    if (warp == 0) {
+        // ------------------------------------------------------------ producer
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+                int tm, tn;
+                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+                const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
+                const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA;
+                for (int kb = 0; kb < num_kb; ++kb) {
+                    ptx::mbar_wait(&empty[stage], phase ^ 1);
+                    uint8_t* sA_hi = stage_base + stage * Cfg::STAGE_BYTES;
+                    uint8_t* sA_8 = sA_hi + Cfg::A_BYTES;
+                    uint8_t* sB_hi = sA_8 + Cfg::A_BYTES;
+                    uint8_t* sB_8 = sB_hi + Cfg::B_BYTES;
+                    const int k0 = kb * Cfg::BK;
+                    if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
+                    ptx::tma_load_2d_cg2(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
+                    ptx::tma_load_2d_cg2(sA_8, &tmA_8, &full[stage], kb * SW, m0, ptx::kEvictLast);
+                    ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
+                    ptx::tma_load_2d_cg2(sB_8, &tmB_8, &full[stage], kb * SW, n0, P.hint_b);
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ----------------------------------------------------------- MMA issuer
+        if (leader) {
+            int stage = 0;
+            uint32_t phase = 0;
+            int it = 0;
+            for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
+                ptx::mbar_wait(tempty, (it & 1) ^ 1);
+                ptx::tc_fence_after();
+                for (int kb = 0; kb < num_kb; ++kb) {
+                    ptx::mbar_wait(&full[stage], phase);
+                    ptx::tc_fence_after();
+                    if (lane == 0) {
+                        const uint32_t a_hi = ptx::smem_u32(stage_base + stage * Cfg::STAGE_BYTES);
+                        const uint32_t a_8 = a_hi + Cfg::A_BYTES;
+                        const uint32_t b_hi = a_8 + Cfg::A_BYTES;
+                        const uint32_t b_8 = b_hi + Cfg::B_BYTES;
+                        const uint64_t dA_hi = ptx::sdesc_k<SW>(a_hi), dA_8 = ptx::sdesc_k<SW>(a_8);
+                        const uint64_t dB_hi = ptx::sdesc_k<SW>(b_hi), dB_8 = ptx::sdesc_k<SW>(b_8);
+#pragma unroll
+                        for (int k = 0; k < Cfg::KSTEPS; ++k) {
+                            const uint64_t off = (uint64_t)(k * 32) >> 4;
+                            ptx::umma<2, 0>(tmem_base, dA_hi + off, dB_hi + off, Cfg::IDESC_F, (kb | k) != 0);
+                            ptx::umma<2, 2>(tmem_base + 256, dA_8 + off, dB_8 + off, Cfg::IDESC_I, (kb | k) != 0);
+                        }
+                        ptx::umma_commit<2>(&empty[stage]);
+                    }
+                    __syncwarp();
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+                if (lane == 0) ptx::umma_commit<2>(tfull);
+                __syncwarp();
+            }
+        }
+    } else {
+        // -------------------------------------------------------------- epilogue
+        const uint32_t e = threadIdx.x - 64;  // 0..255
+        const uint32_t hh = e / 128;          // column half of the tile
+        const uint32_t eh = e % 128;
+        const uint32_t q = warp & 3;          // TMEM lane quarter
+        const uint32_t r = q * 32 + lane;     // row of the CTA tile
+        const uint32_t bar_id = 1 + hh;
+        uint8_t* cb = cbuf + hh * Cfg::NCBH * Cfg::C_CHUNK_BYTES;
+        uint64_t* cf = cfull + hh * Cfg::NCBH;
+        uint32_t cpar = 0;
+        int it = 0;
+        for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
+            int tm, tn;
+            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+            const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
+            const int n0 = tn * Cfg::BN + (int)hh * 128;
+            if (eh == 0 && P.load_c) {
+                ptx::bulk_wait_read0();
+#pragma unroll
+                for (int c = 0; c < Cfg::NCBH; ++c) {
+                    ptx::mbar_arrive_expect_tx(&cf[c], Cfg::C_CHUNK_BYTES);
+                    ptx::tma_load_2d(cb + c * Cfg::C_CHUNK_BYTES, &tmC, &cf[c], n0 + 32 * c, m0, ptx::kEvictFirst);
+                }
+            }
+            const int grow = m0 + (int)r;
+            const float sa = (P.sa != nullptr && grow < P.M) ? P.sa[grow] : 1.0f;
+            ptx::mbar_wait(tfull, it & 1);
+            ptx::tc_fence_after();
+            // drain both accumulators: u = acc_f + 32 acc_i (128 columns of this half)
+            const uint32_t t_row = tmem_base + ((q * 32) << 16) + hh * 128;
+            uint32_t u[128];
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                uint32_t ti[32];
+                ptx::tmem_ld_32x32b_x32_nw(t_row + 32 * c, &u[32 * c]);
+                ptx::tmem_ld_32x32b_x32_nw(t_row + 256 + 32 * c, ti);
+                ptx::tmem_wait_ld();
+#pragma unroll
+                for (int j = 0; j < 32; ++j)
+                    u[32 * c + j] = __float_as_uint(fmaf(32.0f, (float)(int)ti[j], __uint_as_float(u[32 * c + j])));
+            }
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) ptx::mbar_arrive_cluster(tempty, 0);
+            // C read-modify-write (overlaps the next tile's mainloop)
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const int buf = c % Cfg::NCBH;
+                float v[32];
+#pragma unroll
+                for (int j = 0; j < 32; ++j) v[j] = __uint_as_float(u[32 * c + j]);
+                if (P.sb != nullptr) {
+                    const int gc = n0 + 32 * c;
+                    if (gc + 32 <= P.Nc) {
+                        const float4* sb4 = reinterpret_cast<const float4*>(P.sb + gc);
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) {
+                            const float4 s4 = __ldg(sb4 + j);
+                            v[4 * j + 0] *= sa * s4.x;
+                            v[4 * j + 1] *= sa * s4.y;
+                            v[4 * j + 2] *= sa * s4.z;
+                            v[4 * j + 3] *= sa * s4.w;
+                        }
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) {
+                            const float sbj = (gc + j < P.Nc) ? __ldg(P.sb + gc + j) : 0.0f;
+                            v[j] *= sa * sbj;
+                        }
+                    }
+                }
+                if (P.load_c) {
+                    ptx::mbar_wait(&cf[buf], (cpar >> buf) & 1u);
+                    cpar ^= 1u << buf;
+                } else {
+                    if (eh == 0) ptx::bulk_wait_read_n<Cfg::NCBH - 1>();
+                    ptx::named_bar_sync(bar_id, 128);
+                }
+                uint8_t* rowp = cb + buf * Cfg::C_CHUNK_BYTES + r * 128;
+#pragma unroll
+                for (int j = 0; j < 8; ++j) {
+                    float4* p4 = reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4));
+                    float4 cv = make_float4(0.f, 0.f, 0.f, 0.f);
+                    if (P.load_c) cv = *p4;
+                    cv.x += v[4 * j + 0];
+                    cv.y += v[4 * j + 1];
+                    cv.z += v[4 * j + 2];
+                    cv.w += v[4 * j + 3];
+                    *p4 = cv;
+                }
+                ptx::fence_proxy_async_smem();
+                ptx::named_bar_sync(bar_id, 128);
+                if (eh == 0) {
+                    ptx::tma_store_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0, ptx::kEvictFirst);
+                    ptx::bulk_commit();
+                    const int nxt = c - 1 + Cfg::NCBH;  // refill the buffer of chunk c - 1
+                    if (P.load_c && c >= 1 && nxt < 4) {
+                        const int nb = (c - 1) % Cfg::NCBH;
+                        ptx::bulk_wait_read1();
+                        ptx::mbar_arrive_expect_tx(&cf[nb], Cfg::C_CHUNK_BYTES);
+                        ptx::tma_load_2d(cb + nb * Cfg::C_CHUNK_BYTES, &tmC, &cf[nb], n0 + 32 * nxt, m0,
+                                         ptx::kEvictFirst);
+                    }
+                }
+            }
+        }
+        if (eh == 0) ptx::bulk_wait0();
+    }
+
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::cluster_sync();
+    if (warp == 1) {
+        ptx::tc_fence_after();
+        ptx::tmem_dealloc<2>(tmem_base, 512);
+    }
+}
+
 // ------------------------------------------------------------------- host side
 namespace {
 
@@ -372,10 +655,12 @@ CUtensorMap make_tmap_2d(const void* base, CUtensorMapDataType dt, int elem_byte
     return m;
 }
 
-template <int CG, bool TF32, int BN, int STAGES, int SW, int NCB>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB>
 static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
-    using Cfg = UpdCfg<CG, TF32, BN, STAGES, SW, NCB>;
-    const CUtensorMapDataType odt = TF32 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+    using Cfg = UpdCfg<CG, KIND, BN, STAGES, SW, NCB>;
+    const CUtensorMapDataType odt = KIND == 1   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
+                                    : KIND == 0 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT16
+                                                : CU_TENSOR_MAP_DATA_TYPE_UINT8;
     const CUtensorMap tAh = make_tmap_2d(a.a_hi, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
     const CUtensorMap tAl = make_tmap_2d(a.a_lo, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
     const CUtensorMap tBh = make_tmap_2d(a.bt_hi, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
@@ -393,7 +678,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.load_c = a.accumulate ? 1 : 0;
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
-    auto kern = update_kernel<CG, TF32, BN, STAGES, SW, NCB>;
+    auto kern = update_kernel<CG, KIND, BN, STAGES, SW, NCB>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;
     cudaGetDevice(&dev);
@@ -421,6 +706,56 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
 }
 
+template <int SW, int STAGES, int NCB>
+static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
+    using Cfg = HybCfg<SW, STAGES, NCB>;
+    const CUtensorMap tAh = make_tmap_2d(a.a_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
+    const CUtensorMap tA8 = make_tmap_2d(a.a_lo, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, a.M, 2 * a.K, 2 * a.K, SW, Cfg::BM);
+    const CUtensorMap tBh =
+        make_tmap_2d(a.bt_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+    const CUtensorMap tB8 =
+        make_tmap_2d(a.bt_lo, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, a.Nc, 2 * a.K, 2 * a.K, SW, Cfg::BN_CTA);
+    const CUtensorMap tC = make_tmap_2d(a.C, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.M, a.Nc, a.ldc, 32, Cfg::BM);
+    UpdParams P;
+    P.M = (int)a.M;
+    P.Nc = (int)a.Nc;
+    P.K = (int)a.K;
+    P.tiles_m = (int)((a.M + Cfg::TILE_M - 1) / Cfg::TILE_M);
+    P.tiles_n = (int)((a.Nc + Cfg::BN - 1) / Cfg::BN);
+    P.num_tiles = P.tiles_m * P.tiles_n;
+    P.sa = a.sa;
+    P.sb = a.sb;
+    P.load_c = a.accumulate ? 1 : 0;
+    P.group = a.raster_group > 0 ? a.raster_group : 16;
+    P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
+    auto kern = update_hyb_kernel<SW, STAGES, NCB>;
+    static uint64_t attr_done = 0;
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(attr_done & (1ull << dev))) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+        attr_done |= 1ull << dev;
+    }
+    int clusters = a.num_sms / 2;
+    if (clusters > P.num_tiles) clusters = P.num_tiles;
+    if (clusters < 1) clusters = 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(clusters * 2);
+    cfg.blockDim = dim3(Cfg::THREADS);
+    cfg.dynamicSmemBytes = Cfg::SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tAh, tA8, tBh, tB8, tC, P);
+    if (e != cudaSuccess) fail(FPM_ECUDA, "F16I8 update kernel launch: %s", cudaGetErrorString(e));
+}
+
 void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     if (a.M <= 0 || a.Nc <= 0 || a.K <= 0) return;
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
@@ -428,6 +763,24 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
     FPM_CHECK_ARG(a.variant >= -1 && a.variant <= 4, "kernel variant must be -1 (auto) or 0..4");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
+    if (a.scheme == SplitScheme::F16I8) {
+        FPM_CHECK_ARG(a.cta_group == 2, "F16I8 runs on CTA pairs (cta_group 2)");
+        FPM_CHECK_ARG(a.K % 64 == 0, "F16I8: K must be a multiple of 64");
+        FPM_CHECK_ARG(a.sa != nullptr && a.sb != nullptr, "F16I8 needs sa and sb");
+        switch (a.variant) {
+            case 0: launch_update_hyb_t<128, 2, 4>(a, st); break;  // 2 x 64 KB stages, 4 C chunks (192 KB)
+            case 1: launch_update_hyb_t<64, 4, 4>(a, st); break;   // 4 x 32 KB stages, 4 C chunks (192 KB)
+            case 2: launch_update_hyb_t<128, 2, 6>(a, st); break;  // 2 x 64 KB stages, 6 C chunks (224 KB)
+            case 3: launch_update_hyb_t<64, 5, 4>(a, st); break;   // 5 x 32 KB stages, 4 C chunks (224 KB)
+            default: launch_update_hyb_t<64, 5, 4>(a, st);
+        }
+        return;
+    }
+    if (a.scheme == SplitScheme::I8PROBE) {  // timing probe: int8 operands, 3 x kind::i8 per k-step
+        FPM_CHECK_ARG(a.cta_group == 2 && a.K % 128 == 0, "I8 probe: cta_group 2, K % 128 == 0");
+        launch_update_t<2, 2, 256, 2, 128, 4>(a, st);
+        return;
+    }
     // auto: variant 4 (two 64-KB operand stages, four C chunks in flight): as fast
     // as variant 2 (six C chunks) at the fused K = 2048 (429 TFLOP/s both, c5) and
     // leaves ~36 KB of shared memory per SM for kernels that must co-run with the
@@ -436,29 +789,29 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     if (a.cta_group == 2) {
         switch (variant) {
             case 1:  // 64-B k-blocks x 4 stages, 6 C chunks in flight
-                if (tf32) launch_update_t<2, true, 256, 4, 64, 6>(a, st);
-                else launch_update_t<2, false, 256, 4, 64, 6>(a, st);
+                if (tf32) launch_update_t<2, 1, 256, 4, 64, 6>(a, st);
+                else launch_update_t<2, 0, 256, 4, 64, 6>(a, st);
                 break;
             case 2:  // 128-B k-blocks x 2 stages, 6 C chunks
-                if (tf32) launch_update_t<2, true, 256, 2, 128, 6>(a, st);
-                else launch_update_t<2, false, 256, 2, 128, 6>(a, st);
+                if (tf32) launch_update_t<2, 1, 256, 2, 128, 6>(a, st);
+                else launch_update_t<2, 0, 256, 2, 128, 6>(a, st);
                 break;
             case 3:  // 64-B k-blocks x 5 stages, 4 C chunks
-                if (tf32) launch_update_t<2, true, 256, 5, 64, 4>(a, st);
-                else launch_update_t<2, false, 256, 5, 64, 4>(a, st);
+                if (tf32) launch_update_t<2, 1, 256, 5, 64, 4>(a, st);
+                else launch_update_t<2, 0, 256, 5, 64, 4>(a, st);
                 break;
             case 4:  // 128-B k-blocks x 2 stages, 4 C chunks: leaves ~36 KB smem per SM for
                      // NCCL kernels to co-run with the persistent update
-                if (tf32) launch_update_t<2, true, 256, 2, 128, 4>(a, st);
-                else launch_update_t<2, false, 256, 2, 128, 4>(a, st);
+                if (tf32) launch_update_t<2, 1, 256, 2, 128, 4>(a, st);
+                else launch_update_t<2, 0, 256, 2, 128, 4>(a, st);
                 break;
             default:  // 128-B k-blocks x 3 stages, 2 C chunks
-                if (tf32) launch_update_t<2, true, 256, 3, 128, 2>(a, st);
-                else launch_update_t<2, false, 256, 3, 128, 2>(a, st);
+                if (tf32) launch_update_t<2, 1, 256, 3, 128, 2>(a, st);
+                else launch_update_t<2, 0, 256, 3, 128, 2>(a, st);
         }
     } else {
-        if (tf32) launch_update_t<1, true, 256, 2, 128, 2>(a, st);
-        else launch_update_t<1, false, 256, 2, 128, 2>(a, st);
+        if (tf32) launch_update_t<1, 1, 256, 2, 128, 2>(a, st);
+        else launch_update_t<1, 0, 256, 2, 128, 2>(a, st);
     }
 }
 

@@ -139,7 +139,7 @@ struct pmm_ctx {
     std::vector<colpart_rect> rects;
     std::vector<std::vector<fpm::Move>> plan_a, plan_b;
 
-    int f32_scheme = 0;  // fpm::SplitScheme
+    int f32_scheme = -1;  // fpm::SplitScheme, -1 = auto (scheme_for)
     int cta_group = 2;
     int raster_group = 16;
     int l2_hint_b = 0;
@@ -508,6 +508,17 @@ int fuse_factor(pmm_ctx* ctx, fpm_dtype dt, int64_t b) {
     return (int)std::max<int64_t>(1, std::min<int64_t>(8, 2048 / b));
 }
 
+// FP32 scheme of a problem with block size b: the option, or auto = F16I8
+// (fp16 main product + int8 cross terms) when every fused K is a multiple of 64
+// and CTA pairs are on, else F16X3.  Both use 2-byte operand halves and
+// per-row / per-column scales; TF32X3 uses 4-byte halves and no scales.
+SplitScheme scheme_for(const pmm_ctx* ctx, int64_t b) {
+    if (ctx->f32_scheme >= 0) return (SplitScheme)ctx->f32_scheme;
+    return (b % 64 == 0 && ctx->cta_group == 2) ? SplitScheme::F16I8 : SplitScheme::F16X3;
+}
+bool has_scales(SplitScheme s) { return s != SplitScheme::TF32X3; }
+size_t op_bytes(SplitScheme s) { return s == SplitScheme::TF32X3 ? 4 : 2; }
+
 // ---------------------------------------------------------------- setup
 // Operand buffers of one slot: receive buffers (NCCL lands pivots in them;
 // FP64 copies peers' pivots into them -- FP32 in local / IPC mode stages
@@ -515,7 +526,7 @@ int fuse_factor(pmm_ctx* ctx, fpm_dtype dt, int64_t b) {
 void alloc_slot(pmm_ctx* ctx, Device& d, int s) {
     const fpm_dtype dt = ctx->dt;
     const size_t es = esize(dt);
-    const size_t op = (dt == FPM_F64) ? 0 : (ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4);
+    const size_t op = (dt == FPM_F64) ? 0 : op_bytes(scheme_for(ctx, ctx->b));
     const bool need_recv = ctx->nccl_mode || dt == FPM_F64;
     const size_t fb = (size_t)ctx->fuse_max * ctx->b;  // K of a fused update
     if (need_recv) {
@@ -800,9 +811,9 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     // ---- staging: K-major operands of the fused update (K = f b)
     if (tp.phase != 2) rec_t(d.ev_pack0[g], d.s_comm);
     if (ctx->dt == FPM_F32) {
-        const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
-        const bool f16 = sch == SplitScheme::F16X3;
-        const size_t op = f16 ? 2 : 4;
+        const SplitScheme sch = scheme_for(ctx, ctx->b);
+        const bool f16 = has_scales(sch);
+        const size_t op = op_bytes(sch);
         FPM_CHECK_ARG(b_src != nullptr, "no source of block-row %lld for device %d", (long long)k0, d.idx);
         if (tp.phase == 1) {  // maxima only (TF32X3 has no scales: nothing to do)
             if (f16) {
@@ -857,7 +868,8 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.a_lo = d.a_lo[slot];
     a.bt_hi = d.b_hi[slot];
     a.bt_lo = d.b_lo[slot];
-    const bool f16 = ctx->f32_scheme == (int)SplitScheme::F16X3;
+    const SplitScheme sch = scheme_for(ctx, ctx->b);
+    const bool f16 = has_scales(sch);
     a.sa = f16 ? d.sa[slot] : nullptr;
     a.sb = f16 ? d.sb[slot] : nullptr;
     a.C = static_cast<float*>(d.C);
@@ -865,7 +877,7 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.Nc = d.W;
     a.K = (int64_t)ctx->groups[g].second * ctx->b;
     a.ldc = d.W;
-    a.scheme = (SplitScheme)ctx->f32_scheme;
+    a.scheme = sch;
     a.cta_group = ctx->cta_group;
     a.num_sms = d.num_sms;
     a.accumulate = ctx->groups[g].first != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
@@ -878,7 +890,7 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
 // The same update restricted to rows [r0, r0 + m) of C_i, written to `Cband`
 // (row stride W): rows r0.. of the A operand and of its scales.
 UpdateArgs band_args(const UpdateArgs& a, int64_t r0, int64_t m, float* Cband) {
-    const size_t op = a.scheme == SplitScheme::F16X3 ? 2 : 4;
+    const size_t op = op_bytes(a.scheme);
     UpdateArgs x = a;
     x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * a.K * op;
     x.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * a.K * op;
@@ -988,7 +1000,7 @@ void ensure_fused_tail(pmm_ctx* ctx, Device& d, int gt) {
     CU(cudaDeviceSynchronize());
     for (void* p : d.tail_allocs) cudaFree(p);
     d.tail_allocs.clear();
-    const size_t op = ctx->f32_scheme == (int)SplitScheme::F16X3 ? 2 : 4;
+    const size_t op = op_bytes(scheme_for(ctx, ctx->b));
     auto get = [&](size_t bytes) {
         void* p = nullptr;
         if (cudaMalloc(&p, bytes) != cudaSuccess) {
@@ -1521,8 +1533,8 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
     }
     const int64_t L = mmax * b;
     const size_t es = dt == FPM_F64 ? 8 : 4;
-    const SplitScheme sch = (SplitScheme)ctx->f32_scheme;
-    const size_t op = sch == SplitScheme::F16X3 ? 2 : 4;
+    const SplitScheme sch = scheme_for(ctx, b);
+    const size_t op = op_bytes(sch);
     // the kernel as the k-loop runs it: f fused pivots per update (K = f b)
     const int f = fuse_factor(ctx, dt, b);
     const int64_t fb = (int64_t)f * b;
@@ -1613,8 +1625,8 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 launch_split_cols(static_cast<const float*>(s.Bp), L, fb, Lx, sch, s.bh, s.bl, s.sb, st);
                 UpdateArgs a;
                 a.a_hi = s.ah; a.a_lo = s.al; a.bt_hi = s.bh; a.bt_lo = s.bl;
-                a.sa = sch == SplitScheme::F16X3 ? s.sa : nullptr;
-                a.sb = sch == SplitScheme::F16X3 ? s.sb : nullptr;
+                a.sa = has_scales(sch) ? s.sa : nullptr;
+                a.sb = has_scales(sch) ? s.sb : nullptr;
                 a.C = static_cast<float*>(s.C);
                 a.M = Lx; a.Nc = Lx; a.K = fb; a.ldc = Lx;
                 a.scheme = sch;
@@ -1910,7 +1922,8 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value == 0 || value == 1, "graph must be 0 or 1");
             ctx->graph = (int)value;
         } else if (k == "f32_scheme") {
-            FPM_CHECK_ARG(value == 0 || value == 1, "f32_scheme must be 0 or 1");
+            FPM_CHECK_ARG(value == -1 || value == 0 || value == 1 || value == 3,
+                          "f32_scheme must be -1 (auto), 0 (F16X3), 1 (TF32X3) or 3 (F16I8)");
             if (ctx->f32_scheme != (int)value) ctx->have_problem = false;  // operand buffers change size
             ctx->f32_scheme = (int)value;
         } else if (k == "cta_group") {
@@ -2104,8 +2117,8 @@ extern "C" int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, co
 extern "C" int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64_t K, int32_t scheme, void* hi,
                                void* lo, float* inv_scale, void* stream) {
     return guarded([&] {
-        FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
-        FPM_CHECK_ARG(scheme == 1 || inv_scale != nullptr, "F16X3 needs inv_scale");
+        FPM_CHECK_ARG(scheme == 0 || scheme == 1 || scheme == 3, "scheme must be 0, 1 or 3");
+        FPM_CHECK_ARG(scheme == 1 || inv_scale != nullptr, "F16X3 / F16I8 need inv_scale");
         fpm::launch_split_rows(src, ld, rows, K, (fpm::SplitScheme)scheme, hi, lo, inv_scale,
                                static_cast<cudaStream_t>(stream));
     });
@@ -2114,7 +2127,7 @@ extern "C" int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64
 extern "C" int fpm_k_split_cols_f32(const float* src, int64_t ld, int64_t K, int64_t W, int32_t scheme, void* hi,
                                     void* lo, float* inv_scale, void* stream) {
     return guarded([&] {
-        FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
+        FPM_CHECK_ARG(scheme == 0 || scheme == 1 || scheme == 3, "scheme must be 0, 1 or 3");
         fpm::launch_split_cols(src, ld, K, W, (fpm::SplitScheme)scheme, hi, lo, inv_scale,
                                static_cast<cudaStream_t>(stream));
     });
@@ -2138,14 +2151,14 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
                                 int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms, int32_t accumulate,
                                 int32_t variant, void* stream) {
     return guarded([&] {
-        FPM_CHECK_ARG(scheme == 0 || scheme == 1, "scheme must be 0 or 1");
+        FPM_CHECK_ARG(scheme >= 0 && scheme <= 3, "scheme must be 0, 1, 2 (int8 timing probe) or 3");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
         FPM_CHECK_ARG(variant >= -1 && variant <= 4, "variant must be -1 (auto) or 0..4");
-        FPM_CHECK_ARG(scheme == 1 || (sa && sb), "F16X3 needs sa and sb");
+        FPM_CHECK_ARG(scheme == 1 || scheme == 2 || (sa && sb), "F16X3 / F16I8 need sa and sb");
         fpm::UpdateArgs a;
         a.a_hi = a_hi; a.a_lo = a_lo; a.bt_hi = bt_hi; a.bt_lo = bt_lo;
-        a.sa = scheme == 0 ? sa : nullptr;
-        a.sb = scheme == 0 ? sb : nullptr;
+        a.sa = (scheme == 0 || scheme == 3) ? sa : nullptr;
+        a.sb = (scheme == 0 || scheme == 3) ? sb : nullptr;
         a.C = C; a.M = M; a.Nc = Nc; a.K = K; a.ldc = ldc;
         a.scheme = (fpm::SplitScheme)scheme;
         a.cta_group = cta_group;
