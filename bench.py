@@ -111,7 +111,7 @@ def committed_traffic(N: int, b: int, args):
     """DRAM bytes per update launch from the committed ncu capture of the same
     configuration (profiles/ncu_traffic.json), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    variant = (3 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
+    variant = (0 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
     key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}")
     if args.gpus != 1 or not os.path.exists(path):

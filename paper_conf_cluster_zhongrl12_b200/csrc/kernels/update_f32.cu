@@ -375,7 +375,7 @@ struct HybCfg {
     static constexpr uint32_t IDESC_I = ptx::idesc_s32acc_s8(TILE_M, BN);
     static constexpr int THREADS = 320;  // producer, MMA, 8 epilogue warps
     static_assert(SW == 128 || SW == 64, "swizzle width");
-    static_assert(NCB % 2 == 0 && NCBH >= 2 && NCBH <= 4, "C ring: 2..4 chunks per half");
+    static_assert(NCB % 2 == 0 && NCBH >= 1 && NCBH <= 4, "C ring: 1..4 chunks per half");
     static_assert(SMEM <= 232448, "shared memory budget");
 };
 
@@ -525,14 +525,14 @@ __global__ void __launch_bounds__(320, 1)
             const uint32_t t_row = tmem_base + ((q * 32) << 16) + hh * 128;
             uint32_t u[128];
 #pragma unroll
-            for (int c = 0; c < 4; ++c) {
-                uint32_t ti[32];
-                ptx::tmem_ld_32x32b_x32_nw(t_row + 32 * c, &u[32 * c]);
-                ptx::tmem_ld_32x32b_x32_nw(t_row + 256 + 32 * c, ti);
+            for (int c = 0; c < 8; ++c) {
+                uint32_t ti[16];
+                ptx::tmem_ld_32x32b_x16_nw(t_row + 16 * c, &u[16 * c]);
+                ptx::tmem_ld_32x32b_x16_nw(t_row + 256 + 16 * c, ti);
                 ptx::tmem_wait_ld();
 #pragma unroll
-                for (int j = 0; j < 32; ++j)
-                    u[32 * c + j] = __float_as_uint(fmaf(32.0f, (float)(int)ti[j], __uint_as_float(u[32 * c + j])));
+                for (int j = 0; j < 16; ++j)
+                    u[16 * c + j] = __float_as_uint(fmaf(32.0f, (float)(int)ti[j], __uint_as_float(u[16 * c + j])));
             }
             ptx::tc_fence_before();
             __syncwarp();
@@ -588,13 +588,23 @@ __global__ void __launch_bounds__(320, 1)
                 if (eh == 0) {
                     ptx::tma_store_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0, ptx::kEvictFirst);
                     ptx::bulk_commit();
-                    const int nxt = c - 1 + Cfg::NCBH;  // refill the buffer of chunk c - 1
-                    if (P.load_c && c >= 1 && nxt < 4) {
-                        const int nb = (c - 1) % Cfg::NCBH;
-                        ptx::bulk_wait_read1();
-                        ptx::mbar_arrive_expect_tx(&cf[nb], Cfg::C_CHUNK_BYTES);
-                        ptx::tma_load_2d(cb + nb * Cfg::C_CHUNK_BYTES, &tmC, &cf[nb], n0 + 32 * nxt, m0,
-                                         ptx::kEvictFirst);
+                    if constexpr (Cfg::NCBH == 1) {
+                        // one buffer per half: the next chunk's load waits for this store to read it
+                        // (the C read-modify-write is off the MMA's critical path)
+                        if (P.load_c && c + 1 < 4) {
+                            ptx::bulk_wait_read0();
+                            ptx::mbar_arrive_expect_tx(&cf[0], Cfg::C_CHUNK_BYTES);
+                            ptx::tma_load_2d(cb, &tmC, &cf[0], n0 + 32 * (c + 1), m0, ptx::kEvictFirst);
+                        }
+                    } else {
+                        const int nxt = c - 1 + Cfg::NCBH;  // refill the buffer of chunk c - 1
+                        if (P.load_c && c >= 1 && nxt < 4) {
+                            const int nb = (c - 1) % Cfg::NCBH;
+                            ptx::bulk_wait_read1();
+                            ptx::mbar_arrive_expect_tx(&cf[nb], Cfg::C_CHUNK_BYTES);
+                            ptx::tma_load_2d(cb + nb * Cfg::C_CHUNK_BYTES, &tmC, &cf[nb], n0 + 32 * nxt, m0,
+                                             ptx::kEvictFirst);
+                        }
                     }
                 }
             }
@@ -769,10 +779,10 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
         FPM_CHECK_ARG(a.sa != nullptr && a.sb != nullptr, "F16I8 needs sa and sb");
         switch (a.variant) {
             case 0: launch_update_hyb_t<128, 2, 4>(a, st); break;  // 2 x 64 KB stages, 4 C chunks (192 KB)
-            case 1: launch_update_hyb_t<64, 4, 4>(a, st); break;   // 4 x 32 KB stages, 4 C chunks (192 KB)
+            case 1: launch_update_hyb_t<128, 3, 2>(a, st); break;  // 3 x 64 KB stages, 2 C chunks (224 KB)
             case 2: launch_update_hyb_t<128, 2, 6>(a, st); break;  // 2 x 64 KB stages, 6 C chunks (224 KB)
             case 3: launch_update_hyb_t<64, 5, 4>(a, st); break;   // 5 x 32 KB stages, 4 C chunks (224 KB)
-            default: launch_update_hyb_t<64, 5, 4>(a, st);
+            default: launch_update_hyb_t<128, 2, 4>(a, st);  // variant 0 (measured best, c5: 520 vs 490 TFLOP/s)
         }
         return;
     }
