@@ -276,9 +276,14 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
                int32_t nsizes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out);
 
 /* Tuning / selection knobs (all optional):
- *   "f32_scheme": 0 = F16X3 (default: x 2^e = h0 + h1 in fp16, per-row
- *                 power-of-two scales, 3 kind::f16 MMAs), 1 = TF32X3
- *                 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  DESIGN.md Q15.
+ *   "f32_scheme": -1 = auto (default): 3 when b % 64 == 0 and cta_group is
+ *                 2, else 0.  3 = F16I8 (x 2^e = h0 + h1, h0 fp16 with a
+ *                 per-row power-of-two scale; int8 codes q = rint(x 2^e / 256),
+ *                 l = rint(8 h1); one kind::f16 MMA for h0 h0' and one kind::i8
+ *                 MMA for 32 (q l' + l q'); error fixed-point relative to the
+ *                 row maximum, ~2^-18; Q15b).  0 = F16X3 (h0, h1 both
+ *                 fp16, 3 kind::f16 MMAs, 2^-22 relative to each element).
+ *                 1 = TF32X3 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  Q15.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
  *   "kernel_variant": -1 (auto, default) or 0..3, see fpm_k_update_f32.
  *   "fuse":       pivots fused into one rank-(f b) update (FP32): 0 = auto
@@ -363,6 +368,10 @@ int pmm_set_device_option(pmm_ctx* ctx, int32_t dev, const char* key, int64_t va
  * tensor cores (reading Q15).  scheme 0 (F16X3): hi/lo are fp16 rows x K,
  * inv_scale[rows] receives 2^-e of each row.  scheme 1 (TF32X3): hi/lo are
  * fp32 rows x K holding tf32 values; inv_scale unused (may be NULL).
+ * scheme 3 (F16I8, Q15b): hi = fp16 h0 rows x K; lo = int8 codes, 2 K bytes
+ * per row, one 128-byte row [q of 64 | l of 64] per 64-wide k-block (the
+ * fpm_k_split_cols_f32 output is [l | q], so one int8 product of the two
+ * gives both cross terms); K % 64 == 0.
  * K % 4 == 0, ld % 4 == 0. */
 int fpm_k_split_f32(const float* src, int64_t ld, int64_t rows, int64_t K, int32_t scheme,
                     void* hi, void* lo, float* inv_scale, void* stream);
@@ -387,6 +396,12 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * k-blocks x 3 stages + 2 C chunks in flight, 1 = 64-byte x 4 + 6, 2 = 128-byte
  * x 2 + 6, 3 = 64-byte x 5 + 4, 4 = 128-byte x 2 + 4 (leaves ~36 KB smem per
  * SM for NCCL / staging kernels co-running with the update); -1 = auto (4).
+ * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
+ * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks (auto),
+ * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4.
+ * scheme 2 is a timing probe (int8 operands, three kind::i8 MMAs per k-step,
+ * s32 accumulator converted to float): it measures the int8 tensor path, its
+ * result is not a product of FP32 operands.
  * Requires K % 8 == 0, ldc % 4 == 0. */
 int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, const void* bt_lo,
                      const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,

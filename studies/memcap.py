@@ -174,7 +174,7 @@ def main():
         "config": {"b": b, "ns": ns, "p": p, "names": names, "sm_caps": caps, "c_cap_bytes": c_caps,
                    "ncal": args.ncal, "x_cal": x_cal, "sizes": sizes, "ooc_keep": args.ooc_keep, "ooc_buffers": args.ooc_buffers,
                    "sampling": "concurrent (all devices at once)" if args.concurrent else "exclusive",
-                   "dtype": "f32 (F16X3)", "sm_partition": args.sm_partition,
+                   "dtype": "f32 (auto scheme: F16I8 for b % 64 == 0, DESIGN Q15b)", "sm_partition": args.sm_partition,
                    "gpu": "1x B200; devices emulated by SM caps, device memory by C caps (C_i out of core above)"},
         "pcie": pcie, "fpm_sample_s": t_sample, "models": sample_info, "table": table,
     }

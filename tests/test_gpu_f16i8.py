@@ -175,3 +175,17 @@ def test_update_f16i8_rejects_ragged_k():
     C = torch.zeros((M, Nc), device="cuda")
     with pytest.raises(pkg.FpmError):
         pkg.k_update_f32(h, z, h, z, s, s, C, M, Nc, K, Nc, S, 2)
+
+
+def test_update_f16i8_intra_row_dynamic_range_is_normwise():
+    """Entries spanning 2^0 .. 2^-20 inside each row / column: F16I8's error is
+    bounded relative to the row and column maxima (reading Q15b), F16X3's
+    relative to the elements -- the documented difference between the two."""
+    M, Nc, K = 256, 320, 512
+    rng = np.random.default_rng(11)
+    A = (synth.rect(1, 4096, 0, 0, M, K).astype(np.float64) * 2.0 ** -rng.integers(0, 21, (M, K))).astype(np.float32)
+    B = (synth.rect(2, 4096, 0, 0, K, Nc).astype(np.float64) * 2.0 ** -rng.integers(0, 21, (K, Nc))).astype(np.float32)
+    C = _update(A, B, np.zeros((M, Nc), np.float32))
+    ref = og.gemm(A, B)
+    den = np.abs(A).astype(np.float64).max(1, keepdims=True) * np.abs(B).astype(np.float64).max(0, keepdims=True)
+    assert np.max(np.abs(C - ref) / den) <= K * 2.0 ** -16
