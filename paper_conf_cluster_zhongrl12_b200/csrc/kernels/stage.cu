@@ -418,7 +418,28 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
             slot_c = slot_c + 1 == F64_ST ? 0 : slot_c + 1;
         }
         // epilogue: this group's next chunks are already in flight, the other
-        // group keeps the DMMA pipe busy
+        // group keeps the DMMA pipe busy.  Interior tiles: the four C loads of
+        // a DMMA row are issued together (one global round trip per row, not
+        // one per element); edge tiles take the guarded path.
+        const bool interior = m0 + F64_BM <= M && n0 + F64_BN <= Nc && (ldc & 1) == 0 &&
+                              (reinterpret_cast<uintptr_t>(C) & 15) == 0;
+        if (interior) {
+#pragma unroll
+            for (int i = 0; i < 4; ++i) {
+                double2* rowp = reinterpret_cast<double2*>(C + (m0 + wm + i * 8 + lane / 4) * ldc + n0 + wn +
+                                                           2 * (lane % 4));
+                double2 c[4];
+#pragma unroll
+                for (int j = 0; j < 4; ++j) c[j] = accumulate ? __ldcs(rowp + 4 * j) : make_double2(0.0, 0.0);
+#pragma unroll
+                for (int j = 0; j < 4; ++j) {
+                    c[j].x += acc[i][j][0];
+                    c[j].y += acc[i][j][1];
+                    __stcs(rowp + 4 * j, c[j]);
+                }
+            }
+            continue;
+        }
 #pragma unroll
         for (int i = 0; i < 4; ++i)
 #pragma unroll

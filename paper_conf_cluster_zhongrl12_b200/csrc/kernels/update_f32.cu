@@ -87,7 +87,7 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
     tn = r / gm;
 }
 
-template <int CG, int KIND, int BN, int STAGES, int SW, int NCB>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1>
 __global__ void __launch_bounds__(192, 1)
     update_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
                   const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
@@ -201,9 +201,13 @@ __global__ void __launch_bounds__(192, 1)
 #pragma unroll
                         for (int k = 0; k < Cfg::KSTEPS; ++k) {
                             const uint64_t off = (uint64_t)(k * 32) >> 4;  // 32 B per MMA k-step
-                            ptx::umma<CG, KIND>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC, (kb | k) != 0);
-                            ptx::umma<CG, KIND>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
-                            ptx::umma<CG, KIND>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
+#pragma unroll
+                            for (int rep = 0; rep < MREP; ++rep) {  // MREP > 1: timing probe only
+                                ptx::umma<CG, KIND>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC,
+                                                    (kb | k | rep) != 0);
+                                ptx::umma<CG, KIND>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
+                                ptx::umma<CG, KIND>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
+                            }
                         }
                         ptx::umma_commit<CG>(&empty[stage]);
                     }
@@ -665,7 +669,7 @@ CUtensorMap make_tmap_2d(const void* base, CUtensorMapDataType dt, int elem_byte
     return m;
 }
 
-template <int CG, int KIND, int BN, int STAGES, int SW, int NCB>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1>
 static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = UpdCfg<CG, KIND, BN, STAGES, SW, NCB>;
     const CUtensorMapDataType odt = KIND == 1   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
@@ -688,7 +692,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.load_c = a.accumulate ? 1 : 0;
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
-    auto kern = update_kernel<CG, KIND, BN, STAGES, SW, NCB>;
+    auto kern = update_kernel<CG, KIND, BN, STAGES, SW, NCB, MREP>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;
     cudaGetDevice(&dev);
@@ -788,7 +792,8 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     }
     if (a.scheme == SplitScheme::I8PROBE) {  // timing probe: int8 operands, 3 x kind::i8 per k-step
         FPM_CHECK_ARG(a.cta_group == 2 && a.K % 128 == 0, "I8 probe: cta_group 2, K % 128 == 0");
-        launch_update_t<2, 2, 256, 2, 128, 4>(a, st);
+        if (a.variant == 1) launch_update_t<2, 2, 256, 2, 128, 4, 2>(a, st);  // twice the MMAs, same bytes
+        else launch_update_t<2, 2, 256, 2, 128, 4>(a, st);
         return;
     }
     // auto: variant 4 (two 64-KB operand stages, four C chunks in flight): as fast

@@ -48,6 +48,8 @@ q = lambda r, lim: torch.randint(-lim, lim + 1, (r, 2 * K), device=dev, dtype=to
 qa, qla, qb, qlb = q(M, 127), q(M, 64), q(N, 127), q(N, 64)
 res.append(run("i8x3 K=4096 (same bytes)", lambda: pkg.k_update_f32(qa, qla, qb, qlb, sa, sb, C, M, N, 2 * K, N, scheme=2),
                3 * 2 * M * N * 2 * K))
+res.append(run("i8x6 K=4096 (same bytes, twice the MMAs)", lambda: pkg.k_update_f32(qa, qla, qb, qlb, sa, sb, C, M, N, 2 * K, N, scheme=2, variant=1),
+               6 * 2 * M * N * 2 * K))
 res.append(run("f16x3 K=2048 again", lambda: pkg.k_update_f32(ah, al, bh, bl, sa, sb, C, M, N, K, N, scheme=0), 3 * 2 * M * N * K))
 os.makedirs("gpurun_out", exist_ok=True)
 json.dump(res, open("gpurun_out/i8_energy.json", "w"), indent=1)
