@@ -398,7 +398,9 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * SM for NCCL / staging kernels co-running with the update); -1 = auto (4).
  * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
  * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks (auto),
- * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4.
+ * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 4 = variant
+ * 0 on clusters of two CTA pairs that multicast the B^T tiles (grid = the
+ * co-resident clusters of 4).
  * scheme 2 is a timing probe (int8 operands, three kind::i8 MMAs per k-step,
  * s32 accumulator converted to float): it measures the int8 tensor path, its
  * result is not a product of FP32 operands.
@@ -407,6 +409,14 @@ int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* bt_hi, cons
                      const float* sa, const float* sb, float* C, int64_t M, int64_t Nc, int64_t K,
                      int64_t ldc, int32_t scheme, int32_t cta_group, int32_t num_sms,
                      int32_t accumulate, int32_t variant, void* stream);
+
+/* Diagnostic counters of the F16I8 update's MMA issuer (the leader CTA of
+ * each pair, lane 0; clock64 cycles summed over CTAs and launches): op 1 =
+ * reset and enable for subsequent launches, 0 = disable, 2 = read into
+ * out[4] = {cycles waiting for TMEM (the epilogue's drain of the previous tile),
+ * cycles waiting for operands (TMA), cycles of the issuer loop, tiles}.
+ * Current CUDA device; synchronise before reading. */
+int fpm_k_prof(int32_t op, uint64_t* out);
 
 /* Rank-b update in FP64 on DMMA: C (M x Nc, ldc) (+)= A (M x K, lda) x Bt^T,
  * Bt (Nc x K); accumulate = 0 overwrites C. */

@@ -254,6 +254,16 @@ def k_update_f32(a_hi, a_lo, bt_hi, bt_lo, sa, sb, C, M, Nc, K, ldc, scheme=SCHE
                                num_sms, 1 if accumulate else 0, variant, _stream(stream)))
 
 
+def k_prof(op: int):
+    """F16I8 MMA-issuer wait counters (fpm_k_prof): op 1 reset + enable, 0 disable,
+    2 read -> dict(tmem_wait, operand_wait, issuer, tiles) in cycles summed over CTAs."""
+    out = (ctypes.c_uint64 * 4)()
+    check(lib.fpm_k_prof(op, out))
+    if op == 2:
+        return {"tmem_wait": out[0], "operand_wait": out[1], "issuer": out[2], "tiles": out[3]}
+    return None
+
+
 def k_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate=True, stream=None):
     check(lib.fpm_k_update_f64(_lib._ptr(A), lda, _lib._ptr(Bt), _lib._ptr(C), M, Nc, K, ldc,
                                1 if accumulate else 0, _stream(stream)))

@@ -116,6 +116,7 @@ _SIGS = {
     "fpm_k_update_f32": ([vp, vp, vp, vp, vp, vp, vp, i64, i64, i64, i64, i32, i32, i32, i32, i32, vp],
                          ctypes.c_int),
     "fpm_k_update_f64": ([vp, i64, vp, vp, i64, i64, i64, i64, i32, vp], ctypes.c_int),
+    "fpm_k_prof": ([i32, ctypes.POINTER(u64)], ctypes.c_int),
     "fpm_k_fill_synthetic": ([vp, i32, i64, u64, i64, i64, i64, i64, i64, i32, vp], ctypes.c_int),
 }
 for _name, (_args, _res) in _SIGS.items():

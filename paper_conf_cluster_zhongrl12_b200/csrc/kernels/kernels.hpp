@@ -38,6 +38,9 @@ struct UpdateArgs {
 };
 
 // C += A . Bt^T  (the rank-b update)
+// Diagnostic counters of the F16I8 MMA issuer: op 1 = reset + enable, 0 = disable,
+// 2 = read the 4 counters (current device) into out.
+void update_prof(int op, unsigned long long* out);
 void launch_update_f32(const UpdateArgs& a, cudaStream_t st);
 
 // Split an FP32 panel (rows x K, row stride ld) into the two operand halves.

@@ -99,6 +99,18 @@ __device__ __forceinline__ void tma_load_2d_cg2(void* smem_dst, const void* tmap
         "l"(reinterpret_cast<uint64_t>(tmap)), "r"(bar_leader), "r"(c0), "r"(c1), "l"(cache_hint)
         : "memory");
 }
+// 2-SM variant with multicast: the box lands at the same smem offset in every
+// CTA of `mask`; each destination's complete_tx goes to the barrier of the
+// leader CTA of that destination's pair.
+__device__ __forceinline__ void tma_load_2d_cg2_mc(void* smem_dst, const void* tmap, uint64_t* bar, int32_t c0,
+                                                   int32_t c1, uint16_t mask, uint64_t cache_hint) {
+    const uint32_t bar_leader = smem_u32(bar) & 0xFEFFFFFFu;
+    asm volatile(
+        "cp.async.bulk.tensor.2d.cta_group::2.shared::cluster.global.mbarrier::complete_tx::bytes.multicast::cluster"
+        ".L2::cache_hint [%0], [%1, {%3, %4}], [%2], %5, %6;" ::"r"(smem_u32(smem_dst)),
+        "l"(reinterpret_cast<uint64_t>(tmap)), "r"(bar_leader), "r"(c0), "r"(c1), "h"(mask), "l"(cache_hint)
+        : "memory");
+}
 __device__ __forceinline__ void tma_store_2d(const void* tmap, const void* smem_src, int32_t c0, int32_t c1) {
     asm volatile("cp.async.bulk.tensor.2d.global.shared::cta.bulk_group [%0, {%2, %3}], [%1];" ::"l"(
                      reinterpret_cast<uint64_t>(tmap)),
@@ -201,6 +213,15 @@ __device__ __forceinline__ void umma_commit(uint64_t* bar) {
                 smem_u32(bar)),
             "h"((uint16_t)0x3)
             : "memory");
+}
+
+// cta_group::2 commit arriving on `bar` in every CTA of `mask` (cluster ranks).
+__device__ __forceinline__ void umma_commit_mask(uint64_t* bar, uint16_t mask) {
+    asm volatile(
+        "tcgen05.commit.cta_group::2.mbarrier::arrive::one.shared::cluster.multicast::cluster.b64 [%0], %1;" ::"r"(
+            smem_u32(bar)),
+        "h"(mask)
+        : "memory");
 }
 
 // 32 lanes x 32 consecutive 32-bit columns: thread t gets row (lane base + t).

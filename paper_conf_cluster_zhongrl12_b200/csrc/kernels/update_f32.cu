@@ -72,7 +72,15 @@ struct UpdParams {
     int load_c;       // 1: C += A B^T (read-modify-write), 0: C = A B^T (first iteration)
     int group;        // raster group (tile-rows)
     uint64_t hint_b;  // L2 policy of the B^T tiles (A tiles: evict_last, C: evict_first)
+    int prof;         // F16I8: accumulate MMA-issuer wait cycles into g_hyb_prof (fpm_k_prof)
 };
+
+// Diagnostic counters of the F16I8 MMA issuer (leader CTAs, lane 0), summed over
+// the CTAs of every profiled launch: [0] cycles waiting for TMEM (the epilogue's
+// drain), [1] cycles waiting for operands (TMA), [2] cycles of the issuer loop,
+// [3] tiles.
+__device__ unsigned long long g_hyb_prof[4];
+static bool g_prof_on = false;
 
 // Grouped raster over tiles so concurrently running CTAs share A / B tiles in L2:
 // groups of G tile-rows, column-major inside a group (A rows of the group stay
@@ -383,7 +391,12 @@ struct HybCfg {
     static_assert(SMEM <= 232448, "shared memory budget");
 };
 
-template <int SW, int STAGES, int NCB>
+// MC = 2: clusters of two CTA pairs stacked along M (tile-rows 2 i and 2 i + 1)
+// sharing the B^T tiles: each CTA loads a quarter of the pair's B^T rows and
+// multicasts it to the CTA in the same position of the other pair, so the L2
+// reads of B^T halve (A: unchanged).  A stage's smem is then written by two
+// producers, so its release waits for both pairs' MMAs (empty count 2).
+template <int SW, int STAGES, int NCB, int MC = 1>
 __global__ void __launch_bounds__(320, 1)
     update_hyb_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_8,
                       const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_8,
@@ -403,15 +416,20 @@ __global__ void __launch_bounds__(320, 1)
 
     const uint32_t warp = threadIdx.x / 32;
     const uint32_t lane = threadIdx.x % 32;
-    const uint32_t rank = ptx::cluster_ctarank();
+    const uint32_t crank = ptx::cluster_ctarank();
+    const uint32_t rank = crank & 1;        // position in the CTA pair
+    const uint32_t pr = crank >> 1;         // pair of the cluster (MC = 2)
     const bool leader = rank == 0;
-    const int cluster_id = blockIdx.x / 2;
-    const int num_clusters = gridDim.x / 2;
+    const int cluster_id = blockIdx.x / (2 * MC);
+    const int num_clusters = gridDim.x / (2 * MC);
+    const int tiles_mc = (P.tiles_m + MC - 1) / MC;  // cluster tiles: MC tile-rows each
+    const int num_ct = tiles_mc * P.tiles_n;
+    const int group = P.group / MC > 0 ? P.group / MC : 1;
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
             ptx::mbar_init(&full[s], 1);
-            ptx::mbar_init(&empty[s], 1);
+            ptx::mbar_init(&empty[s], MC);
         }
         ptx::mbar_init(tfull, 1);
         ptx::mbar_init(tempty, 8 * 2);  // every epilogue warp of both CTAs
@@ -441,11 +459,12 @@ __global__ void __launch_bounds__(320, 1)
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+            for (int t = cluster_id; t < num_ct; t += num_clusters) {
                 int tm, tn;
-                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+                tile_coords(t, tiles_mc, P.tiles_n, group, tm, tn);
+                tm = tm * MC + (int)pr;
                 const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
-                const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA;
+                const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA + (int)pr * (Cfg::BN_CTA / MC);
                 for (int kb = 0; kb < num_kb; ++kb) {
                     ptx::mbar_wait(&empty[stage], phase ^ 1);
                     uint8_t* sA_hi = stage_base + stage * Cfg::STAGE_BYTES;
@@ -456,8 +475,15 @@ __global__ void __launch_bounds__(320, 1)
                     if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
                     ptx::tma_load_2d_cg2(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
                     ptx::tma_load_2d_cg2(sA_8, &tmA_8, &full[stage], kb * SW, m0, ptx::kEvictLast);
-                    ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
-                    ptx::tma_load_2d_cg2(sB_8, &tmB_8, &full[stage], kb * SW, n0, P.hint_b);
+                    if constexpr (MC == 1) {
+                        ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
+                        ptx::tma_load_2d_cg2(sB_8, &tmB_8, &full[stage], kb * SW, n0, P.hint_b);
+                    } else {  // this CTA's quarter of the B^T rows, to itself and its counterpart
+                        const uint16_t mask = (uint16_t)((1u << rank) | (1u << (rank + 2)));
+                        const int off = (int)pr * (Cfg::BN_CTA / MC) * SW;
+                        ptx::tma_load_2d_cg2_mc(sB_hi + off, &tmB_hi, &full[stage], k0, n0, mask, P.hint_b);
+                        ptx::tma_load_2d_cg2_mc(sB_8 + off, &tmB_8, &full[stage], kb * SW, n0, mask, P.hint_b);
+                    }
                     if (++stage == STAGES) { stage = 0; phase ^= 1; }
                 }
             }
@@ -468,11 +494,17 @@ __global__ void __launch_bounds__(320, 1)
             int stage = 0;
             uint32_t phase = 0;
             int it = 0;
-            for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
+            long long w_tmem = 0, w_ops = 0;
+            const long long t_begin = clock64();
+            for (int t = cluster_id; t < num_ct; t += num_clusters, ++it) {
+                long long c0 = P.prof ? clock64() : 0;
                 ptx::mbar_wait(tempty, (it & 1) ^ 1);
+                if (P.prof) w_tmem += clock64() - c0;
                 ptx::tc_fence_after();
                 for (int kb = 0; kb < num_kb; ++kb) {
+                    if (P.prof) c0 = clock64();
                     ptx::mbar_wait(&full[stage], phase);
+                    if (P.prof) w_ops += clock64() - c0;
                     ptx::tc_fence_after();
                     if (lane == 0) {
                         const uint32_t a_hi = ptx::smem_u32(stage_base + stage * Cfg::STAGE_BYTES);
@@ -487,13 +519,19 @@ __global__ void __launch_bounds__(320, 1)
                             ptx::umma<2, 0>(tmem_base, dA_hi + off, dB_hi + off, Cfg::IDESC_F, (kb | k) != 0);
                             ptx::umma<2, 2>(tmem_base + 256, dA_8 + off, dB_8 + off, Cfg::IDESC_I, (kb | k) != 0);
                         }
-                        ptx::umma_commit<2>(&empty[stage]);
+                        ptx::umma_commit_mask(&empty[stage], MC == 1 ? 0x3 : 0xF);  // every producer writing the slot
                     }
                     __syncwarp();
                     if (++stage == STAGES) { stage = 0; phase ^= 1; }
                 }
-                if (lane == 0) ptx::umma_commit<2>(tfull);
+                if (lane == 0) ptx::umma_commit_mask(tfull, (uint16_t)(0x3u << (2 * pr)));
                 __syncwarp();
+            }
+            if (P.prof && lane == 0) {
+                atomicAdd(&g_hyb_prof[0], (unsigned long long)w_tmem);
+                atomicAdd(&g_hyb_prof[1], (unsigned long long)w_ops);
+                atomicAdd(&g_hyb_prof[2], (unsigned long long)(clock64() - t_begin));
+                atomicAdd(&g_hyb_prof[3], (unsigned long long)it);
             }
         }
     } else {
@@ -508,9 +546,10 @@ __global__ void __launch_bounds__(320, 1)
         uint64_t* cf = cfull + hh * Cfg::NCBH;
         uint32_t cpar = 0;
         int it = 0;
-        for (int t = cluster_id; t < P.num_tiles; t += num_clusters, ++it) {
+        for (int t = cluster_id; t < num_ct; t += num_clusters, ++it) {
             int tm, tn;
-            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+            tile_coords(t, tiles_mc, P.tiles_n, group, tm, tn);
+            tm = tm * MC + (int)pr;
             const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
             const int n0 = tn * Cfg::BN + (int)hh * 128;
             if (eh == 0 && P.load_c) {
@@ -540,7 +579,7 @@ __global__ void __launch_bounds__(320, 1)
             }
             ptx::tc_fence_before();
             __syncwarp();
-            if (lane == 0) ptx::mbar_arrive_cluster(tempty, 0);
+            if (lane == 0) ptx::mbar_arrive_cluster(tempty, 2 * pr);
             // C read-modify-write (overlaps the next tile's mainloop)
 #pragma unroll
             for (int c = 0; c < 4; ++c) {
@@ -692,6 +731,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.load_c = a.accumulate ? 1 : 0;
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
+    P.prof = 0;
     auto kern = update_kernel<CG, KIND, BN, STAGES, SW, NCB, MREP>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;
@@ -720,15 +760,15 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
 }
 
-template <int SW, int STAGES, int NCB>
+template <int SW, int STAGES, int NCB, int MC = 1>
 static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = HybCfg<SW, STAGES, NCB>;
     const CUtensorMap tAh = make_tmap_2d(a.a_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
     const CUtensorMap tA8 = make_tmap_2d(a.a_lo, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, a.M, 2 * a.K, 2 * a.K, SW, Cfg::BM);
     const CUtensorMap tBh =
-        make_tmap_2d(a.bt_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+        make_tmap_2d(a.bt_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA / MC);
     const CUtensorMap tB8 =
-        make_tmap_2d(a.bt_lo, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, a.Nc, 2 * a.K, 2 * a.K, SW, Cfg::BN_CTA);
+        make_tmap_2d(a.bt_lo, CU_TENSOR_MAP_DATA_TYPE_UINT8, 1, a.Nc, 2 * a.K, 2 * a.K, SW, Cfg::BN_CTA / MC);
     const CUtensorMap tC = make_tmap_2d(a.C, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.M, a.Nc, a.ldc, 32, Cfg::BM);
     UpdParams P;
     P.M = (int)a.M;
@@ -742,32 +782,60 @@ static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
     P.load_c = a.accumulate ? 1 : 0;
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
-    auto kern = update_hyb_kernel<SW, STAGES, NCB>;
+    P.prof = g_prof_on ? 1 : 0;
+    auto kern = update_hyb_kernel<SW, STAGES, NCB, MC>;
     static uint64_t attr_done = 0;
+    static int max_clusters[64] = {};  // co-resident clusters of 2 MC CTAs, per device
     int dev = 0;
     cudaGetDevice(&dev);
-    if (!(attr_done & (1ull << dev))) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
-        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
-        attr_done |= 1ull << dev;
-    }
-    int clusters = a.num_sms / 2;
-    if (clusters > P.num_tiles) clusters = P.num_tiles;
-    if (clusters < 1) clusters = 1;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(clusters * 2);
     cfg.blockDim = dim3(Cfg::THREADS);
     cfg.dynamicSmemBytes = Cfg::SMEM;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.x = 2 * MC;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    if (!(attr_done & (1ull << dev))) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+        if (MC > 1) {
+            // a persistent grid must be co-resident: clusters of 4 do not tile every GPC
+            int sms = 0;
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            cfg.gridDim = dim3((unsigned)(sms / (2 * MC) * 2 * MC));
+            int n = 0;
+            e = cudaOccupancyMaxActiveClusters(&n, kern, &cfg);
+            if (e != cudaSuccess || n < 1) fail(FPM_ECUDA, "cudaOccupancyMaxActiveClusters: %s", cudaGetErrorString(e));
+            if (dev < 64) max_clusters[dev] = n;
+        }
+        attr_done |= 1ull << dev;
+    }
+    const int num_ct = ((P.tiles_m + MC - 1) / MC) * P.tiles_n;
+    int clusters = a.num_sms / (2 * MC);
+    if (MC > 1 && dev < 64 && max_clusters[dev] > 0 && clusters > max_clusters[dev]) clusters = max_clusters[dev];
+    if (clusters > num_ct) clusters = num_ct;
+    if (clusters < 1) clusters = 1;
+    cfg.gridDim = dim3(clusters * 2 * MC);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tAh, tA8, tBh, tB8, tC, P);
     if (e != cudaSuccess) fail(FPM_ECUDA, "F16I8 update kernel launch: %s", cudaGetErrorString(e));
+}
+
+void update_prof(int op, unsigned long long* out) {
+    if (op == 1) {
+        const unsigned long long z[4] = {0, 0, 0, 0};
+        const cudaError_t e = cudaMemcpyToSymbol(g_hyb_prof, z, sizeof(z));
+        if (e != cudaSuccess) fail(FPM_ECUDA, "prof reset: %s", cudaGetErrorString(e));
+        g_prof_on = true;
+    } else if (op == 0) {
+        g_prof_on = false;
+    } else {
+        const cudaError_t e = cudaMemcpyFromSymbol(out, g_hyb_prof, 4 * sizeof(unsigned long long));
+        if (e != cudaSuccess) fail(FPM_ECUDA, "prof read: %s", cudaGetErrorString(e));
+    }
 }
 
 void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
@@ -786,6 +854,7 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
             case 1: launch_update_hyb_t<128, 3, 2>(a, st); break;  // 3 x 64 KB stages, 2 C chunks (224 KB)
             case 2: launch_update_hyb_t<128, 2, 6>(a, st); break;  // 2 x 64 KB stages, 6 C chunks (224 KB)
             case 3: launch_update_hyb_t<64, 5, 4>(a, st); break;   // 5 x 32 KB stages, 4 C chunks (224 KB)
+            case 4: launch_update_hyb_t<128, 2, 4, 2>(a, st); break;  // variant 0 on clusters of 2 pairs, B multicast
             default: launch_update_hyb_t<128, 2, 4>(a, st);  // variant 0 (measured best, c5: 520 vs 490 TFLOP/s)
         }
         return;

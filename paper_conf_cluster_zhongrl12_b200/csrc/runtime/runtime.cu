@@ -2172,6 +2172,14 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
     });
 }
 
+extern "C" int fpm_k_prof(int32_t op, uint64_t* out) {
+    return guarded([&] {
+        FPM_CHECK_ARG(op >= 0 && op <= 2, "op must be 0, 1 or 2");
+        FPM_CHECK_ARG(op != 2 || out != nullptr, "null out");
+        fpm::update_prof(op, reinterpret_cast<unsigned long long*>(out));
+    });
+}
+
 extern "C" int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, int64_t M, int64_t Nc,
                                 int64_t K, int64_t ldc, int32_t accumulate, void* stream) {
     return guarded([&] {
