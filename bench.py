@@ -334,8 +334,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             log("e2e failed:", repr(ex))
             e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:200]}
 
-    cpu = None
-    if rank == 0 and not args.no_cpu_baseline:
+    cpu = None  # the oracle baseline is timed at N = 1 only (rank 0); N > 1 lines carry null
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
         g, cores, desc, _ = oracle_sample(N)
         cpu = {"value": g, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc}
 
