@@ -147,6 +147,9 @@ def oracle_sample(N: int, reps: int = 1):
 def run_reference(args, rank: int):
     if rank != 0:
         return
+    # rank 0 alone runs: give the oracle every host core (torchrun exports OMP_NUM_THREADS=1)
+    from oracle import gemm as og
+    og.set_num_threads(len(os.sched_getaffinity(0)))
     N = args.N
     vals, times = [], []
     for i in range(args.warmup + args.steps):

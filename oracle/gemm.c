@@ -66,3 +66,15 @@ int oracle_num_threads(void)
     return 1;
 #endif
 }
+
+/* Thread count of the OpenMP loops above (timing only; the result does not
+ * depend on it).  bench.py's reference arm runs on rank 0 alone under
+ * torchrun, which exports OMP_NUM_THREADS=1. */
+void oracle_set_num_threads(int n)
+{
+#ifdef _OPENMP
+    if (n > 0) omp_set_num_threads(n);
+#else
+    (void)n;
+#endif
+}

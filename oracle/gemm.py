@@ -37,12 +37,19 @@ def _load():
             fn.argtypes = [i64, i64, i64, vp, i64, vp, i64, vp, i64]
             fn.restype = None
         lib.oracle_num_threads.restype = ctypes.c_int
+        lib.oracle_set_num_threads.argtypes = [ctypes.c_int]
+        lib.oracle_set_num_threads.restype = None
         _lib = lib
     return _lib
 
 
 def num_threads() -> int:
     return int(_load().oracle_num_threads())
+
+
+def set_num_threads(n: int) -> None:
+    """OpenMP threads of the oracle loops (timing only; results do not depend on it)."""
+    _load().oracle_set_num_threads(int(n))
 
 
 def gemm(A: np.ndarray, B: np.ndarray) -> np.ndarray:
