@@ -113,7 +113,8 @@ def committed_traffic(N: int, b: int, args):
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     variant = (0 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
-    key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}")
+    G = args.raster_group if args.raster_group > 0 else (12 if args.scheme == "f16i8" else 16)
+    key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}") + ("" if G == 16 else f"_r{G}")
     if args.gpus != 1 or not os.path.exists(path):
         return None
     entry = json.load(open(path)).get(key)
@@ -471,7 +472,7 @@ def main():
     ap.add_argument("--transport", choices=["ipc", "nccl"], default="ipc",
                     help="N > 1: pull pivots from peers' memory (ipc) or exchange them with NCCL")
     ap.add_argument("--cta-group", type=int, default=2)
-    ap.add_argument("--raster-group", type=int, default=16)
+    ap.add_argument("--raster-group", type=int, default=0, help="0 = auto (12 for F16I8, 16 otherwise)")
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")

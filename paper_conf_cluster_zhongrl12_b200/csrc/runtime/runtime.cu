@@ -141,7 +141,7 @@ struct pmm_ctx {
 
     int f32_scheme = -1;  // fpm::SplitScheme, -1 = auto (scheme_for)
     int cta_group = 2;
-    int raster_group = 16;
+    int raster_group = 0;  // 0 = auto: 12 for F16I8, 16 otherwise (measured, c5)
     int l2_hint_b = 0;
     int kernel_variant = -1;  // auto
     int fuse = 0;             // pivots per update (0 = auto)
@@ -881,7 +881,7 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.cta_group = ctx->cta_group;
     a.num_sms = d.num_sms;
     a.accumulate = ctx->groups[g].first != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
-    a.raster_group = ctx->raster_group;
+    a.raster_group = ctx->raster_group > 0 ? ctx->raster_group : (sch == SplitScheme::F16I8 ? 12 : 16);
     a.l2_hint_b = ctx->l2_hint_b;
     a.variant = ctx->kernel_variant;  // -1: auto (variant 4, leaves smem for co-running kernels)
     return a;
@@ -1632,7 +1632,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.scheme = sch;
                 a.cta_group = ctx->cta_group;
                 a.num_sms = s.d->num_sms;
-                a.raster_group = ctx->raster_group;
+                a.raster_group = ctx->raster_group > 0 ? ctx->raster_group : (sch == SplitScheme::F16I8 ? 12 : 16);
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
                 if (ooc) {
@@ -1964,7 +1964,7 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= 0 && value <= 2, "l2_hint_b must be 0 (normal), 1 (first) or 2 (last)");
             ctx->l2_hint_b = (int)value;
         } else if (k == "raster_group") {
-            FPM_CHECK_ARG(value >= 1 && value <= 4096, "raster_group must be in [1, 4096]");
+            FPM_CHECK_ARG(value >= 0 && value <= 4096, "raster_group must be 0 (auto) or in [1, 4096]");
             ctx->raster_group = (int)value;
         } else {
             fpm::fail(FPM_EINVAL, "unknown option '%s'", key);
