@@ -316,9 +316,19 @@ __global__ void __launch_bounds__(256) fill_k(T* dst, int64_t ld, uint64_t seed,
 // fragment loads (lane -> row lane/4, column lane%4) are conflict-free per
 // half-warp.  Measured (ncu, L = 8192, K = 512): the previous 128 x 128
 // single-group design kept the DMMA pipe 73 % busy.
+// K per cp.async chunk: 32 (2 stages, one group barrier per 32 K) measured 31.2
+// vs 30.4 TFLOP/s at L = 8192, K = 512 (config 1's fused K) and 20.7 vs 21.4 at
+// K = 64; 16 (3 stages) kept selectable.
+#ifndef FPM_F64_BK
+#define FPM_F64_BK 32
+#endif
+#if FPM_F64_BK == 32
+constexpr int F64_BM = 64, F64_BN = 128, F64_BK = 32, F64_LD = 36, F64_ST = 2, F64_GROUPS = 2;
+#else
 constexpr int F64_BM = 64, F64_BN = 128, F64_BK = 16, F64_LD = 20, F64_ST = 3, F64_GROUPS = 2;
+#endif
 constexpr int F64_GROUP_DOUBLES = F64_ST * (F64_BM + F64_BN) * F64_LD;
-constexpr int F64_SMEM = F64_GROUPS * F64_GROUP_DOUBLES * 8;  // 184320 B
+constexpr int F64_SMEM = F64_GROUPS * F64_GROUP_DOUBLES * 8;  // 184320 B (BK 16) / 221184 B (BK 32)
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool valid) {
     const uint32_t s = static_cast<uint32_t>(__cvta_generic_to_shared(smem));
@@ -354,13 +364,14 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
     auto advance_load = [&]() {
         if (lt < tiles) {
             const int64_t m0 = (lt / tiles_n) * F64_BM, n0 = (lt % tiles_n) * F64_BN, k0 = lkb * F64_BK;
-            // A: 64 rows x 16 doubles = 512 16-B chunks (2 per thread); B: 128 rows (4 per thread)
+            // A: 64 rows x BK doubles (BK / 2 16-B chunks per row); B: 128 rows
+            constexpr int CPR = F64_BK / 2, A_IT = F64_BM * CPR / 256, B_IT = F64_BN * CPR / 256;
 #pragma unroll
-            for (int it = 0; it < 6; ++it) {
+            for (int it = 0; it < A_IT + B_IT; ++it) {
                 const int idx = gtid + it * 256;
-                const bool isA = it < 2;
-                const int j = isA ? idx : idx - 512;
-                const int r = j / 8, c2 = (j % 8) * 2;
+                const bool isA = it < A_IT;
+                const int j = isA ? idx : idx - A_IT * 256;
+                const int r = j / CPR, c2 = (j % CPR) * 2;
                 const int64_t gk = k0 + c2;
                 const bool ka = gk < K;  // K even: a 2-element chunk is all in or all out
                 if (isA) {
