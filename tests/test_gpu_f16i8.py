@@ -189,3 +189,21 @@ def test_update_f16i8_intra_row_dynamic_range_is_normwise():
     ref = og.gemm(A, B)
     den = np.abs(A).astype(np.float64).max(1, keepdims=True) * np.abs(B).astype(np.float64).max(0, keepdims=True)
     assert np.max(np.abs(C - ref) / den) <= K * 2.0 ** -16
+
+
+def test_prof_counters_count_tiles_and_reset():
+    """fpm_k_prof: the MMA issuer's counters see every tile of a profiled launch,
+    stay at zero while disabled, and reset on enable."""
+    M, Nc, K = 512, 768, 128
+    A = synth.rect(1, 4096, 0, 0, M, K)
+    B = synth.rect(2, 4096, 0, 0, K, Nc)
+    pkg.k_prof(1)
+    _update(A, B, np.zeros((M, Nc), np.float32))
+    pr = pkg.k_prof(2)
+    pkg.k_prof(0)
+    assert pr["tiles"] == (M // 256) * (Nc // 256)          # 256 x 256 tiles, one count per CTA pair
+    assert 0 < pr["tmem_wait"] + pr["operand_wait"] <= pr["issuer"]
+    pkg.k_prof(1)
+    pkg.k_prof(0)
+    _update(A, B, np.zeros((M, Nc), np.float32))             # disabled: not counted
+    assert pkg.k_prof(2)["tiles"] == 0
