@@ -325,6 +325,15 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 row / column over all of them (maxima merged first), so each
  *                 band takes a single update and one read-modify-write of C;
  *                 0: one update per tail group and band.
+ *   "tail_stream": 1 (default): pmm_run on a context whose one device holds
+ *                 the whole problem uploads the fused tail's B rows first and
+ *                 its A rows band by band (a 4-byte-per-element staging buffer
+ *                 of H x tail_K), staging and updating each band as it lands,
+ *                 so the copy of C to the host overlaps the last uploads; the
+ *                 tail may then be longer (the uploads under the groups before
+ *                 it are 8 B per element for those groups + 4 B for the tail's
+ *                 B).  Same results bit for bit as 0 (all tail pivots uploaded
+ *                 before the tail starts).
  *   "sm_partition": how an SM cap is enforced.  0 (default): the cap is the
  *                 grid of the persistent update kernel (one CTA per SM); other
  *                 kernels of the device are not confined, and devices sharing a

@@ -112,6 +112,12 @@ struct Device {
     std::vector<void*> tail_allocs;
     cudaEvent_t ev_tpack0 = nullptr, ev_tpack1 = nullptr;  // staging of the fused tail (second pass)
     bool tail_fused_run = false;  // the current k-loop stages its tail into kFusedSlot
+    // band-streamed tail (pmm_run, one device holding all of A and B): the tail's
+    // A rows arrive band by band into tail_rows (H x tail_K, row-major)
+    bool tail_streamed_run = false;
+    float* tail_rows = nullptr;
+    std::vector<cudaEvent_t> ev_band_up, ev_band_st;  // per band: rows uploaded, rows staged
+    cudaEvent_t ev_tail_b = nullptr;                  // tail B rows uploaded
     std::vector<void*> allocs;
     int64_t launches = 0;                   // library kernels launched (running count)
 
@@ -154,6 +160,7 @@ struct pmm_ctx {
     int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
     int64_t tail_band = 2048; // rows of C_i per band of the tail (multiple of 256)
     int tail_fuse = 1;        // local / IPC FP32: the tail as one fused operand (1) or per group (0)
+    int tail_stream = 1;      // pmm_run on one device: the tail's B rows first, its A rows band by band
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
     std::vector<std::pair<int64_t, int>> groups;  // (first pivot, pivots) of each update
@@ -344,6 +351,7 @@ void free_problem(Device& d) {
     d.tail_allocs.clear();
     d.tail_K = d.tail_K_alloc = 0;
     d.tmax_a = d.tmax_b = nullptr;
+    d.tail_rows = nullptr;
     for (int s = 0; s < kSlots; ++s) {
         d.a_recv[s] = d.b_recv[s] = d.bt[s] = d.a_hi[s] = d.a_lo[s] = d.b_hi[s] = d.b_lo[s] = nullptr;
         d.sa[s] = d.sb[s] = nullptr;
@@ -394,8 +402,13 @@ void destroy_device(Device& d) {
         if (d.ev_ready[s]) cudaEventDestroy(d.ev_ready[s]);
         if (d.ev_free[s]) cudaEventDestroy(d.ev_free[s]);
     }
-    for (cudaEvent_t e : {d.ev_start, d.ev_stop, d.ev_io0, d.ev_io1, d.ev_tpack0, d.ev_tpack1})
+    for (cudaEvent_t e : {d.ev_start, d.ev_stop, d.ev_io0, d.ev_io1, d.ev_tpack0, d.ev_tpack1, d.ev_tail_b})
         if (e) cudaEventDestroy(e);
+    for (auto* v : {&d.ev_band_up, &d.ev_band_st}) {
+        for (cudaEvent_t e : *v) cudaEventDestroy(e);
+        v->clear();
+    }
+    d.ev_tail_b = nullptr;
     for (auto& e : d.ev_join) {
         if (e) cudaEventDestroy(e);
         e = nullptr;
@@ -965,16 +978,27 @@ struct HostDst {
 // at ~3 TFLOP/s per SM (measured) -- but, when the inputs are streamed in
 // (pmm_run), no more than leaves the uploads (8 B per element of C_i) under the
 // groups before the tail: the tail's staging needs its pivots on the device.
+//
+// Band-streamed tail (one device, pmm_run, `tail_stream`): the tail needs its B
+// rows (4 B per element of C_i) before it starts and its A rows only band by
+// band, so the uploads under the groups before the tail are 8 B per element for
+// those groups plus 4 B for the tail's B: X (4 u + 4 u) + (1 - X) 4 u <= X c,
+// i.e. the non-tail fraction X >= r / (1 - r), r = 4 u / c.
+bool streamed_tail_ok(const pmm_ctx* ctx);
 int tail_groups(pmm_ctx* ctx, bool streamed) {
     const int G = (int)ctx->groups.size();
     if (ctx->dt != FPM_F32 || ctx->e2e_tail == 0 || G == 0) return 0;
     if (ctx->e2e_tail > 0) return std::min({ctx->e2e_tail, G, kMaxTail});
+    const double rate_per_sm = scheme_for(ctx, ctx->b) == SplitScheme::F16I8 ? 3.6e12 : 3.0e12;  // measured, c5
     double r = 0.0;
     for (auto& d : ctx->devs)
-        if (d.live() && !d.ooc) r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (3.0e12 * d.num_sms)));
+        if (d.live() && !d.ooc) r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (rate_per_sm * d.num_sms)));
     if (r == 0.0) return 0;
     int L = (int)std::ceil(G * 1.05 * r);
-    if (streamed) L = std::min(L, G - (int)std::ceil(G * 2.0 * r));
+    if (streamed && streamed_tail_ok(ctx) && r < 0.5)
+        L = std::min(L, (int)std::floor(G * (1.0 - r / (1.0 - r))));
+    else if (streamed)
+        L = std::min(L, G - (int)std::ceil(G * 2.0 * r));
     return std::max(1, std::min({L, G, kMaxTail}));
 }
 
@@ -990,12 +1014,19 @@ void ensure_tail_slots(pmm_ctx* ctx, Device& d, int L) {
 // instead of one per group.  The same sum per element as the group-major
 // loop, with one scale per row over the tail instead of one per group.
 bool use_fused_tail(const pmm_ctx* ctx) { return ctx->tail_fuse && ctx->dt == FPM_F32 && !ctx->nccl_mode; }
+// One device holding the whole problem (p = 1, local): its tail operand can be
+// staged from rows that arrive band by band.
+bool streamed_tail_ok(const pmm_ctx* ctx) {
+    return ctx->tail_stream && use_fused_tail(ctx) && !ctx->ipc_mode && ctx->devs.size() == 1 &&
+           ctx->devs[0].live() && !ctx->devs[0].ooc && ctx->devs[0].rect.h * ctx->b == ctx->N &&
+           ctx->devs[0].rect.w * ctx->b == ctx->N;
+}
 
-void ensure_fused_tail(pmm_ctx* ctx, Device& d, int gt) {
+void ensure_fused_tail(pmm_ctx* ctx, Device& d, int gt, bool rows) {
     int64_t K = 0;
     for (size_t g = gt; g < ctx->groups.size(); ++g) K += (int64_t)ctx->groups[g].second * ctx->b;
     d.tail_K = K;
-    if (K <= d.tail_K_alloc) return;
+    if (K <= d.tail_K_alloc && (d.tail_rows != nullptr || !rows)) return;
     CU(cudaSetDevice(d.cuda_dev));
     CU(cudaDeviceSynchronize());
     for (void* p : d.tail_allocs) cudaFree(p);
@@ -1019,6 +1050,7 @@ void ensure_fused_tail(pmm_ctx* ctx, Device& d, int gt) {
     d.sb[s] = static_cast<float*>(get((size_t)d.W * sizeof(float)));
     d.tmax_a = static_cast<unsigned*>(get((size_t)d.H * sizeof(unsigned)));
     d.tmax_b = static_cast<unsigned*>(get((size_t)d.W * sizeof(unsigned)));
+    d.tail_rows = rows ? static_cast<float*>(get((size_t)d.H * K * sizeof(float))) : nullptr;
     d.tail_K_alloc = K;
 }
 
@@ -1130,11 +1162,14 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
         d.tail_fused_run = false;
+        d.tail_streamed_run = false;
         if (L > 0 && d.live() && !d.ooc) {
             // before the timed region (cudaMalloc synchronises)
             if (use_fused_tail(ctx)) {
-                ensure_fused_tail(ctx, d, (int)ctx->groups.size() - L);
+                const bool rows = host != nullptr && streamed_tail_ok(ctx);
+                ensure_fused_tail(ctx, d, (int)ctx->groups.size() - L, rows);
                 d.tail_fused_run = true;
+                d.tail_streamed_run = rows;
             } else {
                 ensure_tail_slots(ctx, d, L);
             }
@@ -1175,6 +1210,102 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
 }
 
 // Everything from ev_start to ev_stop of one k-loop, on the devices' streams.
+// Band-streamed fused tail (pmm_run with one device holding all of A, B and C;
+// option "tail_stream").  Every element of C needs the last pivot, so no band of
+// C can leave before the tail's pivots arrived -- but a band needs only ITS rows
+// of the tail's A panels.  So the tail's B rows (one copy) are uploaded first,
+// then its A rows band by band into `tail_rows` (H x tail_K, row-major: one 2D
+// copy per band); B is staged once, each band's A rows as they land, and band
+// j's update and device -> host copy start as soon as its rows are staged: the
+// D2H of early bands overlaps the H2D of later ones.  Same operand, scales
+// (per-row over the tail's K, per-column over its rows) and sums as the fused
+// tail of issue_tail.
+void issue_tail_streamed(pmm_ctx* ctx, Device& d, int gt, const HostSrc& h, const HostDst& out) {
+    const int64_t b = ctx->b;
+    const int64_t kt = ctx->groups[gt].first;  // first tail pivot
+    const int64_t K = d.tail_K;
+    FPM_CHECK_ARG(kt * b + K == ctx->N && d.tail_rows != nullptr, "streamed tail: inconsistent tail");
+    const SplitScheme sch = scheme_for(ctx, b);
+    const size_t op = op_bytes(sch);
+    const colpart_rect& r = d.rect;
+    CU(cudaSetDevice(d.cuda_dev));
+    const auto bands = tail_bands(d.H, ctx->tail_band);
+    while (d.ev_band_up.size() < bands.size()) {
+        cudaEvent_t e1, e2;
+        CU(cudaEventCreateWithFlags(&e1, cudaEventDisableTiming));
+        CU(cudaEventCreateWithFlags(&e2, cudaEventDisableTiming));
+        d.ev_band_up.push_back(e1);
+        d.ev_band_st.push_back(e2);
+    }
+    if (!d.ev_tail_b) CU(cudaEventCreateWithFlags(&d.ev_tail_b, cudaEventDisableTiming));
+    const int64_t R0 = r.row0 * b - h.row_base, C0 = r.col0 * b - h.col_base;
+    // uploads (behind the non-tail groups' on s_up): the tail's B rows, then A by bands
+    {
+        const char* src = static_cast<const char*>(h.B) + ((size_t)(R0 + kt * b) * h.ld + (size_t)C0) * 4;
+        char* dst = static_cast<char*>(d.B) + (size_t)kt * b * d.W * 4;
+        CU(cudaMemcpy2DAsync(dst, d.W * 4, src, h.ld * 4, d.W * 4, K, cudaMemcpyHostToDevice, d.s_up));
+        CU(cudaEventRecord(d.ev_tail_b, d.s_up));
+    }
+    for (size_t j = 0; j < bands.size(); ++j) {
+        const int64_t r0 = bands[j].first, m = bands[j].second;
+        const char* src = static_cast<const char*>(h.A) + ((size_t)(R0 + r0) * h.ld + (size_t)(C0 + kt * b)) * 4;
+        CU(cudaMemcpy2DAsync(d.tail_rows + (size_t)r0 * K, K * 4, src, h.ld * 4, K * 4, m, cudaMemcpyHostToDevice,
+                             d.s_up));
+        CU(cudaEventRecord(d.ev_band_up[j], d.s_up));
+    }
+    for (int64_t k = kt; k < ctx->n; ++k) CU(cudaEventRecord(d.ev_up[k], d.s_up));  // every tail pivot landed
+    // staging on the comm stream: B once (column maxima over the tail's rows), then A band by band
+    // (the tail groups' own staging events stay empty: the staging is booked on ev_tpack0..1)
+    for (int g = gt; g < (int)ctx->groups.size(); ++g) {
+        rec_t(d.ev_pack0[g], d.s_comm);
+        rec_t(d.ev_pack1[g], d.s_comm);
+    }
+    rec_t(d.ev_tpack0, d.s_comm);
+    CU(cudaStreamWaitEvent(d.s_comm, d.ev_tail_b, 0));
+    launch_split_cols(static_cast<const float*>(d.B) + (size_t)kt * b * d.W, d.W, K, d.W, sch, d.b_hi[kFusedSlot],
+                      d.b_lo[kFusedSlot], d.sb[kFusedSlot], d.s_comm, K, nullptr);
+    d.launches += has_scales(sch) ? 3 : 1;
+    CU(cudaEventRecord(d.ev_ready[kFusedSlot], d.s_comm));
+    for (size_t j = 0; j < bands.size(); ++j) {
+        const int64_t r0 = bands[j].first, m = bands[j].second;
+        CU(cudaStreamWaitEvent(d.s_comm, d.ev_band_up[j], 0));
+        launch_split_rows_seg(d.tail_rows + (size_t)r0 * K, K, 0, 1, m, K, K, sch,
+                              static_cast<char*>(d.a_hi[kFusedSlot]) + (size_t)r0 * K * op,
+                              static_cast<char*>(d.a_lo[kFusedSlot]) + (size_t)r0 * K * op,
+                              d.sa[kFusedSlot] ? d.sa[kFusedSlot] + r0 : nullptr, d.s_comm, nullptr);
+        d.launches += 1;
+        CU(cudaEventRecord(d.ev_band_st[j], d.s_comm));
+    }
+    rec_t(d.ev_tpack1, d.s_comm);
+    // updates band by band, each band's copy to the host right after its update
+    CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[kFusedSlot], 0));
+    CU(cudaEventRecord(d.ev_upd0[gt], d.s_comp));
+    UpdateArgs fa = f32_args(ctx, d, gt, kFusedSlot);
+    fa.K = K;
+    fa.accumulate = true;  // the groups before the tail wrote C
+    const int64_t oR0 = r.row0 * b - out.row_base, oC0 = r.col0 * b - out.col_base;
+    float* C = static_cast<float*>(d.C);
+    for (size_t j = 0; j < bands.size(); ++j) {
+        const int64_t r0 = bands[j].first, m = bands[j].second;
+        CU(cudaStreamWaitEvent(d.s_comp, d.ev_band_st[j], 0));
+        launch_update_f32(band_args(fa, r0, m, C + (size_t)r0 * d.W), d.s_comp);
+        d.launches += 1;
+        CU(cudaEventRecord(d.bp.done[0], d.s_comp));
+        if (r0 + m >= d.H) CU(cudaEventRecord(d.ev_io0, d.s_comp));  // last band updated
+        CU(cudaStreamWaitEvent(d.bp.s_d2h, d.bp.done[0], 0));
+        char* dst = static_cast<char*>(out.C) + ((size_t)(oR0 + r0) * out.ld + (size_t)oC0) * 4;
+        CU(cudaMemcpy2DAsync(dst, out.ld * 4, C + (size_t)r0 * d.W, d.W * 4, d.W * 4, m, cudaMemcpyDeviceToHost,
+                             d.bp.s_d2h));
+    }
+    CU(cudaEventRecord(d.ev_upd1[gt], d.s_comp));
+    for (int g = gt + 1; g < (int)ctx->groups.size(); ++g) {  // the tail's time is booked on its first group
+        CU(cudaEventRecord(d.ev_upd0[g], d.s_comp));
+        CU(cudaEventRecord(d.ev_upd1[g], d.s_comp));
+    }
+    CU(cudaEventRecord(d.ev_free[kFusedSlot], d.s_comp));
+    CU(cudaEventRecord(d.ev_io1, d.bp.s_d2h));  // C_i in host memory
+}
+
 void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, int64_t* bytes_out) {
     const int ngroups = (int)ctx->groups.size();
     const int gt = ngroups - L;  // first tail group
@@ -1194,12 +1325,14 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     auto slot_of = [&](const Device& d, int g) {
         return in_tail(d, g) ? (d.tail_fused_run ? kFusedSlot : 2 + (g - gt)) : (g & 1);
     };
+    // band-streamed tail: its uploads, staging and updates are issued after the loop
+    auto streamed_tail = [&](const Device& d, int g) { return in_tail(d, g) && d.tail_streamed_run; };
     for (int g = 0; g < ngroups; ++g) {
         const int64_t k0 = ctx->groups[g].first;
         if (streamed)
             for (int64_t k = k0; k < k0 + ctx->groups[g].second; ++k)
                 for (auto& d : ctx->devs)
-                    if (d.live()) issue_upload(ctx, d, k, *host);
+                    if (d.live() && !streamed_tail(d, g)) issue_upload(ctx, d, k, *host);
         if (ctx->nccl_mode) {
             // every rank takes part in the NCCL calls, live or not
             Device& d = ctx->devs[0];
@@ -1214,7 +1347,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
             continue;
         }
         for (auto& d : ctx->devs)
-            if (d.live()) {
+            if (d.live() && !streamed_tail(d, g)) {
                 const int slot = slot_of(d, g);
                 if (in_tail(d, g) && d.tail_fused_run) {  // fused tail, pass 1: merge the maxima
                     if (g == gt) {
@@ -1232,7 +1365,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     // fused tail, pass 2: split every tail group with the merged maxima into its
     // K range of the tail operand
     for (auto& d : ctx->devs) {
-        if (L == 0 || !d.live() || d.ooc || !d.tail_fused_run) continue;
+        if (L == 0 || !d.live() || d.ooc || !d.tail_fused_run || d.tail_streamed_run) continue;
         CU(cudaSetDevice(d.cuda_dev));
         rec_t(d.ev_tpack0, d.s_comm);
         int64_t k_off = 0;
@@ -1244,8 +1377,11 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
         CU(cudaEventRecord(d.ev_ready[kFusedSlot], d.s_comm));
     }
     if (L > 0)
-        for (auto& d : ctx->devs)
-            if (d.live() && !d.ooc) issue_tail(ctx, d, gt, L, *out);
+        for (auto& d : ctx->devs) {
+            if (!d.live() || d.ooc) continue;
+            if (d.tail_streamed_run) issue_tail_streamed(ctx, d, gt, *host, *out);
+            else issue_tail(ctx, d, gt, L, *out);
+        }
     for (auto& d : ctx->devs) {
         CU(cudaSetDevice(d.cuda_dev));
         if (d.ooc) bp_join(d.bp, d.s_comp);  // C_i is complete once its last band is back in host memory
@@ -1933,6 +2069,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= 0 && value <= 8, "fuse must be 0 (auto) or 1..8");
             if (ctx->fuse != (int)value) ctx->have_problem = false;  // staging buffers change size
             ctx->fuse = (int)value;
+        } else if (k == "tail_stream") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "tail_stream must be 0 or 1");
+            ctx->tail_stream = (int)value;
         } else if (k == "e2e_tail") {
             FPM_CHECK_ARG(value >= -1 && value <= fpm::kMaxTail, "e2e_tail must be -1 (auto), 0 (off) or 1..%d",
                           fpm::kMaxTail);

@@ -137,3 +137,32 @@ def test_e2e_tail_option_errors():
         for bad in (-2, 17):
             with pytest.raises(pkg.FpmError):
                 ctx.set_option("e2e_tail", bad)
+
+
+@pytest.mark.parametrize("tail", [-1, 1, 3, 16])
+@pytest.mark.parametrize("N,b", [(4096, 256), (2304, 96)])
+def test_band_streamed_tail_matches_fused_tail(tail, N, b):
+    """pmm_run on one device (option "tail_stream"): the tail's B rows are
+    uploaded first and its A rows band by band, each band staged and updated as
+    it lands.  Same operand, scales and sums as the fused tail: C bit-identical
+    to tail_stream = 0, and within the FP32 tolerance of the oracle (integers:
+    exact)."""
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n])
+    for dist in (synth.DIST_PM1, synth.DIST_INT):
+        A = synth.rect(5, N, 0, 0, N, N, dist)
+        B = synth.rect(6, N, 0, 0, N, N, dist)
+        out = []
+        for stream in (0, 1):
+            C = np.full((N, N), np.nan, np.float32)
+            with pkg.Context.local([0]) as ctx:
+                ctx.set_option("e2e_tail", tail)
+                ctx.set_option("tail_stream", stream)
+                ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+            out.append(C)
+        assert np.array_equal(out[0], out[1])
+        ref = og.gemm(A, B)
+        if dist == synth.DIST_INT:
+            assert np.array_equal(out[1].astype(np.float64), ref)
+        else:
+            assert og.rel_fro(out[1], ref) <= 1e-5
