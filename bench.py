@@ -202,6 +202,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         c.set_option("kernel_variant", args.kernel_variant)
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
+        c.set_option("e2e_tail", args.e2e_tail)
         return c
 
     transport = args.transport if world > 1 else "none (p = 1)"
@@ -479,6 +480,7 @@ def main():
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
     ap.add_argument("--e2e-steps", type=int, default=2)
     ap.add_argument("--tail-stream", type=int, default=1, help="pmm_run option tail_stream (e2e, one device)")
+    ap.add_argument("--e2e-tail", type=int, default=-1, help="pmm_run option e2e_tail (-1 auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-hetero", action="store_true",
                     help="skip the emulated-heterogeneity measurement (c4 analogue) added at N = 1")
