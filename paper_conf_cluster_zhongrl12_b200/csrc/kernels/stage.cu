@@ -327,6 +327,14 @@ constexpr int F64_BM = 64, F64_BN = 128, F64_BK = 32, F64_LD = 36, F64_ST = 2, F
 #else
 constexpr int F64_BM = 64, F64_BN = 128, F64_BK = 16, F64_LD = 20, F64_ST = 3, F64_GROUPS = 2;
 #endif
+// Warps per group and warp tile width: 8 warps of 32 x 32 (FPM_F64_WIDE 0, the
+// default) or 4 warps of 32 x 64 (1: 32 independent DMMAs per k-step per warp;
+// measured the same, 31.1 vs 31.2 TFLOP/s at L = 8192, K = 512).
+#ifndef FPM_F64_WIDE
+#define FPM_F64_WIDE 0
+#endif
+constexpr int F64_WTN = FPM_F64_WIDE ? 64 : 32, F64_GW = FPM_F64_WIDE ? 4 : 8;
+constexpr int F64_GT = F64_GW * 32, F64_THREADS = F64_GROUPS * F64_GT, F64_NJ = F64_WTN / 8;
 constexpr int F64_GROUP_DOUBLES = F64_ST * (F64_BM + F64_BN) * F64_LD;
 constexpr int F64_SMEM = F64_GROUPS * F64_GROUP_DOUBLES * 8;  // 184320 B (BK 16) / 221184 B (BK 32)
 
@@ -336,21 +344,22 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool va
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
 }
 
-__device__ __forceinline__ void group_bar(int id) { asm volatile("bar.sync %0, 256;" ::"r"(id) : "memory"); }
+__device__ __forceinline__ void group_bar(int id) { asm volatile("bar.sync %0, %1;" ::"r"(id), "n"(F64_GT) : "memory"); }
 
 // A may be segmented along K (fused pivots, each pivot's H x b panel stored on
 // its own): element (r, k) at A + (k / seg) * seg_stride + r * lda + k % seg.
 // seg is even, so the two consecutive k of a 16-byte copy share a segment.
-__global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict__ A, int64_t lda, int64_t seg,
+__global__ void __launch_bounds__(F64_THREADS, 1) update_f64_k(const double* __restrict__ A, int64_t lda, int64_t seg,
                                                        int64_t seg_stride, const double* __restrict__ Bt,
                                                        double* __restrict__ C, int64_t M, int64_t Nc, int64_t K,
                                                        int64_t ldc, int accumulate) {
     extern __shared__ double sm64[];
-    const int grp = threadIdx.x / 256, gtid = threadIdx.x % 256;
+    const int grp = threadIdx.x / F64_GT, gtid = threadIdx.x % F64_GT;
     double* As = sm64 + grp * F64_GROUP_DOUBLES;       // [ST][BM][LD]
     double* Bs = As + F64_ST * F64_BM * F64_LD;        // [ST][BN][LD]
     const int warp = gtid / 32, lane = threadIdx.x % 32;
-    const int wm = (warp / 4) * 32, wn = (warp % 4) * 32;
+    constexpr int WARPS_N = F64_BN / F64_WTN;
+    const int wm = (warp / WARPS_N) * 32, wn = (warp % WARPS_N) * F64_WTN;
     const int64_t tiles_n = (Nc + F64_BN - 1) / F64_BN;
     const int64_t tiles = ((M + F64_BM - 1) / F64_BM) * tiles_n;
     const int64_t nk = (K + F64_BK - 1) / F64_BK;
@@ -365,12 +374,12 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
         if (lt < tiles) {
             const int64_t m0 = (lt / tiles_n) * F64_BM, n0 = (lt % tiles_n) * F64_BN, k0 = lkb * F64_BK;
             // A: 64 rows x BK doubles (BK / 2 16-B chunks per row); B: 128 rows
-            constexpr int CPR = F64_BK / 2, A_IT = F64_BM * CPR / 256, B_IT = F64_BN * CPR / 256;
+            constexpr int CPR = F64_BK / 2, A_IT = F64_BM * CPR / F64_GT, B_IT = F64_BN * CPR / F64_GT;
 #pragma unroll
             for (int it = 0; it < A_IT + B_IT; ++it) {
-                const int idx = gtid + it * 256;
+                const int idx = gtid + it * F64_GT;
                 const bool isA = it < A_IT;
-                const int j = isA ? idx : idx - A_IT * 256;
+                const int j = isA ? idx : idx - A_IT * F64_GT;
                 const int r = j / CPR, c2 = (j % CPR) * 2;
                 const int64_t gk = k0 + c2;
                 const bool ka = gk < K;  // K even: a 2-element chunk is all in or all out
@@ -398,11 +407,11 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
     int slot_c = 0;
     for (int64_t t = first; t < tiles; t += stride) {
         const int64_t m0 = (t / tiles_n) * F64_BM, n0 = (t % tiles_n) * F64_BN;
-        double acc[4][4][2];
+        double acc[4][F64_NJ][2];
 #pragma unroll
         for (int i = 0; i < 4; ++i)
 #pragma unroll
-            for (int j = 0; j < 4; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
+            for (int j = 0; j < F64_NJ; ++j) acc[i][j][0] = acc[i][j][1] = 0.0;
 
         for (int64_t kb = 0; kb < nk; ++kb) {
             asm volatile("cp.async.wait_group %0;" ::"n"(F64_ST - 2) : "memory");
@@ -412,15 +421,15 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
             const double* bs = Bs + slot_c * F64_BN * F64_LD;
 #pragma unroll
             for (int kk = 0; kk < F64_BK; kk += 4) {
-                double a[4], b[4];
+                double a[4], b[F64_NJ];
 #pragma unroll
                 for (int i = 0; i < 4; ++i) a[i] = as[(wm + i * 8 + lane / 4) * F64_LD + kk + lane % 4];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) b[j] = bs[(wn + j * 8 + lane / 4) * F64_LD + kk + lane % 4];
+                for (int j = 0; j < F64_NJ; ++j) b[j] = bs[(wn + j * 8 + lane / 4) * F64_LD + kk + lane % 4];
 #pragma unroll
                 for (int i = 0; i < 4; ++i)
 #pragma unroll
-                    for (int j = 0; j < 4; ++j)
+                    for (int j = 0; j < F64_NJ; ++j)
                         asm volatile(
                             "mma.sync.aligned.m8n8k4.row.col.f64.f64.f64.f64 {%0, %1}, {%2}, {%3}, {%0, %1};"
                             : "+d"(acc[i][j][0]), "+d"(acc[i][j][1])
@@ -439,11 +448,11 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
             for (int i = 0; i < 4; ++i) {
                 double2* rowp = reinterpret_cast<double2*>(C + (m0 + wm + i * 8 + lane / 4) * ldc + n0 + wn +
                                                            2 * (lane % 4));
-                double2 c[4];
+                double2 c[F64_NJ];
 #pragma unroll
-                for (int j = 0; j < 4; ++j) c[j] = accumulate ? __ldcs(rowp + 4 * j) : make_double2(0.0, 0.0);
+                for (int j = 0; j < F64_NJ; ++j) c[j] = accumulate ? __ldcs(rowp + 4 * j) : make_double2(0.0, 0.0);
 #pragma unroll
-                for (int j = 0; j < 4; ++j) {
+                for (int j = 0; j < F64_NJ; ++j) {
                     c[j].x += acc[i][j][0];
                     c[j].y += acc[i][j][1];
                     __stcs(rowp + 4 * j, c[j]);
@@ -454,7 +463,7 @@ __global__ void __launch_bounds__(512, 1) update_f64_k(const double* __restrict_
 #pragma unroll
         for (int i = 0; i < 4; ++i)
 #pragma unroll
-            for (int j = 0; j < 4; ++j) {
+            for (int j = 0; j < F64_NJ; ++j) {
                 const int64_t gm = m0 + wm + i * 8 + lane / 4;
                 const int64_t gn = n0 + wn + j * 8 + 2 * (lane % 4);
                 if (gm >= M) continue;
@@ -608,7 +617,7 @@ void launch_update_f64(const double* A, int64_t lda, const double* Bt, double* C
     int sms = num_sms;
     if (sms <= 0) cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
     const unsigned grid = (unsigned)std::min<int64_t>((tiles + 1) / 2, std::max(1, sms));  // 1 CTA (2 tile groups) per SM
-    update_f64_k<<<grid, 512, F64_SMEM, st>>>(A, lda, seg, seg_stride, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
+    update_f64_k<<<grid, F64_THREADS, F64_SMEM, st>>>(A, lda, seg, seg_stride, Bt, C, M, Nc, K, ldc, accumulate ? 1 : 0);
     check_launch("update_f64");
 }
 
