@@ -313,3 +313,48 @@ def test_full_size_sampled_parity(N, b):
                 B_cols[c0] = synth.rect(2, N, 0, c0, N, 64)
             ref = og.gemm(A_rows, B_cols[c0])
             assert og.rel_fro(got, ref) <= 1e-5, (r0, c0, og.rel_fro(got, ref))
+
+
+@pytest.mark.parametrize("sm_partition", [0, 1])
+def test_c4_full_size_sampled_parity(sm_partition):
+    """Config 4 at full size (N = 32768, b = 512, 8 devices with the SM caps of the
+    heterogeneity study, grid caps or green partitions), an FPM partition of
+    synthetic speed functions and the column arrangement: sampled blocks of C
+    in every device's rectangle (corners and an interior block) vs the oracle."""
+    N, b = 32768, 512
+    free, _ = torch.cuda.mem_get_info(0)
+    if free < 3.3 * 3 * N * N * 4:
+        pytest.skip("not enough device memory")
+    n = N // b
+    caps = [30, 26, 24, 20, 16, 14, 10, 6]
+    sizes = [1, 4, 16, 64, 256, 1024, 4096]
+    models = [(sizes, [c * (1.0 - 0.5 / (1 + x / 16.0)) for x in sizes]) for c in caps]
+    d = pkg.fpm_partition(n * n, models)
+    rects = pkg.colpart_arrange(n, d)
+    try:
+        ctx = pkg.Context.local([0] * 8, sm_caps=caps)
+    except pkg.FpmError:
+        pytest.skip("SM caps not available")
+    with ctx:
+        ctx.set_option("sm_partition", sm_partition)
+        try:
+            ctx.setup(N, b, rects, pkg.FPM_F32)
+        except pkg.FpmError as ex:
+            if sm_partition:
+                pytest.skip(f"green partitions unavailable: {ex}")
+            raise
+        ctx.fill_synthetic(1, 2, pkg.FPM_DIST_PM1)
+        st = ctx.compute(zero_c=True)
+        assert st.t_compute_s > 0
+        B_cols = {}
+        for (col, r_0, c_0, h, w) in rects:
+            if h * w == 0:
+                continue
+            R0, C0, H, W = r_0 * b, c_0 * b, h * b, w * b
+            for (r0, c0) in [(R0, C0), (R0 + H - 16, C0 + W - 64), (R0 + H // 2, C0 + W // 2)]:
+                got = ctx.download_block(r0, c0, 16, 64)
+                A_rows = synth.rect(1, N, r0, 0, 16, N)
+                if c0 not in B_cols:
+                    B_cols[c0] = synth.rect(2, N, 0, c0, N, 64)
+                ref = og.gemm(A_rows, B_cols[c0])
+                assert og.rel_fro(got, ref) <= 1e-5, (r0, c0, og.rel_fro(got, ref))
