@@ -411,8 +411,9 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks (auto),
  * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 4 = variant
  * 0 on clusters of two CTA pairs that multicast the B^T tiles (grid = the
- * co-resident clusters of 4), 9 = timing probe (no operand loads, no C
- * traffic: the MMAs and the TMEM drain only; C is not written).
+ * co-resident clusters of 4); timing probes (C is not a product): 9 = no
+ * operand loads and no C traffic (the MMAs and the TMEM drain only), 10 =
+ * operand loads but no C traffic, 11 = C traffic but no operand loads.
  * scheme 2 is a timing probe (int8 operands, three kind::i8 MMAs per k-step,
  * s32 accumulator converted to float): it measures the int8 tensor path, its
  * result is not a product of FP32 operands.

@@ -396,10 +396,11 @@ struct HybCfg {
 // multicasts it to the CTA in the same position of the other pair, so the L2
 // reads of B^T halve (A: unchanged).  A stage's smem is then written by two
 // producers, so its release waits for both pairs' MMAs (empty count 2).
-// PROBE (timing only, variant 9): no operand loads and no C traffic -- the MMAs
-// run on whatever stage 0 holds and the epilogue only drains TMEM: the
-// instruction mix's own throughput at the power cap.
-template <int SW, int STAGES, int NCB, int MC = 1, bool PROBE = false>
+// PROBE (timing only): 1 (variant 9) no operand loads and no C traffic -- the
+// MMAs run on whatever stage 0 holds and the epilogue only drains TMEM: the
+// instruction mix's own throughput at the power cap; 2 (variant 10) operand
+// loads but no C traffic; 3 (variant 11) C traffic but no operand loads.
+template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0>
 __global__ void __launch_bounds__(320, 1)
     update_hyb_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_8,
                       const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_8,
@@ -459,7 +460,7 @@ __global__ void __launch_bounds__(320, 1)
 
     if (warp == 0) {
         // ------------------------------------------------------------ producer
-        if (lane == 0 && !PROBE) {
+        if (lane == 0 && PROBE != 1 && PROBE != 3) {
             int stage = 0;
             uint32_t phase = 0;
             for (int t = cluster_id; t < num_ct; t += num_clusters) {
@@ -506,7 +507,7 @@ __global__ void __launch_bounds__(320, 1)
                 ptx::tc_fence_after();
                 for (int kb = 0; kb < num_kb; ++kb) {
                     if (P.prof) c0 = clock64();
-                    if (!PROBE) ptx::mbar_wait(&full[stage], phase);
+                    if (PROBE != 1 && PROBE != 3) ptx::mbar_wait(&full[stage], phase);
                     if (P.prof) w_ops += clock64() - c0;
                     ptx::tc_fence_after();
                     if (lane == 0) {
@@ -522,10 +523,10 @@ __global__ void __launch_bounds__(320, 1)
                             ptx::umma<2, 0>(tmem_base, dA_hi + off, dB_hi + off, Cfg::IDESC_F, (kb | k) != 0);
                             ptx::umma<2, 2>(tmem_base + 256, dA_8 + off, dB_8 + off, Cfg::IDESC_I, (kb | k) != 0);
                         }
-                        if (!PROBE) ptx::umma_commit_mask(&empty[stage], MC == 1 ? 0x3 : 0xF);  // every producer writing the slot
+                        if (PROBE != 1 && PROBE != 3) ptx::umma_commit_mask(&empty[stage], MC == 1 ? 0x3 : 0xF);  // every producer writing the slot
                     }
                     __syncwarp();
-                    if (!PROBE && ++stage == STAGES) { stage = 0; phase ^= 1; }
+                    if (PROBE != 1 && PROBE != 3 && ++stage == STAGES) { stage = 0; phase ^= 1; }
                 }
                 if (lane == 0) ptx::umma_commit_mask(tfull, (uint16_t)(0x3u << (2 * pr)));
                 __syncwarp();
@@ -583,7 +584,7 @@ __global__ void __launch_bounds__(320, 1)
             ptx::tc_fence_before();
             __syncwarp();
             if (lane == 0) ptx::mbar_arrive_cluster(tempty, 2 * pr);
-            if constexpr (PROBE) {  // keep the drained values live, touch nothing else
+            if constexpr (PROBE == 1 || PROBE == 2) {  // keep the drained values live, touch nothing else
                 uint32_t x = 0;
 #pragma unroll
                 for (int j = 0; j < 128; ++j) x ^= u[j];
@@ -770,7 +771,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
 }
 
-template <int SW, int STAGES, int NCB, int MC = 1, bool PROBE = false>
+template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0>
 static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = HybCfg<SW, STAGES, NCB>;
     const CUtensorMap tAh = make_tmap_2d(a.a_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
@@ -853,7 +854,7 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
-    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 4) || (a.variant == 9 && a.scheme == SplitScheme::F16I8),
+    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 4) || (a.variant >= 9 && a.variant <= 11 && a.scheme == SplitScheme::F16I8),
                   "kernel variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
     if (a.scheme == SplitScheme::F16I8) {
@@ -866,7 +867,9 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
             case 2: launch_update_hyb_t<128, 2, 6>(a, st); break;  // 2 x 64 KB stages, 6 C chunks (224 KB)
             case 3: launch_update_hyb_t<64, 5, 4>(a, st); break;   // 5 x 32 KB stages, 4 C chunks (224 KB)
             case 4: launch_update_hyb_t<128, 2, 4, 2>(a, st); break;  // variant 0 on clusters of 2 pairs, B multicast
-            case 9: launch_update_hyb_t<128, 2, 4, 1, true>(a, st); break;  // timing probe: MMAs + TMEM drain only
+            case 9: launch_update_hyb_t<128, 2, 4, 1, 1>(a, st); break;   // timing probe: MMAs + TMEM drain only
+            case 10: launch_update_hyb_t<128, 2, 4, 1, 2>(a, st); break;  // probe: + operand loads, no C traffic
+            case 11: launch_update_hyb_t<128, 2, 4, 1, 3>(a, st); break;  // probe: + C traffic, no operand loads
             default: launch_update_hyb_t<128, 2, 4>(a, st);  // variant 0 (measured best, c5: 520 vs 490 TFLOP/s)
         }
         return;

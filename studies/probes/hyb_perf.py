@@ -47,7 +47,7 @@ res = []
 for scheme, name in ((pkg.SCHEME_F16X3, "F16X3"), (pkg.SCHEME_F16I8, "F16I8"), (pkg.SCHEME_F16X3, "F16X3"), (pkg.SCHEME_F16I8, "F16I8")):
     pkg.k_split_f32(srcA, K, N, K, scheme, ah, al, sa)
     pkg.k_split_cols_f32(srcB, N, K, N, scheme, bh, bl, sb)
-    for v in ((0, 9) if scheme == pkg.SCHEME_F16I8 else (-1,)):
+    for v in ((0, 9, 10, 11) if scheme == pkg.SCHEME_F16I8 else (-1,)):
         res.append(run(f"{name} v{v}", lambda: pkg.k_update_f32(ah, al, bh, bl, sa, sb, C, N, N, K, N, scheme=scheme, variant=v),
                        2 * N * N * K))
 # parity of the two schemes on one launch (overwrite mode)
