@@ -111,7 +111,7 @@ def committed_traffic(N: int, b: int, args):
     """DRAM bytes per update launch from the committed ncu capture of the same
     configuration (profiles/ncu_traffic.json), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    variant = (0 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
+    variant = (6 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
     G = args.raster_group if args.raster_group > 0 else (12 if args.scheme == "f16i8" else 16)
     key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}") + ("" if G == 16 else f"_r{G}")

@@ -285,7 +285,9 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 fp16, 3 kind::f16 MMAs, 2^-22 relative to each element).
  *                 1 = TF32X3 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  Q15.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
- *   "kernel_variant": -1 (auto, default) or 0..3, see fpm_k_update_f32.
+ *   "kernel_variant": -1 (auto, default: F16X3 4, F16I8 6 -- 5 in NCCL
+ *                 contexts, whose kernels need shared memory beside the
+ *                 update) or 0..6, see fpm_k_update_f32.
  *   "fuse":       pivots fused into one rank-(f b) update (FP32): 0 = auto
  *                 (f = min(8, max(1, 2048 / b))), else 1..8.  Groups never
  *                 straddle a column or row boundary of the arrangement, so a
@@ -408,8 +410,11 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * x 2 + 6, 3 = 64-byte x 5 + 4, 4 = 128-byte x 2 + 4 (leaves ~36 KB smem per
  * SM for NCCL / staging kernels co-running with the update); -1 = auto (4).
  * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
- * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks (auto),
- * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 4 = variant
+ * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks,
+ * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 5 = variant
+ * 0 and 6 = variant 1 with C updated by TMA reduce-add (the L2 adds the scaled
+ * accumulator; C is never loaded into shared memory; 6 is the auto choice),
+ * 4 = variant
  * 0 on clusters of two CTA pairs that multicast the B^T tiles (grid = the
  * co-resident clusters of 4); timing probes (C is not a product): 9 = no
  * operand loads and no C traffic (the MMAs and the TMEM drain only), 10 =

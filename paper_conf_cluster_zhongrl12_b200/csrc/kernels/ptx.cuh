@@ -125,6 +125,15 @@ __device__ __forceinline__ void tma_store_2d_hint(const void* tmap, const void* 
         "r"(smem_u32(smem_src)), "r"(c0), "r"(c1), "l"(cache_hint)
         : "memory");
 }
+// C (+)= smem tile in L2: TMA reduce-add (f32 from the tensor map), bulk group.
+__device__ __forceinline__ void tma_reduce_add_2d_hint(const void* tmap, const void* smem_src, int32_t c0, int32_t c1,
+                                                       uint64_t cache_hint) {
+    asm volatile(
+        "cp.reduce.async.bulk.tensor.2d.global.shared::cta.add.bulk_group.L2::cache_hint [%0, {%2, %3}], [%1], %4;" ::"l"(
+            reinterpret_cast<uint64_t>(tmap)),
+        "r"(smem_u32(smem_src)), "r"(c0), "r"(c1), "l"(cache_hint)
+        : "memory");
+}
 __device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;" ::: "memory"); }
 __device__ __forceinline__ void bulk_wait_read0() {
     asm volatile("cp.async.bulk.wait_group.read 0;" ::: "memory");

@@ -400,7 +400,9 @@ struct HybCfg {
 // MMAs run on whatever stage 0 holds and the epilogue only drains TMEM: the
 // instruction mix's own throughput at the power cap; 2 (variant 10) operand
 // loads but no C traffic; 3 (variant 11) C traffic but no operand loads.
-template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0>
+// RED: the C update is a TMA reduce-add of the scaled accumulator (the L2 adds),
+// so C is never loaded into shared memory.
+template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0, bool RED = false>
 __global__ void __launch_bounds__(320, 1)
     update_hyb_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_8,
                       const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_8,
@@ -556,7 +558,7 @@ __global__ void __launch_bounds__(320, 1)
             tm = tm * MC + (int)pr;
             const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
             const int n0 = tn * Cfg::BN + (int)hh * 128;
-            if (eh == 0 && P.load_c) {
+            if (eh == 0 && P.load_c && !RED) {
                 ptx::bulk_wait_read0();
 #pragma unroll
                 for (int c = 0; c < Cfg::NCBH; ++c) {
@@ -618,7 +620,7 @@ __global__ void __launch_bounds__(320, 1)
                         }
                     }
                 }
-                if (P.load_c) {
+                if (P.load_c && !RED) {
                     ptx::mbar_wait(&cf[buf], (cpar >> buf) & 1u);
                     cpar ^= 1u << buf;
                 } else {
@@ -630,7 +632,7 @@ __global__ void __launch_bounds__(320, 1)
                 for (int j = 0; j < 8; ++j) {
                     float4* p4 = reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4));
                     float4 cv = make_float4(0.f, 0.f, 0.f, 0.f);
-                    if (P.load_c) cv = *p4;
+                    if (P.load_c && !RED) cv = *p4;
                     cv.x += v[4 * j + 0];
                     cv.y += v[4 * j + 1];
                     cv.z += v[4 * j + 2];
@@ -640,9 +642,14 @@ __global__ void __launch_bounds__(320, 1)
                 ptx::fence_proxy_async_smem();
                 ptx::named_bar_sync(bar_id, 128);
                 if (eh == 0) {
-                    ptx::tma_store_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0, ptx::kEvictFirst);
+                    if (RED && P.load_c)
+                        ptx::tma_reduce_add_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
+                                                    ptx::kEvictFirst);
+                    else
+                        ptx::tma_store_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0, ptx::kEvictFirst);
                     ptx::bulk_commit();
-                    if constexpr (Cfg::NCBH == 1) {
+                    if constexpr (RED) {
+                    } else if constexpr (Cfg::NCBH == 1) {
                         // one buffer per half: the next chunk's load waits for this store to read it
                         // (the C read-modify-write is off the MMA's critical path)
                         if (P.load_c && c + 1 < 4) {
@@ -771,7 +778,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
 }
 
-template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0>
+template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0, bool RED = false>
 static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = HybCfg<SW, STAGES, NCB>;
     const CUtensorMap tAh = make_tmap_2d(a.a_hi, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
@@ -794,7 +801,7 @@ static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
     P.prof = g_prof_on ? 1 : 0;
-    auto kern = update_hyb_kernel<SW, STAGES, NCB, MC, PROBE>;
+    auto kern = update_hyb_kernel<SW, STAGES, NCB, MC, PROBE, RED>;
     static uint64_t attr_done = 0;
     static int max_clusters[64] = {};  // co-resident clusters of 2 MC CTAs, per device
     int dev = 0;
@@ -854,7 +861,9 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
-    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 4) || (a.variant >= 9 && a.variant <= 11 && a.scheme == SplitScheme::F16I8),
+    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 4) ||
+                      (a.variant >= 5 && a.variant <= 11 && a.variant != 7 && a.variant != 8 &&
+                       a.scheme == SplitScheme::F16I8),
                   "kernel variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
     if (a.scheme == SplitScheme::F16I8) {
@@ -867,10 +876,13 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
             case 2: launch_update_hyb_t<128, 2, 6>(a, st); break;  // 2 x 64 KB stages, 6 C chunks (224 KB)
             case 3: launch_update_hyb_t<64, 5, 4>(a, st); break;   // 5 x 32 KB stages, 4 C chunks (224 KB)
             case 4: launch_update_hyb_t<128, 2, 4, 2>(a, st); break;  // variant 0 on clusters of 2 pairs, B multicast
+            case 5: launch_update_hyb_t<128, 2, 4, 1, 0, true>(a, st); break;  // variant 0, C by TMA reduce-add
+            case 6: launch_update_hyb_t<128, 3, 2, 1, 0, true>(a, st); break;  // 3 stages, C by TMA reduce-add
             case 9: launch_update_hyb_t<128, 2, 4, 1, 1>(a, st); break;   // timing probe: MMAs + TMEM drain only
             case 10: launch_update_hyb_t<128, 2, 4, 1, 2>(a, st); break;  // probe: + operand loads, no C traffic
             case 11: launch_update_hyb_t<128, 2, 4, 1, 3>(a, st); break;  // probe: + C traffic, no operand loads
-            default: launch_update_hyb_t<128, 2, 4>(a, st);  // variant 0 (measured best, c5: 520 vs 490 TFLOP/s)
+            default:  // variant 6: 3 x 64-KB operand stages, C by TMA reduce-add (c5: 545-549 vs 521 for variant 0)
+                launch_update_hyb_t<128, 3, 2, 1, 0, true>(a, st);
         }
         return;
     }

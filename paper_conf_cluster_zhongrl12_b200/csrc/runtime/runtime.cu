@@ -896,7 +896,10 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.accumulate = ctx->groups[g].first != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
     a.raster_group = ctx->raster_group > 0 ? ctx->raster_group : (sch == SplitScheme::F16I8 ? 12 : 16);
     a.l2_hint_b = ctx->l2_hint_b;
-    a.variant = ctx->kernel_variant;  // -1: auto (variant 4, leaves smem for co-running kernels)
+    a.variant = ctx->kernel_variant;  // -1: auto (F16X3: variant 4; F16I8: 6)
+    // NCCL kernels need shared memory to co-run with the persistent update:
+    // F16I8 then takes variant 5 (198 KB) instead of 6 (224 KB)
+    if (a.variant < 0 && ctx->nccl_mode && sch == SplitScheme::F16I8) a.variant = 5;
     return a;
 }
 
@@ -2097,7 +2100,7 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value == 0 || value == 1, "ooc_keep must be 0 or 1");
             ctx->ooc_keep = (int)value;
         } else if (k == "kernel_variant") {
-            FPM_CHECK_ARG(value >= -1 && value <= 4, "kernel_variant must be -1 (auto) or 0..4");
+            FPM_CHECK_ARG(value >= -1 && value <= 6, "kernel_variant must be -1 (auto) or 0..6 (5, 6: F16I8 only)");
             ctx->kernel_variant = (int)value;
         } else if (k == "l2_hint_b") {
             FPM_CHECK_ARG(value >= 0 && value <= 2, "l2_hint_b must be 0 (normal), 1 (first) or 2 (last)");
@@ -2292,7 +2295,7 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
     return guarded([&] {
         FPM_CHECK_ARG(scheme >= 0 && scheme <= 3, "scheme must be 0, 1, 2 (int8 timing probe) or 3");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
-        FPM_CHECK_ARG((variant >= -1 && variant <= 4) || (variant >= 9 && variant <= 11 && scheme == 3),
+        FPM_CHECK_ARG((variant >= -1 && variant <= 4) || (variant >= 5 && variant <= 11 && scheme == 3),
                       "variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
         FPM_CHECK_ARG(scheme == 1 || scheme == 2 || (sa && sb), "F16X3 / F16I8 need sa and sb");
         fpm::UpdateArgs a;

@@ -113,7 +113,7 @@ SHAPES = [(128, 256, 64), (300, 520, 128), (1000, 1000, 512), (64, 40, 64), (1, 
           (777, 264, 192), (520, 1032, 2048)]
 
 
-@pytest.mark.parametrize("variant", [-1, 0, 1, 2, 4])
+@pytest.mark.parametrize("variant", [-1, 0, 1, 2, 4, 5, 6])
 @pytest.mark.parametrize("M,Nc,K", SHAPES)
 def test_update_f16i8_random(variant, M, Nc, K):
     A = synth.rect(1, 4096, 0, 0, M, K)
@@ -124,7 +124,7 @@ def test_update_f16i8_random(variant, M, Nc, K):
     assert og.rel_fro(C, ref) <= 1e-5
 
 
-@pytest.mark.parametrize("variant", [-1, 0, 1, 2, 4])
+@pytest.mark.parametrize("variant", [-1, 0, 1, 2, 4, 5, 6])
 def test_update_f16i8_integer_exact(variant):
     M, Nc, K = 520, 776, 512
     A = synth.rect(4, 4096, 0, 0, M, K, synth.DIST_INT)
