@@ -992,14 +992,14 @@ int tail_groups(pmm_ctx* ctx, bool streamed) {
     const int G = (int)ctx->groups.size();
     if (ctx->dt != FPM_F32 || ctx->e2e_tail == 0 || G == 0) return 0;
     if (ctx->e2e_tail > 0) return std::min({ctx->e2e_tail, G, kMaxTail});
-    const double rate_per_sm = scheme_for(ctx, ctx->b) == SplitScheme::F16I8 ? 3.6e12 : 3.0e12;  // measured, c5
+    const double rate_per_sm = scheme_for(ctx, ctx->b) == SplitScheme::F16I8 ? 3.9e12 : 3.0e12;  // measured, c5
     double r = 0.0;
     for (auto& d : ctx->devs)
         if (d.live() && !d.ooc) r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (rate_per_sm * d.num_sms)));
     if (r == 0.0) return 0;
     int L = (int)std::ceil(G * 1.05 * r);
-    if (streamed && streamed_tail_ok(ctx) && r < 0.5)  // 0.9: the tail may start a little late (measured, c5:
-        L = std::min(L, (int)std::floor(G * (1.0 - 0.9 * r / (1.0 - r))));  // L = 10 of 25 best, 8: -4 %)
+    if (streamed && streamed_tail_ok(ctx) && r < 0.5)  // 0.55: the tail may start somewhat late (measured, c5:
+        L = std::min(L, (int)std::floor(G * (1.0 - 0.55 * r / (1.0 - r))));  // L = 12 of 25 best, 8: -4 %, 16: -8 %)
     else if (streamed)
         L = std::min(L, G - (int)std::ceil(G * 2.0 * r));
     return std::max(1, std::min({L, G, kMaxTail}));
