@@ -408,7 +408,9 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * shared-memory split between the operand ring and the C ring: 0 = 128-byte
  * k-blocks x 3 stages + 2 C chunks in flight, 1 = 64-byte x 4 + 6, 2 = 128-byte
  * x 2 + 6, 3 = 64-byte x 5 + 4, 4 = 128-byte x 2 + 4 (leaves ~36 KB smem per
- * SM for NCCL / staging kernels co-running with the update); -1 = auto (4).
+ * SM for NCCL / staging kernels co-running with the update), 5 = 128-byte x 3
+ * + 2 with C updated by TMA reduce-add (C never loaded into shared memory);
+ * -1 = auto (4).
  * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
  * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks,
  * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 5 = variant

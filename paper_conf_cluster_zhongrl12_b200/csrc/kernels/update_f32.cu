@@ -95,7 +95,7 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
     tn = r / gm;
 }
 
-template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1, bool RED = false>
 __global__ void __launch_bounds__(192, 1)
     update_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
                   const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
@@ -244,7 +244,7 @@ __global__ void __launch_bounds__(192, 1)
             const int n0 = tn * BN;
             const int acc = it & 1;
             const uint32_t acc_par = (it >> 1) & 1;
-            if (e == 0 && P.load_c) {
+            if (e == 0 && P.load_c && !RED) {
                 ptx::bulk_wait_read0();
                 for (int c = 0; c < NCB && c < Cfg::N_CHUNKS; ++c) {
                     ptx::mbar_arrive_expect_tx(&cfull[c], Cfg::C_CHUNK_BYTES);
@@ -295,7 +295,7 @@ __global__ void __launch_bounds__(192, 1)
                         }
                     }
                 }
-                if (P.load_c) {
+                if (P.load_c && !RED) {
                     ptx::mbar_wait(&cfull[buf], (cpar >> buf) & 1u);
                     cpar ^= 1u << buf;
                 } else {
@@ -309,7 +309,7 @@ __global__ void __launch_bounds__(192, 1)
                 for (int j = 0; j < 8; ++j) {
                     float4* p4 = reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4));
                     float4 cv = make_float4(0.f, 0.f, 0.f, 0.f);
-                    if (P.load_c) cv = *p4;
+                    if (P.load_c && !RED) cv = *p4;
                     cv.x += v[4 * j + 0];
                     cv.y += v[4 * j + 1];
                     cv.z += v[4 * j + 2];
@@ -319,11 +319,15 @@ __global__ void __launch_bounds__(192, 1)
                 ptx::fence_proxy_async_smem();
                 ptx::named_bar_sync(1, 128);
                 if (e == 0) {
-                    ptx::tma_store_2d_hint(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
-                                           ptx::kEvictFirst);
+                    if (RED && P.load_c)
+                        ptx::tma_reduce_add_2d_hint(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
+                                                    ptx::kEvictFirst);
+                    else
+                        ptx::tma_store_2d_hint(&tmC, cbuf + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
+                                               ptx::kEvictFirst);
                     ptx::bulk_commit();
                     const int nxt = c - 1 + NCB;  // refill the buffer of chunk c - 1
-                    if (P.load_c && c >= 1 && nxt < Cfg::N_CHUNKS) {
+                    if (P.load_c && !RED && c >= 1 && nxt < Cfg::N_CHUNKS) {
                         const int nb = (c - 1) % NCB;
                         ptx::bulk_wait_read1();  // store of chunk c - 1 has read its buffer
                         ptx::mbar_arrive_expect_tx(&cfull[nb], Cfg::C_CHUNK_BYTES);
@@ -726,7 +730,7 @@ CUtensorMap make_tmap_2d(const void* base, CUtensorMapDataType dt, int elem_byte
     return m;
 }
 
-template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1>
+template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1, bool RED = false>
 static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = UpdCfg<CG, KIND, BN, STAGES, SW, NCB>;
     const CUtensorMapDataType odt = KIND == 1   ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32
@@ -750,7 +754,7 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     P.group = a.raster_group > 0 ? a.raster_group : 16;
     P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
     P.prof = 0;
-    auto kern = update_kernel<CG, KIND, BN, STAGES, SW, NCB, MREP>;
+    auto kern = update_kernel<CG, KIND, BN, STAGES, SW, NCB, MREP, RED>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;
     cudaGetDevice(&dev);
@@ -861,8 +865,8 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
-    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 4) ||
-                      (a.variant >= 5 && a.variant <= 11 && a.variant != 7 && a.variant != 8 &&
+    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 5) ||
+                      (a.variant >= 6 && a.variant <= 11 && a.variant != 7 && a.variant != 8 &&
                        a.scheme == SplitScheme::F16I8),
                   "kernel variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
@@ -910,6 +914,10 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
             case 3:  // 64-B k-blocks x 5 stages, 4 C chunks
                 if (tf32) launch_update_t<2, 1, 256, 5, 64, 4>(a, st);
                 else launch_update_t<2, 0, 256, 5, 64, 4>(a, st);
+                break;
+            case 5:  // 128-B k-blocks x 3 stages, 2 C chunks, C by TMA reduce-add
+                if (tf32) launch_update_t<2, 1, 256, 3, 128, 2, 1, true>(a, st);
+                else launch_update_t<2, 0, 256, 3, 128, 2, 1, true>(a, st);
                 break;
             case 4:  // 128-B k-blocks x 2 stages, 4 C chunks: leaves ~36 KB smem per SM for
                      // NCCL kernels to co-run with the persistent update

@@ -2295,7 +2295,7 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
     return guarded([&] {
         FPM_CHECK_ARG(scheme >= 0 && scheme <= 3, "scheme must be 0, 1, 2 (int8 timing probe) or 3");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
-        FPM_CHECK_ARG((variant >= -1 && variant <= 4) || (variant >= 5 && variant <= 11 && scheme == 3),
+        FPM_CHECK_ARG((variant >= -1 && variant <= 5) || (variant >= 6 && variant <= 11 && scheme == 3),
                       "variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
         FPM_CHECK_ARG(scheme == 1 || scheme == 2 || (sa && sb), "F16X3 / F16I8 need sa and sb");
         fpm::UpdateArgs a;

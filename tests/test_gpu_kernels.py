@@ -147,7 +147,7 @@ def test_transpose_bit_exact(dt, rows, cols):
     assert np.array_equal(out.cpu().numpy(), x[:, :cols].T)
 
 
-KCFG = ["1", "2v0", "2v1", "2v2", "2v3", "2v4"]   # cta_group 1; cta_group 2 with smem variants 0..4
+KCFG = ["1", "2v0", "2v1", "2v2", "2v3", "2v4", "2v5"]   # cta_group 1; cta_group 2 with smem variants 0..5 (5: reduce-add C)
 
 
 def _update_f32(A, B, C0, scheme, cg, num_sms=0, accumulate=True):
