@@ -47,7 +47,7 @@ res = []
 for scheme, name in ((pkg.SCHEME_F16X3, "F16X3"), (pkg.SCHEME_F16I8, "F16I8"), (pkg.SCHEME_F16X3, "F16X3"), (pkg.SCHEME_F16I8, "F16I8")):
     pkg.k_split_f32(srcA, K, N, K, scheme, ah, al, sa)
     pkg.k_split_cols_f32(srcB, N, K, N, scheme, bh, bl, sb)
-    for v in ((0, 9, 10, 11) if scheme == pkg.SCHEME_F16I8 else (-1,)):
+    for v in ((6, 9, 10, 11) if scheme == pkg.SCHEME_F16I8 else (-1,)):
         res.append(run(f"{name} v{v}", lambda: pkg.k_update_f32(ah, al, bh, bl, sa, sb, C, N, N, K, N, scheme=scheme, variant=v),
                        2 * N * N * K))
 # parity of the two schemes on one launch (overwrite mode)
@@ -67,7 +67,7 @@ json.dump(res, open("gpurun_out/hyb_perf.json", "w"), indent=1)
 # MMA-issuer wait counters (fpm_k_prof) over 5 launches of the default F16I8 kernel
 pkg.k_split_f32(srcA, K, N, K, pkg.SCHEME_F16I8, ah, al, sa)
 pkg.k_split_cols_f32(srcB, N, K, N, pkg.SCHEME_F16I8, bh, bl, sb)
-for v in (0,):
+for v in (0, 6):
     torch.cuda.synchronize(); pkg.k_prof(1)
     for _ in range(5):
         pkg.k_update_f32(ah, al, bh, bl, sa, sb, C, N, N, K, N, scheme=pkg.SCHEME_F16I8, variant=v)
