@@ -33,7 +33,7 @@ sys.path.insert(0, ROOT)
 METRIC = "partitioned GEMM GFLOPS & % tensor peak at 1/2/4/8 B200; FPM load imbalance %"
 UNIT = "GFLOP/s"
 N_DEFAULT, B_DEFAULT = 49152, 1024
-ORACLE_ROWS, ORACLE_COLS = 64, 1024   # bounded sample for the CPU oracle
+ORACLE_ROWS, ORACLE_COLS = 2048, 1024   # bounded sample for the CPU oracle (~206 GFLOP at c5, ~5 s on 16 cores)
 
 
 def log(*a):
@@ -127,7 +127,7 @@ def oracle_sample(N: int, reps: int = 1):
     C[0:R, 0:S] = A[0:R, :] B[:, 0:S] of the workload; returns (GFLOP/s, cores, desc)."""
     import synth
     from oracle import gemm as og
-    R, S = ORACLE_ROWS, ORACLE_COLS
+    R, S = min(ORACLE_ROWS, N), min(ORACLE_COLS, N)
     sa, sb = synth.seeds_for_config(4)
     A = synth.rect(sa, N, 0, 0, R, N)
     B = synth.rect(sb, N, 0, 0, N, S)
