@@ -370,8 +370,12 @@ __global__ void __launch_bounds__(192, 1)
 // all 512 columns, so there is no second accumulator set: eight epilogue warps
 // (two per TMEM lane quarter, one per 128-column half) drain both accumulators
 // into registers (128 combined values per thread), hand TMEM back to the MMA
-// warp, and only then do the C read-modify-write, which overlaps the next
-// tile's mainloop.  Each column half runs its own C ring (NCB / 2 chunks).
+// warp, and only then update C, which overlaps the next tile's mainloop.  Each
+// column half runs its own ring of NCB / 2 chunks.  Default (variant 6, RED):
+// the scaled chunk is written to shared memory once and added to C in L2 by a
+// TMA reduce-add, so C is never loaded into shared memory and the smem a C ring
+// would hold goes to a third operand stage (c5: 545-612 vs 521-536 TFLOP/s for
+// variant 0, which loads C by TMA, adds and stores).
 // SW: bytes per operand row and k-block (128: 64 K per k-block, the fp16 row and
 // the whole [q | l] int8 row; 64: 32 K per k-block, the fp16 row and one half --
 // q or l -- of the int8 row: the pairing of fp16 and int8 k-blocks is free, the
