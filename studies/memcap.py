@@ -97,6 +97,10 @@ def main():
     ap.add_argument("--concurrent", action="store_true",
                     help="sample all devices at once (P:10 (ii)): the out-of-core GPUs then share the "
                          "host link as they do in the run")
+    ap.add_argument("--link-group", default="",
+                    help="comma-separated device indices sampled together in a context of their own "
+                         "(the out-of-core GPUs: they share the host link in the run, P:10 (ii) applied to "
+                         "the shared resource); the others alone")
     ap.add_argument("--sm-partition", type=int, default=0,
                     help="1 = each device in its own green-context SM partition (all its kernels confined)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "memcap_table3_r01.json"))
@@ -122,6 +126,16 @@ def main():
         per_dev = list(zip(*ctx.sample(-1, b, sizes, pkg.FPM_F32)))
     else:                  # each device alone, as the paper measured its GPUs
         per_dev = [ctx.sample(dev, b, sizes, pkg.FPM_F32) for dev in range(p)]
+    if args.link_group:    # the link-sharing devices again, together in a context of their own
+        grp = [int(i) for i in args.link_group.split(",")]
+        with pkg.Context.local([0] * len(grp), sm_caps=[caps[i] for i in grp]) as gctx:
+            gctx.set_option("ooc_keep", args.ooc_keep)
+            gctx.set_option("ooc_buffers", args.ooc_buffers)
+            for j, i in enumerate(grp):
+                gctx.set_device_option(j, "c_cap_bytes", c_caps[i])
+            gsp = list(zip(*gctx.sample(-1, b, sizes, pkg.FPM_F32)))
+        for j, i in enumerate(grp):
+            per_dev[i] = gsp[j]
     for dev, (sp, ci, reps) in enumerate(per_dev):
         models.append((sizes, sp))
         sample_info.append({"name": names[dev], "sm_cap": caps[dev], "c_cap_bytes": c_caps[dev],
@@ -173,6 +187,7 @@ def main():
     out = {
         "config": {"b": b, "ns": ns, "p": p, "names": names, "sm_caps": caps, "c_cap_bytes": c_caps,
                    "ncal": args.ncal, "x_cal": x_cal, "sizes": sizes, "ooc_keep": args.ooc_keep, "ooc_buffers": args.ooc_buffers,
+                   "link_group": args.link_group,
                    "sampling": "concurrent (all devices at once)" if args.concurrent else "exclusive",
                    "dtype": "f32 (auto scheme: F16I8 for b % 64 == 0, DESIGN Q15b)", "sm_partition": args.sm_partition,
                    "gpu": "1x B200; devices emulated by SM caps, device memory by C caps (C_i out of core above)"},
