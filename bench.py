@@ -30,6 +30,10 @@ import time
 ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
+# the arithmetic the FP32 path computes in (inputs, outputs and accumulation FP32)
+DTYPE = {"f16x3": "f32 (F16X3: 3 fp16 tcgen05 products per FP32 MAC, FP32 accumulate)",
+         "tf32x3": "f32 (TF32X3: 3 tf32 tcgen05 products per FP32 MAC, FP32 accumulate)",
+         "f16i8": "f32-emulated-f16i8 (fp16 + int8 products, row-max fixed point: NOT FP32-class)"}
 METRIC = "partitioned GEMM GFLOPS & % tensor peak at 1/2/4/8 B200; FPM load imbalance %"
 UNIT = "GFLOP/s"
 N_DEFAULT, B_DEFAULT = 49152, 1024
@@ -122,9 +126,10 @@ def committed_traffic(N: int, b: int, args):
 
 
 # ----------------------------------------------------------------- oracle
-def oracle_sample(N: int, reps: int = 1):
+def oracle_sample(N: int, reps: int = 1, want_c: bool = False):
     """Time the CPU oracle (plain triple loop, FP64 accumulation) on the block
-    C[0:R, 0:S] = A[0:R, :] B[:, 0:S] of the workload; returns (GFLOP/s, cores, desc)."""
+    C[0:R, 0:S] = A[0:R, :] B[:, 0:S] of the workload; returns (GFLOP/s, cores,
+    desc, seconds[, C block])."""
     import synth
     from oracle import gemm as og
     R, S = min(ORACLE_ROWS, N), min(ORACLE_COLS, N)
@@ -135,13 +140,42 @@ def oracle_sample(N: int, reps: int = 1):
     ts = []
     for _ in range(reps):
         t0 = time.perf_counter()
-        og.gemm(A, B)
+        Cs = og.gemm(A, B)
         ts.append(time.perf_counter() - t0)
     t = min(ts)
     flops = 2.0 * R * S * N
     desc = (f"C[0:{R},0:{S}] = A[0:{R},:] B[:,0:{S}] of the N={N} workload (K={N}); "
             f"{flops / 1e9:.2f} GFLOP per step, oracle triple loop (gcc -O2, OpenMP, FP64 accumulation)")
+    if want_c:
+        return flops / t / 1e9, og.num_threads(), desc, t, Cs
     return flops / t / 1e9, og.num_threads(), desc, t
+
+
+def e2e_parity(N: int, hC, oracle_block) -> dict:
+    """Parity of the timed e2e output (pmm_run, default options) against the
+    oracle on sampled blocks (exact oracle on a sample of C):
+    the top-left block the CPU baseline computes anyway, plus the bottom-right
+    corner and an interior block computed here.  Tolerance 1e-5 rel-Fro (FP32)."""
+    import numpy as np
+
+    import synth
+    from oracle import gemm as og
+    sa, sb = synth.seeds_for_config(4)
+    C = hC.numpy() if hasattr(hC, "numpy") else np.asarray(hC)
+    R, S = oracle_block.shape
+    blocks = [("top-left", 0, 0, R, S, oracle_block)]
+    for name, r0, c0, h, w in (("bottom-right", N - 256, N - 256, 256, 256),
+                               ("interior", N // 2 - 100, N // 3 - 60, 200, 120)):
+        A = synth.rect(sa, N, r0, 0, h, N)
+        B = synth.rect(sb, N, 0, c0, N, w)
+        blocks.append((name, r0, c0, h, w, og.gemm(A, B)))
+    out = []
+    for name, r0, c0, h, w, ref in blocks:
+        out.append({"block": name, "rows": [r0, r0 + h], "cols": [c0, c0 + w],
+                    "rel_fro": float(og.rel_fro(C[r0:r0 + h, c0:c0 + w], ref))})
+    worst = max(b["rel_fro"] for b in out)
+    return {"what": "e2e output C (host, pmm_run) vs the CPU oracle on sampled blocks", "tol": 1e-5,
+            "blocks": out, "max_rel_fro": worst, "ok": bool(worst <= 1e-5)}
 
 
 # ----------------------------------------------------------------- main arms
@@ -332,24 +366,28 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None}
 
     # ---- end to end through pmm_run with pinned host buffers
-    e2e = None
+    e2e, hC = None, None
     if args.e2e_steps > 0:
         try:
-            e2e = run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc)
+            e2e, hC = run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc)
         except Exception as ex:  # report, do not hide
             log("e2e failed:", repr(ex))
             e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:200]}
 
-    cpu = None  # the oracle baseline is timed at N = 1 only (rank 0); N > 1 lines carry null
+    cpu, parity = None, None  # the oracle baseline is timed at N = 1 only (rank 0); N > 1 lines carry null
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        g, cores, desc, _ = oracle_sample(N)
+        g, cores, desc, _, c_block = oracle_sample(N, want_c=True)
         cpu = {"value": g, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc}
+        if hC is not None:
+            parity = e2e_parity(N, hC, c_block)
+            if not parity["ok"]:
+                log("PARITY FAILURE of the e2e output:", json.dumps(parity))
 
     if rank == 0:
         line = {
             "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
             "warmup": args.warmup, "ms_per_step": 1e3 * total_t / args.steps, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None, "dtype": DTYPE[args.scheme], "data": "synthetic",
             "config": {
                 "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
                 "N": N, "b": b, "p": p, "partition": d, "rects": rects,
@@ -370,6 +408,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             },
             "roofline": roofline,
             "cpu_baseline": cpu,
+            "parity": parity,
             "e2e": e2e,
             "gpu_launches": launches,
             "clocks": clk,
@@ -384,6 +423,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 log("hetero failed:", repr(ex))
                 line["hetero"] = {"error": repr(ex)[:200]}
         print(json.dumps(line), flush=True)
+        if parity is not None and not parity["ok"]:
+            sys.exit(3)
 
 
 def run_hetero(peak_tflops: float) -> dict:
@@ -455,11 +496,12 @@ def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc):
         if i > 0:  # first call is a warm-up
             ts.append(t_all)
     t = statistics.median(ts)
-    return {"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
+    return ({"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
             "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
             "device_kloop_s": st.t_compute_s if st else None, "download_s": st.t_download_s if st else None,
             "timing": ("host wall clock: upload + barrier + pmm_compute_into (IPC), max over ranks"
-                       if ipc else "host wall clock around the blocking pmm_run call, max over ranks")}
+                       if ipc else "host wall clock around the blocking pmm_run call, max over ranks")},
+            hC if (live and len(rects) == 1) else None)   # N = 1: hC is all of C
 
 
 def main():
@@ -470,7 +512,9 @@ def main():
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
     ap.add_argument("--N", type=int, default=N_DEFAULT)
     ap.add_argument("--b", type=int, default=B_DEFAULT)
-    ap.add_argument("--scheme", choices=["f16i8", "f16x3", "tf32x3"], default="f16i8")
+    ap.add_argument("--scheme", choices=["f16i8", "f16x3", "tf32x3"], default="f16x3",
+                    help="FP32 arithmetic: f16x3 (default, FP32-class), tf32x3, or f16i8 (opt-in, "
+                         "fixed point relative to the row maximum: not FP32-class, DESIGN Q15b)")
     ap.add_argument("--transport", choices=["ipc", "nccl"], default="ipc",
                     help="N > 1: pull pivots from peers' memory (ipc) or exchange them with NCCL")
     ap.add_argument("--cta-group", type=int, default=2)
@@ -478,7 +522,7 @@ def main():
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
-    ap.add_argument("--e2e-steps", type=int, default=2)
+    ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--tail-stream", type=int, default=1, help="pmm_run option tail_stream (e2e, one device)")
     ap.add_argument("--e2e-tail", type=int, default=-1, help="pmm_run option e2e_tail (-1 auto)")
     ap.add_argument("--no-cpu-baseline", action="store_true")

@@ -276,14 +276,16 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
                int32_t nsizes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out);
 
 /* Tuning / selection knobs (all optional):
- *   "f32_scheme": -1 = auto (default): 3 when b % 64 == 0 and cta_group is
- *                 2, else 0.  3 = F16I8 (x 2^e = h0 + h1, h0 fp16 with a
- *                 per-row power-of-two scale; int8 codes q = rint(x 2^e / 256),
- *                 l = rint(8 h1); one kind::f16 MMA for h0 h0' and one kind::i8
- *                 MMA for 32 (q l' + l q'); error fixed-point relative to the
- *                 row maximum, ~2^-18; Q15b).  0 = F16X3 (h0, h1 both
- *                 fp16, 3 kind::f16 MMAs, 2^-22 relative to each element).
- *                 1 = TF32X3 (x = hi + lo in tf32, 3 kind::tf32 MMAs).  Q15.
+ *   "f32_scheme": -1 = auto (default) = 0.  0 = F16X3 (x 2^e = h0 + h1, both
+ *                 fp16, 2^e a per-row / per-column power of two; 3 kind::f16
+ *                 MMAs; 2^-22 relative to each element: FP32-class, Q15).
+ *                 1 = TF32X3 (x = hi + lo in tf32, 3 kind::tf32 MMAs).
+ *                 3 = F16I8, opt-in only, NOT FP32-class: int8 codes
+ *                 q = rint(x 2^e / 256), l = rint(8 h1); one kind::f16 MMA for
+ *                 h0 h0' and one kind::i8 MMA for 32 (q l' + l q'); the error
+ *                 is fixed point relative to the row maximum (~2^-18 of it,
+ *                 normwise, not elementwise; Q15b); needs cta_group
+ *                 2, b % 64 == 0 and K <= 131072 per update.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
  *   "kernel_variant": -1 (auto, default: F16X3 4, F16I8 6 -- 5 in NCCL
  *                 contexts, whose kernels need shared memory beside the

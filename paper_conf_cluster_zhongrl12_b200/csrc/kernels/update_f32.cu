@@ -349,7 +349,7 @@ __global__ void __launch_bounds__(192, 1)
     }
 }
 
-// ------------------------------------------------------------ F16I8 (default)
+// ---------------------------------------------- F16I8 (opt-in, not FP32-class)
 // FP32 operand x of a row (A) / column (B) with the F16X3 power-of-two scale
 // 2^e (row maximum in [2^14, 2^15)):  x 2^e = h0 + h1, h0 = fp16_rn(x 2^e),
 // |h1| <= 8, and two int8 codes q = clamp(rint(x 2^e / 256), +-127),
@@ -358,7 +358,9 @@ __global__ void __launch_bounds__(192, 1)
 //                     ~ h0a h0b            (kind::f16, exact products, fp32 sum)
 //                     + 32 (qa lb + la qb) (kind::i8, exact s32 sum)
 // with the dropped h1a h1b and the q rounding of the cross terms at the 2^-18
-// level (relative Frobenius error ~3e-6 on U[-1,1), tolerance 1e-5).  The int8
+// level of the row maximum: fixed point per row, so accurate to ~3e-6 rel-Fro
+// on U[-1,1) but NOT elementwise FP32-class on inputs with a large dynamic
+// range (Q15b) -- an explicit opt-in (f32_scheme 3).  The int8
 // operand of a 64-wide k-block is one 128-byte row [q(64) | l(64)] for A and
 // [l(64) | q(64)] for B^T, so ONE kind::i8 product over 128 bytes gives both
 // cross terms.  Per k-block: 4 f16 MMAs (K = 16 each) + 4 i8 MMAs (K = 32 each)
@@ -877,6 +879,9 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     if (a.scheme == SplitScheme::F16I8) {
         FPM_CHECK_ARG(a.cta_group == 2, "F16I8 runs on CTA pairs (cta_group 2)");
         FPM_CHECK_ARG(a.K % 64 == 0, "F16I8: K must be a multiple of 64");
+        // the s32 accumulator takes up to 2 * 127 * 64 = 16256 per k of one 64-wide block,
+        // i.e. < 2^31 only for K <= 131072 (no wrap-around of the exact int8 cross terms)
+        FPM_CHECK_ARG(a.K <= 131072, "F16I8: K must be <= 131072 per update (s32 accumulator range)");
         FPM_CHECK_ARG(a.sa != nullptr && a.sb != nullptr, "F16I8 needs sa and sb");
         switch (a.variant) {
             case 0: launch_update_hyb_t<128, 2, 4>(a, st); break;  // 2 x 64 KB stages, 4 C chunks (192 KB)

@@ -521,13 +521,17 @@ int fuse_factor(pmm_ctx* ctx, fpm_dtype dt, int64_t b) {
     return (int)std::max<int64_t>(1, std::min<int64_t>(8, 2048 / b));
 }
 
-// FP32 scheme of a problem with block size b: the option, or auto = F16I8
-// (fp16 main product + int8 cross terms) when every fused K is a multiple of 64
-// and CTA pairs are on, else F16X3.  Both use 2-byte operand halves and
-// per-row / per-column scales; TF32X3 uses 4-byte halves and no scales.
+// FP32 scheme of a problem: the option, or auto = F16X3 (three fp16 products,
+// 22 significant bits per operand relative to the element itself: FP32-class,
+// DESIGN.md Q15).  F16I8 (fp16 main product + int8 cross terms, fixed point
+// relative to the row maximum, Q15b) is narrower than FP32 on inputs with a
+// large dynamic range, so it is an explicit opt-in only.  F16X3 and F16I8 use
+// 2-byte operand halves and per-row / per-column scales; TF32X3 uses 4-byte
+// halves and no scales.
 SplitScheme scheme_for(const pmm_ctx* ctx, int64_t b) {
+    (void)b;
     if (ctx->f32_scheme >= 0) return (SplitScheme)ctx->f32_scheme;
-    return (b % 64 == 0 && ctx->cta_group == 2) ? SplitScheme::F16I8 : SplitScheme::F16X3;
+    return SplitScheme::F16X3;
 }
 bool has_scales(SplitScheme s) { return s != SplitScheme::TF32X3; }
 size_t op_bytes(SplitScheme s) { return s == SplitScheme::TF32X3 ? 4 : 2; }

@@ -137,7 +137,7 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
         st1 = one.compute()
     return {
         "config": {"N": N, "b": b, "p": p, "sm_caps": list(caps), "ncal": ncal, "x_cal": x_cal, "x_even": x_even,
-                   "sizes": sizes, "dtype": "f32 (auto scheme: F16I8 for b % 64 == 0, DESIGN Q15b)", "sm_partition": sm_partition,
+                   "sizes": sizes, "dtype": "f32 (auto scheme: F16X3, DESIGN Q15)", "sm_partition": sm_partition,
                    "gpu": "1x B200, devices emulated by SM caps",
                    "sampling": "exclusive" if exclusive else "concurrent (all devices at once)"},
         "fpm_sample_s": t_sample, "models": sample_info, "partitions": results,

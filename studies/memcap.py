@@ -114,12 +114,16 @@ def main():
 
     pcie = pcie_bandwidth()
     print("pcie", pcie, flush=True)
+    def apply_options(c, devs):
+        """Every option of the run on context c whose devices are `devs` (indices into caps)."""
+        c.set_option("sm_partition", args.sm_partition)
+        c.set_option("ooc_keep", args.ooc_keep)
+        c.set_option("ooc_buffers", args.ooc_buffers)
+        for j, i in enumerate(devs):
+            c.set_device_option(j, "c_cap_bytes", c_caps[i])
+
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
-    ctx.set_option("sm_partition", args.sm_partition)
-    ctx.set_option("ooc_keep", args.ooc_keep)
-    ctx.set_option("ooc_buffers", args.ooc_buffers)
-    for dev, cap in enumerate(c_caps):
-        ctx.set_device_option(dev, "c_cap_bytes", cap)
+    apply_options(ctx, range(p))
     t0 = time.perf_counter()
     models, sample_info = [], []
     if args.concurrent:
@@ -129,10 +133,7 @@ def main():
     if args.link_group:    # the link-sharing devices again, together in a context of their own
         grp = [int(i) for i in args.link_group.split(",")]
         with pkg.Context.local([0] * len(grp), sm_caps=[caps[i] for i in grp]) as gctx:
-            gctx.set_option("ooc_keep", args.ooc_keep)
-            gctx.set_option("ooc_buffers", args.ooc_buffers)
-            for j, i in enumerate(grp):
-                gctx.set_device_option(j, "c_cap_bytes", c_caps[i])
+            apply_options(gctx, grp)
             gsp = list(zip(*gctx.sample(-1, b, sizes, pkg.FPM_F32)))
         for j, i in enumerate(grp):
             per_dev[i] = gsp[j]
@@ -189,7 +190,7 @@ def main():
                    "ncal": args.ncal, "x_cal": x_cal, "sizes": sizes, "ooc_keep": args.ooc_keep, "ooc_buffers": args.ooc_buffers,
                    "link_group": args.link_group,
                    "sampling": "concurrent (all devices at once)" if args.concurrent else "exclusive",
-                   "dtype": "f32 (auto scheme: F16I8 for b % 64 == 0, DESIGN Q15b)", "sm_partition": args.sm_partition,
+                   "dtype": "f32 (auto scheme: F16X3, DESIGN Q15)", "sm_partition": args.sm_partition,
                    "gpu": "1x B200; devices emulated by SM caps, device memory by C caps (C_i out of core above)"},
         "pcie": pcie, "fpm_sample_s": t_sample, "models": sample_info, "table": table,
     }

@@ -79,6 +79,30 @@ def matrix_pm1(seed: int, N: int, dtype=np.float32) -> np.ndarray:
     return rect(seed, N, 0, 0, N, N, DIST_PM1, dtype)
 
 
+# Stress distributions for the FP32 parity tests: inputs whose
+# magnitudes vary inside a row, which fixed-point-per-row schemes cannot carry.
+# Drawn from independent streams of the same counter-based generator.
+_STREAM2 = 0x632BE59BD9B4E019
+_STREAM3 = 0x8CB92BA72F3D8DD7
+
+
+def gaussian(seed: int, N: int, r0: int, c0: int, h: int, w: int, dtype=np.float32) -> np.ndarray:
+    """N(0, 1) by Box-Muller from two 53-bit uniforms of the element's counter."""
+    idx = _indices(N, r0, c0, h, w)
+    u1 = ((_hash(seed, idx) >> np.uint64(11)).astype(np.float64) + 1.0) * 2.0 ** -53   # (0, 1]
+    u2 = (_hash(seed ^ _STREAM2, idx) >> np.uint64(11)).astype(np.float64) * 2.0 ** -53
+    return (np.sqrt(-2.0 * np.log(u1)) * np.cos(2.0 * np.pi * u2)).astype(dtype)
+
+
+def lognormal_signed(seed: int, N: int, r0: int, c0: int, h: int, w: int, sigma: float = 1.0,
+                     dtype=np.float32) -> np.ndarray:
+    """Random sign times exp(sigma g), g ~ N(0, 1): magnitudes spread over
+    e^(+-4 sigma) inside every row and column."""
+    g = gaussian(seed, N, r0, c0, h, w, np.float64)
+    sgn = np.where((_hash(seed ^ _STREAM3, _indices(N, r0, c0, h, w)) >> np.uint64(63)) == 0, 1.0, -1.0)
+    return (sgn * np.exp(sigma * g)).astype(dtype)
+
+
 def matrix_int(seed: int, N: int, dtype=np.float32) -> np.ndarray:
     return rect(seed, N, 0, 0, N, N, DIST_INT, dtype)
 

@@ -1,4 +1,4 @@
-"""F16I8, the default FP32 scheme of the rank-b update (reading Q15b):
+"""F16I8, the opt-in (not FP32-class) FP32 scheme of the rank-b update (reading Q15b):
 x 2^e = h0 + h1 (h0 fp16), int8 codes q = clamp(rint(x 2^e / 256), +-127) and
 l = rint(8 h1); C += 2^-(ea+eb) (h0a h0b' + 32 (qa lb' + la qb')) with the fp16
 product on kind::f16 and the two cross terms as ONE kind::i8 product.

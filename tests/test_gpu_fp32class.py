@@ -1,0 +1,206 @@
+"""The DEFAULT FP32 path is FP32-class (Q15; PAPER.md P:33, P:39, P:77:
+the paper's experiments are single precision; north_star: C within 1e-5
+relative Frobenius error of the oracle).
+
+Inputs whose magnitudes vary inside every row and column -- Gaussian,
+signed lognormal (sigma = 1: e^(+-4) spread) and pivot blocks anti-scaled by
+8^(+-1) along K -- are exactly where a scheme that is fixed point relative to
+the row maximum (F16I8, Q15b, opt-in only) loses accuracy.  Every test here
+runs with default options (no "f32_scheme", no "fuse", no tail option), at a
+single fused update (K = 2048), at the fused download tail (one operand over
+many pivots, one scale per row), and at the bench's full e2e size (c5,
+N = 49152: sampled rows and blocks of the host C vs the oracle, plus
+Freivalds' check on all of C)."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import gemm as og
+
+pytestmark = pytest.mark.gpu
+
+torch = pytest.importorskip("torch")
+import paper_conf_cluster_zhongrl12_b200 as pkg  # noqa: E402
+
+TOL = 1e-5
+DISTS = ["pm1", "gauss", "lognormal1", "antiscaled8"]
+
+
+@pytest.fixture(autouse=True)
+def _cuda():
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    yield
+
+
+def _antiscale(A, B, b, factor=8.0):
+    """Block-column k of A times factor^s_k, block-row k of B times factor^-s_k,
+    s_k = +1, -1, +1, ... (powers of two: exact; the product is unchanged in
+    magnitude but every row's magnitudes differ by factor^2 between pivots)."""
+    n = A.shape[1] // b
+    for k in range(n):
+        s = np.float32(factor if k % 2 == 0 else 1.0 / factor)
+        A[:, k * b:(k + 1) * b] *= s
+        B[k * b:(k + 1) * b, :] /= s
+
+
+def make_inputs(dist, N, b, seed=21):
+    if dist == "pm1":
+        A, B = synth.rect(seed, N, 0, 0, N, N), synth.rect(seed + 1, N, 0, 0, N, N)
+    elif dist == "gauss":
+        A, B = synth.gaussian(seed, N, 0, 0, N, N), synth.gaussian(seed + 1, N, 0, 0, N, N)
+    elif dist == "lognormal1":
+        A = synth.lognormal_signed(seed, N, 0, 0, N, N, 1.0)
+        B = synth.lognormal_signed(seed + 1, N, 0, 0, N, N, 1.0)
+    elif dist == "antiscaled8":
+        A, B = synth.rect(seed, N, 0, 0, N, N), synth.rect(seed + 1, N, 0, 0, N, N)
+        _antiscale(A, B, b)
+    else:
+        raise ValueError(dist)
+    return np.ascontiguousarray(A), np.ascontiguousarray(B)
+
+
+@pytest.mark.parametrize("dist", DISTS)
+@pytest.mark.parametrize("p", [1, 3])
+def test_default_path_one_fused_update(dist, p):
+    """N = 2048, b = 1024: the two pivots are ONE fused update of K = 2048 (auto
+    fuse), one scale per row over both, through pmm_run with default options."""
+    N, b = 2048, 1024
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n] if p == 1 else [2, 1, 1])
+    A, B = make_inputs(dist, N, b)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0] * p) as ctx:
+        ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+    err = og.rel_fro(C, og.gemm(A, B))
+    assert err <= TOL, (dist, p, err)
+
+
+@pytest.mark.parametrize("dist", DISTS)
+def test_default_path_k2048_b512_multi_device(dist):
+    """b = 512 (configs 3 / 4): four pivots fused per update (K = 2048), three
+    devices whose A slices come from several holders."""
+    N, b = 2048, 512
+    n = N // b
+    rects = pkg.colpart_arrange(n, [8, 4, 4])
+    A, B = make_inputs(dist, N, b, seed=31)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0, 0, 0]) as ctx:
+        ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+    err = og.rel_fro(C, og.gemm(A, B))
+    assert err <= TOL, (dist, err)
+
+
+def _sampled_check(C, A, B, rows, cols):
+    """rel-Fro of whole sampled rows and whole sampled columns of C vs the oracle."""
+    errs = []
+    ref_r = og.gemm(np.ascontiguousarray(A[rows, :]), B)
+    errs.append(og.rel_fro(C[rows, :], ref_r))
+    ref_c = og.gemm(A, np.ascontiguousarray(B[:, cols]))
+    errs.append(og.rel_fro(C[:, cols], ref_c))
+    return max(errs)
+
+
+def _freivalds(C, A, B, nvec=4, seed=0, chunk=4096):
+    """max over +-1 vectors x of ||C x - A (B x)|| / ||A (B x)|| (FP64, row chunks)."""
+    rng = np.random.default_rng(seed)
+    X = rng.choice([-1.0, 1.0], size=(C.shape[1], nvec))
+    BX = np.zeros((B.shape[0], nvec))
+    for r in range(0, B.shape[0], chunk):
+        BX[r:r + chunk] = B[r:r + chunk].astype(np.float64) @ X
+    num = np.zeros(nvec)
+    den = np.zeros(nvec)
+    for r in range(0, A.shape[0], chunk):
+        ref = A[r:r + chunk].astype(np.float64) @ BX
+        got = C[r:r + chunk].astype(np.float64) @ X
+        num += np.sum((got - ref) ** 2, axis=0)
+        den += np.sum(ref ** 2, axis=0)
+    return float(np.max(np.sqrt(num / den)))
+
+
+@pytest.mark.parametrize("dist", DISTS)
+def test_default_path_fused_tail(dist):
+    """N = 12288, b = 1024 through pmm_run with default options on one device:
+    the band-streamed fused download tail stages several fused groups as ONE
+    operand (K up to tail_K) with one scale per row / column over all of it."""
+    N, b = 12288, 1024
+    n = N // b
+    A, B = make_inputs(dist, N, b, seed=41)
+    C = np.full((N, N), np.nan, np.float32)
+    with pkg.Context.local([0]) as ctx:
+        st = ctx.run(A, B, C, N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+        assert st.updates >= 1
+    assert not np.isnan(C).any()
+    rng = np.random.default_rng(5)
+    rows = np.unique(np.concatenate([[0, N - 1], rng.integers(0, N, 14)]))
+    cols = np.unique(np.concatenate([[0, N - 1], rng.integers(0, N, 14)]))
+    err = _sampled_check(C, A, B, rows, cols)
+    assert err <= TOL, (dist, err)
+    fr = _freivalds(C, A, B)
+    assert fr <= 10 * TOL, (dist, fr)
+
+
+@pytest.mark.parametrize("stress", ["pm1", "antiscaled8"])
+def test_c5_e2e_full_size(stress):
+    """The bench's e2e call at c5 (N = 49152, b = 1024, p = 1): pmm_run with
+    default options on pinned host buffers (band-streamed fused tail), inputs
+    the bench's (seeds 5, 6 from the counter-based generator), optionally
+    anti-scaled along K.  Sampled rows (all columns), corner / interior blocks
+    vs the oracle; Freivalds on all of C."""
+    N, b = 49152, 1024
+    n = N // b
+    free, _ = torch.cuda.mem_get_info(0)
+    if free < 3.5 * 3 * N * N * 4:
+        pytest.skip("not enough device memory")
+    hA = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
+    hB = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
+    hC = torch.empty((N, N), dtype=torch.float32, pin_memory=True)
+    tmp = torch.empty((N, N), dtype=torch.float32, device="cuda")
+    sa, sb = synth.seeds_for_config(4)
+    pkg.k_fill_synthetic(tmp, pkg.FPM_F32, N, sa, N, 0, 0, N, N)
+    hA.copy_(tmp)
+    pkg.k_fill_synthetic(tmp, pkg.FPM_F32, N, sb, N, 0, 0, N, N)
+    hB.copy_(tmp)
+    del tmp
+    torch.cuda.empty_cache()
+    A, B, C = hA.numpy(), hB.numpy(), hC.numpy()
+    # the device generator is the host generator (tests/test_gpu_kernels.py); spot-check here too
+    np.testing.assert_array_equal(A[N - 3:N, N - 70:N], synth.rect(sa, N, N - 3, N - 70, 3, 70))
+    if stress == "antiscaled8":
+        _antiscale(A, B, b)
+    C.fill(np.nan)
+    with pkg.Context.local([0]) as ctx:
+        ctx.run(A, B, C, N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+    assert not np.isnan(C[::97, ::89]).any()
+    rng = np.random.default_rng(49152)
+    rows = np.unique(np.concatenate([[0, N - 1, N // 2], rng.integers(0, N, 9)]))
+    err_rows = og.rel_fro(C[rows, :], og.gemm(np.ascontiguousarray(A[rows, :]), B))
+    assert err_rows <= TOL, (stress, "rows", err_rows)
+    for (r0, c0) in [(0, 0), (N - 64, N - 64), (0, N - 64), (N - 64, 0), (20000, 31000)]:
+        ref = og.gemm(np.ascontiguousarray(A[r0:r0 + 64, :]), np.ascontiguousarray(B[:, c0:c0 + 64]))
+        e = og.rel_fro(C[r0:r0 + 64, c0:c0 + 64], ref)
+        assert e <= TOL, (stress, r0, c0, e)
+    fr = _freivalds(C, A, B, chunk=2048)
+    assert fr <= 10 * TOL, (stress, fr)
+
+
+def test_f16i8_opt_in_is_not_fp32_class():
+    """The opt-in F16I8 scheme (Q15b) is fixed point relative to the row maximum:
+    on anti-scaled pivot blocks it misses 1e-5 (documented limit), while it
+    still meets its own normwise bound K 2^-16 max|A| max|B| per element and
+    the default scheme meets 1e-5 on the same input."""
+    N, b = 2048, 1024
+    A, B = make_inputs("antiscaled8", N, b, seed=51)
+    ref = og.gemm(A, B)
+    out = {}
+    for scheme in (pkg.SCHEME_F16I8, -1):
+        C = np.full((N, N), np.nan, np.float32)
+        with pkg.Context.local([0]) as ctx:
+            ctx.set_option("f32_scheme", scheme)
+            ctx.run(A, B, C, N, b, [(0, 0, 0, 2, 2)], pkg.FPM_F32)
+        out[scheme] = C
+    assert og.rel_fro(out[-1], ref) <= TOL
+    e8 = og.rel_fro(out[pkg.SCHEME_F16I8], ref)
+    assert e8 > TOL, e8   # if this ever passes, F16I8's documented limit (Q15b) is wrong
+    bound = N * 2.0 ** -16 * np.abs(A).max(axis=1)[:, None] * np.abs(B).max(axis=0)[None, :]
+    assert np.all(np.abs(out[pkg.SCHEME_F16I8] - ref) <= bound)

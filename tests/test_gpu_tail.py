@@ -40,7 +40,7 @@ def test_run_with_tail_parity(tail, p, tail_fuse):
     assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
 
 
-@pytest.mark.parametrize("scheme", [pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])
+@pytest.mark.parametrize("scheme", [-1, pkg.SCHEME_F16X3, pkg.SCHEME_TF32X3])   # -1: the default (auto)
 def test_fused_tail_common_scale_over_groups(scheme):
     """Fused tail: every row / column takes ONE F16X3 scale over all tail pivots
     (maxima merged across groups and holders).  Block-columns of A and

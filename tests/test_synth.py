@@ -43,3 +43,18 @@ def test_known_hash_values():
 
 def test_seeds_differ():
     assert not np.array_equal(synth.matrix_pm1(1, 32), synth.matrix_pm1(2, 32))
+
+
+def test_stress_distributions_moments_and_windows():
+    """Gaussian / signed-lognormal stress inputs: right moments, and a window of
+    the global matrix equals the same entries of the whole matrix (counter-based)."""
+    N = 600
+    g = synth.gaussian(7, N, 0, 0, N, N, np.float64)
+    assert abs(g.mean()) < 0.01 and abs(g.std() - 1.0) < 0.01
+    assert abs(np.mean(g ** 4) - 3.0) < 0.1            # Gaussian kurtosis
+    np.testing.assert_array_equal(synth.gaussian(7, N, 100, 50, 30, 40, np.float64), g[100:130, 50:90])
+    lg = synth.lognormal_signed(7, N, 0, 0, N, N, 1.0, np.float64)
+    mag = np.log(np.abs(lg))
+    assert abs(mag.mean()) < 0.01 and abs(mag.std() - 1.0) < 0.01
+    assert abs((lg > 0).mean() - 0.5) < 0.01
+    np.testing.assert_array_equal(synth.lognormal_signed(7, N, 5, 9, 3, 4, 1.0, np.float64), lg[5:8, 9:13])
