@@ -115,7 +115,7 @@ def committed_traffic(N: int, b: int, args):
     """DRAM bytes per update launch from the committed ncu capture of the same
     configuration (profiles/ncu_traffic.json), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    variant = (6 if args.scheme == "f16i8" else 4) if args.kernel_variant < 0 else args.kernel_variant
+    variant = (6 if args.scheme == "f16i8" else 7) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
     G = args.raster_group if args.raster_group > 0 else (12 if args.scheme == "f16i8" else 16)
     key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}") + ("" if G == 16 else f"_r{G}")
@@ -234,6 +234,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         c.set_option("raster_group", args.raster_group)
         c.set_option("l2_hint_b", args.l2_hint_b)
         c.set_option("kernel_variant", args.kernel_variant)
+        c.set_option("chunk_k", args.chunk_k)
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
         c.set_option("e2e_tail", args.e2e_tail)
@@ -392,7 +393,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
                 "N": N, "b": b, "p": p, "partition": d, "rects": rects,
                 "f32_scheme": args.scheme, "cta_group": args.cta_group, "raster_group": args.raster_group,
-                "kernel_variant": args.kernel_variant, "fuse": args.fuse,
+                "kernel_variant": args.kernel_variant, "chunk_k": args.chunk_k, "fuse": args.fuse,
                 "update_launches_per_step": upd_launches,
                 "transport": transport,
                 "l2": (f"inputs larger than L2 (A, B, C {N * N * 4 / 1e9:.2f} GB each)" if N * N * 4 > 126e6
@@ -521,6 +522,7 @@ def main():
     ap.add_argument("--raster-group", type=int, default=0, help="0 = auto (12 for F16I8, 16 otherwise)")
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
+    ap.add_argument("--chunk-k", type=int, default=0, help="K per TMEM accumulation (variants 7/8; 0 auto = 512)")
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--tail-stream", type=int, default=1, help="pmm_run option tail_stream (e2e, one device)")

@@ -169,7 +169,26 @@ int colpart_plan_step(int64_t n, int32_t p, const colpart_rect* rects, int64_t k
  * emulation (BASELINE north_star): the persistent rank-b update kernel, which
  * holds one SM per CTA, runs with a grid of `cap` CTAs.  Pivot
  * transfers between devices are device-to-device copies on the receivers'
- * communication streams.  Errors: FPM_EINVAL, FPM_ECUDA, FPM_EUNSUPPORTED. */
+ * communication streams.
+ *
+ * cuda_devices[i] = FPM_CPU_DEVICE makes device i a host-CPU device (PAPER.md
+ * a socket of c cores executing the GEMM kernel
+ * simultaneously): sm_caps[i] = c cores (0 = every core left), taken as
+ * consecutive cores of the process's affinity mask after those of earlier CPU
+ * devices -- and after the first core when the context drives GPUs (a
+ * core dedicated to the GPU); pmm_set_device_option "cpu_first_core" moves
+ * them.  Its A_i, B_i, C_i live in host memory (pinned and mapped when GPUs
+ * are present: their staging kernels read its pivots directly); its update is
+ * the host GEMM of fpm_k_cpu_gemm on its c pinned cores, rows split evenly;
+ * its k-loop runs on a thread of its own, concurrently with the GPU devices'
+ * streams, pulling pivots held by GPU devices device -> host one update group
+ * ahead.  A CPU device is a device of the partition chosen by the caller,
+ * never a fallback: GPU devices' updates always run on their GPUs.  Contexts
+ * with only CPU devices need no GPU.  Not available in NCCL / IPC contexts;
+ * fpm_sample(dev = -1) is FPM_EUNSUPPORTED with CPU devices (sample each).
+ * Errors: FPM_EINVAL, FPM_ECUDA, FPM_EUNSUPPORTED (SM cap or cores not
+ * available). */
+#define FPM_CPU_DEVICE (-1)
 int pmm_create_local(int32_t p, const int32_t* cuda_devices, const int32_t* sm_caps,
                      pmm_ctx** out);
 
@@ -287,9 +306,13 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 normwise, not elementwise; Q15b); needs cta_group
  *                 2, b % 64 == 0 and K <= 131072 per update.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
- *   "kernel_variant": -1 (auto, default: F16X3 4, F16I8 6 -- 5 in NCCL
+ *   "kernel_variant": -1 (auto, default: F16X3 / TF32X3 7, F16I8 6; in NCCL
  *                 contexts, whose kernels need shared memory beside the
- *                 update) or 0..6, see fpm_k_update_f32.
+ *                 update, 8 and 5) or 0..8, see fpm_k_update_f32.
+ *   "chunk_k":    variants 7 / 8: K summed per TMEM accumulation before the
+ *                 epilogue adds it to its FP32 register sum (0 = auto = 512;
+ *                 DESIGN.md Q15c: the tensor cores' accumulation error grows
+ *                 with the MMAs folded into one sum).
  *   "fuse":       pivots fused into one rank-(f b) update (FP32): 0 = auto
  *                 (f = min(8, max(1, 2048 / b))), else 1..8.  Groups never
  *                 straddle a column or row boundary of the arrangement, so a
@@ -412,7 +435,11 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * x 2 + 6, 3 = 64-byte x 5 + 4, 4 = 128-byte x 2 + 4 (leaves ~36 KB smem per
  * SM for NCCL / staging kernels co-running with the update), 5 = 128-byte x 3
  * + 2 with C updated by TMA reduce-add (C never loaded into shared memory);
- * -1 = auto (4).
+ * variants 0..5 sum a whole update in one TMEM accumulation.  7 (auto) =
+ * chunked accumulation: every 512 of K is a fresh TMEM accumulation drained
+ * into per-thread FP32 register sums (round-to-nearest), C written once per
+ * tile by TMA reduce-add (store when accumulate = 0), 3 x 64-KB operand
+ * stages; 8 = the same with 2 stages.  -1 = auto (7).
  * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
  * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks,
  * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 5 = variant
@@ -449,6 +476,31 @@ int fpm_k_update_f64(const double* A, int64_t lda, const double* Bt, double* C, 
  * starting at global (r0, c0); dt = FPM_F32 or FPM_F64; dist = fpm_dist. */
 int fpm_k_fill_synthetic(void* dst, int32_t dt, int64_t ld, uint64_t seed, int64_t N, int64_t r0,
                          int64_t c0, int64_t rows, int64_t cols, int32_t dist, void* stream);
+
+/* ---------------------------------------------------- host-CPU devices */
+
+/* Host-CPU rank-b update kernel of the CPU devices (a
+ * socket of c cores executing the GEMM kernel simultaneously; SURVEY §8(f)
+ * NEXT-3), callable on its own: C (M x N, ldc) (+)= A (M x K) x B (K x N, ldb),
+ * host pointers, row-major, dt = FPM_F32 (FP32 FMA arithmetic: SGEMM) or
+ * FPM_F64.  A is read in K-segments of `seg` columns:
+ * A(i, k) = A[(k / seg) * seg_stride + i * lda + k % seg] (seg = K,
+ * seg_stride = 0 for a plain row-major A) -- the layout of a device's
+ * block-column panels.  threads: worker threads (rows of C split evenly across
+ * them), pinned to the first `threads` cores of this process's affinity mask
+ * when pin != 0, else unpinned.  accumulate = 0 overwrites C.  Needs no GPU.
+ * Errors: FPM_EINVAL (bad shape, threads < 1). */
+int fpm_k_cpu_gemm(int32_t dt, int64_t M, int64_t N, int64_t K, const void* A, int64_t lda, int64_t seg,
+                   int64_t seg_stride, const void* B, int64_t ldb, void* C, int64_t ldc, int32_t accumulate,
+                   int32_t threads, int32_t pin);
+
+/* Micro-kernel instruction set of the CPU GEMM on this host: writes
+ * "avx512", "avx2" or "generic" (NUL-terminated, at most cap bytes). */
+int fpm_cpu_isa(char* out, int32_t cap);
+
+/* Host cores this process may use (its affinity mask), ascending: writes
+ * min(count, cap) core ids to cores_out and the count to *count. */
+int fpm_cpu_cores(int32_t* cores_out, int32_t cap, int32_t* count);
 
 #ifdef __cplusplus
 }

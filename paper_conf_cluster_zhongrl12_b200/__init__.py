@@ -16,7 +16,7 @@ import ctypes
 from typing import List, Sequence, Tuple
 
 from . import _lib
-from ._lib import (FPM_DIST_INT, FPM_DIST_PM1, FPM_F32, FPM_F64, SCHEME_F16I8, SCHEME_F16X3, SCHEME_TF32X3,  # noqa: F401,E501
+from ._lib import (FPM_CPU_DEVICE, FPM_DIST_INT, FPM_DIST_PM1, FPM_F32, FPM_F64, SCHEME_F16I8, SCHEME_F16X3, SCHEME_TF32X3,  # noqa: F401,E501
                    FpmError, PmmStats, check, lib)
 
 Model = Tuple[Sequence[int], Sequence[float]]
@@ -272,3 +272,37 @@ def k_update_f64(A, lda, Bt, C, M, Nc, K, ldc, accumulate=True, stream=None):
 def k_fill_synthetic(dst, dtype, ld, seed, N, r0, c0, rows, cols, dist=FPM_DIST_PM1, stream=None):
     check(lib.fpm_k_fill_synthetic(_lib._ptr(dst), dtype, ld, seed, N, r0, c0, rows, cols, dist,
                                    _stream(stream)))
+
+
+# ------------------------------------------------------- host-CPU devices
+def k_cpu_gemm(A, B, C, accumulate: bool = False, threads: int = 1, pin: bool = False,
+               M: int | None = None, N: int | None = None, K: int | None = None,
+               lda: int | None = None, seg: int = 0, seg_stride: int = 0, ldb: int | None = None,
+               ldc: int | None = None) -> None:
+    """The CPU devices' GEMM (include/fpmpmm.h fpm_k_cpu_gemm) on host numpy
+    arrays: C (+)= A B, FP32 or FP64 (from C's dtype)."""
+    import numpy as np
+    dt = FPM_F64 if C.dtype == np.float64 else FPM_F32
+    M = C.shape[0] if M is None else M
+    N = C.shape[1] if N is None else N
+    K = B.shape[0] if K is None else K
+    lda = (A.strides[0] // A.itemsize) if lda is None else lda
+    ldb = (B.strides[0] // B.itemsize) if ldb is None else ldb
+    ldc = (C.strides[0] // C.itemsize) if ldc is None else ldc
+    check(lib.fpm_k_cpu_gemm(dt, int(M), int(N), int(K), _lib._ptr(A), int(lda), int(seg), int(seg_stride),
+                             _lib._ptr(B), int(ldb), _lib._ptr(C), int(ldc), 1 if accumulate else 0, int(threads),
+                             1 if pin else 0))
+
+
+def cpu_isa() -> str:
+    buf = ctypes.create_string_buffer(16)
+    check(lib.fpm_cpu_isa(buf, 16))
+    return buf.value.decode()
+
+
+def cpu_cores() -> list:
+    n = _lib.i32(0)
+    check(lib.fpm_cpu_cores(None, 0, ctypes.byref(n)))
+    arr = (_lib.i32 * max(1, n.value))()
+    check(lib.fpm_cpu_cores(arr, n.value, ctypes.byref(n)))
+    return list(arr[:n.value])

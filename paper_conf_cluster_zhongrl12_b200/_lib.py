@@ -29,7 +29,8 @@ FPM_DIST_INT = 1
 
 SCHEME_F16X3 = 0
 SCHEME_TF32X3 = 1
-SCHEME_F16I8 = 3      # fp16 main product + int8 cross terms (default for b % 64 == 0)
+SCHEME_F16I8 = 3      # fp16 main product + int8 cross terms (opt-in: not FP32-class, DESIGN Q15b)
+FPM_CPU_DEVICE = -1   # cuda_devices[i] of a host-CPU device (pmm_create_local)
 
 i32, i64, u64, dbl, vp = ctypes.c_int32, ctypes.c_int64, ctypes.c_uint64, ctypes.c_double, ctypes.c_void_p
 
@@ -118,6 +119,9 @@ _SIGS = {
     "fpm_k_update_f64": ([vp, i64, vp, vp, i64, i64, i64, i64, i32, vp], ctypes.c_int),
     "fpm_k_prof": ([i32, ctypes.POINTER(u64)], ctypes.c_int),
     "fpm_k_fill_synthetic": ([vp, i32, i64, u64, i64, i64, i64, i64, i64, i32, vp], ctypes.c_int),
+    "fpm_k_cpu_gemm": ([i32, i64, i64, i64, vp, i64, i64, i64, vp, i64, vp, i64, i32, i32, i32], ctypes.c_int),
+    "fpm_cpu_isa": ([ctypes.c_char_p, i32], ctypes.c_int),
+    "fpm_cpu_cores": ([ctypes.POINTER(i32), i32, ctypes.POINTER(i32)], ctypes.c_int),
 }
 for _name, (_args, _res) in _SIGS.items():
     _fn = getattr(lib, _name)

@@ -73,6 +73,7 @@ struct UpdParams {
     int group;        // raster group (tile-rows)
     uint64_t hint_b;  // L2 policy of the B^T tiles (A tiles: evict_last, C: evict_first)
     int prof;         // F16I8: accumulate MMA-issuer wait cycles into g_hyb_prof (fpm_k_prof)
+    int chunk_kb;     // chunked kernel: k-blocks per TMEM accumulation
 };
 
 // Diagnostic counters of the F16I8 MMA issuer (leader CTAs, lane 0), summed over
@@ -346,6 +347,263 @@ __global__ void __launch_bounds__(192, 1)
     if (warp == 1) {
         ptx::tc_fence_after();
         ptx::tmem_dealloc<CG>(tmem_base, Cfg::TMEM_COLS);
+    }
+}
+
+
+// ------------------------------------ F16X3 / TF32X3, chunked accumulation (default)
+// The tensor cores add every MMA's products into the FP32 accumulator with a
+// truncated (not round-to-nearest) alignment, so the accumulation error of one
+// TMEM sum grows with the number of MMAs folded into it: F16X3 over one K =
+// 4096 sum measured 1.3e-5 rel-Fro, over the fused tail's K = 24576 4.0e-5
+// (U[-1,1); reading Q15c).  This kernel bounds it: the K range of a tile is cut
+// into chunks of chunk_kb k-blocks; each chunk is a fresh TMEM accumulation
+// (double-buffered: 2 x 256 columns), which the epilogue drains and adds to a
+// per-thread FP32 register sum (round-to-nearest), so each element carries the
+// error of a K = 512 accumulation plus one FP32 rounding per chunk -- like an
+// SGEMM's blocked accumulation -- whatever the update's K.  C is written once
+// per tile: the scaled sum staged in shared memory and added to C by a TMA
+// reduce-add (C never enters shared memory), or stored when the update
+// overwrites C.  Eight epilogue warps (two per TMEM lane quarter, one per
+// 128-column half of the 256-column tile) each hold 128 running sums.
+//   warp 0: TMA producer (A hi/lo, B^T hi/lo k-blocks, 128-byte swizzle)
+//   warp 1: TMEM allocation + single-thread tcgen05.mma issuer (leader CTA)
+//   warps 2-9: epilogue
+template <int KIND, int STAGES, int NCB>
+struct AccCfg {
+    static constexpr int BM = 128, TILE_M = 256, BN = 256, BN_CTA = 128, SW = 128;
+    static constexpr int ELEM = KIND == 1 ? 4 : 2;
+    static constexpr int BK = SW / ELEM;
+    static constexpr int KSTEPS = SW / 32;
+    static constexpr int A_BYTES = BM * SW, B_BYTES = BN_CTA * SW;
+    static constexpr int STAGE_BYTES = 2 * (A_BYTES + B_BYTES);
+    static constexpr int NCBH = NCB / 2;
+    static constexpr int C_CHUNK_BYTES = BM * 128;
+    static constexpr int BAR_BYTES = 8 * (2 * STAGES + 4) + 16;
+    static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + NCB * C_CHUNK_BYTES + BAR_BYTES;
+    static constexpr uint32_t IDESC = ptx::idesc_f32acc(TILE_M, BN, KIND == 1);
+    static constexpr int THREADS = 320;
+    static_assert(NCB % 2 == 0 && NCBH >= 1 && NCBH <= 4, "C staging: 1..4 chunks per half");
+    static_assert(SMEM <= 232448, "shared memory budget");
+};
+
+template <int KIND, int STAGES, int NCB>
+__global__ void __launch_bounds__(320, 1)
+    update_acc_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
+                      const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
+                      const __grid_constant__ CUtensorMap tmC, const UpdParams P) {
+    using Cfg = AccCfg<KIND, STAGES, NCB>;
+    extern __shared__ uint8_t smem_raw[];
+    uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
+    uint8_t* stage_base = smem;
+    uint8_t* cbuf = smem + STAGES * Cfg::STAGE_BYTES;
+    uint64_t* bars = reinterpret_cast<uint64_t*>(cbuf + NCB * Cfg::C_CHUNK_BYTES);
+    uint64_t* full = bars;                     // [STAGES]
+    uint64_t* empty = bars + STAGES;           // [STAGES]
+    uint64_t* tfull = bars + 2 * STAGES;       // [2]
+    uint64_t* tempty = bars + 2 * STAGES + 2;  // [2]
+    uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 4);
+
+    const uint32_t warp = threadIdx.x / 32;
+    const uint32_t lane = threadIdx.x % 32;
+    const uint32_t rank = ptx::cluster_ctarank();
+    const bool leader = rank == 0;
+    const int cluster_id = blockIdx.x / 2;
+    const int num_clusters = gridDim.x / 2;
+
+    if (threadIdx.x == 0) {
+        for (int s = 0; s < STAGES; ++s) {
+            ptx::mbar_init(&full[s], 1);
+            ptx::mbar_init(&empty[s], 1);
+        }
+        for (int a = 0; a < 2; ++a) {
+            ptx::mbar_init(&tfull[a], 1);
+            ptx::mbar_init(&tempty[a], 8 * 2);  // every epilogue warp of both CTAs
+        }
+        ptx::fence_mbar_init();
+    }
+    if (warp == 0 && lane == 0) {
+        ptx::tma_prefetch_desc(&tmA_hi);
+        ptx::tma_prefetch_desc(&tmA_lo);
+        ptx::tma_prefetch_desc(&tmB_hi);
+        ptx::tma_prefetch_desc(&tmB_lo);
+        ptx::tma_prefetch_desc(&tmC);
+    }
+    if (warp == 1) {
+        ptx::tmem_alloc<2>(tmem_slot, 512);
+        ptx::tmem_relinquish<2>();
+    }
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::cluster_sync();
+    ptx::tc_fence_after();
+    const uint32_t tmem_base = *tmem_slot;
+    const int num_kb = (P.K + Cfg::BK - 1) / Cfg::BK;
+    const int ckb = P.chunk_kb > 0 ? P.chunk_kb : num_kb;
+
+    if (warp == 0) {
+        // ------------------------------------------------------------ producer
+        if (lane == 0) {
+            int stage = 0;
+            uint32_t phase = 0;
+            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+                int tm, tn;
+                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+                const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
+                const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA;
+                for (int kb = 0; kb < num_kb; ++kb) {
+                    ptx::mbar_wait(&empty[stage], phase ^ 1);
+                    uint8_t* sA_hi = stage_base + stage * Cfg::STAGE_BYTES;
+                    uint8_t* sA_lo = sA_hi + Cfg::A_BYTES;
+                    uint8_t* sB_hi = sA_lo + Cfg::A_BYTES;
+                    uint8_t* sB_lo = sB_hi + Cfg::B_BYTES;
+                    const int k0 = kb * Cfg::BK;
+                    if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
+                    ptx::tma_load_2d_cg2(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
+                    ptx::tma_load_2d_cg2(sA_lo, &tmA_lo, &full[stage], k0, m0, ptx::kEvictLast);
+                    ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
+                    ptx::tma_load_2d_cg2(sB_lo, &tmB_lo, &full[stage], k0, n0, P.hint_b);
+                    if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                }
+            }
+        }
+    } else if (warp == 1) {
+        // ----------------------------------------------------------- MMA issuer
+        if (leader) {
+            int stage = 0;
+            uint32_t phase = 0;
+            int it = 0;  // accumulations issued (chunks over all tiles)
+            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+                for (int kb0 = 0; kb0 < num_kb; kb0 += ckb, ++it) {
+                    const int acc = it & 1;
+                    ptx::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);
+                    ptx::tc_fence_after();
+                    const uint32_t d_tmem = tmem_base + acc * Cfg::BN;
+                    const int kb1 = min(kb0 + ckb, num_kb);
+                    for (int kb = kb0; kb < kb1; ++kb) {
+                        ptx::mbar_wait(&full[stage], phase);
+                        ptx::tc_fence_after();
+                        if (lane == 0) {
+                            const uint32_t a_hi = ptx::smem_u32(stage_base + stage * Cfg::STAGE_BYTES);
+                            const uint32_t a_lo = a_hi + Cfg::A_BYTES;
+                            const uint32_t b_hi = a_lo + Cfg::A_BYTES;
+                            const uint32_t b_lo = b_hi + Cfg::B_BYTES;
+                            const uint64_t dA_hi = ptx::sdesc_k<128>(a_hi), dA_lo = ptx::sdesc_k<128>(a_lo);
+                            const uint64_t dB_hi = ptx::sdesc_k<128>(b_hi), dB_lo = ptx::sdesc_k<128>(b_lo);
+#pragma unroll
+                            for (int k = 0; k < Cfg::KSTEPS; ++k) {
+                                const uint64_t off = (uint64_t)(k * 32) >> 4;  // 32 B per MMA k-step
+                                // small products first, the h0 h0' product last (Q15)
+                                ptx::umma<2, KIND>(d_tmem, dA_lo + off, dB_hi + off, Cfg::IDESC,
+                                                   (kb != kb0 || k != 0) ? 1u : 0u);
+                                ptx::umma<2, KIND>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
+                                ptx::umma<2, KIND>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
+                            }
+                            ptx::umma_commit<2>(&empty[stage]);
+                        }
+                        __syncwarp();
+                        if (++stage == STAGES) { stage = 0; phase ^= 1; }
+                    }
+                    if (lane == 0) ptx::umma_commit<2>(&tfull[acc]);
+                    __syncwarp();
+                }
+            }
+        }
+    } else {
+        // -------------------------------------------------------------- epilogue
+        const uint32_t e = threadIdx.x - 64;  // 0..255
+        const uint32_t hh = e / 128;          // 128-column half of the tile
+        const uint32_t eh = e % 128;
+        const uint32_t q = warp & 3;          // TMEM lane quarter this warp may access
+        const uint32_t r = q * 32 + lane;     // row of the CTA tile
+        const uint32_t bar_id = 1 + hh;
+        uint8_t* cb = cbuf + hh * Cfg::NCBH * Cfg::C_CHUNK_BYTES;
+        int it = 0;
+        for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+            int tm, tn;
+            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+            const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
+            const int n0 = tn * Cfg::BN + (int)hh * 128;
+            float s[128];
+            for (int kb0 = 0; kb0 < num_kb; kb0 += ckb, ++it) {
+                const int acc = it & 1;
+                ptx::mbar_wait(&tfull[acc], (it >> 1) & 1);
+                ptx::tc_fence_after();
+                const uint32_t t_row = tmem_base + ((q * 32) << 16) + acc * Cfg::BN + hh * 128;
+#pragma unroll
+                for (int c = 0; c < 8; ++c) {
+                    uint32_t u[16];
+                    ptx::tmem_ld_32x32b_x16_nw(t_row + 16 * c, u);
+                    ptx::tmem_wait_ld();
+                    if (kb0 == 0) {
+#pragma unroll
+                        for (int j = 0; j < 16; ++j) s[16 * c + j] = __uint_as_float(u[j]);
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 16; ++j) s[16 * c + j] = __fadd_rn(s[16 * c + j], __uint_as_float(u[j]));
+                    }
+                }
+                // accumulator read: hand it back to the MMA warp
+                ptx::tc_fence_before();
+                __syncwarp();
+                if (lane == 0) ptx::mbar_arrive_cluster(&tempty[acc], 0);
+            }
+            // C update of this tile: C (+)= 2^-(ea+eb) s, once per tile (overlaps the next tile's MMAs)
+            const int grow = m0 + (int)r;
+            const float sa = (P.sa != nullptr && grow < P.M) ? P.sa[grow] : 1.0f;
+#pragma unroll
+            for (int c = 0; c < 4; ++c) {
+                const int buf = c % Cfg::NCBH;
+                float* v = s + 32 * c;
+                if (P.sb != nullptr) {
+                    const int gc = n0 + 32 * c;
+                    if (gc + 32 <= P.Nc) {
+                        const float4* sb4 = reinterpret_cast<const float4*>(P.sb + gc);
+#pragma unroll
+                        for (int j = 0; j < 8; ++j) {
+                            const float4 s4 = __ldg(sb4 + j);
+                            v[4 * j + 0] *= sa * s4.x;
+                            v[4 * j + 1] *= sa * s4.y;
+                            v[4 * j + 2] *= sa * s4.z;
+                            v[4 * j + 3] *= sa * s4.w;
+                        }
+                    } else {
+#pragma unroll
+                        for (int j = 0; j < 32; ++j) {
+                            const float sbj = (gc + j < P.Nc) ? __ldg(P.sb + gc + j) : 0.0f;
+                            v[j] *= sa * sbj;
+                        }
+                    }
+                }
+                // the buffer's previous TMA (chunk c - NCBH) has read it
+                if (eh == 0) ptx::bulk_wait_read_n<Cfg::NCBH - 1>();
+                ptx::named_bar_sync(bar_id, 128);
+                uint8_t* rowp = cb + buf * Cfg::C_CHUNK_BYTES + r * 128;
+#pragma unroll
+                for (int j = 0; j < 8; ++j)
+                    *reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4)) =
+                        make_float4(v[4 * j + 0], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+                ptx::fence_proxy_async_smem();
+                ptx::named_bar_sync(bar_id, 128);
+                if (eh == 0) {
+                    if (P.load_c)
+                        ptx::tma_reduce_add_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
+                                                    ptx::kEvictFirst);
+                    else
+                        ptx::tma_store_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0, ptx::kEvictFirst);
+                    ptx::bulk_commit();
+                }
+            }
+        }
+        if (eh == 0) ptx::bulk_wait0();
+    }
+
+    ptx::tc_fence_before();
+    __syncthreads();
+    ptx::cluster_sync();
+    if (warp == 1) {
+        ptx::tc_fence_after();
+        ptx::tmem_dealloc<2>(tmem_base, 512);
     }
 }
 
@@ -788,6 +1046,59 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
     if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
 }
 
+
+template <int KIND, int STAGES, int NCB>
+static void launch_update_acc_t(const UpdateArgs& a, cudaStream_t st) {
+    using Cfg = AccCfg<KIND, STAGES, NCB>;
+    const CUtensorMapDataType odt = KIND == 1 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
+    const CUtensorMap tAh = make_tmap_2d(a.a_hi, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
+    const CUtensorMap tAl = make_tmap_2d(a.a_lo, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
+    const CUtensorMap tBh = make_tmap_2d(a.bt_hi, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+    const CUtensorMap tBl = make_tmap_2d(a.bt_lo, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+    const CUtensorMap tC = make_tmap_2d(a.C, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.M, a.Nc, a.ldc, 32, Cfg::BM);
+    UpdParams P;
+    P.M = (int)a.M;
+    P.Nc = (int)a.Nc;
+    P.K = (int)a.K;
+    P.tiles_m = (int)((a.M + Cfg::TILE_M - 1) / Cfg::TILE_M);
+    P.tiles_n = (int)((a.Nc + Cfg::BN - 1) / Cfg::BN);
+    P.num_tiles = P.tiles_m * P.tiles_n;
+    P.sa = a.sa;
+    P.sb = a.sb;
+    P.load_c = a.accumulate ? 1 : 0;
+    P.group = a.raster_group > 0 ? a.raster_group : 16;
+    P.hint_b = a.l2_hint_b == 2 ? ptx::kEvictLast : (a.l2_hint_b == 1 ? ptx::kEvictFirst : ptx::kEvictNormal);
+    P.prof = 0;
+    const int chunk_k = a.chunk_k > 0 ? a.chunk_k : 512;
+    P.chunk_kb = (chunk_k + Cfg::BK - 1) / Cfg::BK;
+    auto kern = update_acc_kernel<KIND, STAGES, NCB>;
+    static uint64_t attr_done = 0;  // one bit per CUDA device
+    int dev = 0;
+    cudaGetDevice(&dev);
+    if (!(attr_done & (1ull << dev))) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+        attr_done |= 1ull << dev;
+    }
+    int clusters = a.num_sms / 2;
+    if (clusters > P.num_tiles) clusters = P.num_tiles;
+    if (clusters < 1) clusters = 1;
+    cudaLaunchConfig_t cfg = {};
+    cfg.gridDim = dim3(clusters * 2);
+    cfg.blockDim = dim3(Cfg::THREADS);
+    cfg.dynamicSmemBytes = Cfg::SMEM;
+    cfg.stream = st;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tAh, tAl, tBh, tBl, tC, P);
+    if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
+}
+
 template <int SW, int STAGES, int NCB, int MC = 1, int PROBE = 0, bool RED = false>
 static void launch_update_hyb_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = HybCfg<SW, STAGES, NCB>;
@@ -871,10 +1182,11 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.ldc % 4 == 0 && a.ldc >= a.Nc, "ldc must be >= Nc and a multiple of 4");
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
-    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 5) ||
+    FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 5) || ((a.variant == 7 || a.variant == 8) && a.scheme != SplitScheme::F16I8) ||
                       (a.variant >= 6 && a.variant <= 11 && a.variant != 7 && a.variant != 8 &&
                        a.scheme == SplitScheme::F16I8),
-                  "kernel variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
+                  "kernel variant must be -1 (auto), 0..5, 7, 8 (F16X3 / TF32X3) or 6, 9..11 (F16I8)");
+    FPM_CHECK_ARG(a.chunk_k >= 0, "chunk_k must be >= 0");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
     if (a.scheme == SplitScheme::F16I8) {
         FPM_CHECK_ARG(a.cta_group == 2, "F16I8 runs on CTA pairs (cta_group 2)");
@@ -905,13 +1217,20 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
         else launch_update_t<2, 2, 256, 2, 128, 4>(a, st);
         return;
     }
-    // auto: variant 4 (two 64-KB operand stages, four C chunks in flight): as fast
-    // as variant 2 (six C chunks) at the fused K = 2048 (429 TFLOP/s both, c5) and
-    // leaves ~36 KB of shared memory per SM for kernels that must co-run with the
-    // persistent update (NCCL, staging of other emulated devices)
-    const int variant = a.variant >= 0 ? a.variant : 4;
+    // auto: variant 7 (chunked accumulation, three 64-KB operand stages, C by TMA
+    // reduce-add): the FP32-class error bound at every K (Q15c).  Variants 0..5
+    // accumulate a whole update in one TMEM sum (error grows with K).
+    const int variant = a.variant >= 0 ? a.variant : 7;
     if (a.cta_group == 2) {
         switch (variant) {
+            case 7:  // chunked accumulation, 3 stages + 2 C staging chunks (224 KB)
+                if (tf32) launch_update_acc_t<1, 3, 2>(a, st);
+                else launch_update_acc_t<0, 3, 2>(a, st);
+                break;
+            case 8:  // chunked accumulation, 2 stages + 2 C staging chunks (160 KB): room for NCCL kernels
+                if (tf32) launch_update_acc_t<1, 2, 2>(a, st);
+                else launch_update_acc_t<0, 2, 2>(a, st);
+                break;
             case 1:  // 64-B k-blocks x 4 stages, 6 C chunks in flight
                 if (tf32) launch_update_t<2, 1, 256, 4, 64, 6>(a, st);
                 else launch_update_t<2, 0, 256, 4, 64, 6>(a, st);

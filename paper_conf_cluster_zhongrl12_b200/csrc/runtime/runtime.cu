@@ -14,13 +14,18 @@
 #include <cuda_runtime.h>
 
 #include <algorithm>
+#include <chrono>
 #include <cmath>
+#include <cstdlib>
 #include <cstring>
+#include <exception>
 #include <memory>
 #include <string>
+#include <thread>
 #include <vector>
 
 #include "../common.hpp"
+#include "../host/cpu_device.hpp"
 #include "../host/host_algos.hpp"
 #include "../kernels/kernels.hpp"
 #include "green.hpp"
@@ -121,6 +126,21 @@ struct Device {
     std::vector<void*> allocs;
     int64_t launches = 0;                   // library kernels launched (running count)
 
+    // host-CPU device (cuda_dev = FPM_CPU_DEVICE; a socket
+    // of c cores running the GEMM kernel together): A_i, B_i, C_i in host memory
+    // (pinned and mapped when the context has GPUs, so their staging kernels read
+    // this device's pivots directly), its update on a team of pinned cores
+    bool cpu = false;
+    int cores = 0;                          // c
+    int first_core = -1;                    // index of its first core in the affinity mask
+    cpu::Team* team = nullptr;
+    std::vector<void*> plain_allocs;        // host memory without a GPU in the context
+    void* h_arecv[2] = {}, *h_brecv[2] = {}; // gathered pivots of a group
+    std::vector<std::pair<int, cudaStream_t>> pulls;  // (CUDA ordinal, stream) of device -> host pivot pulls
+    std::vector<double> cpu_pack_s, cpu_upd_s;         // per group, last k-loop
+    double cpu_loop_s = 0.0;                // last k-loop, wall time
+    int64_t cpu_bytes = 0;                  // pivot bytes received in the last k-loop
+
     bool live() const { return H > 0 && W > 0; }
 };
 
@@ -150,6 +170,7 @@ struct pmm_ctx {
     int raster_group = 0;  // 0 = auto: 12 for F16I8, 16 otherwise (measured, c5)
     int l2_hint_b = 0;
     int kernel_variant = -1;  // auto
+    int chunk_k = 0;          // F16X3 / TF32X3 default kernel: K per TMEM accumulation (0 auto = 512)
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
@@ -184,14 +205,26 @@ void* dalloc(Device& d, size_t bytes) {
     return p;
 }
 
-void* halloc(Device& d, size_t bytes) {
+void* halloc(Device& d, size_t bytes, unsigned flags = cudaHostAllocPortable) {
     void* p = nullptr;
-    cudaError_t e = cudaHostAlloc(&p, bytes, cudaHostAllocPortable);
+    cudaError_t e = cudaHostAlloc(&p, bytes, flags);
     if (e != cudaSuccess) {
         cudaGetLastError();
         fail(FPM_ENOMEM, "cudaHostAlloc(%zu): %s", bytes, cudaGetErrorString(e));
     }
     d.host_allocs.push_back(p);
+    return p;
+}
+
+// Memory of a CPU device: pinned and mapped (device-accessible through its UVA
+// address, so GPU devices' staging kernels pull its pivots directly) when the
+// context drives GPUs, plain aligned host memory otherwise.
+void* cpu_mem(Device& d, size_t bytes, bool pinned) {
+    if (bytes == 0) return nullptr;
+    if (pinned) return halloc(d, bytes, cudaHostAllocPortable | cudaHostAllocMapped);
+    void* p = nullptr;
+    if (posix_memalign(&p, 64, bytes) != 0) fail(FPM_ENOMEM, "host allocation of %zu bytes failed", bytes);
+    d.plain_allocs.push_back(p);
     return p;
 }
 
@@ -332,6 +365,17 @@ void bp_join(BandPipe& bp, cudaStream_t s) {
 }
 
 void free_problem(Device& d) {
+    if (d.cpu) {
+        for (auto& ps : d.pulls) cudaStreamSynchronize(ps.second);
+        for (void* p : d.plain_allocs) std::free(p);
+        d.plain_allocs.clear();
+        for (void* p : d.host_allocs) cudaFreeHost(p);
+        d.host_allocs.clear();
+        d.A = d.B = d.C = nullptr;
+        for (int s = 0; s < 2; ++s) d.h_arecv[s] = d.h_brecv[s] = nullptr;
+        d.H = d.W = 0;
+        return;
+    }
     cudaSetDevice(d.cuda_dev);
     if (d.bp.s_d2h) cudaStreamSynchronize(d.bp.s_d2h);
     bp_release_bands(d.bp);
@@ -361,6 +405,14 @@ void free_problem(Device& d) {
 }
 
 void init_device(Device& d) {
+    if (d.cpu) {  // a team of c worker threads pinned to its cores (P:10 (i))
+        const std::vector<int> all = cpu::allowed_cores();
+        if (d.cores < 1 || d.first_core < 0 || d.first_core + d.cores > (int)all.size())
+            fail(FPM_EUNSUPPORTED, "CPU device %d: cores [%d, %d) outside the %zu cores of the affinity mask", d.idx,
+                 d.first_core, d.first_core + d.cores, all.size());
+        d.team = cpu::team_create(std::vector<int>(all.begin() + d.first_core, all.begin() + d.first_core + d.cores));
+        return;
+    }
     CU(cudaSetDevice(d.cuda_dev));
     int sms = 0;
     CU(cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, d.cuda_dev));
@@ -396,6 +448,16 @@ void init_device(Device& d) {
 
 void destroy_device(Device& d) {
     free_problem(d);
+    if (d.cpu) {
+        for (auto& ps : d.pulls) {
+            cudaSetDevice(ps.first);
+            cudaStreamDestroy(ps.second);
+        }
+        d.pulls.clear();
+        cpu::team_destroy(d.team);
+        d.team = nullptr;
+        return;
+    }
     cudaSetDevice(d.cuda_dev);
     bp_destroy(d.bp);
     for (int s = 0; s < kSlots; ++s) {
@@ -469,17 +531,17 @@ void set_sm_partition(pmm_ctx* ctx, bool green) {
     std::vector<GreenPartition> parts(ctx->devs.size());
     if (green) {
         for (auto& d : ctx->devs)
-            if (d.sm_cap == 0)
+            if (!d.cpu && d.sm_cap == 0)
                 fail(FPM_EUNSUPPORTED, "sm_partition = 1 needs an SM cap on every device (device %d has none)", d.idx);
         try {
             std::vector<int> gpus;
             for (auto& d : ctx->devs)
-                if (std::find(gpus.begin(), gpus.end(), d.cuda_dev) == gpus.end()) gpus.push_back(d.cuda_dev);
+                if (!d.cpu && std::find(gpus.begin(), gpus.end(), d.cuda_dev) == gpus.end()) gpus.push_back(d.cuda_dev);
             for (int g : gpus) {  // one split per GPU: the partitions of its devices are disjoint
                 std::vector<size_t> on;
                 std::vector<int> caps;
                 for (size_t i = 0; i < ctx->devs.size(); ++i)
-                    if (ctx->devs[i].cuda_dev == g) {
+                    if (!ctx->devs[i].cpu && ctx->devs[i].cuda_dev == g) {
                         on.push_back(i);
                         caps.push_back(ctx->devs[i].sm_cap);
                     }
@@ -492,9 +554,12 @@ void set_sm_partition(pmm_ctx* ctx, bool green) {
         }
     }
     close_peers(ctx);
-    for (auto& d : ctx->devs) destroy_device(d);
+    for (auto& d : ctx->devs)
+        if (!d.cpu) destroy_device(d);
+        else free_problem(d);
     ctx->have_problem = false;
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
+        if (ctx->devs[i].cpu) continue;
         ctx->devs[i].green = parts[i];
         init_device(ctx->devs[i]);
     }
@@ -510,6 +575,28 @@ const void* src_A(pmm_ctx* ctx, int q) {
 const void* src_B(pmm_ctx* ctx, int q) {
     if (ctx->ipc_mode) return q == ctx->rank ? ctx->devs[0].B : ctx->peer_B[q];
     return local_dev(ctx, q)->B;
+}
+
+bool has_gpu(const pmm_ctx* ctx) {
+    for (auto& d : ctx->devs)
+        if (!d.cpu) return true;
+    return false;
+}
+bool has_cpu(const pmm_ctx* ctx) {
+    for (auto& d : ctx->devs)
+        if (d.cpu) return true;
+    return false;
+}
+
+// A CPU device's stream for pulling pivots out of GPU `cuda_dev`'s memory.
+cudaStream_t pull_stream(Device& d, int cuda_dev) {
+    for (auto& ps : d.pulls)
+        if (ps.first == cuda_dev) return ps.second;
+    cudaStream_t s = nullptr;
+    CU(cudaSetDevice(cuda_dev));
+    CU(cudaStreamCreateWithFlags(&s, cudaStreamNonBlocking));
+    d.pulls.push_back({cuda_dev, s});
+    return s;
 }
 
 // Pivots fused per update (FP32 only): option "fuse", 0 = auto = K of about 2048
@@ -616,7 +703,27 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
     ctx->fuse_max = f;
 
     const size_t es = esize(dt);
+    const bool pinned = has_gpu(ctx);
     for (auto& d : ctx->devs) {
+        if (d.cpu) {  // host rectangles; receive buffers for the pivots of one group (two slots)
+            d.rect = rects[d.idx];
+            d.H = d.rect.h * b;
+            d.W = d.rect.w * b;
+            if (!d.live()) {
+                d.H = d.W = 0;
+                continue;
+            }
+            const size_t HW = (size_t)d.H * d.W;
+            d.A = cpu_mem(d, HW * es, pinned);
+            d.B = cpu_mem(d, HW * es, pinned);
+            d.C = cpu_mem(d, HW * es, false);
+            std::memset(d.C, 0, HW * es);
+            for (int s = 0; s < 2; ++s) {
+                d.h_arecv[s] = cpu_mem(d, (size_t)d.H * f * b * es, pinned);
+                d.h_brecv[s] = cpu_mem(d, (size_t)f * b * d.W * es, pinned);
+            }
+            continue;
+        }
         CU(cudaSetDevice(d.cuda_dev));
         d.rect = rects[d.idx];
         d.H = d.rect.h * b;
@@ -662,6 +769,7 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         NC(nccl().CommSplit(ctx->world_comm, color, ctx->rank, &ctx->col_comm, nullptr));
     }
     for (auto& d : ctx->devs) {
+        if (d.cpu) continue;
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaDeviceSynchronize());
     }
@@ -900,10 +1008,11 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.accumulate = ctx->groups[g].first != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
     a.raster_group = ctx->raster_group > 0 ? ctx->raster_group : (sch == SplitScheme::F16I8 ? 12 : 16);
     a.l2_hint_b = ctx->l2_hint_b;
-    a.variant = ctx->kernel_variant;  // -1: auto (F16X3: variant 4; F16I8: 6)
+    a.variant = ctx->kernel_variant;  // -1: auto (F16X3 / TF32X3: variant 7; F16I8: 6)
+    a.chunk_k = ctx->chunk_k;
     // NCCL kernels need shared memory to co-run with the persistent update:
-    // F16I8 then takes variant 5 (198 KB) instead of 6 (224 KB)
-    if (a.variant < 0 && ctx->nccl_mode && sch == SplitScheme::F16I8) a.variant = 5;
+    // F16I8 then takes variant 5 (198 KB) instead of 6 (224 KB), F16X3 8 (2 stages) instead of 7
+    if (a.variant < 0 && ctx->nccl_mode) a.variant = sch == SplitScheme::F16I8 ? 5 : 8;
     return a;
 }
 
@@ -999,7 +1108,8 @@ int tail_groups(pmm_ctx* ctx, bool streamed) {
     const double rate_per_sm = scheme_for(ctx, ctx->b) == SplitScheme::F16I8 ? 3.9e12 : 3.0e12;  // measured, c5
     double r = 0.0;
     for (auto& d : ctx->devs)
-        if (d.live() && !d.ooc) r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (rate_per_sm * d.num_sms)));
+        if (d.live() && !d.ooc && !d.cpu)
+            r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (rate_per_sm * d.num_sms)));
     if (r == 0.0) return 0;
     int L = (int)std::ceil(G * 1.05 * r);
     if (streamed && streamed_tail_ok(ctx) && r < 0.5)  // 0.55: the tail may start somewhat late (measured, c5:
@@ -1024,7 +1134,7 @@ bool use_fused_tail(const pmm_ctx* ctx) { return ctx->tail_fuse && ctx->dt == FP
 // One device holding the whole problem (p = 1, local): its tail operand can be
 // staged from rows that arrive band by band.
 bool streamed_tail_ok(const pmm_ctx* ctx) {
-    return ctx->tail_stream && use_fused_tail(ctx) && !ctx->ipc_mode && ctx->devs.size() == 1 &&
+    return ctx->tail_stream && use_fused_tail(ctx) && !ctx->ipc_mode && ctx->devs.size() == 1 && !ctx->devs[0].cpu &&
            ctx->devs[0].live() && !ctx->devs[0].ooc && ctx->devs[0].rect.h * ctx->b == ctx->N &&
            ctx->devs[0].rect.w * ctx->b == ctx->N;
 }
@@ -1147,6 +1257,143 @@ void capture_kloop(pmm_ctx* ctx);
 void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<char>* tail_done, int64_t bytes,
                   int64_t launches);
 
+// ------------------------------------------------------------ CPU devices
+// The k-loop of a host-CPU device (P:15's iteration on a socket, P:18 kernel):
+// per update group, gather A(rows_i, k0..kl) and B(k0..kl, cols_i) into host
+// receive buffers -- pieces held by GPU devices are pulled device -> host on
+// this device's pull streams, pieces of CPU devices copied -- then
+// C_i (+)= A B with the team's GEMM.  The next group's pulls are issued before
+// the current GEMM (two slots), so they overlap it.  Pivot sources are resident
+// inputs that the loop never writes, so no ordering with the GPU streams is
+// needed (pmm_compute's inputs are resident before it starts).
+void cpu_kloop(pmm_ctx* ctx, Device& d) {
+    using clk = std::chrono::steady_clock;
+    const auto t_begin = clk::now();
+    const int G = (int)ctx->groups.size();
+    const size_t es = esize(ctx->dt);
+    const int64_t b = ctx->b;
+    const colpart_rect& r = d.rect;
+    d.cpu_pack_s.assign(G, 0.0);
+    d.cpu_upd_s.assign(G, 0.0);
+    d.cpu_bytes = 0;
+    struct Op {
+        const void* A = nullptr;
+        int64_t seg_stride = 0;  // A: f panels of H x b (row stride b), seg_stride apart
+        const void* B = nullptr; // B: f b rows of W
+        std::vector<cudaStream_t> wait;
+    };
+    auto secs = [](clk::time_point a, clk::time_point z) { return std::chrono::duration<double>(z - a).count(); };
+    auto gather = [&](int g, int slot) {
+        const auto t0 = clk::now();
+        Op op;
+        const int64_t k0 = ctx->groups[g].first;
+        const int f = ctx->groups[g].second;
+        auto copy = [&](void* dst, const void* src, size_t bytes, const Device* q) {
+            if (q->cpu) {
+                std::memcpy(dst, src, bytes);
+            } else {
+                cudaStream_t st = pull_stream(d, q->cuda_dev);
+                CU(cudaSetDevice(q->cuda_dev));
+                CU(cudaMemcpyAsync(dst, src, bytes, cudaMemcpyDeviceToHost, st));
+                if (std::find(op.wait.begin(), op.wait.end(), st) == op.wait.end()) op.wait.push_back(st);
+            }
+            d.cpu_bytes += (int64_t)bytes;
+        };
+        if (r.col0 <= k0 && k0 < r.col0 + r.w) {  // own block-columns
+            op.A = static_cast<const char*>(d.A) + (size_t)(k0 - r.col0) * d.H * b * es;
+        } else {
+            for (const Move& m : ctx->plan_a[k0]) {
+                if (m.dst != d.idx) continue;
+                const Device* q = local_dev(ctx, m.src);
+                const colpart_rect& qr = ctx->rects[m.src];
+                const int64_t qH = qr.h * b;
+                const size_t cnt = (size_t)(m.end - m.begin) * b * b * es;
+                const char* src = static_cast<const char*>(q->A) +
+                                  ((size_t)(k0 - qr.col0) * qH * b + (size_t)(m.begin - qr.row0) * b * b) * es;
+                for (int j = 0; j < f; ++j)
+                    copy(static_cast<char*>(d.h_arecv[slot]) + ((size_t)j * d.H * b + (size_t)(m.begin - r.row0) * b * b) * es,
+                         src + (size_t)j * qH * b * es, cnt, q);
+            }
+            op.A = d.h_arecv[slot];
+        }
+        op.seg_stride = d.H * b;
+        if (r.row0 <= k0 && k0 < r.row0 + r.h) {  // own block-rows
+            op.B = static_cast<const char*>(d.B) + (size_t)(k0 - r.row0) * b * d.W * es;
+        } else {
+            for (const Move& m : ctx->plan_b[k0]) {
+                if (m.dst != d.idx) continue;
+                const Device* q = local_dev(ctx, m.src);
+                const colpart_rect& orr = ctx->rects[m.src];
+                copy(d.h_brecv[slot], static_cast<const char*>(q->B) + (size_t)(k0 - orr.row0) * b * d.W * es,
+                     (size_t)f * b * d.W * es, q);
+                op.B = d.h_brecv[slot];
+            }
+        }
+        FPM_CHECK_ARG(op.B != nullptr, "no source of block-row %lld for CPU device %d", (long long)k0, d.idx);
+        d.cpu_pack_s[g] += secs(t0, clk::now());
+        return op;
+    };
+    auto wait = [&](const Op& op) {
+        for (cudaStream_t st : op.wait) CU(cudaStreamSynchronize(st));
+    };
+    Op cur = gather(0, 0);
+    wait(cur);
+    for (int g = 0; g < G; ++g) {
+        Op nxt;
+        if (g + 1 < G) nxt = gather(g + 1, (g + 1) & 1);  // pulls of the next group under this GEMM
+        const int64_t K = (int64_t)ctx->groups[g].second * b;
+        const bool acc = ctx->groups[g].first != 0;  // the first update writes C_i = A(0..) B(0..)
+        const auto t0 = clk::now();
+        if (ctx->dt == FPM_F32)
+            cpu::gemm_f32(d.team, d.H, d.W, K, static_cast<const float*>(cur.A), b, b, cur.seg_stride,
+                          static_cast<const float*>(cur.B), d.W, static_cast<float*>(d.C), d.W, acc);
+        else
+            cpu::gemm_f64(d.team, d.H, d.W, K, static_cast<const double*>(cur.A), b, b, cur.seg_stride,
+                          static_cast<const double*>(cur.B), d.W, static_cast<double*>(d.C), d.W, acc);
+        d.cpu_upd_s[g] = secs(t0, clk::now());
+        if (g + 1 < G) {
+            wait(nxt);
+            cur = nxt;
+        }
+    }
+    d.cpu_loop_s = secs(t_begin, clk::now());
+}
+
+// Runs every live CPU device's k-loop on a thread of its own for the lifetime
+// of the object; join() waits and re-throws the first failure.
+struct CpuLoops {
+    std::vector<std::thread> threads;
+    std::vector<std::exception_ptr> errs;
+    explicit CpuLoops(pmm_ctx* ctx) {
+        size_t n = 0;
+        for (auto& d : ctx->devs) n += (d.cpu && d.live()) ? 1 : 0;
+        errs.assign(n, nullptr);  // sized before any thread holds a pointer into it
+        size_t i = 0;
+        for (auto& d : ctx->devs) {
+            if (!d.cpu || !d.live()) continue;
+            Device* dp = &d;
+            std::exception_ptr* e = &errs[i++];
+            threads.emplace_back([ctx, dp, e] {
+                try {
+                    cpu_kloop(ctx, *dp);
+                } catch (...) {
+                    *e = std::current_exception();
+                }
+            });
+        }
+    }
+    void join() {
+        for (auto& t : threads)
+            if (t.joinable()) t.join();
+        for (auto& e : errs)
+            if (e) std::rethrow_exception(e);
+    }
+    ~CpuLoops() {
+        for (auto& t : threads)
+            if (t.joinable()) t.join();
+    }
+};
+
 void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const HostDst* out = nullptr,
              std::vector<char>* tail_done = nullptr) {
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
@@ -1170,7 +1417,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
         Device& d = ctx->devs[i];
         d.tail_fused_run = false;
         d.tail_streamed_run = false;
-        if (L > 0 && d.live() && !d.ooc) {
+        if (L > 0 && d.live() && !d.ooc && !d.cpu) {
             // before the timed region (cudaMalloc synchronises)
             if (use_fused_tail(ctx)) {
                 const bool rows = host != nullptr && streamed_tail_ok(ctx);
@@ -1189,7 +1436,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
         d.bp.bytes = 0;
     }
     for (auto& d : ctx->devs) {
-        if (!d.live()) continue;
+        if (!d.live() || d.cpu) continue;
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaStreamSynchronize(d.s_comp));
         CU(cudaStreamSynchronize(d.s_comm));
@@ -1198,7 +1445,11 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     // captured on first use and replayed (option "graph")
     // (not with green partitions: measured, replays lose the per-device SM
     // confinement -- c4 analogue 0.37 s replayed vs 0.23 s issued eagerly)
-    const bool use_graph = ctx->graph && !host && !out && !ctx->nccl_mode && !ctx->sm_partition;
+    const bool use_graph = ctx->graph && !host && !out && !ctx->nccl_mode && !ctx->sm_partition && !has_cpu(ctx);
+    FPM_CHECK_ARG(!(host && has_cpu(ctx)), "streamed host input with CPU devices (pmm_run uploads first)");
+    // CPU devices run their k-loops on their own threads, concurrently with the
+    // GPU devices' streams (their pivots come from resident buffers only)
+    CpuLoops cpu_loops(ctx);
     int64_t bytes = 0, launches = 0;
     if (use_graph) {
         if (!ctx->gexec) capture_kloop(ctx);
@@ -1213,6 +1464,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
         launches = -launches0;
         for (auto& d : ctx->devs) launches += d.launches;
     }
+    cpu_loops.join();
     finish_kloop(ctx, st, host != nullptr, tail_done, bytes, launches);
 }
 
@@ -1317,6 +1569,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     const int ngroups = (int)ctx->groups.size();
     const int gt = ngroups - L;  // first tail group
     for (auto& d : ctx->devs) {
+        if (d.cpu) continue;
         CU(cudaSetDevice(d.cuda_dev));
         rec_t(d.ev_start, d.s_comp);
         if (!g_capturing) {  // (a capture forks every stream from its origin instead)
@@ -1328,7 +1581,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     int64_t bytes = 0;
     // tail devices take tail groups from slots 2.. and update them band-major
     // after the loop; everyone else (and every group before gt) as usual
-    auto in_tail = [&](const Device& d, int g) { return g >= gt && d.live() && !d.ooc; };
+    auto in_tail = [&](const Device& d, int g) { return g >= gt && d.live() && !d.ooc && !d.cpu; };
     auto slot_of = [&](const Device& d, int g) {
         return in_tail(d, g) ? (d.tail_fused_run ? kFusedSlot : 2 + (g - gt)) : (g & 1);
     };
@@ -1339,7 +1592,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
         if (streamed)
             for (int64_t k = k0; k < k0 + ctx->groups[g].second; ++k)
                 for (auto& d : ctx->devs)
-                    if (d.live() && !streamed_tail(d, g)) issue_upload(ctx, d, k, *host);
+                    if (d.live() && !d.cpu && !streamed_tail(d, g)) issue_upload(ctx, d, k, *host);
         if (ctx->nccl_mode) {
             // every rank takes part in the NCCL calls, live or not
             Device& d = ctx->devs[0];
@@ -1354,7 +1607,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
             continue;
         }
         for (auto& d : ctx->devs)
-            if (d.live() && !streamed_tail(d, g)) {
+            if (d.live() && !d.cpu && !streamed_tail(d, g)) {
                 const int slot = slot_of(d, g);
                 if (in_tail(d, g) && d.tail_fused_run) {  // fused tail, pass 1: merge the maxima
                     if (g == gt) {
@@ -1367,12 +1620,12 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
                 }
             }
         for (auto& d : ctx->devs)
-            if (d.live() && !in_tail(d, g)) issue_update(ctx, d, g, g & 1);
+            if (d.live() && !d.cpu && !in_tail(d, g)) issue_update(ctx, d, g, g & 1);
     }
     // fused tail, pass 2: split every tail group with the merged maxima into its
     // K range of the tail operand
     for (auto& d : ctx->devs) {
-        if (L == 0 || !d.live() || d.ooc || !d.tail_fused_run || d.tail_streamed_run) continue;
+        if (L == 0 || !d.live() || d.ooc || d.cpu || !d.tail_fused_run || d.tail_streamed_run) continue;
         CU(cudaSetDevice(d.cuda_dev));
         rec_t(d.ev_tpack0, d.s_comm);
         int64_t k_off = 0;
@@ -1385,11 +1638,12 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     }
     if (L > 0)
         for (auto& d : ctx->devs) {
-            if (!d.live() || d.ooc) continue;
+            if (!d.live() || d.ooc || d.cpu) continue;
             if (d.tail_streamed_run) issue_tail_streamed(ctx, d, gt, *host, *out);
             else issue_tail(ctx, d, gt, L, *out);
         }
     for (auto& d : ctx->devs) {
+        if (d.cpu) continue;
         CU(cudaSetDevice(d.cuda_dev));
         if (d.ooc) bp_join(d.bp, d.s_comp);  // C_i is complete once its last band is back in host memory
         rec_t(d.ev_stop, d.s_comp);
@@ -1472,6 +1726,11 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
     double t_max = 0.0, t_tail_copy = 0.0;
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
+        if (d.cpu) {
+            if (d.live()) t_max = std::max(t_max, d.cpu_loop_s);
+            bytes += d.live() ? d.cpu_bytes : 0;
+            continue;
+        }
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventSynchronize(d.ev_stop));
         CU(cudaStreamSynchronize(d.s_comm));
@@ -1490,7 +1749,7 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
         if (streamed) {
             double tu = 0.0;  // until the last host->device panel landed
             for (auto& d : ctx->devs)
-                if (d.live()) tu = std::max(tu, (double)elapsed_ms(d.ev_start, d.ev_up[ctx->n - 1]) * 1e-3);
+                if (d.live() && !d.cpu) tu = std::max(tu, (double)elapsed_ms(d.ev_start, d.ev_up[ctx->n - 1]) * 1e-3);
             st->t_upload_s = tu;
         }
         st->iters = ctx->n;
@@ -1508,12 +1767,16 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
         for (auto& d : ctx->devs) {
             if (!d.live()) continue;
             double comp = 0.0, upd = 0.0;
-            for (int g = 0; g < ngroups; ++g) {
+            for (int g = 0; g < ngroups && d.cpu; ++g) {  // host-timed gather + GEMM of each group
+                comp += d.cpu_pack_s[g] + d.cpu_upd_s[g];
+                upd += d.cpu_upd_s[g];
+            }
+            for (int g = 0; g < ngroups && !d.cpu; ++g) {
                 const double u = elapsed_ms(d.ev_upd0[g], d.ev_upd1[g]) * 1e-3;
                 comp += u + elapsed_ms(d.ev_pack0[g], d.ev_pack1[g]) * 1e-3;
                 upd += u;
             }
-            if (d.tail_fused_run) comp += elapsed_ms(d.ev_tpack0, d.ev_tpack1) * 1e-3;
+            if (d.tail_fused_run && !d.cpu) comp += elapsed_ms(d.ev_tpack0, d.ev_tpack1) * 1e-3;
             if (d.idx < FPM_MAX_DEVICES) {
                 st->per_dev_compute_s[d.idx] = comp;
                 st->per_dev_update_s[d.idx] = upd;
@@ -1550,8 +1813,18 @@ void upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld, int64_t row_
     for (auto& d : ctx->devs) {
         if (!d.live()) continue;
         check_window(ctx, d, ld, row_base, col_base);
-        CU(cudaSetDevice(d.cuda_dev));
         const int64_t R0 = d.rect.row0 * b - row_base, C0 = d.rect.col0 * b - col_base;
+        if (d.cpu) {  // host to host: block-column panels of A, rows of B
+            for (int64_t c = 0; c < d.rect.w; ++c)
+                copy_rows(static_cast<char*>(d.A) + (size_t)c * d.H * b * es, b * es,
+                          static_cast<const char*>(A) + ((size_t)R0 * ld + (size_t)(C0 + c * b)) * es, ld * es, b * es,
+                          d.H);
+            copy_rows(d.B, d.W * es, static_cast<const char*>(B) + ((size_t)R0 * ld + (size_t)C0) * es, ld * es,
+                      d.W * es, d.H);
+            std::memset(d.C, 0, (size_t)d.H * d.W * es);
+            continue;
+        }
+        CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventRecord(d.ev_io0, d.s_comp));
         for (int64_t c = 0; c < d.rect.w; ++c) {
             const char* src = static_cast<const char*>(A) + ((size_t)R0 * ld + (size_t)(C0 + c * b)) * es;
@@ -1564,7 +1837,7 @@ void upload(pmm_ctx* ctx, const void* A, const void* B, int64_t ld, int64_t row_
         CU(cudaEventRecord(d.ev_io1, d.s_comp));
     }
     for (auto& d : ctx->devs) {
-        if (!d.live()) continue;
+        if (!d.live() || d.cpu) continue;
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaEventSynchronize(d.ev_io1));
         t = std::max(t, (double)elapsed_ms(d.ev_io0, d.ev_io1) * 1e-3);
@@ -1583,12 +1856,16 @@ void download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t col_b
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
         if (!d.live() || (skip && (*skip)[i])) continue;
-        copied[i] = 1;
         check_window(ctx, d, ld, row_base, col_base);
-        CU(cudaSetDevice(d.cuda_dev));
         const int64_t R0 = d.rect.row0 * b - row_base, C0 = d.rect.col0 * b - col_base;
-        CU(cudaEventRecord(d.ev_io0, d.s_comp));
         char* dst = static_cast<char*>(C) + ((size_t)R0 * ld + (size_t)C0) * es;
+        if (d.cpu) {
+            copy_rows(dst, ld * es, d.C, d.W * es, d.W * es, d.H);
+            continue;
+        }
+        copied[i] = 1;
+        CU(cudaSetDevice(d.cuda_dev));
+        CU(cudaEventRecord(d.ev_io0, d.s_comp));
         if (d.ooc) {  // C_i already in host memory (compute joined its band copies)
             CU(cudaStreamSynchronize(d.bp.s_d2h));
             copy_rows(dst, ld * es, d.hC, d.W * es, d.W * es, d.H);
@@ -1614,8 +1891,16 @@ void fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int dist) {
     const int64_t b = ctx->b;
     for (auto& d : ctx->devs) {
         if (!d.live()) continue;
-        CU(cudaSetDevice(d.cuda_dev));
         const int64_t R0 = d.rect.row0 * b, C0 = d.rect.col0 * b;
+        if (d.cpu) {  // the same counter-based generator on the host
+            for (int64_t c = 0; c < d.rect.w; ++c)
+                cpu::fill_synthetic(d.team, static_cast<char*>(d.A) + (size_t)c * d.H * b * es, f64, b, seed_a, ctx->N,
+                                    R0, C0 + c * b, d.H, b, dist);
+            cpu::fill_synthetic(d.team, d.B, f64, d.W, seed_b, ctx->N, R0, C0, d.H, d.W, dist);
+            std::memset(d.C, 0, (size_t)d.H * d.W * es);
+            continue;
+        }
+        CU(cudaSetDevice(d.cuda_dev));
         for (int64_t c = 0; c < d.rect.w; ++c)
             launch_fill_synthetic(static_cast<char*>(d.A) + (size_t)c * d.H * b * es, f64, b, seed_a, ctx->N, R0,
                                   C0 + c * b, d.H, b, dist, d.s_comp);
@@ -1623,7 +1908,7 @@ void fill_synthetic(pmm_ctx* ctx, uint64_t seed_a, uint64_t seed_b, int dist) {
         if (!d.ooc) CU(cudaMemsetAsync(d.C, 0, (size_t)d.H * d.W * es, d.s_comp));
     }
     for (auto& d : ctx->devs) {
-        if (!d.live()) continue;
+        if (!d.live() || d.cpu) continue;
         CU(cudaSetDevice(d.cuda_dev));
         CU(cudaStreamSynchronize(d.s_comp));
     }
@@ -1649,20 +1934,8 @@ double t975(int df) {
 // between the maximum number of processes"), which captures the contention of
 // devices emulated on one GPU; each repetition launches the kernel on all
 // devices and times each on its own stream.  Outputs are then p x nsizes.
-void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes, int nsizes, double* speeds,
-            double* ci, int32_t* reps_out) {
-    FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype");
-    FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 && b >= 8 : b % 32 == 0 && b >= 32, "bad block size b");
-    FPM_CHECK_ARG(nsizes >= 1 && sizes && speeds, "bad sizes");
-    std::vector<Device*> devs;
-    if (dev == -1) {
-        for (auto& d : ctx->devs) devs.push_back(&d);
-    } else {
-        Device* d = local_dev(ctx, dev);
-        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
-        devs.push_back(d);
-    }
-    int64_t mmax = 0;
+// Side of each sample size x = m^2 blocks (P:18 sqrt(x) x sqrt(x) submatrices).
+std::vector<int64_t> sample_sides(const int64_t* sizes, int nsizes) {
     std::vector<int64_t> ms(nsizes);
     for (int j = 0; j < nsizes; ++j) {
         const int64_t x = sizes[j];
@@ -1672,8 +1945,89 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         while ((m + 1) * (m + 1) <= x) ++m;
         FPM_CHECK_ARG(m * m == x, "size %lld is not a perfect square (P:18 sqrt(x) x sqrt(x))", (long long)x);
         ms[j] = m;
-        mmax = std::max(mmax, m);
     }
+    return ms;
+}
+
+// Speed function of a CPU device: its kernel C (m b x m b) += A (m b x f b) B
+// (f b x m b) -- the k-loop's fused update -- run by all c cores of the device
+// at once, each on m b / c rows ("the speed of a socket executing the ACML
+// kernels simultaneously on c cores, with the problem size x / c on each
+// core"; P:10 (ii) synchronised cores), host-timed (the synchronous approach,
+// P:10), repeated under the same statistical stop rule as the GPU devices (Q8).
+void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vector<int64_t>& ms, double* speeds,
+                double* ci, int32_t* reps_out) {
+    using clk = std::chrono::steady_clock;
+    const int64_t fb = (int64_t)fuse_factor(ctx, dt, b) * b;
+    const int64_t L = *std::max_element(ms.begin(), ms.end()) * b;
+    const size_t es = esize(dt);
+    struct Buf {
+        void* p = nullptr;
+        ~Buf() { std::free(p); }
+    } A, B, C;
+    auto get = [&](Buf& x, size_t bytes) {
+        if (posix_memalign(&x.p, 64, std::max<size_t>(bytes, 64)) != 0) fail(FPM_ENOMEM, "host allocation failed");
+    };
+    get(A, (size_t)L * fb * es);
+    get(B, (size_t)fb * L * es);
+    get(C, (size_t)L * L * es);
+    cpu::fill_synthetic(d.team, A.p, dt == FPM_F64, fb, 101, L, 0, 0, L, fb, FPM_DIST_PM1);
+    cpu::fill_synthetic(d.team, B.p, dt == FPM_F64, L, 102, L, 0, 0, fb, L, FPM_DIST_PM1);
+    std::memset(C.p, 0, (size_t)L * L * es);
+    for (size_t j = 0; j < ms.size(); ++j) {
+        const int64_t Lx = ms[j] * b;
+        auto run = [&] {
+            const auto t0 = clk::now();
+            if (dt == FPM_F32)
+                cpu::gemm_f32(d.team, Lx, Lx, fb, static_cast<const float*>(A.p), fb, fb, 0,
+                              static_cast<const float*>(B.p), L, static_cast<float*>(C.p), Lx, true);
+            else
+                cpu::gemm_f64(d.team, Lx, Lx, fb, static_cast<const double*>(A.p), fb, fb, 0,
+                              static_cast<const double*>(B.p), L, static_cast<double*>(C.p), Lx, true);
+            return std::chrono::duration<double>(clk::now() - t0).count();
+        };
+        run();
+        run();  // two warm-ups
+        std::vector<double> ts;
+        double mean = 0.0, half = 0.0;
+        for (int r = 0; r < 50; ++r) {
+            ts.push_back(run());
+            const int nr = (int)ts.size();
+            mean = 0.0;
+            for (double t : ts) mean += t;
+            mean /= nr;
+            double var = 0.0;
+            for (double t : ts) var += (t - mean) * (t - mean);
+            var = nr > 1 ? var / (nr - 1) : 0.0;
+            half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
+            if (nr >= 5 && half <= 0.025 * mean) break;
+        }
+        const double x = (double)(ms[j] * ms[j]);
+        speeds[j] = 2.0 * x * (double)b * (double)b * (double)fb / mean;
+        if (ci) ci[j] = mean > 0 ? half / mean : 0.0;
+        if (reps_out) reps_out[j] = (int32_t)ts.size();
+    }
+}
+
+void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes, int nsizes, double* speeds,
+            double* ci, int32_t* reps_out) {
+    FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype");
+    FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 && b >= 8 : b % 32 == 0 && b >= 32, "bad block size b");
+    FPM_CHECK_ARG(nsizes >= 1 && sizes && speeds, "bad sizes");
+    const std::vector<int64_t> ms = sample_sides(sizes, nsizes);
+    std::vector<Device*> devs;
+    if (dev == -1) {
+        if (has_cpu(ctx))
+            fail(FPM_EUNSUPPORTED, "concurrent sampling (dev = -1) of a context with CPU devices: sample each "
+                                   "device (P:11: GPUs and sockets were measured separately)");
+        for (auto& d : ctx->devs) devs.push_back(&d);
+    } else {
+        Device* d = local_dev(ctx, dev);
+        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
+        if (d->cpu) return sample_cpu(ctx, *d, dt, b, ms, speeds, ci, reps_out);
+        devs.push_back(d);
+    }
+    const int64_t mmax = *std::max_element(ms.begin(), ms.end());
     const int64_t L = mmax * b;
     const size_t es = dt == FPM_F64 ? 8 : 4;
     const SplitScheme sch = scheme_for(ctx, b);
@@ -1778,6 +2132,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.raster_group = ctx->raster_group > 0 ? ctx->raster_group : (sch == SplitScheme::F16I8 ? 12 : 16);
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
+                a.chunk_k = ctx->chunk_k;
                 if (ooc) {
                     banded_update(s.mem.bp, ring_at(s.d, Lx), s.hC, Lx, (size_t)Lx * 4, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
@@ -1884,15 +2239,38 @@ extern "C" int pmm_create_local(int32_t p, const int32_t* cuda_devices, const in
         *out = nullptr;
         FPM_CHECK_ARG(p >= 1 && p <= FPM_MAX_DEVICES, "p = %d out of [1, %d]", p, FPM_MAX_DEVICES);
         FPM_CHECK_ARG(cuda_devices != nullptr, "null cuda_devices");
+        bool any_gpu = false;
+        for (int i = 0; i < p; ++i) {
+            FPM_CHECK_ARG(cuda_devices[i] >= 0 || cuda_devices[i] == FPM_CPU_DEVICE, "bad device %d",
+                          cuda_devices[i]);
+            any_gpu = any_gpu || cuda_devices[i] >= 0;
+        }
         int count = 0;
-        CU(cudaGetDeviceCount(&count));
+        if (any_gpu) CU(cudaGetDeviceCount(&count));
+        // CPU devices: consecutive cores of the affinity mask; with GPUs in the
+        // context the first core stays with the thread that drives them ("a
+        // CPU core is usually dedicated to deal with the GPU")
+        const int ncores = (int)fpm::cpu::allowed_cores().size();
+        int next_core = any_gpu ? 1 : 0;
         auto ctx = std::make_unique<pmm_ctx>();
         ctx->devs.resize(p);
         try {
             for (int i = 0; i < p; ++i) {
-                FPM_CHECK_ARG(cuda_devices[i] >= 0 && cuda_devices[i] < count, "CUDA device %d out of range",
-                              cuda_devices[i]);
                 ctx->devs[i].idx = i;
+                if (cuda_devices[i] == FPM_CPU_DEVICE) {
+                    fpm::Device& d = ctx->devs[i];
+                    d.cpu = true;
+                    d.cuda_dev = -1;
+                    d.cores = (sm_caps && sm_caps[i] > 0) ? sm_caps[i] : ncores - next_core;
+                    d.first_core = next_core;
+                    if (d.cores < 1 || next_core + d.cores > ncores)
+                        fpm::fail(FPM_EUNSUPPORTED, "CPU device %d: %d cores requested, %d of %d left", i, d.cores,
+                                  ncores - next_core, ncores);
+                    next_core += d.cores;
+                    fpm::init_device(d);
+                    continue;
+                }
+                FPM_CHECK_ARG(cuda_devices[i] < count, "CUDA device %d out of range", cuda_devices[i]);
                 ctx->devs[i].cuda_dev = cuda_devices[i];
                 ctx->devs[i].sm_cap = sm_caps ? sm_caps[i] : 0;
                 fpm::init_device(ctx->devs[i]);
@@ -1901,7 +2279,7 @@ extern "C" int pmm_create_local(int32_t p, const int32_t* cuda_devices, const in
             for (int i = 0; i < p; ++i)
                 for (int j = 0; j < p; ++j) {
                     const int a = cuda_devices[i], c = cuda_devices[j];
-                    if (a == c) continue;
+                    if (a == c || a < 0 || c < 0) continue;
                     int can = 0;
                     cudaDeviceCanAccessPeer(&can, a, c);
                     if (can) {
@@ -2104,8 +2482,12 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value == 0 || value == 1, "ooc_keep must be 0 or 1");
             ctx->ooc_keep = (int)value;
         } else if (k == "kernel_variant") {
-            FPM_CHECK_ARG(value >= -1 && value <= 6, "kernel_variant must be -1 (auto) or 0..6 (5, 6: F16I8 only)");
+            FPM_CHECK_ARG(value >= -1 && value <= 8,
+                          "kernel_variant must be -1 (auto) or 0..8 (6: F16I8 only; 7, 8: F16X3 / TF32X3 only)");
             ctx->kernel_variant = (int)value;
+        } else if (k == "chunk_k") {
+            FPM_CHECK_ARG(value >= 0 && value <= (1 << 20), "chunk_k must be 0 (auto = 512) or a positive K");
+            ctx->chunk_k = (int)value;
         } else if (k == "l2_hint_b") {
             FPM_CHECK_ARG(value >= 0 && value <= 2, "l2_hint_b must be 0 (normal), 1 (first) or 2 (last)");
             ctx->l2_hint_b = (int)value;
@@ -2125,7 +2507,24 @@ extern "C" int pmm_set_device_option(pmm_ctx* ctx, int32_t dev, const char* key,
         FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
         fpm::drop_graph(ctx);
         const std::string k(key);
-        if (k == "c_cap_bytes") {
+        if (k == "cpu_first_core") {  // CPU device: move its team to cores [value, value + c) of the affinity mask
+            FPM_CHECK_ARG(d->cpu, "cpu_first_core applies to CPU devices only");
+            FPM_CHECK_ARG(value >= 0, "cpu_first_core must be >= 0");
+            if (d->first_core != (int)value) {
+                const int old = d->first_core;
+                fpm::cpu::team_destroy(d->team);
+                d->team = nullptr;
+                d->first_core = (int)value;
+                try {
+                    fpm::init_device(*d);
+                } catch (...) {
+                    d->first_core = old;
+                    fpm::init_device(*d);
+                    throw;
+                }
+            }
+        } else if (k == "c_cap_bytes") {
+            FPM_CHECK_ARG(!d->cpu, "c_cap_bytes applies to GPU devices");
             FPM_CHECK_ARG(value >= 0, "c_cap_bytes must be >= 0");
             if (d->c_cap != value) ctx->have_problem = false;  // C_i placement changes
             d->c_cap = value;
@@ -2203,6 +2602,11 @@ extern "C" int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t 
             if (!d.live()) continue;
             const int64_t R0 = d.rect.row0 * b, C0 = d.rect.col0 * b;
             if (r0 >= R0 && c0 >= C0 && r0 + rows <= R0 + d.H && c0 + cols <= C0 + d.W) {
+                const size_t off0 = ((size_t)(r0 - R0) * d.W + (size_t)(c0 - C0)) * es;
+                if (d.cpu) {
+                    fpm::copy_rows(C_host, ld * es, static_cast<const char*>(d.C) + off0, d.W * es, cols * es, rows);
+                    return;
+                }
                 CU(cudaSetDevice(d.cuda_dev));
                 CU(cudaStreamSynchronize(d.s_comp));
                 const size_t off = ((size_t)(r0 - R0) * d.W + (size_t)(c0 - C0)) * es;
@@ -2243,7 +2647,16 @@ extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int6
         const fpm::HostDst out{C, ld, row_base, col_base};
         pmm_stats local;
         std::vector<char> done;
-        fpm::compute(ctx, &local, &host, &out, &done);  // host panels streamed in, C streamed out
+        if (fpm::has_cpu(ctx)) {
+            // CPU devices pull pivots from resident rectangles: every device's
+            // inputs are in place before the k-loop (C still streamed out)
+            double tu = 0.0;
+            fpm::upload(ctx, A, B, ld, row_base, col_base, &tu);
+            fpm::compute(ctx, &local, nullptr, &out, &done);
+            local.t_upload_s = tu;
+        } else {
+            fpm::compute(ctx, &local, &host, &out, &done);  // host panels streamed in, C streamed out
+        }
         double td = 0.0;
         fpm::download(ctx, C, ld, row_base, col_base, &td, &done);  // devices without a tail
         local.t_download_s = std::max(local.t_download_s, td);
@@ -2299,8 +2712,9 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
     return guarded([&] {
         FPM_CHECK_ARG(scheme >= 0 && scheme <= 3, "scheme must be 0, 1, 2 (int8 timing probe) or 3");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
-        FPM_CHECK_ARG((variant >= -1 && variant <= 5) || (variant >= 6 && variant <= 11 && scheme == 3),
-                      "variant must be -1 (auto) or 0..4 (9: F16I8 timing probe)");
+        FPM_CHECK_ARG((variant >= -1 && variant <= 5) || ((variant == 7 || variant == 8) && scheme != 3) ||
+                          (variant >= 6 && variant <= 11 && variant != 7 && variant != 8 && scheme == 3),
+                      "variant must be -1 (auto), 0..5, 7, 8, or 6, 9..11 with F16I8");
         FPM_CHECK_ARG(scheme == 1 || scheme == 2 || (sa && sb), "F16X3 / F16I8 need sa and sb");
         fpm::UpdateArgs a;
         a.a_hi = a_hi; a.a_lo = a_lo; a.bt_hi = bt_hi; a.bt_lo = bt_lo;
