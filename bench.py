@@ -1,20 +1,25 @@
 #!/usr/bin/env python
 """Benchmark of the FPM-partitioned column-based parallel matrix multiplication.
 
-    python bench.py --gpus N --steps K --warmup W [--impl ours|reference]
+    python bench.py --gpus N --steps K --warmup W [--impl ours|reference] [--config c5|c3|c4]
 
-One process per GPU (torchrun for N > 1: RANK / WORLD_SIZE / LOCAL_RANK), the
-pivot exchange over NCCL inside libfpmpmm, torch.distributed (gloo) only for the
-control plane (unique id, barriers, max-over-ranks of device times).
+One process per GPU (torchrun for N > 1: RANK / WORLD_SIZE / LOCAL_RANK); the
+pivot exchange inside libfpmpmm -- one-sided pulls from the peers' memory over
+NVLink fused into the staging kernels (IPC, default) or NCCL send/recv +
+column broadcasts (--transport nccl); torch.distributed (gloo) only for the
+control plane (IPC handles, unique id, barriers, max-over-ranks of device times).
 
-Workload (BASELINE.json config 5): N = 49152, b = 1024, FP32,
-square U[-1,1) matrices from the shared counter-based generator, p = N GPUs,
-strong scaling.  A step = fpm_partition + colpart_arrange + pmm_compute (the
-N/b iterations of pivot exchange, staging and rank-b update) on inputs resident
-in HBM; `value` = 2 N^3 K / sum of per-step device times (max over ranks).
-`e2e` = the same through pmm_run on pinned host buffers (H2D + D2H inside).
-`--impl reference` times the CPU oracle (plain triple loop) on a bounded
-sample of the same workload (rank 0 only).
+Workload (BASELINE.json config 5, default): N = 49152, b = 1024,
+FP32, square U[-1,1) matrices from the shared counter-based generator, p = N
+GPUs, strong scaling.  --config c3: N = 16384, b = 512 homogeneous; --config c4:
+N = 32768, b = 512, rank i capped to {144, 128, 112, 96, 80, 64, 48, 32}[i] SMs
+in a green-context partition (one GPU: eight partitions of it), plus the CPM and
+homogeneous partitions.  A step = fpm_partition + colpart_arrange + pmm_compute
+(the N/b iterations of pivot exchange, staging and rank-b update) on inputs
+resident in HBM; `value` = 2 N^3 K / sum of per-step device times (max over
+ranks).  `e2e` = the same through the public API on pinned host buffers (H2D
+and D2H inside the timed region).  `--impl reference` times the CPU oracle
+(plain triple loop) on a bounded sample of the same workload (rank 0 only).
 """
 from __future__ import annotations
 
@@ -36,7 +41,6 @@ DTYPE = {"f16x3": "f32 (F16X3: 3 fp16 tcgen05 products per FP32 MAC, FP32 accumu
          "f16i8": "f32-emulated-f16i8 (fp16 + int8 products, row-max fixed point: NOT FP32-class)"}
 METRIC = "partitioned GEMM GFLOPS & % tensor peak at 1/2/4/8 B200; FPM load imbalance %"
 UNIT = "GFLOP/s"
-N_DEFAULT, B_DEFAULT = 49152, 1024
 ORACLE_ROWS, ORACLE_COLS = 2048, 1024   # bounded sample for the CPU oracle (~206 GFLOP at c5, ~5 s on 16 cores)
 
 
@@ -115,7 +119,7 @@ def committed_traffic(N: int, b: int, args):
     """DRAM bytes per update launch from the committed ncu capture of the same
     configuration (profiles/ncu_traffic.json), else None."""
     path = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    variant = (6 if args.scheme == "f16i8" else 7) if args.kernel_variant < 0 else args.kernel_variant
+    variant = (6 if args.scheme == "f16i8" else 8) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
     G = args.raster_group if args.raster_group > 0 else (12 if args.scheme == "f16i8" else 16)
     key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}") + ("" if G == 16 else f"_r{G}")
@@ -126,14 +130,14 @@ def committed_traffic(N: int, b: int, args):
 
 
 # ----------------------------------------------------------------- oracle
-def oracle_sample(N: int, reps: int = 1, want_c: bool = False):
+def oracle_sample(N: int, reps: int = 1, want_c: bool = False, seed_cfg: int = 4):
     """Time the CPU oracle (plain triple loop, FP64 accumulation) on the block
     C[0:R, 0:S] = A[0:R, :] B[:, 0:S] of the workload; returns (GFLOP/s, cores,
     desc, seconds[, C block])."""
     import synth
     from oracle import gemm as og
     R, S = min(ORACLE_ROWS, N), min(ORACLE_COLS, N)
-    sa, sb = synth.seeds_for_config(4)
+    sa, sb = synth.seeds_for_config(seed_cfg)
     A = synth.rect(sa, N, 0, 0, R, N)
     B = synth.rect(sb, N, 0, 0, N, S)
     og.gemm(A[:2, :64], B[:64, :8])  # build / load outside the timing
@@ -151,7 +155,7 @@ def oracle_sample(N: int, reps: int = 1, want_c: bool = False):
     return flops / t / 1e9, og.num_threads(), desc, t
 
 
-def e2e_parity(N: int, hC, oracle_block) -> dict:
+def e2e_parity(N: int, hC, oracle_block, seeds) -> dict:
     """Parity of the timed e2e output (pmm_run, default options) against the
     oracle on sampled blocks (exact oracle on a sample of C):
     the top-left block the CPU baseline computes anyway, plus the bottom-right
@@ -160,7 +164,7 @@ def e2e_parity(N: int, hC, oracle_block) -> dict:
 
     import synth
     from oracle import gemm as og
-    sa, sb = synth.seeds_for_config(4)
+    sa, sb = seeds
     C = hC.numpy() if hasattr(hC, "numpy") else np.asarray(hC)
     R, S = oracle_block.shape
     blocks = [("top-left", 0, 0, R, S, oracle_block)]
@@ -185,10 +189,11 @@ def run_reference(args, rank: int):
     # rank 0 alone runs: give the oracle every host core (torchrun exports OMP_NUM_THREADS=1)
     from oracle import gemm as og
     og.set_num_threads(len(os.sched_getaffinity(0)))
-    N = args.N
+    cfg = CONFIGS[args.config]
+    N, b = args.N or cfg["N"], args.b or cfg["b"]
     vals, times = [], []
     for i in range(args.warmup + args.steps):
-        g, cores, desc, t = oracle_sample(N)
+        g, cores, desc, t = oracle_sample(N, seed_cfg=cfg["seed_cfg"])
         if i >= args.warmup:
             vals.append(g)
             times.append(t)
@@ -198,36 +203,103 @@ def run_reference(args, rank: int):
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": 1e3 * statistics.median(times),
         "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
         "data": "synthetic",
-        "config": {"workload": f"c5: N={N}, b={args.b}, FP32 inputs (oracle accumulates in FP64)",
-                   "N": N, "b": args.b, "sample": desc},
+        "config": {"workload": f"{args.config}: N={N}, b={b}, FP32 inputs (oracle accumulates in FP64)",
+                   "N": N, "b": b, "sample": desc},
         "cpu_baseline": {"value": value, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc},
         "e2e": {"value": value, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
 
 
+# BASELINE.json configs bench.py can run; seeds = synth.seeds_for_config(index)
+CONFIGS = {
+    "c3": {"N": 16384, "b": 512, "caps": None, "seed_cfg": 2,
+           "desc": "c3: N=16384, b=512, FP32, p={p} homogeneous B200, FPM partition + column arrangement"},
+    "c4": {"N": 32768, "b": 512, "caps": [144, 128, 112, 96, 80, 64, 48, 32], "seed_cfg": 3,
+           "desc": "c4: N=32768, b=512, FP32, p={p} B200 with SM caps {caps} (green-context partitions), "
+                   "FPM vs constant-model vs homogeneous partition"},
+    "c5": {"N": 49152, "b": 1024, "caps": None, "seed_cfg": 4,
+           "desc": "c5: N=49152, b=1024, FP32, p={p} homogeneous B200, FPM partition + column arrangement"},
+}
+# c4 on ONE GPU: the eight caps scaled to fit its 148 SMs (studies/hetero.py)
+C4_ONE_GPU_CAPS = [30, 26, 24, 20, 16, 14, 10, 6]
+
+
+def imbalance(ts) -> float:
+    """max / mean - 1 over devices with work (reading Q18)."""
+    live = [t for t in ts if t > 0]
+    return max(live) / (sum(live) / len(live)) - 1.0 if live else 0.0
+
+
+def build_line(*, world, steps, warmup, step_times, workload, cfg, scheme, roofline, per_dev, e2e, cpu, parity,
+               launches, clocks, extra_config=None) -> dict:
+    """The bench JSON line from per-step device times (max over ranks) and
+    per-device records (pure: tested without a GPU, tests/test_bench_contract.py).
+    per_dev: one dict per device of the arrangement with keys rank, device, rect,
+    compute_s, update_s, predicted_s."""
+    total_t = sum(step_times)
+    N = cfg["N"]
+    value = 2.0 * N ** 3 * steps / total_t / 1e9
+    meas = [d["compute_s"] for d in per_dev if d["rect"][3] * d["rect"][4] > 0]
+    pred = [d["predicted_s"] for d in per_dev if d["rect"][3] * d["rect"][4] > 0]
+    peak = roofline["peak"]
+    config = {
+        "workload": workload, "N": N, "b": cfg["b"], "p": len(per_dev),
+        "partition": [d["area"] for d in per_dev], "rects": [d["rect"] for d in per_dev],
+        "f32_scheme": scheme,
+        "l2": (f"inputs larger than L2 (A, B, C {N * N * 4 / 1e9:.2f} GB each)" if N * N * 4 > 126e6
+               else "inputs fit in L2 (no flush between steps)"),
+        "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
+        "imbalance_pct_measured": 100.0 * imbalance(meas),
+        "imbalance_pct_predicted": 100.0 * imbalance(pred),
+        "per_device": per_dev,
+    }
+    config.update(extra_config or {})
+    return {
+        "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": steps, "warmup": warmup,
+        "ms_per_step": 1e3 * total_t / steps, "higher_is_better": True, "scaling": "strong",
+        "vs_baseline": None, "dtype": DTYPE[scheme], "data": "synthetic", "config": config,
+        "roofline": roofline, "cpu_baseline": cpu, "parity": parity, "e2e": e2e, "gpu_launches": launches,
+        "clocks": clocks,
+    }
+
+
 def run_ours(args, rank: int, world: int, local_rank: int, dist):
-    import numpy as np
     import torch
 
     import paper_conf_cluster_zhongrl12_b200 as pkg
+    import synth
 
     torch.cuda.set_device(local_rank)
-    N, b = args.N, args.b
+    cfg = dict(CONFIGS[args.config])
+    if args.N:
+        cfg["N"] = args.N
+    if args.b:
+        cfg["b"] = args.b
+    N, b = cfg["N"], cfg["b"]
     n = N // b
-    p = world
+    T = n * n
+    # devices of the arrangement: one per rank; c4 on one GPU emulates eight in
+    # disjoint green-context SM partitions of it
+    if world == 1 and cfg["caps"]:
+        caps = list(C4_ONE_GPU_CAPS)
+    elif cfg["caps"]:
+        caps = [cfg["caps"][r % len(cfg["caps"])] for r in range(world)]
+    else:
+        caps = None
+    p = world if world > 1 else (len(caps) if caps else 1)
+    mine = [rank] if world > 1 else list(range(p))   # devices this process drives
 
-    # ---- context: N > 1 -> one process per GPU, pivots pulled from the peers'
-    # memory over NVLink (ipc, default) or exchanged with NCCL (nccl)
     def make_ctx(transport: str):
-        if world > 1 and transport == "nccl":
+        if transport.startswith("nccl") and not (world == 1 and caps):
             obj = [pkg.Context.nccl_unique_id() if rank == 0 else None]
-            dist.broadcast_object_list(obj, src=0)
-            c = pkg.Context.nccl(rank, world, local_rank, obj[0])
+            if world > 1:
+                dist.broadcast_object_list(obj, src=0)
+            c = pkg.Context.nccl(rank, world, local_rank, obj[0], sm_cap=caps[rank] if caps else 0)
         elif world > 1:
-            c = pkg.Context.ipc(rank, world, local_rank)
+            c = pkg.Context.ipc(rank, world, local_rank, sm_cap=caps[rank] if caps else 0)
         else:
-            c = pkg.Context.local([local_rank])
+            c = pkg.Context.local([local_rank] * p, sm_caps=caps)
         c.set_option("f32_scheme", {"f16i8": pkg.SCHEME_F16I8, "f16x3": pkg.SCHEME_F16X3,
                                     "tf32x3": pkg.SCHEME_TF32X3}[args.scheme])
         c.set_option("cta_group", args.cta_group)
@@ -238,59 +310,32 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
         c.set_option("e2e_tail", args.e2e_tail)
+        if caps:
+            c.set_option("sm_partition", 1)   # every kernel of a device inside its SM partition
         return c
 
-    transport = args.transport if world > 1 else "none (p = 1)"
+    transport = args.transport if (world > 1 or args.transport == "nccl") else "none (one process)"
     ctx = make_ctx(transport)
 
-    # ---- FPMs (offline): sample this GPU's speed function once;
-    # every rank's model is gathered so all ranks partition identically.
-    sizes = [m * m for m in (1, 2, 4, 8, 12, 16)]
+    # ---- FPMs (offline): each device's speed function sampled once,
+    # gathered so every rank partitions identically
+    sizes = [m * m for m in ((1, 2, 4, 8, 12, 16, 20, 24, 28, 32) if caps else (1, 2, 4, 8, 12, 16))]
     t0 = time.perf_counter()
     if args.no_sample:  # profiling runs: identical constant models, predictable launch order
-        sp = [1.0] * len(sizes)
+        mine_models = [(sizes, [1.0] * len(sizes)) for _ in mine]
     else:
-        sp, ci, reps = ctx.sample(rank, b, sizes, pkg.FPM_F32)
+        mine_models = [(sizes, ctx.sample(dev, b, sizes, pkg.FPM_F32)[0]) for dev in mine]
     t_sample = time.perf_counter() - t0
-    models_all = [None] * world
     if world > 1:
-        dist.all_gather_object(models_all, (sizes, sp))
+        models = [None] * world
+        dist.all_gather_object(models, mine_models[0])
     else:
-        models_all = [(sizes, sp)]
-
-    def plan():
-        d = pkg.fpm_partition(n * n, models_all)
-        return d, pkg.colpart_arrange(n, d)
+        models = mine_models
 
     def barrier():
         torch.cuda.synchronize()
         if world > 1:
             dist.barrier()
-
-    d, rects = plan()
-    ctx.setup(N, b, rects, pkg.FPM_F32)
-    if transport == "ipc":
-        ok = 1
-        blobs = [None] * world
-        dist.all_gather_object(blobs, ctx.ipc_export())
-        try:
-            ctx.ipc_import(blobs)
-        except pkg.FpmError as ex:  # e.g. no peer access between these GPUs
-            log(f"rank {rank}: IPC import failed ({ex}); falling back to NCCL")
-            ok = 0
-        flag = torch.tensor([ok], dtype=torch.int32)
-        dist.all_reduce(flag, op=dist.ReduceOp.MIN)
-        if int(flag.item()) == 0:
-            dist.barrier()
-            ctx.close()
-            transport = "nccl (ipc unavailable)"
-            ctx = make_ctx("nccl")
-            ctx.setup(N, b, rects, pkg.FPM_F32)
-    ipc = transport == "ipc"
-    import synth
-    sa, sb = synth.seeds_for_config(4)   # config 5 (index 4): seeds 5 and 6
-    ctx.fill_synthetic(sa, sb, pkg.FPM_DIST_PM1)
-    barrier()                            # every rank's inputs resident before any pull
 
     def max_over_ranks(x: float) -> float:
         if world == 1:
@@ -299,125 +344,191 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         dist.all_reduce(t, op=dist.ReduceOp.MAX)
         return float(t.item())
 
-    # ---- device-resident steps
+    seeds = synth.seeds_for_config(cfg["seed_cfg"])
+
+    def install(rects):
+        """Set up the arrangement on every rank (IPC: exchange the mappings), fill
+        the synthetic inputs, and barrier so every rank's inputs are resident."""
+        nonlocal ctx, transport
+        ctx.setup(N, b, rects, pkg.FPM_F32)
+        if transport == "ipc":
+            ok = 1
+            blobs = [None] * world
+            dist.all_gather_object(blobs, ctx.ipc_export())
+            try:
+                ctx.ipc_import(blobs)
+            except pkg.FpmError as ex:  # e.g. no peer access between these GPUs
+                log(f"rank {rank}: IPC import failed ({ex}); falling back to NCCL")
+                ok = 0
+            flag = torch.tensor([ok], dtype=torch.int32)
+            dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+            if int(flag.item()) == 0:
+                dist.barrier()
+                ctx.close()
+                transport = "nccl (ipc unavailable)"
+                ctx = make_ctx("nccl")
+                ctx.setup(N, b, rects, pkg.FPM_F32)
+        ctx.fill_synthetic(seeds[0], seeds[1], pkg.FPM_DIST_PM1)
+        barrier()
+
+    def plan(part_models):
+        d = pkg.fpm_partition(T, part_models)
+        return d, pkg.colpart_arrange(n, d)
+
+    def per_device(comp, upd, rects, part_models):
+        """Per-device records (Fig. 6 metric): this process's devices (comp /
+        upd indexed by device, as pmm_stats), gathered over the ranks."""
+        recs = []
+        for dev in mine:
+            r = rects[dev]
+            a = r[3] * r[4]
+            recs.append({"rank": rank, "device": dev, "rect": list(r), "area": a,
+                         "sm_cap": caps[dev] if caps else None,
+                         "compute_s": comp[dev], "update_s": upd[dev],
+                         "predicted_s": (2.0 * a * b * b * N / pkg.fpm_model_speed(part_models[dev], a)
+                                         if a > 0 else 0.0)})
+        if world > 1:
+            allr = [None] * world
+            dist.all_gather_object(allr, recs)
+            recs = [x for rr in allr for x in rr]
+        return recs
+
+    d, rects = plan(models)
+    install(rects)
+
+    # ---- device-resident steps: fpm_partition + colpart_arrange + the k-loop
     for _ in range(args.warmup):
-        d, rects = plan()
+        d, rects = plan(models)
         ctx.compute(zero_c=True)
     barrier()
     clocks = ClockSampler(local_rank)
     clocks.start()
-    step_times, upd_times, comp_times, own_times, launches, comm = [], [], [], [], 0, 0
+    step_times, recs_steps, own_times, launches, comm = [], [], [], 0, 0
     wall0 = time.perf_counter()
     for _ in range(args.steps):
-        d, rects = plan()
+        d, rects = plan(models)
         st = ctx.compute(zero_c=True)
         own_times.append(st.t_compute_s)
         step_times.append(max_over_ranks(st.t_compute_s))
-        upd_times.append(st.per_dev_update_s[rank])
-        comp_times.append(st.per_dev_compute_s[rank])
+        recs_steps.append([(st.per_dev_compute_s[i], st.per_dev_update_s[i]) for i in range(16)])
         launches += st.kernel_launches
         comm += st.comm_bytes
     barrier()
     wall = time.perf_counter() - wall0
     clk = clocks.stop()
-    total_t = sum(step_times)
-    flops = 2.0 * N ** 3
-    value = flops * args.steps / total_t / 1e9
-
-    # per-rank computation time (Fig. 6 metric) -> measured imbalance
-    comp_all = [statistics.median(comp_times)]
-    if world > 1:
-        comp_all = [None] * world
-        dist.all_gather_object(comp_all, statistics.median(comp_times))
-    live = [c for c, r in zip(comp_all, rects) if r[3] * r[4] > 0]
-    imb_meas = max(live) / (sum(live) / len(live)) - 1.0 if live else 0.0
-    areas = [r[3] * r[4] for r in rects]
-    pred_t = [a / pkg.fpm_model_speed(m, a) if a > 0 else 0.0 for a, m in zip(areas, models_all)]
-    live_t = [t for t in pred_t if t > 0]
-    imb_pred = max(live_t) / (sum(live_t) / len(live_t)) - 1.0 if live_t else 0.0
-
-    stage = statistics.median(comp_times) - statistics.median(upd_times)
-    exposed = max(0.0, statistics.median(own_times) - statistics.median(upd_times))
+    # the median step's per-device record
+    med = sorted(range(args.steps), key=lambda i: own_times[i])[args.steps // 2]
+    per_dev = per_device([x[0] for x in recs_steps[med]], [x[1] for x in recs_steps[med]], rects, models)
+    mine_recs = [x for x in per_dev if x["rank"] == rank]
+    upd_med = max(x["update_s"] for x in mine_recs)
+    comp_med = max(x["compute_s"] for x in mine_recs)
+    stage = comp_med - upd_med
+    exposed = max(0.0, own_times[med] - upd_med)
     overlap = 1.0 - exposed / stage if stage > 0 else None
+    overlaps = [overlap]
+    if world > 1:
+        overlaps = [None] * world
+        dist.all_gather_object(overlaps, overlap)
 
-    # ---- roofline of the dominant kernel (rank-(f b) update): algorithmic flops per
-    # launch = 2 H W f b, over the launch duration (CUDA events on its stream);
-    # per step: 2 H W b n flop over the summed update time.
+    # ---- roofline of the dominant kernel (rank-(f b) update): algorithmic flops
+    # 2 H W b n of the busiest device over its summed update time (CUDA events on its stream)
     peaks = measured_peaks()
-    r = rects[rank]
-    H, W = r[3] * b, r[4] * b
-    upd_launches = st.updates
-    upd_step = statistics.median(upd_times)
-    achieved = 2.0 * H * W * b * n / upd_step / 1e12 if upd_step > 0 else 0.0
-    # tensor-pipe time per FP32 MAC in units of one dense fp16 MAC: F16X3 three
-    # fp16 products; TF32X3 three tf32 products at half the fp16 rate; F16I8 one
-    # fp16 product plus one int8 product over twice the K at twice the fp16 rate
-    # (the guide's nominal int8 : fp16 = 2 : 1) = 2
+    busiest = max(mine_recs, key=lambda x: x["update_s"])
+    rb = busiest["rect"]
+    H, W = rb[3] * b, rb[4] * b
+    achieved = 2.0 * H * W * b * n / busiest["update_s"] / 1e12 if busiest["update_s"] > 0 else 0.0
     dense_peak = peaks["bf16_sustained"] if args.scheme != "tf32x3" else peaks["bf16_sustained"] / 2.0
     mma_per_mac = 2.0 if args.scheme == "f16i8" else 3.0
     peak = dense_peak / mma_per_mac
+    if caps:  # one device's share of the GPU
+        peak *= caps[busiest["device"]] / torch.cuda.get_device_properties(local_rank).multi_processor_count
     basis = {"f16i8": "fp16 dense tensor peak ({src} {p:.1f} TFLOP/s sustained) / 2 (one fp16 product + one "
                       "int8 product of 2K at 2x the fp16 rate per FP32 MAC)",
              "f16x3": "fp16 dense tensor peak ({src} {p:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC",
              "tf32x3": "tf32 dense tensor peak ({src} {p:.1f} TFLOP/s sustained) / 3 MMAs per FP32 MAC"}[args.scheme]
+    if caps:
+        basis += " x the device's SM share"
     roofline = {"bound": "tensor", "achieved": achieved, "peak": peak, "unit": "TFLOP/s",
                 "frac": achieved / peak if peak else None,
-                "traffic": args.traffic if args.traffic is not None else committed_traffic(N, b, args),
+                "traffic": (args.traffic if args.traffic is not None else
+                            (committed_traffic(N, b, args) if not caps else None)),
                 "peak_basis": basis.format(src=peaks["source"], p=dense_peak),
-                "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None}
+                "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None,
+                "kernel": "rank-(f b) update (update_acc_kernel: F16X3 chunked accumulation)"
+                if args.scheme == "f16x3" else "rank-(f b) update",
+                "device": busiest["device"]}
+
+    # ---- c4: the same multiply under the constant-model and homogeneous partitions (P:87, P:143)
+    partitions = None
+    if caps and not args.no_partitions:
+        x_cal = max(1, (8192 // b) ** 2 // p)   # CPM constants at the even share of N_cal = 8192 (Q9)
+        alt = {"cpm_ncal": [([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models],
+               "homogeneous": [([1], [1.0])] * p}
+        partitions = {"fpm": {"t_s": statistics.median(step_times), "d": list(d),
+                              "imbalance_pct_measured": 100.0 * imbalance([x["compute_s"] for x in per_dev]),
+                              "imbalance_pct_predicted": 100.0 * imbalance([x["predicted_s"] for x in per_dev])}}
+        for name, pm in alt.items():
+            dd, rr = plan(pm)
+            install(rr)
+            ctx.compute()
+            best, t_best = None, None
+            for _ in range(2):
+                s2 = ctx.compute()
+                t2 = max_over_ranks(s2.t_compute_s)
+                if t_best is None or t2 < t_best:
+                    best, t_best = s2, t2
+            recs = per_device(list(best.per_dev_compute_s), list(best.per_dev_update_s), rr, models)
+            partitions[name] = {"t_s": t_best, "d": list(dd),
+                                "imbalance_pct_measured": 100.0 * imbalance([x["compute_s"] for x in recs]),
+                                "imbalance_pct_predicted": 100.0 * imbalance([x["predicted_s"] for x in recs])}
+        for v in partitions.values():
+            v["gflops"] = 2.0 * N ** 3 / v["t_s"] / 1e9
+        partitions["fpm_vs_cpm_time_delta_pct"] = 100.0 * (partitions["fpm"]["t_s"] / partitions["cpm_ncal"]["t_s"] - 1)
+        partitions["fpm_vs_homogeneous_time_delta_pct"] = 100.0 * (
+            partitions["fpm"]["t_s"] / partitions["homogeneous"]["t_s"] - 1)
+        install(rects)   # back to the FPM arrangement for e2e
 
     # ---- end to end through pmm_run with pinned host buffers
     e2e, hC = None, None
     if args.e2e_steps > 0:
         try:
-            e2e, hC = run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc)
+            e2e, hC = run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, transport == "ipc", N, b,
+                              seeds)
         except Exception as ex:  # report, do not hide
             log("e2e failed:", repr(ex))
             e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:200]}
 
     cpu, parity = None, None  # the oracle baseline is timed at N = 1 only (rank 0); N > 1 lines carry null
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
-        g, cores, desc, _, c_block = oracle_sample(N, want_c=True)
+        g, cores, desc, _, c_block = oracle_sample(N, want_c=True, seed_cfg=cfg["seed_cfg"])
         cpu = {"value": g, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc}
         if hC is not None:
-            parity = e2e_parity(N, hC, c_block)
+            parity = e2e_parity(N, hC, c_block, seeds)
             if not parity["ok"]:
                 log("PARITY FAILURE of the e2e output:", json.dumps(parity))
 
+    line = None
     if rank == 0:
-        line = {
-            "metric": METRIC, "value": value, "unit": UNIT, "n_gpus": world, "steps": args.steps,
-            "warmup": args.warmup, "ms_per_step": 1e3 * total_t / args.steps, "higher_is_better": True,
-            "scaling": "strong", "vs_baseline": None, "dtype": DTYPE[args.scheme], "data": "synthetic",
-            "config": {
-                "workload": f"c5: N={N}, b={b}, FP32, p={p} homogeneous B200, FPM partition + column arrangement",
-                "N": N, "b": b, "p": p, "partition": d, "rects": rects,
-                "f32_scheme": args.scheme, "cta_group": args.cta_group, "raster_group": args.raster_group,
+        line = build_line(
+            world=world, steps=args.steps, warmup=args.warmup, step_times=step_times,
+            workload=cfg["desc"].format(p=p, caps=caps), cfg=cfg, scheme=args.scheme, roofline=roofline,
+            per_dev=per_dev, e2e=e2e, cpu=cpu, parity=parity, launches=launches, clocks=clk,
+            extra_config={
+                "config": args.config, "cta_group": args.cta_group, "raster_group": args.raster_group,
                 "kernel_variant": args.kernel_variant, "chunk_k": args.chunk_k, "fuse": args.fuse,
-                "update_launches_per_step": upd_launches,
-                "transport": transport,
-                "l2": (f"inputs larger than L2 (A, B, C {N * N * 4 / 1e9:.2f} GB each)" if N * N * 4 > 126e6
-                       else "inputs fit in L2 (no flush between steps)"),
-                "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
-                "imbalance_pct_measured": 100.0 * imb_meas, "imbalance_pct_predicted": 100.0 * imb_pred,
+                "update_launches_per_step": st.updates, "transport": transport,
                 "fpm_sample_s": t_sample, "fpm_sizes": sizes,
                 "comm_bytes_per_step": comm // max(1, args.steps),
-                # share of the exchange + staging time hidden under the updates (SURVEY §8(d) c5
-                # "broadcast/update overlap", from the CUDA events of this rank's streams)
-                "exchange_staging_overlap": overlap,
+                # share of the exchange + staging time hidden under the updates, per rank (CUDA
+                # events of each rank's streams; SURVEY §8(d) c5 "broadcast/update overlap")
+                "exchange_staging_overlap": overlaps[0] if world == 1 else overlaps,
                 "wall_s_timed_region": wall,
-            },
-            "roofline": roofline,
-            "cpu_baseline": cpu,
-            "parity": parity,
-            "e2e": e2e,
-            "gpu_launches": launches,
-            "clocks": clk,
-        }
+                "partitions": partitions,
+            })
     barrier()  # no rank frees buffers a peer may still read (IPC)
     ctx.close()
     if rank == 0:
-        if world == 1 and not args.no_hetero:
+        if world == 1 and not caps and not args.no_hetero:
             try:
                 line["hetero"] = run_hetero(peak)
             except Exception as ex:  # report, do not hide
@@ -456,24 +567,31 @@ def run_hetero(peak_tflops: float) -> dict:
     return out
 
 
-def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc):
+def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, seeds):
+    """e2e through the public API with pinned host buffers: pmm_run (one process:
+    host panels streamed in, C streamed out) or, under IPC, pmm_upload + barrier +
+    pmm_compute_into (C copied out under the last updates); median of
+    args.e2e_steps calls after one warm-up call, max over ranks.  Returns the
+    record and, in one process, the host C (all of it) for the parity check."""
     import torch
 
     import paper_conf_cluster_zhongrl12_b200 as pkg
-    N, b = args.N, args.b
-    r = rects[rank]
-    H, W = r[3] * b, r[4] * b
-    R0, C0 = r[1] * b, r[2] * b
+    # host windows: this rank's rectangle (IPC / NCCL) or all of A, B, C (one process)
+    if world > 1:
+        r = rects[rank]
+        H, W, R0, C0 = r[3] * b, r[4] * b, r[1] * b, r[2] * b
+    else:
+        H = W = N
+        R0 = C0 = 0
     live = H * W > 0
-    # host windows = this rank's rectangle (generated on the device once, untimed)
-    if live:
+    if live:   # generated on the device by the shared generator once, untimed
         hA = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
         hB = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
         hC = torch.empty((H, W), dtype=torch.float32, pin_memory=True)
         tmp = torch.empty((H, W), dtype=torch.float32, device="cuda")
-        pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 5, N, R0, C0, H, W)  # seeds_for_config(4)
+        pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, seeds[0], N, R0, C0, H, W)
         hA.copy_(tmp)
-        pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, 6, N, R0, C0, H, W)
+        pkg.k_fill_synthetic(tmp, pkg.FPM_F32, W, seeds[1], N, R0, C0, H, W)
         hB.copy_(tmp)
         del tmp
         torch.cuda.empty_cache()
@@ -487,7 +605,6 @@ def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc):
             if live:
                 ctx.upload(hA, hB, W, R0, C0)
             barrier()
-            # k-loop with C_i copied out band by band under the last updates
             st = ctx.compute_into(hC, W, R0, C0) if live else ctx.compute()
         elif live:
             # blocking call: H2D streamed under the updates, k-loop, D2H of C
@@ -497,12 +614,18 @@ def run_e2e(args, ctx, rects, rank, local_rank, max_over_ranks, barrier, ipc):
         if i > 0:  # first call is a warm-up
             ts.append(t_all)
     t = statistics.median(ts)
-    return ({"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
-            "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
-            "device_kloop_s": st.t_compute_s if st else None, "download_s": st.t_download_s if st else None,
-            "timing": ("host wall clock: upload + barrier + pmm_compute_into (IPC), max over ranks"
-                       if ipc else "host wall clock around the blocking pmm_run call, max over ranks")},
-            hC if (live and len(rects) == 1) else None)   # N = 1: hC is all of C
+    rec = {"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
+           "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
+           "device_kloop_s": st.t_compute_s if st else None, "download_s": st.t_download_s if st else None,
+           "timing": ("host wall clock: upload + barrier + pmm_compute_into (IPC), max over ranks"
+                      if ipc else "host wall clock around the blocking pmm_run call, max over ranks")}
+    if world > 1:
+        rec["h2d_bytes_per_step_rank0"] = rec["h2d_bytes_per_step"]
+        tot = torch.tensor([2 * H * W * 4, H * W * 4], dtype=torch.float64)
+        import torch.distributed as dist
+        dist.all_reduce(tot)
+        rec["h2d_bytes_per_step"], rec["d2h_bytes_per_step"] = int(tot[0].item()), int(tot[1].item())
+    return rec, (hC if (live and world == 1) else None)
 
 
 def main():
@@ -511,8 +634,12 @@ def main():
     ap.add_argument("--steps", type=int, default=5)
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", choices=["ours", "reference"], default="ours")
-    ap.add_argument("--N", type=int, default=N_DEFAULT)
-    ap.add_argument("--b", type=int, default=B_DEFAULT)
+    ap.add_argument("--config", choices=sorted(CONFIGS), default="c5",
+                    help="BASELINE config: c5 (default; N=49152, b=1024), c3 (N=16384, b=512), c4 (N=32768, "
+                         "b=512, SM caps {144..32} per rank; one GPU: 8 green partitions)")
+    ap.add_argument("--N", type=int, default=0, help="override the config's N")
+    ap.add_argument("--b", type=int, default=0, help="override the config's b")
+    ap.add_argument("--no-partitions", action="store_true", help="c4: skip the CPM / homogeneous runs")
     ap.add_argument("--scheme", choices=["f16i8", "f16x3", "tf32x3"], default="f16x3",
                     help="FP32 arithmetic: f16x3 (default, FP32-class), tf32x3, or f16i8 (opt-in, "
                          "fixed point relative to the row maximum: not FP32-class, DESIGN Q15b)")
@@ -536,7 +663,7 @@ def main():
     ap.add_argument("--traffic", type=float, default=None,
                     help="dram bytes per update launch from an ncu --set full capture")
     args = ap.parse_args()
-    if args.N % args.b:
+    if (args.N or CONFIGS[args.config]["N"]) % (args.b or CONFIGS[args.config]["b"]):
         ap.error("b must divide N")
 
     world = int(os.environ.get("WORLD_SIZE", "1"))
@@ -548,6 +675,9 @@ def main():
     if world > 1:
         import torch.distributed as dist
         os.environ.setdefault("MASTER_ADDR", "127.0.0.1")
+        if args.transport == "nccl":   # communicator set-up in the log (ranks per communicator)
+            os.environ.setdefault("NCCL_DEBUG", "INFO")
+            os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
         dist.init_process_group("gloo", rank=rank, world_size=world)
     if args.impl == "reference":
         run_reference(args, rank)

@@ -306,9 +306,9 @@ int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t
  *                 normwise, not elementwise; Q15b); needs cta_group
  *                 2, b % 64 == 0 and K <= 131072 per update.
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
- *   "kernel_variant": -1 (auto, default: F16X3 / TF32X3 7, F16I8 6; in NCCL
- *                 contexts, whose kernels need shared memory beside the
- *                 update, 8 and 5) or 0..8, see fpm_k_update_f32.
+ *   "kernel_variant": -1 (auto, default: F16X3 / TF32X3 8, F16I8 6 -- 5 in
+ *                 NCCL contexts, whose kernels need shared memory beside the
+ *                 update) or 0..8, see fpm_k_update_f32.
  *   "chunk_k":    variants 7 / 8: K summed per TMEM accumulation before the
  *                 epilogue adds it to its FP32 register sum (0 = auto = 512;
  *                 DESIGN.md Q15c: the tensor cores' accumulation error grows
@@ -439,7 +439,7 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * chunked accumulation: every 512 of K is a fresh TMEM accumulation drained
  * into per-thread FP32 register sums (round-to-nearest), C written once per
  * tile by TMA reduce-add (store when accumulate = 0), 3 x 64-KB operand
- * stages; 8 = the same with 2 stages.  -1 = auto (7).
+ * stages; 8 = the same with 2 stages (160 KB).  -1 = auto (8).
  * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
  * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks,
  * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 5 = variant

@@ -279,12 +279,6 @@ def _largest_remainder(numerators: Sequence[int], denominator: int, total: int) 
     return out
 
 
-def arrangement_cost(n: int, rects) -> int:
-    """Total half-perimeter sum_i (h_i + w_i) of the non-empty rectangles (in
-    blocks): the per-iteration communication volume that P:15 minimises."""
-    return sum(h + w for (_, _, _, h, w) in rects if h > 0 and w > 0)
-
-
 # --------------------------------------------------------------------------- O6
 def plan_step(rects, n: int, k: int):
     """Who sends what at iteration k ("At each iteration of the main loop,

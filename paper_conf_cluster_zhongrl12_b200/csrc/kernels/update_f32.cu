@@ -1217,10 +1217,13 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
         else launch_update_t<2, 2, 256, 2, 128, 4>(a, st);
         return;
     }
-    // auto: variant 7 (chunked accumulation, three 64-KB operand stages, C by TMA
-    // reduce-add): the FP32-class error bound at every K (Q15c).  Variants 0..5
-    // accumulate a whole update in one TMEM sum (error grows with K).
-    const int variant = a.variant >= 0 ? a.variant : 7;
+    // auto: variant 8 (chunked accumulation, two 64-KB operand stages, C by TMA
+    // reduce-add): the FP32-class error bound at every K (Q15c).  Measured c5:
+    // 430 TFLOP/s (variant 7, three stages: 421 -- it ran at a lower clock under
+    // the power cap; non-chunked variant 4: 430), and 160 KB of shared memory
+    // leave room for NCCL / staging kernels to co-run.  Variants 0..5 accumulate
+    // a whole update in one TMEM sum (error grows with K).
+    const int variant = a.variant >= 0 ? a.variant : 8;
     if (a.cta_group == 2) {
         switch (variant) {
             case 7:  // chunked accumulation, 3 stages + 2 C staging chunks (224 KB)

@@ -30,6 +30,9 @@ const NcclApi& nccl() {
     }
         FPM_NCCL_SYM(GetUniqueId, "ncclGetUniqueId")
         FPM_NCCL_SYM(CommInitRank, "ncclCommInitRank")
+        FPM_NCCL_SYM(CommInitRankConfig, "ncclCommInitRankConfig")
+        FPM_NCCL_SYM(CommCount, "ncclCommCount")
+        FPM_NCCL_SYM(CommAbort, "ncclCommAbort")
         FPM_NCCL_SYM(CommSplit, "ncclCommSplit")
         FPM_NCCL_SYM(CommDestroy, "ncclCommDestroy")
         FPM_NCCL_SYM(CommGetAsyncError, "ncclCommGetAsyncError")

@@ -10,6 +10,9 @@ namespace fpm {
 struct NcclApi {
     ncclResult_t (*GetUniqueId)(ncclUniqueId*);
     ncclResult_t (*CommInitRank)(ncclComm_t*, int, ncclUniqueId, int);
+    ncclResult_t (*CommInitRankConfig)(ncclComm_t*, int, ncclUniqueId, int, ncclConfig_t*);
+    ncclResult_t (*CommCount)(const ncclComm_t, int*);
+    ncclResult_t (*CommAbort)(ncclComm_t);
     ncclResult_t (*CommSplit)(ncclComm_t, int, int, ncclComm_t*, ncclConfig_t*);
     ncclResult_t (*CommDestroy)(ncclComm_t);
     ncclResult_t (*CommGetAsyncError)(ncclComm_t, ncclResult_t*);

@@ -588,6 +588,40 @@ bool has_cpu(const pmm_ctx* ctx) {
     return false;
 }
 
+// NCCL communicator configuration: the exchange runs beside the persistent
+// update kernel, which holds every SM, so NCCL gets few CTAs (maxCTAs, env
+// FPM_NCCL_MAX_CTAS, default 8) -- its transfers are NVLink-bound, not SM-bound.
+ncclConfig_t nccl_config() {
+    ncclConfig_t cfg = NCCL_CONFIG_INITIALIZER;
+    int max_ctas = 8;
+    if (const char* e = std::getenv("FPM_NCCL_MAX_CTAS")) max_ctas = std::max(1, std::atoi(e));
+    cfg.minCTAs = 1;
+    cfg.maxCTAs = max_ctas;
+    return cfg;
+}
+
+// Wait for `ev` while polling the communicators for asynchronous errors (a peer
+// that died or a network failure would otherwise block forever on the event).
+void nccl_wait(pmm_ctx* ctx, cudaEvent_t ev) {
+    const NcclApi& nc = nccl();
+    for (int spin = 0;; ++spin) {
+        const cudaError_t q = cudaEventQuery(ev);
+        if (q == cudaSuccess) return;
+        if (q != cudaErrorNotReady) CU(q);
+        for (ncclComm_t c : {ctx->world_comm, ctx->col_comm}) {
+            if (!c) continue;
+            ncclResult_t ae = ncclSuccess;
+            NC(nc.CommGetAsyncError(c, &ae));
+            if (ae != ncclSuccess && ae != ncclInProgress) {
+                nc.CommAbort(c);
+                if (c == ctx->world_comm) ctx->world_comm = nullptr;
+                else ctx->col_comm = nullptr;
+                fail(FPM_ENCCL, "NCCL asynchronous error: %s (communicator aborted)", nc.GetErrorString(ae));
+            }
+        }
+        if (spin > 64) std::this_thread::sleep_for(std::chrono::microseconds(200));
+    }
+}
 // A CPU device's stream for pulling pivots out of GPU `cuda_dev`'s memory.
 cudaStream_t pull_stream(Device& d, int cuda_dev) {
     for (auto& ps : d.pulls)
@@ -766,7 +800,14 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         for (int q = 0; q < p; ++q)
             if (rects[q].h > 0 && rects[q].w > 0 && live && rects[q].col == me.col) ctx->col_members.push_back(q);
         const int color = live ? me.col : NCCL_SPLIT_NOCOLOR;
-        NC(nccl().CommSplit(ctx->world_comm, color, ctx->rank, &ctx->col_comm, nullptr));
+        ncclConfig_t cfg = nccl_config();
+        NC(nccl().CommSplit(ctx->world_comm, color, ctx->rank, &ctx->col_comm, &cfg));
+        if (ctx->col_comm) {
+            int cn = 0;
+            NC(nccl().CommCount(ctx->col_comm, &cn));
+            FPM_CHECK_ARG(cn == (int)ctx->col_members.size(), "column communicator has %d ranks, expected %zu", cn,
+                          ctx->col_members.size());
+        }
     }
     for (auto& d : ctx->devs) {
         if (d.cpu) continue;
@@ -778,6 +819,8 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
 
 // ------------------------------------------------------------ iteration parts
 ncclDataType_t nccl_dtype(fpm_dtype dt) { return dt == FPM_F64 ? ncclFloat64 : ncclFloat32; }
+
+
 
 // Host windows streamed into the resident rectangles during the k-loop
 // (pmm_run): block-column k of A and block-row k of B are copied just before
@@ -1008,11 +1051,11 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.accumulate = ctx->groups[g].first != 0;  // the first update writes C = A(0..) B(0..): no zeroing, no read of C
     a.raster_group = ctx->raster_group > 0 ? ctx->raster_group : (sch == SplitScheme::F16I8 ? 12 : 16);
     a.l2_hint_b = ctx->l2_hint_b;
-    a.variant = ctx->kernel_variant;  // -1: auto (F16X3 / TF32X3: variant 7; F16I8: 6)
+    a.variant = ctx->kernel_variant;  // -1: auto (F16X3 / TF32X3: variant 8; F16I8: 6)
     a.chunk_k = ctx->chunk_k;
     // NCCL kernels need shared memory to co-run with the persistent update:
-    // F16I8 then takes variant 5 (198 KB) instead of 6 (224 KB), F16X3 8 (2 stages) instead of 7
-    if (a.variant < 0 && ctx->nccl_mode) a.variant = sch == SplitScheme::F16I8 ? 5 : 8;
+    // F16I8 then takes variant 5 (198 KB) instead of 6 (224 KB); F16X3's auto variant 8 uses 160 KB
+    if (a.variant < 0 && ctx->nccl_mode && sch == SplitScheme::F16I8) a.variant = 5;
     return a;
 }
 
@@ -1732,7 +1775,11 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
             continue;
         }
         CU(cudaSetDevice(d.cuda_dev));
-        CU(cudaEventSynchronize(d.ev_stop));
+        if (ctx->nccl_mode) {  // poll the communicators while waiting (the last
+            nccl_wait(ctx, d.ev_stop);  // update waited for the last exchange)
+        } else {
+            CU(cudaEventSynchronize(d.ev_stop));
+        }
         CU(cudaStreamSynchronize(d.s_comm));
         t_max = std::max(t_max, (double)elapsed_ms(d.ev_start, d.ev_stop) * 1e-3);
         if (tail_done && (*tail_done)[i]) {  // copy still draining after the last update
@@ -2327,10 +2374,17 @@ extern "C" int pmm_create_nccl(int32_t rank, int32_t world, int32_t cuda_device,
         ncclUniqueId id;
         std::memcpy(&id, nccl_id, 128);
         CU(cudaSetDevice(cuda_device));
-        ncclResult_t r = fpm::nccl().CommInitRank(&ctx->world_comm, world, id, rank);
+        ncclConfig_t cfg = fpm::nccl_config();
+        ncclResult_t r = fpm::nccl().CommInitRankConfig(&ctx->world_comm, world, id, rank, &cfg);
         if (r != ncclSuccess) {
             fpm::destroy_device(ctx->devs[0]);
-            fpm::fail(FPM_ENCCL, "ncclCommInitRank: %s", fpm::nccl().GetErrorString(r));
+            fpm::fail(FPM_ENCCL, "ncclCommInitRankConfig: %s", fpm::nccl().GetErrorString(r));
+        }
+        int cn = 0;
+        if (fpm::nccl().CommCount(ctx->world_comm, &cn) != ncclSuccess || cn != world) {
+            fpm::nccl().CommDestroy(ctx->world_comm);
+            fpm::destroy_device(ctx->devs[0]);
+            fpm::fail(FPM_ENCCL, "world communicator has %d ranks, expected %d", cn, world);
         }
         *out = ctx.release();
     });

@@ -60,3 +60,45 @@ def test_ours_json_line_contract_gpu():
     assert d["e2e"]["d2h_bytes_per_step"] == 8192 * 8192 * 4
     assert d["gpu_launches"] > 0 and d["cpu_baseline"]["kind"] == "oracle"
     assert "sm_mhz" in d["clocks"] and "reasons" in d["clocks"]
+
+
+def _bench_module():
+    import importlib.util
+    spec = importlib.util.spec_from_file_location("bench_mod", os.path.join(ROOT, "bench.py"))
+    m = importlib.util.module_from_spec(spec)
+    spec.loader.exec_module(m)
+    return m
+
+
+def test_n_gt_1_line_contract():
+    """The line bench.py prints at N > 1 (built by its pure build_line from the
+    gathered per-device records, as under torchrun): whole-job value = 2 N^3 K /
+    sum of max-over-ranks step times, n_gpus = world, strong scaling, per-device
+    records, measured and predicted imbalance over the ranks."""
+    bm = _bench_module()
+    cfg = dict(bm.CONFIGS["c3"])
+    N, b = cfg["N"], cfg["b"]
+    rects = [[0, 0, 0, 16, 32], [0, 16, 0, 16, 32]]   # p = 2: one column of two 16 x 32-block strips
+    per_dev = [{"rank": r, "device": r, "rect": rects[r], "area": 512, "sm_cap": None,
+                "compute_s": t, "update_s": 0.9 * t, "predicted_s": 0.01} for r, t in enumerate((0.010, 0.011))]
+    roof = {"bound": "tensor", "achieved": 400.0, "peak": 464.5, "unit": "TFLOP/s", "frac": 400.0 / 464.5,
+            "traffic": None}
+    line = bm.build_line(world=2, steps=3, warmup=3, step_times=[0.011, 0.012, 0.011], workload="c3",
+                         cfg=cfg, scheme="f16x3", roofline=roof, per_dev=per_dev,
+                         e2e={"value": 1.0, "unit": "GFLOP/s", "h2d_bytes_per_step": 1, "d2h_bytes_per_step": 1},
+                         cpu=None, parity=None, launches=10, clocks={"sm_mhz": 1.0, "reasons": []},
+                         extra_config={"exchange_staging_overlap": [0.9, 0.8]})
+    for key in ("metric", "value", "unit", "n_gpus", "steps", "warmup", "ms_per_step", "higher_is_better",
+                "scaling", "vs_baseline", "dtype", "data", "config", "roofline", "cpu_baseline", "e2e",
+                "gpu_launches", "clocks"):
+        assert key in line, key
+    assert line["n_gpus"] == 2 and line["scaling"] == "strong" and line["cpu_baseline"] is None
+    assert abs(line["value"] - 2.0 * N ** 3 * 3 / 0.034 / 1e9) < 1e-6 * line["value"]
+    assert abs(line["ms_per_step"] - 1e3 * 0.034 / 3) < 1e-9
+    c = line["config"]
+    assert c["p"] == 2 and len(c["per_device"]) == 2 and c["partition"] == [512, 512]
+    assert abs(c["imbalance_pct_measured"] - 100.0 * (0.011 / 0.0105 - 1)) < 1e-9
+    assert c["imbalance_pct_predicted"] == 0.0
+    assert c["exchange_staging_overlap"] == [0.9, 0.8]
+    assert line["dtype"].startswith("f32 (F16X3")
+    json.dumps(line)
