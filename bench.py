@@ -568,9 +568,9 @@ def run_hetero(peak_tflops: float) -> dict:
 
 
 def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, seeds):
-    """e2e through the public API with pinned host buffers: pmm_run (one process:
-    host panels streamed in, C streamed out) or, under IPC, pmm_upload + barrier +
-    pmm_compute_into (C copied out under the last updates); median of
+    """e2e through the public API with pinned host buffers: pmm_run (host panels
+    streamed in under the k-loop, C streamed out; under IPC every rank streams
+    its own window and peers' pulls wait on its progress flag); median of
     args.e2e_steps calls after one warm-up call, max over ranks.  Returns the
     record and, in one process, the host C (all of it) for the parity check."""
     import torch
@@ -600,12 +600,8 @@ def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, s
     for i in range(args.e2e_steps + 1):
         barrier()
         t0 = time.perf_counter()
-        if ipc:
-            # peers pull from each other's resident inputs: upload, barrier, k-loop, download
-            if live:
-                ctx.upload(hA, hB, W, R0, C0)
-            barrier()
-            st = ctx.compute_into(hC, W, R0, C0) if live else ctx.compute()
+        if ipc and not live:
+            st = ctx.compute()   # takes part in the exchange only
         elif live:
             # blocking call: H2D streamed under the updates, k-loop, D2H of C
             st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32, ld=W, row_base=R0, col_base=C0)
@@ -617,8 +613,9 @@ def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, s
     rec = {"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
            "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
            "device_kloop_s": st.t_compute_s if st else None, "download_s": st.t_download_s if st else None,
-           "timing": ("host wall clock: upload + barrier + pmm_compute_into (IPC), max over ranks"
-                      if ipc else "host wall clock around the blocking pmm_run call, max over ranks")}
+           "timing": ("host wall clock around the blocking pmm_run call (IPC: each rank's window streamed in, "
+                      "peers' pulls ordered by its progress flag), max over ranks" if ipc else
+                      "host wall clock around the blocking pmm_run call, max over ranks")}
     if world > 1:
         rec["h2d_bytes_per_step_rank0"] = rec["h2d_bytes_per_step"]
         tot = torch.tensor([2 * H * W * 4, H * W * 4], dtype=torch.float64)

@@ -294,6 +294,18 @@ int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int6
 int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t* sizes,
                int32_t nsizes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out);
 
+/* The same timing procedure on rectangles: shapes = nshapes (h, w) pairs in
+ * blocks (C of h b x w b; speeds_out[j] = 2 h w b^3 f / t, attributed to the
+ * area x = h w).  P:18: the speed "does not vary with the nearly square shapes
+ * of submatrices", so the rectangles a column arrangement hands out are valid
+ * sample points of the FPM -- the operating-point refinement of reading Q26
+ * samples each device at its own rectangle.  dev = -1: every device of the
+ * context at once, each on its own shapes (shapes device-major, p x nshapes x 2;
+ * outputs p x nshapes), i.e. under the contention of the run.  CPU devices
+ * (dev >= 0 only) and out-of-core GPU sizes are sampled as by fpm_sample. */
+int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t* shapes,
+                     int32_t nshapes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out);
+
 /* Tuning / selection knobs (all optional):
  *   "f32_scheme": -1 = auto (default) = 0.  0 = F16X3 (x 2^e = h0 + h1, both
  *                 fp16, 2^e a per-row / per-column power of two; 3 kind::f16

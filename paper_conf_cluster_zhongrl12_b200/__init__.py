@@ -211,6 +211,25 @@ class Context:
         return cut(sp), cut(ci), cut(reps)
 
 
+    def sample_rects(self, dev: int, b: int, shapes, dtype: int = FPM_F32):
+        """Speed points on rectangles (include/fpmpmm.h fpm_sample_rects): shapes =
+        [(h, w), ...] blocks; dev = -1: one such list per device of the context,
+        all sampled at once.  Returns (speeds, ci, reps) (lists per device for -1)."""
+        per_dev = shapes if dev == -1 else [shapes]
+        n = len(per_dev[0])
+        flat = [int(v) for dev_shapes in per_dev for hw in dev_shapes for v in hw]
+        rows = len(per_dev)
+        arr = (_lib.i64 * len(flat))(*flat)
+        sp = (ctypes.c_double * (n * rows))()
+        ci = (ctypes.c_double * (n * rows))()
+        reps = (ctypes.c_int32 * (n * rows))()
+        check(lib.fpm_sample_rects(self._h, int(dev), int(dtype), int(b), arr, n, sp, ci, reps))
+        if dev != -1:
+            return list(sp), list(ci), list(reps)
+        cut = lambda a: [list(a[i * n:(i + 1) * n]) for i in range(rows)]  # noqa: E731
+        return cut(sp), cut(ci), cut(reps)
+
+
 def fpm_sample(ctx: Context, dev: int, b: int, sizes: Sequence[int], dtype: int = FPM_F32):
     """Speed points s(x) = 2 x b^3 / t(x) of the rank-b kernel."""
     return ctx.sample(dev, b, sizes, dtype)

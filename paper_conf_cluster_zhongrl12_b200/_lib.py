@@ -111,6 +111,8 @@ _SIGS = {
                  ctypes.POINTER(PmmStats)], ctypes.c_int),
     "fpm_sample": ([vp, i32, ctypes.c_int, i64, ctypes.POINTER(i64), i32, ctypes.POINTER(dbl),
                     ctypes.POINTER(dbl), ctypes.POINTER(i32)], ctypes.c_int),
+    "fpm_sample_rects": ([vp, i32, ctypes.c_int, i64, ctypes.POINTER(i64), i32, ctypes.POINTER(dbl),
+                          ctypes.POINTER(dbl), ctypes.POINTER(i32)], ctypes.c_int),
     "fpm_k_split_f32": ([vp, i64, i64, i64, i32, vp, vp, vp, vp], ctypes.c_int),
     "fpm_k_split_cols_f32": ([vp, i64, i64, i64, i32, vp, vp, vp, vp], ctypes.c_int),
     "fpm_k_transpose": ([vp, i32, i64, i64, i64, vp, vp], ctypes.c_int),

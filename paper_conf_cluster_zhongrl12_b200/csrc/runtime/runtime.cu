@@ -11,6 +11,7 @@
 //                   record free[slot]
 // so the exchange and staging of k+1 run under the update of k (P:40/P:68
 // overlap principle; "broadcast horizontally and vertically").
+#include <cuda.h>
 #include <cuda_runtime.h>
 
 #include <algorithm>
@@ -100,6 +101,9 @@ struct Device {
     int64_t H = 0, W = 0;  // rectangle in elements
     void* A = nullptr;     // w block-columns, each H x b row-major (K-major panels)
     void* B = nullptr;     // H x W row-major (h block-rows of b x W)
+    // IPC: upload progress of this rank's panels, at the end of B's allocation
+    // (so peers map it with B): (epoch << 16) | (k + 1) once panels 0..k landed
+    uint64_t* up_flag = nullptr;
     void* C = nullptr;     // H x W row-major
     // operand slots: 0, 1 double-buffer the k-loop; 2 .. 2+tail_slots-1 hold the
     // groups of the download-overlapped tail (compute_into, allocated on demand)
@@ -156,7 +160,9 @@ struct pmm_ctx {
     std::vector<int> col_members;  // global ranks of my column, sorted
     // IPC mode: peers' resident A_q, B_q mapped into this process
     std::vector<void*> peer_A, peer_B;
+    std::vector<uint64_t*> peer_flag;  // peers' upload-progress flags (streamed pmm_run)
     bool peers_ready = false;
+    uint64_t epoch = 0;                // streamed runs issued (the same sequence on every rank)
 
     bool have_problem = false;
     int64_t N = 0, b = 0, n = 0;
@@ -390,6 +396,7 @@ void free_problem(Device& d) {
         v->clear();
     }
     d.A = d.B = d.C = nullptr;
+    d.up_flag = nullptr;
     d.tail_slots = 0;
     for (void* p : d.tail_allocs) cudaFree(p);
     d.tail_allocs.clear();
@@ -514,6 +521,7 @@ void close_peers(pmm_ctx* ctx) {
             if (ptr) cudaIpcCloseMemHandle(ptr);
             ptr = nullptr;
         }
+    std::fill(ctx->peer_flag.begin(), ctx->peer_flag.end(), nullptr);
     ctx->peers_ready = false;
 }
 
@@ -576,6 +584,34 @@ const void* src_B(pmm_ctx* ctx, int q) {
     if (ctx->ipc_mode) return q == ctx->rank ? ctx->devs[0].B : ctx->peer_B[q];
     return local_dev(ctx, q)->B;
 }
+
+// Stream memory operations (driver API, resolved at run time): the streamed
+// IPC pmm_run orders a peer's pulls after this rank's uploads through a 64-bit
+// progress flag in device memory instead of IPC events.
+struct StreamMemOps {
+    CUresult (*write64)(CUstream, CUdeviceptr, cuuint64_t, unsigned) = nullptr;
+    CUresult (*wait64)(CUstream, CUdeviceptr, cuuint64_t, unsigned) = nullptr;
+};
+const StreamMemOps& stream_mem_ops() {
+    static StreamMemOps ops;
+    static bool done = false;
+    if (!done) {
+        cudaDriverEntryPointQueryResult q;
+        void* p = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWriteValue64", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            ops.write64 = reinterpret_cast<decltype(ops.write64)>(p);
+        p = nullptr;
+        if (cudaGetDriverEntryPoint("cuStreamWaitValue64", &p, cudaEnableDefault, &q) == cudaSuccess &&
+            q == cudaDriverEntryPointSuccess)
+            ops.wait64 = reinterpret_cast<decltype(ops.wait64)>(p);
+        cudaGetLastError();
+        done = true;
+    }
+    if (!ops.write64 || !ops.wait64) fail(FPM_EUNSUPPORTED, "cuStreamWriteValue64 / cuStreamWaitValue64 unavailable");
+    return ops;
+}
+uint64_t flag_value(uint64_t epoch, int64_t k) { return (epoch << 16) | (uint64_t)(k + 1); }
 
 bool has_gpu(const pmm_ctx* ctx) {
     for (auto& d : ctx->devs)
@@ -768,7 +804,9 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         }
         const size_t HW = (size_t)d.H * d.W;
         d.A = dalloc(d, HW * es);
-        d.B = dalloc(d, HW * es);
+        d.B = dalloc(d, HW * es + 256);  // + the upload-progress flag (IPC peers map it with B)
+        d.up_flag = reinterpret_cast<uint64_t*>(static_cast<char*>(d.B) + (HW * es + 63) / 64 * 64);
+        CU(cudaMemsetAsync(d.up_flag, 0, 8, d.s_comp));
         d.ooc = d.c_cap > 0 && (int64_t)(HW * es) > d.c_cap;
         if (d.ooc) {  // C_i in pinned host memory, streamed through two band buffers
             d.ring = ring_for(d.c_cap, d.H, d.W, es, ctx->ooc_buffers);
@@ -850,6 +888,24 @@ void issue_upload(pmm_ctx* ctx, Device& d, int64_t k, const HostSrc& h) {
         CU(cudaMemcpy2DAsync(dst, d.W * es, src, h.ld * es, d.W * es, b, cudaMemcpyHostToDevice, d.s_up));
     }
     CU(cudaEventRecord(d.ev_up[k], d.s_up));
+    if (ctx->ipc_mode)  // peers pulling this rank's panels wait for the flag (after the copies above)
+        if (stream_mem_ops().write64(reinterpret_cast<CUstream>(d.s_up), reinterpret_cast<CUdeviceptr>(d.up_flag),
+                                     flag_value(ctx->epoch, k), 0) != CUDA_SUCCESS)
+            fail(FPM_ECUDA, "cuStreamWriteValue64 failed");
+}
+
+// The comm stream of device d waits until holder / owner q's panels through
+// pivot kl have landed (streamed input): q's upload event in one process, q's
+// progress flag in peer memory under IPC.
+void wait_panels(pmm_ctx* ctx, Device& d, int q, int64_t kl) {
+    if (q == d.idx) return;  // own panels: the ev_up wait issued by issue_comm
+    if (!ctx->ipc_mode) {
+        CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, q)->ev_up[kl], 0));
+        return;
+    }
+    if (stream_mem_ops().wait64(reinterpret_cast<CUstream>(d.s_comm), reinterpret_cast<CUdeviceptr>(ctx->peer_flag[q]),
+                                flag_value(ctx->epoch, kl), CU_STREAM_WAIT_VALUE_GEQ) != CUDA_SUCCESS)
+        fail(FPM_ECUDA, "cuStreamWaitValue64 failed");
 }
 
 // Exchange + staging of update group g (pivots k0 .. k0+f-1) on device d's comm
@@ -906,7 +962,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
             const size_t cnt = (size_t)(m.end - m.begin) * b * b;
             const char* src = static_cast<const char*>(src_A(ctx, m.src)) +
                               ((size_t)(k0 - qr.col0) * qH * b + (size_t)(m.begin - qr.row0) * b * b) * es;
-            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[kl], 0));
+            if (streamed) wait_panels(ctx, d, m.src, kl);
             if (fused) {
                 a_pieces.push_back(Piece{src, qH * b, (m.begin - r.row0) * b, (m.end - m.begin) * b});
             } else {  // FP64: copy the f panels' rows into the receive buffer
@@ -932,7 +988,7 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
             if (m.dst != d.idx) continue;
             const colpart_rect& orr = ctx->rects[m.src];
             const char* src = static_cast<const char*>(src_B(ctx, m.src)) + (size_t)(k0 - orr.row0) * b * d.W * es;
-            if (streamed && !ctx->ipc_mode) CU(cudaStreamWaitEvent(d.s_comm, local_dev(ctx, m.src)->ev_up[kl], 0));
+            if (streamed) wait_panels(ctx, d, m.src, kl);
             if (fused) {
                 b_src = src;
             } else {
@@ -1442,7 +1498,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
     if (ctx->ipc_mode && !ctx->peers_ready)
         fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
-    FPM_CHECK_ARG(!(ctx->ipc_mode && host), "IPC mode has no streamed host input (peers cannot be ordered)");
+    if (ctx->ipc_mode && host) ++ctx->epoch;  // this run's progress-flag values (every rank in step)
     // streamed input: the grouping that starts with single pivots (setup)
     struct GroupSwap {
         pmm_ctx* c;
@@ -1996,17 +2052,30 @@ std::vector<int64_t> sample_sides(const int64_t* sizes, int nsizes) {
     return ms;
 }
 
-// Speed function of a CPU device: its kernel C (m b x m b) += A (m b x f b) B
-// (f b x m b) -- the k-loop's fused update -- run by all c cores of the device
-// at once, each on m b / c rows ("the speed of a socket executing the ACML
+// Sample shapes: h x w blocks (C is h b x w b); the square sizes of fpm_sample
+// are m x m, fpm_sample_rects takes any rectangle (the speed "does not
+// vary with the nearly square shapes"; the operating-point refinement samples
+// the rectangles the arrangement gave each device, reading Q26).
+struct Shape {
+    int64_t h, w;
+};
+
+// Speed function of a CPU device: its kernel C (h b x w b) += A (h b x f b) B
+// (f b x w b) -- the k-loop's fused update -- run by all c cores of the device
+// at once, each on h b / c rows ("the speed of a socket executing the ACML
 // kernels simultaneously on c cores, with the problem size x / c on each
 // core"; P:10 (ii) synchronised cores), host-timed (the synchronous approach,
 // P:10), repeated under the same statistical stop rule as the GPU devices (Q8).
-void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vector<int64_t>& ms, double* speeds,
+void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vector<Shape>& shp, double* speeds,
                 double* ci, int32_t* reps_out) {
     using clk = std::chrono::steady_clock;
     const int64_t fb = (int64_t)fuse_factor(ctx, dt, b) * b;
-    const int64_t L = *std::max_element(ms.begin(), ms.end()) * b;
+    int64_t Hm = 0, Wm = 0, area = 0;
+    for (const Shape& x : shp) {
+        Hm = std::max(Hm, x.h * b);
+        Wm = std::max(Wm, x.w * b);
+        area = std::max(area, x.h * x.w * b * b);
+    }
     const size_t es = esize(dt);
     struct Buf {
         void* p = nullptr;
@@ -2015,22 +2084,22 @@ void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vec
     auto get = [&](Buf& x, size_t bytes) {
         if (posix_memalign(&x.p, 64, std::max<size_t>(bytes, 64)) != 0) fail(FPM_ENOMEM, "host allocation failed");
     };
-    get(A, (size_t)L * fb * es);
-    get(B, (size_t)fb * L * es);
-    get(C, (size_t)L * L * es);
-    cpu::fill_synthetic(d.team, A.p, dt == FPM_F64, fb, 101, L, 0, 0, L, fb, FPM_DIST_PM1);
-    cpu::fill_synthetic(d.team, B.p, dt == FPM_F64, L, 102, L, 0, 0, fb, L, FPM_DIST_PM1);
-    std::memset(C.p, 0, (size_t)L * L * es);
-    for (size_t j = 0; j < ms.size(); ++j) {
-        const int64_t Lx = ms[j] * b;
+    get(A, (size_t)Hm * fb * es);
+    get(B, (size_t)fb * Wm * es);
+    get(C, (size_t)area * es);
+    cpu::fill_synthetic(d.team, A.p, dt == FPM_F64, fb, 101, std::max(Hm, Wm), 0, 0, Hm, fb, FPM_DIST_PM1);
+    cpu::fill_synthetic(d.team, B.p, dt == FPM_F64, Wm, 102, std::max(Hm, Wm), 0, 0, fb, Wm, FPM_DIST_PM1);
+    std::memset(C.p, 0, (size_t)area * es);
+    for (size_t j = 0; j < shp.size(); ++j) {
+        const int64_t Mx = shp[j].h * b, Nx = shp[j].w * b;
         auto run = [&] {
             const auto t0 = clk::now();
             if (dt == FPM_F32)
-                cpu::gemm_f32(d.team, Lx, Lx, fb, static_cast<const float*>(A.p), fb, fb, 0,
-                              static_cast<const float*>(B.p), L, static_cast<float*>(C.p), Lx, true);
+                cpu::gemm_f32(d.team, Mx, Nx, fb, static_cast<const float*>(A.p), fb, fb, 0,
+                              static_cast<const float*>(B.p), Wm, static_cast<float*>(C.p), Nx, true);
             else
-                cpu::gemm_f64(d.team, Lx, Lx, fb, static_cast<const double*>(A.p), fb, fb, 0,
-                              static_cast<const double*>(B.p), L, static_cast<double*>(C.p), Lx, true);
+                cpu::gemm_f64(d.team, Mx, Nx, fb, static_cast<const double*>(A.p), fb, fb, 0,
+                              static_cast<const double*>(B.p), Wm, static_cast<double*>(C.p), Nx, true);
             return std::chrono::duration<double>(clk::now() - t0).count();
         };
         run();
@@ -2049,33 +2118,17 @@ void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vec
             half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
             if (nr >= 5 && half <= 0.025 * mean) break;
         }
-        const double x = (double)(ms[j] * ms[j]);
+        const double x = (double)(shp[j].h * shp[j].w);
         speeds[j] = 2.0 * x * (double)b * (double)b * (double)fb / mean;
         if (ci) ci[j] = mean > 0 ? half / mean : 0.0;
         if (reps_out) reps_out[j] = (int32_t)ts.size();
     }
 }
 
-void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes, int nsizes, double* speeds,
-            double* ci, int32_t* reps_out) {
-    FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype");
-    FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 && b >= 8 : b % 32 == 0 && b >= 32, "bad block size b");
-    FPM_CHECK_ARG(nsizes >= 1 && sizes && speeds, "bad sizes");
-    const std::vector<int64_t> ms = sample_sides(sizes, nsizes);
-    std::vector<Device*> devs;
-    if (dev == -1) {
-        if (has_cpu(ctx))
-            fail(FPM_EUNSUPPORTED, "concurrent sampling (dev = -1) of a context with CPU devices: sample each "
-                                   "device (P:11: GPUs and sockets were measured separately)");
-        for (auto& d : ctx->devs) devs.push_back(&d);
-    } else {
-        Device* d = local_dev(ctx, dev);
-        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
-        if (d->cpu) return sample_cpu(ctx, *d, dt, b, ms, speeds, ci, reps_out);
-        devs.push_back(d);
-    }
-    const int64_t mmax = *std::max_element(ms.begin(), ms.end());
-    const int64_t L = mmax * b;
+// devs[i] samples shapes[i][0 .. nshapes) (all devices at once when more than one).
+void sample_gpu(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vector<std::vector<Shape>>& shapes,
+                fpm_dtype dt, int64_t b, double* speeds, double* ci, int32_t* reps_out) {
+    const int nsizes = (int)shapes[0].size();
     const size_t es = dt == FPM_F64 ? 8 : 4;
     const SplitScheme sch = scheme_for(ctx, b);
     const size_t op = op_bytes(sch);
@@ -2090,6 +2143,7 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
         void *C = nullptr, *Ap = nullptr, *Bp = nullptr, *Bt = nullptr;
         void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
         float *sa = nullptr, *sb = nullptr;
+        int64_t Hm = 0, Wm = 0;  // largest rows / columns of C over this device's shapes
         cudaEvent_t e0 = nullptr, e1 = nullptr;
         std::vector<double> ts;
         int runs = 0;  // runs at the current size (out-of-core band order alternates)
@@ -2104,59 +2158,67 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             if (e1) cudaEventDestroy(e1);
         }
     };
-    // sizes whose C exceeds the device's C cap run out of core (as in the k-loop)
-    auto ooc_at = [&](const Device* d, int64_t Lx) { return d->c_cap > 0 && (int64_t)(Lx * Lx * es) > d->c_cap; };
-    auto ring_at = [&](const Device* d, int64_t Lx) { return ring_for(d->c_cap, Lx, Lx, es, ctx->ooc_buffers); };
+    // shapes whose C exceeds the device's C cap run out of core (as in the k-loop)
+    auto ooc_at = [&](const Device* d, int64_t Mx, int64_t Nx) {
+        return d->c_cap > 0 && (int64_t)(Mx * Nx * es) > d->c_cap;
+    };
+    auto ring_at = [&](const Device* d, int64_t Mx, int64_t Nx) {
+        return ring_for(d->c_cap, Mx, Nx, es, ctx->ooc_buffers);
+    };
     std::vector<std::unique_ptr<Scratch>> S;
-    for (Device* d : devs) {
+    for (size_t i = 0; i < devs.size(); ++i) {
+        Device* d = devs[i];
         S.emplace_back(new Scratch);
         Scratch& s = *S.back();
         s.d = d;
         s.mem.cuda_dev = d->cuda_dev;
         CU(cudaSetDevice(d->cuda_dev));
-        int64_t Lin = 0, Lout = 0, nbands = 0;
+        int64_t in_area = 0, out_area = 0, nbands = 0;
         size_t band_bytes = 0;
-        for (int j = 0; j < nsizes; ++j) {
-            const int64_t Lx = ms[j] * b;
-            if (!ooc_at(d, Lx)) {
-                Lin = std::max(Lin, Lx);
+        for (const Shape& x : shapes[i]) {
+            const int64_t Mx = x.h * b, Nx = x.w * b;
+            s.Hm = std::max(s.Hm, Mx);
+            s.Wm = std::max(s.Wm, Nx);
+            if (!ooc_at(d, Mx, Nx)) {
+                in_area = std::max(in_area, Mx * Nx);
                 continue;
             }
-            Lout = std::max(Lout, Lx);
-            const int64_t rows = ring_at(d, Lx).rows;
-            nbands = std::max(nbands, (Lx + rows - 1) / rows);
-            band_bytes = std::max(band_bytes, (size_t)rows * Lx * es);
+            out_area = std::max(out_area, Mx * Nx);
+            const int64_t rows = ring_at(d, Mx, Nx).rows;
+            nbands = std::max(nbands, (Mx + rows - 1) / rows);
+            band_bytes = std::max(band_bytes, (size_t)rows * Nx * es);
         }
-        s.C = dalloc(s.mem, (size_t)Lin * Lin * es);
-        if (Lout > 0) {
+        s.C = dalloc(s.mem, (size_t)in_area * es);
+        if (out_area > 0) {
             bp_init(s.mem.bp);
-            s.hC = static_cast<char*>(halloc(s.mem, (size_t)Lout * Lout * es));
-            std::memset(s.hC, 0, (size_t)Lout * Lout * es);
+            s.hC = static_cast<char*>(halloc(s.mem, (size_t)out_area * es));
+            std::memset(s.hC, 0, (size_t)out_area * es);
             bp_alloc_bands(s.mem, s.mem.bp, ctx->ooc_buffers, band_bytes, nbands);
         }
-        s.Ap = dalloc(s.mem, (size_t)L * fb * es);
-        s.Bp = dalloc(s.mem, (size_t)fb * L * es);
-        s.Bt = dalloc(s.mem, (size_t)L * fb * es);
+        const int64_t L = std::max(s.Hm, s.Wm);
+        s.Ap = dalloc(s.mem, (size_t)s.Hm * fb * es);
+        s.Bp = dalloc(s.mem, (size_t)fb * s.Wm * es);
+        s.Bt = dalloc(s.mem, (size_t)s.Wm * fb * es);
         if (dt == FPM_F32) {
-            s.ah = dalloc(s.mem, (size_t)L * fb * op);
-            s.al = dalloc(s.mem, (size_t)L * fb * op);
-            s.bh = dalloc(s.mem, (size_t)L * fb * op);
-            s.bl = dalloc(s.mem, (size_t)L * fb * op);
-            s.sa = static_cast<float*>(dalloc(s.mem, (size_t)L * 4));
-            s.sb = static_cast<float*>(dalloc(s.mem, (size_t)L * 4));
+            s.ah = dalloc(s.mem, (size_t)s.Hm * fb * op);
+            s.al = dalloc(s.mem, (size_t)s.Hm * fb * op);
+            s.bh = dalloc(s.mem, (size_t)s.Wm * fb * op);
+            s.bl = dalloc(s.mem, (size_t)s.Wm * fb * op);
+            s.sa = static_cast<float*>(dalloc(s.mem, (size_t)s.Hm * 4));
+            s.sb = static_cast<float*>(dalloc(s.mem, (size_t)s.Wm * 4));
         }
         CU(cudaEventCreate(&s.e0));
         CU(cudaEventCreate(&s.e1));
-        launch_fill_synthetic(s.Ap, dt == FPM_F64, fb, 101, L, 0, 0, L, fb, FPM_DIST_PM1, d->s_comp);
-        launch_fill_synthetic(s.Bp, dt == FPM_F64, L, 102, L, 0, 0, fb, L, FPM_DIST_PM1, d->s_comp);
-        if (s.C) CU(cudaMemsetAsync(s.C, 0, (size_t)Lin * Lin * es, d->s_comp));
+        launch_fill_synthetic(s.Ap, dt == FPM_F64, fb, 101, L, 0, 0, s.Hm, fb, FPM_DIST_PM1, d->s_comp);
+        launch_fill_synthetic(s.Bp, dt == FPM_F64, s.Wm, 102, L, 0, 0, fb, s.Wm, FPM_DIST_PM1, d->s_comp);
+        if (s.C) CU(cudaMemsetAsync(s.C, 0, (size_t)in_area * es, d->s_comp));
     }
 
     for (int j = 0; j < nsizes; ++j) {
-        const int64_t Lx = ms[j] * b;
-        auto run = [&](Scratch& s) {
+        auto run = [&](Scratch& s, const Shape& x) {
+            const int64_t Mx = x.h * b, Nx = x.w * b;
             const cudaStream_t st = s.d->s_comp;
-            const bool ooc = ooc_at(s.d, Lx);
+            const bool ooc = ooc_at(s.d, Mx, Nx);
             // out of core: the k-loop's steady state (bands kept and order reversed
             // between consecutive updates)
             BandCall bc;
@@ -2165,14 +2227,14 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             bc.keep_tail = ctx->ooc_keep;
             ++s.runs;
             if (dt == FPM_F32) {
-                launch_split_rows(static_cast<const float*>(s.Ap), fb, Lx, fb, sch, s.ah, s.al, s.sa, st);
-                launch_split_cols(static_cast<const float*>(s.Bp), L, fb, Lx, sch, s.bh, s.bl, s.sb, st);
+                launch_split_rows(static_cast<const float*>(s.Ap), fb, Mx, fb, sch, s.ah, s.al, s.sa, st);
+                launch_split_cols(static_cast<const float*>(s.Bp), s.Wm, fb, Nx, sch, s.bh, s.bl, s.sb, st);
                 UpdateArgs a;
                 a.a_hi = s.ah; a.a_lo = s.al; a.bt_hi = s.bh; a.bt_lo = s.bl;
                 a.sa = has_scales(sch) ? s.sa : nullptr;
                 a.sb = has_scales(sch) ? s.sb : nullptr;
                 a.C = static_cast<float*>(s.C);
-                a.M = Lx; a.Nc = Lx; a.K = fb; a.ldc = Lx;
+                a.M = Mx; a.Nc = Nx; a.K = fb; a.ldc = Nx;
                 a.scheme = sch;
                 a.cta_group = ctx->cta_group;
                 a.num_sms = s.d->num_sms;
@@ -2181,31 +2243,31 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                 a.variant = ctx->kernel_variant;
                 a.chunk_k = ctx->chunk_k;
                 if (ooc) {
-                    banded_update(s.mem.bp, ring_at(s.d, Lx), s.hC, Lx, (size_t)Lx * 4, bc, st,
+                    banded_update(s.mem.bp, ring_at(s.d, Mx, Nx), s.hC, Mx, (size_t)Nx * 4, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
-                                      UpdateArgs x = a;
-                                      x.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
-                                      x.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * fb * op;
-                                      x.sa = a.sa ? a.sa + r0 : nullptr;
-                                      x.C = static_cast<float*>(band);
-                                      x.M = m;
-                                      launch_update_f32(x, st);
+                                      UpdateArgs y = a;
+                                      y.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
+                                      y.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * fb * op;
+                                      y.sa = a.sa ? a.sa + r0 : nullptr;
+                                      y.C = static_cast<float*>(band);
+                                      y.M = m;
+                                      launch_update_f32(y, st);
                                   });
                 } else {
                     launch_update_f32(a, st);
                 }
             } else {  // FP64: the fused update of the k-loop (K = f b, A rows contiguous here)
-                launch_transpose_f64(static_cast<const double*>(s.Bp), L, fb, Lx, static_cast<double*>(s.Bt), st);
+                launch_transpose_f64(static_cast<const double*>(s.Bp), s.Wm, fb, Nx, static_cast<double*>(s.Bt), st);
                 if (ooc) {
-                    banded_update(s.mem.bp, ring_at(s.d, Lx), s.hC, Lx, (size_t)Lx * 8, bc, st,
+                    banded_update(s.mem.bp, ring_at(s.d, Mx, Nx), s.hC, Mx, (size_t)Nx * 8, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
                                       launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * fb, fb,
                                                         static_cast<const double*>(s.Bt), static_cast<double*>(band),
-                                                        m, Lx, fb, Lx, true, s.d->num_sms, st);
+                                                        m, Nx, fb, Nx, true, s.d->num_sms, st);
                                   });
                 } else {
                     launch_update_f64(static_cast<const double*>(s.Ap), fb, static_cast<const double*>(s.Bt),
-                                      static_cast<double*>(s.C), Lx, Lx, fb, Lx, true, s.d->num_sms, st);
+                                      static_cast<double*>(s.C), Mx, Nx, fb, Nx, true, s.d->num_sms, st);
                 }
             }
             if (ooc) bp_join(s.mem.bp, st);  // the update is done when C is back in host memory
@@ -2216,11 +2278,12 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             sp->runs = 0;
         }
         for (int w = 0; w < 2; ++w)
-            for (auto& sp : S) {
-                CU(cudaSetDevice(sp->d->cuda_dev));
-                CU(cudaEventRecord(sp->e0, sp->d->s_comp));
-                run(*sp);
-                CU(cudaEventRecord(sp->e1, sp->d->s_comp));
+            for (size_t i = 0; i < S.size(); ++i) {
+                Scratch& sp = *S[i];
+                CU(cudaSetDevice(sp.d->cuda_dev));
+                CU(cudaEventRecord(sp.e0, sp.d->s_comp));
+                run(sp, shapes[i][j]);
+                CU(cudaEventRecord(sp.e1, sp.d->s_comp));
             }
         // Concurrent sampling: every device must stay busy for the whole window
         // (P:10 (ii): resources "shared between the maximum number of
@@ -2238,11 +2301,12 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
                                   : (int)std::min<double>(64.0, std::max(1.0, std::round(t_max / std::max(sp->t_warm, 1e-9))));
         for (int r = 0; r < 50; ++r) {
             // all devices run every repetition, so contention stays the same until the last converges
-            for (auto& sp : S) {
-                CU(cudaSetDevice(sp->d->cuda_dev));
-                CU(cudaEventRecord(sp->e0, sp->d->s_comp));
-                for (int i = 0; i < sp->k; ++i) run(*sp);
-                CU(cudaEventRecord(sp->e1, sp->d->s_comp));
+            for (size_t i = 0; i < S.size(); ++i) {
+                Scratch& sp = *S[i];
+                CU(cudaSetDevice(sp.d->cuda_dev));
+                CU(cudaEventRecord(sp.e0, sp.d->s_comp));
+                for (int q = 0; q < sp.k; ++q) run(sp, shapes[i][j]);
+                CU(cudaEventRecord(sp.e1, sp.d->s_comp));
             }
             bool all_done = true;
             for (auto& sp : S) {
@@ -2263,15 +2327,50 @@ void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes
             }
             if (all_done) break;
         }
-        const double x = (double)(ms[j] * ms[j]);
         for (size_t i = 0; i < S.size(); ++i) {
             const Scratch& s = *S[i];
             // one timed run = f pivots of the x-block kernel: 2 x b^3 f flop
+            const double x = (double)(shapes[i][j].h * shapes[i][j].w);
             speeds[i * nsizes + j] = 2.0 * x * (double)b * (double)b * (double)fb / s.mean;
             if (ci) ci[i * nsizes + j] = s.mean > 0 ? s.half / s.mean : 0.0;
             if (reps_out) reps_out[i * nsizes + j] = (int32_t)s.ts.size();
         }
     }
+}
+
+// fpm_sample / fpm_sample_rects: shapes per device (dev = -1: every device of
+// the context at once, shapes device-major, p x nshapes).
+void sample_shapes(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const std::vector<std::vector<Shape>>& shapes,
+                   double* speeds, double* ci, int32_t* reps_out) {
+    FPM_CHECK_ARG(dt == FPM_F32 || dt == FPM_F64, "unknown dtype");
+    FPM_CHECK_ARG(dt == FPM_F64 ? b % 8 == 0 && b >= 8 : b % 32 == 0 && b >= 32, "bad block size b");
+    FPM_CHECK_ARG(!shapes.empty() && !shapes[0].empty() && speeds, "bad sizes");
+    for (const auto& v : shapes)
+        for (const Shape& x : v) FPM_CHECK_ARG(x.h >= 1 && x.w >= 1, "shape %lld x %lld", (long long)x.h, (long long)x.w);
+    std::vector<Device*> devs;
+    if (dev == -1) {
+        if (has_cpu(ctx))
+            fail(FPM_EUNSUPPORTED, "concurrent sampling (dev = -1) of a context with CPU devices: sample each "
+                                   "device (P:11: GPUs and sockets were measured separately)");
+        for (auto& d : ctx->devs) devs.push_back(&d);
+    } else {
+        Device* d = local_dev(ctx, dev);
+        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);
+        if (d->cpu) return sample_cpu(ctx, *d, dt, b, shapes[0], speeds, ci, reps_out);
+        devs.push_back(d);
+    }
+    FPM_CHECK_ARG(shapes.size() == devs.size(), "expected shapes for %zu devices", devs.size());
+    sample_gpu(ctx, devs, shapes, dt, b, speeds, ci, reps_out);
+}
+
+void sample(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const int64_t* sizes, int nsizes, double* speeds,
+            double* ci, int32_t* reps_out) {
+    FPM_CHECK_ARG(nsizes >= 1 && sizes && speeds, "bad sizes");
+    const std::vector<int64_t> ms = sample_sides(sizes, nsizes);
+    std::vector<Shape> sq;
+    for (int64_t m : ms) sq.push_back({m, m});
+    const size_t ndev = dev == -1 ? ctx->devs.size() : 1;
+    sample_shapes(ctx, dev, dt, b, std::vector<std::vector<Shape>>(ndev, sq), speeds, ci, reps_out);
 }
 
 }  // namespace
@@ -2404,6 +2503,7 @@ extern "C" int pmm_create_ipc(int32_t rank, int32_t world, int32_t cuda_device, 
         ctx->world = world;
         ctx->peer_A.assign(world, nullptr);
         ctx->peer_B.assign(world, nullptr);
+        ctx->peer_flag.assign(world, nullptr);
         ctx->devs.resize(1);
         ctx->devs[0].idx = rank;
         ctx->devs[0].cuda_dev = cuda_device;
@@ -2468,6 +2568,8 @@ extern "C" int pmm_ipc_import(pmm_ctx* ctx, const uint8_t* blobs, int32_t world)
             if (q == ctx->rank || !blob.live) continue;
             CU(cudaIpcOpenMemHandle(&ctx->peer_A[q], blob.A, cudaIpcMemLazyEnablePeerAccess));
             CU(cudaIpcOpenMemHandle(&ctx->peer_B[q], blob.B, cudaIpcMemLazyEnablePeerAccess));
+            const size_t qHW = (size_t)(r.h * ctx->b) * (size_t)(r.w * ctx->b) * fpm::esize(ctx->dt);
+            ctx->peer_flag[q] = reinterpret_cast<uint64_t*>(static_cast<char*>(ctx->peer_B[q]) + (qHW + 63) / 64 * 64);
         }
         ctx->peers_ready = true;
     });
@@ -2690,9 +2792,9 @@ extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int6
                 const colpart_rect &x = ctx->rects[i], &y = rects[i];
                 same = same && x.col == y.col && x.row0 == y.row0 && x.col0 == y.col0 && x.h == y.h && x.w == y.w;
             }
-        if (ctx->ipc_mode)
-            fpm::fail(FPM_EUNSUPPORTED, "pmm_run is not available on IPC contexts: use pmm_upload, a barrier across "
-                                        "the ranks, pmm_compute, pmm_download");
+        if (ctx->ipc_mode && !(same && ctx->peers_ready))
+            fpm::fail(FPM_EUNSUPPORTED, "pmm_run on an IPC context needs the same problem set up and the peers "
+                                        "imported first (pmm_setup, pmm_ipc_export / import on every rank)");
         if (!same) fpm::setup(ctx, N, b, p, rects, dt);
         FPM_CHECK_ARG(A && B && C, "null host matrix");
         for (auto& d : ctx->devs)
@@ -2723,6 +2825,20 @@ extern "C" int fpm_sample(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, co
     return guarded([&] {
         FPM_CHECK_ARG(ctx != nullptr, "null ctx");
         fpm::sample(ctx, dev, dt, b, sizes, nsizes, speeds_out, rel_ci95_out, reps_out);
+    });
+}
+
+extern "C" int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const int64_t* shapes,
+                                int32_t nshapes, double* speeds_out, double* rel_ci95_out, int32_t* reps_out) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr && shapes != nullptr, "null argument");
+        FPM_CHECK_ARG(nshapes >= 1, "nshapes must be >= 1");
+        const size_t ndev = dev == -1 ? ctx->devs.size() : 1;
+        std::vector<std::vector<fpm::Shape>> shp(ndev);
+        for (size_t i = 0; i < ndev; ++i)
+            for (int j = 0; j < nshapes; ++j)
+                shp[i].push_back({shapes[(i * nshapes + j) * 2], shapes[(i * nshapes + j) * 2 + 1]});
+        fpm::sample_shapes(ctx, dev, dt, b, shp, speeds_out, rel_ci95_out, reps_out);
     });
 }
 

@@ -91,6 +91,8 @@ def main():
     ap.add_argument("--c-caps-mib", default="1024,512,0,0,0,0")
     ap.add_argument("--ncal", type=int, default=40, help="CPM calibration problem, in blocks per side")
     ap.add_argument("--sizes", default="2,4,6,8,10,12,14,16,18,20,22,23,24,26,28,30,32,33,34,36,40,44,48,52,56")
+    ap.add_argument("--cpu-sizes", default="2,4,8,12,16,20,24",
+                    help="sample sides of CPU devices (their speed is flat beyond; the model is constant past the end)")
     ap.add_argument("--reps", type=int, default=2)
     ap.add_argument("--ooc-keep", type=int, default=1)
     ap.add_argument("--ooc-buffers", type=int, default=2, help="R band buffers (2 = the paper's C0, C1)")
@@ -103,14 +105,22 @@ def main():
                          "the shared resource); the others alone")
     ap.add_argument("--sm-partition", type=int, default=0,
                     help="1 = each device in its own green-context SM partition (all its kernels confined)")
+    ap.add_argument("--refine", type=int, default=0,
+                    help="FPM: rounds of operating-point refinement (reading Q26): sample every device at the "
+                         "rectangle the arrangement gave it, all devices at once, add the points, re-partition")
+    ap.add_argument("--arrange", choices=["paper", "fpm"], default="paper",
+                    help="FPM partition arranged by colpart_arrange (paper) or colpart_arrange_fpm (Q25)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "memcap_table3_r01.json"))
     args = ap.parse_args()
-    caps = [int(c) for c in args.caps.split(",")]
+    # "cpuN": a host-CPU device of N pinned cores (NEXT-3: the paper's sockets, P:18 s_c(x))
+    cpu_dev = [c.startswith("cpu") for c in args.caps.split(",")]
+    caps = [int(c[3:]) if c.startswith("cpu") else int(c) for c in args.caps.split(",")]
     names = args.names.split(",")
     c_caps = [int(c) << 20 for c in args.c_caps_mib.split(",")]
     p, b = len(caps), args.b
     ns = [int(x) for x in args.ns.split(",")]
     sizes = [int(m) ** 2 for m in args.sizes.split(",")]
+    cpu_sizes = [int(m) ** 2 for m in args.cpu_sizes.split(",")]
 
     pcie = pcie_bandwidth()
     print("pcie", pcie, flush=True)
@@ -120,16 +130,17 @@ def main():
         c.set_option("ooc_keep", args.ooc_keep)
         c.set_option("ooc_buffers", args.ooc_buffers)
         for j, i in enumerate(devs):
-            c.set_device_option(j, "c_cap_bytes", c_caps[i])
+            if not cpu_dev[i]:
+                c.set_device_option(j, "c_cap_bytes", c_caps[i])
 
-    ctx = pkg.Context.local([0] * p, sm_caps=caps)
+    ctx = pkg.Context.local([pkg.FPM_CPU_DEVICE if c else 0 for c in cpu_dev], sm_caps=caps)
     apply_options(ctx, range(p))
     t0 = time.perf_counter()
     models, sample_info = [], []
     if args.concurrent:
         per_dev = list(zip(*ctx.sample(-1, b, sizes, pkg.FPM_F32)))
     else:                  # each device alone, as the paper measured its GPUs
-        per_dev = [ctx.sample(dev, b, sizes, pkg.FPM_F32) for dev in range(p)]
+        per_dev = [ctx.sample(dev, b, cpu_sizes if cpu_dev[dev] else sizes, pkg.FPM_F32) for dev in range(p)]
     if args.link_group:    # the link-sharing devices again, together in a context of their own
         grp = [int(i) for i in args.link_group.split(",")]
         with pkg.Context.local([0] * len(grp), sm_caps=[caps[i] for i in grp]) as gctx:
@@ -138,8 +149,9 @@ def main():
         for j, i in enumerate(grp):
             per_dev[i] = gsp[j]
     for dev, (sp, ci, reps) in enumerate(per_dev):
-        models.append((sizes, sp))
-        sample_info.append({"name": names[dev], "sm_cap": caps[dev], "c_cap_bytes": c_caps[dev],
+        models.append((cpu_sizes if cpu_dev[dev] else sizes, sp))
+        sample_info.append({"name": names[dev], "sm_cap": None if cpu_dev[dev] else caps[dev],
+                            "cpu_cores": caps[dev] if cpu_dev[dev] else None, "c_cap_bytes": c_caps[dev],
                             "speeds_gflops": [s / 1e9 for s in sp], "rel_ci95": ci, "reps": reps})
         print(f"{names[dev]}: " + " ".join(f"{m}:{s / 1e12:.1f}" for m, s in
                                            zip(args.sizes.split(","), sp)), flush=True)
@@ -147,13 +159,52 @@ def main():
 
     x_cal = max(1, args.ncal * args.ncal // p)
     cpm_models = [([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models]
+
+    def refine(n, T, mods):
+        """Operating-point refinement (Q26, the partial-FPM idea of [5]): the
+        partition's own rectangles are sampled -- every device at once, so the
+        shared host link is contended as in the run (P:10 (ii)) -- and added to
+        the models until the partition stops changing."""
+        mods = [(list(xs), list(ss)) for xs, ss in mods]
+        hist, d_prev = [], None
+        for r in range(args.refine):
+            d = pkg.fpm_partition(T, mods)
+            rects = arrange(n, d, mods)
+            if d == d_prev:
+                break
+            shapes = [[(max(1, rc[3]), max(1, rc[4]))] for rc in rects]
+            if any(cpu_dev):   # CPU devices are sampled on their own (fpm_sample_rects dev >= 0)
+                sp = [ctx.sample_rects(i, b, shapes[i], pkg.FPM_F32)[0] for i in range(p)]
+            else:
+                sp, _, _ = ctx.sample_rects(-1, b, shapes, pkg.FPM_F32)
+            for i, rc in enumerate(rects):
+                if rc[3] * rc[4] == 0:
+                    continue
+                x, sv = rc[3] * rc[4], sp[i][0]
+                xs, ss = mods[i]
+                if x in xs:
+                    ss[xs.index(x)] = sv
+                else:
+                    k = sum(1 for v in xs if v < x)
+                    xs.insert(k, x)
+                    ss.insert(k, sv)
+            hist.append({"d": d, "areas": [rc[3] * rc[4] for rc in rects],
+                         "sampled_tflops": [v[0] / 1e12 for v in sp]})
+            d_prev = d
+        return mods, hist
+
+    def arrange(n, d, mods):
+        return pkg.colpart_arrange_fpm(n, d, mods) if args.arrange == "fpm" else pkg.colpart_arrange(n, d)
+
     table = []
     for n in ns:
         N, T = n * b, n * n
         row = {"n": n, "N": N}
-        for name, mods in (("fpm", models), ("cpm", cpm_models), ("homogeneous", [([1], [1.0])] * p)):
+        fpm_models, hist = refine(n, T, models) if args.refine else (models, [])
+        row["refine"] = hist
+        for name, mods in (("fpm", fpm_models), ("cpm", cpm_models), ("homogeneous", [([1], [1.0])] * p)):
             d = pkg.fpm_partition(T, mods)
-            rects = pkg.colpart_arrange(n, d)
+            rects = arrange(n, d, mods) if name == "fpm" else pkg.colpart_arrange(n, d)
             ctx.setup(N, b, rects, pkg.FPM_F32)
             ctx.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
             ctx.compute()
@@ -166,7 +217,7 @@ def main():
             per_dev = list(best.per_dev_compute_s[:p])
             # FPM-predicted k-loop time: 2 a b^2 N flop at the model's speed s(a)
             pred = [2.0 * a * b * b * N / pkg.fpm_model_speed(m, a) if a > 0 else 0.0
-                    for a, m in zip(areas, models)]
+                    for a, m in zip(areas, fpm_models)]
             row[name] = {
                 "d": d, "areas": areas, "rects": rects,
                 "t_total_s": best.t_compute_s, "gflops": best.gflops,
@@ -186,9 +237,10 @@ def main():
     ctx.close()
 
     out = {
-        "config": {"b": b, "ns": ns, "p": p, "names": names, "sm_caps": caps, "c_cap_bytes": c_caps,
+        "config": {"b": b, "ns": ns, "p": p, "names": names, "sm_caps": caps, "cpu_devices": cpu_dev,
+                   "c_cap_bytes": c_caps,
                    "ncal": args.ncal, "x_cal": x_cal, "sizes": sizes, "ooc_keep": args.ooc_keep, "ooc_buffers": args.ooc_buffers,
-                   "link_group": args.link_group,
+                   "link_group": args.link_group, "refine_rounds": args.refine, "arrange": args.arrange,
                    "sampling": "concurrent (all devices at once)" if args.concurrent else "exclusive",
                    "dtype": "f32 (auto scheme: F16X3, DESIGN Q15)", "sm_partition": args.sm_partition,
                    "gpu": "1x B200; devices emulated by SM caps, device memory by C caps (C_i out of core above)"},

@@ -98,3 +98,64 @@ def test_ipc_three_ranks_mixed_columns():
     assert len({r[0] for r in rects}) == 2
     out = _run(3, rects, N, b, 1)
     assert all(ok is True for (_, ok, _, _) in out), out
+
+
+def _worker_run(rank, world, port, rects, N, b, reps, q):
+    """pmm_run on an IPC context: each rank streams its own host window in (k
+    order, its progress flag written after each pivot's panels) while peers
+    wait on that flag in their streams before pulling; C streamed out."""
+    import sys
+    sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+    import torch.distributed as dist
+
+    import paper_conf_cluster_zhongrl12_b200 as pkg
+    import synth
+    try:
+        torch.cuda.set_device(0)
+        dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
+        col, r0, c0, h, w = rects[rank]
+        H, W = h * b, w * b
+        A = synth.rect(11, N, r0 * b, c0 * b, H, W, synth.DIST_INT)
+        B = synth.rect(12, N, r0 * b, c0 * b, H, W, synth.DIST_INT)
+        results = []
+        with pkg.Context.ipc(rank, world, 0) as ctx:
+            ctx.setup(N, b, rects, pkg.FPM_F32)
+            blobs = [None] * world
+            dist.all_gather_object(blobs, ctx.ipc_export())
+            ctx.ipc_import(blobs)
+            for it in range(reps):           # repeated runs: the flag epochs must not confuse the waits
+                C = np.full((H, W), np.nan, np.float32)
+                dist.barrier()
+                ctx.run(A, B, C, N, b, rects, pkg.FPM_F32, ld=W, row_base=r0 * b, col_base=c0 * b)
+                results.append(C)
+            dist.barrier()
+        from oracle import gemm as og
+        ref = og.gemm(synth.rect(11, N, r0 * b, 0, H, N, synth.DIST_INT),
+                      synth.rect(12, N, 0, c0 * b, N, W, synth.DIST_INT))
+        ok = all(np.array_equal(C.astype(np.float64), ref) for C in results)
+        q.put((rank, ok, 0.0, 0))
+        dist.destroy_process_group()
+    except Exception as e:  # pragma: no cover
+        q.put((rank, repr(e), -1.0, -1))
+
+
+@pytest.mark.parametrize("world,d", [(2, [40, 24]), (3, [70, 44, 30])])
+def test_ipc_streamed_pmm_run(world, d):
+    """pmm_run on IPC contexts (the bench's e2e at N > 1): host windows streamed
+    in under the k-loop, integer inputs bit-exact, three repeated runs."""
+    import paper_conf_cluster_zhongrl12_b200 as pkg
+    N, b = 1536 if world == 3 else 1024, 128
+    n = N // b
+    rects = pkg.colpart_arrange(n, d if world == 2 else d)
+    if world == 2:
+        rects = pkg.colpart_arrange(n, [40, 24])
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_run, args=(r, world, port, rects, N, b, 3, q)) for r in range(world)]
+    for p in procs:
+        p.start()
+    out = sorted(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    assert all(ok is True for (_, ok, _, _) in out), out
