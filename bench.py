@@ -549,7 +549,7 @@ def run_hetero(peak_tflops: float) -> dict:
     from studies import hetero
     caps = [30, 26, 24, 20, 16, 14, 10, 6]   # config 4's {144 .. 32} scaled to fit 148 SMs
     t0 = time.perf_counter()
-    res = hetero.c4_study(caps, N=32768, b=512, reps=2, insitu=1, graph=0, sm_partition=1, log=log)
+    res = hetero.c4_study(caps, N=32768, b=512, reps=2, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3)
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     capped_peak = peak_tflops * sum(caps) / sms
     out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "
@@ -558,6 +558,7 @@ def run_hetero(peak_tflops: float) -> dict:
            "capped_aggregate_peak_tflops": capped_peak, "fpm_sample_s": res["fpm_sample_s"]}
     for name, r in res["partitions"].items():
         out[name] = {"t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],
+                     "refine_rounds": len(r.get("refine_history", [])) or None,
                      "imbalance_pct_measured": 100.0 * r["imbalance_measured"],
                      "imbalance_pct_predicted": 100.0 * r["imbalance_predicted"],
                      "pct_of_capped_peak": 100.0 * r["gflops"] / 1e3 / capped_peak}

@@ -3,7 +3,7 @@
 with devices emulated by SM caps — each device a persistent update grid of
 `cap` SMs — run concurrently on the same GPU):
 
-  c1  N = 512, b = 64, FP64, 2 devices capped {144, 48}: FPMs from 8 sample
+  c1  N = 512, b = 64, FP64, 2 devices in disjoint green partitions {100, 48}: FPMs from 8 sample
       sizes -> fpm_partition -> colpart_arrange -> pmm_run (host A, B, C),
       checked against the CPU oracle (rel-Fro <= 1e-12), oracle time reported.
   c3  N = 16384, b = 512, FP32: p = 1 on the whole GPU; p = 2, 4, 8 homogeneous
@@ -55,7 +55,8 @@ def c1():
     sa, sb = synth.seeds_for_config(0)
     A = synth.rect(sa, N, 0, 0, N, N, dtype=np.float64)
     B = synth.rect(sb, N, 0, 0, N, N, dtype=np.float64)
-    with pkg.Context.local([0, 0], sm_caps=[144, 48]) as ctx:
+    with pkg.Context.local([0, 0], sm_caps=[100, 48]) as ctx:
+        ctx.set_option("sm_partition", 1)   # disjoint SM partitions (reading Q13)
         models = [(sizes, ctx.sample(dev, b, sizes, pkg.FPM_F64)[0]) for dev in range(2)]
         t0 = time.perf_counter()
         d = pkg.fpm_partition(n * n, models)
@@ -69,7 +70,7 @@ def c1():
     t0 = time.perf_counter()
     ref = og.gemm(A, B)
     t_oracle = time.perf_counter() - t0
-    return {"N": N, "b": b, "dtype": "f64", "sm_caps": [144, 48], "partition": d, "rects": rects,
+    return {"N": N, "b": b, "dtype": "f64", "sm_caps": [100, 48], "sm_partition": 1, "partition": d, "rects": rects,
             "models_gflops": [[s / 1e9 for s in m[1]] for m in models],
             "host_partition_arrange_s": t_host, "pmm_run_wall_s": t_run, "k_loop_s": st.t_compute_s,
             "rel_fro": og.rel_fro(C, ref), "oracle_s": t_oracle, "oracle_threads": og.num_threads()}

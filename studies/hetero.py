@@ -39,7 +39,7 @@ def imbalance(ts):
 
 
 def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, graph=1, sm_partition=0,
-             exclusive=True, log=print) -> dict:
+             exclusive=True, log=print, refine_rounds=0) -> dict:
     """Sample each emulated device's FPM, then run the multiply under the FPM,
     CPM (N_cal and self-calibrated), homogeneous and in-situ corrected FPM
     partitions; returns the result dict written by main()."""
@@ -87,9 +87,19 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
             out.append((m[0], [s * r for s in m[1]]))
         return out
 
+    # operating-point refinement (reading Q26): every device timed on its own
+    # rectangle, all at once, points added to the models, partition repeated
+    refined = {}
+    if refine_rounds > 0:
+        from studies import refine as rf
+        for arr in ("paper", "fpm"):
+            mods_r, hist, d_r, rects_r = rf.refine(ctx, n, b, models, refine_rounds, arrange=arr, log=log)
+            refined["fpm_refined" + ("_arr" if arr == "fpm" else "")] = (mods_r, hist, d_r, rects_r)
+
     # "_arr": the same partition arranged by colpart_arrange_fpm (integer widths
     # and heights chosen on the models, reading Q25) instead of colpart_arrange
     order = [("fpm", parts["fpm"]), ("fpm_arr", parts["fpm"])]
+    order += [(k, v[2]) for k, v in refined.items()]
     order += [(k, v) for k, v in parts.items() if k != "fpm"]
     for it in range(insitu):
         order += [(f"fpm_insitu{it + 1}", None), (f"fpm_insitu{it + 1}_arr", None)]
@@ -100,7 +110,9 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
             cur_models = corrected(cur_models, prev)
         if d is None:
             d = pkg.fpm_partition(T, cur_models)
-        if name.endswith("_arr"):
+        if name in refined:
+            rects = refined[name][3]
+        elif name.endswith("_arr"):
             rects = pkg.colpart_arrange_fpm(n, d, cur_models if name.startswith("fpm_insitu") else models)
         else:
             rects = pkg.colpart_arrange(n, d)
@@ -115,8 +127,10 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
         areas = [r[3] * r[4] for r in rects]
         per_dev = list(best.per_dev_compute_s[:p])
         # FPM-predicted k-loop time: 2 a b^2 N flop at the model's speed s(a)
+        pred_models = (refined[name][0] if name in refined else
+                       cur_models if name.startswith("fpm_insitu") else models)
         pred = [2.0 * a * b * b * N / pkg.fpm_model_speed(m, a) if a > 0 else 0.0
-                for a, m in zip(areas, cur_models if name.startswith("fpm_insitu") else models)]
+                for a, m in zip(areas, pred_models)]
         results[name] = {
             "d": d, "areas": areas, "rects": rects,
             "t_total_s": best.t_compute_s, "gflops": best.gflops,
@@ -125,6 +139,8 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
             "predicted_time_s": max(pred),
             "comm_bytes": best.comm_bytes,
         }
+        if name in refined:
+            results[name]["refine_history"] = refined[name][1]
         log(f"{name:12s} t={best.t_compute_s:8.4f}s  {best.gflops / 1e3:8.1f} TFLOP/s  "
             f"imb meas={100 * imbalance(per_dev):6.2f}%  pred={100 * imbalance(pred):6.2f}%  d={d}")
     ctx.close()
@@ -162,11 +178,13 @@ def main():
     ap.add_argument("--graph", type=int, default=1, help="pmm_compute as a replayed CUDA graph (option graph)")
     ap.add_argument("--sm-partition", type=int, default=0,
                     help="1 = each device in its own green-context SM partition (all its kernels confined)")
+    ap.add_argument("--refine", type=int, default=0, help="rounds of operating-point refinement (Q26)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
     args = ap.parse_args()
     caps = [int(c) for c in args.caps.split(",")]
     out = c4_study(caps, args.N, args.b, [int(m) ** 2 for m in args.sizes.split(",")], args.ncal, args.reps,
-                   args.insitu, args.graph, args.sm_partition, args.exclusive, log=lambda s: print(s, flush=True))
+                   args.insitu, args.graph, args.sm_partition, args.exclusive, log=lambda s: print(s, flush=True),
+                   refine_rounds=args.refine)
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)

@@ -271,19 +271,24 @@ def test_fpm_sample_all_devices_concurrently():
 
 
 def test_config1_fp64_two_capped_devices():
-    """BASELINE config 1: N=512, b=64, FP64, two devices with SM caps {144, 48}:
-    FPMs from 8 sample sizes -> partition -> arrangement -> multiply."""
+    """BASELINE config 1: N=512, b=64, FP64, two emulated devices in DISJOINT
+    green-context SM partitions of the GPU, caps {100, 48} (reading Q13): FPMs
+    from 8 sample sizes -> partition (bit-exact vs the oracle) -> arrangement ->
+    multiply (within 1e-12 of the oracle)."""
+    from oracle import fpm as ofpm
     N, b = 512, 64
     n = N // b
     sizes = [m * m for m in range(1, 9)]
-    with pkg.Context.local([0, 0], sm_caps=[144, 48]) as ctx:
+    with pkg.Context.local([0, 0], sm_caps=[100, 48]) as ctx:
+        ctx.set_option("sm_partition", 1)
         models = []
         for dev in range(2):
             sp, _, _ = ctx.sample(dev, b, sizes, pkg.FPM_F64)
             models.append((sizes, sp))
         d = pkg.fpm_partition(n * n, models)
-        assert sum(d) == n * n
+        assert sum(d) == n * n and d == ofpm.partition(n * n, models)
         rects = pkg.colpart_arrange(n, d)
+        assert rects == ofpm.arrange(n, d)
         A, B, C, _ = _run(ctx, N, b, rects, pkg.FPM_F64, seeds=(1, 2))
         assert og.rel_fro(C, og.gemm(A, B)) <= 1e-12
 
