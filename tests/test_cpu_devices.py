@@ -193,3 +193,34 @@ def test_cpu_device_options_and_errors():
         C = np.empty((N, N), np.float32)
         ctx.run(A, B, C, N, b, [(0, 0, 0, 4, 4)], pkg.FPM_F32)        # still works after the failed move
         assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+def test_sample_rects_and_operating_point_refinement():
+    """fpm_sample_rects on a CPU device (any rectangle, speed attributed to
+    x = h w) and the operating-point refinement loop (studies/refine.py,
+    reading Q26) on two CPU devices: it terminates, every round's partition sums
+    to T, and the refined models contain the sampled areas."""
+    if NCORES < 2:
+        pytest.skip("needs 2 host cores")
+    from studies import refine as rf
+    n, b = 12, 64
+    with pkg.Context.local([CPU, CPU], sm_caps=[1, 1]) as ctx:
+        sp, ci, reps = ctx.sample_rects(0, b, [(2, 3), (3, 2), (4, 4)], pkg.FPM_F32)
+        assert len(sp) == 3 and all(s > 0 for s in sp) and all(r >= 5 for r in reps)
+        sizes = [1, 4, 16]
+        models = [(sizes, ctx.sample(i, b, sizes, pkg.FPM_F32)[0]) for i in range(2)]
+        mods, hist, d, rects = rf.refine(ctx, n, b, models, rounds=3, concurrent=False)
+        assert sum(d) == n * n and 1 <= len(hist) <= 3
+        for h in hist:
+            assert sum(h["d"]) == n * n
+            for i, a in enumerate(h["areas"]):
+                if a > 0:
+                    assert a in mods[i][0]
+        assert rects == pkg.colpart_arrange(n, d)
+
+
+def test_refine_add_point():
+    from studies import refine as rf
+    assert rf.add_point(([1, 4, 9], [1.0, 2.0, 3.0]), 6, 2.5) == ([1, 4, 6, 9], [1.0, 2.0, 2.5, 3.0])
+    assert rf.add_point(([1, 4], [1.0, 2.0]), 4, 5.0) == ([1, 4], [1.0, 5.0])
+    assert rf.add_point(([4], [2.0]), 1, 1.0) == ([1, 4], [1.0, 2.0])

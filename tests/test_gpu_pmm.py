@@ -363,3 +363,20 @@ def test_c4_full_size_sampled_parity(sm_partition):
                     B_cols[c0] = synth.rect(2, N, 0, c0, N, 64)
                 ref = og.gemm(A_rows, B_cols[c0])
                 assert og.rel_fro(got, ref) <= 1e-5, (r0, c0, og.rel_fro(got, ref))
+
+
+def test_sample_rects_gpu():
+    """fpm_sample_rects (reading Q26): a square rectangle times like fpm_sample's
+    square size (within the sampling noise), a near-square rectangle of the
+    same area likewise, and dev = -1 samples every device on its own
+    shape at once (2 devices: the 96-SM device's larger rectangle)."""
+    with pkg.Context.local([0, 0], sm_caps=[96, 48]) as ctx:
+        sq, _, _ = ctx.sample(0, 512, [64], pkg.FPM_F32)
+        r, ci, reps = ctx.sample_rects(0, 512, [(8, 8), (4, 16)], pkg.FPM_F32)
+        assert all(v > 0 for v in r) and all(n >= 5 for n in reps)
+        assert abs(r[0] / sq[0] - 1) < 0.15
+        assert abs(r[1] / r[0] - 1) < 0.2
+        sp, _, _ = ctx.sample_rects(-1, 512, [[(12, 12)], [(6, 6)]], pkg.FPM_F32)
+        assert len(sp) == 2 and sp[0][0] > sp[1][0] > 0
+        with pytest.raises(pkg.FpmError):
+            ctx.sample_rects(0, 512, [(0, 4)], pkg.FPM_F32)
