@@ -321,10 +321,33 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     # gathered so every rank partitions identically
     sizes = [m * m for m in ((1, 2, 4, 8, 12, 16, 20, 24, 28, 32) if caps else (1, 2, 4, 8, 12, 16))]
     t0 = time.perf_counter()
+    fpm_source = "sampled"
     if args.no_sample:  # profiling runs: identical constant models, predictable launch order
         mine_models = [(sizes, [1.0] * len(sizes)) for _ in mine]
+        fpm_source = "constant (profiling)"
     else:
-        mine_models = [(sizes, ctx.sample(dev, b, sizes, pkg.FPM_F32)[0]) for dev in mine]
+        from paper_conf_cluster_zhongrl12_b200 import fpm_store
+        meta = [{"device": torch.cuda.get_device_name(local_rank), "kind": "gpu",
+                 "sm_cap": caps[dev] if caps else 0, "cores": None, "dtype": "f32", "b": b,
+                 "scheme": args.scheme, "fuse": args.fuse} for dev in mine]
+        cache = (f"{args.fpm_cache}.rank{rank}" if world > 1 else args.fpm_cache) if args.fpm_cache else None
+        mine_models = None
+        if cache and os.path.exists(cache):   # FPMs built in advance, reused if measured alike
+            try:
+                recs = fpm_store.load(cache, expect=meta)
+                if all(r["x"] == sizes for r in recs):
+                    mine_models = fpm_store.models(recs)
+                    fpm_source = f"loaded from {cache}"
+            except ValueError as ex:
+                log(f"rank {rank}: FPM cache not used: {ex}")
+        if mine_models is None:
+            recs = []
+            for dev, m in zip(mine, meta):
+                sp, ci, reps = ctx.sample(dev, b, sizes, pkg.FPM_F32)
+                recs.append(fpm_store.record(sizes, sp, ci, reps, **m))
+            mine_models = fpm_store.models(recs)
+            if cache:
+                fpm_store.save(cache, recs)
     t_sample = time.perf_counter() - t0
     if world > 1:
         models = [None] * world
@@ -517,7 +540,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "config": args.config, "cta_group": args.cta_group, "raster_group": args.raster_group,
                 "kernel_variant": args.kernel_variant, "chunk_k": args.chunk_k, "fuse": args.fuse,
                 "update_launches_per_step": st.updates, "transport": transport,
-                "fpm_sample_s": t_sample, "fpm_sizes": sizes,
+                "fpm_sample_s": t_sample, "fpm_sizes": sizes, "fpm_models": fpm_source,
                 "comm_bytes_per_step": comm // max(1, args.steps),
                 # share of the exchange + staging time hidden under the updates, per rank (CUDA
                 # events of each rank's streams; SURVEY §8(d) c5 "broadcast/update overlap")
@@ -656,6 +679,9 @@ def main():
     ap.add_argument("--no-hetero", action="store_true",
                     help="skip the emulated-heterogeneity measurement (c4 analogue) added at N = 1")
     ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")
+    ap.add_argument("--fpm-cache", default="",
+                    help="FPM model file: reused when it was measured on the same device / cap / b / scheme, "
+                         "else sampled and written (per rank under torchrun: PATH.rankR)")
     ap.add_argument("--same-gpu", action="store_true",
                     help="testing only: put every rank on cuda:0 (IPC transport works within one GPU)")
     ap.add_argument("--traffic", type=float, default=None,

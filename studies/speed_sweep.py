@@ -4,12 +4,12 @@
 (1) Standalone kernel curve (the Fig. 3 analogue): the update kernel
     alone, C_i += A(b) B(b) with an L x L C and K = b in {512, 64}, L from 64 to
     16384 (x1.5 / x2 steps), uncapped and SM-capped; GFLOPS and fraction of the
-    tensor roofline of the FP32 scheme (--scheme: f16i8 default, f16x3).  Timed with CUDA events on the launching stream over
+    tensor roofline of the FP32 scheme (--scheme: f16x3 default, f16i8).  Timed with CUDA events on the launching stream over
     repeated launches (inputs resident; C is 1 GB at L = 16384).
 (2) Model points: fpm_sample at x = m^2 blocks (m = 1..32, b = 512), i.e. the
     FPM the partitioner consumes (P:18 sqrt(x) x sqrt(x)).
 
-Writes profiles/speed_sweep_r01_<scheme>.json.
+Writes profiles/speed_sweep_r02_<scheme>.json.
 """
 from __future__ import annotations
 
@@ -69,12 +69,12 @@ def time_update(L, K, cap, scheme, reps=20):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--caps", default="0,74,30")
-    ap.add_argument("--scheme", choices=sorted(SCHEMES), default="f16i8")
+    ap.add_argument("--scheme", choices=sorted(SCHEMES), default="f16x3")
     ap.add_argument("--out", default=None)
     args = ap.parse_args()
     scheme, per_mac, basis = SCHEMES[args.scheme]
     if args.out is None:
-        args.out = os.path.join(ROOT, "profiles", f"speed_sweep_r01_{args.scheme}.json")
+        args.out = os.path.join(ROOT, "profiles", f"speed_sweep_r02_{args.scheme}.json")
     caps = [int(c) for c in args.caps.split(",")]
     burst, sustained = peak_alg_tflops(per_mac)
     torch.cuda.set_device(0)
