@@ -39,7 +39,7 @@ def imbalance(ts):
 
 
 def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, graph=1, sm_partition=0,
-             exclusive=True, log=print, refine_rounds=0) -> dict:
+             exclusive=True, log=print, refine_rounds=0, options=None) -> dict:
     """Sample each emulated device's FPM, then run the multiply under the FPM,
     CPM (N_cal and self-calibrated), homogeneous and in-situ corrected FPM
     partitions; returns the result dict written by main()."""
@@ -51,6 +51,8 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
     ctx = pkg.Context.local([0] * p, sm_caps=caps)
     ctx.set_option("sm_partition", sm_partition)
     ctx.set_option("graph", graph)
+    for k, v in (options or {}).items():
+        ctx.set_option(k, v)
     t0 = time.perf_counter()
     models, sample_info = [], []
     if exclusive:   # each device alone (how the paper measured its GPUs)
@@ -94,6 +96,7 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
         from studies import refine as rf
         for arr in ("paper", "fpm"):
             mods_r, hist, d_r, rects_r = rf.refine(ctx, n, b, models, refine_rounds, arrange=arr, log=log)
+            # (synchronised level correction of the exclusive models, Q26)
             refined["fpm_refined" + ("_arr" if arr == "fpm" else "")] = (mods_r, hist, d_r, rects_r)
 
     # "_arr": the same partition arranged by colpart_arrange_fpm (integer widths
@@ -179,12 +182,14 @@ def main():
     ap.add_argument("--sm-partition", type=int, default=0,
                     help="1 = each device in its own green-context SM partition (all its kernels confined)")
     ap.add_argument("--refine", type=int, default=0, help="rounds of operating-point refinement (Q26)")
+    ap.add_argument("--option", action="append", default=[], help="context option key=value (repeatable)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hetero_c4_r01.json"))
     args = ap.parse_args()
     caps = [int(c) for c in args.caps.split(",")]
     out = c4_study(caps, args.N, args.b, [int(m) ** 2 for m in args.sizes.split(",")], args.ncal, args.reps,
                    args.insitu, args.graph, args.sm_partition, args.exclusive, log=lambda s: print(s, flush=True),
-                   refine_rounds=args.refine)
+                   refine_rounds=args.refine,
+                   options={kv.split("=")[0]: int(kv.split("=")[1]) for kv in args.option})
     os.makedirs(os.path.dirname(args.out), exist_ok=True)
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)

@@ -106,8 +106,10 @@ def main():
     ap.add_argument("--sm-partition", type=int, default=0,
                     help="1 = each device in its own green-context SM partition (all its kernels confined)")
     ap.add_argument("--refine", type=int, default=0,
-                    help="FPM: rounds of operating-point refinement (reading Q26): sample every device at the "
-                         "rectangle the arrangement gave it, all devices at once, add the points, re-partition")
+                    help="FPM: rounds of synchronised level correction (reading Q26): every device timed on the "
+                         "rectangle it was given, all at once, its model rescaled, re-partition (fpm_refined)")
+    ap.add_argument("--cliff", type=int, default=1,
+                    help="1: bracket each capped GPU's memory cliff with two near-square samples (Q26)")
     ap.add_argument("--arrange", choices=["paper", "fpm"], default="paper",
                     help="FPM partition arranged by colpart_arrange (paper) or colpart_arrange_fpm (Q25)")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "memcap_table3_r01.json"))
@@ -160,51 +162,34 @@ def main():
     x_cal = max(1, args.ncal * args.ncal // p)
     cpm_models = [([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models]
 
-    def refine(n, T, mods):
-        """Operating-point refinement (Q26, the partial-FPM idea of [5]): the
-        partition's own rectangles are sampled -- every device at once, so the
-        shared host link is contended as in the run (P:10 (ii)) -- and added to
-        the models until the partition stops changing."""
-        mods = [(list(xs), list(ss)) for xs, ss in mods]
-        hist, d_prev = [], None
-        for r in range(args.refine):
-            d = pkg.fpm_partition(T, mods)
-            rects = arrange(n, d, mods)
-            if d == d_prev:
-                break
-            shapes = [[(max(1, rc[3]), max(1, rc[4]))] for rc in rects]
-            if any(cpu_dev):   # CPU devices are sampled on their own (fpm_sample_rects dev >= 0)
-                sp = [ctx.sample_rects(i, b, shapes[i], pkg.FPM_F32)[0] for i in range(p)]
-            else:
-                sp, _, _ = ctx.sample_rects(-1, b, shapes, pkg.FPM_F32)
-            for i, rc in enumerate(rects):
-                if rc[3] * rc[4] == 0:
-                    continue
-                x, sv = rc[3] * rc[4], sp[i][0]
-                xs, ss = mods[i]
-                if x in xs:
-                    ss[xs.index(x)] = sv
-                else:
-                    k = sum(1 for v in xs if v < x)
-                    xs.insert(k, x)
-                    ss.insert(k, sv)
-            hist.append({"d": d, "areas": [rc[3] * rc[4] for rc in rects],
-                         "sampled_tflops": [v[0] / 1e12 for v in sp]})
-            d_prev = d
-        return mods, hist
-
     def arrange(n, d, mods):
         return pkg.colpart_arrange_fpm(n, d, mods) if args.arrange == "fpm" else pkg.colpart_arrange(n, d)
+
+    from studies import refine as rf
+    splits = [None] * p
+    if args.cliff:   # bracket each capped GPU device's memory cliff with two samples (Q26)
+        for i in range(p):
+            if c_caps[i] and not cpu_dev[i]:
+                models[i] = rf.cliff_points(ctx, i, b, models[i], c_caps[i])
+                splits[i] = rf.cliff_areas(c_caps[i], b)[0][0]
+                sample_info[i]["cliff_points"] = [(x, s / 1e9) for x, s in zip(*models[i])
+                                                  if x not in sizes]
 
     table = []
     for n in ns:
         N, T = n * b, n * n
         row = {"n": n, "N": N}
-        fpm_models, hist = refine(n, T, models) if args.refine else (models, [])
-        row["refine"] = hist
-        for name, mods in (("fpm", fpm_models), ("cpm", cpm_models), ("homogeneous", [([1], [1.0])] * p)):
+        parts = [("fpm", models, None)]
+        if args.refine:
+            r_models, hist, r_d, r_rects = rf.refine(ctx, n, b, models, args.refine, arrange=args.arrange,
+                                                      concurrent=not any(cpu_dev), splits=splits,
+                                                      log=lambda m: print(m, flush=True))
+            row["refine"] = hist
+            parts.append(("fpm_refined", r_models, r_rects))
+        parts += [("cpm", cpm_models, None), ("homogeneous", [([1], [1.0])] * p, None)]
+        for name, mods, given in parts:
             d = pkg.fpm_partition(T, mods)
-            rects = arrange(n, d, mods) if name == "fpm" else pkg.colpart_arrange(n, d)
+            rects = given if given is not None else (arrange(n, d, mods) if name == "fpm" else pkg.colpart_arrange(n, d))
             ctx.setup(N, b, rects, pkg.FPM_F32)
             ctx.fill_synthetic(5, 6, pkg.FPM_DIST_PM1)
             ctx.compute()
@@ -217,7 +202,7 @@ def main():
             per_dev = list(best.per_dev_compute_s[:p])
             # FPM-predicted k-loop time: 2 a b^2 N flop at the model's speed s(a)
             pred = [2.0 * a * b * b * N / pkg.fpm_model_speed(m, a) if a > 0 else 0.0
-                    for a, m in zip(areas, fpm_models)]
+                    for a, m in zip(areas, mods if name.startswith("fpm") else models)]
             row[name] = {
                 "d": d, "areas": areas, "rects": rects,
                 "t_total_s": best.t_compute_s, "gflops": best.gflops,
@@ -233,6 +218,10 @@ def main():
                   + f"  ooc={row[name]['ooc']}", flush=True)
         row["fpm_vs_cpm_time_delta"] = row["fpm"]["t_total_s"] / row["cpm"]["t_total_s"] - 1.0
         row["fpm_vs_homogeneous_time_delta"] = row["fpm"]["t_total_s"] / row["homogeneous"]["t_total_s"] - 1.0
+        if "fpm_refined" in row:
+            row["fpm_refined_vs_cpm_time_delta"] = row["fpm_refined"]["t_total_s"] / row["cpm"]["t_total_s"] - 1.0
+            row["fpm_refined_vs_homogeneous_time_delta"] = (row["fpm_refined"]["t_total_s"] /
+                                                             row["homogeneous"]["t_total_s"] - 1.0)
         table.append(row)
     ctx.close()
 
@@ -241,6 +230,7 @@ def main():
                    "c_cap_bytes": c_caps,
                    "ncal": args.ncal, "x_cal": x_cal, "sizes": sizes, "ooc_keep": args.ooc_keep, "ooc_buffers": args.ooc_buffers,
                    "link_group": args.link_group, "refine_rounds": args.refine, "arrange": args.arrange,
+                   "cliff_points": args.cliff,
                    "sampling": "concurrent (all devices at once)" if args.concurrent else "exclusive",
                    "dtype": "f32 (auto scheme: F16X3, DESIGN Q15)", "sm_partition": args.sm_partition,
                    "gpu": "1x B200; devices emulated by SM caps, device memory by C caps (C_i out of core above)"},
@@ -250,7 +240,8 @@ def main():
     with open(args.out, "w") as f:
         json.dump(out, f, indent=1)
     print(json.dumps([{"n": r["n"], "fpm_vs_cpm": r["fpm_vs_cpm_time_delta"],
-                       "fpm_vs_homogeneous": r["fpm_vs_homogeneous_time_delta"]} for r in table]))
+                       "fpm_vs_homogeneous": r["fpm_vs_homogeneous_time_delta"],
+                       "fpm_refined_vs_homogeneous": r.get("fpm_refined_vs_homogeneous_time_delta")} for r in table]))
 
 
 if __name__ == "__main__":

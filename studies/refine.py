@@ -1,22 +1,34 @@
-"""Operating-point refinement of the FPMs (reading Q26).
+"""FPM construction helpers beyond the square size sweep (reading Q26).
 
 The speed functions are sampled in advance on sqrt(x) x sqrt(x) submatrices
-(P:18).  Between two sample sizes the model is a straight segment, which
-misses a memory cliff that lies between them, and each device was timed alone,
-so resources shared in the run (a host link, the power budget of a GPU that
-several emulated devices share) are not in the model.  Refinement: partition,
-arrange, then time every device on the very rectangle it was given -- all
-devices at once (P:10 (ii): "processes are synchronised ... the resources will
-be shared between the maximum number of processes") -- add those points to the
-models (the speed does not vary with the nearly square shapes, so a
-rectangle of area h w is a sample of x = h w) and repeat until the partition
-stops changing.  This is the partial-model idea of [5]: the model is
-made exact where the partitioner looks.
+(P:18), each device alone.  Two things such a model can miss:
 
-Orchestration only: sampling (fpm_sample_rects), partitioning and arranging
-are library calls.
+1. **A memory cliff between two sample sizes.**  A device whose C_i must fit a
+   memory cap is fast up to x_in = cap / (b^2 s) blocks and out of core above
+   (Fig. 3).  With squares only, the cliff lies between m^2 and
+   (m+1)^2 and the linear segment across it promises intermediate speeds that
+   do not exist.  `cliff_points` samples the largest in-core area and the
+   smallest out-of-core area as nearly square rectangles (the speed "does
+   not vary with the nearly square shapes") and adds them, so the model drops
+   within a few blocks, where the device does.
+
+2. **Resources shared in the run.**  Devices measured alone do not see the
+   host link, power budget or memory system they share with the others when
+   all run (P:10 (ii): measure "synchronised" processes, so "the resources
+   will be shared between the maximum number of processes").  `refine` times
+   every device on the very rectangle the partition gave it, all devices at
+   once (fpm_sample_rects dev = -1: each repeats its kernel to fill a common
+   window), and rescales the device's model by measured / modelled speed at
+   that point -- the shape stays the one of the size sweep, the level becomes
+   the synchronised one; for a capped device only the points on the same side
+   of its cliff -- then re-partitions, until the partition stops changing.
+
+Orchestration only: sampling (fpm_sample / fpm_sample_rects), partitioning and
+arranging are library calls.
 """
 from __future__ import annotations
+
+import math
 
 import paper_conf_cluster_zhongrl12_b200 as pkg
 
@@ -33,14 +45,66 @@ def add_point(model, x, s):
     return xs, ss
 
 
-def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=pkg.FPM_F32, log=None):
-    """Returns (refined models, history, d, rects) for T = n^2 blocks.
-    arrange: "paper" (colpart_arrange) or "fpm" (colpart_arrange_fpm on the
-    current models).  concurrent: sample all devices at once (fpm_sample_rects
-    dev = -1; contexts with CPU devices sample each device alone)."""
+def near_square(x, max_aspect=2.0):
+    """A rectangle (h, w), h <= w, h w = x, with the smallest aspect ratio
+    w / h <= max_aspect, or None."""
+    best = None
+    for h in range(int(math.isqrt(x)), 0, -1):
+        if x % h == 0:
+            w = x // h
+            if w / h <= max_aspect:
+                best = (h, w)
+            break
+    return best
+
+
+def cliff_areas(cap_bytes, b, es=4, max_aspect=2.0):
+    """(largest in-core area, smallest out-of-core area) in blocks, each with a
+    nearly square rectangle: ((x_in, (h, w)), (x_out, (h, w)))."""
+    x_cap = cap_bytes // (b * b * es)
+    x_in = x_cap
+    while x_in > 0 and near_square(x_in, max_aspect) is None:
+        x_in -= 1
+    x_out = x_cap + 1
+    while near_square(x_out, max_aspect) is None:
+        x_out += 1
+    return (x_in, near_square(x_in, max_aspect)), (x_out, near_square(x_out, max_aspect))
+
+
+def cliff_points(ctx, dev, b, model, cap_bytes, dtype=pkg.FPM_F32, es=4):
+    """Model with the two points that bracket device dev's memory cliff."""
+    (x_in, r_in), (x_out, r_out) = cliff_areas(cap_bytes, b, es)
+    shapes = [r for r in (r_in, r_out) if r is not None]
+    sp, _, _ = ctx.sample_rects(dev, b, shapes, dtype)
+    m = model
+    for (x, _), s in zip([p for p in ((x_in, r_in), (x_out, r_out)) if p[1] is not None], sp):
+        m = add_point(m, x, s)
+    return m
+
+
+def rescale(model, x_op, s_op, split=None):
+    """The model times s_op / model(x_op): all points, or -- with a cliff at
+    `split` (largest in-core area) -- those on x_op's side of it."""
+    r = s_op / pkg.fpm_model_speed(model, x_op)
+    xs, ss = list(model[0]), list(model[1])
+    for i, x in enumerate(xs):
+        if split is None or (x <= split) == (x_op <= split):
+            ss[i] *= r
+    return xs, ss, r
+
+
+def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=pkg.FPM_F32, splits=None,
+           log=None):
+    """Synchronised level correction: returns (models, history, d, rects) for
+    T = n^2 blocks.  arrange: "paper" (colpart_arrange) or "fpm"
+    (colpart_arrange_fpm on the current models); concurrent: sample all devices
+    at once (contexts with CPU devices: each device alone); splits: per device
+    the largest in-core area (None: no cliff)."""
     T = n * n
     p = len(models)
+    base = [(list(xs), list(ss)) for xs, ss in models]   # the size sweep's shapes
     mods = [(list(xs), list(ss)) for xs, ss in models]
+    splits = splits or [None] * p
 
     def place(m):
         d = pkg.fpm_partition(T, m)
@@ -56,14 +120,20 @@ def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=
             sp = [row[0] for row in sp]
         else:
             sp = [ctx.sample_rects(i, b, shapes[i], dtype)[0][0] for i in range(p)]
+        ratios = []
         for i, r in enumerate(rects):
-            if r[3] * r[4] > 0:
-                mods[i] = add_point(mods[i], r[3] * r[4], sp[i])
+            x = r[3] * r[4]
+            if x > 0:
+                xs, ss, k = rescale(base[i], x, sp[i], splits[i])
+                mods[i] = (xs, ss)
+                ratios.append(k)
+            else:
+                ratios.append(None)
         hist.append({"round": it, "d": list(d), "areas": [r[3] * r[4] for r in rects],
-                     "sampled_gflops": [v / 1e9 for v in sp]})
+                     "sampled_gflops": [v / 1e9 for v in sp], "level_ratio": ratios})
         d_new, rects_new = place(mods)
         if log:
-            log(f"refine {it}: d={d} -> {d_new}")
+            log(f"refine {it}: d={d} -> {d_new}  ratios={[round(k, 3) if k else None for k in ratios]}")
         if d_new == d:
             break
         d, rects = d_new, rects_new

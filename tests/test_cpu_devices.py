@@ -197,9 +197,10 @@ def test_cpu_device_options_and_errors():
 
 def test_sample_rects_and_operating_point_refinement():
     """fpm_sample_rects on a CPU device (any rectangle, speed attributed to
-    x = h w) and the operating-point refinement loop (studies/refine.py,
-    reading Q26) on two CPU devices: it terminates, every round's partition sums
-    to T, and the refined models contain the sampled areas."""
+    x = h w) and the synchronised level correction (studies/refine.py, reading
+    Q26) on two CPU devices: it terminates, every round's partition sums to T,
+    and each refined model is its size-sweep model times one ratio (the shape
+    is kept), the ratio = sampled / modelled speed at the operating point."""
     if NCORES < 2:
         pytest.skip("needs 2 host cores")
     from studies import refine as rf
@@ -213,10 +214,30 @@ def test_sample_rects_and_operating_point_refinement():
         assert sum(d) == n * n and 1 <= len(hist) <= 3
         for h in hist:
             assert sum(h["d"]) == n * n
-            for i, a in enumerate(h["areas"]):
-                if a > 0:
-                    assert a in mods[i][0]
-        assert rects == pkg.colpart_arrange(n, d)
+        last = hist[-1]
+        for i in range(2):
+            assert mods[i][0] == sizes
+            k = last["level_ratio"][i]
+            assert all(abs(a - k * s0) <= 1e-9 * a for a, s0 in zip(mods[i][1], models[i][1]))
+            x = last["areas"][i]
+            assert abs(pkg.fpm_model_speed(mods[i], x) - last["sampled_gflops"][i] * 1e9) <= 1e-6 * pkg.fpm_model_speed(mods[i], x)
+
+
+def test_cliff_areas_and_rescale():
+    """Cliff bracketing: 1 GiB of FP32 C at b = 512 holds 1024 blocks (32 x 32);
+    1025 = 25 x 41 is not nearly square, the smallest out-of-core area with a
+    rectangle of aspect <= 2 is 1026 = 27 x 38.  rescale() keeps the other
+    side of a cliff untouched."""
+    from studies import refine as rf
+    (x_in, r_in), (x_out, r_out) = rf.cliff_areas(1 << 30, 512)
+    assert (x_in, r_in) == (1024, (32, 32))
+    assert x_out > 1024 and r_out[0] * r_out[1] == x_out and r_out[1] / r_out[0] <= 2.0
+    assert all(rf.near_square(x) is None for x in range(1025, x_out))
+    m = ([1, 4, 1024, x_out, 2000], [1.0, 2.0, 3.0, 1.0, 1.0])
+    xs, ss, k = rf.rescale(m, 2000, 0.5, split=1024)
+    assert k == 0.5 and ss == [1.0, 2.0, 3.0, 0.5, 0.5]
+    xs, ss, k = rf.rescale(m, 4, 4.0)
+    assert k == 2.0 and ss == [2.0, 4.0, 6.0, 2.0, 2.0]
 
 
 def test_refine_add_point():
