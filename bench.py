@@ -572,12 +572,21 @@ def run_hetero(peak_tflops: float) -> dict:
     from studies import hetero
     caps = [30, 26, 24, 20, 16, 14, 10, 6]   # config 4's {144 .. 32} scaled to fit 148 SMs
     t0 = time.perf_counter()
-    res = hetero.c4_study(caps, N=32768, b=512, reps=2, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3)
+    res = hetero.c4_study(caps, N=32768, b=512, reps=2, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3,
+                          refine_arrange=("fpm",))
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     capped_peak = peak_tflops * sum(caps) / sms
     out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "
                         f"SM partitions {caps}; FPMs sampled per device alone (P:11), "
                         f"{len(res['config']['sizes'])} sizes"),
+           "partitions": {"fpm": "FPM partition of the exclusive size-sweep models, paper arrangement",
+                          "fpm_arr": "the same, FPM-chosen integer arrangement (Q25)",
+                          "fpm_refined_arr": "FPM after synchronised level correction at the operating point "
+                                             "(Q26), FPM-chosen integer arrangement",
+                          "cpm_ncal": "constant models at the even share of N_cal = 8192 (Q9)",
+                          "cpm_self": "constant models at this run's even share",
+                          "homogeneous": "equal areas",
+                          "fpm_insitu1": "models rescaled by one FPM run's own per-device times (side study)"},
            "capped_aggregate_peak_tflops": capped_peak, "fpm_sample_s": res["fpm_sample_s"]}
     for name, r in res["partitions"].items():
         out[name] = {"t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],

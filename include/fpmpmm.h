@@ -385,7 +385,9 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *                 the devices' streams: set it before pmm_setup.
  *   "raster_group": tile-rows per L2 raster group of the update (0 = auto,
  *                 the default: 12 for F16I8, 16 for F16X3 / TF32X3, measured
- *                 at c5).
+ *                 at c5, times the device's share of the SMs of its GPU among
+ *                 the context's devices on it, at least 1: devices sharing a
+ *                 GPU share its L2, so their A groups must fit it together).
  *   "l2_hint_b":  L2 policy of the B^T operand tiles: 0 normal (default),
  *                 1 evict-first, 2 evict-last.
  * FPM_EINVAL on unknown key or value. */

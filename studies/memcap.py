@@ -166,12 +166,13 @@ def main():
         return pkg.colpart_arrange_fpm(n, d, mods) if args.arrange == "fpm" else pkg.colpart_arrange(n, d)
 
     from studies import refine as rf
-    splits = [None] * p
+    splits, cliffs = [None] * p, [None] * p
     if args.cliff:   # bracket each capped GPU device's memory cliff with two samples (Q26)
         for i in range(p):
             if c_caps[i] and not cpu_dev[i]:
                 models[i] = rf.cliff_points(ctx, i, b, models[i], c_caps[i])
-                splits[i] = rf.cliff_areas(c_caps[i], b)[0][0]
+                (x_in, r_in), (x_out, r_out) = rf.cliff_areas(c_caps[i], b)
+                splits[i], cliffs[i] = x_in, (r_in, r_out)
                 sample_info[i]["cliff_points"] = [(x, s / 1e9) for x, s in zip(*models[i])
                                                   if x not in sizes]
 
@@ -182,7 +183,7 @@ def main():
         parts = [("fpm", models, None)]
         if args.refine:
             r_models, hist, r_d, r_rects = rf.refine(ctx, n, b, models, args.refine, arrange=args.arrange,
-                                                      concurrent=not any(cpu_dev), splits=splits,
+                                                      concurrent=not any(cpu_dev), splits=splits, cliffs=cliffs,
                                                       log=lambda m: print(m, flush=True))
             row["refine"] = hist
             parts.append(("fpm_refined", r_models, r_rects))

@@ -94,17 +94,22 @@ def rescale(model, x_op, s_op, split=None):
 
 
 def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=pkg.FPM_F32, splits=None,
-           log=None):
+           cliffs=None, log=None):
     """Synchronised level correction: returns (models, history, d, rects) for
     T = n^2 blocks.  arrange: "paper" (colpart_arrange) or "fpm"
     (colpart_arrange_fpm on the current models); concurrent: sample all devices
     at once (contexts with CPU devices: each device alone); splits: per device
-    the largest in-core area (None: no cliff)."""
+    the largest in-core area (None: no cliff); cliffs: per device the two
+    bracketing rectangles ((h, w) in core, (h, w) out of core) -- a capped
+    device is then also timed, in the same synchronised window, on the cliff
+    rectangle on the other side of its operating point, so both sides of its
+    model get their synchronised level."""
     T = n * n
     p = len(models)
     base = [(list(xs), list(ss)) for xs, ss in models]   # the size sweep's shapes
     mods = [(list(xs), list(ss)) for xs, ss in models]
     splits = splits or [None] * p
+    cliffs = cliffs or [None] * p
 
     def place(m):
         d = pkg.fpm_partition(T, m)
@@ -114,26 +119,36 @@ def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=
     d, rects = place(mods)
     hist = []
     for it in range(rounds):
-        shapes = [[(max(1, r[3]), max(1, r[4]))] for r in rects]
+        shapes = []
+        for i, r in enumerate(rects):
+            op = (max(1, r[3]), max(1, r[4]))
+            other = op
+            if splits[i] is not None and cliffs[i] is not None and r[3] * r[4] > 0:
+                other = cliffs[i][1] if r[3] * r[4] <= splits[i] else cliffs[i][0]
+            shapes.append([op, other])
         if concurrent:
             sp, _, _ = ctx.sample_rects(-1, b, shapes, dtype)
-            sp = [row[0] for row in sp]
         else:
-            sp = [ctx.sample_rects(i, b, shapes[i], dtype)[0][0] for i in range(p)]
+            sp = [ctx.sample_rects(i, b, shapes[i], dtype)[0] for i in range(p)]
         ratios = []
         for i, r in enumerate(rects):
             x = r[3] * r[4]
-            if x > 0:
-                xs, ss, k = rescale(base[i], x, sp[i], splits[i])
-                mods[i] = (xs, ss)
-                ratios.append(k)
-            else:
+            if x <= 0:
                 ratios.append(None)
+                continue
+            xs, ss, k = rescale(base[i], x, sp[i][0], splits[i])
+            if splits[i] is not None and shapes[i][1] != shapes[i][0]:   # the other side of the cliff
+                xo = shapes[i][1][0] * shapes[i][1][1]
+                xs, ss, k2 = rescale((xs, ss), xo, sp[i][1], splits[i])
+                ratios.append((k, k2))
+            else:
+                ratios.append(k)
+            mods[i] = (xs, ss)
         hist.append({"round": it, "d": list(d), "areas": [r[3] * r[4] for r in rects],
-                     "sampled_gflops": [v / 1e9 for v in sp], "level_ratio": ratios})
+                     "sampled_gflops": [v[0] / 1e9 for v in sp], "level_ratio": ratios})
         d_new, rects_new = place(mods)
         if log:
-            log(f"refine {it}: d={d} -> {d_new}  ratios={[round(k, 3) if k else None for k in ratios]}")
+            log(f"refine {it}: d={d} -> {d_new}  ratios={ratios}")
         if d_new == d:
             break
         d, rects = d_new, rects_new
