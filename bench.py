@@ -630,14 +630,39 @@ def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, s
         torch.cuda.empty_cache()
     barrier()
     ts, st = [], None
+    streamed = True   # IPC: streamed pmm_run (peer progress flags); fallback: upload + barrier + compute_into
+
+    def ipc_resident_call():
+        if live:
+            ctx.upload(hA, hB, W, R0, C0)
+        barrier()
+        return ctx.compute_into(hC, W, R0, C0) if live else ctx.compute()
+
     for i in range(args.e2e_steps + 1):
         barrier()
         t0 = time.perf_counter()
         if ipc and not live:
             st = ctx.compute()   # takes part in the exchange only
+        elif ipc and not streamed:
+            st = ipc_resident_call()
         elif live:
             # blocking call: H2D streamed under the updates, k-loop, D2H of C
-            st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32, ld=W, row_base=R0, col_base=C0)
+            try:
+                st = ctx.run(hA, hB, hC, N, b, rects, pkg.FPM_F32, ld=W, row_base=R0, col_base=C0)
+            except pkg.FpmError as ex:
+                if not ipc or i > 0:
+                    raise
+                log(f"rank {rank}: streamed IPC pmm_run failed ({ex}); using upload + barrier + compute_into")
+                streamed = False
+        if ipc and i == 0:   # every rank takes the same path from here on
+            flag = torch.tensor([1 if streamed else 0], dtype=torch.int32)
+            import torch.distributed as dist
+            dist.all_reduce(flag, op=dist.ReduceOp.MIN)
+            if int(flag.item()) == 0 and streamed:
+                streamed = False
+            if not streamed:
+                barrier()
+                st = ipc_resident_call()
         t_host = time.perf_counter() - t0
         t_all = max_over_ranks(t_host)
         if i > 0:  # first call is a warm-up
@@ -646,8 +671,9 @@ def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, s
     rec = {"value": 2.0 * N ** 3 / t / 1e9, "unit": UNIT, "h2d_bytes_per_step": 2 * H * W * 4,
            "d2h_bytes_per_step": H * W * 4, "steps": len(ts), "ms_per_step": 1e3 * t,
            "device_kloop_s": st.t_compute_s if st else None, "download_s": st.t_download_s if st else None,
-           "timing": ("host wall clock around the blocking pmm_run call (IPC: each rank's window streamed in, "
-                      "peers' pulls ordered by its progress flag), max over ranks" if ipc else
+           "timing": (("host wall clock around the blocking pmm_run call (IPC: each rank's window streamed in, "
+                       "peers' pulls ordered by its progress flag), max over ranks") if (ipc and streamed) else
+                      "host wall clock: pmm_upload + barrier + pmm_compute_into (IPC), max over ranks" if ipc else
                       "host wall clock around the blocking pmm_run call, max over ranks")}
     if world > 1:
         rec["h2d_bytes_per_step_rank0"] = rec["h2d_bytes_per_step"]
