@@ -307,6 +307,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         c.set_option("l2_hint_b", args.l2_hint_b)
         c.set_option("kernel_variant", args.kernel_variant)
         c.set_option("chunk_k", args.chunk_k)
+        c.set_option("raster_snake", args.raster_snake)
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
         c.set_option("e2e_tail", args.e2e_tail)
@@ -538,7 +539,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             per_dev=per_dev, e2e=e2e, cpu=cpu, parity=parity, launches=launches, clocks=clk,
             extra_config={
                 "config": args.config, "cta_group": args.cta_group, "raster_group": args.raster_group,
-                "kernel_variant": args.kernel_variant, "chunk_k": args.chunk_k, "fuse": args.fuse,
+                "kernel_variant": args.kernel_variant, "chunk_k": args.chunk_k, "raster_snake": args.raster_snake,
+                "fuse": args.fuse,
                 "update_launches_per_step": st.updates, "transport": transport,
                 "fpm_sample_s": t_sample, "fpm_sizes": sizes, "fpm_models": fpm_source,
                 "comm_bytes_per_step": comm // max(1, args.steps),
@@ -705,6 +707,7 @@ def main():
     ap.add_argument("--raster-group", type=int, default=0, help="0 = auto (12 for F16I8, 16 otherwise)")
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
+    ap.add_argument("--raster-snake", type=int, default=0, help="serpentine raster over groups (0/1)")
     ap.add_argument("--chunk-k", type=int, default=0, help="K per TMEM accumulation (variants 7/8; 0 auto = 512)")
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
     ap.add_argument("--e2e-steps", type=int, default=5)

@@ -32,6 +32,7 @@ struct UpdateArgs {
     bool accumulate = true;  // false: C = A . Bt^T (no read of C)
     int raster_group = 16;   // tile-rows per raster group (L2 reuse)
     int l2_hint_b = 0;       // B^T tile L2 policy: 0 evict_normal, 1 evict_first, 2 evict_last
+    bool raster_snake = false;  // variants 7 / 8: odd raster groups walk the columns backwards
     int variant = -1;        // smem split (cta_group 2): -1 auto (= 8), 4 = SW128 x 2 + 4 C chunks,
                              // 0 = SW128 x 3 stages + 2 C chunks, 1 = SW64 x 4 + 6,
                              // 2 = SW128 x 2 + 6, 3 = SW64 x 5 + 4,

@@ -74,6 +74,7 @@ struct UpdParams {
     uint64_t hint_b;  // L2 policy of the B^T tiles (A tiles: evict_last, C: evict_first)
     int prof;         // F16I8: accumulate MMA-issuer wait cycles into g_hyb_prof (fpm_k_prof)
     int chunk_kb;     // chunked kernel: k-blocks per TMEM accumulation
+    int snake;        // chunked kernel: serpentine raster over groups
 };
 
 // Diagnostic counters of the F16I8 MMA issuer (leader CTAs, lane 0), summed over
@@ -86,7 +87,10 @@ static bool g_prof_on = false;
 // Grouped raster over tiles so concurrently running CTAs share A / B tiles in L2:
 // groups of G tile-rows, column-major inside a group (A rows of the group stay
 // resident while the B^T tiles stream once per group).
-__device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int G, int& tm, int& tn) {
+// snake: odd groups walk the columns right to left, so a group starts on the
+// B^T column tiles the previous group used last (still in L2).
+__device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int G, int& tm, int& tn,
+                                            bool snake = false) {
     const int per_group = G * tiles_n;
     const int g = t / per_group;
     const int first_m = g * G;
@@ -94,6 +98,7 @@ __device__ __forceinline__ void tile_coords(int t, int tiles_m, int tiles_n, int
     const int r = t - g * per_group;
     tm = first_m + r % gm;
     tn = r / gm;
+    if (snake && (g & 1)) tn = tiles_n - 1 - tn;
 }
 
 template <int CG, int KIND, int BN, int STAGES, int SW, int NCB, int MREP = 1, bool RED = false>
@@ -448,7 +453,7 @@ __global__ void __launch_bounds__(320, 1)
             uint32_t phase = 0;
             for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
                 int tm, tn;
-                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn, P.snake != 0);
                 const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
                 const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA;
                 for (int kb = 0; kb < num_kb; ++kb) {
@@ -521,7 +526,7 @@ __global__ void __launch_bounds__(320, 1)
         int it = 0;
         for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
             int tm, tn;
-            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn);
+            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn, P.snake != 0);
             const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
             const int n0 = tn * Cfg::BN + (int)hh * 128;
             float s[128];
@@ -1071,6 +1076,7 @@ static void launch_update_acc_t(const UpdateArgs& a, cudaStream_t st) {
     P.prof = 0;
     const int chunk_k = a.chunk_k > 0 ? a.chunk_k : 512;
     P.chunk_kb = (chunk_k + Cfg::BK - 1) / Cfg::BK;
+    P.snake = a.raster_snake ? 1 : 0;
     auto kern = update_acc_kernel<KIND, STAGES, NCB>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;

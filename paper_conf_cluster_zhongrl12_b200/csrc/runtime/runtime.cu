@@ -177,6 +177,7 @@ struct pmm_ctx {
     int l2_hint_b = 0;
     int kernel_variant = -1;  // auto
     int chunk_k = 0;          // F16X3 / TF32X3 default kernel: K per TMEM accumulation (0 auto = 512)
+    int raster_snake = 0;     // F16X3 / TF32X3 default kernel: serpentine raster over groups
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
@@ -1125,6 +1126,7 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     a.l2_hint_b = ctx->l2_hint_b;
     a.variant = ctx->kernel_variant;  // -1: auto (F16X3 / TF32X3: variant 8; F16I8: 6)
     a.chunk_k = ctx->chunk_k;
+    a.raster_snake = ctx->raster_snake != 0;
     // NCCL kernels need shared memory to co-run with the persistent update:
     // F16I8 then takes variant 5 (198 KB) instead of 6 (224 KB); F16X3's auto variant 8 uses 160 KB
     if (a.variant < 0 && ctx->nccl_mode && sch == SplitScheme::F16I8) a.variant = 5;
@@ -2258,6 +2260,7 @@ void sample_gpu(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vecto
                 a.l2_hint_b = ctx->l2_hint_b;
                 a.variant = ctx->kernel_variant;
                 a.chunk_k = ctx->chunk_k;
+                a.raster_snake = ctx->raster_snake != 0;
                 if (ooc) {
                     banded_update(s.mem.bp, ring_at(s.d, Mx, Nx), s.hC, Mx, (size_t)Nx * 4, bc, st,
                                   [&](int64_t r0, int64_t m, void* band) {
@@ -2657,6 +2660,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= -1 && value <= 8,
                           "kernel_variant must be -1 (auto) or 0..8 (6: F16I8 only; 7, 8: F16X3 / TF32X3 only)");
             ctx->kernel_variant = (int)value;
+        } else if (k == "raster_snake") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "raster_snake must be 0 or 1");
+            ctx->raster_snake = (int)value;
         } else if (k == "chunk_k") {
             FPM_CHECK_ARG(value >= 0 && value <= (1 << 20), "chunk_k must be 0 (auto = 512) or a positive K");
             ctx->chunk_k = (int)value;

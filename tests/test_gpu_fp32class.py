@@ -229,3 +229,29 @@ def test_chunked_accumulation_bounds_error_at_long_k(chunk_k):
     rows = np.arange(0, N, 257)
     err = og.rel_fro(C[rows, :], og.gemm(np.ascontiguousarray(A[rows, :]), B))
     assert err <= TOL, (chunk_k, err)
+
+
+@pytest.mark.parametrize("opts", [{"raster_snake": 1}, {"raster_group": 1}, {"raster_group": 3, "raster_snake": 1},
+                                  {"chunk_k": 128}])
+def test_tile_order_and_chunking_options_keep_c_bit_identical(opts):
+    """Raster group / serpentine order only reorder the tiles; every element's
+    sums are the same, so C is bit-identical to the default (one device and
+    three devices sharing the GPU, whose auto raster groups differ).  A smaller
+    chunk changes where the register sums split K, but not the tolerance."""
+    N, b = 2048, 256
+    n = N // b
+    A, B = make_inputs("gauss", N, b, seed=71)
+    for d in ([n * n], [32, 20, 12]):
+        rects = pkg.colpart_arrange(n, d)
+        out = []
+        for o in ({}, opts):
+            C = np.full((N, N), np.nan, np.float32)
+            with pkg.Context.local([0] * len(d)) as ctx:
+                for k, v in o.items():
+                    ctx.set_option(k, v)
+                ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+            out.append(C)
+        if "chunk_k" in opts:
+            assert og.rel_fro(out[1], og.gemm(A, B)) <= TOL
+        else:
+            assert np.array_equal(out[0], out[1]), (opts, d)
