@@ -255,3 +255,27 @@ def test_tile_order_and_chunking_options_keep_c_bit_identical(opts):
             assert og.rel_fro(out[1], og.gemm(A, B)) <= TOL
         else:
             assert np.array_equal(out[0], out[1]), (opts, d)
+
+
+@pytest.mark.parametrize("N,b,fuse,d", [(32, 32, 1, [1]), (96, 32, 1, [5, 4]), (4096, 2048, 1, [4]),
+                                        (1600, 320, 0, [13, 12]), (2304, 64, 8, [600, 300, 200, 196])])
+def test_default_kernel_edge_shapes(N, b, fuse, d):
+    """The default chunked kernel at the edges: one 32 x 32 block (smaller than
+    a tile, K far below one chunk), K = 32 updates, b = 2048 (K = 2048 per
+    update, the largest block), ragged tiles with b = 320, and K = 512 fused
+    groups of 8 b = 64 pivots over four devices; integer inputs must come out
+    bit-exact, U[-1,1) within 1e-5."""
+    n = N // b
+    rects = pkg.colpart_arrange(n, d)
+    for dist in (synth.DIST_INT, synth.DIST_PM1):
+        A = synth.rect(81, N, 0, 0, N, N, dist)
+        B = synth.rect(82, N, 0, 0, N, N, dist)
+        C = np.full((N, N), np.nan, np.float32)
+        with pkg.Context.local([0] * len(d)) as ctx:
+            ctx.set_option("fuse", fuse)
+            ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+        ref = og.gemm(A, B)
+        if dist == synth.DIST_INT:
+            np.testing.assert_array_equal(C.astype(np.float64), ref)
+        else:
+            assert og.rel_fro(C, ref) <= TOL
