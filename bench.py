@@ -252,6 +252,10 @@ def build_line(*, world, steps, warmup, step_times, workload, cfg, scheme, roofl
         "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
         "imbalance_pct_measured": 100.0 * imbalance(meas),
         "imbalance_pct_predicted": 100.0 * imbalance(pred),
+        # the same over the devices' k-loop spans (start to their last update's end):
+        # staging that overlaps a device's updates counted once
+        "imbalance_pct_span": 100.0 * imbalance([d.get("span_s", 0.0) for d in per_dev
+                                                  if d["rect"][3] * d["rect"][4] > 0]),
         "per_device": per_dev,
     }
     config.update(extra_config or {})
@@ -399,7 +403,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         d = pkg.fpm_partition(T, part_models)
         return d, pkg.colpart_arrange(n, d)
 
-    def per_device(comp, upd, rects, part_models):
+    def per_device(comp, upd, span, rects, part_models):
         """Per-device records (Fig. 6 metric): this process's devices (comp /
         upd indexed by device, as pmm_stats), gathered over the ranks."""
         recs = []
@@ -408,7 +412,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             a = r[3] * r[4]
             recs.append({"rank": rank, "device": dev, "rect": list(r), "area": a,
                          "sm_cap": caps[dev] if caps else None,
-                         "compute_s": comp[dev], "update_s": upd[dev],
+                         "compute_s": comp[dev], "update_s": upd[dev], "span_s": span[dev],
                          "predicted_s": (2.0 * a * b * b * N / pkg.fpm_model_speed(part_models[dev], a)
                                          if a > 0 else 0.0)})
         if world > 1:
@@ -434,7 +438,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         st = ctx.compute(zero_c=True)
         own_times.append(st.t_compute_s)
         step_times.append(max_over_ranks(st.t_compute_s))
-        recs_steps.append([(st.per_dev_compute_s[i], st.per_dev_update_s[i]) for i in range(16)])
+        recs_steps.append([(st.per_dev_compute_s[i], st.per_dev_update_s[i], st.per_dev_span_s[i]) for i in range(16)])
         launches += st.kernel_launches
         comm += st.comm_bytes
     barrier()
@@ -442,7 +446,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     clk = clocks.stop()
     # the median step's per-device record
     med = sorted(range(args.steps), key=lambda i: own_times[i])[args.steps // 2]
-    per_dev = per_device([x[0] for x in recs_steps[med]], [x[1] for x in recs_steps[med]], rects, models)
+    per_dev = per_device([x[0] for x in recs_steps[med]], [x[1] for x in recs_steps[med]],
+                         [x[2] for x in recs_steps[med]], rects, models)
     mine_recs = [x for x in per_dev if x["rank"] == rank]
     upd_med = max(x["update_s"] for x in mine_recs)
     comp_med = max(x["compute_s"] for x in mine_recs)
@@ -501,7 +506,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 t2 = max_over_ranks(s2.t_compute_s)
                 if t_best is None or t2 < t_best:
                     best, t_best = s2, t2
-            recs = per_device(list(best.per_dev_compute_s), list(best.per_dev_update_s), rr, models)
+            recs = per_device(list(best.per_dev_compute_s), list(best.per_dev_update_s), list(best.per_dev_span_s),
+                              rr, models)
             partitions[name] = {"t_s": t_best, "d": list(dd),
                                 "imbalance_pct_measured": 100.0 * imbalance([x["compute_s"] for x in recs]),
                                 "imbalance_pct_predicted": 100.0 * imbalance([x["predicted_s"] for x in recs])}
@@ -594,6 +600,7 @@ def run_hetero(peak_tflops: float) -> dict:
         out[name] = {"t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],
                      "refine_rounds": len(r.get("refine_history", [])) or None,
                      "imbalance_pct_measured": 100.0 * r["imbalance_measured"],
+                     "imbalance_pct_span": 100.0 * r.get("imbalance_span", 0.0),
                      "imbalance_pct_predicted": 100.0 * r["imbalance_predicted"],
                      "pct_of_capped_peak": 100.0 * r["gflops"] / 1e3 / capped_peak}
     out["fpm_vs_cpm_time_delta_pct"] = 100.0 * res["fpm_vs_cpm_ncal_time_delta"]

@@ -95,6 +95,9 @@ typedef struct {
     int64_t updates;                            /* rank-(f b) update launches (f pivots fused)    */
     int64_t ooc_devices;                        /* bit i: device i held C_i out of core           */
     int64_t ooc_bytes;                          /* C bytes streamed host <-> device (out of core) */
+    double  per_dev_span_s[FPM_MAX_DEVICES];    /* k-loop start to the device's last update end:
+                                                   when it finished (staging that overlaps its
+                                                   updates counted once)                        */
 } pmm_stats;
 
 typedef struct pmm_ctx pmm_ctx;

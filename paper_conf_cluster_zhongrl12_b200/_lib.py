@@ -53,7 +53,7 @@ class PmmStats(ctypes.Structure):
         ("per_dev_compute_s", dbl * FPM_MAX_DEVICES), ("per_dev_update_s", dbl * FPM_MAX_DEVICES),
         ("gflops", dbl), ("imbalance", dbl), ("iters", i64), ("comm_bytes", i64),
         ("kernel_launches", i64), ("updates", i64),
-        ("ooc_devices", i64), ("ooc_bytes", i64),
+        ("ooc_devices", i64), ("ooc_bytes", i64), ("per_dev_span_s", dbl * FPM_MAX_DEVICES),
     ]
 
     def as_dict(self, p: int | None = None) -> dict:
@@ -66,6 +66,7 @@ class PmmStats(ctypes.Structure):
             "gflops": self.gflops, "imbalance": self.imbalance, "iters": self.iters,
             "comm_bytes": self.comm_bytes, "kernel_launches": self.kernel_launches, "updates": self.updates,
             "ooc_devices": self.ooc_devices, "ooc_bytes": self.ooc_bytes,
+            "per_dev_span_s": list(self.per_dev_span_s[:p]),
         }
 
 

@@ -1841,10 +1841,12 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
                   int64_t launches) {
     const int ngroups = (int)ctx->groups.size();
     double t_max = 0.0, t_tail_copy = 0.0;
+    std::vector<double> span(ctx->devs.size(), 0.0);
     for (size_t i = 0; i < ctx->devs.size(); ++i) {
         Device& d = ctx->devs[i];
         if (d.cpu) {
             if (d.live()) t_max = std::max(t_max, d.cpu_loop_s);
+            if (d.live()) span[i] = d.cpu_loop_s;
             bytes += d.live() ? d.cpu_bytes : 0;
             continue;
         }
@@ -1855,6 +1857,7 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
             CU(cudaEventSynchronize(d.ev_stop));
         }
         CU(cudaStreamSynchronize(d.s_comm));
+        span[i] = d.live() ? (double)elapsed_ms(d.ev_start, d.ev_stop) * 1e-3 : 0.0;
         t_max = std::max(t_max, (double)elapsed_ms(d.ev_start, d.ev_stop) * 1e-3);
         if (tail_done && (*tail_done)[i]) {  // copy still draining after the last update
             CU(cudaEventSynchronize(d.ev_io1));
@@ -1907,6 +1910,8 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
             ++cnt;
         }
         st->imbalance = (cnt > 0 && sum > 0) ? mx / (sum / cnt) - 1.0 : 0.0;
+        for (size_t i = 0; i < ctx->devs.size(); ++i)
+            if (ctx->devs[i].idx < FPM_MAX_DEVICES) st->per_dev_span_s[ctx->devs[i].idx] = span[i];
     }
 }
 

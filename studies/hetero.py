@@ -129,6 +129,7 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
                 best = st
         areas = [r[3] * r[4] for r in rects]
         per_dev = list(best.per_dev_compute_s[:p])
+        spans = list(best.per_dev_span_s[:p])
         # FPM-predicted k-loop time: 2 a b^2 N flop at the model's speed s(a)
         pred_models = (refined[name][0] if name in refined else
                        cur_models if name.startswith("fpm_insitu") else models)
@@ -139,6 +140,7 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
             "t_total_s": best.t_compute_s, "gflops": best.gflops,
             "per_dev_compute_s": per_dev,
             "imbalance_measured": imbalance(per_dev), "imbalance_predicted": imbalance(pred),
+            "per_dev_span_s": spans, "imbalance_span": imbalance([t for t, a in zip(spans, areas) if a > 0]),
             "predicted_time_s": max(pred),
             "comm_bytes": best.comm_bytes,
         }

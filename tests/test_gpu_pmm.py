@@ -380,3 +380,21 @@ def test_sample_rects_gpu():
         assert len(sp) == 2 and sp[0][0] > sp[1][0] > 0
         with pytest.raises(pkg.FpmError):
             ctx.sample_rects(0, 512, [(0, 4)], pkg.FPM_F32)
+
+
+def test_per_device_span_stats():
+    """pmm_stats.per_dev_span_s: every live device's k-loop span is positive, at
+    most the k-loop time (its maximum), at least its summed update time; a
+    zero-area device reports 0."""
+    N, b = 2048, 256
+    n = N // b
+    rects = pkg.colpart_arrange(n, [40, 24, 0])
+    with pkg.Context.local([0, 0, 0]) as ctx:
+        ctx.setup(N, b, rects, pkg.FPM_F32)
+        ctx.fill_synthetic(1, 2, pkg.FPM_DIST_PM1)
+        st = ctx.compute()
+        for i in range(2):
+            assert 0 < st.per_dev_update_s[i] <= st.per_dev_span_s[i] * 1.001
+            assert st.per_dev_span_s[i] <= st.t_compute_s * 1.001
+        assert max(st.per_dev_span_s[:2]) == pytest.approx(st.t_compute_s, rel=1e-6)
+        assert st.per_dev_span_s[2] == 0.0
