@@ -565,9 +565,42 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             except Exception as ex:  # report, do not hide
                 log("hetero failed:", repr(ex))
                 line["hetero"] = {"error": repr(ex)[:200]}
+        if world == 1:
+            line["fig7"] = fig7_summary()
         print(json.dumps(line), flush=True)
         if parity is not None and not parity["ok"]:
             sys.exit(3)
+
+
+def fig7_summary() -> dict | None:
+    """The memory-cliff study (Table III / Fig. 7 analogue, NEXT-2) summarised
+    from its committed records (`studies/memcap.py`, several minutes of GPU
+    time: not re-run inside the bench): per layout and n, the time of each
+    partition and FPM's delta against CPM and the homogeneous split."""
+    out = {"source": "committed study records, not re-measured in this run", "layouts": {}}
+    for layout in ("sockets", "cores"):
+        path = os.path.join(ROOT, "profiles", f"memcap_fig7_r02_{layout}.json")
+        if not os.path.exists(path):
+            continue
+        d = json.load(open(path))
+        rows, ok_cpm, ok_hom = [], True, True
+        for r in d["table"]:
+            f = r.get("fpm_refined", r["fpm"])
+            row = {"n": r["n"], "fpm_s": f["t_total_s"], "fpm_static_s": r["fpm"]["t_total_s"],
+                   "cpm_s": r["cpm"]["t_total_s"], "homogeneous_s": r["homogeneous"]["t_total_s"]}
+            row["fpm_vs_cpm_pct"] = 100.0 * (row["fpm_s"] / row["cpm_s"] - 1)
+            row["fpm_vs_homogeneous_pct"] = 100.0 * (row["fpm_s"] / row["homogeneous_s"] - 1)
+            ok_cpm = ok_cpm and row["fpm_vs_cpm_pct"] <= 1.0     # within 1 % counts as a tie
+            ok_hom = ok_hom and row["fpm_vs_homogeneous_pct"] <= 1.0
+            rows.append(row)
+        out["layouts"][layout] = {
+            "file": os.path.relpath(path, ROOT), "devices": d["config"]["names"],
+            "sm_caps": d["config"]["sm_caps"], "c_cap_bytes": d["config"]["c_cap_bytes"],
+            "fpm": "cliff-bracketed FPMs with synchronised level correction (DESIGN Q26)",
+            "fpm_no_slower_than_cpm_every_n": ok_cpm, "fpm_no_slower_than_homogeneous_every_n": ok_hom,
+            "tie_tolerance_pct": 1.0,
+            "rows": rows}
+    return out if out["layouts"] else None
 
 
 def run_hetero(peak_tflops: float) -> dict:
