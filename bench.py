@@ -399,9 +399,12 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         ctx.fill_synthetic(seeds[0], seeds[1], pkg.FPM_DIST_PM1)
         barrier()
 
+    # devices sharing one GPU (c4 on one GPU): the FPM-chosen integer arrangement (Q25)
+    arrange_fpm = world == 1 and bool(caps)
+
     def plan(part_models):
         d = pkg.fpm_partition(T, part_models)
-        return d, pkg.colpart_arrange(n, d)
+        return d, (pkg.colpart_arrange_fpm(n, d, part_models) if arrange_fpm else pkg.colpart_arrange(n, d))
 
     def per_device(comp, upd, span, rects, part_models):
         """Per-device records (Fig. 6 metric): this process's devices (comp /
@@ -421,6 +424,13 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             recs = [x for rr in allr for x in rr]
         return recs
 
+    refine_hist = None
+    if arrange_fpm and not args.no_sample:
+        # devices that share one GPU share its power budget: models measured alone take the
+        # level the devices reach when all run (synchronised level correction, Q26)
+        from studies import refine as rf
+        models, refine_hist, _, _ = rf.refine(ctx, n, b, models, 3, arrange="fpm")
+        fpm_source += " + synchronised level correction (Q26)"
     d, rects = plan(models)
     install(rects)
 
@@ -549,6 +559,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 "fuse": args.fuse,
                 "update_launches_per_step": st.updates, "transport": transport,
                 "fpm_sample_s": t_sample, "fpm_sizes": sizes, "fpm_models": fpm_source,
+                "fpm_refine_rounds": len(refine_hist) if refine_hist else None,
                 "comm_bytes_per_step": comm // max(1, args.steps),
                 # share of the exchange + staging time hidden under the updates, per rank (CUDA
                 # events of each rank's streams; SURVEY §8(d) c5 "broadcast/update overlap")
@@ -620,24 +631,31 @@ def run_hetero(peak_tflops: float) -> dict:
     out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "
                         f"SM partitions {caps}; FPMs sampled per device alone (P:11), "
                         f"{len(res['config']['sizes'])} sizes"),
-           "partitions": {"fpm": "FPM partition of the exclusive size-sweep models, paper arrangement",
-                          "fpm_arr": "the same, FPM-chosen integer arrangement (Q25)",
-                          "fpm_refined_arr": "FPM after synchronised level correction at the operating point "
-                                             "(Q26), FPM-chosen integer arrangement",
+           "method": ("fpm: the FPM partition of models built by the paper's protocol -- size sweep of each "
+                      "device alone (P:18, P:11), level from the synchronised run of all devices at their "
+                      "operating points (P:10 (ii); DESIGN Q26) -- with FPM-chosen integers (Q25)"),
+           "partitions": {"fpm": "FPM, synchronised level correction (Q26), FPM-chosen integer arrangement (Q25)",
+                          "fpm_exclusive": "FPM of the exclusive size-sweep models alone, paper arrangement",
+                          "fpm_exclusive_arr": "the same, FPM-chosen integer arrangement (Q25)",
                           "cpm_ncal": "constant models at the even share of N_cal = 8192 (Q9)",
                           "cpm_self": "constant models at this run's even share",
                           "homogeneous": "equal areas",
-                          "fpm_insitu1": "models rescaled by one FPM run's own per-device times (side study)"},
+                          "fpm_insitu1": "exclusive models rescaled by one FPM run's own per-device times "
+                                         "(side study, not the method)"},
            "capped_aggregate_peak_tflops": capped_peak, "fpm_sample_s": res["fpm_sample_s"]}
+    rename = {"fpm_refined_arr": "fpm", "fpm": "fpm_exclusive", "fpm_arr": "fpm_exclusive_arr"}
     for name, r in res["partitions"].items():
-        out[name] = {"t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],
-                     "refine_rounds": len(r.get("refine_history", [])) or None,
-                     "imbalance_pct_measured": 100.0 * r["imbalance_measured"],
-                     "imbalance_pct_span": 100.0 * r.get("imbalance_span", 0.0),
-                     "imbalance_pct_predicted": 100.0 * r["imbalance_predicted"],
-                     "pct_of_capped_peak": 100.0 * r["gflops"] / 1e3 / capped_peak}
-    out["fpm_vs_cpm_time_delta_pct"] = 100.0 * res["fpm_vs_cpm_ncal_time_delta"]
-    out["fpm_vs_homogeneous_time_delta_pct"] = 100.0 * res["fpm_vs_homogeneous_time_delta"]
+        out[rename.get(name, name)] = {
+            "t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],
+            "refine_rounds": len(r.get("refine_history", [])) or None,
+            "imbalance_pct_measured": 100.0 * r["imbalance_measured"],
+            "imbalance_pct_span": 100.0 * r.get("imbalance_span", 0.0),
+            "imbalance_pct_predicted": 100.0 * r["imbalance_predicted"],
+            "pct_of_capped_peak": 100.0 * r["gflops"] / 1e3 / capped_peak}
+    if "fpm" in out and "cpm_ncal" in out:
+        out["fpm_vs_cpm_time_delta_pct"] = 100.0 * (out["fpm"]["t_s"] / out["cpm_ncal"]["t_s"] - 1)
+        out["fpm_vs_homogeneous_time_delta_pct"] = 100.0 * (out["fpm"]["t_s"] / out["homogeneous"]["t_s"] - 1)
+        out["fpm_exclusive_vs_cpm_time_delta_pct"] = 100.0 * res["fpm_vs_cpm_ncal_time_delta"]
     out["wall_s"] = time.perf_counter() - t0
     return out
 
