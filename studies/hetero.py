@@ -141,6 +141,7 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
             "per_dev_compute_s": per_dev,
             "imbalance_measured": imbalance(per_dev), "imbalance_predicted": imbalance(pred),
             "per_dev_span_s": spans, "imbalance_span": imbalance([t for t, a in zip(spans, areas) if a > 0]),
+            "per_dev_update_s": list(best.per_dev_update_s[:p]),
             "predicted_time_s": max(pred),
             "comm_bytes": best.comm_bytes,
         }
