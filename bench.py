@@ -469,6 +469,22 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         overlaps = [None] * world
         dist.all_gather_object(overlaps, overlap)
 
+    # ---- the exchange against NVLink ("NVLink bandwidth for the
+    # broadcasts"): pivot bytes this rank pulled per step over its staging time (the
+    # pulls are fused into the staging kernels, so this is a lower bound of the link rate)
+    ex = None
+    if world > 1:
+        mine_bytes = comm / max(1, args.steps)
+        rate = mine_bytes / stage / 1e9 if stage > 0 and mine_bytes > 0 else None
+        rates = [None] * world
+        dist.all_gather_object(rates, rate)
+        peer = "same GPU (--same-gpu): HBM, not NVLink" if args.same_gpu else "NVLink 5, 900 GB/s per direction"
+        valid = [r for r in rates if r]
+        ex = {"bound": "nvlink", "unit": "GB/s", "peak": 900.0, "peak_basis": "B200 NVLink 5 nominal per direction "
+              "(/opt/skills/guides/B200_PROFILING.md)", "achieved_per_rank": rates,
+              "achieved": max(valid) if valid else None, "frac": (max(valid) / 900.0) if valid else None,
+              "path": peer, "what": "pivot bytes pulled per step / the rank's staging time (pull fused into the split)"}
+
     # ---- roofline of the dominant kernel (rank-(f b) update): algorithmic flops
     # 2 H W b n of the busiest device over its summed update time (CUDA events on its stream)
     peaks = measured_peaks()
@@ -564,6 +580,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 # share of the exchange + staging time hidden under the updates, per rank (CUDA
                 # events of each rank's streams; SURVEY §8(d) c5 "broadcast/update overlap")
                 "exchange_staging_overlap": overlaps[0] if world == 1 else overlaps,
+                "exchange_roofline": ex,
                 "wall_s_timed_region": wall,
                 "partitions": partitions,
             })

@@ -53,6 +53,9 @@ def test_two_ranks_same_gpu_line(config, N, b):
     assert isinstance(c["exchange_staging_overlap"], list) and len(c["exchange_staging_overlap"]) == 2
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 2 * N * N * 4
     assert d["roofline"]["frac"] > 0 and d["gpu_launches"] > 0 and d["cpu_baseline"] is None
+    ex = c["exchange_roofline"]
+    assert ex["bound"] == "nvlink" and ex["peak"] == 900.0 and len(ex["achieved_per_rank"]) == 2
+    assert ex["achieved"] > 0 and "same GPU" in ex["path"]
     if config == "c4":
         assert [x["sm_cap"] for x in c["per_device"]] == [144, 128]
         parts = c["partitions"]
