@@ -187,8 +187,11 @@ int colpart_plan_step(int64_t n, int32_t p, const colpart_rect* rects, int64_t k
  * streams, pulling pivots held by GPU devices device -> host one update group
  * ahead.  A CPU device is a device of the partition chosen by the caller,
  * never a fallback: GPU devices' updates always run on their GPUs.  Contexts
- * with only CPU devices need no GPU.  Not available in NCCL / IPC contexts;
- * fpm_sample(dev = -1) is FPM_EUNSUPPORTED with CPU devices (sample each).
+ * with only CPU devices need no GPU.  Not available in NCCL / IPC contexts.
+ * fpm_sample(dev = -1) on a context with CPU devices runs every device on a
+ * host thread of its own, all repetitions in step: each device runs its kernel
+ * for the same wall-clock window (>= 4 runs of the slowest) and its speed is
+ * its completed runs over that time (P:10 (ii) synchronised measurement).
  * Errors: FPM_EINVAL, FPM_ECUDA, FPM_EUNSUPPORTED (SM cap or cores not
  * available). */
 #define FPM_CPU_DEVICE (-1)

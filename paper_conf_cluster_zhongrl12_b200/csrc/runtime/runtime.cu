@@ -20,7 +20,9 @@
 #include <cstdlib>
 #include <cstring>
 #include <exception>
+#include <condition_variable>
 #include <memory>
+#include <mutex>
 #include <string>
 #include <thread>
 #include <vector>
@@ -2083,68 +2085,220 @@ struct Shape {
     int64_t h, w;
 };
 
-// Speed function of a CPU device: its kernel C (h b x w b) += A (h b x f b) B
-// (f b x w b) -- the k-loop's fused update -- run by all c cores of the device
-// at once, each on h b / c rows ("the speed of a socket executing the ACML
-// kernels simultaneously on c cores, with the problem size x / c on each
-// core"; P:10 (ii) synchronised cores), host-timed (the synchronous approach,
-// P:10), repeated under the same statistical stop rule as the GPU devices (Q8).
+// One CPU device's sampling kernel: C (h b x w b) += A (h b x f b) B (f b x w b)
+// -- the k-loop's fused update -- on all c cores of the device at once, each on
+// h b / c rows ("the speed of a socket executing the ACML kernels
+// simultaneously on c cores, with the problem size x / c on each core"
+// (ii) synchronised cores), host-timed (the synchronous approach).
+struct CpuRunner {
+    Device* d;
+    fpm_dtype dt;
+    int64_t b, fb, Hm = 0, Wm = 0;
+    void *A = nullptr, *B = nullptr, *C = nullptr;
+    CpuRunner(pmm_ctx* ctx, Device* dev, fpm_dtype dt_, int64_t b_, const std::vector<Shape>& shp)
+        : d(dev), dt(dt_), b(b_), fb((int64_t)fuse_factor(ctx, dt_, b_) * b_) {
+        int64_t area = 0;
+        for (const Shape& x : shp) {
+            Hm = std::max(Hm, x.h * b);
+            Wm = std::max(Wm, x.w * b);
+            area = std::max(area, x.h * x.w * b * b);
+        }
+        const size_t es = esize(dt);
+        auto get = [&](void*& p, size_t bytes) {
+            if (posix_memalign(&p, 64, std::max<size_t>(bytes, 64)) != 0) fail(FPM_ENOMEM, "host allocation failed");
+        };
+        get(A, (size_t)Hm * fb * es);
+        get(B, (size_t)fb * Wm * es);
+        get(C, (size_t)area * es);
+        cpu::fill_synthetic(d->team, A, dt == FPM_F64, fb, 101, std::max(Hm, Wm), 0, 0, Hm, fb, FPM_DIST_PM1);
+        cpu::fill_synthetic(d->team, B, dt == FPM_F64, Wm, 102, std::max(Hm, Wm), 0, 0, fb, Wm, FPM_DIST_PM1);
+        std::memset(C, 0, (size_t)area * es);
+    }
+    ~CpuRunner() {
+        std::free(A);
+        std::free(B);
+        std::free(C);
+    }
+    double flops(const Shape& x) const { return 2.0 * (double)(x.h * x.w) * (double)b * (double)b * (double)fb; }
+    // one run, completed on return
+    void run(const Shape& x) {
+        const int64_t Mx = x.h * b, Nx = x.w * b;
+        if (dt == FPM_F32)
+            cpu::gemm_f32(d->team, Mx, Nx, fb, static_cast<const float*>(A), fb, fb, 0, static_cast<const float*>(B),
+                          Wm, static_cast<float*>(C), Nx, true);
+        else
+            cpu::gemm_f64(d->team, Mx, Nx, fb, static_cast<const double*>(A), fb, fb, 0,
+                          static_cast<const double*>(B), Wm, static_cast<double*>(C), Nx, true);
+    }
+};
+
+// One GPU device's sampling kernel, as the k-loop runs it: staging (split /
+// transpose) of an f-pivot group and the fused rank-(f b) update on an h b x w b
+// C; shapes whose C exceeds the device's C cap run out of core through the band
+// ring in the k-loop's steady state (bands kept, order reversed).
+struct GpuRunner {
+    pmm_ctx* ctx;
+    Device* d;
+    fpm_dtype dt;
+    int64_t b, fb;
+    size_t es, op;
+    SplitScheme sch;
+    Device mem;          // owns the allocations (and the band pipeline of out-of-core sizes)
+    char* hC = nullptr;  // pinned host C for sizes above the device's C cap
+    void *C = nullptr, *Ap = nullptr, *Bp = nullptr, *Bt = nullptr;
+    void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
+    float *sa = nullptr, *sb = nullptr;
+    int64_t Hm = 0, Wm = 0;  // largest rows / columns of C over this device's shapes
+    int runs = 0;            // runs at the current size (out-of-core band order alternates)
+
+    bool ooc_at(int64_t Mx, int64_t Nx) const { return d->c_cap > 0 && (int64_t)(Mx * Nx * es) > d->c_cap; }
+    Ring ring_at(int64_t Mx, int64_t Nx) const { return ring_for(d->c_cap, Mx, Nx, es, ctx->ooc_buffers); }
+    double flops(const Shape& x) const { return 2.0 * (double)(x.h * x.w) * (double)b * (double)b * (double)fb; }
+
+    GpuRunner(pmm_ctx* c, Device* dev, fpm_dtype dt_, int64_t b_, const std::vector<Shape>& shp)
+        : ctx(c), d(dev), dt(dt_), b(b_), fb((int64_t)fuse_factor(c, dt_, b_) * b_), es(dt_ == FPM_F64 ? 8 : 4),
+          op(op_bytes(scheme_for(c, b_))), sch(scheme_for(c, b_)) {
+        mem.cuda_dev = d->cuda_dev;
+        CU(cudaSetDevice(d->cuda_dev));
+        int64_t in_area = 0, out_area = 0, nbands = 0;
+        size_t band_bytes = 0;
+        for (const Shape& x : shp) {
+            const int64_t Mx = x.h * b, Nx = x.w * b;
+            Hm = std::max(Hm, Mx);
+            Wm = std::max(Wm, Nx);
+            if (!ooc_at(Mx, Nx)) {
+                in_area = std::max(in_area, Mx * Nx);
+                continue;
+            }
+            out_area = std::max(out_area, Mx * Nx);
+            const int64_t rows = ring_at(Mx, Nx).rows;
+            nbands = std::max(nbands, (Mx + rows - 1) / rows);
+            band_bytes = std::max(band_bytes, (size_t)rows * Nx * es);
+        }
+        C = dalloc(mem, (size_t)in_area * es);
+        if (out_area > 0) {
+            bp_init(mem.bp);
+            hC = static_cast<char*>(halloc(mem, (size_t)out_area * es));
+            std::memset(hC, 0, (size_t)out_area * es);
+            bp_alloc_bands(mem, mem.bp, ctx->ooc_buffers, band_bytes, nbands);
+        }
+        const int64_t L = std::max(Hm, Wm);
+        Ap = dalloc(mem, (size_t)Hm * fb * es);
+        Bp = dalloc(mem, (size_t)fb * Wm * es);
+        Bt = dalloc(mem, (size_t)Wm * fb * es);
+        if (dt == FPM_F32) {
+            ah = dalloc(mem, (size_t)Hm * fb * op);
+            al = dalloc(mem, (size_t)Hm * fb * op);
+            bh = dalloc(mem, (size_t)Wm * fb * op);
+            bl = dalloc(mem, (size_t)Wm * fb * op);
+            sa = static_cast<float*>(dalloc(mem, (size_t)Hm * 4));
+            sb = static_cast<float*>(dalloc(mem, (size_t)Wm * 4));
+        }
+        launch_fill_synthetic(Ap, dt == FPM_F64, fb, 101, L, 0, 0, Hm, fb, FPM_DIST_PM1, d->s_comp);
+        launch_fill_synthetic(Bp, dt == FPM_F64, Wm, 102, L, 0, 0, fb, Wm, FPM_DIST_PM1, d->s_comp);
+        if (C) CU(cudaMemsetAsync(C, 0, (size_t)in_area * es, d->s_comp));
+    }
+    ~GpuRunner() {
+        free_problem(mem);
+        bp_destroy(mem.bp);
+    }
+
+    // enqueue one run on the device's compute stream
+    void run(const Shape& x) {
+        const int64_t Mx = x.h * b, Nx = x.w * b;
+        const cudaStream_t st = d->s_comp;
+        const bool ooc = ooc_at(Mx, Nx);
+        BandCall bc;
+        bc.reverse = ctx->ooc_keep && (runs & 1);
+        bc.kept_head = ctx->ooc_keep && runs > 0;
+        bc.keep_tail = ctx->ooc_keep;
+        ++runs;
+        if (dt == FPM_F32) {
+            launch_split_rows(static_cast<const float*>(Ap), fb, Mx, fb, sch, ah, al, sa, st);
+            launch_split_cols(static_cast<const float*>(Bp), Wm, fb, Nx, sch, bh, bl, sb, st);
+            UpdateArgs a;
+            a.a_hi = ah; a.a_lo = al; a.bt_hi = bh; a.bt_lo = bl;
+            a.sa = has_scales(sch) ? sa : nullptr;
+            a.sb = has_scales(sch) ? sb : nullptr;
+            a.C = static_cast<float*>(C);
+            a.M = Mx; a.Nc = Nx; a.K = fb; a.ldc = Nx;
+            a.scheme = sch;
+            a.cta_group = ctx->cta_group;
+            a.num_sms = d->num_sms;
+            a.raster_group = raster_group_for(ctx, *d, sch);
+            a.l2_hint_b = ctx->l2_hint_b;
+            a.variant = ctx->kernel_variant;
+            a.chunk_k = ctx->chunk_k;
+            a.raster_snake = ctx->raster_snake != 0;
+            if (ooc) {
+                banded_update(mem.bp, ring_at(Mx, Nx), hC, Mx, (size_t)Nx * 4, bc, st,
+                              [&](int64_t r0, int64_t m, void* band) {
+                                  UpdateArgs y = a;
+                                  y.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
+                                  y.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * fb * op;
+                                  y.sa = a.sa ? a.sa + r0 : nullptr;
+                                  y.C = static_cast<float*>(band);
+                                  y.M = m;
+                                  launch_update_f32(y, st);
+                              });
+            } else {
+                launch_update_f32(a, st);
+            }
+        } else {  // FP64: the fused update of the k-loop (K = f b, A rows contiguous here)
+            launch_transpose_f64(static_cast<const double*>(Bp), Wm, fb, Nx, static_cast<double*>(Bt), st);
+            if (ooc) {
+                banded_update(mem.bp, ring_at(Mx, Nx), hC, Mx, (size_t)Nx * 8, bc, st,
+                              [&](int64_t r0, int64_t m, void* band) {
+                                  launch_update_f64(static_cast<const double*>(Ap) + (size_t)r0 * fb, fb,
+                                                    static_cast<const double*>(Bt), static_cast<double*>(band), m,
+                                                    Nx, fb, Nx, true, d->num_sms, st);
+                              });
+            } else {
+                launch_update_f64(static_cast<const double*>(Ap), fb, static_cast<const double*>(Bt),
+                                  static_cast<double*>(C), Mx, Nx, fb, Nx, true, d->num_sms, st);
+            }
+        }
+        if (ooc) bp_join(mem.bp, st);  // the update is done when C is back in host memory
+    }
+};
+
+// Q8's stop rule over repetition times: (mean, 95 % half-width, converged).
+struct RepStats {
+    std::vector<double> ts;
+    double mean = 0.0, half = 0.0;
+    bool add(double t) {
+        ts.push_back(t);
+        const int nr = (int)ts.size();
+        mean = 0.0;
+        for (double v : ts) mean += v;
+        mean /= nr;
+        double var = 0.0;
+        for (double v : ts) var += (v - mean) * (v - mean);
+        var = nr > 1 ? var / (nr - 1) : 0.0;
+        half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
+        return nr >= 5 && half <= 0.025 * mean;
+    }
+};
+
+// Speed function of a CPU device alone, repeated under the stop rule (Q8).
 void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vector<Shape>& shp, double* speeds,
                 double* ci, int32_t* reps_out) {
     using clk = std::chrono::steady_clock;
-    const int64_t fb = (int64_t)fuse_factor(ctx, dt, b) * b;
-    int64_t Hm = 0, Wm = 0, area = 0;
-    for (const Shape& x : shp) {
-        Hm = std::max(Hm, x.h * b);
-        Wm = std::max(Wm, x.w * b);
-        area = std::max(area, x.h * x.w * b * b);
-    }
-    const size_t es = esize(dt);
-    struct Buf {
-        void* p = nullptr;
-        ~Buf() { std::free(p); }
-    } A, B, C;
-    auto get = [&](Buf& x, size_t bytes) {
-        if (posix_memalign(&x.p, 64, std::max<size_t>(bytes, 64)) != 0) fail(FPM_ENOMEM, "host allocation failed");
-    };
-    get(A, (size_t)Hm * fb * es);
-    get(B, (size_t)fb * Wm * es);
-    get(C, (size_t)area * es);
-    cpu::fill_synthetic(d.team, A.p, dt == FPM_F64, fb, 101, std::max(Hm, Wm), 0, 0, Hm, fb, FPM_DIST_PM1);
-    cpu::fill_synthetic(d.team, B.p, dt == FPM_F64, Wm, 102, std::max(Hm, Wm), 0, 0, fb, Wm, FPM_DIST_PM1);
-    std::memset(C.p, 0, (size_t)area * es);
+    CpuRunner R(ctx, &d, dt, b, shp);
     for (size_t j = 0; j < shp.size(); ++j) {
-        const int64_t Mx = shp[j].h * b, Nx = shp[j].w * b;
         auto run = [&] {
             const auto t0 = clk::now();
-            if (dt == FPM_F32)
-                cpu::gemm_f32(d.team, Mx, Nx, fb, static_cast<const float*>(A.p), fb, fb, 0,
-                              static_cast<const float*>(B.p), Wm, static_cast<float*>(C.p), Nx, true);
-            else
-                cpu::gemm_f64(d.team, Mx, Nx, fb, static_cast<const double*>(A.p), fb, fb, 0,
-                              static_cast<const double*>(B.p), Wm, static_cast<double*>(C.p), Nx, true);
+            R.run(shp[j]);
             return std::chrono::duration<double>(clk::now() - t0).count();
         };
         run();
         run();  // two warm-ups
-        std::vector<double> ts;
-        double mean = 0.0, half = 0.0;
-        for (int r = 0; r < 50; ++r) {
-            ts.push_back(run());
-            const int nr = (int)ts.size();
-            mean = 0.0;
-            for (double t : ts) mean += t;
-            mean /= nr;
-            double var = 0.0;
-            for (double t : ts) var += (t - mean) * (t - mean);
-            var = nr > 1 ? var / (nr - 1) : 0.0;
-            half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
-            if (nr >= 5 && half <= 0.025 * mean) break;
-        }
-        const double x = (double)(shp[j].h * shp[j].w);
-        speeds[j] = 2.0 * x * (double)b * (double)b * (double)fb / mean;
-        if (ci) ci[j] = mean > 0 ? half / mean : 0.0;
-        if (reps_out) reps_out[j] = (int32_t)ts.size();
+        RepStats st;
+        for (int r = 0; r < 50; ++r)
+            if (st.add(run())) break;
+        speeds[j] = R.flops(shp[j]) / st.mean;
+        if (ci) ci[j] = st.mean > 0 ? st.half / st.mean : 0.0;
+        if (reps_out) reps_out[j] = (int32_t)st.ts.size();
     }
 }
 
@@ -2152,162 +2306,39 @@ void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vec
 void sample_gpu(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vector<std::vector<Shape>>& shapes,
                 fpm_dtype dt, int64_t b, double* speeds, double* ci, int32_t* reps_out) {
     const int nsizes = (int)shapes[0].size();
-    const size_t es = dt == FPM_F64 ? 8 : 4;
-    const SplitScheme sch = scheme_for(ctx, b);
-    const size_t op = op_bytes(sch);
-    // the kernel as the k-loop runs it: f fused pivots per update (K = f b)
-    const int f = fuse_factor(ctx, dt, b);
-    const int64_t fb = (int64_t)f * b;
-
     struct Scratch {
-        Device* d = nullptr;
-        Device mem;  // owns the allocations (and the band pipeline of out-of-core sizes)
-        char* hC = nullptr;  // pinned host C for sizes above the device's C cap
-        void *C = nullptr, *Ap = nullptr, *Bp = nullptr, *Bt = nullptr;
-        void *ah = nullptr, *al = nullptr, *bh = nullptr, *bl = nullptr;
-        float *sa = nullptr, *sb = nullptr;
-        int64_t Hm = 0, Wm = 0;  // largest rows / columns of C over this device's shapes
+        std::unique_ptr<GpuRunner> R;
         cudaEvent_t e0 = nullptr, e1 = nullptr;
-        std::vector<double> ts;
-        int runs = 0;  // runs at the current size (out-of-core band order alternates)
+        RepStats st;
         int k = 1;            // kernel runs per timed repetition (concurrent sampling)
         double t_warm = 0.0;  // last warm-up run
-        double mean = 0.0, half = 0.0;
         bool done = false;
         ~Scratch() {
-            free_problem(mem);
-            bp_destroy(mem.bp);
             if (e0) cudaEventDestroy(e0);
             if (e1) cudaEventDestroy(e1);
         }
     };
-    // shapes whose C exceeds the device's C cap run out of core (as in the k-loop)
-    auto ooc_at = [&](const Device* d, int64_t Mx, int64_t Nx) {
-        return d->c_cap > 0 && (int64_t)(Mx * Nx * es) > d->c_cap;
-    };
-    auto ring_at = [&](const Device* d, int64_t Mx, int64_t Nx) {
-        return ring_for(d->c_cap, Mx, Nx, es, ctx->ooc_buffers);
-    };
     std::vector<std::unique_ptr<Scratch>> S;
     for (size_t i = 0; i < devs.size(); ++i) {
-        Device* d = devs[i];
         S.emplace_back(new Scratch);
         Scratch& s = *S.back();
-        s.d = d;
-        s.mem.cuda_dev = d->cuda_dev;
-        CU(cudaSetDevice(d->cuda_dev));
-        int64_t in_area = 0, out_area = 0, nbands = 0;
-        size_t band_bytes = 0;
-        for (const Shape& x : shapes[i]) {
-            const int64_t Mx = x.h * b, Nx = x.w * b;
-            s.Hm = std::max(s.Hm, Mx);
-            s.Wm = std::max(s.Wm, Nx);
-            if (!ooc_at(d, Mx, Nx)) {
-                in_area = std::max(in_area, Mx * Nx);
-                continue;
-            }
-            out_area = std::max(out_area, Mx * Nx);
-            const int64_t rows = ring_at(d, Mx, Nx).rows;
-            nbands = std::max(nbands, (Mx + rows - 1) / rows);
-            band_bytes = std::max(band_bytes, (size_t)rows * Nx * es);
-        }
-        s.C = dalloc(s.mem, (size_t)in_area * es);
-        if (out_area > 0) {
-            bp_init(s.mem.bp);
-            s.hC = static_cast<char*>(halloc(s.mem, (size_t)out_area * es));
-            std::memset(s.hC, 0, (size_t)out_area * es);
-            bp_alloc_bands(s.mem, s.mem.bp, ctx->ooc_buffers, band_bytes, nbands);
-        }
-        const int64_t L = std::max(s.Hm, s.Wm);
-        s.Ap = dalloc(s.mem, (size_t)s.Hm * fb * es);
-        s.Bp = dalloc(s.mem, (size_t)fb * s.Wm * es);
-        s.Bt = dalloc(s.mem, (size_t)s.Wm * fb * es);
-        if (dt == FPM_F32) {
-            s.ah = dalloc(s.mem, (size_t)s.Hm * fb * op);
-            s.al = dalloc(s.mem, (size_t)s.Hm * fb * op);
-            s.bh = dalloc(s.mem, (size_t)s.Wm * fb * op);
-            s.bl = dalloc(s.mem, (size_t)s.Wm * fb * op);
-            s.sa = static_cast<float*>(dalloc(s.mem, (size_t)s.Hm * 4));
-            s.sb = static_cast<float*>(dalloc(s.mem, (size_t)s.Wm * 4));
-        }
+        s.R.reset(new GpuRunner(ctx, devs[i], dt, b, shapes[i]));
         CU(cudaEventCreate(&s.e0));
         CU(cudaEventCreate(&s.e1));
-        launch_fill_synthetic(s.Ap, dt == FPM_F64, fb, 101, L, 0, 0, s.Hm, fb, FPM_DIST_PM1, d->s_comp);
-        launch_fill_synthetic(s.Bp, dt == FPM_F64, s.Wm, 102, L, 0, 0, fb, s.Wm, FPM_DIST_PM1, d->s_comp);
-        if (s.C) CU(cudaMemsetAsync(s.C, 0, (size_t)in_area * es, d->s_comp));
     }
-
     for (int j = 0; j < nsizes; ++j) {
-        auto run = [&](Scratch& s, const Shape& x) {
-            const int64_t Mx = x.h * b, Nx = x.w * b;
-            const cudaStream_t st = s.d->s_comp;
-            const bool ooc = ooc_at(s.d, Mx, Nx);
-            // out of core: the k-loop's steady state (bands kept and order reversed
-            // between consecutive updates)
-            BandCall bc;
-            bc.reverse = ctx->ooc_keep && (s.runs & 1);
-            bc.kept_head = ctx->ooc_keep && s.runs > 0;
-            bc.keep_tail = ctx->ooc_keep;
-            ++s.runs;
-            if (dt == FPM_F32) {
-                launch_split_rows(static_cast<const float*>(s.Ap), fb, Mx, fb, sch, s.ah, s.al, s.sa, st);
-                launch_split_cols(static_cast<const float*>(s.Bp), s.Wm, fb, Nx, sch, s.bh, s.bl, s.sb, st);
-                UpdateArgs a;
-                a.a_hi = s.ah; a.a_lo = s.al; a.bt_hi = s.bh; a.bt_lo = s.bl;
-                a.sa = has_scales(sch) ? s.sa : nullptr;
-                a.sb = has_scales(sch) ? s.sb : nullptr;
-                a.C = static_cast<float*>(s.C);
-                a.M = Mx; a.Nc = Nx; a.K = fb; a.ldc = Nx;
-                a.scheme = sch;
-                a.cta_group = ctx->cta_group;
-                a.num_sms = s.d->num_sms;
-                a.raster_group = raster_group_for(ctx, *s.d, sch);
-                a.l2_hint_b = ctx->l2_hint_b;
-                a.variant = ctx->kernel_variant;
-                a.chunk_k = ctx->chunk_k;
-                a.raster_snake = ctx->raster_snake != 0;
-                if (ooc) {
-                    banded_update(s.mem.bp, ring_at(s.d, Mx, Nx), s.hC, Mx, (size_t)Nx * 4, bc, st,
-                                  [&](int64_t r0, int64_t m, void* band) {
-                                      UpdateArgs y = a;
-                                      y.a_hi = static_cast<const char*>(a.a_hi) + (size_t)r0 * fb * op;
-                                      y.a_lo = static_cast<const char*>(a.a_lo) + (size_t)r0 * fb * op;
-                                      y.sa = a.sa ? a.sa + r0 : nullptr;
-                                      y.C = static_cast<float*>(band);
-                                      y.M = m;
-                                      launch_update_f32(y, st);
-                                  });
-                } else {
-                    launch_update_f32(a, st);
-                }
-            } else {  // FP64: the fused update of the k-loop (K = f b, A rows contiguous here)
-                launch_transpose_f64(static_cast<const double*>(s.Bp), s.Wm, fb, Nx, static_cast<double*>(s.Bt), st);
-                if (ooc) {
-                    banded_update(s.mem.bp, ring_at(s.d, Mx, Nx), s.hC, Mx, (size_t)Nx * 8, bc, st,
-                                  [&](int64_t r0, int64_t m, void* band) {
-                                      launch_update_f64(static_cast<const double*>(s.Ap) + (size_t)r0 * fb, fb,
-                                                        static_cast<const double*>(s.Bt), static_cast<double*>(band),
-                                                        m, Nx, fb, Nx, true, s.d->num_sms, st);
-                                  });
-                } else {
-                    launch_update_f64(static_cast<const double*>(s.Ap), fb, static_cast<const double*>(s.Bt),
-                                      static_cast<double*>(s.C), Mx, Nx, fb, Nx, true, s.d->num_sms, st);
-                }
-            }
-            if (ooc) bp_join(s.mem.bp, st);  // the update is done when C is back in host memory
-        };
         for (auto& sp : S) {
-            sp->ts.clear();
+            sp->st = RepStats{};
             sp->done = false;
-            sp->runs = 0;
+            sp->R->runs = 0;
         }
         for (int w = 0; w < 2; ++w)
             for (size_t i = 0; i < S.size(); ++i) {
                 Scratch& sp = *S[i];
-                CU(cudaSetDevice(sp.d->cuda_dev));
-                CU(cudaEventRecord(sp.e0, sp.d->s_comp));
-                run(sp, shapes[i][j]);
-                CU(cudaEventRecord(sp.e1, sp.d->s_comp));
+                CU(cudaSetDevice(sp.R->d->cuda_dev));
+                CU(cudaEventRecord(sp.e0, sp.R->d->s_comp));
+                sp.R->run(shapes[i][j]);
+                CU(cudaEventRecord(sp.e1, sp.R->d->s_comp));
             }
         // Concurrent sampling: every device must stay busy for the whole window
         // (P:10 (ii): resources "shared between the maximum number of
@@ -2315,7 +2346,7 @@ void sample_gpu(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vecto
         // times per repetition and each run is timed as the window / k.
         double t_max = 0.0;
         for (auto& sp : S) {
-            CU(cudaSetDevice(sp->d->cuda_dev));
+            CU(cudaSetDevice(sp->R->d->cuda_dev));
             CU(cudaEventSynchronize(sp->e1));
             sp->t_warm = elapsed_ms(sp->e0, sp->e1) * 1e-3;
             t_max = std::max(t_max, sp->t_warm);
@@ -2327,37 +2358,137 @@ void sample_gpu(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vecto
             // all devices run every repetition, so contention stays the same until the last converges
             for (size_t i = 0; i < S.size(); ++i) {
                 Scratch& sp = *S[i];
-                CU(cudaSetDevice(sp.d->cuda_dev));
-                CU(cudaEventRecord(sp.e0, sp.d->s_comp));
-                for (int q = 0; q < sp.k; ++q) run(sp, shapes[i][j]);
-                CU(cudaEventRecord(sp.e1, sp.d->s_comp));
+                CU(cudaSetDevice(sp.R->d->cuda_dev));
+                CU(cudaEventRecord(sp.e0, sp.R->d->s_comp));
+                for (int q = 0; q < sp.k; ++q) sp.R->run(shapes[i][j]);
+                CU(cudaEventRecord(sp.e1, sp.R->d->s_comp));
             }
             bool all_done = true;
             for (auto& sp : S) {
-                Scratch& s = *sp;
-                CU(cudaSetDevice(s.d->cuda_dev));
-                CU(cudaEventSynchronize(s.e1));
-                s.ts.push_back(elapsed_ms(s.e0, s.e1) * 1e-3 / s.k);
-                const int nr = (int)s.ts.size();
-                s.mean = 0.0;
-                for (double t : s.ts) s.mean += t;
-                s.mean /= nr;
-                double var = 0.0;
-                for (double t : s.ts) var += (t - s.mean) * (t - s.mean);
-                var = nr > 1 ? var / (nr - 1) : 0.0;
-                s.half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
-                s.done = nr >= 5 && s.half <= 0.025 * s.mean;
-                all_done = all_done && s.done;
+                CU(cudaSetDevice(sp->R->d->cuda_dev));
+                CU(cudaEventSynchronize(sp->e1));
+                sp->done = sp->st.add(elapsed_ms(sp->e0, sp->e1) * 1e-3 / sp->k);
+                all_done = all_done && sp->done;
             }
             if (all_done) break;
         }
         for (size_t i = 0; i < S.size(); ++i) {
             const Scratch& s = *S[i];
             // one timed run = f pivots of the x-block kernel: 2 x b^3 f flop
-            const double x = (double)(shapes[i][j].h * shapes[i][j].w);
-            speeds[i * nsizes + j] = 2.0 * x * (double)b * (double)b * (double)fb / s.mean;
-            if (ci) ci[i * nsizes + j] = s.mean > 0 ? s.half / s.mean : 0.0;
-            if (reps_out) reps_out[i * nsizes + j] = (int32_t)s.ts.size();
+            speeds[i * nsizes + j] = s.R->flops(shapes[i][j]) / s.st.mean;
+            if (ci) ci[i * nsizes + j] = s.st.mean > 0 ? s.st.half / s.st.mean : 0.0;
+            if (reps_out) reps_out[i * nsizes + j] = (int32_t)s.st.ts.size();
+        }
+    }
+}
+
+// Synchronised sampling of a context with CPU devices (dev = -1; P:10 (ii)):
+// every device -- GPU or CPU -- runs on a host thread of its own, all start each
+// repetition together at a barrier and keep running their kernel for the same
+// wall-clock window (long enough for >= 4 runs of the slowest); a device's
+// speed is its completed runs' flops over their time.  Repetitions follow Q8.
+void sample_sync(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vector<std::vector<Shape>>& shapes,
+                 fpm_dtype dt, int64_t b, double* speeds, double* ci, int32_t* reps_out) {
+    using clk = std::chrono::steady_clock;
+    const int nsizes = (int)shapes[0].size();
+    const size_t P = devs.size();
+    std::vector<std::unique_ptr<GpuRunner>> G(P);
+    std::vector<std::unique_ptr<CpuRunner>> Cr(P);
+    for (size_t i = 0; i < P; ++i) {
+        if (devs[i]->cpu) Cr[i].reset(new CpuRunner(ctx, devs[i], dt, b, shapes[i]));
+        else G[i].reset(new GpuRunner(ctx, devs[i], dt, b, shapes[i]));
+    }
+    for (size_t i = 0; i < P; ++i)
+        if (G[i]) {
+            CU(cudaSetDevice(devs[i]->cuda_dev));
+            CU(cudaStreamSynchronize(devs[i]->s_comp));
+        }
+    // one run, completed on return (GPU: enqueue and wait for its stream)
+    auto run_once = [&](size_t i, const Shape& x) {
+        if (Cr[i]) {
+            Cr[i]->run(x);
+        } else {
+            CU(cudaSetDevice(devs[i]->cuda_dev));
+            G[i]->run(x);
+            CU(cudaStreamSynchronize(devs[i]->s_comp));
+        }
+    };
+    auto flops = [&](size_t i, const Shape& x) { return Cr[i] ? Cr[i]->flops(x) : G[i]->flops(x); };
+    for (int j = 0; j < nsizes; ++j) {
+        std::vector<RepStats> st(P);
+        std::vector<double> t_run(P, 0.0), rate(P, 0.0);
+        std::vector<std::exception_ptr> errs(P);
+        double window = 0.0;
+        for (size_t i = 0; i < P; ++i)
+            if (G[i]) G[i]->runs = 0;
+        // phase 0: warm-ups (each device alone, then the window from the slowest)
+        for (size_t i = 0; i < P; ++i) {
+            run_once(i, shapes[i][j]);
+            const auto t0 = clk::now();
+            run_once(i, shapes[i][j]);
+            t_run[i] = std::chrono::duration<double>(clk::now() - t0).count();
+            window = std::max(window, 4.0 * t_run[i]);
+        }
+        window = std::max(window, 0.02);
+        bool stop = false;
+        std::mutex mu;
+        std::condition_variable cv;
+        int arrived = 0;
+        uint64_t gen = 0;
+        auto barrier = [&] {
+            std::unique_lock<std::mutex> lk(mu);
+            const uint64_t g = gen;
+            if (++arrived == (int)P) {
+                arrived = 0;
+                ++gen;
+                cv.notify_all();
+            } else {
+                cv.wait(lk, [&] { return gen != g; });
+            }
+        };
+        std::vector<std::thread> th;
+        std::vector<char> failed(P, 0);
+        for (size_t i = 0; i < P; ++i)
+            th.emplace_back([&, i] {
+                // a failing device keeps arriving at the barriers (nobody waits forever)
+                for (int r = 0; r < 50; ++r) {
+                    barrier();                               // everyone starts the window together
+                    if (!failed[i]) {
+                        try {
+                            const auto t0 = clk::now();
+                            int runs = 0;
+                            double t_done = 0.0;
+                            do {
+                                run_once(i, shapes[i][j]);
+                                ++runs;
+                                t_done = std::chrono::duration<double>(clk::now() - t0).count();
+                            } while (t_done < window);
+                            rate[i] = (double)runs / t_done;  // runs per second
+                        } catch (...) {
+                            errs[i] = std::current_exception();
+                            failed[i] = 1;
+                        }
+                    }
+                    barrier();                               // window over for everyone
+                    if (i == 0) {
+                        bool all = true, bad = false;
+                        for (size_t q = 0; q < P; ++q) {
+                            bad = bad || failed[q];
+                            if (!failed[q]) all = st[q].add(1.0 / rate[q]) && all;
+                        }
+                        stop = all || bad;
+                    }
+                    barrier();
+                    if (stop) break;
+                }
+            });
+        for (auto& t : th) t.join();
+        for (auto& e : errs)
+            if (e) std::rethrow_exception(e);
+        for (size_t i = 0; i < P; ++i) {
+            speeds[i * nsizes + j] = flops(i, shapes[i][j]) / st[i].mean;
+            if (ci) ci[i * nsizes + j] = st[i].mean > 0 ? st[i].half / st[i].mean : 0.0;
+            if (reps_out) reps_out[i * nsizes + j] = (int32_t)st[i].ts.size();
         }
     }
 }
@@ -2373,10 +2504,11 @@ void sample_shapes(pmm_ctx* ctx, int dev, fpm_dtype dt, int64_t b, const std::ve
         for (const Shape& x : v) FPM_CHECK_ARG(x.h >= 1 && x.w >= 1, "shape %lld x %lld", (long long)x.h, (long long)x.w);
     std::vector<Device*> devs;
     if (dev == -1) {
-        if (has_cpu(ctx))
-            fail(FPM_EUNSUPPORTED, "concurrent sampling (dev = -1) of a context with CPU devices: sample each "
-                                   "device (P:11: GPUs and sockets were measured separately)");
         for (auto& d : ctx->devs) devs.push_back(&d);
+        if (has_cpu(ctx)) {  // host threads for every device, windows in step (P:10 (ii))
+            FPM_CHECK_ARG(shapes.size() == devs.size(), "expected shapes for %zu devices", devs.size());
+            return sample_sync(ctx, devs, shapes, dt, b, speeds, ci, reps_out);
+        }
     } else {
         Device* d = local_dev(ctx, dev);
         FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this context", dev);

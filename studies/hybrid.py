@@ -62,6 +62,8 @@ def main():
     ap.add_argument("--gpu-sizes", default="1,2,4,6,8,10,12,14,16,18,20,24,28,32,36,40,44")
     ap.add_argument("--cpu-sizes", default="1,2,4,8,12,16")
     ap.add_argument("--reps", type=int, default=2)
+    ap.add_argument("--refine", type=int, default=0,
+                    help="rounds of synchronised level correction (Q26): partition 'fpm_refined'")
     ap.add_argument("--out", default=os.path.join(ROOT, "profiles", "hybrid_r02.json"))
     args = ap.parse_args()
     b = args.b
@@ -83,6 +85,8 @@ def main():
         sp = ctx.sample(i, b, sizes, pkg.FPM_F32)[0]
         models.append((sizes, sp))
         print(names[i], " ".join(f"{x}:{s / 1e9:.0f}" for x, s in zip(sizes, sp)), flush=True)
+    from studies import refine as rf
+    models[0] = rf.cliff_points(ctx, 0, b, models[0], args.gpu_c_cap_mib << 20)   # bracket the GPU's cliff (Q26)
     t_sample = time.perf_counter() - t0
     cpus = pkg.Context.local([CPU] * len(sockets), sm_caps=sockets)
     gpu = pkg.Context.local([0], sm_caps=[args.gpu_sms])
@@ -100,21 +104,33 @@ def main():
         st, per = timed_run(gpu, N, b, [(0, 0, 0, n, n)], 1, args.reps)
         row["gpu"] = {"t_s": st.t_compute_s, "gflops": st.gflops, "ooc": bool(st.ooc_devices & 1)}
         x_cal = max(1, args.ncal * args.ncal // p)
-        parts = {"fpm": models, "cpm": [([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models],
-                 "homogeneous": [([1], [1.0])] * p}
-        for name, mods in parts.items():
+        parts = {"fpm": (models, None), "cpm": ([([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models], None),
+                 "homogeneous": ([([1], [1.0])] * p, None)}
+        if args.refine:
+            (x_in, r_in), (x_out, r_out) = rf.cliff_areas(args.gpu_c_cap_mib << 20, b)
+            r_models, hist, r_d, r_rects = rf.refine(ctx, n, b, models, args.refine, arrange="fpm", concurrent=True,
+                                                      splits=[x_in] + [None] * (p - 1),
+                                                      cliffs=[(r_in, r_out)] + [None] * (p - 1))
+            parts["fpm_refined"] = (r_models, r_rects)
+            row["refine"] = hist
+        for name, (mods, given) in parts.items():
             d = pkg.fpm_partition(T, mods)
-            rects = pkg.colpart_arrange(n, d)
+            rects = given if given is not None else pkg.colpart_arrange(n, d)
             st, per = timed_run(ctx, N, b, rects, p, args.reps)
             row[name] = {"d": d, "areas": [r[3] * r[4] for r in rects], "t_s": st.t_compute_s, "gflops": st.gflops,
                          "per_dev_compute_s": per, "imbalance": imbalance(per), "ooc": bool(st.ooc_devices & 1)}
         row["fpm_vs_cpm"] = row["fpm"]["t_s"] / row["cpm"]["t_s"] - 1
         row["fpm_vs_homogeneous"] = row["fpm"]["t_s"] / row["homogeneous"]["t_s"] - 1
         row["fpm_vs_gpu_alone"] = row["fpm"]["t_s"] / row["gpu"]["t_s"] - 1
+        if "fpm_refined" in row:
+            row["fpm_refined_vs_cpm"] = row["fpm_refined"]["t_s"] / row["cpm"]["t_s"] - 1
+            row["fpm_refined_vs_gpu_alone"] = row["fpm_refined"]["t_s"] / row["gpu"]["t_s"] - 1
         table.append(row)
+        ref = row.get("fpm_refined")
         print(f"n={n}: cpus {row['cpus']['t_s']:.3f}s gpu {row['gpu']['t_s']:.3f}s fpm {row['fpm']['t_s']:.3f}s "
-              f"(imb {100 * row['fpm']['imbalance']:.1f}%, d={row['fpm']['d']}) cpm {row['cpm']['t_s']:.3f}s "
-              f"homog {row['homogeneous']['t_s']:.3f}s", flush=True)
+              f"(imb {100 * row['fpm']['imbalance']:.1f}%, d={row['fpm']['d']}) "
+              + (f"refined {ref['t_s']:.3f}s (imb {100 * ref['imbalance']:.1f}%, d={ref['d']}) " if ref else "")
+              + f"cpm {row['cpm']['t_s']:.3f}s homog {row['homogeneous']['t_s']:.3f}s", flush=True)
     for c in (ctx, cpus, gpu):
         c.close()
     out = {"config": {"b": b, "ns": ns, "gpu_sm_cap": args.gpu_sms, "gpu_c_cap_bytes": args.gpu_c_cap_mib << 20,

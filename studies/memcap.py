@@ -183,7 +183,7 @@ def main():
         parts = [("fpm", models, None)]
         if args.refine:
             r_models, hist, r_d, r_rects = rf.refine(ctx, n, b, models, args.refine, arrange=args.arrange,
-                                                      concurrent=not any(cpu_dev), splits=splits, cliffs=cliffs,
+                                                      concurrent=True, splits=splits, cliffs=cliffs,
                                                       log=lambda m: print(m, flush=True))
             row["refine"] = hist
             parts.append(("fpm_refined", r_models, r_rects))

@@ -98,7 +98,8 @@ def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=
     """Synchronised level correction: returns (models, history, d, rects) for
     T = n^2 blocks.  arrange: "paper" (colpart_arrange) or "fpm"
     (colpart_arrange_fpm on the current models); concurrent: sample all devices
-    at once (contexts with CPU devices: each device alone); splits: per device
+    at once (with CPU devices: every device on its own host thread, windows in
+    step); splits: per device
     the largest in-core area (None: no cliff); cliffs: per device the two
     bracketing rectangles ((h, w) in core, (h, w) out of core) -- a capped
     device is then also timed, in the same synchronised window, on the cliff

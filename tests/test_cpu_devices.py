@@ -150,8 +150,22 @@ def test_cpu_device_fpm_sample_procedure():
         assert all(c <= 0.025 or r == 50 for c, r in zip(ci, reps))
         with pytest.raises(pkg.FpmError):
             ctx.sample(0, 64, [2], pkg.FPM_F32)
-        with pytest.raises(pkg.FpmError):
-            ctx.sample(-1, 64, [1], pkg.FPM_F32)   # concurrent sampling with CPU devices: unsupported
+
+
+def test_cpu_devices_synchronised_sampling():
+    """fpm_sample(dev = -1) on CPU devices: all devices' windows in step (P:10
+    (ii)); per-device lists of positive speeds under the Q8 stop rule, and
+    fpm_sample_rects(-1) with a rectangle per device."""
+    if NCORES < 2:
+        pytest.skip("needs 2 host cores")
+    with pkg.Context.local([CPU, CPU], sm_caps=[1, 1]) as ctx:
+        sp, ci, reps = ctx.sample(-1, 64, [1, 4], pkg.FPM_F32)
+        assert len(sp) == 2 and all(len(r) == 2 for r in sp)
+        assert all(v > 0 for r in sp for v in r)
+        assert all(5 <= n <= 50 for r in reps for n in r)
+        assert all(c <= 0.025 or n == 50 for cr, rr in zip(ci, reps) for c, n in zip(cr, rr))
+        sp2, _, _ = ctx.sample_rects(-1, 64, [[(2, 3)], [(1, 2)]], pkg.FPM_F32)
+        assert len(sp2) == 2 and sp2[0][0] > 0 and sp2[1][0] > 0
 
 
 def test_cpu_device_fpm_partition_end_to_end():
