@@ -429,7 +429,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         # devices that share one GPU share its power budget: models measured alone take the
         # level the devices reach when all run (synchronised level correction, Q26)
         from studies import refine as rf
-        models, refine_hist, _, _ = rf.refine(ctx, n, b, models, 3, arrange="fpm")
+        models, refine_hist, _, _ = rf.refine(ctx, n, b, models, 3, arrange="fpm", ci_permille=10)
         fpm_source += " + synchronised level correction (Q26)"
     d, rects = plan(models)
     install(rects)
@@ -641,8 +641,8 @@ def run_hetero(peak_tflops: float) -> dict:
     from studies import hetero
     caps = [30, 26, 24, 20, 16, 14, 10, 6]   # config 4's {144 .. 32} scaled to fit 148 SMs
     t0 = time.perf_counter()
-    res = hetero.c4_study(caps, N=32768, b=512, reps=2, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3,
-                          refine_arrange=("fpm",))
+    res = hetero.c4_study(caps, N=32768, b=512, reps=3, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3,
+                          refine_arrange=("fpm",), refine_ci_permille=10)
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     capped_peak = peak_tflops * sum(caps) / sms
     out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "

@@ -389,6 +389,9 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *                 it.  Needs a cap on every device and the caps of the devices
  *                 of one GPU to fit it (FPM_EUNSUPPORTED otherwise).  Rebuilds
  *                 the devices' streams: set it before pmm_setup.
+ *   "sample_rel_ci_permille": fpm_sample's stop rule, the 95 % confidence
+ *                 half-width in thousandths of the mean (default 25 = 2.5 %,
+ *                 reading Q8; at most 50 repetitions either way).
  *   "raster_group": tile-rows per L2 raster group of the update (0 = auto,
  *                 the default: 12 for F16I8, 16 for F16X3 / TF32X3, measured
  *                 at c5, times the device's share of the SMs of its GPU among

@@ -180,6 +180,7 @@ struct pmm_ctx {
     int kernel_variant = -1;  // auto
     int chunk_k = 0;          // F16X3 / TF32X3 default kernel: K per TMEM accumulation (0 auto = 512)
     int raster_snake = 0;     // F16X3 / TF32X3 default kernel: serpentine raster over groups
+    double sample_rel_ci = 0.025;  // fpm_sample stop rule: 95 % half-width / mean (Q8)
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
@@ -2266,6 +2267,7 @@ struct GpuRunner {
 struct RepStats {
     std::vector<double> ts;
     double mean = 0.0, half = 0.0;
+    double rel = 0.025;  // stop when the 95 % half-width is <= rel x mean (option "sample_rel_ci")
     bool add(double t) {
         ts.push_back(t);
         const int nr = (int)ts.size();
@@ -2276,7 +2278,7 @@ struct RepStats {
         for (double v : ts) var += (v - mean) * (v - mean);
         var = nr > 1 ? var / (nr - 1) : 0.0;
         half = nr > 1 ? t975(nr - 1) * std::sqrt(var / nr) : 0.0;
-        return nr >= 5 && half <= 0.025 * mean;
+        return nr >= 5 && half <= rel * mean;
     }
 };
 
@@ -2294,6 +2296,7 @@ void sample_cpu(pmm_ctx* ctx, Device& d, fpm_dtype dt, int64_t b, const std::vec
         run();
         run();  // two warm-ups
         RepStats st;
+        st.rel = ctx->sample_rel_ci;
         for (int r = 0; r < 50; ++r)
             if (st.add(run())) break;
         speeds[j] = R.flops(shp[j]) / st.mean;
@@ -2329,6 +2332,7 @@ void sample_gpu(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vecto
     for (int j = 0; j < nsizes; ++j) {
         for (auto& sp : S) {
             sp->st = RepStats{};
+            sp->st.rel = ctx->sample_rel_ci;
             sp->done = false;
             sp->R->runs = 0;
         }
@@ -2416,6 +2420,7 @@ void sample_sync(pmm_ctx* ctx, const std::vector<Device*>& devs, const std::vect
     auto flops = [&](size_t i, const Shape& x) { return Cr[i] ? Cr[i]->flops(x) : G[i]->flops(x); };
     for (int j = 0; j < nsizes; ++j) {
         std::vector<RepStats> st(P);
+        for (auto& x : st) x.rel = ctx->sample_rel_ci;
         std::vector<double> t_run(P, 0.0), rate(P, 0.0);
         std::vector<std::exception_ptr> errs(P);
         double window = 0.0;
@@ -2797,6 +2802,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= -1 && value <= 8,
                           "kernel_variant must be -1 (auto) or 0..8 (6: F16I8 only; 7, 8: F16X3 / TF32X3 only)");
             ctx->kernel_variant = (int)value;
+        } else if (k == "sample_rel_ci_permille") {
+            FPM_CHECK_ARG(value >= 1 && value <= 500, "sample_rel_ci_permille must be in [1, 500]");
+            ctx->sample_rel_ci = value / 1000.0;
         } else if (k == "raster_snake") {
             FPM_CHECK_ARG(value == 0 || value == 1, "raster_snake must be 0 or 1");
             ctx->raster_snake = (int)value;

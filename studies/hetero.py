@@ -39,7 +39,8 @@ def imbalance(ts):
 
 
 def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, graph=1, sm_partition=0,
-             exclusive=True, log=print, refine_rounds=0, options=None, refine_arrange=("paper", "fpm")) -> dict:
+             exclusive=True, log=print, refine_rounds=0, options=None, refine_arrange=("paper", "fpm"),
+             refine_ci_permille=None) -> dict:
     """Sample each emulated device's FPM, then run the multiply under the FPM,
     CPM (N_cal and self-calibrated), homogeneous and in-situ corrected FPM
     partitions; returns the result dict written by main()."""
@@ -95,7 +96,8 @@ def c4_study(caps, N=32768, b=512, sizes=None, ncal=8192, reps=2, insitu=2, grap
     if refine_rounds > 0:
         from studies import refine as rf
         for arr in refine_arrange:
-            mods_r, hist, d_r, rects_r = rf.refine(ctx, n, b, models, refine_rounds, arrange=arr, log=log)
+            mods_r, hist, d_r, rects_r = rf.refine(ctx, n, b, models, refine_rounds, arrange=arr, log=log,
+                                                   ci_permille=refine_ci_permille)
             # (synchronised level correction of the exclusive models, Q26)
             refined["fpm_refined" + ("_arr" if arr == "fpm" else "")] = (mods_r, hist, d_r, rects_r)
 

@@ -94,7 +94,7 @@ def rescale(model, x_op, s_op, split=None):
 
 
 def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=pkg.FPM_F32, splits=None,
-           cliffs=None, log=None):
+           cliffs=None, log=None, ci_permille=None):
     """Synchronised level correction: returns (models, history, d, rects) for
     T = n^2 blocks.  arrange: "paper" (colpart_arrange) or "fpm"
     (colpart_arrange_fpm on the current models); concurrent: sample all devices
@@ -104,7 +104,15 @@ def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=
     bracketing rectangles ((h, w) in core, (h, w) out of core) -- a capped
     device is then also timed, in the same synchronised window, on the cliff
     rectangle on the other side of its operating point, so both sides of its
-    model get their synchronised level."""
+    model get their synchronised level.  ci_permille: the sampling stop rule
+    for these timings (option "sample_rel_ci_permille"; restored to Q8's 25
+    afterwards) -- a level ratio carries its sample's noise into the partition."""
+    if ci_permille is not None:
+        ctx.set_option("sample_rel_ci_permille", int(ci_permille))
+        try:
+            return refine(ctx, n, b, models, rounds, arrange, concurrent, dtype, splits, cliffs, log, None)
+        finally:
+            ctx.set_option("sample_rel_ci_permille", 25)
     T = n * n
     p = len(models)
     base = [(list(xs), list(ss)) for xs, ss in models]   # the size sweep's shapes
