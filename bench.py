@@ -312,6 +312,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         c.set_option("kernel_variant", args.kernel_variant)
         c.set_option("chunk_k", args.chunk_k)
         c.set_option("raster_snake", args.raster_snake)
+        c.set_option("share_b", args.share_b)
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
         c.set_option("e2e_tail", args.e2e_tail)
@@ -589,7 +590,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
     if rank == 0:
         if world == 1 and not caps and not args.no_hetero:
             try:
-                line["hetero"] = run_hetero(peak)
+                line["hetero"] = run_hetero(peak, args.share_b)
             except Exception as ex:  # report, do not hide
                 log("hetero failed:", repr(ex))
                 line["hetero"] = {"error": repr(ex)[:200]}
@@ -631,7 +632,7 @@ def fig7_summary() -> dict | None:
     return out if out["layouts"] else None
 
 
-def run_hetero(peak_tflops: float) -> dict:
+def run_hetero(peak_tflops: float, share_b: int = 1) -> dict:
     """The metric's 'FPM load imbalance %' under emulated heterogeneity (SURVEY
     §8(d) c4 analogue, studies/hetero.py): 8 devices on this GPU in disjoint
     green-context SM partitions, FPMs sampled per device, the multiply under
@@ -642,7 +643,7 @@ def run_hetero(peak_tflops: float) -> dict:
     caps = [30, 26, 24, 20, 16, 14, 10, 6]   # config 4's {144 .. 32} scaled to fit 148 SMs
     t0 = time.perf_counter()
     res = hetero.c4_study(caps, N=32768, b=512, reps=3, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3,
-                          refine_arrange=("fpm",), refine_ci_permille=10)
+                          refine_arrange=("fpm",), refine_ci_permille=10, options={"share_b": share_b})
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     capped_peak = peak_tflops * sum(caps) / sms
     out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "
@@ -783,6 +784,8 @@ def main():
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
     ap.add_argument("--raster-snake", type=int, default=0, help="serpentine raster over groups (0/1)")
+    ap.add_argument("--share-b", type=int, default=1,
+                    help="column members on the B owner's GPU read its staged B operand (0/1; local contexts)")
     ap.add_argument("--chunk-k", type=int, default=0, help="K per TMEM accumulation (variants 7/8; 0 auto = 512)")
     ap.add_argument("--fuse", type=int, default=0, help="pivots fused per update (0 auto = K of about 2048)")
     ap.add_argument("--e2e-steps", type=int, default=5)

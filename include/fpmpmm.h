@@ -389,6 +389,12 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *                 it.  Needs a cap on every device and the caps of the devices
  *                 of one GPU to fit it (FPM_EUNSUPPORTED otherwise).  Rebuilds
  *                 the devices' streams: set it before pmm_setup.
+ *   "share_b":    1 (default): in a local FP32 context, a device whose column's
+ *                 B pivot owner is another device on the same GPU reads the
+ *                 owner's staged (split, transposed) B operand instead of
+ *                 staging its own copy (update groups outside the download
+ *                 tail; the owner's next staging into that slot waits for
+ *                 those updates); 0: every device stages its own.
  *   "sample_rel_ci_permille": fpm_sample's stop rule, the 95 % confidence
  *                 half-width in thousandths of the mean (default 25 = 2.5 %,
  *                 reading Q8; at most 50 repetitions either way).

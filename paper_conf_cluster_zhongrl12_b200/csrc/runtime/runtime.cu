@@ -114,6 +114,9 @@ struct Device {
     void* a_hi[kSlots] = {}, *a_lo[kSlots] = {}, *b_hi[kSlots] = {}, *b_lo[kSlots] = {};
     float* sa[kSlots] = {}, *sb[kSlots] = {};
     const void* a_op[kSlots] = {};          // FP64: A operand of the slot
+    int b_from[kSlots] = {};                // FP32 slots 0, 1: device whose staged B operand this slot's
+                                            // update reads (its own index, or the column's B owner on the
+                                            // same GPU: option "share_b")
     int tail_slots = 0;                     // slots 2.. allocated
     // fused tail (kFusedSlot): the tail's pivots staged as one K = tail_K operand
     // with common F16X3 scales (maxima merged in tmax_a / tmax_b first)
@@ -181,6 +184,7 @@ struct pmm_ctx {
     int chunk_k = 0;          // F16X3 / TF32X3 default kernel: K per TMEM accumulation (0 auto = 512)
     int raster_snake = 0;     // F16X3 / TF32X3 default kernel: serpentine raster over groups
     double sample_rel_ci = 0.025;  // fpm_sample stop rule: 95 % half-width / mean (Q8)
+    int share_b = 1;          // local FP32: column members on the B owner's GPU read its staged B operand
     int fuse = 0;             // pivots per update (0 = auto)
     int fuse_max = 1;         // resolved for the current problem
     int ooc_keep = 1;         // out-of-core: keep the last R bands, reverse every other update
@@ -818,6 +822,7 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
         d.rect = rects[d.idx];
         d.H = d.rect.h * b;
         d.W = d.rect.w * b;
+        for (int s = 0; s < kSlots; ++s) d.b_from[s] = d.idx;
         if (!d.live()) {
             d.H = d.W = 0;
             continue;
@@ -940,8 +945,23 @@ struct TailPhase {
     int64_t k_off = 0;
 };
 
+// The B owner of update group g for device d's column, if d may read that
+// owner's staged B operand instead of staging its own copy: local FP32 context,
+// a double-buffered slot (not the tail), the owner another GPU device on the
+// same GPU (its L2 serves the re-reads; peer addresses bypass it).
+Device* shared_b_owner(pmm_ctx* ctx, const Device& d, int g, int slot) {
+    if (!ctx->share_b || ctx->dt != FPM_F32 || ctx->nccl_mode || ctx->ipc_mode || d.cpu || slot >= 2) return nullptr;
+    const int64_t k0 = ctx->groups[g].first;
+    for (const Move& m : ctx->plan_b[k0]) {
+        if (m.dst != d.idx || m.src == d.idx) continue;
+        Device* q = local_dev(ctx, m.src);
+        if (q && !q->cpu && q->cuda_dev == d.cuda_dev && q->live() && q->W == d.W) return q;
+    }
+    return nullptr;
+}
+
 int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, bool streamed,
-                   TailPhase tp = TailPhase{}) {
+                   TailPhase tp = TailPhase{}, bool share = false) {
     const size_t es = esize(ctx->dt);
     const int64_t b = ctx->b;
     const int64_t k0 = ctx->groups[g].first;
@@ -951,6 +971,14 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     int64_t bytes = 0;
     CU(cudaSetDevice(d.cuda_dev));
     if (!first_use) CU(cudaStreamWaitEvent(d.s_comm, d.ev_free[slot], 0));
+    // shared B operands: this slot's buffers may still be read by the column members
+    // whose previous update took its B from here -- wait for those updates too
+    if (!first_use && tp.phase == 0 && slot < 2)
+        for (auto& q : ctx->devs)
+            if (&q != &d && !q.cpu && q.live() && q.b_from[slot] == d.idx)
+                CU(cudaStreamWaitEvent(d.s_comm, q.ev_free[slot], 0));
+    Device* b_owner = (share && tp.phase == 0) ? shared_b_owner(ctx, d, g, slot) : nullptr;
+    if (slot < 2 && tp.phase == 0) d.b_from[slot] = b_owner ? b_owner->idx : d.idx;
     // streamed input: this device's own panels of the group have landed (the
     // upload stream runs ahead, in k order)
     if (streamed) CU(cudaStreamWaitEvent(d.s_comm, d.ev_up[kl], 0));
@@ -1090,9 +1118,13 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
                         static_cast<char*>(d.a_lo[slot]) + (size_t)pc.row_off * ld_out * op + ko,
                         d.sa[slot] + pc.row_off, d.s_comm, ga ? ga + pc.row_off : nullptr);
             }
-            launch_split_cols(static_cast<const float*>(b_src), d.W, fb, d.W, sch,
-                              static_cast<char*>(d.b_hi[slot]) + ko, static_cast<char*>(d.b_lo[slot]) + ko,
-                              d.sb[slot], d.s_comm, ld_out, gb);
+            if (b_owner) {
+                d.launches -= (f16 && gb == nullptr) ? 3 : 1;   // the owner stages this B operand
+            } else {
+                launch_split_cols(static_cast<const float*>(b_src), d.W, fb, d.W, sch,
+                                  static_cast<char*>(d.b_hi[slot]) + ko, static_cast<char*>(d.b_lo[slot]) + ko,
+                                  d.sb[slot], d.s_comm, ld_out, gb);
+            }
         }
     } else {
         d.a_op[slot] = a_src;  // f panels of H x b, H b apart (own block-columns or the receive buffer)
@@ -1110,12 +1142,14 @@ UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     UpdateArgs a;
     a.a_hi = d.a_hi[slot];
     a.a_lo = d.a_lo[slot];
-    a.bt_hi = d.b_hi[slot];
-    a.bt_lo = d.b_lo[slot];
+    // the B operand: this device's, or the column owner's on the same GPU (share_b)
+    const Device* bd = (slot < 2 && d.b_from[slot] != d.idx) ? local_dev(ctx, d.b_from[slot]) : &d;
+    a.bt_hi = bd->b_hi[slot];
+    a.bt_lo = bd->b_lo[slot];
     const SplitScheme sch = scheme_for(ctx, ctx->b);
     const bool f16 = has_scales(sch);
     a.sa = f16 ? d.sa[slot] : nullptr;
-    a.sb = f16 ? d.sb[slot] : nullptr;
+    a.sb = f16 ? bd->sb[slot] : nullptr;
     a.C = static_cast<float*>(d.C);
     a.M = d.H;
     a.Nc = d.W;
@@ -1154,6 +1188,8 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
     const int f = ctx->groups[g].second;
     CU(cudaSetDevice(d.cuda_dev));
     CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
+    if (ctx->dt == FPM_F32 && slot < 2 && d.b_from[slot] != d.idx)  // the owner staged this update's B
+        CU(cudaStreamWaitEvent(d.s_comp, local_dev(ctx, d.b_from[slot])->ev_ready[slot], 0));
     rec_t(d.ev_upd0[g], d.s_comp);
     // out-of-core band order: reversed every other update, the last two
     // bands kept on the device between updates (option "ooc_keep")
@@ -1736,7 +1772,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
                     }
                     bytes += issue_comm(ctx, d, g, slot, false, streamed, TailPhase{1, 0});
                 } else {
-                    bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed);
+                    bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed, TailPhase{}, g < gt);
                 }
             }
         for (auto& d : ctx->devs)
@@ -2802,6 +2838,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value >= -1 && value <= 8,
                           "kernel_variant must be -1 (auto) or 0..8 (6: F16I8 only; 7, 8: F16X3 / TF32X3 only)");
             ctx->kernel_variant = (int)value;
+        } else if (k == "share_b") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "share_b must be 0 or 1");
+            ctx->share_b = (int)value;
         } else if (k == "sample_rel_ci_permille") {
             FPM_CHECK_ARG(value >= 1 && value <= 500, "sample_rel_ci_permille must be in [1, 500]");
             ctx->sample_rel_ci = value / 1000.0;

@@ -398,3 +398,30 @@ def test_per_device_span_stats():
             assert st.per_dev_span_s[i] <= st.t_compute_s * 1.001
         assert max(st.per_dev_span_s[:2]) == pytest.approx(st.t_compute_s, rel=1e-6)
         assert st.per_dev_span_s[2] == 0.0
+
+
+@pytest.mark.parametrize("graph", [1, 0])
+def test_shared_b_operand_bit_identical(graph):
+    """Option share_b (default on): column members on the B owner's GPU read its
+    staged B operand.  The operand is the same bytes either way (same rows,
+    same column maxima), so C is bit-identical to share_b = 0, with the k-loop
+    replayed as a graph or issued eagerly, and repeated computes agree."""
+    N, b = 3072, 256
+    n = N // b
+    rects = pkg.colpart_arrange(n, [40, 36, 30, 20, 18])
+    assert len({r[0] for r in rects}) < 5     # some columns hold several devices
+    out = []
+    for share in (1, 0):
+        with pkg.Context.local([0] * 5) as ctx:
+            ctx.set_option("graph", graph)
+            ctx.set_option("share_b", share)
+            ctx.setup(N, b, rects, pkg.FPM_F32)
+            ctx.fill_synthetic(1, 2, pkg.FPM_DIST_PM1)
+            ctx.compute()
+            ctx.compute()
+            C = np.empty((N, N), np.float32)
+            ctx.download(C, N)
+            out.append(C)
+    assert np.array_equal(out[0], out[1])
+    ref = og.gemm(synth.rect(1, N, 0, 0, N, N), synth.rect(2, N, 0, 0, N, N))
+    assert og.rel_fro(out[0], ref) <= 1e-5
