@@ -21,7 +21,9 @@ The speed functions are sampled in advance on sqrt(x) x sqrt(x) submatrices
    window), and rescales the device's model by measured / modelled speed at
    that point -- the shape stays the one of the size sweep, the level becomes
    the synchronised one; for a capped device only the points on the same side
-   of its cliff -- then re-partitions, until the partition stops changing.
+   of its cliff -- then re-partitions, until the partition stops changing; if it
+   does not within the rounds, the candidate with the smallest measured
+   makespan is kept.
 
 Orchestration only: sampling (fpm_sample / fpm_sample_rects), partitioning and
 arranging are library calls.
@@ -126,7 +128,9 @@ def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=
         return d, r
 
     d, rects = place(mods)
+    placed_by = [(list(xs), list(ss)) for xs, ss in mods]   # the models this candidate was placed with
     hist = []
+    best = None   # (measured makespan, d, rects, models): the best partition actually timed
     for it in range(rounds):
         shapes = []
         for i, r in enumerate(rects):
@@ -153,12 +157,22 @@ def refine(ctx, n, b, models, rounds=3, arrange="paper", concurrent=True, dtype=
             else:
                 ratios.append(k)
             mods[i] = (xs, ss)
+        # this candidate's makespan as measured in the synchronised window (a run's time is
+        # proportional to area / speed at the operating point)
+        span = max((r[3] * r[4]) / sp[i][0] for i, r in enumerate(rects) if r[3] * r[4] > 0)
+        if best is None or span < best[0]:
+            best = (span, list(d), list(rects), placed_by)
         hist.append({"round": it, "d": list(d), "areas": [r[3] * r[4] for r in rects],
-                     "sampled_gflops": [v[0] / 1e9 for v in sp], "level_ratio": ratios})
+                     "sampled_gflops": [v[0] / 1e9 for v in sp], "level_ratio": ratios,
+                     "measured_makespan_rel": span})
         d_new, rects_new = place(mods)
         if log:
             log(f"refine {it}: d={d} -> {d_new}  ratios={ratios}")
-        if d_new == d:
-            break
+        if d_new == d:   # converged: the partition the corrected models place is the one just timed
+            return mods, hist, d, rects
         d, rects = d_new, rects_new
-    return mods, hist, d, rects
+        placed_by = [(list(xs), list(ss)) for xs, ss in mods]
+    # not converged within `rounds` (e.g. oscillating across a memory cliff): the best
+    # partition that was actually timed, with the models that placed it
+    _, d, rects, m = best
+    return m, hist, d, rects

@@ -228,13 +228,20 @@ def test_sample_rects_and_operating_point_refinement():
         assert sum(d) == n * n and 1 <= len(hist) <= 3
         for h in hist:
             assert sum(h["d"]) == n * n
-        last = hist[-1]
+        # the returned partition is one that was timed: the converged one (last round) or
+        # the candidate with the smallest measured makespan
+        assert d in [h["d"] for h in hist]
+        chosen = [h for h in hist if h["d"] == d][-1]
+        assert chosen is hist[-1] or chosen["measured_makespan_rel"] == min(h["measured_makespan_rel"] for h in hist)
         for i in range(2):
-            assert mods[i][0] == sizes
-            k = last["level_ratio"][i]
+            assert mods[i][0] == sizes   # the shape of the size sweep is kept: one ratio per device
+            k = mods[i][1][0] / models[i][1][0]
             assert all(abs(a - k * s0) <= 1e-9 * a for a, s0 in zip(mods[i][1], models[i][1]))
-            x = last["areas"][i]
-            assert abs(pkg.fpm_model_speed(mods[i], x) - last["sampled_gflops"][i] * 1e9) <= 1e-6 * pkg.fpm_model_speed(mods[i], x)
+        if chosen is hist[-1] and len(hist) < 3:   # converged: the models carry that round's levels
+            for i in range(2):
+                x = chosen["areas"][i]
+                assert abs(pkg.fpm_model_speed(mods[i], x) - chosen["sampled_gflops"][i] * 1e9) <= \
+                    1e-6 * pkg.fpm_model_speed(mods[i], x)
 
 
 def test_cliff_areas_and_rescale():
