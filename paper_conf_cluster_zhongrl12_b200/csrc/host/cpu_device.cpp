@@ -153,8 +153,6 @@ void team_destroy(Team* t) {
     delete t;
 }
 
-int team_size(const Team* t) { return t ? t->n : 0; }
-
 // ------------------------------------------------------------------ micro-kernels
 namespace {
 

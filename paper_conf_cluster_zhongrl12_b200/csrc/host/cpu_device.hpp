@@ -24,7 +24,6 @@ std::vector<int> allowed_cores();
 // Worker threads pinned one per core (cores empty: `n` unpinned threads).
 Team* team_create(const std::vector<int>& cores, int n = 0);
 void team_destroy(Team* t);
-int team_size(const Team* t);
 // Instruction set of the micro-kernels in use: "avx512", "avx2" or "generic".
 const char* isa();
 
