@@ -240,8 +240,10 @@ def build_line(*, world, steps, warmup, step_times, workload, cfg, scheme, roofl
     total_t = sum(step_times)
     N = cfg["N"]
     value = 2.0 * N ** 3 * steps / total_t / 1e9
-    meas = [d["compute_s"] for d in per_dev if d["rect"][3] * d["rect"][4] > 0]
-    pred = [d["predicted_s"] for d in per_dev if d["rect"][3] * d["rect"][4] > 0]
+    live = [d for d in per_dev if d["rect"][3] * d["rect"][4] > 0]
+    meas = [d.get("span_s", 0.0) for d in live]          # when each device finished (P:9)
+    comp = [d["compute_s"] for d in live]                # sum of its staging + update event times
+    pred = [d["predicted_s"] for d in live]
     peak = roofline["peak"]
     config = {
         "workload": workload, "N": N, "b": cfg["b"], "p": len(per_dev),
@@ -250,12 +252,14 @@ def build_line(*, world, steps, warmup, step_times, workload, cfg, scheme, roofl
         "l2": (f"inputs larger than L2 (A, B, C {N * N * 4 / 1e9:.2f} GB each)" if N * N * 4 > 126e6
                else "inputs fit in L2 (no flush between steps)"),
         "pct_tensor_peak": 100.0 * value / 1e3 / (peak * world) if peak else None,
+        # load imbalance (reading Q18): max / mean - 1 of the devices' finish times -- the
+        # k-loop span of each device, start to its last update's end (P:9: "all processors
+        # complete their work within the same time"); also over the sums of each device's
+        # staging + update event times (round 1's measure, which counts staging that runs
+        # under the device's own updates a second time) and as the FPMs predict it
         "imbalance_pct_measured": 100.0 * imbalance(meas),
+        "imbalance_pct_compute_sum": 100.0 * imbalance(comp),
         "imbalance_pct_predicted": 100.0 * imbalance(pred),
-        # the same over the devices' k-loop spans (start to their last update's end):
-        # staging that overlaps a device's updates counted once
-        "imbalance_pct_span": 100.0 * imbalance([d.get("span_s", 0.0) for d in per_dev
-                                                  if d["rect"][3] * d["rect"][4] > 0]),
         "per_device": per_dev,
     }
     config.update(extra_config or {})
@@ -521,7 +525,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         alt = {"cpm_ncal": [([1], [pkg.fpm_model_speed(m, x_cal)]) for m in models],
                "homogeneous": [([1], [1.0])] * p}
         partitions = {"fpm": {"t_s": statistics.median(step_times), "d": list(d),
-                              "imbalance_pct_measured": 100.0 * imbalance([x["compute_s"] for x in per_dev]),
+                              "imbalance_pct_measured": 100.0 * imbalance([x["span_s"] for x in per_dev]),
+                              "imbalance_pct_compute_sum": 100.0 * imbalance([x["compute_s"] for x in per_dev]),
                               "imbalance_pct_predicted": 100.0 * imbalance([x["predicted_s"] for x in per_dev])}}
         for name, pm in alt.items():
             dd, rr = plan(pm)
@@ -536,7 +541,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
             recs = per_device(list(best.per_dev_compute_s), list(best.per_dev_update_s), list(best.per_dev_span_s),
                               rr, models)
             partitions[name] = {"t_s": t_best, "d": list(dd),
-                                "imbalance_pct_measured": 100.0 * imbalance([x["compute_s"] for x in recs]),
+                                "imbalance_pct_measured": 100.0 * imbalance([x["span_s"] for x in recs]),
+                                "imbalance_pct_compute_sum": 100.0 * imbalance([x["compute_s"] for x in recs]),
                                 "imbalance_pct_predicted": 100.0 * imbalance([x["predicted_s"] for x in recs])}
         for v in partitions.values():
             v["gflops"] = 2.0 * N ** 3 / v["t_s"] / 1e9
@@ -666,8 +672,8 @@ def run_hetero(peak_tflops: float, share_b: int = 1) -> dict:
         out[rename.get(name, name)] = {
             "t_s": r["t_total_s"], "gflops": r["gflops"], "d": r["d"],
             "refine_rounds": len(r.get("refine_history", [])) or None,
-            "imbalance_pct_measured": 100.0 * r["imbalance_measured"],
-            "imbalance_pct_span": 100.0 * r.get("imbalance_span", 0.0),
+            "imbalance_pct_measured": 100.0 * r.get("imbalance_span", 0.0),
+            "imbalance_pct_compute_sum": 100.0 * r["imbalance_measured"],
             "imbalance_pct_predicted": 100.0 * r["imbalance_predicted"],
             "pct_of_capped_peak": 100.0 * r["gflops"] / 1e3 / capped_peak}
     if "fpm" in out and "cpm_ncal" in out:

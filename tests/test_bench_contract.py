@@ -80,7 +80,8 @@ def test_n_gt_1_line_contract():
     N, b = cfg["N"], cfg["b"]
     rects = [[0, 0, 0, 16, 32], [0, 16, 0, 16, 32]]   # p = 2: one column of two 16 x 32-block strips
     per_dev = [{"rank": r, "device": r, "rect": rects[r], "area": 512, "sm_cap": None,
-                "compute_s": t, "update_s": 0.9 * t, "predicted_s": 0.01} for r, t in enumerate((0.010, 0.011))]
+                "compute_s": t, "update_s": 0.9 * t, "span_s": sp, "predicted_s": 0.01}
+               for r, (t, sp) in enumerate(((0.010, 0.0100), (0.011, 0.0104)))]
     roof = {"bound": "tensor", "achieved": 400.0, "peak": 464.5, "unit": "TFLOP/s", "frac": 400.0 / 464.5,
             "traffic": None}
     line = bm.build_line(world=2, steps=3, warmup=3, step_times=[0.011, 0.012, 0.011], workload="c3",
@@ -97,7 +98,8 @@ def test_n_gt_1_line_contract():
     assert abs(line["ms_per_step"] - 1e3 * 0.034 / 3) < 1e-9
     c = line["config"]
     assert c["p"] == 2 and len(c["per_device"]) == 2 and c["partition"] == [512, 512]
-    assert abs(c["imbalance_pct_measured"] - 100.0 * (0.011 / 0.0105 - 1)) < 1e-9
+    assert abs(c["imbalance_pct_measured"] - 100.0 * (0.0104 / 0.0102 - 1)) < 1e-9      # finish times
+    assert abs(c["imbalance_pct_compute_sum"] - 100.0 * (0.011 / 0.0105 - 1)) < 1e-9
     assert c["imbalance_pct_predicted"] == 0.0
     assert c["exchange_staging_overlap"] == [0.9, 0.8]
     assert line["dtype"].startswith("f32 (F16X3")
