@@ -320,6 +320,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
         c.set_option("e2e_tail", args.e2e_tail)
+        if args.tail_band:
+            c.set_option("tail_band", args.tail_band)
         if caps:
             c.set_option("sm_partition", 1)   # every kernel of a device inside its SM partition
         return c
@@ -797,6 +799,7 @@ def main():
     ap.add_argument("--e2e-steps", type=int, default=5)
     ap.add_argument("--tail-stream", type=int, default=1, help="pmm_run option tail_stream (e2e, one device)")
     ap.add_argument("--e2e-tail", type=int, default=-1, help="pmm_run option e2e_tail (-1 auto)")
+    ap.add_argument("--tail-band", type=int, default=0, help="pmm_run option tail_band (rows, multiple of 256; 0 default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-hetero", action="store_true",
                     help="skip the emulated-heterogeneity measurement (c4 analogue) added at N = 1")
