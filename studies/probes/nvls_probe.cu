@@ -51,6 +51,23 @@ int main() {
             if (r == CUDA_SUCCESS) cuMemRelease(t);
         }
     }
+    for (unsigned nd = 2; nd <= 8; nd *= 2) {   // teams larger than the GPUs present
+        CUmulticastObjectProp q = mp; q.numDevices = nd; q.size = gran;
+        CUmemGenericAllocationHandle t; CUresult r = cuMulticastCreate(&t, &q);
+        const char* es = nullptr; cuGetErrorString(r, &es);
+        printf("{\"try_num_devices\": %u, \"rc\": %d, \"err\": \"%s\"}\n", nd, (int)r, es ? es : "");
+        if (r == CUDA_SUCCESS) {
+            CUresult ra = cuMulticastAddDevice(t, dev);
+            CUmemAllocationProp pq = {};
+            pq.type = CU_MEM_ALLOCATION_TYPE_PINNED; pq.location.type = CU_MEM_LOCATION_TYPE_DEVICE; pq.location.id = 0;
+            pq.requestedHandleTypes = (CUmemAllocationHandleType)q.handleTypes;
+            CUmemGenericAllocationHandle ph2; CUresult rc = cuMemCreate(&ph2, gran, &pq, 0);
+            CUresult rb = rc == CUDA_SUCCESS ? cuMulticastBindMem(t, 0, ph2, 0, gran, 0) : rc;
+            printf("{\"add_rc\": %d, \"create_rc\": %d, \"bind_rc\": %d}\n", (int)ra, (int)rc, (int)rb);
+            if (rc == CUDA_SUCCESS) cuMemRelease(ph2);
+            cuMemRelease(t);
+        }
+    }
     mp.handleTypes = CU_MEM_HANDLE_TYPE_NONE;
     CUmemGenericAllocationHandle mch; CK(cuMulticastCreate(&mch, &mp));
     CK(cuMulticastAddDevice(mch, dev));
