@@ -272,7 +272,9 @@ def build_line(*, world, steps, warmup, step_times, workload, cfg, scheme, roofl
     }
 
 
-def run_ours(args, rank: int, world: int, local_rank: int, dist):
+def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = True) -> dict | None:
+    """One bench run of args.config; rank 0 returns (and, with `emit`, prints) the
+    JSON line, the other ranks return None."""
     import torch
 
     import paper_conf_cluster_zhongrl12_b200 as pkg
@@ -604,9 +606,54 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist):
                 line["hetero"] = {"error": repr(ex)[:200]}
         if world == 1:
             line["fig7"] = fig7_summary()
-        print(json.dumps(line), flush=True)
         if parity is not None and not parity["ok"]:
+            print(json.dumps(line), flush=True)
             sys.exit(3)
+        if emit:
+            print(json.dumps(line), flush=True)
+    return line
+
+
+def run_hetero_multi(args, rank: int, world: int, local_rank: int, dist) -> dict | None:
+    """N > 1: the heterogeneity measurement on the job's own GPUs -- config 4
+    (N = 32768, b = 512, rank i capped to {144, 128, ..., 32}[i] SMs in a green
+    partition of its GPU) run through the same code path as
+    `--config c4`: FPMs sampled per rank, FPM / CPM(N_cal) / homogeneous
+    partitions, max-over-ranks device times.  Rank 0 returns the summary."""
+    import copy
+
+    import torch
+    h = copy.copy(args)
+    h.config, h.N, h.b = "c4", args.hetero_N, 0
+    h.steps, h.warmup, h.e2e_steps = 3, 3, 0
+    h.no_cpu_baseline, h.no_partitions, h.fpm_cache = True, False, ""
+    h.traffic = None
+    t0 = time.perf_counter()
+    hl = run_ours(h, rank, world, local_rank, dist, emit=False)
+    if rank != 0:
+        return None
+    c = hl["config"]
+    sms = torch.cuda.get_device_properties(local_rank).multi_processor_count
+    caps = [x["sm_cap"] for x in c["per_device"]]
+    mma_per_mac = 2.0 if args.scheme == "f16i8" else 3.0
+    peaks = measured_peaks()
+    dense = peaks["bf16_sustained"] if args.scheme != "tf32x3" else peaks["bf16_sustained"] / 2.0
+    capped_peak = dense / mma_per_mac * sum(caps) / sms
+    out = {"workload": c["workload"], "N": c["N"], "b": c["b"], "sm_caps": caps,
+           "source": "bench.py --config c4 path run inside this job across its ranks (one GPU each, "
+                     "green-context partitions)",
+           "method": "fpm: each rank's FPM sampled on its own capped GPU (P:18), gathered, fpm_partition + "
+                     "colpart_arrange (P:9, P:15)",
+           "capped_aggregate_peak_tflops": capped_peak, "value_gflops": hl["value"],
+           "roofline_frac_busiest": hl["roofline"]["frac"], "transport": c["transport"]}
+    for name, r in (c["partitions"] or {}).items():
+        if not isinstance(r, dict):
+            continue
+        out[name] = dict(r, pct_of_capped_peak=100.0 * r["gflops"] / 1e3 / capped_peak)
+    for k in ("fpm_vs_cpm_time_delta_pct", "fpm_vs_homogeneous_time_delta_pct"):
+        out[k] = (c["partitions"] or {}).get(k)
+    out["wall_s"] = time.perf_counter() - t0
+    return out
 
 
 def fig7_summary() -> dict | None:
@@ -802,7 +849,10 @@ def main():
     ap.add_argument("--tail-band", type=int, default=0, help="pmm_run option tail_band (rows, multiple of 256; 0 default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--no-hetero", action="store_true",
-                    help="skip the emulated-heterogeneity measurement (c4 analogue) added at N = 1")
+                    help="skip the heterogeneity measurement added to the line: N = 1 the c4 analogue on "
+                         "eight green partitions of the GPU, N > 1 config 4 across the job's GPUs")
+    ap.add_argument("--hetero-N", type=int, default=32768,
+                    help="N > 1: matrix size of the config-4 heterogeneity run (b = 512)")
     ap.add_argument("--no-sample", action="store_true", help="skip fpm_sample (profiling runs)")
     ap.add_argument("--fpm-cache", default="",
                     help="FPM model file: reused when it was measured on the same device / cap / b / scheme, "
@@ -827,11 +877,25 @@ def main():
         if args.transport == "nccl":   # communicator set-up in the log (ranks per communicator)
             os.environ.setdefault("NCCL_DEBUG", "INFO")
             os.environ.setdefault("NCCL_DEBUG_SUBSYS", "INIT")
-        dist.init_process_group("gloo", rank=rank, world_size=world)
+        import datetime
+        # a rank that fails between collectives surfaces as an error on the others
+        # after this long instead of hanging the job
+        dist.init_process_group("gloo", rank=rank, world_size=world, timeout=datetime.timedelta(minutes=10))
     if args.impl == "reference":
         run_reference(args, rank)
     else:
-        run_ours(args, rank, world, local_rank, dist)
+        line = run_ours(args, rank, world, local_rank, dist, emit=False)
+        if world > 1 and args.config != "c4" and not args.no_hetero:
+            # every rank takes part; a failure is reported in the line, not hidden
+            try:
+                het = run_hetero_multi(args, rank, world, local_rank, dist)
+            except Exception as ex:  # pragma: no cover (GPU only)
+                log(f"rank {rank}: multi-GPU hetero failed:", repr(ex))
+                het = {"error": repr(ex)[:200]}
+            if rank == 0:
+                line["hetero"] = het
+        if rank == 0:
+            print(json.dumps(line), flush=True)
     if dist is not None:
         dist.barrier()
         dist.destroy_process_group()

@@ -272,6 +272,18 @@ int pmm_download(pmm_ctx* ctx, void* C, int64_t ld, int64_t row_base, int64_t co
 int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t rows, int64_t cols, void* C_host,
                        int64_t ld);
 
+/* Timeline of the last k-loop on local GPU device `dev` (arrangement index),
+ * per update group g (f pivots fused, in k order): out[4g .. 4g+3] = start and
+ * end of its staging (pivot exchange + pack) and start and end of
+ * its rank-(f b) update (a7), in seconds after the loop's start event, from the
+ * CUDA events on the device's streams -- the per-iteration view behind the
+ * Fig. 6 computation times.  Groups of a download-overlapped tail or
+ * of a phase the loop did not time are NaN.  out: cap doubles (caller-owned;
+ * 4 per group); *count = number of groups (written even when cap is short).
+ * Blocks until the loop finished.  FPM_EINVAL for a CPU device or one this
+ * process does not drive; FPM_ESTATE before pmm_setup. */
+int pmm_group_times(pmm_ctx* ctx, int32_t dev, double* out, int32_t cap, int32_t* count);
+
 /* Whole call on host matrices: setup (if the problem changed), then the N/b
  * iterations with the inputs streamed from the host windows (block-column k of
  * A and block-row k of B are copied host -> device on the communication stream

@@ -187,6 +187,15 @@ class Context:
                                      out.strides[0] // out.itemsize))
         return out
 
+    def group_times(self, dev: int) -> list:
+        """[(staging start, staging end, update start, update end)] per update group
+        of the last k-loop on device `dev`, seconds after its start (pmm_group_times)."""
+        cnt = ctypes.c_int32(0)
+        check(lib.pmm_group_times(self._h, int(dev), None, 0, ctypes.byref(cnt)))
+        buf = (ctypes.c_double * (4 * cnt.value))()
+        check(lib.pmm_group_times(self._h, int(dev), buf, 4 * cnt.value, ctypes.byref(cnt)))
+        return [tuple(buf[4 * g: 4 * g + 4]) for g in range(cnt.value)]
+
     def run(self, A, B, C, N: int, b: int, rects: Sequence[Rect], dtype: int = FPM_F32,
             ld: int | None = None, row_base: int = 0, col_base: int = 0) -> PmmStats:
         st = PmmStats()

@@ -108,6 +108,7 @@ _SIGS = {
     "pmm_compute": ([vp, i32, ctypes.POINTER(PmmStats)], ctypes.c_int),
     "pmm_download": ([vp, vp, i64, i64, i64], ctypes.c_int),
     "pmm_download_block": ([vp, i64, i64, i64, i64, vp, i64], ctypes.c_int),
+    "pmm_group_times": ([vp, i32, ctypes.POINTER(dbl), i32, ctypes.POINTER(i32)], ctypes.c_int),
     "pmm_run": ([vp, vp, vp, vp, i64, i64, i32, ctypes.POINTER(ColpartRect), ctypes.c_int, i64, i64, i64,
                  ctypes.POINTER(PmmStats)], ctypes.c_int),
     "fpm_sample": ([vp, i32, ctypes.c_int, i64, ctypes.POINTER(i64), i32, ctypes.POINTER(dbl),

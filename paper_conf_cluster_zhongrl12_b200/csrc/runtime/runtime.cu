@@ -2987,6 +2987,35 @@ extern "C" int pmm_download_block(pmm_ctx* ctx, int64_t r0, int64_t c0, int64_t 
     });
 }
 
+extern "C" int pmm_group_times(pmm_ctx* ctx, int32_t dev, double* out, int32_t cap, int32_t* count) {
+    return guarded([&] {
+        FPM_CHECK_ARG(ctx != nullptr && count != nullptr && (cap == 0 || out != nullptr), "null argument");
+        if (!ctx->have_problem) fpm::fail(FPM_ESTATE, "pmm_group_times before pmm_setup");
+        fpm::Device* d = fpm::local_dev(ctx, dev);
+        FPM_CHECK_ARG(d != nullptr, "device %d is not driven by this process", dev);
+        FPM_CHECK_ARG(!d->cpu, "device %d is a host-CPU device (its times are host-timed)", dev);
+        const int ng = d->live() ? (int)ctx->groups.size() : 0;
+        *count = ng;
+        if (ng == 0) return;
+        CU(cudaSetDevice(d->cuda_dev));
+        CU(cudaEventSynchronize(d->ev_stop));
+        auto rel = [&](cudaEvent_t e) {  // seconds after ev_start; NaN for an event this loop did not record
+            float ms = 0.0f;
+            if (cudaEventElapsedTime(&ms, d->ev_start, e) != cudaSuccess) {
+                cudaGetLastError();
+                return std::nan("");
+            }
+            return (double)ms * 1e-3;
+        };
+        for (int g = 0; g < ng && 4 * g + 3 < cap; ++g) {
+            out[4 * g + 0] = rel(d->ev_pack0[g]);
+            out[4 * g + 1] = rel(d->ev_pack1[g]);
+            out[4 * g + 2] = rel(d->ev_upd0[g]);
+            out[4 * g + 3] = rel(d->ev_upd1[g]);
+        }
+    });
+}
+
 extern "C" int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int64_t b, int32_t p,
                        const colpart_rect* rects, fpm_dtype dt, int64_t ld, int64_t row_base, int64_t col_base,
                        pmm_stats* stats) {

@@ -44,7 +44,7 @@ def _torchrun(nproc, args, timeout=600):
 @pytest.mark.parametrize("config,N,b", [("c5", 8192, 1024), ("c3", 4096, 512), ("c4", 4096, 512)])
 def test_two_ranks_same_gpu_line(config, N, b):
     d, _ = _torchrun(2, ["--gpus", "2", "--steps", "2", "--warmup", "3", "--same-gpu", "--config", config,
-                         "--N", str(N), "--b", str(b), "--e2e-steps", "1"])
+                         "--N", str(N), "--b", str(b), "--e2e-steps", "1", "--hetero-N", "4096"])
     assert d["n_gpus"] == 2 and d["scaling"] == "strong" and d["value"] > 0
     c = d["config"]
     assert c["p"] == 2 and len(c["per_device"]) == 2 and c["transport"] == "ipc"
@@ -61,6 +61,15 @@ def test_two_ranks_same_gpu_line(config, N, b):
         parts = c["partitions"]
         for name in ("fpm", "cpm_ncal", "homogeneous"):
             assert parts[name]["t_s"] > 0 and sum(parts[name]["d"]) == (N // b) ** 2
+        assert "hetero" not in d   # the line is itself the heterogeneity run
+    else:   # N > 1 lines carry config 4 run across the job's ranks (here at N = 4096)
+        h = d["hetero"]
+        assert "error" not in h, h
+        assert h["N"] == 4096 and h["b"] == 512 and h["sm_caps"] == [144, 128]
+        for name in ("fpm", "cpm_ncal", "homogeneous"):
+            assert h[name]["t_s"] > 0 and sum(h[name]["d"]) == (4096 // 512) ** 2
+            assert h[name]["pct_of_capped_peak"] > 0
+        assert h["capped_aggregate_peak_tflops"] > 0 and h["transport"] == "ipc"
 
 
 def test_nccl_transport_one_rank_line():

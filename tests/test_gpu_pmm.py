@@ -401,6 +401,34 @@ def test_per_device_span_stats():
 
 
 @pytest.mark.parametrize("graph", [1, 0])
+def test_group_times_timeline(graph):
+    """pmm_group_times: one (staging start, end, update start, end) record per
+    update group; each interval ordered, a group's update starts after its own
+    staging ended, updates follow each other on the compute stream, and their
+    summed length is the per-device update time of pmm_stats."""
+    N, b = 2048, 256
+    n = N // b
+    rects = pkg.colpart_arrange(n, [40, 24])
+    with pkg.Context.local([0, 0]) as ctx:
+        ctx.set_option("graph", graph)
+        ctx.setup(N, b, rects, pkg.FPM_F32)
+        ctx.fill_synthetic(1, 2, pkg.FPM_DIST_PM1)
+        ctx.compute()
+        st = ctx.compute()
+        for dev in range(2):
+            tl = ctx.group_times(dev)
+            assert len(tl) == st.updates
+            prev_end = 0.0
+            for p0, p1, u0, u1 in tl:
+                assert 0.0 <= p0 <= p1 <= u0 <= u1 <= st.t_compute_s * 1.001
+                assert u0 >= prev_end * 0.999999
+                prev_end = u1
+            assert sum(u1 - u0 for _, _, u0, u1 in tl) == pytest.approx(st.per_dev_update_s[dev], rel=1e-4)
+        with pytest.raises(pkg.FpmError):
+            ctx.group_times(5)
+
+
+@pytest.mark.parametrize("graph", [1, 0])
 def test_shared_b_operand_bit_identical(graph):
     """Option share_b (default on): column members on the B owner's GPU read its
     staged B operand.  The operand is the same bytes either way (same rows,
