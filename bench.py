@@ -319,6 +319,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
         c.set_option("chunk_k", args.chunk_k)
         c.set_option("raster_snake", args.raster_snake)
         c.set_option("share_b", args.share_b)
+        c.set_option("fused_staging", args.fused_staging)
         c.set_option("fuse", args.fuse)
         c.set_option("tail_stream", args.tail_stream)
         c.set_option("e2e_tail", args.e2e_tail)
@@ -583,6 +584,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
             extra_config={
                 "config": args.config, "cta_group": args.cta_group, "raster_group": args.raster_group,
                 "kernel_variant": args.kernel_variant, "chunk_k": args.chunk_k, "raster_snake": args.raster_snake,
+                "fused_staging": args.fused_staging,
                 "fuse": args.fuse,
                 "update_launches_per_step": st.updates, "transport": transport,
                 "fpm_sample_s": t_sample, "fpm_sizes": sizes, "fpm_models": fpm_source,
@@ -839,6 +841,8 @@ def main():
     ap.add_argument("--l2-hint-b", type=int, default=0, help="0 evict_normal, 1 evict_first, 2 evict_last")
     ap.add_argument("--kernel-variant", type=int, default=-1, help="update kernel smem split (-1 auto, 0..3)")
     ap.add_argument("--raster-snake", type=int, default=0, help="serpentine raster over groups (0/1)")
+    ap.add_argument("--fused-staging", type=int, default=1,
+                    help="resident k-loop: the update kernel's staging warp stages the next group (0/1)")
     ap.add_argument("--share-b", type=int, default=1,
                     help="column members on the B owner's GPU read its staged B operand (0/1; local contexts)")
     ap.add_argument("--chunk-k", type=int, default=0, help="K per TMEM accumulation (variants 7/8; 0 auto = 512)")

@@ -17,6 +17,41 @@ enum class SplitScheme : int {
     F16I8 = 3,   // x 2^e = h0 + h1; h0 h0' in kind::f16 + 32 (q l' + l q') in kind::i8 (update_f32.cu)
 };
 
+// The next update group's F16X3 staging, run by a staging warp of
+// the chunked update kernel (variants 7 / 8) while its MMAs run: the persistent
+// update holds every SM, so standalone staging kernels could only run between
+// two updates (measured: 0.44 ms per group at c5, 1.9 % of the step).  The
+// arithmetic is the standalone kernels' (split_math.cuh), so the staged
+// operands are the same bits.  A: pieces of the device's rows, each nseg
+// segments of K elements (segment j of row r at src + j seg_stride + r lda),
+// written to rows row_off.. of a_hi / a_lo (row stride ld_out) with their
+// inverse scales in sa.  B: the block-row(s) b_src (Kb x W, row stride ldb)
+// transposed into b_hi / b_lo (W x Kb, row stride Kb), column maxima in bmax,
+// inverse scales in sb.  ctr: two zeroed counters for the grid barrier between
+// the maxima and the split of B (the kernel leaves them zeroed).
+constexpr int kMaxStagePieces = 16;
+struct StagePiece {
+    const float* src;
+    int64_t seg_stride, row_off, rows;
+};
+struct StageJob {
+    int active = 0;
+    int npieces = 0;
+    int nseg = 1;
+    int64_t K = 0, lda = 0, ld_out = 0;
+    StagePiece a[kMaxStagePieces] = {};
+    void* a_hi = nullptr;
+    void* a_lo = nullptr;
+    float* sa = nullptr;
+    const float* b_src = nullptr;
+    int64_t ldb = 0, Kb = 0, W = 0;
+    void* b_hi = nullptr;
+    void* b_lo = nullptr;
+    float* sb = nullptr;
+    unsigned* bmax = nullptr;
+    unsigned* ctr = nullptr;
+};
+
 struct UpdateArgs {
     const void* a_hi;   // M x K, K-major (row-major, ld = K), fp16 or tf32-in-fp32
     const void* a_lo;
@@ -41,6 +76,7 @@ struct UpdateArgs {
     int chunk_k = 0;         // variants 7 / 8: K per TMEM accumulation (0 auto = 512); each chunk's
                              // sum is drained and added to a per-thread FP32 register sum, so the
                              // tensor-core accumulation error stays that of a short K (DESIGN Q15c)
+    StageJob stage;          // variants 7 / 8, F16X3: the next group's staging (inactive by default)
 };
 
 // C += A . Bt^T  (the rank-b update)

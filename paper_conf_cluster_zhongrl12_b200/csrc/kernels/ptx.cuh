@@ -306,5 +306,16 @@ __host__ __device__ constexpr uint32_t idesc_s32acc_s8(int M, int N) {
 __device__ __forceinline__ void named_bar_sync(uint32_t id, uint32_t nthreads) {
     asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
+// Named barrier 1 or 2 (warp-uniform `which`), each with immediate operands: a
+// barrier id held in a register makes ptxas reserve all 16 barriers of the CTA,
+// and a CTA holding all 16 keeps every other kernel's CTAs off its SM (measured:
+// the staging kernels then wait for the persistent update to finish).
+template <int NT>
+__device__ __forceinline__ void bar_sync_1or2(uint32_t which) {
+    if (which == 0)
+        asm volatile("bar.sync 1, %0;" ::"n"(NT) : "memory");
+    else
+        asm volatile("bar.sync 2, %0;" ::"n"(NT) : "memory");
+}
 
 }  // namespace fpm::ptx

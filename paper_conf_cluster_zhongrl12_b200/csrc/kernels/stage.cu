@@ -9,6 +9,7 @@
 #include <cstdint>
 
 #include "kernels.hpp"
+#include "split_math.cuh"
 
 namespace fpm {
 
@@ -20,19 +21,6 @@ __device__ __forceinline__ float tf32_rna(float x) {
     return __uint_as_float(r);
 }
 
-__device__ __forceinline__ float warp_max(float v) {
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) v = fmaxf(v, __shfl_xor_sync(0xffffffffu, v, o));
-    return v;
-}
-
-// Power-of-two F16X3 scale 2^s that puts the maximum m in [2^14, 2^15).
-__device__ __forceinline__ int f16x3_shift(float m) {
-    int e = 0;
-    if (m > 0.0f) frexpf(m, &e);  // m < 2^e
-    int s = (m > 0.0f) ? 15 - e : 0;
-    return s < -126 ? -126 : (s > 127 ? 127 : s);
-}
 
 // F16I8 codes of a scaled element xs = x 2^s (update_f32.cu): h0 = fp16_rn(xs),
 // q = clamp(rint(xs / 256), +-127), l = rint(8 (xs - h0)) (|l| <= 64).
@@ -98,8 +86,7 @@ __global__ void __launch_bounds__(256) split_rows_f16(const float* __restrict__ 
                 if constexpr (I8) {
                     h[q] = f16i8_codes(x[q], qc[q], lc[q]);
                 } else {
-                    h[q] = __float2half_rn(x[q]);
-                    l[q] = __float2half_rn(x[q] - __half2float(h[q]));
+                    f16x3_split((&v.x)[q], scale, h[q], l[q]);
                 }
             }
             h2[2 * i] = __halves2half2(h[0], h[1]);
@@ -148,9 +135,15 @@ __global__ void __launch_bounds__(256) split_rows_tf32(const float* __restrict__
 // the persistent update kernel (they waited for it to finish, even with the
 // max-shared carveout and ~34 KB left per SM), while these must run under it.
 // A warp reads 8 rows x 32 columns (128 B coalesced per row; lane = column),
-// each lane writes its column's 8 values as 16 B of output row `column`; the 8
-// warps of a CTA fill 128 B of each output row, merged into full sectors in L2.
-constexpr int kColTileK = 64;     // rows of B (= K of the output) per CTA: 8 warps x 8 rows
+// each lane writes its column's 8 values as 16 B of output row `column`; the 4
+// warps of a CTA fill 64 B of each output row, merged into full sectors in L2.
+// The split runs in CTAs of 128 threads: it needs ~60 registers per thread, and
+// the persistent update (320 threads x 168 registers) leaves 11 776 registers
+// of an SM free -- 4 warps fit beside it, 8 did not, so a 256-thread split
+// waited for the update to finish (measured: 0.41 ms exposed per update group
+// at c5, pmm_group_times).
+constexpr int kColTileK = 32;     // rows of B (= K of the output) per CTA: 4 warps x 8 rows
+constexpr int kColThreads = 128;
 constexpr int kColMaxRows = 256;  // rows per CTA of the maxima pass: 8 warps x 32 rows
 constexpr int kColsPerCta = 128;  // 32 lanes x 4 columns (float4 loads)
 
@@ -184,7 +177,7 @@ __global__ void __launch_bounds__(256) colmax_tile_k(const float* __restrict__ s
 // I8 (F16I8): `lo` holds int8 codes as 128-byte rows per 64-wide k-block:
 // [l of the 64 | q of the 64] (the B side of the cross-term product).
 template <bool F16, bool I8 = false>
-__global__ void __launch_bounds__(256) split_cols_t(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
+__global__ void __launch_bounds__(kColThreads) split_cols_t(const float* __restrict__ src, int64_t ld, int64_t K, int64_t W,
                                                     int64_t ld_out, void* __restrict__ hi, void* __restrict__ lo,
                                                     const unsigned* __restrict__ m_bits,
                                                     float* __restrict__ inv_scale) {
@@ -216,8 +209,7 @@ __global__ void __launch_bounds__(256) split_cols_t(const float* __restrict__ sr
                 if constexpr (I8) {
                     h[i] = f16i8_codes(xs, qc[i], lc[i]);
                 } else {
-                    h[i] = __float2half_rn(xs);
-                    l[i] = __float2half_rn(xs - __half2float(h[i]));
+                    f16x3_split(x[c][i], scale, h[i], l[i]);
                 }
             }
             *reinterpret_cast<uint4*>(static_cast<__half*>(hi) + orow) = *reinterpret_cast<uint4*>(h);
@@ -344,7 +336,14 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, bool va
     asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;" ::"r"(s), "l"(gmem), "r"(n) : "memory");
 }
 
-__device__ __forceinline__ void group_bar(int id) { asm volatile("bar.sync %0, %1;" ::"r"(id), "n"(F64_GT) : "memory"); }
+// named barrier 1 + grp with immediate operands (a register id would reserve
+// all 16 barriers of the CTA and keep other kernels off the SM)
+__device__ __forceinline__ void group_bar(int grp) {
+    if (grp == 0)
+        asm volatile("bar.sync 1, %0;" ::"n"(F64_GT) : "memory");
+    else
+        asm volatile("bar.sync 2, %0;" ::"n"(F64_GT) : "memory");
+}
 
 // A may be segmented along K (fused pivots, each pivot's H x b panel stored on
 // its own): element (r, k) at A + (k / seg) * seg_stride + r * lda + k % seg.
@@ -415,7 +414,7 @@ __global__ void __launch_bounds__(F64_THREADS, 1) update_f64_k(const double* __r
 
         for (int64_t kb = 0; kb < nk; ++kb) {
             asm volatile("cp.async.wait_group %0;" ::"n"(F64_ST - 2) : "memory");
-            group_bar(1 + grp);  // chunk visible to the group; the slot refilled next is free
+            group_bar(grp);  // chunk visible to the group; the slot refilled next is free
             advance_load();
             const double* as = As + slot_c * F64_BM * F64_LD;
             const double* bs = Bs + slot_c * F64_BN * F64_LD;
@@ -545,18 +544,18 @@ void launch_split_cols(const float* src, int64_t ld, int64_t K, int64_t W, Split
         if (i8) FPM_CHECK_ARG(K % 64 == 0 && ld_out % 64 == 0, "F16I8 split: K and ld_out multiples of 64");
         auto kern = i8 ? split_cols_t<true, true> : split_cols_t<true, false>;
         if (given_max) {
-            kern<<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, given_max, inv_scale);
+            kern<<<grid, kColThreads, 0, st>>>(src, ld, K, W, ld_out, hi, lo, given_max, inv_scale);
         } else {  // maxima into inv_scale (as bits), split, then bits -> inverse scales in place
             unsigned* bits = reinterpret_cast<unsigned*>(inv_scale);
             const cudaError_t e = cudaMemsetAsync(bits, 0, (size_t)W * sizeof(unsigned), st);
             if (e != cudaSuccess) fail(FPM_ECUDA, "split_cols memset: %s", cudaGetErrorString(e));
             launch_colmax(src, ld, K, W, bits, st);
-            kern<<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, bits, nullptr);
+            kern<<<grid, kColThreads, 0, st>>>(src, ld, K, W, ld_out, hi, lo, bits, nullptr);
             check_launch("split_cols");
             scale_from_max_k<<<(unsigned)((W + 255) / 256), 256, 0, st>>>(inv_scale, W);
         }
     } else {
-        split_cols_t<false><<<grid, 256, 0, st>>>(src, ld, K, W, ld_out, hi, lo, nullptr, nullptr);
+        split_cols_t<false><<<grid, kColThreads, 0, st>>>(src, ld, K, W, ld_out, hi, lo, nullptr, nullptr);
     }
     check_launch("split_cols");
 }

@@ -36,6 +36,7 @@
 
 #include "kernels.hpp"
 #include "ptx.cuh"
+#include "split_math.cuh"
 
 namespace fpm {
 
@@ -75,6 +76,7 @@ struct UpdParams {
     int prof;         // F16I8: accumulate MMA-issuer wait cycles into g_hyb_prof (fpm_k_prof)
     int chunk_kb;     // chunked kernel: k-blocks per TMEM accumulation
     int snake;        // chunked kernel: serpentine raster over groups
+    StageJob stg;     // chunked kernel, F16X3: the next group's staging (staging warp)
 };
 
 // Diagnostic counters of the F16I8 MMA issuer (leader CTAs, lane 0), summed over
@@ -356,6 +358,134 @@ __global__ void __launch_bounds__(192, 1)
 }
 
 
+// ---------------------------------------------------- staging warp (StageJob)
+__device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
+    unsigned v;
+    asm volatile("ld.acquire.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(p) : "memory");
+    return v;
+}
+
+// One warp per CTA stages the next update group while this one's MMAs run
+// (kernels.hpp StageJob): B column maxima (one warp per 128-column chunk over
+// all Kb rows, so plain stores, no atomics), the A rows (warp per row: maximum
+// over the fused row, then the split -- split_rows_f16), a grid barrier over
+// the staging warps (every CTA of the persistent grid is resident), then B's
+// split + transpose in (128 columns) x (8 rows) units (split_cols_t) with the
+// inverse scales.  Same arithmetic as the standalone kernels (split_math.cuh).
+__device__ __forceinline__ unsigned __halves2ushort2(__half a, __half b) {
+    return (unsigned)__half_as_ushort(a) | ((unsigned)__half_as_ushort(b) << 16);
+}
+
+__device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int ncta, int lane) {
+    const int64_t nchunks = (J.W + 127) / 128;
+    // ---- B: column maxima
+    for (int64_t ch = cta; ch < nchunks; ch += ncta) {
+        const int64_t col = ch * 128 + 4 * lane;
+        if (col < J.W) {  // W % 4 == 0: a lane's four columns are all in or all out
+            float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
+            const float* p = J.b_src + col;
+#pragma unroll 8
+            for (int64_t k = 0; k < J.Kb; ++k) {
+                const float4 v = __ldcs(reinterpret_cast<const float4*>(p + k * J.ldb));
+                m.x = fmaxf(m.x, fabsf(v.x));
+                m.y = fmaxf(m.y, fabsf(v.y));
+                m.z = fmaxf(m.z, fabsf(v.z));
+                m.w = fmaxf(m.w, fabsf(v.w));
+            }
+            *reinterpret_cast<uint4*>(J.bmax + col) =
+                make_uint4(__float_as_uint(m.x), __float_as_uint(m.y), __float_as_uint(m.z), __float_as_uint(m.w));
+        }
+    }
+    // ---- A: rows of every piece (one warp per row)
+    int64_t rtot = 0;
+    for (int i = 0; i < J.npieces; ++i) rtot += J.a[i].rows;
+    const int64_t n4 = J.K / 4;
+    for (int64_t g = cta; g < rtot; g += ncta) {
+        int pi = 0;
+        int64_t r = g;
+        while (r >= J.a[pi].rows) r -= J.a[pi++].rows;
+        const StagePiece& pc = J.a[pi];
+        float m = 0.0f;
+        for (int j = 0; j < J.nseg; ++j) {
+            const float4* s4 = reinterpret_cast<const float4*>(pc.src + j * pc.seg_stride + r * J.lda);
+#pragma unroll 4
+            for (int64_t i = lane; i < n4; i += 32) {
+                const float4 v = s4[i];
+                m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+            }
+        }
+        m = warp_max(m);
+        const int sh = f16x3_shift(m);
+        const float scale = ldexpf(1.0f, sh);
+        const int64_t orow = pc.row_off + r;
+        if (lane == 0) J.sa[orow] = ldexpf(1.0f, -sh);
+        for (int j = 0; j < J.nseg; ++j) {
+            const float4* s4 = reinterpret_cast<const float4*>(pc.src + j * pc.seg_stride + r * J.lda);
+            __half2* h2 = reinterpret_cast<__half2*>(static_cast<__half*>(J.a_hi) + orow * J.ld_out + j * J.K);
+            __half2* l2 = reinterpret_cast<__half2*>(static_cast<__half*>(J.a_lo) + orow * J.ld_out + j * J.K);
+#pragma unroll 4
+            for (int64_t i = lane; i < n4; i += 32) {
+                const float4 v = __ldcs(s4 + i);
+                __half h[4], l[4];
+#pragma unroll
+                for (int q = 0; q < 4; ++q) f16x3_split((&v.x)[q], scale, h[q], l[q]);
+                // streaming stores: the staged halves must not push the running
+                // update's raster-group operands out of L2
+                __stcs(reinterpret_cast<uint2*>(h2) + i, make_uint2(__halves2ushort2(h[0], h[1]), __halves2ushort2(h[2], h[3])));
+                __stcs(reinterpret_cast<uint2*>(l2) + i, make_uint2(__halves2ushort2(l[0], l[1]), __halves2ushort2(l[2], l[3])));
+            }
+        }
+    }
+    // ---- grid barrier: every staging warp's B maxima are written
+    __syncwarp();
+    if (lane == 0) {
+        __threadfence();
+        atomicAdd(J.ctr, 1u);
+        while (ld_acquire_u32(J.ctr) < (unsigned)ncta) __nanosleep(256);
+    }
+    __syncwarp();
+    // ---- B: split + transpose, (128 columns) x (8 rows of Kb) per unit
+    const int64_t nk8 = J.Kb / 8;
+    const int64_t units = nchunks * nk8;
+    for (int64_t u = cta; u < units; u += ncta) {
+        const int64_t ch = u / nk8, kk = (u - ch * nk8) * 8;
+        const int64_t col = ch * 128 + 4 * lane;
+        if (col >= J.W) continue;
+        float x[4][8];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {
+            const float4 v = __ldcs(reinterpret_cast<const float4*>(J.b_src + (kk + i) * J.ldb + col));
+            x[0][i] = v.x;
+            x[1][i] = v.y;
+            x[2][i] = v.z;
+            x[3][i] = v.w;
+        }
+        const uint4 mb = __ldcg(reinterpret_cast<const uint4*>(J.bmax + col));
+        const unsigned mbits[4] = {mb.x, mb.y, mb.z, mb.w};
+#pragma unroll
+        for (int c = 0; c < 4; ++c) {
+            const int sh = f16x3_shift(__uint_as_float(mbits[c]));
+            const float scale = ldexpf(1.0f, sh);
+            if (kk == 0) J.sb[col + c] = ldexpf(1.0f, -sh);
+            __align__(16) __half h[8], l[8];
+#pragma unroll
+            for (int i = 0; i < 8; ++i) f16x3_split(x[c][i], scale, h[i], l[i]);
+            const int64_t orow = (col + c) * J.Kb + kk;
+            __stcs(reinterpret_cast<uint4*>(static_cast<__half*>(J.b_hi) + orow), *reinterpret_cast<uint4*>(h));
+            __stcs(reinterpret_cast<uint4*>(static_cast<__half*>(J.b_lo) + orow), *reinterpret_cast<uint4*>(l));
+        }
+    }
+    // ---- departure: the last staging warp re-arms the barrier for the next launch
+    __syncwarp();
+    if (lane == 0) {
+        const unsigned d = atomicAdd(J.ctr + 1, 1u);
+        if (d == (unsigned)ncta - 1) {
+            J.ctr[0] = 0;
+            J.ctr[1] = 0;
+        }
+    }
+}
+
 // ------------------------------------ F16X3 / TF32X3, chunked accumulation (default)
 // The tensor cores add every MMA's products into the FP32 accumulator with a
 // truncated (not round-to-nearest) alignment, so the accumulation error of one
@@ -374,6 +504,7 @@ __global__ void __launch_bounds__(192, 1)
 //   warp 0: TMA producer (A hi/lo, B^T hi/lo k-blocks, 128-byte swizzle)
 //   warp 1: TMEM allocation + single-thread tcgen05.mma issuer (leader CTA)
 //   warps 2-9: epilogue
+//   warp 10: staging of the next update group (StageJob, when given)
 template <int KIND, int STAGES, int NCB>
 struct AccCfg {
     static constexpr int BM = 128, TILE_M = 256, BN = 256, BN_CTA = 128, SW = 128;
@@ -387,16 +518,16 @@ struct AccCfg {
     static constexpr int BAR_BYTES = 8 * (2 * STAGES + 4) + 16;
     static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + NCB * C_CHUNK_BYTES + BAR_BYTES;
     static constexpr uint32_t IDESC = ptx::idesc_f32acc(TILE_M, BN, KIND == 1);
-    static constexpr int THREADS = 320;
+    static constexpr int THREADS = 352;  // producer, MMA, 8 epilogue warps, staging warp
     static_assert(NCB % 2 == 0 && NCBH >= 1 && NCBH <= 4, "C staging: 1..4 chunks per half");
     static_assert(SMEM <= 232448, "shared memory budget");
 };
 
 template <int KIND, int STAGES, int NCB>
-__global__ void __launch_bounds__(320, 1)
+__global__ void __maxnreg__(168)
     update_acc_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
                       const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
-                      const __grid_constant__ CUtensorMap tmC, const UpdParams P) {
+                      const __grid_constant__ CUtensorMap tmC, const __grid_constant__ UpdParams P) {
     using Cfg = AccCfg<KIND, STAGES, NCB>;
     extern __shared__ uint8_t smem_raw[];
     uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) & ~uintptr_t(1023));
@@ -514,6 +645,9 @@ __global__ void __launch_bounds__(320, 1)
                 }
             }
         }
+    } else if (warp == 10) {
+        // ------------------------------------------------ staging of the next group
+        if (P.stg.active) stage_next_group(P.stg, blockIdx.x, gridDim.x, lane);
     } else {
         // -------------------------------------------------------------- epilogue
         const uint32_t e = threadIdx.x - 64;  // 0..255
@@ -521,7 +655,6 @@ __global__ void __launch_bounds__(320, 1)
         const uint32_t eh = e % 128;
         const uint32_t q = warp & 3;          // TMEM lane quarter this warp may access
         const uint32_t r = q * 32 + lane;     // row of the CTA tile
-        const uint32_t bar_id = 1 + hh;
         uint8_t* cb = cbuf + hh * Cfg::NCBH * Cfg::C_CHUNK_BYTES;
         int it = 0;
         for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
@@ -582,14 +715,14 @@ __global__ void __launch_bounds__(320, 1)
                 }
                 // the buffer's previous TMA (chunk c - NCBH) has read it
                 if (eh == 0) ptx::bulk_wait_read_n<Cfg::NCBH - 1>();
-                ptx::named_bar_sync(bar_id, 128);
+                ptx::bar_sync_1or2<128>(hh);
                 uint8_t* rowp = cb + buf * Cfg::C_CHUNK_BYTES + r * 128;
 #pragma unroll
                 for (int j = 0; j < 8; ++j)
                     *reinterpret_cast<float4*>(rowp + ((j ^ (r & 7)) << 4)) =
                         make_float4(v[4 * j + 0], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
                 ptx::fence_proxy_async_smem();
-                ptx::named_bar_sync(bar_id, 128);
+                ptx::bar_sync_1or2<128>(hh);
                 if (eh == 0) {
                     if (P.load_c)
                         ptx::tma_reduce_add_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
@@ -820,7 +953,6 @@ __global__ void __launch_bounds__(320, 1)
         const uint32_t eh = e % 128;
         const uint32_t q = warp & 3;          // TMEM lane quarter
         const uint32_t r = q * 32 + lane;     // row of the CTA tile
-        const uint32_t bar_id = 1 + hh;
         uint8_t* cb = cbuf + hh * Cfg::NCBH * Cfg::C_CHUNK_BYTES;
         uint64_t* cf = cfull + hh * Cfg::NCBH;
         uint32_t cpar = 0;
@@ -898,7 +1030,7 @@ __global__ void __launch_bounds__(320, 1)
                     cpar ^= 1u << buf;
                 } else {
                     if (eh == 0) ptx::bulk_wait_read_n<Cfg::NCBH - 1>();
-                    ptx::named_bar_sync(bar_id, 128);
+                    ptx::bar_sync_1or2<128>(hh);
                 }
                 uint8_t* rowp = cb + buf * Cfg::C_CHUNK_BYTES + r * 128;
 #pragma unroll
@@ -913,7 +1045,7 @@ __global__ void __launch_bounds__(320, 1)
                     *p4 = cv;
                 }
                 ptx::fence_proxy_async_smem();
-                ptx::named_bar_sync(bar_id, 128);
+                ptx::bar_sync_1or2<128>(hh);
                 if (eh == 0) {
                     if (RED && P.load_c)
                         ptx::tma_reduce_add_2d_hint(&tmC, cb + buf * Cfg::C_CHUNK_BYTES, n0 + 32 * c, m0,
@@ -1077,6 +1209,14 @@ static void launch_update_acc_t(const UpdateArgs& a, cudaStream_t st) {
     const int chunk_k = a.chunk_k > 0 ? a.chunk_k : 512;
     P.chunk_kb = (chunk_k + Cfg::BK - 1) / Cfg::BK;
     P.snake = a.raster_snake ? 1 : 0;
+    P.stg = a.stage;
+    if (P.stg.active) {
+        FPM_CHECK_ARG(KIND == 0, "in-kernel staging is F16X3 only");
+        FPM_CHECK_ARG(P.stg.npieces >= 1 && P.stg.npieces <= kMaxStagePieces && P.stg.K % 4 == 0 &&
+                          P.stg.Kb % 8 == 0 && P.stg.W % 4 == 0 && P.stg.ldb % 4 == 0 && P.stg.lda % 4 == 0 &&
+                          P.stg.ctr != nullptr && P.stg.bmax != nullptr,
+                      "bad staging job");
+    }
     auto kern = update_acc_kernel<KIND, STAGES, NCB>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
     int dev = 0;

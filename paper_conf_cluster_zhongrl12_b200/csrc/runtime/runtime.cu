@@ -126,6 +126,11 @@ struct Device {
     std::vector<void*> tail_allocs;
     cudaEvent_t ev_tpack0 = nullptr, ev_tpack1 = nullptr;  // staging of the fused tail (second pass)
     bool tail_fused_run = false;  // the current k-loop stages its tail into kFusedSlot
+    // in-kernel staging (option "fused_staging"): update g stages group g + 1
+    // with its staging warp; B column maxima and the grid-barrier counters
+    bool fs_run = false;
+    unsigned* stg_bmax = nullptr;
+    unsigned* stg_ctr = nullptr;
     // band-streamed tail (pmm_run, one device holding all of A and B): the tail's
     // A rows arrive band by band into tail_rows (H x tail_K, row-major)
     bool tail_streamed_run = false;
@@ -195,6 +200,7 @@ struct pmm_ctx {
     int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
     int64_t tail_band = 2048; // rows of C_i per band of the tail (multiple of 256)
     int tail_fuse = 1;        // local / IPC FP32: the tail as one fused operand (1) or per group (0)
+    int fused_staging = 1;    // resident FP32 F16X3 k-loop: the update kernel stages the next group
     int tail_stream = 1;      // pmm_run on one device: the tail's B rows first, its A rows band by band
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
@@ -411,6 +417,8 @@ void free_problem(Device& d) {
     d.tail_K = d.tail_K_alloc = 0;
     d.tmax_a = d.tmax_b = nullptr;
     d.tail_rows = nullptr;
+    d.stg_bmax = d.stg_ctr = nullptr;
+    d.fs_run = false;
     for (int s = 0; s < kSlots; ++s) {
         d.a_recv[s] = d.b_recv[s] = d.bt[s] = d.a_hi[s] = d.a_lo[s] = d.b_hi[s] = d.b_lo[s] = nullptr;
         d.sa[s] = d.sb[s] = nullptr;
@@ -841,6 +849,11 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
             d.C = dalloc(d, HW * es);
         }
         for (int s = 0; s < 2; ++s) alloc_slot(ctx, d, s);
+        if (dt == FPM_F32) {  // in-kernel staging: B column maxima, grid-barrier counters (zeroed)
+            d.stg_bmax = static_cast<unsigned*>(dalloc(d, (size_t)d.W * sizeof(unsigned)));
+            d.stg_ctr = static_cast<unsigned*>(dalloc(d, 2 * sizeof(unsigned)));
+            CU(cudaMemsetAsync(d.stg_ctr, 0, 2 * sizeof(unsigned), d.s_comp));
+        }
         for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1, &d.ev_up}) {
             v->resize(n);
             for (auto& e : *v) CU(cudaEventCreate(&e));
@@ -1137,6 +1150,82 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
     return tp.phase == 2 ? 0 : bytes;
 }
 
+// In-kernel staging (option "fused_staging", kernels.hpp StageJob) for device d
+// in this k-loop: resident inputs (no host streaming), FP32 F16X3 on the chunked
+// kernel (variants 7 / 8, CTA pairs), local or IPC pulls (not NCCL: its
+// receives complete on their own schedule), C_i in core, the only GPU device of
+// this context on its GPU (the staging warps meet at a grid barrier, so every
+// CTA of the update must be resident at once), and a grid of >= 32 CTAs.
+bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
+    if (!ctx->fused_staging || ctx->dt != FPM_F32 || ctx->nccl_mode || streamed || d.cpu || d.ooc || !d.live())
+        return false;
+    if (scheme_for(ctx, ctx->b) != SplitScheme::F16X3 || ctx->cta_group != 2) return false;
+    if (!(ctx->kernel_variant == -1 || ctx->kernel_variant == 7 || ctx->kernel_variant == 8)) return false;
+    if (!d.stg_bmax || !d.stg_ctr) return false;
+    for (const auto& q : ctx->devs)
+        if (&q != &d && !q.cpu && q.cuda_dev == d.cuda_dev && q.live()) return false;
+    const int64_t tiles = ((d.H + 255) / 256) * ((d.W + 255) / 256);
+    return 2 * std::min<int64_t>(d.num_sms / 2, tiles) >= 32;
+}
+
+// The staging of update group g into operand slot `slot` of device d as a job
+// for the previous update's staging warp: the same sources as issue_comm's
+// FP32 local / IPC path (own panels, or the holders' / owner's resident memory).
+// Returns the pivot bytes pulled from other devices; job.active = 0 when the
+// group has more A pieces than a job holds.
+int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob& J) {
+    const int64_t b = ctx->b;
+    const int64_t k0 = ctx->groups[g].first;
+    const int f = ctx->groups[g].second;
+    const int64_t fb = (int64_t)f * b;
+    const colpart_rect& r = d.rect;
+    int64_t bytes = 0;
+    J = StageJob{};
+    J.nseg = f;
+    J.K = b;
+    J.lda = b;
+    J.ld_out = fb;
+    if (r.col0 <= k0 && k0 < r.col0 + r.w) {  // own block-columns: f panels of H x b
+        J.a[0] = StagePiece{static_cast<const float*>(d.A) + (size_t)(k0 - r.col0) * d.H * b, d.H * b, 0, d.H};
+        J.npieces = 1;
+    } else {
+        for (const Move& m : ctx->plan_a[k0]) {
+            if (m.dst != d.idx) continue;
+            if (J.npieces == kMaxStagePieces) return 0;
+            const colpart_rect& qr = ctx->rects[m.src];
+            const int64_t qH = qr.h * b;
+            const float* src = static_cast<const float*>(src_A(ctx, m.src)) +
+                               ((size_t)(k0 - qr.col0) * qH * b + (size_t)(m.begin - qr.row0) * b * b);
+            J.a[J.npieces++] = StagePiece{src, qH * b, (m.begin - r.row0) * b, (m.end - m.begin) * b};
+            bytes += (m.end - m.begin) * b * b * 4 * f;
+        }
+    }
+    if (r.row0 <= k0 && k0 < r.row0 + r.h) {
+        J.b_src = static_cast<const float*>(d.B) + (size_t)(k0 - r.row0) * b * d.W;
+    } else {
+        for (const Move& m : ctx->plan_b[k0]) {
+            if (m.dst != d.idx) continue;
+            const colpart_rect& orr = ctx->rects[m.src];
+            J.b_src = static_cast<const float*>(src_B(ctx, m.src)) + (size_t)(k0 - orr.row0) * b * d.W;
+            bytes += fb * d.W * 4;
+        }
+    }
+    if (J.npieces == 0 || J.b_src == nullptr) return 0;
+    J.ldb = d.W;
+    J.Kb = fb;
+    J.W = d.W;
+    J.a_hi = d.a_hi[slot];
+    J.a_lo = d.a_lo[slot];
+    J.sa = d.sa[slot];
+    J.b_hi = d.b_hi[slot];
+    J.b_lo = d.b_lo[slot];
+    J.sb = d.sb[slot];
+    J.bmax = d.stg_bmax;
+    J.ctr = d.stg_ctr;
+    J.active = 1;
+    return bytes;
+}
+
 // FP32 update of group g from operand slot `slot` over all of C_i.
 UpdateArgs f32_args(pmm_ctx* ctx, const Device& d, int g, int slot) {
     UpdateArgs a;
@@ -1183,11 +1272,17 @@ UpdateArgs band_args(const UpdateArgs& a, int64_t r0, int64_t m, float* Cband) {
     return x;
 }
 
-void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
+void issue_update(pmm_ctx* ctx, Device& d, int g, int slot, const StageJob* next = nullptr,
+                  bool staged_in_kernel = false) {
     const int64_t k0 = ctx->groups[g].first;
     const int f = ctx->groups[g].second;
     CU(cudaSetDevice(d.cuda_dev));
-    CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
+    if (staged_in_kernel) {  // update g - 1 staged this group on this stream: nothing to wait for
+        rec_t(d.ev_pack0[g], d.s_comp);
+        rec_t(d.ev_pack1[g], d.s_comp);
+    } else {
+        CU(cudaStreamWaitEvent(d.s_comp, d.ev_ready[slot], 0));
+    }
     if (ctx->dt == FPM_F32 && slot < 2 && d.b_from[slot] != d.idx)  // the owner staged this update's B
         CU(cudaStreamWaitEvent(d.s_comp, local_dev(ctx, d.b_from[slot])->ev_ready[slot], 0));
     rec_t(d.ev_upd0[g], d.s_comp);
@@ -1199,7 +1294,8 @@ void issue_update(pmm_ctx* ctx, Device& d, int g, int slot) {
     bc.kept_head = ctx->ooc_keep && g > 0;
     bc.keep_tail = ctx->ooc_keep && g + 1 < (int)ctx->groups.size();
     if (ctx->dt == FPM_F32) {
-        const UpdateArgs a = f32_args(ctx, d, g, slot);
+        UpdateArgs a = f32_args(ctx, d, g, slot);
+        if (next) a.stage = *next;
         if (d.ooc) {
             // out of core: the same update, one row band of C_i at a time (rows
             // r0.. of the A operand and its scales, the band buffer as C)
@@ -1743,6 +1839,10 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     };
     // band-streamed tail: its uploads, staging and updates are issued after the loop
     auto streamed_tail = [&](const Device& d, int g) { return in_tail(d, g) && d.tail_streamed_run; };
+    // in-kernel staging: group g >= 1 (not in the tail) was staged by update g - 1
+    for (auto& d : ctx->devs) d.fs_run = fused_staging_ok(ctx, d, streamed);
+    auto staged_in_kernel = [&](const Device& d, int g) { return d.fs_run && g >= 1 && !in_tail(d, g); };
+    std::vector<char> job_ok(ctx->devs.size(), 0);  // the previous update carried this group's job
     for (int g = 0; g < ngroups; ++g) {
         const int64_t k0 = ctx->groups[g].first;
         if (streamed)
@@ -1762,8 +1862,9 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
             }
             continue;
         }
-        for (auto& d : ctx->devs)
-            if (d.live() && !d.cpu && !streamed_tail(d, g)) {
+        for (size_t di = 0; di < ctx->devs.size(); ++di) {
+            Device& d = ctx->devs[di];
+            if (d.live() && !d.cpu && !streamed_tail(d, g) && !(staged_in_kernel(d, g) && job_ok[di])) {
                 const int slot = slot_of(d, g);
                 if (in_tail(d, g) && d.tail_fused_run) {  // fused tail, pass 1: merge the maxima
                     if (g == gt) {
@@ -1775,8 +1876,22 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
                     bytes += issue_comm(ctx, d, g, slot, g < 2 && slot < 2, streamed, TailPhase{}, g < gt);
                 }
             }
-        for (auto& d : ctx->devs)
-            if (d.live() && !d.cpu && !in_tail(d, g)) issue_update(ctx, d, g, g & 1);
+        }
+        for (size_t di = 0; di < ctx->devs.size(); ++di) {
+            Device& d = ctx->devs[di];
+            if (!d.live() || d.cpu || in_tail(d, g)) continue;
+            const bool here = staged_in_kernel(d, g) && job_ok[di];
+            StageJob job;
+            job_ok[di] = 0;
+            if (d.fs_run && g + 1 < ngroups && !in_tail(d, g + 1)) {
+                const int64_t nb = build_stage_job(ctx, d, g + 1, (g + 1) & 1, job);
+                if (job.active) {
+                    bytes += nb;
+                    job_ok[di] = 1;
+                }
+            }
+            issue_update(ctx, d, g, g & 1, job.active ? &job : nullptr, here);
+        }
     }
     // fused tail, pass 2: split every tail group with the merged maxima into its
     // K range of the tail operand
@@ -2841,6 +2956,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
         } else if (k == "share_b") {
             FPM_CHECK_ARG(value == 0 || value == 1, "share_b must be 0 or 1");
             ctx->share_b = (int)value;
+        } else if (k == "fused_staging") {
+            FPM_CHECK_ARG(value == 0 || value == 1, "fused_staging must be 0 or 1");
+            ctx->fused_staging = (int)value;
         } else if (k == "sample_rel_ci_permille") {
             FPM_CHECK_ARG(value >= 1 && value <= 500, "sample_rel_ci_permille must be in [1, 500]");
             ctx->sample_rel_ci = value / 1000.0;

@@ -22,7 +22,7 @@ def _free_port():
         return s.getsockname()[1]
 
 
-def _worker(rank, world, port, rects, N, b, dist_kind, q):
+def _worker(rank, world, port, rects, N, b, dist_kind, q, opts=None):
     import sys
     sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
     import torch.distributed as dist
@@ -34,6 +34,8 @@ def _worker(rank, world, port, rects, N, b, dist_kind, q):
         torch.cuda.set_device(0)
         dist.init_process_group("gloo", init_method=f"tcp://127.0.0.1:{port}", rank=rank, world_size=world)
         with pkg.Context.ipc(rank, world, 0) as ctx:
+            for k, v in (opts or {}).items():
+                ctx.set_option(k, v)
             ctx.setup(N, b, rects, pkg.FPM_F32)
             blobs = [None] * world
             dist.all_gather_object(blobs, ctx.ipc_export())
@@ -41,7 +43,8 @@ def _worker(rank, world, port, rects, N, b, dist_kind, q):
             ctx.fill_synthetic(1, 2, dist_kind)
             torch.cuda.synchronize()
             dist.barrier()                       # every rank's inputs are resident
-            st = ctx.compute()
+            for _ in range(2):                   # repeated: the staging barrier re-arms
+                st = ctx.compute()
             col, r0, c0, h, w = rects[rank]
             ok, err = True, 0.0
             if h * w:
@@ -61,11 +64,12 @@ def _worker(rank, world, port, rects, N, b, dist_kind, q):
         q.put((rank, repr(e), -1.0, -1))
 
 
-def _run(world, rects, N, b, dist_kind):
+def _run(world, rects, N, b, dist_kind, opts=None):
     ctx = mp.get_context("spawn")
     q = ctx.Queue()
     port = _free_port()
-    procs = [ctx.Process(target=_worker, args=(r, world, port, rects, N, b, dist_kind, q)) for r in range(world)]
+    procs = [ctx.Process(target=_worker, args=(r, world, port, rects, N, b, dist_kind, q, opts))
+             for r in range(world)]
     for p in procs:
         p.start()
     out = sorted(q.get(timeout=300) for _ in range(world))
@@ -97,6 +101,21 @@ def test_ipc_three_ranks_mixed_columns():
     rects = pkg.colpart_arrange(n, [70, 44, 30])             # one 2-device column, one 1-device column
     assert len({r[0] for r in rects}) == 2
     out = _run(3, rects, N, b, 1)
+    assert all(ok is True for (_, ok, _, _) in out), out
+
+
+@pytest.mark.parametrize("fused", [1, 0])
+def test_ipc_fused_staging_pulls_peer_pieces(fused):
+    """In-kernel staging on IPC contexts (the driver's N > 1 bench path): the
+    staging warp of update g pulls group g + 1's A slices from the holders'
+    and B from the owner's resident memory (several pieces per job); integer
+    inputs bit-exact, with the option on and off."""
+    import paper_conf_cluster_zhongrl12_b200 as pkg
+    N, b = 4096, 256
+    n = N // b
+    rects = pkg.colpart_arrange(n, [120, 80, 56])            # a two-device column and a one-device column
+    assert len({r[0] for r in rects}) == 2
+    out = _run(3, rects, N, b, 1, {"fused_staging": fused})
     assert all(ok is True for (_, ok, _, _) in out), out
 
 

@@ -428,6 +428,38 @@ def test_group_times_timeline(graph):
             ctx.group_times(5)
 
 
+@pytest.mark.parametrize("N,b,fuse", [(3072, 256, 0), (2880, 96, 3), (4096, 512, 1), (1024, 128, 2)])
+@pytest.mark.parametrize("graph", [1, 0])
+def test_fused_staging_bit_identical(N, b, fuse, graph):
+    """Option fused_staging (default on): update g's staging warp stages group
+    g + 1 (kernels.hpp StageJob) instead of the standalone split kernels between
+    the updates.  Same arithmetic (split_math.cuh), so C is bit-identical with
+    the option off, eager or graph-replayed, with ragged column chunks (W not a
+    multiple of 128), one / several pivots per update, and repeated computes
+    (the grid-barrier counters re-arm); and C matches the oracle."""
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n])
+    out = []
+    for fs in (1, 0):
+        with pkg.Context.local([0]) as ctx:
+            ctx.set_option("graph", graph)
+            ctx.set_option("fuse", fuse)
+            ctx.set_option("fused_staging", fs)
+            ctx.setup(N, b, rects, pkg.FPM_F32)
+            ctx.fill_synthetic(1, 2, pkg.FPM_DIST_PM1)
+            for _ in range(3):
+                st = ctx.compute()
+            C = np.empty((N, N), np.float32)
+            ctx.download(C, N)
+            out.append((C, st.kernel_launches, ctx.group_times(0)))
+    assert np.array_equal(out[0][0], out[1][0])
+    assert out[0][1] < out[1][1]          # no standalone staging kernels after the first group
+    tl = out[0][2]
+    assert all(p1 - p0 < 1e-4 for p0, p1, _, _ in tl[1:])   # staged inside the updates (no staging interval)
+    ref = og.gemm(synth.rect(1, N, 0, 0, N, N), synth.rect(2, N, 0, 0, N, N))
+    assert og.rel_fro(out[0][0], ref) <= 1e-5
+
+
 @pytest.mark.parametrize("graph", [1, 0])
 def test_shared_b_operand_bit_identical(graph):
     """Option share_b (default on): column members on the B owner's GPU read its
