@@ -50,6 +50,12 @@ struct StageJob {
     float* sb = nullptr;
     unsigned* bmax = nullptr;
     unsigned* ctr = nullptr;
+    // streamed inputs (pmm_run): progress flags of the devices holding this
+    // group's pieces (own, local or IPC peer memory) that must reach `need`
+    // ((epoch << 16) | (last pivot + 1)) before the staging reads them
+    int nwait = 0;
+    const unsigned long long* wait_flag[kMaxStagePieces + 1] = {};
+    unsigned long long need = 0;
 };
 
 struct UpdateArgs {

@@ -376,8 +376,19 @@ __device__ __forceinline__ unsigned __halves2ushort2(__half a, __half b) {
     return (unsigned)__half_as_ushort(a) | ((unsigned)__half_as_ushort(b) << 16);
 }
 
+__device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned long long* p) {
+    unsigned long long v;
+    asm volatile("ld.acquire.sys.global.u64 %0, [%1];" : "=l"(v) : "l"(p) : "memory");
+    return v;
+}
+
 __device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int ncta, int lane) {
     const int64_t nchunks = (J.W + 127) / 128;
+    // streamed inputs: wait until every holder's panels of the group have landed
+    if (lane == 0)
+        for (int i = 0; i < J.nwait; ++i)
+            while (ld_acquire_sys_u64(J.wait_flag[i]) < J.need) __nanosleep(1000);
+    __syncwarp();
     // ---- B: column maxima
     for (int64_t ch = cta; ch < nchunks; ch += ncta) {
         const int64_t col = ch * 128 + 4 * lane;

@@ -200,7 +200,8 @@ struct pmm_ctx {
     int e2e_tail = -1;        // groups of the download-overlapped tail (-1 auto, 0 off)
     int64_t tail_band = 2048; // rows of C_i per band of the tail (multiple of 256)
     int tail_fuse = 1;        // local / IPC FP32: the tail as one fused operand (1) or per group (0)
-    int fused_staging = 1;    // resident FP32 F16X3 k-loop: the update kernel stages the next group
+    int fused_staging = 1;    // FP32 F16X3 k-loop: the update kernel stages the next group
+    bool stream_flags = false;  // this streamed run writes upload-progress flags (in-kernel staging)
     int tail_stream = 1;      // pmm_run on one device: the tail's B rows first, its A rows band by band
     int sm_partition = 0;     // 0: SM caps as persistent grid sizes; 1: green-context partitions
     int ooc_buffers = 8;      // out-of-core: up to R band buffers in the C cap (2 = the paper's C0, C1)
@@ -926,7 +927,9 @@ void issue_upload(pmm_ctx* ctx, Device& d, int64_t k, const HostSrc& h) {
         CU(cudaMemcpy2DAsync(dst, d.W * es, src, h.ld * es, d.W * es, b, cudaMemcpyHostToDevice, d.s_up));
     }
     CU(cudaEventRecord(d.ev_up[k], d.s_up));
-    if (ctx->ipc_mode)  // peers pulling this rank's panels wait for the flag (after the copies above)
+    // peers pulling this rank's panels (IPC) and in-kernel staging wait for the
+    // flag (after the copies above)
+    if (ctx->ipc_mode || ctx->stream_flags)
         if (stream_mem_ops().write64(reinterpret_cast<CUstream>(d.s_up), reinterpret_cast<CUdeviceptr>(d.up_flag),
                                      flag_value(ctx->epoch, k), 0) != CUDA_SUCCESS)
             fail(FPM_ECUDA, "cuStreamWriteValue64 failed");
@@ -1156,9 +1159,18 @@ int64_t issue_comm(pmm_ctx* ctx, Device& d, int g, int slot, bool first_use, boo
 // receives complete on their own schedule), C_i in core, the only GPU device of
 // this context on its GPU (the staging warps meet at a grid barrier, so every
 // CTA of the update must be resident at once), and a grid of >= 32 CTAs.
-bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
-    if (!ctx->fused_staging || ctx->dt != FPM_F32 || ctx->nccl_mode || streamed || d.cpu || d.ooc || !d.live())
+bool stream_ops_available() {
+    try {
+        stream_mem_ops();
+        return true;
+    } catch (...) {
         return false;
+    }
+}
+
+bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
+    if (!ctx->fused_staging || ctx->dt != FPM_F32 || ctx->nccl_mode || d.cpu || d.ooc || !d.live()) return false;
+    if (streamed && (has_cpu(ctx) || !stream_ops_available())) return false;
     if (scheme_for(ctx, ctx->b) != SplitScheme::F16X3 || ctx->cta_group != 2) return false;
     if (!(ctx->kernel_variant == -1 || ctx->kernel_variant == 7 || ctx->kernel_variant == 8)) return false;
     if (!d.stg_bmax || !d.stg_ctr) return false;
@@ -1168,12 +1180,21 @@ bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
     return 2 * std::min<int64_t>(d.num_sms / 2, tiles) >= 32;
 }
 
+// The upload-progress flag of device q as device d reads it (own / local
+// device memory, or the IPC peer mapping).
+const unsigned long long* flag_of(pmm_ctx* ctx, const Device& d, int q) {
+    if (q == d.idx) return reinterpret_cast<const unsigned long long*>(d.up_flag);
+    if (ctx->ipc_mode) return reinterpret_cast<const unsigned long long*>(ctx->peer_flag[q]);
+    return reinterpret_cast<const unsigned long long*>(local_dev(ctx, q)->up_flag);
+}
+
 // The staging of update group g into operand slot `slot` of device d as a job
 // for the previous update's staging warp: the same sources as issue_comm's
-// FP32 local / IPC path (own panels, or the holders' / owner's resident memory).
+// FP32 local / IPC path (own panels, or the holders' / owner's resident memory;
+// streamed: after their progress flags show the group's panels landed).
 // Returns the pivot bytes pulled from other devices; job.active = 0 when the
 // group has more A pieces than a job holds.
-int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob& J) {
+int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob& J, bool streamed) {
     const int64_t b = ctx->b;
     const int64_t k0 = ctx->groups[g].first;
     const int f = ctx->groups[g].second;
@@ -1185,9 +1206,17 @@ int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob
     J.K = b;
     J.lda = b;
     J.ld_out = fb;
+    auto wait_for = [&](int q) {
+        if (!streamed) return;
+        const unsigned long long* fl = flag_of(ctx, d, q);
+        for (int i = 0; i < J.nwait; ++i)
+            if (J.wait_flag[i] == fl) return;
+        J.wait_flag[J.nwait++] = fl;
+    };
     if (r.col0 <= k0 && k0 < r.col0 + r.w) {  // own block-columns: f panels of H x b
         J.a[0] = StagePiece{static_cast<const float*>(d.A) + (size_t)(k0 - r.col0) * d.H * b, d.H * b, 0, d.H};
         J.npieces = 1;
+        wait_for(d.idx);
     } else {
         for (const Move& m : ctx->plan_a[k0]) {
             if (m.dst != d.idx) continue;
@@ -1197,19 +1226,23 @@ int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob
             const float* src = static_cast<const float*>(src_A(ctx, m.src)) +
                                ((size_t)(k0 - qr.col0) * qH * b + (size_t)(m.begin - qr.row0) * b * b);
             J.a[J.npieces++] = StagePiece{src, qH * b, (m.begin - r.row0) * b, (m.end - m.begin) * b};
+            wait_for(m.src);
             bytes += (m.end - m.begin) * b * b * 4 * f;
         }
     }
     if (r.row0 <= k0 && k0 < r.row0 + r.h) {
         J.b_src = static_cast<const float*>(d.B) + (size_t)(k0 - r.row0) * b * d.W;
+        wait_for(d.idx);
     } else {
         for (const Move& m : ctx->plan_b[k0]) {
             if (m.dst != d.idx) continue;
             const colpart_rect& orr = ctx->rects[m.src];
             J.b_src = static_cast<const float*>(src_B(ctx, m.src)) + (size_t)(k0 - orr.row0) * b * d.W;
+            wait_for(m.src);
             bytes += fb * d.W * 4;
         }
     }
+    J.need = streamed ? flag_value(ctx->epoch, k0 + f - 1) : 0;
     if (J.npieces == 0 || J.b_src == nullptr) return 0;
     J.ldb = d.W;
     J.Kb = fb;
@@ -1651,7 +1684,7 @@ void compute(pmm_ctx* ctx, pmm_stats* st, const HostSrc* host = nullptr, const H
     if (!ctx->have_problem) fail(FPM_ESTATE, "pmm_compute before pmm_setup");
     if (ctx->ipc_mode && !ctx->peers_ready)
         fail(FPM_ESTATE, "IPC context: pmm_ipc_import must follow pmm_setup before pmm_compute");
-    if (ctx->ipc_mode && host) ++ctx->epoch;  // this run's progress-flag values (every rank in step)
+    if (host) ++ctx->epoch;  // this run's progress-flag values (IPC: every rank in step)
     // streamed input: the grouping that starts with single pivots (setup)
     struct GroupSwap {
         pmm_ctx* c;
@@ -1840,7 +1873,11 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
     // band-streamed tail: its uploads, staging and updates are issued after the loop
     auto streamed_tail = [&](const Device& d, int g) { return in_tail(d, g) && d.tail_streamed_run; };
     // in-kernel staging: group g >= 1 (not in the tail) was staged by update g - 1
-    for (auto& d : ctx->devs) d.fs_run = fused_staging_ok(ctx, d, streamed);
+    ctx->stream_flags = false;
+    for (auto& d : ctx->devs) {
+        d.fs_run = fused_staging_ok(ctx, d, streamed);
+        ctx->stream_flags = ctx->stream_flags || (d.fs_run && streamed);
+    }
     auto staged_in_kernel = [&](const Device& d, int g) { return d.fs_run && g >= 1 && !in_tail(d, g); };
     std::vector<char> job_ok(ctx->devs.size(), 0);  // the previous update carried this group's job
     for (int g = 0; g < ngroups; ++g) {
@@ -1884,7 +1921,7 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
             StageJob job;
             job_ok[di] = 0;
             if (d.fs_run && g + 1 < ngroups && !in_tail(d, g + 1)) {
-                const int64_t nb = build_stage_job(ctx, d, g + 1, (g + 1) & 1, job);
+                const int64_t nb = build_stage_job(ctx, d, g + 1, (g + 1) & 1, job, streamed);
                 if (job.active) {
                     bytes += nb;
                     job_ok[di] = 1;

@@ -119,7 +119,7 @@ def test_ipc_fused_staging_pulls_peer_pieces(fused):
     assert all(ok is True for (_, ok, _, _) in out), out
 
 
-def _worker_run(rank, world, port, rects, N, b, reps, q):
+def _worker_run(rank, world, port, rects, N, b, reps, q, opts=None):
     """pmm_run on an IPC context: each rank streams its own host window in (k
     order, its progress flag written after each pivot's panels) while peers
     wait on that flag in their streams before pulling; C streamed out."""
@@ -138,6 +138,8 @@ def _worker_run(rank, world, port, rects, N, b, reps, q):
         B = synth.rect(12, N, r0 * b, c0 * b, H, W, synth.DIST_INT)
         results = []
         with pkg.Context.ipc(rank, world, 0) as ctx:
+            for k, v in (opts or {}).items():
+                ctx.set_option(k, v)
             ctx.setup(N, b, rects, pkg.FPM_F32)
             blobs = [None] * world
             dist.all_gather_object(blobs, ctx.ipc_export())
@@ -175,6 +177,28 @@ def test_ipc_streamed_pmm_run(world, d):
     for p in procs:
         p.start()
     out = sorted(q.get(timeout=300) for _ in range(world))
+    for p in procs:
+        p.join(timeout=60)
+    assert all(ok is True for (_, ok, _, _) in out), out
+
+
+@pytest.mark.parametrize("fused", [1, 0])
+def test_ipc_streamed_fused_staging(fused):
+    """pmm_run on IPC contexts at a size where the update's staging warp stages
+    the next group: it waits in-kernel for the holders' upload-progress flags
+    (own and peers') before pulling; integer inputs bit-exact over repeated runs."""
+    import paper_conf_cluster_zhongrl12_b200 as pkg
+    N, b = 4096, 256
+    n = N // b
+    rects = pkg.colpart_arrange(n, [120, 80, 56])
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    procs = [ctx.Process(target=_worker_run, args=(r, 3, port, rects, N, b, 2, q, {"fused_staging": fused}))
+             for r in range(3)]
+    for p in procs:
+        p.start()
+    out = sorted(q.get(timeout=300) for _ in range(3))
     for p in procs:
         p.join(timeout=60)
     assert all(ok is True for (_, ok, _, _) in out), out

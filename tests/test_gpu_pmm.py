@@ -460,6 +460,34 @@ def test_fused_staging_bit_identical(N, b, fuse, graph):
     assert og.rel_fro(out[0][0], ref) <= 1e-5
 
 
+@pytest.mark.parametrize("N,b,dist", [(4096, 512, synth.DIST_INT), (3072, 256, synth.DIST_PM1)])
+@pytest.mark.parametrize("tail_stream", [1, 0])
+def test_fused_staging_streamed_run(N, b, dist, tail_stream):
+    """pmm_run (host panels streamed in under the k-loop) with in-kernel
+    staging: the staging warp waits for the upload-progress flag of the next
+    group's panels; C bit-identical to fused_staging = 0 over repeated runs
+    (the flag epochs advance), integer inputs bit-exact vs the oracle."""
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n])
+    A = synth.rect(1, N, 0, 0, N, N, dist)
+    B = synth.rect(2, N, 0, 0, N, N, dist)
+    out = []
+    for fs in (1, 0):
+        with pkg.Context.local([0]) as ctx:
+            ctx.set_option("fused_staging", fs)
+            ctx.set_option("tail_stream", tail_stream)
+            for _ in range(2):
+                C = np.full((N, N), np.nan, dtype=np.float32)
+                ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+            out.append(C)
+    assert np.array_equal(out[0], out[1])
+    ref = og.gemm(A, B)
+    if dist == synth.DIST_INT:
+        assert np.array_equal(out[0].astype(np.float64), ref)
+    else:
+        assert og.rel_fro(out[0], ref) <= 1e-5
+
+
 @pytest.mark.parametrize("graph", [1, 0])
 def test_shared_b_operand_bit_identical(graph):
     """Option share_b (default on): column members on the B owner's GPU read its
