@@ -122,7 +122,9 @@ def committed_traffic(N: int, b: int, args):
     variant = (6 if args.scheme == "f16i8" else 8) if args.kernel_variant < 0 else args.kernel_variant
     fuse = args.fuse if args.fuse > 0 else max(1, min(8, 2048 // b))
     G = args.raster_group if args.raster_group > 0 else (12 if args.scheme == "f16i8" else 16)
-    key = f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}") + ("" if G == 16 else f"_r{G}")
+    fs = getattr(args, "fused_staging", 0) and args.scheme == "f16x3" and variant in (7, 8)
+    key = (f"{N}_{b}_{args.scheme}_v{variant}" + ("" if fuse == 1 else f"_f{fuse}") + ("" if G == 16 else f"_r{G}")
+           + ("_fs" if fs else ""))
     if args.gpus != 1 or not os.path.exists(path):
         return None
     entry = json.load(open(path)).get(key)
@@ -472,12 +474,17 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
     upd_med = max(x["update_s"] for x in mine_recs)
     comp_med = max(x["compute_s"] for x in mine_recs)
     stage = comp_med - upd_med
-    exposed = max(0.0, own_times[med] - upd_med)
-    overlap = 1.0 - exposed / stage if stage > 0 else None
-    overlaps = [overlap]
+    exposed = max(0.0, own_times[med] - upd_med)   # k-loop time with no update running
+    # with in-kernel staging the later groups' staging runs inside the updates
+    # (their staging intervals are empty), so a ratio over staging intervals
+    # would mean nothing: the exposed time per step is reported instead
+    fused = bool(args.fused_staging) and args.scheme == "f16x3"
+    overlap = (1.0 - exposed / stage) if (stage > 0 and not fused) else None
+    overlaps, exposeds = [overlap], [exposed]
     if world > 1:
-        overlaps = [None] * world
+        overlaps, exposeds = [None] * world, [None] * world
         dist.all_gather_object(overlaps, overlap)
+        dist.all_gather_object(exposeds, exposed)
 
     # ---- the exchange against NVLink ("NVLink bandwidth for the
     # broadcasts"): pivot bytes this rank pulled per step over its staging time (the
@@ -519,7 +526,8 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
                             (committed_traffic(N, b, args) if not caps else None)),
                 "peak_basis": basis.format(src=peaks["source"], p=dense_peak),
                 "tensor_pipe_frac": achieved * mma_per_mac / dense_peak if dense_peak else None,
-                "kernel": "rank-(f b) update (update_acc_kernel: F16X3 chunked accumulation)"
+                "kernel": ("rank-(f b) update (update_acc_kernel: F16X3 chunked accumulation"
+                           + (", staging the next group in its staging warp)" if args.fused_staging else ")"))
                 if args.scheme == "f16x3" else "rank-(f b) update",
                 "device": busiest["device"]}
 
@@ -593,6 +601,9 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
                 # share of the exchange + staging time hidden under the updates, per rank (CUDA
                 # events of each rank's streams; SURVEY §8(d) c5 "broadcast/update overlap")
                 "exchange_staging_overlap": overlaps[0] if world == 1 else overlaps,
+                # per step: k-loop time during which no update kernel ran (the first group's
+                # staging, launch gaps, and any staging between updates), per rank
+                "exposed_between_updates_ms": (1e3 * exposeds[0]) if world == 1 else [1e3 * x for x in exposeds],
                 "exchange_roofline": ex,
                 "wall_s_timed_region": wall,
                 "partitions": partitions,

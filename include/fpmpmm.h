@@ -407,6 +407,16 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *                 staging its own copy (update groups outside the download
  *                 tail; the owner's next staging into that slot waits for
  *                 those updates); 0: every device stages its own.
+ *   "fused_staging": 1 (default): FP32 F16X3 on the default update kernel --
+ *                 update g's staging warp stages group g + 1 (the pivot pulls
+ *                 from the holders' / owner's memory, the split, the B
+ *                 transpose) while its MMAs run, instead of the standalone
+ *                 staging kernels, which cannot run beside the persistent
+ *                 update and so sat between two updates.  Applies to a GPU
+ *                 device that is the only device of the context on its GPU,
+ *                 in core, not in NCCL mode, with a grid of >= 32 CTAs; under
+ *                 pmm_run the warp first waits for the holders' upload-progress
+ *                 flags.  Bit-identical C.  0: standalone staging kernels.
  *   "sample_rel_ci_permille": fpm_sample's stop rule, the 95 % confidence
  *                 half-width in thousandths of the mean (default 25 = 2.5 %,
  *                 reading Q8; at most 50 repetitions either way).

@@ -1377,9 +1377,10 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     // auto: variant 8 (chunked accumulation, two 64-KB operand stages, C by TMA
     // reduce-add): the FP32-class error bound at every K (Q15c).  Measured c5:
     // 430 TFLOP/s (variant 7, three stages: 421 -- it ran at a lower clock under
-    // the power cap; non-chunked variant 4: 430), and 160 KB of shared memory
-    // leave room for NCCL / staging kernels to co-run.  Variants 0..5 accumulate
-    // a whole update in one TMEM sum (error grows with K).
+    // the power cap; non-chunked variant 4: 430).  No other kernel's CTAs fit
+    // beside it (measured: 320 -- now 352 -- threads x 168 registers), so the
+    // next group's staging runs in its own staging warp (StageJob).  Variants
+    // 0..5 accumulate a whole update in one TMEM sum (error grows with K).
     const int variant = a.variant >= 0 ? a.variant : 8;
     if (a.cta_group == 2) {
         switch (variant) {

@@ -51,6 +51,7 @@ def test_two_ranks_same_gpu_line(config, N, b):
     assert {x["rank"] for x in c["per_device"]} == {0, 1}
     assert sum(c["partition"]) == (N // b) ** 2
     assert isinstance(c["exchange_staging_overlap"], list) and len(c["exchange_staging_overlap"]) == 2
+    assert len(c["exposed_between_updates_ms"]) == 2
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 2 * N * N * 4
     assert d["roofline"]["frac"] > 0 and d["gpu_launches"] > 0 and d["cpu_baseline"] is None
     ex = c["exchange_roofline"]

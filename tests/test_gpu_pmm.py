@@ -137,13 +137,20 @@ def test_run_on_fpm_arrangement(seed):
 def test_kernel_launch_count():
     """pmm_stats.kernel_launches counts every library kernel of the k-loop: per
     update group one A split, three B-row kernels (maxima, split, scales) for
-    F16X3 or one for TF32X3, and the update."""
+    F16X3 or one for TF32X3, and the update; with in-kernel staging (F16X3
+    default) only the first group's staging kernels run, the later groups are
+    staged by the previous update's staging warp."""
     N, b = 2048, 128
     n = N // b
     with pkg.Context.local([0]) as ctx:
         ctx.set_option("fuse", 8)
         ctx.setup(N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
         ctx.fill_synthetic(1, 2)
+        for graph in (0, 1):
+            ctx.set_option("graph", graph)
+            st = ctx.compute()
+            assert st.updates == 2 and st.kernel_launches == (1 + 3) + 2
+        ctx.set_option("fused_staging", 0)
         for graph in (0, 1):
             ctx.set_option("graph", graph)
             st = ctx.compute()
