@@ -413,10 +413,14 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *                 transpose) while its MMAs run, instead of the standalone
  *                 staging kernels, which cannot run beside the persistent
  *                 update and so sat between two updates.  Applies to a GPU
- *                 device that is the only device of the context on its GPU,
- *                 in core, not in NCCL mode, with a grid of >= 32 CTAs; under
- *                 pmm_run the warp first waits for the holders' upload-progress
- *                 flags.  Bit-identical C.  0: standalone staging kernels.
+ *                 device that is alone on its GPU in the context or confined
+ *                 to its own green partition, in core, not in NCCL mode, whose
+ *                 rectangle is large enough for the staging warps to finish
+ *                 inside the update (DESIGN 4.8); under pmm_run the warps
+ *                 first wait for the holders' upload-progress flags.  With
+ *                 share_b a column member stages only its A rows.
+ *                 Bit-identical C.  0: standalone staging kernels; 2: in-kernel
+ *                 staging whatever the rectangle size.
  *   "sample_rel_ci_permille": fpm_sample's stop rule, the 95 % confidence
  *                 half-width in thousandths of the mean (default 25 = 2.5 %,
  *                 reading Q8; at most 50 repetitions either way).

@@ -27,8 +27,9 @@ enum class SplitScheme : int {
 // written to rows row_off.. of a_hi / a_lo (row stride ld_out) with their
 // inverse scales in sa.  B: the block-row(s) b_src (Kb x W, row stride ldb)
 // transposed into b_hi / b_lo (W x Kb, row stride Kb), column maxima in bmax,
-// inverse scales in sb.  ctr: two zeroed counters for the grid barrier between
-// the maxima and the split of B (the kernel leaves them zeroed).
+// inverse scales in sb (b_src null: no B -- the device reads another device's
+// staged B operand).  ctr: two zeroed counters for the grid barrier between the
+// maxima and the split of B (the kernel leaves them zeroed).
 constexpr int kMaxStagePieces = 16;
 struct StagePiece {
     const float* src;

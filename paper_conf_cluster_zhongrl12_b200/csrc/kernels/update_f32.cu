@@ -365,13 +365,15 @@ __device__ __forceinline__ unsigned ld_acquire_u32(const unsigned* p) {
     return v;
 }
 
-// One warp per CTA stages the next update group while this one's MMAs run
-// (kernels.hpp StageJob): B column maxima (one warp per 128-column chunk over
-// all Kb rows, so plain stores, no atomics), the A rows (warp per row: maximum
-// over the fused row, then the split -- split_rows_f16), a grid barrier over
-// the staging warps (every CTA of the persistent grid is resident), then B's
-// split + transpose in (128 columns) x (8 rows) units (split_cols_t) with the
-// inverse scales.  Same arithmetic as the standalone kernels (split_math.cuh).
+// Two warps per CTA stage the next update group while this one's MMAs run
+// (kernels.hpp StageJob): B column maxima ((128 columns) x (128 rows) tasks,
+// atomicMax on the float bits, as colmax_tile_k), the A rows (warp per row:
+// maximum over the fused row, then the split -- split_rows_f16), a grid barrier
+// over the staging warps (every CTA of the persistent grid is resident), then
+// B's split + transpose in (128 columns) x (8 rows) units (split_cols_t) with
+// the inverse scales.  Same arithmetic as the standalone kernels
+// (split_math.cuh).  Independent loads are issued in pairs of rows / units so
+// a warp keeps 8-16 KB in flight.
 __device__ __forceinline__ unsigned __halves2ushort2(__half a, __half b) {
     return (unsigned)__half_as_ushort(a) | ((unsigned)__half_as_ushort(b) << 16);
 }
@@ -383,70 +385,100 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned 
 }
 
 __device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int ncta, int lane) {
-    const int64_t nchunks = (J.W + 127) / 128;
+    const int64_t nchunks = J.b_src != nullptr ? (J.W + 127) / 128 : 0;
     // streamed inputs: wait until every holder's panels of the group have landed
     if (lane == 0)
         for (int i = 0; i < J.nwait; ++i)
             while (ld_acquire_sys_u64(J.wait_flag[i]) < J.need) __nanosleep(1000);
     __syncwarp();
-    // ---- B: column maxima
-    for (int64_t ch = cta; ch < nchunks; ch += ncta) {
+    // ---- B: column maxima, (128 columns) x (128 rows) tasks merged with
+    // atomicMax on the bits (bmax is zero here: setup, then the last staging warp
+    // of every launch re-zeroes it)
+    constexpr int64_t kMaxRows = 128;
+    const int64_t nkp = (J.Kb + kMaxRows - 1) / kMaxRows;
+    for (int64_t tsk = cta; tsk < nchunks * nkp; tsk += ncta) {
+        const int64_t ch = tsk / nkp, k0 = (tsk - ch * nkp) * kMaxRows;
         const int64_t col = ch * 128 + 4 * lane;
         if (col < J.W) {  // W % 4 == 0: a lane's four columns are all in or all out
             float4 m = make_float4(0.f, 0.f, 0.f, 0.f);
             const float* p = J.b_src + col;
-#pragma unroll 8
-            for (int64_t k = 0; k < J.Kb; ++k) {
+            const int64_t k1 = min(J.Kb, k0 + kMaxRows);
+#pragma unroll 16
+            for (int64_t k = k0; k < k1; ++k) {
                 const float4 v = __ldcs(reinterpret_cast<const float4*>(p + k * J.ldb));
                 m.x = fmaxf(m.x, fabsf(v.x));
                 m.y = fmaxf(m.y, fabsf(v.y));
                 m.z = fmaxf(m.z, fabsf(v.z));
                 m.w = fmaxf(m.w, fabsf(v.w));
             }
-            *reinterpret_cast<uint4*>(J.bmax + col) =
-                make_uint4(__float_as_uint(m.x), __float_as_uint(m.y), __float_as_uint(m.z), __float_as_uint(m.w));
+            atomicMax(J.bmax + col + 0, __float_as_uint(m.x));
+            atomicMax(J.bmax + col + 1, __float_as_uint(m.y));
+            atomicMax(J.bmax + col + 2, __float_as_uint(m.z));
+            atomicMax(J.bmax + col + 3, __float_as_uint(m.w));
         }
     }
-    // ---- A: rows of every piece (one warp per row)
+    // ---- A: rows of every piece (one warp per row, two rows at a time: their
+    // loads issued together)
     int64_t rtot = 0;
     for (int i = 0; i < J.npieces; ++i) rtot += J.a[i].rows;
     const int64_t n4 = J.K / 4;
-    for (int64_t g = cta; g < rtot; g += ncta) {
-        int pi = 0;
-        int64_t r = g;
-        while (r >= J.a[pi].rows) r -= J.a[pi++].rows;
-        const StagePiece& pc = J.a[pi];
-        float m = 0.0f;
-        for (int j = 0; j < J.nseg; ++j) {
-            const float4* s4 = reinterpret_cast<const float4*>(pc.src + j * pc.seg_stride + r * J.lda);
-#pragma unroll 4
-            for (int64_t i = lane; i < n4; i += 32) {
-                const float4 v = s4[i];
-                m = fmaxf(m, fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+    for (int64_t g0 = cta; g0 < rtot; g0 += 2 * (int64_t)ncta) {
+        const float* base[2] = {nullptr, nullptr};
+        int64_t ss[2] = {0, 0}, orow[2] = {0, 0};
+        bool ok[2];
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+            int64_t r = g0 + t * (int64_t)ncta;
+            ok[t] = r < rtot;
+            if (ok[t]) {
+                int pi = 0;
+                while (r >= J.a[pi].rows) r -= J.a[pi++].rows;
+                base[t] = J.a[pi].src + r * J.lda;
+                ss[t] = J.a[pi].seg_stride;
+                orow[t] = J.a[pi].row_off + r;
             }
         }
-        m = warp_max(m);
-        const int sh = f16x3_shift(m);
-        const float scale = ldexpf(1.0f, sh);
-        const int64_t orow = pc.row_off + r;
-        if (lane == 0) J.sa[orow] = ldexpf(1.0f, -sh);
+        float m[2] = {0.0f, 0.0f};
         for (int j = 0; j < J.nseg; ++j) {
-            const float4* s4 = reinterpret_cast<const float4*>(pc.src + j * pc.seg_stride + r * J.lda);
-            __half2* h2 = reinterpret_cast<__half2*>(static_cast<__half*>(J.a_hi) + orow * J.ld_out + j * J.K);
-            __half2* l2 = reinterpret_cast<__half2*>(static_cast<__half*>(J.a_lo) + orow * J.ld_out + j * J.K);
-#pragma unroll 4
+#pragma unroll 8
             for (int64_t i = lane; i < n4; i += 32) {
-                const float4 v = __ldcs(s4 + i);
-                __half h[4], l[4];
 #pragma unroll
-                for (int q = 0; q < 4; ++q) f16x3_split((&v.x)[q], scale, h[q], l[q]);
-                // streaming stores: the staged halves must not push the running
-                // update's raster-group operands out of L2
-                __stcs(reinterpret_cast<uint2*>(h2) + i, make_uint2(__halves2ushort2(h[0], h[1]), __halves2ushort2(h[2], h[3])));
-                __stcs(reinterpret_cast<uint2*>(l2) + i, make_uint2(__halves2ushort2(l[0], l[1]), __halves2ushort2(l[2], l[3])));
+                for (int t = 0; t < 2; ++t) {
+                    if (!ok[t]) continue;
+                    const float4 v = reinterpret_cast<const float4*>(base[t] + j * ss[t])[i];
+                    m[t] = fmaxf(m[t], fmaxf(fmaxf(fabsf(v.x), fabsf(v.y)), fmaxf(fabsf(v.z), fabsf(v.w))));
+                }
+            }
+        }
+        float scale[2];
+#pragma unroll
+        for (int t = 0; t < 2; ++t) {
+            const int sh = f16x3_shift(warp_max(m[t]));
+            scale[t] = ldexpf(1.0f, sh);
+            if (ok[t] && lane == 0) J.sa[orow[t]] = ldexpf(1.0f, -sh);
+        }
+        for (int j = 0; j < J.nseg; ++j) {
+#pragma unroll 8
+            for (int64_t i = lane; i < n4; i += 32) {
+#pragma unroll
+                for (int t = 0; t < 2; ++t) {
+                    if (!ok[t]) continue;
+                    const float4 v = __ldcs(reinterpret_cast<const float4*>(base[t] + j * ss[t]) + i);
+                    __half h[4], l[4];
+#pragma unroll
+                    for (int q = 0; q < 4; ++q) f16x3_split((&v.x)[q], scale[t], h[q], l[q]);
+                    // streaming stores: the staged halves must not push the running
+                    // update's raster-group operands out of L2
+                    const int64_t o = orow[t] * J.ld_out + j * J.K;
+                    __stcs(reinterpret_cast<uint2*>(static_cast<__half*>(J.a_hi) + o) + i,
+                           make_uint2(__halves2ushort2(h[0], h[1]), __halves2ushort2(h[2], h[3])));
+                    __stcs(reinterpret_cast<uint2*>(static_cast<__half*>(J.a_lo) + o) + i,
+                           make_uint2(__halves2ushort2(l[0], l[1]), __halves2ushort2(l[2], l[3])));
+                }
             }
         }
     }
+    if (J.b_src == nullptr) return;  // A only (the B operand is another device's)
     // ---- grid barrier: every staging warp's B maxima are written
     __syncwarp();
     if (lane == 0) {
@@ -455,42 +487,65 @@ __device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int nc
         while (ld_acquire_u32(J.ctr) < (unsigned)ncta) __nanosleep(256);
     }
     __syncwarp();
-    // ---- B: split + transpose, (128 columns) x (8 rows of Kb) per unit
+    // ---- B: split + transpose, (128 columns) x (8 rows of Kb) per unit; two
+    // units per iteration, their loads issued together
     const int64_t nk8 = J.Kb / 8;
     const int64_t units = nchunks * nk8;
-    for (int64_t u = cta; u < units; u += ncta) {
-        const int64_t ch = u / nk8, kk = (u - ch * nk8) * 8;
-        const int64_t col = ch * 128 + 4 * lane;
-        if (col >= J.W) continue;
-        float x[4][8];
+    for (int64_t u0 = cta; u0 < units; u0 += 2 * (int64_t)ncta) {
+        float x[2][4][8];
+        int64_t col[2], kk[2];
+        bool ok[2];
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {
-            const float4 v = __ldcs(reinterpret_cast<const float4*>(J.b_src + (kk + i) * J.ldb + col));
-            x[0][i] = v.x;
-            x[1][i] = v.y;
-            x[2][i] = v.z;
-            x[3][i] = v.w;
+        for (int t = 0; t < 2; ++t) {
+            const int64_t u = u0 + t * (int64_t)ncta;
+            const int64_t ch = u / nk8;
+            kk[t] = (u - ch * nk8) * 8;
+            col[t] = ch * 128 + 4 * lane;
+            ok[t] = u < units && col[t] < J.W;
+            if (ok[t]) {
+#pragma unroll
+                for (int i = 0; i < 8; ++i) {
+                    const float4 v =
+                        __ldcs(reinterpret_cast<const float4*>(J.b_src + (kk[t] + i) * J.ldb + col[t]));
+                    x[t][0][i] = v.x;
+                    x[t][1][i] = v.y;
+                    x[t][2][i] = v.z;
+                    x[t][3][i] = v.w;
+                }
+            }
         }
-        const uint4 mb = __ldcg(reinterpret_cast<const uint4*>(J.bmax + col));
-        const unsigned mbits[4] = {mb.x, mb.y, mb.z, mb.w};
 #pragma unroll
-        for (int c = 0; c < 4; ++c) {
-            const int sh = f16x3_shift(__uint_as_float(mbits[c]));
-            const float scale = ldexpf(1.0f, sh);
-            if (kk == 0) J.sb[col + c] = ldexpf(1.0f, -sh);
-            __align__(16) __half h[8], l[8];
+        for (int t = 0; t < 2; ++t) {
+            if (!ok[t]) continue;
+            const uint4 mb = __ldcg(reinterpret_cast<const uint4*>(J.bmax + col[t]));
+            const unsigned mbits[4] = {mb.x, mb.y, mb.z, mb.w};
 #pragma unroll
-            for (int i = 0; i < 8; ++i) f16x3_split(x[c][i], scale, h[i], l[i]);
-            const int64_t orow = (col + c) * J.Kb + kk;
-            __stcs(reinterpret_cast<uint4*>(static_cast<__half*>(J.b_hi) + orow), *reinterpret_cast<uint4*>(h));
-            __stcs(reinterpret_cast<uint4*>(static_cast<__half*>(J.b_lo) + orow), *reinterpret_cast<uint4*>(l));
+            for (int c = 0; c < 4; ++c) {
+                const int sh = f16x3_shift(__uint_as_float(mbits[c]));
+                const float scale = ldexpf(1.0f, sh);
+                if (kk[t] == 0) J.sb[col[t] + c] = ldexpf(1.0f, -sh);
+                __align__(16) __half h[8], l[8];
+#pragma unroll
+                for (int i = 0; i < 8; ++i) f16x3_split(x[t][c][i], scale, h[i], l[i]);
+                const int64_t orow = (col[t] + c) * J.Kb + kk[t];
+                __stcs(reinterpret_cast<uint4*>(static_cast<__half*>(J.b_hi) + orow), *reinterpret_cast<uint4*>(h));
+                __stcs(reinterpret_cast<uint4*>(static_cast<__half*>(J.b_lo) + orow), *reinterpret_cast<uint4*>(l));
+            }
         }
     }
-    // ---- departure: the last staging warp re-arms the barrier for the next launch
+    // ---- departure: the last staging warp re-arms the barrier and zeroes the
+    // column maxima for the next launch (every warp has read them by now)
     __syncwarp();
+    unsigned d = 0;
     if (lane == 0) {
-        const unsigned d = atomicAdd(J.ctr + 1, 1u);
-        if (d == (unsigned)ncta - 1) {
+        __threadfence();
+        d = atomicAdd(J.ctr + 1, 1u);
+    }
+    d = __shfl_sync(0xffffffffu, d, 0);
+    if (d == (unsigned)ncta - 1) {
+        __threadfence();
+        for (int64_t c = 4 * lane; c < J.W; c += 128) *reinterpret_cast<uint4*>(J.bmax + c) = make_uint4(0, 0, 0, 0);
+        if (lane == 0) {
             J.ctr[0] = 0;
             J.ctr[1] = 0;
         }
@@ -515,7 +570,7 @@ __device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int nc
 //   warp 0: TMA producer (A hi/lo, B^T hi/lo k-blocks, 128-byte swizzle)
 //   warp 1: TMEM allocation + single-thread tcgen05.mma issuer (leader CTA)
 //   warps 2-9: epilogue
-//   warp 10: staging of the next update group (StageJob, when given)
+//   warps 10-11: staging of the next update group (StageJob, when given)
 template <int KIND, int STAGES, int NCB>
 struct AccCfg {
     static constexpr int BM = 128, TILE_M = 256, BN = 256, BN_CTA = 128, SW = 128;
@@ -529,7 +584,7 @@ struct AccCfg {
     static constexpr int BAR_BYTES = 8 * (2 * STAGES + 4) + 16;
     static constexpr int SMEM = 1024 + STAGES * STAGE_BYTES + NCB * C_CHUNK_BYTES + BAR_BYTES;
     static constexpr uint32_t IDESC = ptx::idesc_f32acc(TILE_M, BN, KIND == 1);
-    static constexpr int THREADS = 352;  // producer, MMA, 8 epilogue warps, staging warp
+    static constexpr int THREADS = 384;  // producer, MMA, 8 epilogue warps, 2 staging warps
     static_assert(NCB % 2 == 0 && NCBH >= 1 && NCBH <= 4, "C staging: 1..4 chunks per half");
     static_assert(SMEM <= 232448, "shared memory budget");
 };
@@ -656,9 +711,9 @@ __global__ void __maxnreg__(168)
                 }
             }
         }
-    } else if (warp == 10) {
+    } else if (warp >= 10) {
         // ------------------------------------------------ staging of the next group
-        if (P.stg.active) stage_next_group(P.stg, blockIdx.x, gridDim.x, lane);
+        if (P.stg.active) stage_next_group(P.stg, 2 * blockIdx.x + (warp - 10), 2 * gridDim.x, lane);
     } else {
         // -------------------------------------------------------------- epilogue
         const uint32_t e = threadIdx.x - 64;  // 0..255
@@ -1224,7 +1279,8 @@ static void launch_update_acc_t(const UpdateArgs& a, cudaStream_t st) {
     if (P.stg.active) {
         FPM_CHECK_ARG(KIND == 0, "in-kernel staging is F16X3 only");
         FPM_CHECK_ARG(P.stg.npieces >= 1 && P.stg.npieces <= kMaxStagePieces && P.stg.K % 4 == 0 &&
-                          P.stg.Kb % 8 == 0 && P.stg.W % 4 == 0 && P.stg.ldb % 4 == 0 && P.stg.lda % 4 == 0 &&
+                          (P.stg.b_src == nullptr || (P.stg.Kb % 8 == 0 && P.stg.W % 4 == 0 && P.stg.ldb % 4 == 0)) &&
+                          P.stg.lda % 4 == 0 &&
                           P.stg.ctr != nullptr && P.stg.bmax != nullptr,
                       "bad staging job");
     }

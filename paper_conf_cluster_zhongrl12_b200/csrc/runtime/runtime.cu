@@ -854,6 +854,7 @@ void setup(pmm_ctx* ctx, int64_t N, int64_t b, int p, const colpart_rect* rects,
             d.stg_bmax = static_cast<unsigned*>(dalloc(d, (size_t)d.W * sizeof(unsigned)));
             d.stg_ctr = static_cast<unsigned*>(dalloc(d, 2 * sizeof(unsigned)));
             CU(cudaMemsetAsync(d.stg_ctr, 0, 2 * sizeof(unsigned), d.s_comp));
+            CU(cudaMemsetAsync(d.stg_bmax, 0, (size_t)d.W * sizeof(unsigned), d.s_comp));
         }
         for (auto* v : {&d.ev_pack0, &d.ev_pack1, &d.ev_upd0, &d.ev_upd1, &d.ev_up}) {
             v->resize(n);
@@ -1174,10 +1175,27 @@ bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
     if (scheme_for(ctx, ctx->b) != SplitScheme::F16X3 || ctx->cta_group != 2) return false;
     if (!(ctx->kernel_variant == -1 || ctx->kernel_variant == 7 || ctx->kernel_variant == 8)) return false;
     if (!d.stg_bmax || !d.stg_ctr) return false;
+    // every CTA must be resident: alone on the GPU, or confined to its own
+    // green partition (devices sharing a GPU under grid caps oversubscribe it).
+    // Devices sharing a GPU stage in-kernel only when forced (option value 2):
+    // measured on the c4 analogue (eight green partitions, shared B operands)
+    // it was no better -- a column owner's update then waits for its members'
+    // previous updates before it may stage their shared B -- and worse with
+    // the FPM-chosen arrangement (profiles/r02v_fused_staging/hetero_*).
+    bool shares_gpu = false;
     for (const auto& q : ctx->devs)
-        if (&q != &d && !q.cpu && q.cuda_dev == d.cuda_dev && q.live()) return false;
+        if (&q != &d && !q.cpu && q.cuda_dev == d.cuda_dev && q.live()) shares_gpu = true;
+    if (shares_gpu && (!d.green.ctx || ctx->fused_staging != 2)) return false;
+    // worth it (option value 1): the two staging warps per CTA must finish well
+    // inside the update -- per group (f b of K) they move about (8 H + 12 W) f b
+    // bytes while the MMAs take 2 H W f b / (CTAs x ~3 TFLOP/s); at ~4 GB/s per
+    // staging warp that is (8 H + 12 W) x kStageCost <= H W (measured crossover,
+    // profiles/r02v_fused_staging/fs_crossover.jsonl: off below ~5000^2).  2 forces it on.
+    constexpr double kStageCost = 250.0;
+    if (ctx->fused_staging == 1 && (8.0 * (double)d.H + 12.0 * (double)d.W) * kStageCost > (double)d.H * (double)d.W)
+        return false;
     const int64_t tiles = ((d.H + 255) / 256) * ((d.W + 255) / 256);
-    return 2 * std::min<int64_t>(d.num_sms / 2, tiles) >= 32;
+    return std::min<int64_t>(d.num_sms / 2, tiles) >= 1;
 }
 
 // The upload-progress flag of device q as device d reads it (own / local
@@ -1194,7 +1212,7 @@ const unsigned long long* flag_of(pmm_ctx* ctx, const Device& d, int q) {
 // streamed: after their progress flags show the group's panels landed).
 // Returns the pivot bytes pulled from other devices; job.active = 0 when the
 // group has more A pieces than a job holds.
-int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob& J, bool streamed) {
+int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob& J, bool streamed, bool with_b) {
     const int64_t b = ctx->b;
     const int64_t k0 = ctx->groups[g].first;
     const int f = ctx->groups[g].second;
@@ -1230,7 +1248,8 @@ int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob
             bytes += (m.end - m.begin) * b * b * 4 * f;
         }
     }
-    if (r.row0 <= k0 && k0 < r.row0 + r.h) {
+    if (!with_b) {  // B: the column owner's staged operand (share_b)
+    } else if (r.row0 <= k0 && k0 < r.row0 + r.h) {
         J.b_src = static_cast<const float*>(d.B) + (size_t)(k0 - r.row0) * b * d.W;
         wait_for(d.idx);
     } else {
@@ -1243,7 +1262,7 @@ int64_t build_stage_job(pmm_ctx* ctx, const Device& d, int g, int slot, StageJob
         }
     }
     J.need = streamed ? flag_value(ctx->epoch, k0 + f - 1) : 0;
-    if (J.npieces == 0 || J.b_src == nullptr) return 0;
+    if (J.npieces == 0 || (with_b && J.b_src == nullptr)) return 0;
     J.ldb = d.W;
     J.Kb = fb;
     J.W = d.W;
@@ -1914,21 +1933,49 @@ void issue_kloop(pmm_ctx* ctx, const HostSrc* host, const HostDst* out, int L, i
                 }
             }
         }
-        for (size_t di = 0; di < ctx->devs.size(); ++di) {
+        // the updates of group g, each carrying the staging of group g + 1 for
+        // its device (in-kernel staging).  With shared B operands (share_b,
+        // green partitions of one GPU) a column member's job stages its A rows
+        // only: it reads the B operand the owner's update stages, whose launch
+        // first waits for the members' updates that read its previous B in that
+        // slot (the b_from values of the slot's previous use).
+        const int nx = g + 1, sx = nx & 1;
+        const size_t nd = ctx->devs.size();
+        std::vector<StageJob> jobs(nd);
+        std::vector<int64_t> job_bytes(nd, 0);
+        std::vector<int> owner_of(nd, -1);  // device index whose B this device's update nx reads
+        for (size_t di = 0; di < nd; ++di) {
+            Device& d = ctx->devs[di];
+            if (!d.live() || d.cpu || in_tail(d, g) || !d.fs_run || nx >= ngroups || in_tail(d, nx)) continue;
+            const Device* ow = shared_b_owner(ctx, d, nx, sx);
+            if (ow && !ow->fs_run) continue;  // the owner stages eagerly: so does this member (issue_comm)
+            job_bytes[di] = build_stage_job(ctx, d, nx, sx, jobs[di], streamed, ow == nullptr);
+            owner_of[di] = ow ? ow->idx : d.idx;
+        }
+        for (size_t di = 0; di < nd; ++di) {  // a member's job needs the owner's (B) job
+            if (!jobs[di].active || owner_of[di] == ctx->devs[di].idx) continue;
+            for (size_t oi = 0; oi < nd; ++oi)
+                if (ctx->devs[oi].idx == owner_of[di] && !jobs[oi].active) jobs[di].active = 0;
+        }
+        for (size_t di = 0; di < nd; ++di) {
             Device& d = ctx->devs[di];
             if (!d.live() || d.cpu || in_tail(d, g)) continue;
             const bool here = staged_in_kernel(d, g) && job_ok[di];
-            StageJob job;
-            job_ok[di] = 0;
-            if (d.fs_run && g + 1 < ngroups && !in_tail(d, g + 1)) {
-                const int64_t nb = build_stage_job(ctx, d, g + 1, (g + 1) & 1, job, streamed);
-                if (job.active) {
-                    bytes += nb;
-                    job_ok[di] = 1;
-                }
+            const StageJob& job = jobs[di];
+            const bool stages_b = job.active && job.b_src != nullptr;
+            if (stages_b && nx >= 2) {  // readers of this device's B in slot sx at group nx - 2
+                CU(cudaSetDevice(d.cuda_dev));
+                for (auto& q : ctx->devs)
+                    if (&q != &d && !q.cpu && q.live() && q.b_from[sx] == d.idx)
+                        CU(cudaStreamWaitEvent(d.s_comp, q.ev_free[sx], 0));
             }
             issue_update(ctx, d, g, g & 1, job.active ? &job : nullptr, here);
+            if (stages_b) CU(cudaEventRecord(d.ev_ready[sx], d.s_comp));  // members' update nx waits for it
+            job_ok[di] = job.active ? 1 : 0;
+            if (job.active) bytes += job_bytes[di];
         }
+        for (size_t di = 0; di < nd; ++di)
+            if (jobs[di].active) ctx->devs[di].b_from[sx] = owner_of[di];
     }
     // fused tail, pass 2: split every tail group with the merged maxima into its
     // K range of the tail operand
@@ -2994,7 +3041,7 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value == 0 || value == 1, "share_b must be 0 or 1");
             ctx->share_b = (int)value;
         } else if (k == "fused_staging") {
-            FPM_CHECK_ARG(value == 0 || value == 1, "fused_staging must be 0 or 1");
+            FPM_CHECK_ARG(value >= 0 && value <= 2, "fused_staging must be 0, 1 (where it pays) or 2 (always)");
             ctx->fused_staging = (int)value;
         } else if (k == "sample_rel_ci_permille") {
             FPM_CHECK_ARG(value >= 1 && value <= 500, "sample_rel_ci_permille must be in [1, 500]");

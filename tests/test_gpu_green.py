@@ -81,3 +81,40 @@ def test_green_partition_errors():
         C = np.zeros((N, N), np.float32)
         ctx.run(A, B, C, N, b, [(0, 0, 0, 4, 4)], pkg.FPM_F32)
         assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
+@pytest.mark.parametrize("share_b", [1, 0])
+@pytest.mark.parametrize("mode", ["compute", "run"])
+def test_green_fused_staging_with_shared_b(share_b, mode):
+    """In-kernel staging on devices confined to green partitions of one GPU
+    (each grid is resident in its own SMs): every update stages its device's
+    next group; with share_b a column member stages only its A rows and reads
+    the B operand its owner's update staged (the owner's launch waits for the
+    members' updates that read its previous B in that slot).  C bit-identical
+    to fused_staging = 0, resident and streamed (pmm_run), integer inputs
+    bit-exact vs the oracle, repeated calls."""
+    N, b = 4096, 256
+    n = N // b
+    caps = [48, 40, 32]
+    rects = pkg.colpart_arrange(n, [120, 80, 56])
+    assert len({r[0] for r in rects}) == 2                   # one column holds two devices
+    A = synth.rect(11, N, 0, 0, N, N, synth.DIST_INT)
+    B = synth.rect(12, N, 0, 0, N, N, synth.DIST_INT)
+    out = []
+    for fs in (2, 0):
+        with pkg.Context.local([0] * 3, sm_caps=caps) as ctx:
+            ctx.set_option("sm_partition", 1)
+            ctx.set_option("share_b", share_b)
+            ctx.set_option("fused_staging", fs)
+            C = np.full((N, N), np.nan, np.float32)
+            for _ in range(2):
+                if mode == "run":
+                    ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+                else:
+                    ctx.setup(N, b, rects, pkg.FPM_F32)
+                    ctx.upload(A, B, N)
+                    st = ctx.compute()
+                    ctx.download(C, N)
+            out.append(C)
+    assert np.array_equal(out[0], out[1])
+    assert np.array_equal(out[0].astype(np.float64), og.gemm(A, B))

@@ -104,7 +104,7 @@ def test_ipc_three_ranks_mixed_columns():
     assert all(ok is True for (_, ok, _, _) in out), out
 
 
-@pytest.mark.parametrize("fused", [1, 0])
+@pytest.mark.parametrize("fused", [2, 0])
 def test_ipc_fused_staging_pulls_peer_pieces(fused):
     """In-kernel staging on IPC contexts (the driver's N > 1 bench path): the
     staging warp of update g pulls group g + 1's A slices from the holders'
@@ -182,7 +182,7 @@ def test_ipc_streamed_pmm_run(world, d):
     assert all(ok is True for (_, ok, _, _) in out), out
 
 
-@pytest.mark.parametrize("fused", [1, 0])
+@pytest.mark.parametrize("fused", [2, 0])
 def test_ipc_streamed_fused_staging(fused):
     """pmm_run on IPC contexts at a size where the update's staging warp stages
     the next group: it waits in-kernel for the holders' upload-progress flags

@@ -144,6 +144,7 @@ def test_kernel_launch_count():
     n = N // b
     with pkg.Context.local([0]) as ctx:
         ctx.set_option("fuse", 8)
+        ctx.set_option("fused_staging", 2)
         ctx.setup(N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
         ctx.fill_synthetic(1, 2)
         for graph in (0, 1):
@@ -447,7 +448,7 @@ def test_fused_staging_bit_identical(N, b, fuse, graph):
     n = N // b
     rects = pkg.colpart_arrange(n, [n * n])
     out = []
-    for fs in (1, 0):
+    for fs in (2, 0):   # 2: in-kernel staging at these (small) sizes too
         with pkg.Context.local([0]) as ctx:
             ctx.set_option("graph", graph)
             ctx.set_option("fuse", fuse)
@@ -479,7 +480,7 @@ def test_fused_staging_streamed_run(N, b, dist, tail_stream):
     A = synth.rect(1, N, 0, 0, N, N, dist)
     B = synth.rect(2, N, 0, 0, N, N, dist)
     out = []
-    for fs in (1, 0):
+    for fs in (2, 0):
         with pkg.Context.local([0]) as ctx:
             ctx.set_option("fused_staging", fs)
             ctx.set_option("tail_stream", tail_stream)
