@@ -166,3 +166,32 @@ def test_band_streamed_tail_matches_fused_tail(tail, N, b):
             assert np.array_equal(out[1].astype(np.float64), ref)
         else:
             assert og.rel_fro(out[1], ref) <= 1e-5
+
+
+@pytest.mark.parametrize("tail", [-1, 1, 3])
+@pytest.mark.parametrize("mode", ["compute_into", "run"])
+def test_fused_staging_with_tail_bit_identical(tail, mode):
+    """In-kernel staging (forced: option fused_staging = 2) up to the download
+    tail: the last non-tail update stages nothing, the tail groups take the
+    standalone staging (fused tail operand / band-streamed tail); C
+    bit-identical to fused_staging = 0, integers bit-exact vs the oracle."""
+    N, b = 4096, 256
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n])
+    A = synth.rect(21, N, 0, 0, N, N, synth.DIST_INT)
+    B = synth.rect(22, N, 0, 0, N, N, synth.DIST_INT)
+    out = []
+    for fs in (2, 0):
+        C = np.full((N, N), np.nan, np.float32)
+        with pkg.Context.local([0]) as ctx:
+            ctx.set_option("fused_staging", fs)
+            ctx.set_option("e2e_tail", tail)
+            if mode == "run":
+                ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+            else:
+                ctx.setup(N, b, rects, pkg.FPM_F32)
+                ctx.upload(A, B, N)
+                ctx.compute_into(C, N)
+        out.append(C)
+    assert np.array_equal(out[0], out[1])
+    assert np.array_equal(out[0].astype(np.float64), og.gemm(A, B))
