@@ -1,0 +1,5 @@
+O=gpurun_out/r02re1; mkdir -p $O
+nvidia-smi > $O/nvidia-smi.txt 2>&1
+timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $O/smoke.log 2>&1; echo "rc=$?" >> $O/smoke.log
+timeout 2400 python -m pytest tests -m gpu -q -p no:cacheprovider > $O/pytest.log 2>&1; echo "rc=$?" >> $O/pytest.log
+timeout 900 python bench.py > $O/bench.json 2> $O/bench.err
