@@ -1415,6 +1415,12 @@ int tail_groups(pmm_ctx* ctx, bool streamed) {
         if (d.live() && !d.ooc && !d.cpu)
             r = std::max(r, (4.0 / 55e9) / (2.0 * (double)ctx->N / (rate_per_sm * d.num_sms)));
     if (r == 0.0) return 0;
+    // host link slower than the updates (r >= 0.5, e.g. N = 16384 on one B200):
+    // the band-streamed tail takes the whole k-loop -- all of B's rows first,
+    // then A's rows band by band, each band's C leaving over the other PCIe
+    // direction while the next band's rows arrive -- so the step is about the
+    // H2D bytes plus one band, instead of H2D plus most of the D2H
+    if (streamed && streamed_tail_ok(ctx) && r >= 0.5) return std::min(G, kMaxTail);
     int L = (int)std::ceil(G * 1.05 * r);
     if (streamed && streamed_tail_ok(ctx) && r < 0.5)  // 0.55: the tail may start somewhat late (measured, c5:
         L = std::min(L, (int)std::floor(G * (1.0 - 0.55 * r / (1.0 - r))));  // L = 12 of 25 best, 8: -4 %, 16: -8 %)
@@ -1845,7 +1851,7 @@ void issue_tail_streamed(pmm_ctx* ctx, Device& d, int gt, const HostSrc& h, cons
     CU(cudaEventRecord(d.ev_upd0[gt], d.s_comp));
     UpdateArgs fa = f32_args(ctx, d, gt, kFusedSlot);
     fa.K = K;
-    fa.accumulate = true;  // the groups before the tail wrote C
+    fa.accumulate = kt != 0;  // the groups before the tail wrote C (none: the tail is the whole k-loop)
     const int64_t oR0 = r.row0 * b - out.row_base, oC0 = r.col0 * b - out.col_base;
     float* C = static_cast<float*>(d.C);
     for (size_t j = 0; j < bands.size(); ++j) {

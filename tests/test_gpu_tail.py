@@ -139,6 +139,33 @@ def test_e2e_tail_option_errors():
                 ctx.set_option("e2e_tail", bad)
 
 
+@pytest.mark.parametrize("stream", [1, 0])
+@pytest.mark.parametrize("mode", ["run", "compute_into"])
+def test_all_tail_repeated_calls(stream, mode):
+    """The whole k-loop in the tail (e2e_tail >= the number of groups), called
+    repeatedly on one context: the tail's first update must overwrite C_i, not
+    add to the previous call's result (the streamed tail once hard-wired
+    accumulation, which a fresh context's zeroed C hid)."""
+    N, b = 2304, 96   # pmm_run groups {0}, {1}, 8, 8, 6: five groups, all in the tail
+    n = N // b
+    rects = pkg.colpart_arrange(n, [n * n])
+    A = synth.rect(7, N, 0, 0, N, N)
+    B = synth.rect(8, N, 0, 0, N, N)
+    ref = og.gemm(A, B)
+    with pkg.Context.local([0]) as ctx:
+        ctx.set_option("e2e_tail", 16)
+        ctx.set_option("tail_stream", stream)
+        for _ in range(3):
+            C = np.full((N, N), np.nan, np.float32)
+            if mode == "run":
+                ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+            else:
+                ctx.setup(N, b, rects, pkg.FPM_F32)
+                ctx.upload(A, B, N, 0, 0)
+                ctx.compute_into(C, N, 0, 0)
+            assert og.rel_fro(C, ref) <= 1e-5
+
+
 @pytest.mark.parametrize("tail", [-1, 1, 3, 16])
 @pytest.mark.parametrize("N,b", [(4096, 256), (2304, 96)])
 def test_band_streamed_tail_matches_fused_tail(tail, N, b):
@@ -156,7 +183,10 @@ def test_band_streamed_tail_matches_fused_tail(tail, N, b):
         for stream in (0, 1):
             C = np.full((N, N), np.nan, np.float32)
             with pkg.Context.local([0]) as ctx:
-                ctx.set_option("e2e_tail", tail)
+                # auto (-1): at these host-link-bound sizes the band-streamed
+                # tail takes the whole k-loop (runtime.cu tail_groups), so the
+                # fused tail it must match is the whole loop too
+                ctx.set_option("e2e_tail", 16 if (tail == -1 and stream == 0) else tail)
                 ctx.set_option("tail_stream", stream)
                 ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
             out.append(C)
