@@ -389,8 +389,12 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *                 so the copy of C to the host overlaps the last uploads; the
  *                 tail may then be longer (the uploads under the groups before
  *                 it are 8 B per element for those groups + 4 B for the tail's
- *                 B).  Same results bit for bit as 0 (all tail pivots uploaded
- *                 before the tail starts).
+ *                 B).  When the host link is slower than the updates (upload
+ *                 time per element of C_i >= half the k-loop's, e.g. N = 16384
+ *                 on a full B200) the auto tail is the whole k-loop (up to 16
+ *                 groups), so a step costs about its H2D bytes plus one band.
+ *                 Same results bit for bit as 0 at the same tail length (all
+ *                 tail pivots uploaded before the tail starts).
  *   "sm_partition": how an SM cap is enforced.  0 (default): the cap is the
  *                 grid of the persistent update kernel (one CTA per SM); other
  *                 kernels of the device are not confined, and devices sharing a
