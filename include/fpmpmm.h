@@ -214,7 +214,14 @@ int pmm_create_nccl(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm
  * iteration loop, so pulls need no synchronisation with the owner.  Protocol:
  * pmm_setup -> pmm_ipc_export (every rank) -> all-gather of the blobs by the
  * caller -> pmm_ipc_import -> pmm_upload / pmm_fill_synthetic -> caller
- * barrier -> pmm_compute -> pmm_download.  pmm_run returns FPM_EUNSUPPORTED. */
+ * barrier -> pmm_compute -> pmm_download; or, after the import, pmm_run on
+ * every rank with its own host window (same problem, else FPM_EUNSUPPORTED):
+ * each rank streams its panels in and writes a 64-bit upload-progress flag per
+ * pivot, and a peer pulls a pivot only after that flag shows it landed.
+ * Failure detection: a k-loop that cannot finish because a peer stopped (its
+ * flag never advances) fails with FPM_ECUDA instead of blocking -- the host
+ * wait gives up after FPM_IPC_TIMEOUT_S seconds (env, default 600, 0 = never)
+ * and the update kernel's staging warps trap after 60 s of waiting. */
 #define FPM_IPC_BLOB_BYTES 256
 int pmm_create_ipc(int32_t rank, int32_t world, int32_t cuda_device, int32_t sm_cap, pmm_ctx** out);
 int pmm_ipc_export(pmm_ctx* ctx, uint8_t blob_out[FPM_IPC_BLOB_BYTES]);

@@ -384,12 +384,30 @@ __device__ __forceinline__ unsigned long long ld_acquire_sys_u64(const unsigned 
     return v;
 }
 
+// Watchdog of the staging warps' two waits (a holder's upload-progress flag,
+// the grid barrier): a wait that cannot finish -- a peer process died before
+// writing its flag, or a CTA of the grid is not resident -- traps after
+// kStageWaitLimitNs instead of spinning forever, so the launch fails with an
+// error the host reports (FPM_ECUDA) rather than hanging the GPU.  Legitimate
+// waits last one group's upload (milliseconds).
+constexpr unsigned long long kStageWaitLimitNs = 60ull * 1000000000ull;
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+    unsigned long long t;
+    asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+    return t;
+}
+
 __device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int ncta, int lane) {
     const int64_t nchunks = J.b_src != nullptr ? (J.W + 127) / 128 : 0;
     // streamed inputs: wait until every holder's panels of the group have landed
     if (lane == 0)
-        for (int i = 0; i < J.nwait; ++i)
-            while (ld_acquire_sys_u64(J.wait_flag[i]) < J.need) __nanosleep(1000);
+        for (int i = 0; i < J.nwait; ++i) {
+            const unsigned long long t0 = globaltimer_ns();
+            while (ld_acquire_sys_u64(J.wait_flag[i]) < J.need) {
+                __nanosleep(1000);
+                if (globaltimer_ns() - t0 > kStageWaitLimitNs) __trap();
+            }
+        }
     __syncwarp();
     // ---- B: column maxima, (128 columns) x (128 rows) tasks merged with
     // atomicMax on the bits (bmax is zero here: setup, then the last staging warp
@@ -484,7 +502,11 @@ __device__ __noinline__ void stage_next_group(const StageJob& J, int cta, int nc
     if (lane == 0) {
         __threadfence();
         atomicAdd(J.ctr, 1u);
-        while (ld_acquire_u32(J.ctr) < (unsigned)ncta) __nanosleep(256);
+        const unsigned long long t0 = globaltimer_ns();
+        while (ld_acquire_u32(J.ctr) < (unsigned)ncta) {
+            __nanosleep(256);
+            if (globaltimer_ns() - t0 > kStageWaitLimitNs) __trap();
+        }
     }
     __syncwarp();
     // ---- B: split + transpose, (128 columns) x (8 rows of Kb) per unit; two

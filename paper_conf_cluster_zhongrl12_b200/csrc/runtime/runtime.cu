@@ -675,6 +675,27 @@ void nccl_wait(pmm_ctx* ctx, cudaEvent_t ev) {
         if (spin > 64) std::this_thread::sleep_for(std::chrono::microseconds(200));
     }
 }
+// IPC contexts: wait for `ev` with a deadline.  The k-loop waits on peers'
+// progress flags (stream waits, and the staging warps' acquire loads, which
+// trap after 60 s); a peer process that stopped would otherwise block this
+// rank forever.  Deadline: env FPM_IPC_TIMEOUT_S (default 600 s; 0 = none).
+void ipc_wait(cudaEvent_t ev) {
+    static const double limit = [] {
+        const char* e = std::getenv("FPM_IPC_TIMEOUT_S");
+        return e ? std::max(0.0, std::atof(e)) : 600.0;
+    }();
+    const auto t0 = std::chrono::steady_clock::now();
+    for (int spin = 0;; ++spin) {
+        const cudaError_t q = cudaEventQuery(ev);
+        if (q == cudaSuccess) return;
+        if (q != cudaErrorNotReady) CU(q);
+        if (limit > 0 && std::chrono::duration<double>(std::chrono::steady_clock::now() - t0).count() > limit)
+            fail(FPM_ECUDA, "IPC k-loop unfinished after %.0f s: a peer's progress flag stopped advancing "
+                            "(peer process stopped?); FPM_IPC_TIMEOUT_S sets the limit", limit);
+        if (spin > 64) std::this_thread::sleep_for(std::chrono::microseconds(200));
+    }
+}
+
 // A CPU device's stream for pulling pivots out of GPU `cuda_dev`'s memory.
 cudaStream_t pull_stream(Device& d, int cuda_dev) {
     for (auto& ps : d.pulls)
@@ -2097,6 +2118,8 @@ void finish_kloop(pmm_ctx* ctx, pmm_stats* st, bool streamed, const std::vector<
         CU(cudaSetDevice(d.cuda_dev));
         if (ctx->nccl_mode) {  // poll the communicators while waiting (the last
             nccl_wait(ctx, d.ev_stop);  // update waited for the last exchange)
+        } else if (ctx->ipc_mode) {
+            ipc_wait(d.ev_stop);
         } else {
             CU(cudaEventSynchronize(d.ev_stop));
         }
