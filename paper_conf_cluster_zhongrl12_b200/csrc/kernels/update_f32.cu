@@ -611,7 +611,7 @@ struct AccCfg {
     static_assert(SMEM <= 232448, "shared memory budget");
 };
 
-template <int KIND, int STAGES, int NCB>
+template <int KIND, int STAGES, int NCB, int MC = 1>
 __global__ void __maxnreg__(168)
     update_acc_kernel(const __grid_constant__ CUtensorMap tmA_hi, const __grid_constant__ CUtensorMap tmA_lo,
                       const __grid_constant__ CUtensorMap tmB_hi, const __grid_constant__ CUtensorMap tmB_lo,
@@ -630,15 +630,24 @@ __global__ void __maxnreg__(168)
 
     const uint32_t warp = threadIdx.x / 32;
     const uint32_t lane = threadIdx.x % 32;
-    const uint32_t rank = ptx::cluster_ctarank();
+    // MC = 2: clusters of two CTA pairs on vertically adjacent tiles (same tile
+    // column): each CTA loads half of its B^T rows and multicasts them to its
+    // counterpart in the other pair, so B^T crosses L2 once per two tiles
+    const uint32_t crank = ptx::cluster_ctarank();
+    const uint32_t rank = crank & 1;  // position in the CTA pair
+    const uint32_t pr = crank >> 1;   // pair of the cluster
     const bool leader = rank == 0;
-    const int cluster_id = blockIdx.x / 2;
-    const int num_clusters = gridDim.x / 2;
+    const int cluster_id = blockIdx.x / (2 * MC);
+    const int num_clusters = gridDim.x / (2 * MC);
+    const int tiles_mc = (P.tiles_m + MC - 1) / MC;  // cluster tiles: MC tile-rows each
+    const int num_ct = tiles_mc * P.tiles_n;
+    const int group = MC == 1 ? P.group : max(1, P.group / MC);
+    const uint16_t pair_mask = (uint16_t)(0x3u << (2 * pr));
 
     if (threadIdx.x == 0) {
         for (int s = 0; s < STAGES; ++s) {
             ptx::mbar_init(&full[s], 1);
-            ptx::mbar_init(&empty[s], 1);
+            ptx::mbar_init(&empty[s], MC);  // the MMAs of every pair writing into the slot
         }
         for (int a = 0; a < 2; ++a) {
             ptx::mbar_init(&tfull[a], 1);
@@ -670,11 +679,12 @@ __global__ void __maxnreg__(168)
         if (lane == 0) {
             int stage = 0;
             uint32_t phase = 0;
-            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+            for (int t = cluster_id; t < num_ct; t += num_clusters) {
                 int tm, tn;
-                tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn, P.snake != 0);
+                tile_coords(t, tiles_mc, P.tiles_n, group, tm, tn, P.snake != 0);
+                tm = tm * MC + (int)pr;
                 const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
-                const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA;
+                const int n0 = tn * Cfg::BN + (int)rank * Cfg::BN_CTA + (int)pr * (Cfg::BN_CTA / MC);
                 for (int kb = 0; kb < num_kb; ++kb) {
                     ptx::mbar_wait(&empty[stage], phase ^ 1);
                     uint8_t* sA_hi = stage_base + stage * Cfg::STAGE_BYTES;
@@ -685,8 +695,15 @@ __global__ void __maxnreg__(168)
                     if (leader) ptx::mbar_arrive_expect_tx(&full[stage], 2 * Cfg::STAGE_BYTES);
                     ptx::tma_load_2d_cg2(sA_hi, &tmA_hi, &full[stage], k0, m0, ptx::kEvictLast);
                     ptx::tma_load_2d_cg2(sA_lo, &tmA_lo, &full[stage], k0, m0, ptx::kEvictLast);
-                    ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
-                    ptx::tma_load_2d_cg2(sB_lo, &tmB_lo, &full[stage], k0, n0, P.hint_b);
+                    if constexpr (MC == 1) {
+                        ptx::tma_load_2d_cg2(sB_hi, &tmB_hi, &full[stage], k0, n0, P.hint_b);
+                        ptx::tma_load_2d_cg2(sB_lo, &tmB_lo, &full[stage], k0, n0, P.hint_b);
+                    } else {  // this CTA's half of the B^T rows, to itself and its counterpart
+                        const uint16_t mask = (uint16_t)((1u << rank) | (1u << (rank + 2)));
+                        const int off = (int)pr * (Cfg::BN_CTA / MC) * Cfg::SW;
+                        ptx::tma_load_2d_cg2_mc(sB_hi + off, &tmB_hi, &full[stage], k0, n0, mask, P.hint_b);
+                        ptx::tma_load_2d_cg2_mc(sB_lo + off, &tmB_lo, &full[stage], k0, n0, mask, P.hint_b);
+                    }
                     if (++stage == STAGES) { stage = 0; phase ^= 1; }
                 }
             }
@@ -697,7 +714,7 @@ __global__ void __maxnreg__(168)
             int stage = 0;
             uint32_t phase = 0;
             int it = 0;  // accumulations issued (chunks over all tiles)
-            for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+            for (int t = cluster_id; t < num_ct; t += num_clusters) {
                 for (int kb0 = 0; kb0 < num_kb; kb0 += ckb, ++it) {
                     const int acc = it & 1;
                     ptx::mbar_wait(&tempty[acc], ((it >> 1) & 1) ^ 1);
@@ -723,12 +740,12 @@ __global__ void __maxnreg__(168)
                                 ptx::umma<2, KIND>(d_tmem, dA_hi + off, dB_lo + off, Cfg::IDESC, 1);
                                 ptx::umma<2, KIND>(d_tmem, dA_hi + off, dB_hi + off, Cfg::IDESC, 1);
                             }
-                            ptx::umma_commit<2>(&empty[stage]);
+                            ptx::umma_commit_mask(&empty[stage], MC == 1 ? 0x3 : 0xF);  // every producer writing the slot
                         }
                         __syncwarp();
                         if (++stage == STAGES) { stage = 0; phase ^= 1; }
                     }
-                    if (lane == 0) ptx::umma_commit<2>(&tfull[acc]);
+                    if (lane == 0) ptx::umma_commit_mask(&tfull[acc], pair_mask);
                     __syncwarp();
                 }
             }
@@ -745,9 +762,10 @@ __global__ void __maxnreg__(168)
         const uint32_t r = q * 32 + lane;     // row of the CTA tile
         uint8_t* cb = cbuf + hh * Cfg::NCBH * Cfg::C_CHUNK_BYTES;
         int it = 0;
-        for (int t = cluster_id; t < P.num_tiles; t += num_clusters) {
+        for (int t = cluster_id; t < num_ct; t += num_clusters) {
             int tm, tn;
-            tile_coords(t, P.tiles_m, P.tiles_n, P.group, tm, tn, P.snake != 0);
+            tile_coords(t, tiles_mc, P.tiles_n, group, tm, tn, P.snake != 0);
+            tm = tm * MC + (int)pr;
             const int m0 = tm * Cfg::TILE_M + (int)rank * Cfg::BM;
             const int n0 = tn * Cfg::BN + (int)hh * 128;
             float s[128];
@@ -772,7 +790,7 @@ __global__ void __maxnreg__(168)
                 // accumulator read: hand it back to the MMA warp
                 ptx::tc_fence_before();
                 __syncwarp();
-                if (lane == 0) ptx::mbar_arrive_cluster(&tempty[acc], 0);
+                if (lane == 0) ptx::mbar_arrive_cluster(&tempty[acc], 2 * pr);
             }
             // C update of this tile: C (+)= 2^-(ea+eb) s, once per tile (overlaps the next tile's MMAs)
             const int grow = m0 + (int)r;
@@ -1272,14 +1290,14 @@ static void launch_update_t(const UpdateArgs& a, cudaStream_t st) {
 }
 
 
-template <int KIND, int STAGES, int NCB>
+template <int KIND, int STAGES, int NCB, int MC = 1>
 static void launch_update_acc_t(const UpdateArgs& a, cudaStream_t st) {
     using Cfg = AccCfg<KIND, STAGES, NCB>;
     const CUtensorMapDataType odt = KIND == 1 ? CU_TENSOR_MAP_DATA_TYPE_FLOAT32 : CU_TENSOR_MAP_DATA_TYPE_FLOAT16;
     const CUtensorMap tAh = make_tmap_2d(a.a_hi, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
     const CUtensorMap tAl = make_tmap_2d(a.a_lo, odt, Cfg::ELEM, a.M, a.K, a.K, Cfg::BK, Cfg::BM);
-    const CUtensorMap tBh = make_tmap_2d(a.bt_hi, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
-    const CUtensorMap tBl = make_tmap_2d(a.bt_lo, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA);
+    const CUtensorMap tBh = make_tmap_2d(a.bt_hi, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA / MC);
+    const CUtensorMap tBl = make_tmap_2d(a.bt_lo, odt, Cfg::ELEM, a.Nc, a.K, a.K, Cfg::BK, Cfg::BN_CTA / MC);
     const CUtensorMap tC = make_tmap_2d(a.C, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 4, a.M, a.Nc, a.ldc, 32, Cfg::BM);
     UpdParams P;
     P.M = (int)a.M;
@@ -1306,30 +1324,42 @@ static void launch_update_acc_t(const UpdateArgs& a, cudaStream_t st) {
                           P.stg.ctr != nullptr && P.stg.bmax != nullptr,
                       "bad staging job");
     }
-    auto kern = update_acc_kernel<KIND, STAGES, NCB>;
+    auto kern = update_acc_kernel<KIND, STAGES, NCB, MC>;
     static uint64_t attr_done = 0;  // one bit per CUDA device
+    static int max_clusters[64] = {};
     int dev = 0;
     cudaGetDevice(&dev);
-    if (!(attr_done & (1ull << dev))) {
-        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
-        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
-        attr_done |= 1ull << dev;
-    }
-    int clusters = a.num_sms / 2;
-    if (clusters > P.num_tiles) clusters = P.num_tiles;
-    if (clusters < 1) clusters = 1;
     cudaLaunchConfig_t cfg = {};
-    cfg.gridDim = dim3(clusters * 2);
     cfg.blockDim = dim3(Cfg::THREADS);
     cfg.dynamicSmemBytes = Cfg::SMEM;
     cfg.stream = st;
     cudaLaunchAttribute attr[1];
     attr[0].id = cudaLaunchAttributeClusterDimension;
-    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.x = 2 * MC;
     attr[0].val.clusterDim.y = 1;
     attr[0].val.clusterDim.z = 1;
     cfg.attrs = attr;
     cfg.numAttrs = 1;
+    if (!(attr_done & (1ull << dev))) {
+        cudaError_t e = cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, Cfg::SMEM);
+        if (e != cudaSuccess) fail(FPM_ECUDA, "cudaFuncSetAttribute: %s", cudaGetErrorString(e));
+        if (MC > 1) {  // the persistent grid (and the staging warps' grid barrier) must be co-resident
+            int sms = 0;
+            cudaDeviceGetAttribute(&sms, cudaDevAttrMultiProcessorCount, dev);
+            cfg.gridDim = dim3((unsigned)(sms / (2 * MC) * 2 * MC));
+            int n = 0;
+            e = cudaOccupancyMaxActiveClusters(&n, kern, &cfg);
+            if (e != cudaSuccess || n < 1) fail(FPM_ECUDA, "cudaOccupancyMaxActiveClusters: %s", cudaGetErrorString(e));
+            if (dev < 64) max_clusters[dev] = n;
+        }
+        attr_done |= 1ull << dev;
+    }
+    const int num_ct = ((P.tiles_m + MC - 1) / MC) * P.tiles_n;
+    int clusters = a.num_sms / (2 * MC);
+    if (MC > 1 && dev < 64 && max_clusters[dev] > 0 && clusters > max_clusters[dev]) clusters = max_clusters[dev];
+    if (clusters > num_ct) clusters = num_ct;
+    if (clusters < 1) clusters = 1;
+    cfg.gridDim = dim3(clusters * 2 * MC);
     cudaError_t e = cudaLaunchKernelEx(&cfg, kern, tAh, tAl, tBh, tBl, tC, P);
     if (e != cudaSuccess) fail(FPM_ECUDA, "update kernel launch: %s", cudaGetErrorString(e));
 }
@@ -1418,9 +1448,10 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
     FPM_CHECK_ARG(a.K % 8 == 0, "K must be a multiple of 8");
     FPM_CHECK_ARG(a.M < (1LL << 31) && a.Nc < (1LL << 31), "matrix too large");
     FPM_CHECK_ARG((a.variant >= -1 && a.variant <= 5) || ((a.variant == 7 || a.variant == 8) && a.scheme != SplitScheme::F16I8) ||
+                      ((a.variant == 12 || a.variant == 13) && a.scheme == SplitScheme::F16X3) ||
                       (a.variant >= 6 && a.variant <= 11 && a.variant != 7 && a.variant != 8 &&
                        a.scheme == SplitScheme::F16I8),
-                  "kernel variant must be -1 (auto), 0..5, 7, 8 (F16X3 / TF32X3) or 6, 9..11 (F16I8)");
+                  "kernel variant must be -1 (auto), 0..5, 7, 8 (F16X3 / TF32X3), 12, 13 (F16X3) or 6, 9..11 (F16I8)");
     FPM_CHECK_ARG(a.chunk_k >= 0, "chunk_k must be >= 0");
     const bool tf32 = a.scheme == SplitScheme::TF32X3;
     if (a.scheme == SplitScheme::F16I8) {
@@ -1469,6 +1500,14 @@ void launch_update_f32(const UpdateArgs& a, cudaStream_t st) {
             case 8:  // chunked accumulation, 2 stages + 2 C staging chunks (160 KB): room for NCCL kernels
                 if (tf32) launch_update_acc_t<1, 2, 2>(a, st);
                 else launch_update_acc_t<0, 2, 2>(a, st);
+                break;
+            case 12:  // variant 8 on clusters of two CTA pairs, B^T multicast (F16X3)
+                FPM_CHECK_ARG(!tf32, "variant 12 is F16X3 only");
+                launch_update_acc_t<0, 2, 2, 2>(a, st);
+                break;
+            case 13:  // variant 7 on clusters of two CTA pairs, B^T multicast (F16X3)
+                FPM_CHECK_ARG(!tf32, "variant 13 is F16X3 only");
+                launch_update_acc_t<0, 3, 2, 2>(a, st);
                 break;
             case 1:  // 64-B k-blocks x 4 stages, 6 C chunks in flight
                 if (tf32) launch_update_t<2, 1, 256, 4, 64, 6>(a, st);

@@ -1194,7 +1194,9 @@ bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
     if (!ctx->fused_staging || ctx->dt != FPM_F32 || ctx->nccl_mode || d.cpu || d.ooc || !d.live()) return false;
     if (streamed && (has_cpu(ctx) || !stream_ops_available())) return false;
     if (scheme_for(ctx, ctx->b) != SplitScheme::F16X3 || ctx->cta_group != 2) return false;
-    if (!(ctx->kernel_variant == -1 || ctx->kernel_variant == 7 || ctx->kernel_variant == 8)) return false;
+    if (!(ctx->kernel_variant == -1 || ctx->kernel_variant == 7 || ctx->kernel_variant == 8 ||
+          ctx->kernel_variant == 12 || ctx->kernel_variant == 13))
+        return false;
     if (!d.stg_bmax || !d.stg_ctr) return false;
     // every CTA must be resident: alone on the GPU, or confined to its own
     // green partition (devices sharing a GPU under grid caps oversubscribe it).
@@ -3063,8 +3065,9 @@ extern "C" int pmm_set_option(pmm_ctx* ctx, const char* key, int64_t value) {
             FPM_CHECK_ARG(value == 0 || value == 1, "ooc_keep must be 0 or 1");
             ctx->ooc_keep = (int)value;
         } else if (k == "kernel_variant") {
-            FPM_CHECK_ARG(value >= -1 && value <= 8,
-                          "kernel_variant must be -1 (auto) or 0..8 (6: F16I8 only; 7, 8: F16X3 / TF32X3 only)");
+            FPM_CHECK_ARG((value >= -1 && value <= 8) || value == 12 || value == 13,
+                          "kernel_variant must be -1 (auto), 0..8 (6: F16I8 only; 7, 8: F16X3 / TF32X3 only) "
+                          "or 12, 13 (F16X3 on clusters of two CTA pairs, B multicast)");
             ctx->kernel_variant = (int)value;
         } else if (k == "share_b") {
             FPM_CHECK_ARG(value == 0 || value == 1, "share_b must be 0 or 1");
@@ -3349,8 +3352,9 @@ extern "C" int fpm_k_update_f32(const void* a_hi, const void* a_lo, const void* 
         FPM_CHECK_ARG(scheme >= 0 && scheme <= 3, "scheme must be 0, 1, 2 (int8 timing probe) or 3");
         FPM_CHECK_ARG(cta_group == 1 || cta_group == 2, "cta_group must be 1 or 2");
         FPM_CHECK_ARG((variant >= -1 && variant <= 5) || ((variant == 7 || variant == 8) && scheme != 3) ||
+                          ((variant == 12 || variant == 13) && scheme == 0) ||
                           (variant >= 6 && variant <= 11 && variant != 7 && variant != 8 && scheme == 3),
-                      "variant must be -1 (auto), 0..5, 7, 8, or 6, 9..11 with F16I8");
+                      "variant must be -1 (auto), 0..5, 7, 8, 12, 13 (F16X3), or 6, 9..11 with F16I8");
         FPM_CHECK_ARG(scheme == 1 || scheme == 2 || (sa && sb), "F16X3 / F16I8 need sa and sb");
         fpm::UpdateArgs a;
         a.a_hi = a_hi; a.a_lo = a_lo; a.bt_hi = bt_hi; a.bt_lo = bt_lo;

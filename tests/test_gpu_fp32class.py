@@ -262,6 +262,31 @@ def test_tile_order_and_chunking_options_keep_c_bit_identical(opts):
             assert np.array_equal(out[0], out[1]), (opts, d)
 
 
+@pytest.mark.parametrize("variant", [12, 13])
+@pytest.mark.parametrize("N,b,d,fused", [(2048, 256, [64], 1), (2048, 256, [64], 2), (1792, 256, [49], 2),
+                                         (1600, 320, [13, 12], 0), (4096, 512, [40, 24], 0)])
+def test_multicast_variants_bit_identical(variant, N, b, d, fused):
+    """Kernel variants 12 / 13 run the default chunked F16X3 update on clusters
+    of two CTA pairs that share each B^T k-block by TMA multicast (half loaded
+    by each pair).  Only the operand delivery changes, so C is bit-identical to
+    the default variant 8: one device (with and without in-kernel staging; an
+    odd number of tile-rows, whose second pair of the last cluster row has no
+    tile), ragged 320-wide blocks, two devices sharing the GPU."""
+    n = N // b
+    rects = pkg.colpart_arrange(n, d)
+    A, B = make_inputs("gauss", N, b, seed=73)
+    out = []
+    for v in (-1, variant):
+        C = np.full((N, N), np.nan, np.float32)
+        with pkg.Context.local([0] * len(d)) as ctx:
+            ctx.set_option("kernel_variant", v)
+            ctx.set_option("fused_staging", fused)
+            ctx.run(A, B, C, N, b, rects, pkg.FPM_F32)
+        out.append(C)
+    assert np.array_equal(out[0], out[1]), (variant, N, b, d)
+    assert og.rel_fro(out[1], og.gemm(A, B)) <= TOL
+
+
 @pytest.mark.parametrize("N,b,fuse,d", [(32, 32, 1, [1]), (96, 32, 1, [5, 4]), (4096, 2048, 1, [4]),
                                         (1600, 320, 0, [13, 12]), (2304, 64, 8, [600, 300, 200, 196])])
 def test_default_kernel_edge_shapes(N, b, fuse, d):
