@@ -345,8 +345,8 @@ int fpm_sample_rects(pmm_ctx* ctx, int32_t dev, fpm_dtype dt, int64_t b, const i
  *   "cta_group":  1 or 2 (default 2: CTA pairs, cta_group::2, 256-row tiles).
  *   "kernel_variant": -1 (auto, default: F16X3 / TF32X3 8, F16I8 6 -- 5 in
  *                 NCCL contexts, whose kernels need shared memory beside the
- *                 update) or 0..8, see fpm_k_update_f32.
- *   "chunk_k":    variants 7 / 8: K summed per TMEM accumulation before the
+ *                 update) or 0..8, 12, 13, see fpm_k_update_f32.
+ *   "chunk_k":    variants 7 / 8 / 12 / 13: K summed per TMEM accumulation before the
  *                 epilogue adds it to its FP32 register sum (0 = auto = 512;
  *                 DESIGN.md Q15c: the tensor cores' accumulation error grows
  *                 with the MMAs folded into one sum).
@@ -501,11 +501,14 @@ int fpm_k_transpose(const void* src, int32_t dt, int64_t ld, int64_t rows, int64
  * x 2 + 6, 3 = 64-byte x 5 + 4, 4 = 128-byte x 2 + 4 (leaves ~36 KB smem per
  * SM for NCCL / staging kernels co-running with the update), 5 = 128-byte x 3
  * + 2 with C updated by TMA reduce-add (C never loaded into shared memory);
- * variants 0..5 sum a whole update in one TMEM accumulation.  7 (auto) =
+ * variants 0..5 sum a whole update in one TMEM accumulation.  7 =
  * chunked accumulation: every 512 of K is a fresh TMEM accumulation drained
  * into per-thread FP32 register sums (round-to-nearest), C written once per
  * tile by TMA reduce-add (store when accumulate = 0), 3 x 64-KB operand
- * stages; 8 = the same with 2 stages (160 KB).  -1 = auto (8).
+ * stages; 8 = the same with 2 stages (160 KB).  12 / 13 (F16X3 only) =
+ * variants 8 / 7 on clusters of two CTA pairs that share each B^T k-block by
+ * TMA multicast (same C bit for bit; measured slower on B200).
+ * -1 = auto (8).
  * scheme 3 (F16I8; cta_group 2, K % 64 == 0; sa / sb required): the
  * fp16 + int8 kernel, variants 0 = 2 x 64-KB stages + 4 C chunks,
  * 1 = 3 stages + 2 chunks, 2 = 2 + 6, 3 = 64-byte k-blocks x 5 + 4, 5 = variant
