@@ -613,7 +613,7 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
     if rank == 0:
         if world == 1 and not caps and not args.no_hetero:
             try:
-                line["hetero"] = run_hetero(peak, args.share_b)
+                line["hetero"] = run_hetero(peak, args.share_b, args.hetero_fused_staging)
             except Exception as ex:  # report, do not hide
                 log("hetero failed:", repr(ex))
                 line["hetero"] = {"error": repr(ex)[:200]}
@@ -700,7 +700,7 @@ def fig7_summary() -> dict | None:
     return out if out["layouts"] else None
 
 
-def run_hetero(peak_tflops: float, share_b: int = 1) -> dict:
+def run_hetero(peak_tflops: float, share_b: int = 1, fused_staging: int = 1) -> dict:
     """The metric's 'FPM load imbalance %' under emulated heterogeneity (SURVEY
     §8(d) c4 analogue, studies/hetero.py): 8 devices on this GPU in disjoint
     green-context SM partitions, FPMs sampled per device, the multiply under
@@ -711,7 +711,8 @@ def run_hetero(peak_tflops: float, share_b: int = 1) -> dict:
     caps = [30, 26, 24, 20, 16, 14, 10, 6]   # config 4's {144 .. 32} scaled to fit 148 SMs
     t0 = time.perf_counter()
     res = hetero.c4_study(caps, N=32768, b=512, reps=3, insitu=1, graph=0, sm_partition=1, log=log, refine_rounds=3,
-                          refine_arrange=("fpm",), refine_ci_permille=10, options={"share_b": share_b})
+                          refine_arrange=("fpm",), refine_ci_permille=10,
+                          options={"share_b": share_b, "fused_staging": fused_staging})
     sms = torch.cuda.get_device_properties(0).multi_processor_count
     capped_peak = peak_tflops * sum(caps) / sms
     out = {"workload": ("c4 analogue: N=32768, b=512, FP32, p=8 devices emulated on one B200 by green-context "
@@ -863,6 +864,8 @@ def main():
     ap.add_argument("--e2e-tail", type=int, default=-1, help="pmm_run option e2e_tail (-1 auto)")
     ap.add_argument("--tail-band", type=int, default=0, help="pmm_run option tail_band (rows, multiple of 256; 0 default)")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--hetero-fused-staging", type=int, default=1,
+                    help="hetero block: option fused_staging of its contexts (1 auto: off for devices sharing a GPU; 2 forced)")
     ap.add_argument("--no-hetero", action="store_true",
                     help="skip the heterogeneity measurement added to the line: N = 1 the c4 analogue on "
                          "eight green partitions of the GPU, N > 1 config 4 across the job's GPUs")
