@@ -184,6 +184,29 @@ def e2e_parity(N: int, hC, oracle_block, seeds) -> dict:
             "blocks": out, "max_rel_fro": worst, "ok": bool(worst <= 1e-5)}
 
 
+def e2e_parity_rank(N: int, hC, window, seeds, rank: int) -> list:
+    """N > 1: sampled 64 x 64 blocks (corners and centre) of this rank's
+    rectangle of the e2e output against the oracle; the operands' full rows and
+    columns come from the same counter-based generator the device filled them
+    with (synth)."""
+    import numpy as np
+
+    import synth
+    from oracle import gemm as og
+    R0, C0, H, W = window
+    sa, sb = seeds
+    C = hC.numpy() if hasattr(hC, "numpy") else np.asarray(hC)
+    h, w = min(64, H), min(64, W)
+    out = []
+    for name, r, c in (("top-left", 0, 0), ("bottom-right", H - h, W - w), ("centre", (H - h) // 2, (W - w) // 2)):
+        A = synth.rect(sa, N, R0 + r, 0, h, N)
+        B = synth.rect(sb, N, 0, C0 + c, N, w)
+        ref = og.gemm(A, B)
+        out.append({"rank": rank, "block": name, "rows": [R0 + r, R0 + r + h], "cols": [C0 + c, C0 + c + w],
+                    "rel_fro": float(og.rel_fro(C[r:r + h, c:c + w], ref))})
+    return out
+
+
 # ----------------------------------------------------------------- main arms
 def run_reference(args, rank: int):
     if rank != 0:
@@ -565,16 +588,19 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
         install(rects)   # back to the FPM arrangement for e2e
 
     # ---- end to end through pmm_run with pinned host buffers
-    e2e, hC = None, None
+    e2e, hC, window = None, None, None
     if args.e2e_steps > 0:
         try:
-            e2e, hC = run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, transport == "ipc", N, b,
-                              seeds)
+            e2e, hC, window = run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, transport == "ipc",
+                                      N, b, seeds)
         except Exception as ex:  # report, do not hide
             log("e2e failed:", repr(ex))
             e2e = {"value": None, "unit": UNIT, "error": repr(ex)[:200]}
 
-    cpu, parity = None, None  # the oracle baseline is timed at N = 1 only (rank 0); N > 1 lines carry null
+    # the oracle leg, after every timed region: at N = 1 rank 0 times the oracle
+    # (cpu_baseline; N > 1 lines carry null) and checks the e2e output with it;
+    # at N > 1 every rank checks sampled blocks of its own rectangle
+    cpu, parity = None, None
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         g, cores, desc, _, c_block = oracle_sample(N, want_c=True, seed_cfg=cfg["seed_cfg"])
         cpu = {"value": g, "unit": UNIT, "cores": cores, "kind": "oracle", "sample": desc}
@@ -582,6 +608,20 @@ def run_ours(args, rank: int, world: int, local_rank: int, dist, emit: bool = Tr
             parity = e2e_parity(N, hC, c_block, seeds)
             if not parity["ok"]:
                 log("PARITY FAILURE of the e2e output:", json.dumps(parity))
+    elif world > 1 and not args.no_cpu_baseline and args.e2e_steps > 0:
+        # every rank checks sampled blocks of its own rectangle of the e2e output
+        # against the oracle; rank 0 reports them all (every rank joins the gather)
+        ok_here = hC is not None and e2e is not None and e2e.get("value") is not None
+        mine = e2e_parity_rank(N, hC, window, seeds, rank) if ok_here else []
+        allb = [None] * world
+        dist.all_gather_object(allb, mine)
+        blocks = [blk for r in allb for blk in r]
+        worst = max((blk["rel_fro"] for blk in blocks), default=0.0)
+        parity = {"what": "e2e output C (each rank's host window, pmm_run) vs the CPU oracle on sampled blocks "
+                          "of every rank's rectangle", "tol": 1e-5, "blocks": blocks, "max_rel_fro": worst,
+                  "ok": bool(blocks) and worst <= 1e-5}
+        if rank == 0 and not parity["ok"]:
+            log("PARITY FAILURE of the e2e output:", json.dumps(parity))
 
     line = None
     if rank == 0:
@@ -828,7 +868,7 @@ def run_e2e(args, ctx, rects, rank, world, max_over_ranks, barrier, ipc, N, b, s
         import torch.distributed as dist
         dist.all_reduce(tot)
         rec["h2d_bytes_per_step"], rec["d2h_bytes_per_step"] = int(tot[0].item()), int(tot[1].item())
-    return rec, (hC if (live and world == 1) else None)
+    return rec, (hC if live else None), (R0, C0, H, W)
 
 
 def main():

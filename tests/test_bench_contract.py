@@ -104,3 +104,29 @@ def test_n_gt_1_line_contract():
     assert c["exchange_staging_overlap"] == [0.9, 0.8]
     assert line["dtype"].startswith("f32 (F16X3")
     json.dumps(line)
+
+
+def test_n_gt_1_rank_parity_blocks():
+    """N > 1: each rank checks sampled blocks of ITS rectangle of the e2e output
+    (host window at rows R0.., columns C0..) against the oracle.  A window equal
+    to the exact product passes; a perturbed element in the centre block or an
+    off-by-one window offset is caught."""
+    import numpy as np
+
+    import synth
+    from oracle import gemm as og
+    bm = _bench_module()
+    N, seeds = 320, (11, 12)
+    R0, C0, H, W = 64, 128, 192, 160
+    A = synth.rect(seeds[0], N, R0, 0, H, N)
+    B = synth.rect(seeds[1], N, 0, C0, N, W)
+    hC = og.gemm(A, B).astype(np.float32)
+    blocks = bm.e2e_parity_rank(N, hC, (R0, C0, H, W), seeds, rank=1)
+    assert [b["block"] for b in blocks] == ["top-left", "bottom-right", "centre"]
+    assert blocks[1]["rows"] == [R0 + H - 64, R0 + H] and blocks[1]["cols"] == [C0 + W - 64, C0 + W]
+    assert all(b["rank"] == 1 and b["rel_fro"] <= 1e-7 for b in blocks)
+    bad = hC.copy()
+    bad[(H - 64) // 2 + 5, (W - 64) // 2 + 7] += 1.0
+    assert bm.e2e_parity_rank(N, bad, (R0, C0, H, W), seeds, 1)[2]["rel_fro"] > 1e-5
+    shifted = bm.e2e_parity_rank(N, hC, (R0 + 1, C0, H, W), seeds, 1)
+    assert max(b["rel_fro"] for b in shifted) > 1e-2

@@ -54,6 +54,10 @@ def test_two_ranks_same_gpu_line(config, N, b):
     assert len(c["exposed_between_updates_ms"]) == 2
     assert d["e2e"]["value"] > 0 and d["e2e"]["h2d_bytes_per_step"] == 2 * N * N * 4
     assert d["roofline"]["frac"] > 0 and d["gpu_launches"] > 0 and d["cpu_baseline"] is None
+    # the e2e output of every rank's rectangle checked against the oracle (3 blocks per rank)
+    par = d["parity"]
+    assert par["ok"] and par["max_rel_fro"] <= 1e-5 and {x["rank"] for x in par["blocks"]} == {0, 1}
+    assert len(par["blocks"]) == 6
     ex = c["exchange_roofline"]
     assert ex["bound"] == "nvlink" and ex["peak"] == 900.0 and len(ex["achieved_per_rank"]) == 2
     assert ex["achieved"] > 0 and "same GPU" in ex["path"]
