@@ -305,8 +305,10 @@ int pmm_run(pmm_ctx* ctx, const void* A, const void* B, void* C, int64_t N, int6
 /* Build a speed function (P:9 kernel-based benchmarking, P:10 (iii) repeated
  * until statistically reliable, P:18 sqrt(x) x sqrt(x) submatrices): for each
  * x = sizes[j] (must be a perfect square m^2), time the computational kernel
- * C += A(b) x B(b) (pivot split + rank-b update) on an (m b) x (m b) C on
- * device `dev` of the context (its SM cap applies) and return
+ * C += A(b) x B(b) (pivot split + rank-b update, as the k-loop runs it: where
+ * its updates stage the next group in-kernel -- option "fused_staging" -- the
+ * timed update stages the next run's operands the same way) on an (m b) x (m b)
+ * C on device `dev` of the context (its SM cap applies) and return
  * speeds_out[j] = 2 x b^3 / t in flop/s.  Repeats until the 95% confidence
  * half-width is <= 2.5% of the mean (>= 5, <= 50 repetitions, reading Q8).
  * dev = -1 samples every device of the context simultaneously (P:10 (ii)

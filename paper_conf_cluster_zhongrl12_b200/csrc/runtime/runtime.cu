@@ -1190,14 +1190,26 @@ bool stream_ops_available() {
     }
 }
 
+// Whether device d's updates on an H x W rectangle stage the next group in
+// their staging warps (the kernel / placement / size rules below), FP32 only.
+// sampling: every other GPU device of the context on d's GPU counts as sharing
+// it (before a problem is set up no device is live; in the run they share it).
+bool fused_staging_applies(const pmm_ctx* ctx, const Device& d, int64_t b, int64_t H, int64_t W,
+                           bool sampling = false);
+
 bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
     if (!ctx->fused_staging || ctx->dt != FPM_F32 || ctx->nccl_mode || d.cpu || d.ooc || !d.live()) return false;
     if (streamed && (has_cpu(ctx) || !stream_ops_available())) return false;
-    if (scheme_for(ctx, ctx->b) != SplitScheme::F16X3 || ctx->cta_group != 2) return false;
+    if (!d.stg_bmax || !d.stg_ctr) return false;
+    return fused_staging_applies(ctx, d, ctx->b, d.H, d.W);
+}
+
+bool fused_staging_applies(const pmm_ctx* ctx, const Device& d, int64_t b, int64_t H, int64_t W, bool sampling) {
+    if (!ctx->fused_staging || ctx->nccl_mode || d.cpu || H <= 0 || W <= 0) return false;
+    if (scheme_for(ctx, b) != SplitScheme::F16X3 || ctx->cta_group != 2) return false;
     if (!(ctx->kernel_variant == -1 || ctx->kernel_variant == 7 || ctx->kernel_variant == 8 ||
           ctx->kernel_variant == 12 || ctx->kernel_variant == 13))
         return false;
-    if (!d.stg_bmax || !d.stg_ctr) return false;
     // every CTA must be resident: alone on the GPU, or confined to its own
     // green partition (devices sharing a GPU under grid caps oversubscribe it).
     // Devices sharing a GPU stage in-kernel only when forced (option value 2):
@@ -1207,7 +1219,7 @@ bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
     // the FPM-chosen arrangement (profiles/r02v_fused_staging/hetero_*).
     bool shares_gpu = false;
     for (const auto& q : ctx->devs)
-        if (&q != &d && !q.cpu && q.cuda_dev == d.cuda_dev && q.live()) shares_gpu = true;
+        if (&q != &d && !q.cpu && q.cuda_dev == d.cuda_dev && (sampling || q.live())) shares_gpu = true;
     if (shares_gpu && (!d.green.ctx || ctx->fused_staging != 2)) return false;
     // worth it (option value 1): the two staging warps per CTA must finish well
     // inside the update -- per group (f b of K) they move about (8 H + 12 W) f b
@@ -1215,9 +1227,9 @@ bool fused_staging_ok(pmm_ctx* ctx, const Device& d, bool streamed) {
     // staging warp that is (8 H + 12 W) x kStageCost <= H W (measured crossover,
     // profiles/r02v_fused_staging/fs_crossover.jsonl: off below ~5000^2).  2 forces it on.
     constexpr double kStageCost = 250.0;
-    if (ctx->fused_staging == 1 && (8.0 * (double)d.H + 12.0 * (double)d.W) * kStageCost > (double)d.H * (double)d.W)
+    if (ctx->fused_staging == 1 && (8.0 * (double)H + 12.0 * (double)W) * kStageCost > (double)H * (double)W)
         return false;
-    const int64_t tiles = ((d.H + 255) / 256) * ((d.W + 255) / 256);
+    const int64_t tiles = ((H + 255) / 256) * ((W + 255) / 256);
     return std::min<int64_t>(d.num_sms / 2, tiles) >= 1;
 }
 
@@ -2402,7 +2414,11 @@ struct CpuRunner {
 // One GPU device's sampling kernel, as the k-loop runs it: staging (split /
 // transpose) of an f-pivot group and the fused rank-(f b) update on an h b x w b
 // C; shapes whose C exceeds the device's C cap run out of core through the band
-// ring in the k-loop's steady state (bands kept, order reversed).
+// ring in the k-loop's steady state (bands kept, order reversed).  Where
+// the k-loop stages the next group inside the update (§4.8, same rule), so
+// does the sampler: each run's update reads one operand set and its staging
+// warps split the panels into the other for the next run, so the timed kernel
+// carries the staging the run pays (hidden, not added).
 struct GpuRunner {
     pmm_ctx* ctx;
     Device* d;
@@ -2417,6 +2433,13 @@ struct GpuRunner {
     float *sa = nullptr, *sb = nullptr;
     int64_t Hm = 0, Wm = 0;  // largest rows / columns of C over this device's shapes
     int runs = 0;            // runs at the current size (out-of-core band order alternates)
+    // in-kernel staging: a second operand set, the staging warps' scratch, and
+    // the shape each set currently holds
+    void *ah2 = nullptr, *al2 = nullptr, *bh2 = nullptr, *bl2 = nullptr;
+    float *sa2 = nullptr, *sb2 = nullptr;
+    unsigned *bmax = nullptr, *ctr = nullptr;
+    int cur = 0;
+    int64_t held[2][2] = {{-1, -1}, {-1, -1}};
 
     bool ooc_at(int64_t Mx, int64_t Nx) const { return d->c_cap > 0 && (int64_t)(Mx * Nx * es) > d->c_cap; }
     Ring ring_at(int64_t Mx, int64_t Nx) const { return ring_for(d->c_cap, Mx, Nx, es, ctx->ooc_buffers); }
@@ -2460,6 +2483,21 @@ struct GpuRunner {
             bl = dalloc(mem, (size_t)Wm * fb * op);
             sa = static_cast<float*>(dalloc(mem, (size_t)Hm * 4));
             sb = static_cast<float*>(dalloc(mem, (size_t)Wm * 4));
+            bool fused = false;
+            for (const Shape& x : shp)
+                fused = fused || (!ooc_at(x.h * b, x.w * b) && fused_staging_applies(ctx, *d, b, x.h * b, x.w * b, true));
+            if (fused) {
+                ah2 = dalloc(mem, (size_t)Hm * fb * op);
+                al2 = dalloc(mem, (size_t)Hm * fb * op);
+                bh2 = dalloc(mem, (size_t)Wm * fb * op);
+                bl2 = dalloc(mem, (size_t)Wm * fb * op);
+                sa2 = static_cast<float*>(dalloc(mem, (size_t)Hm * 4));
+                sb2 = static_cast<float*>(dalloc(mem, (size_t)Wm * 4));
+                bmax = static_cast<unsigned*>(dalloc(mem, (size_t)Wm * sizeof(unsigned)));
+                ctr = static_cast<unsigned*>(dalloc(mem, 2 * sizeof(unsigned)));
+                CU(cudaMemsetAsync(bmax, 0, (size_t)Wm * sizeof(unsigned), d->s_comp));
+                CU(cudaMemsetAsync(ctr, 0, 2 * sizeof(unsigned), d->s_comp));
+            }
         }
         launch_fill_synthetic(Ap, dt == FPM_F64, fb, 101, L, 0, 0, Hm, fb, FPM_DIST_PM1, d->s_comp);
         launch_fill_synthetic(Bp, dt == FPM_F64, Wm, 102, L, 0, 0, fb, Wm, FPM_DIST_PM1, d->s_comp);
@@ -2481,12 +2519,55 @@ struct GpuRunner {
         bc.keep_tail = ctx->ooc_keep;
         ++runs;
         if (dt == FPM_F32) {
-            launch_split_rows(static_cast<const float*>(Ap), fb, Mx, fb, sch, ah, al, sa, st);
-            launch_split_cols(static_cast<const float*>(Bp), Wm, fb, Nx, sch, bh, bl, sb, st);
+            // operand sets: [0] = ah / al / bh / bl / sa / sb, [1] = the *2 buffers
+            void* const AH[2] = {ah, ah2};
+            void* const AL[2] = {al, al2};
+            void* const BH[2] = {bh, bh2};
+            void* const BL[2] = {bl, bl2};
+            float* const SA[2] = {sa, sa2};
+            float* const SB[2] = {sb, sb2};
+            const bool fused = !ooc && ah2 != nullptr && fused_staging_applies(ctx, *d, b, Mx, Nx, true);
+            int s0 = fused ? cur : 0;
+            StageJob job;
+            if (fused) {
+                if (held[s0][0] != Mx || held[s0][1] != Nx) {  // first run at this shape: stage it alone
+                    launch_split_rows(static_cast<const float*>(Ap), fb, Mx, fb, sch, AH[s0], AL[s0], SA[s0], st);
+                    launch_split_cols(static_cast<const float*>(Bp), Wm, fb, Nx, sch, BH[s0], BL[s0], SB[s0], st);
+                }
+                // the update's staging warps stage the same panels into the other set (the next run's)
+                const int s1 = s0 ^ 1;
+                job.nseg = 1;
+                job.K = fb;
+                job.lda = fb;
+                job.ld_out = fb;
+                job.a[0] = StagePiece{static_cast<const float*>(Ap), 0, 0, Mx};
+                job.npieces = 1;
+                job.b_src = static_cast<const float*>(Bp);
+                job.ldb = Wm;
+                job.Kb = fb;
+                job.W = Nx;
+                job.a_hi = AH[s1];
+                job.a_lo = AL[s1];
+                job.sa = SA[s1];
+                job.b_hi = BH[s1];
+                job.b_lo = BL[s1];
+                job.sb = SB[s1];
+                job.bmax = bmax;
+                job.ctr = ctr;
+                job.active = 1;
+                held[s0][0] = held[s1][0] = Mx;
+                held[s0][1] = held[s1][1] = Nx;
+                cur = s1;
+            } else {
+                launch_split_rows(static_cast<const float*>(Ap), fb, Mx, fb, sch, ah, al, sa, st);
+                launch_split_cols(static_cast<const float*>(Bp), Wm, fb, Nx, sch, bh, bl, sb, st);
+                held[0][0] = held[1][0] = -1;  // set 0 now holds a shape the fused path does not track
+            }
             UpdateArgs a;
-            a.a_hi = ah; a.a_lo = al; a.bt_hi = bh; a.bt_lo = bl;
-            a.sa = has_scales(sch) ? sa : nullptr;
-            a.sb = has_scales(sch) ? sb : nullptr;
+            a.a_hi = AH[s0]; a.a_lo = AL[s0]; a.bt_hi = BH[s0]; a.bt_lo = BL[s0];
+            a.sa = has_scales(sch) ? SA[s0] : nullptr;
+            a.sb = has_scales(sch) ? SB[s0] : nullptr;
+            a.stage = job;
             a.C = static_cast<float*>(C);
             a.M = Mx; a.Nc = Nx; a.K = fb; a.ldc = Nx;
             a.scheme = sch;
