@@ -268,6 +268,32 @@ def test_fpm_sample_procedure():
             ctx.sample(0, 256, [3])                        # not a perfect square
 
 
+@pytest.mark.parametrize("cap", [0, 64])
+def test_fpm_sample_through_fused_staging(cap):
+    """Where the k-loop stages the next group inside the update (sizes from
+    about 5000^2 on a device alone on its GPU), fpm_sample times that path:
+    each timed update stages the next run's operands in-kernel.  At such
+    sizes the sampled speeds are positive and converge, in-kernel sampling is
+    no slower than the standalone split + update it replaces (option
+    fused_staging = 0), and the same context's run afterwards is correct."""
+    b, ms = 512, [4, 12, 16]
+    sizes = [m * m for m in ms]
+    caps = [cap] if cap else None
+    with pkg.Context.local([0], sm_caps=caps) as ctx:
+        sp, ci, reps = ctx.sample(0, b, sizes, pkg.FPM_F32)
+        assert all(s > 0 for s in sp) and all(5 <= r <= 50 for r in reps)
+        ctx.set_option("fused_staging", 0)
+        sp0, _, _ = ctx.sample(0, b, sizes, pkg.FPM_F32)
+        ctx.set_option("fused_staging", 1)
+        assert sp[2] >= 0.95 * sp0[2], (sp, sp0)   # 8192^2: in-kernel staging applies
+        N = 2048
+        n = N // b
+        A, B = synth.rect(31, N, 0, 0, N, N), synth.rect(32, N, 0, 0, N, N)
+        C = np.full((N, N), np.nan, np.float32)
+        ctx.run(A, B, C, N, b, [(0, 0, 0, n, n)], pkg.FPM_F32)
+    assert og.rel_fro(C, og.gemm(A, B)) <= 1e-5
+
+
 def test_fpm_sample_all_devices_concurrently():
     """dev = -1: every device sampled at once (P:10 (ii)); a device capped to
     fewer SMs must come out slower at a size that fills the GPU."""
